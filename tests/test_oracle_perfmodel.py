@@ -1,0 +1,182 @@
+"""Pins of oracle/perfmodel.py (Eq. 1, Eq. 2, T_m, Alg. 1 reading) against the
+paper's printed numbers (Table 1; O-proj bound), closed forms
+and brute-force enumeration.  CPU only."""
+import json
+import math
+import os
+
+import pytest
+
+from oracle import perfmodel as PM
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden", "table1_wave_idle.json")
+
+
+def test_eq1_reproduces_table1_columns():
+    """Eq. 1 with the grid of each kernel reproduces the 12 reproducible
+    Table 1 entries to the printed 0.1 %."""
+    t = json.load(open(GOLD))
+    M = t["M"]
+    for row in t["rows"]:
+        sl = row["sl"]
+        got = {"QKV": PM.wave_idle((sl // 128) * (6144 // 256), M),
+               "Attn": PM.wave_idle((sl // 128) * 32, M),
+               "OProj": PM.wave_idle((sl // 128) * (4096 // 256), M)}
+        for k, v in got.items():
+            assert abs(100 * v - row[k]) <= 0.05 + 1e-9, (sl, k, 100 * v, row[k])
+
+
+def test_oproj_theoretical_bound_consistency():
+    """O-proj theoretical utilisation bound 59 % / 79 % = 1 - s."""
+    t = json.load(open(GOLD))["oproj_theoretical_bound_pct"]
+    for sl in (1024, 2048):
+        s = PM.wave_idle((sl // 128) * 16, 108)
+        assert round(100 * (1 - s)) == t[str(sl)]
+
+
+def test_eq1_closed_forms():
+    assert PM.wave_idle(148 * 3, 148) == 0.0
+    assert math.isclose(PM.wave_idle(37, 148), 1 - 37 / 148)
+    assert PM.wave_idle(0, 148) == 0.0
+    assert math.isclose(PM.wave_idle(149, 148), 1 - 149 / 296)
+
+
+def test_eq2_reduces_to_plain_roofline():
+    """m = M, d = p = 1, s = 0 -> max(c/C, b/B)."""
+    for c, b in [(1e12, 1e6), (1e6, 1e12), (3e9, 2e9)]:
+        t = PM.kernel_time(c, b, 1e15, 1e12, 148, 148, 1, 1, 1, 1, 0.0)
+        assert t == max(c / 1e15, b / 1e12)
+
+
+def test_eq2_with_wave_quantization_closed_form():
+    """Compute-bound kernel of g tiles, d = p = 1: Eq. 1 + Eq. 2 give
+    t(m) = c/C * M * ceil(g/m) / g, which is non-increasing in m."""
+    c, C, M, g = 2e12, 1.6e15, 148, 300
+    prev = math.inf
+    for m in range(2, 149, 2):
+        t = PM.kernel_time(c, 0, C, 1, M, m, 1, 1, 1, 1, PM.wave_idle(g, m))
+        assert math.isclose(t, c / C * M * math.ceil(g / m) / g, rel_tol=1e-12)
+        assert t <= prev * (1 + 1e-12)
+        prev = t
+
+
+def test_layer_kernel_inventory_flops():
+    """Flop counts of the inventory: GEMMs 2 n K N; attention 4 hd H x causal
+    pairs, pairs = s(s+1)/2 per prefill request, ctx+1 per decode request."""
+    P = PM.default_params()
+    shape = dict(d=4096, H=32, Hkv=8, hd=128, I=14336, elt=2, q_lens=[512, 100], ctx_lens=[0, 0])
+    ks = {k[0]: k for k in PM.layer_kernels(shape, P, 148)}
+    n = 612
+    assert ks["qkv"][1] == 2.0 * n * 4096 * 6144
+    assert ks["o_proj"][1] == 2.0 * n * 4096 * 4096
+    assert ks["gate_up"][1] == 2.0 * n * 4096 * 2 * 14336
+    assert ks["down"][1] == 2.0 * n * 14336 * 4096
+    assert ks["attn"][1] == 4.0 * 128 * 32 * (512 * 513 // 2 + 100 * 101 // 2)
+    dec = dict(shape, q_lens=[1] * 4, ctx_lens=[10, 20, 30, 40])
+    kd = {k[0]: k for k in PM.layer_kernels(dec, P, 148)}
+    assert kd["attn"][1] == 4.0 * 128 * 32 * (11 + 21 + 31 + 41)
+    assert kd["attn"][2] == 2 * 2 * 8 * 128 * (11 + 21 + 31 + 41) + 2 * 2 * 4 * 32 * 128
+    assert kd["attn"][3] == 4 * 8
+
+
+def test_layer_time_monotone_in_sms():
+    P = PM.default_params()
+    shape = dict(d=4096, H=32, Hkv=8, hd=128, I=14336, elt=2, q_lens=[4096], ctx_lens=[0])
+    ts = [PM.layer_time(shape, P, m, 0) for m in range(8, 149, 2)]
+    # not strictly monotone under split-K re-planning, but close: within 2 %
+    for a, b in zip(ts, ts[1:]):
+        assert b <= a * 1.02
+
+
+def test_interp_piecewise_linear():
+    tab = {"m": [10, 20, 40], "v": [0.5, 0.7, 1.0]}
+    assert PM.interp(tab, 5) == 0.5 and PM.interp(tab, 40) == 1.0 and PM.interp(tab, 100) == 1.0
+    assert math.isclose(PM.interp(tab, 15), 0.6) and math.isclose(PM.interp(tab, 30), 0.85)
+
+
+def test_p90_nearest_rank():
+    assert PM.p90([]) == 0.0
+    assert PM.p90(list(range(1, 11))) == 9
+    assert PM.p90([5]) == 5
+    assert PM.p90(list(range(1, 21))) == 18
+
+
+def test_sm_ranges_partition():
+    sigma = list(range(0, 296, 2))
+    for p in (0, 2, 146, 148):
+        a, b = PM.sm_ranges(p, sigma)
+        assert len(a) == p and set(a).isdisjoint(b) and sorted(a + b) == sorted(sigma)
+
+
+# -------------------------------------------------------------- Alg. 1
+
+MODEL = dict(d=4096, H=32, Hkv=8, hd=128, I=14336, elt=2)
+SLO = {"ttft_norm_ms_per_tok": 1.5, "tpot_ms": 175.0, "w_max": 4, "v_min": 16, "percentile": 0.9}
+
+
+def _state(**kw):
+    s = dict(layers_done=4, total_layers=32, prefill_lens=[2048], prefill_waited_ms=[100.0],
+             pending_lens=[], pending_waited_ms=[], decode_tokens=[50] * 64,
+             decode_elapsed_ms=[50 * 20.0] * 64, decode_mean_ctx=1024, u_k=100, v_k=48)
+    s.update(kw)
+    return s
+
+
+def _eval_all(P, st, slo):
+    return {v: PM.evaluate_split(P, MODEL, st, slo, P["M"] - v, v) for v in PM.candidates(P, slo, 2)}
+
+
+def test_case_both_ok_reduces_decode_to_minimal_feasible():
+    """Alg. 1 l.12-13: both SLOs met -> ReduceDecodeSM: the smallest decode SM
+    count that still meets both SLOs (prefill priority)."""
+    P = PM.default_params()
+    st = _state()
+    ev = _eval_all(P, st, SLO)
+    assert ev[48][0] <= 1 and ev[48][1] <= 1
+    u, k = PM.choose_split(P, MODEL, st, SLO)
+    v = P["M"] - u
+    assert ev[v][0] <= 1 and ev[v][1] <= 1
+    assert all(not (ev[w][0] <= 1 and ev[w][1] <= 1) for w in ev if w < v)
+    assert k >= 1
+
+
+def test_case_both_violated_sets_balanced():
+    """Alg. 1 l.15-16 (R-14): both violated -> argmin of max ratio."""
+    P = PM.default_params()
+    st = _state(prefill_waited_ms=[4000.0], decode_elapsed_ms=[50 * 400.0] * 64)
+    ev = _eval_all(P, st, SLO)
+    assert ev[48][0] > 1 and ev[48][1] > 1
+    u, _ = PM.choose_split(P, MODEL, st, SLO)
+    best = min(max(e[0], e[1]) for e in ev.values())
+    assert max(ev[P["M"] - u][0], ev[P["M"] - u][1]) == best
+
+
+def test_case_tpot_violated_reduces_prefill():
+    """Alg. 1 l.18-19: TTFT ok, TPOT violated, queue short -> smallest decode
+    increase that meets TPOT."""
+    P = PM.default_params()
+    st = _state(v_k=16, u_k=132, decode_tokens=[0] * 64, decode_elapsed_ms=[0.0] * 64,
+                prefill_waited_ms=[0.0])
+    slo = dict(SLO, tpot_ms=20.0)
+    ev = _eval_all(P, st, slo)
+    assert ev[16][0] <= 1 and ev[16][1] > 1
+    u, _ = PM.choose_split(P, MODEL, st, slo)
+    v = P["M"] - u
+    assert v > 16 and ev[v][1] <= 1
+    assert all(ev[w][1] > 1 for w in ev if 16 <= w < v)
+
+
+def test_case_ttft_violated_pauses_decode_when_tpot_allows():
+    """§3.3.3: TTFT violated even at v_min while TPOT holds ->
+    pause decode for the cycle (prefill gets all SMs, k = 0)."""
+    P = PM.default_params()
+    st = _state(prefill_waited_ms=[3053.0], decode_elapsed_ms=[50 * 1.0] * 64)
+    ev = _eval_all(P, st, SLO)
+    assert all(e[0] > 1 for e in ev.values())
+    assert PM.choose_split(P, MODEL, st, SLO) == (P["M"], 0)
+
+
+def test_degenerate_states():
+    P = PM.default_params()
+    assert PM.choose_split(P, MODEL, _state(decode_tokens=[], decode_elapsed_ms=[]), SLO) == (148, 0)
+    assert PM.choose_split(P, MODEL, _state(prefill_lens=[], prefill_waited_ms=[]), SLO) == (0, 32)
