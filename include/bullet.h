@@ -1,0 +1,260 @@
+/*
+ * bullet.h — C ABI of the Bullet co-run hot path on B200 (sm_100a).
+ *
+ * Bullet runs a prefill batch and a decode batch of an LLM at the same time
+ * on disjoint SM partitions of one GPU, re-deciding the partition every
+ * layer-level scheduling cycle with a roofline performance model
+ * (§3.1).  This library is the data-parallel
+ * hot path of that method:
+ *
+ *   bullet_create          model + KV pool, SM probe            (§3.5.2; §3.4)
+ *   bullet_step            one co-run layer step, both phases   (§3.1 step 5 P:L131; §3.3.1)
+ *   bullet_model_predict   Eq. 1 + Eq. 2 + T_m
+ *   bullet_choose_split    Alg. 1 + §3.3.3 search
+ *
+ * Conventions (every call):
+ *   - Returns BULLET_OK (0) or a negative BULLET_E* code; bullet_last_error()
+ *     gives a thread-local message.  Argument validation happens before any
+ *     work is enqueued; a failed call enqueues nothing.
+ *   - Pointers named d_* / documented "device" are CUDA device pointers;
+ *     h_* / "host" are host pointers.  No C++ types, exceptions or torch
+ *     types cross this boundary.  Streams are cudaStream_t passed as void*.
+ *   - Ownership: the caller owns weights, KV pools, hidden buffers, block
+ *     tables and streams, and keeps them alive while the handle uses them.
+ *     The handle owns its workspace, work counters, RoPE table and NCCL
+ *     communicators.
+ *   - Element types: dtype BULLET_DTYPE_BF16 -> weights, KV pool and
+ *     activations are bf16; BULLET_DTYPE_FP32 -> all fp32 (tiny config).
+ *     The residual stream `hidden` is always fp32.
+ *   - The library has no CPU fallback: without a usable sm_100 device
+ *     bullet_create fails with BULLET_ECUDA / BULLET_EUNSUPPORTED.
+ */
+#ifndef BULLET_H
+#define BULLET_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct bullet_handle bullet_handle;
+
+enum {
+  BULLET_OK = 0,
+  BULLET_EINVAL = -1,        /* bad argument / shape */
+  BULLET_ECUDA = -2,         /* CUDA runtime or driver error */
+  BULLET_ENCCL = -3,         /* NCCL error (tensor parallel) */
+  BULLET_ESMRANGE = -4,      /* prefill_sm_count out of [0, N] or off-granularity */
+  BULLET_EKV = -5,           /* block id out of range / request exceeds its block table */
+  BULLET_ENOMEM = -6,        /* workspace allocation failed or batch exceeds max_* */
+  BULLET_EUNSUPPORTED = -7   /* shape the kernels do not support (see bullet_create) */
+};
+
+enum { BULLET_DTYPE_FP32 = 0, BULLET_DTYPE_BF16 = 1 };
+
+/* bullet_step flags */
+enum {
+  BULLET_CORUN = 0,          /* phases concurrently on disjoint SM ranges (the method) */
+  BULLET_TIMESLICED = 1,     /* same kernels on all SMs, prefill then decode (baseline) */
+  BULLET_UNGATED = 2,        /* both phases concurrently on all SMs ("Naive") */
+  BULLET_SMID_LOG = 4        /* record (launch, tile, smid) of every work unit */
+};
+
+/* Model shape (per GPU under tensor parallelism: n_heads, n_kv_heads and
+ * d_ff are the LOCAL counts; d_model is the full hidden size).  The layer is
+ * the Llama pre-norm block (reading R-1; the paper names only
+ * QKV-projection, attention, O-projection and MLP). */
+typedef struct {
+  int n_layers;              /* layers whose weights/pools are registered */
+  int d_model, n_heads, n_kv_heads, head_dim, d_ff;
+  float rms_eps;
+  double rope_theta;
+  int rope_llama3;           /* 1: llama3 inv_freq rescaling (Llama-3.1) */
+  float rope_factor, rope_low_freq, rope_high_freq;
+  int rope_orig_max_pos;
+  int max_position;          /* RoPE table length (max token position + 1) */
+  int qkv_bias;              /* 1: b_qkv present (Qwen2.5) */
+  int dtype;                 /* BULLET_DTYPE_* */
+  int tp_size, tp_rank;      /* 1, 0 without tensor parallelism */
+  int max_prefill_tokens;    /* workspace sizing, prefill phase */
+  int max_decode_tokens;     /* workspace sizing, decode phase */
+} bullet_model_cfg;
+
+/* KV pool: one K and one V array per layer, each
+ * [n_blocks][n_kv_heads][block_size][head_dim] of dtype, row-major.  Token
+ * position p of a request lives in block block_table[r][p / block_size] at
+ * offset p % block_size (index table shared by both phases; a request
+ * moving from prefill to decode keeps its block-table row — copy-free). */
+typedef struct {
+  void *const *d_k;          /* host array of n_layers device pointers */
+  void *const *d_v;
+  int n_blocks, block_size;
+} bullet_kv_pool;
+
+/* Weights of one layer, device pointers, row-major [out][in] (nn.Linear):
+ *   w_qkv     [(H+2Hkv)*hd][d]   rows: q heads, then k heads, then v heads
+ *   b_qkv     [(H+2Hkv)*hd]      or NULL when qkv_bias == 0
+ *   w_o       [d][H*hd]
+ *   w_gate_up [2*I][d]           rows [0,I) gate, [I,2I) up
+ *   w_down    [d][I]
+ *   g_attn, g_mlp [d]            RMSNorm gains
+ * bf16 (or fp32 for BULLET_DTYPE_FP32); b_qkv and gains also of dtype. */
+typedef struct {
+  const void *w_qkv, *b_qkv, *w_o, *w_gate_up, *w_down, *g_attn, *g_mlp;
+} bullet_layer_weights;
+
+/* One phase's batch.  Request r has ctx_lens[r] tokens cached and
+ * q_len_r = cu_seqlens[r+1] - cu_seqlens[r] new tokens at positions
+ * ctx_lens[r] .. ctx_lens[r] + q_len_r - 1.  Prefill: ctx 0 (any ctx works);
+ * decode: q_len 1.  `hidden` rows are the new tokens, request-major; it is
+ * read as x and overwritten with the layer output (fp32 residual stream).
+ * The batch runs layers [layer_begin, layer_end) in order. */
+typedef struct {
+  int n_reqs, n_tokens, max_blocks_per_req;
+  const int32_t *d_cu_seqlens;   /* device [n_reqs+1] */
+  const int32_t *d_ctx_lens;     /* device [n_reqs] */
+  const int32_t *d_block_table;  /* device [n_reqs][max_blocks_per_req] */
+  const int32_t *h_cu_seqlens;   /* host mirrors (validation, planning) */
+  const int32_t *h_ctx_lens;
+  const int32_t *h_block_table;  /* host mirror; NULL skips block-id validation */
+  float *d_hidden;               /* device [n_tokens][d_model] fp32, in/out */
+  int layer_begin, layer_end;
+} bullet_batch;
+
+/* Batch shape for the performance model (host arrays). */
+typedef struct {
+  int n_reqs;
+  const int32_t *q_lens;         /* new tokens per request */
+  const int32_t *ctx_lens;       /* cached tokens per request */
+} bullet_batch_shape;
+
+/* Scheduler state S_k = (P_k, D_k, R_k), P:L193 (§3.3.2); host arrays. */
+typedef struct {
+  int layers_done, total_layers;          /* l_k, total_layers (Alg. 1 l.3) */
+  int n_prefill;                          /* running prefill requests */
+  const int32_t *prefill_lens;
+  const double *prefill_waited_ms;        /* q_i */
+  int n_pending;                          /* w_k */
+  const int32_t *pending_lens;
+  const double *pending_waited_ms;
+  int n_decode;                           /* n_d */
+  const int32_t *decode_tokens;           /* o_i: tokens generated so far */
+  const double *decode_elapsed_ms;        /* d_i: decode time so far */
+  double decode_mean_ctx;
+  int u_k, v_k;                           /* current prefill / decode SMs */
+} bullet_sched_state;
+
+/* SLOs (Table 2) and search bounds. */
+typedef struct {
+  double ttft_norm_ms_per_tok;   /* normalized TTFT: Gamma_ttft(r) = value * input_len_r */
+  double tpot_ms;
+  int w_max;                     /* W_max, Alg. 1 l.18 */
+  int v_min;                     /* minimum decode SMs when co-running */
+  double percentile;             /* 0.9 (Alg. 1 "P90") */
+} bullet_slo;
+
+/* Create a handle on the current CUDA device.  Probes the live SM ids
+ * (%smid) and orders them (sigma).  `nccl_uids`: for tp_size > 1, 2 x 128
+ * bytes (ncclUniqueId of the prefill and the decode communicator, same on
+ * every rank), else NULL.  `perf_params_json`: fitted perf-model
+ * parameters, or NULL for the unfitted roofline (d = p = 1).
+ * Unsupported shapes (BULLET_EUNSUPPORTED): bf16 with d_model, H*hd or d_ff
+ * not multiples of 64; (H+2Hkv)*hd, d_model or d_ff not multiples of 64;
+ * head_dim != 128 for bf16 (64 or 128 for fp32); block_size not in {16}. */
+int bullet_create(const bullet_model_cfg *cfg, const bullet_kv_pool *pool,
+                  const void *nccl_uids, const char *perf_params_json,
+                  bullet_handle **out);
+
+/* Host-only handle for the performance model (no GPU, no allocations):
+ * bullet_model_predict and bullet_choose_split behave as on a full handle
+ * with N = n_sms SMs; every GPU call on it returns BULLET_EUNSUPPORTED.
+ * For planning on a host without a GPU and for CPU tests. */
+int bullet_perf_create(const bullet_model_cfg *cfg, int n_sms, const char *perf_params_json,
+                       bullet_handle **out);
+
+/* Register the weights of one layer (pointers are kept, not copied). */
+int bullet_set_layer_weights(bullet_handle *h, int layer, const bullet_layer_weights *w);
+
+/* SM count N of the device and the split granularity (2 = one TPC). */
+int bullet_num_sms(const bullet_handle *h, int *n_sms, int *granularity);
+
+/* Copy the probed ordered SM list sigma (host int32 [N]) — prefill gets
+ * sigma[0:p), decode sigma[p:N) for prefill_sm_count p. */
+int bullet_sm_order(const bullet_handle *h, int32_t *h_sigma, int cap);
+
+/* One layer step: the prefill batch runs its layers on stream s_prefill and
+ * the decode batch runs its layers on stream s_decode.  With BULLET_CORUN
+ * every kernel of the prefill phase claims work only on the first
+ * prefill_sm_count SMs of sigma and every decode kernel only on the rest
+ * (smid-gated persistent kernels; replaces libsmctrl masks over MPS,
+ * P:L212).  prefill_sm_count = N pauses decode; 0 requires an empty
+ * prefill.  Either batch may be NULL.  Asynchronous: enqueue only.
+ * Errors: EINVAL (shapes), ESMRANGE (split), EKV (block table), ENOMEM
+ * (batch larger than cfg max_*). */
+int bullet_step(bullet_handle *h, const bullet_batch *prefill, const bullet_batch *decode,
+                int prefill_sm_count, int flags, void *s_prefill, void *s_decode);
+
+/* Eq. 2 / T_m: predicted time (microseconds) of one layer of the given
+ * batch on sm_count SMs; corun_sm_count > 0 applies the co-location factors
+ * p_c, p_b. */
+int bullet_model_predict(const bullet_handle *h, const bullet_batch_shape *shape, int sm_count,
+                         int corun_sm_count, double *t_layer_us);
+
+/* Alg. 1 and the §3.3.3 search under the readings
+ * of DESIGN.md §3 (R-14..R-17): returns the prefill SM count for the next
+ * cycle (N = decode paused) and the number of decode layer-steps to co-run
+ * with one prefill layer-step. */
+int bullet_choose_split(const bullet_handle *h, const bullet_sched_state *s, const bullet_slo *slo,
+                        int *prefill_sm_count, int *decode_layer_steps);
+
+/* Device buffer for the smid log used with BULLET_SMID_LOG: int32
+ * [1 + 4*capacity]; entry i = {launch_id, unit, smid, phase}; element 0 is
+ * the entry counter (caller zeroes it).  NULL disables. */
+int bullet_set_smid_log(bullet_handle *h, int32_t *d_log, int capacity);
+
+/* Block until all work the handle enqueued has finished; surfaces
+ * asynchronous CUDA / NCCL errors. */
+int bullet_sync(bullet_handle *h);
+
+/* ncclGetUniqueId into out (128 bytes), for tensor-parallel setup. */
+int bullet_nccl_unique_id(void *out128);
+
+const char *bullet_last_error(void);
+void bullet_destroy(bullet_handle *h);
+
+/* ---- op-level entry points (the same kernels bullet_step launches), for
+ * per-kernel parity tests.  All run on `stream` over the SMs of sigma[lo:hi)
+ * (lo = 0, hi = N for the whole GPU). ---- */
+
+/* C = A B^T with the epilogue `epi` (bf16 A [M][K], B [rowsB][K] for
+ * BULLET_DTYPE_BF16 handles; fp32 otherwise):
+ *   0 F32:      out_f32[M][N] = acc (+ bias[N])                (QKV)
+ *   1 RESID:    out_f32[M][N] = resid[M][N] + acc (in place OK) (O-proj, down)
+ *   2 SILU_MUL: out[M][N/2] = silu(acc[:, j]) * acc[:, silu_half + ... ]:
+ *               B rows [0, N/2) gate, [silu_half, silu_half + N/2) up;
+ *               out of dtype                                    (gate_up)
+ * N = number of B rows used (2 x output columns for SILU_MUL). */
+int bullet_op_gemm(bullet_handle *h, int epi, const void *d_A, int M, int K, const void *d_B,
+                   int N, int silu_half, const void *d_bias, const float *d_resid, void *d_out,
+                   int lo, int hi, void *stream);
+
+int bullet_op_rmsnorm(bullet_handle *h, const float *d_x, int n, const void *d_g, void *d_out,
+                      int lo, int hi, void *stream);
+
+/* RoPE + KV append for `batch` rows: qkv fp32 [n_tokens][(H+2Hkv)*hd] in,
+ * q out [n_tokens][H*hd] (dtype), k/v written to the pool of `layer`. */
+int bullet_op_rope_kv(bullet_handle *h, const bullet_batch *batch, int layer, const float *d_qkv,
+                      void *d_q, int lo, int hi, void *stream);
+
+/* Attention for `batch` rows reading K/V of `layer` through the block
+ * table: q [n_tokens][H*hd] in, o [n_tokens][H*hd] out (dtype).
+ * kind 0: automatic (what bullet_step uses), 1: SIMT kernel, 2: tensor-core
+ * prefill kernel (bf16 only). */
+int bullet_op_attention(bullet_handle *h, const bullet_batch *batch, int layer, const void *d_q,
+                        void *d_o, int kind, int lo, int hi, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BULLET_H */

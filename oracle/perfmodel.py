@@ -130,7 +130,7 @@ def evaluate_split(P, model, state, slo, u, v):
     N, L, lk = P["M"], state["total_layers"], state["layers_done"]
     pre = _phase_shape(model, state["prefill_lens"], [0] * len(state["prefill_lens"]))
     dec = _phase_shape(model, [1] * len(state["decode_tokens"]),
-                       [int(round(state["decode_mean_ctx"]))] * len(state["decode_tokens"]))
+                       [int(math.floor(state["decode_mean_ctx"] + 0.5))] * len(state["decode_tokens"]))
     ms = 1e3
     t_p = layer_time(pre, P, u, v) * ms if state["prefill_lens"] else 0.0
     rem = t_p * (L - lk)                                   # Alg. 1 line 3
@@ -204,7 +204,7 @@ def choose_split(P, model, state, slo, gran=2):
     u = N - v
     t_p = ev[v][2]
     t_d = layer_time(_phase_shape(model, [1] * len(state["decode_tokens"]),
-                                  [int(round(state["decode_mean_ctx"]))] * len(state["decode_tokens"])),
+                                  [int(math.floor(state["decode_mean_ctx"] + 0.5))] * len(state["decode_tokens"])),
                      P, v, u) * 1e3
     k = max(1, int(math.floor(t_p / t_d + 0.5))) if t_d > 0 else 1   # A9: decode steps per prefill layer
     return u, k
@@ -224,6 +224,6 @@ def default_params(M=148, C_tflops=1649.5, B_gbs=6549.4):
         "d_c": {"m": [1, M], "v": [1.0, 1.0]}, "d_b": {"m": [1, M], "v": [1.0, 1.0]},
         "p_c": 1.0, "p_b": 1.0,
         "tiles": {"gemm_bm": 128, "gemm_bn": 256, "gemm_bk": 64, "min_k_blocks": 4,
-                  "attn_bq": 128, "rows_per_unit": 8},
+                  "attn_bq": 64, "rows_per_unit": 8},
         "occ": {"gemm": 1, "attn": 1, "elem": 4},
     }

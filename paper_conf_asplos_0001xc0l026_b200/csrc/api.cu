@@ -1,0 +1,732 @@
+// api.cu — the C ABI of include/bullet.h: handle, validation, per-step
+// planning, kernel launches on the two phase streams, SM gating, perf model
+// and split decision entry points, NCCL tensor parallelism.
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <set>
+#include <string>
+#include <vector>
+
+#include "bullet.h"
+#include "kernels.h"
+#include "perfmodel.h"
+
+using namespace bl;
+
+namespace {
+
+thread_local std::string g_err;
+
+int set_err(int code, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return code;
+}
+
+#define CK(x)                                                                           \
+  do {                                                                                  \
+    cudaError_t e_ = (x);                                                               \
+    if (e_ != cudaSuccess)                                                              \
+      return set_err(BULLET_ECUDA, "%s: %s (%s:%d)", #x, cudaGetErrorString(e_), __FILE__, \
+                     __LINE__);                                                         \
+  } while (0)
+
+// ---------------------------------------------------------------- NCCL (dlopen)
+struct Nccl {
+  void* lib = nullptr;
+  ncclResult_t (*getUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*commInitRankConfig)(ncclComm_t*, int, ncclUniqueId, int, ncclConfig_t*) = nullptr;
+  ncclResult_t (*allReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                            cudaStream_t) = nullptr;
+  ncclResult_t (*commDestroy)(ncclComm_t) = nullptr;
+  const char* (*errStr)(ncclResult_t) = nullptr;
+  bool load() {
+    if (lib) return true;
+    const char* env = getenv("BULLET_NCCL_LIB");
+    lib = dlopen(env ? env : "libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!lib) return false;
+    getUniqueId = (decltype(getUniqueId))dlsym(lib, "ncclGetUniqueId");
+    commInitRankConfig = (decltype(commInitRankConfig))dlsym(lib, "ncclCommInitRankConfig");
+    allReduce = (decltype(allReduce))dlsym(lib, "ncclAllReduce");
+    commDestroy = (decltype(commDestroy))dlsym(lib, "ncclCommDestroy");
+    errStr = (decltype(errStr))dlsym(lib, "ncclGetErrorString");
+    return getUniqueId && commInitRankConfig && allReduce && commDestroy && errStr;
+  }
+} g_nccl;
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+EncodeTiledFn g_encode = nullptr;
+
+int get_encode() {
+  if (g_encode) return BULLET_OK;
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  CK(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
+  if (!fn || q != cudaDriverEntryPointSuccess)
+    return set_err(BULLET_ECUDA, "cuTensorMapEncodeTiled unavailable");
+  g_encode = (EncodeTiledFn)fn;
+  return BULLET_OK;
+}
+
+// 2D bf16 K-major operand [rows][K], box {64, box_rows}, 128-byte swizzle.
+int make_map(CUtensorMap* m, const void* ptr, int rows, int K, int box_rows) {
+  cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)K * 2};
+  cuuint32_t box[2] = {64, (cuuint32_t)box_rows};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = g_encode(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims,
+                        strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                        CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_err(BULLET_ECUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  return BULLET_OK;
+}
+
+struct PhaseWS {
+  float* qkv = nullptr;
+  void *q = nullptr, *o = nullptr, *h = nullptr, *act = nullptr;
+  float* partials = nullptr;
+  size_t partial_floats = 0;
+  int* tile_sems = nullptr;
+  int* counters = nullptr;
+  int n_counters = 0, next_ctr = 0;
+  int2* tiles = nullptr;
+  int* n_tiles = nullptr;
+  int max_tok = 0;
+};
+
+constexpr int GRAN = 2;            // split granularity: one TPC
+constexpr int N_TILE_SEMS = 2048;
+
+}  // namespace
+
+struct bullet_handle {
+  bullet_model_cfg cfg;
+  int dev = 0, n_sms = 0, elt = 2;
+  std::vector<int> sigma;
+  std::vector<bullet_layer_weights> w;
+  std::vector<char> w_set;
+  std::vector<void*> pk, pv;
+  int n_blocks = 0, block_size = 0;
+  float2* rope_cs = nullptr;
+  PhaseWS ph[2];
+  int* op_ctr = nullptr;
+  int32_t* log = nullptr;
+  int log_cap = 0;
+  int launch_seq = 0;
+  PerfParams perf;
+  ncclComm_t comm[2] = {nullptr, nullptr};
+  cudaEvent_t ev_ts = nullptr;
+  bool host_only = false;  // bullet_perf_create: perf model only
+};
+
+namespace {
+
+Gate gate_of(const bullet_handle* h, int lo, int hi) {
+  Gate g;
+  memset(&g, 0, sizeof g);
+  for (int i = lo; i < hi; ++i) {
+    const int s = h->sigma[i];
+    g.m[s >> 5] |= 1u << (s & 31);
+  }
+  return g;
+}
+
+struct Ctx {  // one phase's launch context within a call
+  bullet_handle* h;
+  int phase;
+  Gate gate;
+  int m_sms;
+  bool log;
+  cudaStream_t st;
+  bool op;     // op-level entry: counter = op_ctr, zeroed before each launch
+};
+
+int next_launch(Ctx& c, Launch* L) {
+  memset(L, 0, sizeof *L);
+  L->gate = c.gate;
+  L->log = c.log ? c.h->log : nullptr;
+  L->log_cap = c.h->log_cap;
+  L->launch_id = c.h->launch_seq++;
+  L->phase = c.phase;
+  if (c.op) {
+    CK(cudaMemsetAsync(c.h->op_ctr, 0, sizeof(int), c.st));
+    L->ctr = c.h->op_ctr;
+  } else {
+    PhaseWS& P = c.h->ph[c.phase];
+    if (P.next_ctr >= P.n_counters) return set_err(BULLET_ENOMEM, "work counters exhausted");
+    L->ctr = P.counters + P.next_ctr++;
+  }
+  return BULLET_OK;
+}
+
+int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, int silu_half,
+            const void* bias, const float* resid, void* out, int ldo) {
+  bullet_handle* h = c.h;
+  if (M == 0) return BULLET_OK;
+  GemmArgs a;
+  memset(&a, 0, sizeof a);
+  a.M = M; a.N = N; a.K = K; a.epi = epi; a.silu_half = silu_half; a.bias = bias;
+  a.resid = resid; a.ldo = ldo;
+  if (epi == EPI_SILU) a.out_t = out; else a.out_f32 = (float*)out;
+  int rc = next_launch(c, &a.L);
+  if (rc) return rc;
+  if (h->cfg.dtype == BULLET_DTYPE_FP32) {
+    if (K % 16) return set_err(BULLET_EUNSUPPORTED, "fp32 GEMM needs K %% 16 == 0");
+    a.bn = 64; a.splits = 1;
+    CK(launch_gemm_simt<float>((const float*)A, (const float*)B, a, h->n_sms * 4, c.st));
+    return BULLET_OK;
+  }
+  if (K % 64) return set_err(BULLET_EUNSUPPORTED, "GEMM needs K %% 64 == 0 (K=%d)", K);
+  const int m_tiles = (M + 127) / 128;
+  auto fits = [&](int bn) { return epi == EPI_SILU ? ((N / 2) % (bn / 2) == 0 && N % 2 == 0) : (N % bn == 0); };
+  int bn = 0;
+  if (fits(256) && m_tiles * (N / 256) >= c.m_sms) bn = 256;
+  else if (fits(128)) bn = 128;
+  else if (fits(64)) bn = 64;
+  else if (fits(256)) bn = 256;
+  if (!bn) return set_err(BULLET_EUNSUPPORTED, "GEMM N=%d not tileable", N);
+  const int tiles = m_tiles * (N / bn);
+  const int k_blocks = K / 64;
+  int splits = 1;
+  if (tiles < c.m_sms) {
+    splits = (c.m_sms + tiles - 1) / tiles;
+    splits = std::min(splits, std::max(1, k_blocks / 4));
+    while (splits > 1 && ((size_t)tiles * splits * 128 * bn > h->ph[c.phase].partial_floats ||
+                          tiles > N_TILE_SEMS))
+      --splits;
+  }
+  a.bn = bn; a.splits = splits;
+  a.partials = h->ph[c.phase].partials;
+  a.tile_sems = h->ph[c.phase].tile_sems;
+  CUtensorMap ma, mb;
+  if ((rc = make_map(&ma, A, M, K, 128))) return rc;
+  if ((rc = make_map(&mb, B, N, K, bn / 2))) return rc;
+  CK(launch_gemm_tc(ma, mb, a, h->n_sms, c.st));
+  return BULLET_OK;
+}
+
+int do_rmsnorm(Ctx& c, const float* x, int n, const void* g, void* out) {
+  if (n == 0) return BULLET_OK;
+  NormArgs a;
+  a.x = x; a.g = g; a.out = out; a.n = n; a.d = c.h->cfg.d_model; a.eps = c.h->cfg.rms_eps;
+  int rc = next_launch(c, &a.L);
+  if (rc) return rc;
+  if (c.h->cfg.dtype == BULLET_DTYPE_FP32) CK(launch_rmsnorm<float>(a, c.h->n_sms * 8, c.st));
+  else CK(launch_rmsnorm<__nv_bfloat16>(a, c.h->n_sms * 8, c.st));
+  return BULLET_OK;
+}
+
+int do_rope(Ctx& c, const bullet_batch* b, int layer, const float* qkv, void* q) {
+  bullet_handle* h = c.h;
+  if (b->n_tokens == 0) return BULLET_OK;
+  RopeArgs a;
+  a.qkv = qkv; a.q_out = q; a.pool_k = h->pk[layer]; a.pool_v = h->pv[layer]; a.cs = h->rope_cs;
+  a.cu = b->d_cu_seqlens; a.ctx = b->d_ctx_lens; a.bt = b->d_block_table;
+  a.n_reqs = b->n_reqs; a.max_blocks = b->max_blocks_per_req; a.n_tok = b->n_tokens;
+  a.H = h->cfg.n_heads; a.Hkv = h->cfg.n_kv_heads; a.hd = h->cfg.head_dim; a.B = h->block_size;
+  a.max_pos = h->cfg.max_position;
+  int rc = next_launch(c, &a.L);
+  if (rc) return rc;
+  if (h->cfg.dtype == BULLET_DTYPE_FP32) CK(launch_rope_kv<float>(a, h->n_sms * 8, c.st));
+  else CK(launch_rope_kv<__nv_bfloat16>(a, h->n_sms * 8, c.st));
+  return BULLET_OK;
+}
+
+int max_qlen(const bullet_batch* b) {
+  int mq = 0;
+  for (int r = 0; r < b->n_reqs; ++r) mq = std::max(mq, b->h_cu_seqlens[r + 1] - b->h_cu_seqlens[r]);
+  return mq;
+}
+
+int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* o, int kind) {
+  bullet_handle* h = c.h;
+  if (b->n_tokens == 0) return BULLET_OK;
+  AttnArgs a;
+  memset(&a, 0, sizeof a);
+  a.q = q; a.o = o; a.pool_k = h->pk[layer]; a.pool_v = h->pv[layer];
+  a.cu = b->d_cu_seqlens; a.ctx = b->d_ctx_lens; a.bt = b->d_block_table;
+  a.n_reqs = b->n_reqs; a.max_blocks = b->max_blocks_per_req; a.n_tok = b->n_tokens;
+  a.H = h->cfg.n_heads; a.Hkv = h->cfg.n_kv_heads; a.hd = h->cfg.head_dim; a.B = h->block_size;
+  a.scale = (float)(1.0 / std::sqrt((double)a.hd));
+  const bool bf16 = h->cfg.dtype == BULLET_DTYPE_BF16;
+  if (kind == 0) kind = (bf16 && a.hd == 128 && max_qlen(b) > 1) ? 2 : 1;
+  if (kind == 2) {
+    if (!bf16 || a.hd != 128) return set_err(BULLET_EUNSUPPORTED, "tensor-core attention: bf16, hd 128 only");
+    PhaseWS& P = h->ph[c.phase];
+    a.tiles = P.tiles; a.n_tiles = P.n_tiles;
+    if (c.op) {  // op-level: plan the tile list now
+      PlanArgs pa{nullptr, 0, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ, P.tiles, P.n_tiles};
+      CK(launch_plan(pa, c.st));
+    }
+    int rc = next_launch(c, &a.L);
+    if (rc) return rc;
+    CK(launch_attn_prefill_tc(a, h->n_sms * 2, c.st));
+    return BULLET_OK;
+  }
+  int rc = next_launch(c, &a.L);
+  if (rc) return rc;
+  if (bf16) CK(launch_attn_simt<__nv_bfloat16>(a, h->n_sms * 4, c.st));
+  else CK(launch_attn_simt<float>(a, h->n_sms * 4, c.st));
+  return BULLET_OK;
+}
+
+int allreduce(Ctx& c, float* buf, size_t count) {
+  bullet_handle* h = c.h;
+  ncclResult_t r = g_nccl.allReduce(buf, buf, count, ncclFloat32, ncclSum, h->comm[c.phase], c.st);
+  if (r != ncclSuccess) return set_err(BULLET_ENCCL, "ncclAllReduce: %s", g_nccl.errStr(r));
+  return BULLET_OK;
+}
+
+// One decoder layer of one phase (DESIGN.md §2 steps S1-S9).
+int run_layer(Ctx& c, const bullet_batch* b, int layer) {
+  bullet_handle* h = c.h;
+  PhaseWS& P = h->ph[c.phase];
+  const bullet_layer_weights& w = h->w[layer];
+  const bullet_model_cfg& cf = h->cfg;
+  const int n = b->n_tokens, d = cf.d_model, H = cf.n_heads, Hkv = cf.n_kv_heads, hd = cf.head_dim;
+  const int I = cf.d_ff, nq = (H + 2 * Hkv) * hd;
+  const bool tp = cf.tp_size > 1, lead = cf.tp_rank == 0;
+  int rc;
+  if ((rc = do_rmsnorm(c, b->d_hidden, n, w.g_attn, P.h))) return rc;                       // S1
+  if ((rc = do_gemm(c, EPI_F32, P.h, n, d, w.w_qkv, nq, 0, w.b_qkv, nullptr, P.qkv, nq))) return rc;  // S2
+  if ((rc = do_rope(c, b, layer, P.qkv, P.q))) return rc;                                    // S3
+  if ((rc = do_attention(c, b, layer, P.q, P.o, 0))) return rc;                             // S4
+  // S5: x1 = x + o W_o^T.  Under TP the non-lead ranks write their partial
+  // into hidden and the fp32 all-reduce restores x + sum of partials (S9).
+  if ((rc = do_gemm(c, (!tp || lead) ? EPI_RESID : EPI_F32, P.o, n, H * hd, w.w_o, d, 0, nullptr,
+                    b->d_hidden, b->d_hidden, d))) return rc;
+  if (tp && (rc = allreduce(c, b->d_hidden, (size_t)n * d))) return rc;
+  if ((rc = do_rmsnorm(c, b->d_hidden, n, w.g_mlp, P.h))) return rc;                        // S6
+  if ((rc = do_gemm(c, EPI_SILU, P.h, n, d, w.w_gate_up, 2 * I, I, nullptr, nullptr, P.act, I))) return rc;  // S7
+  if ((rc = do_gemm(c, (!tp || lead) ? EPI_RESID : EPI_F32, P.act, n, I, w.w_down, d, 0, nullptr,
+                    b->d_hidden, b->d_hidden, d))) return rc;                                // S8
+  if (tp && (rc = allreduce(c, b->d_hidden, (size_t)n * d))) return rc;
+  return BULLET_OK;
+}
+
+int validate_batch(const bullet_handle* h, const bullet_batch* b, int phase) {
+  const char* nm = phase == 0 ? "prefill" : "decode";
+  if (b->n_reqs < 0 || b->n_tokens < 0) return set_err(BULLET_EINVAL, "%s: negative sizes", nm);
+  if (b->n_tokens == 0) return BULLET_OK;
+  if (!b->h_cu_seqlens || !b->h_ctx_lens || !b->d_cu_seqlens || !b->d_ctx_lens ||
+      !b->d_block_table || !b->d_hidden)
+    return set_err(BULLET_EINVAL, "%s: null pointer in batch", nm);
+  if (b->h_cu_seqlens[0] != 0 || b->h_cu_seqlens[b->n_reqs] != b->n_tokens)
+    return set_err(BULLET_EINVAL, "%s: cu_seqlens must run 0..n_tokens", nm);
+  if (b->n_tokens > h->ph[phase].max_tok)
+    return set_err(BULLET_ENOMEM, "%s: %d tokens > max %d", nm, b->n_tokens, h->ph[phase].max_tok);
+  if (b->layer_begin < 0 || b->layer_end > h->cfg.n_layers || b->layer_begin > b->layer_end)
+    return set_err(BULLET_EINVAL, "%s: layer range [%d,%d)", nm, b->layer_begin, b->layer_end);
+  for (int l = b->layer_begin; l < b->layer_end; ++l)
+    if (!h->w_set[l]) return set_err(BULLET_EINVAL, "%s: weights of layer %d not set", nm, l);
+  if (b->max_blocks_per_req <= 0) return set_err(BULLET_EINVAL, "%s: max_blocks_per_req", nm);
+  for (int r = 0; r < b->n_reqs; ++r) {
+    const int q = b->h_cu_seqlens[r + 1] - b->h_cu_seqlens[r], cx = b->h_ctx_lens[r];
+    if (q < 0 || cx < 0) return set_err(BULLET_EINVAL, "%s: request %d negative length", nm, r);
+    if (q == 0) continue;
+    if (cx + q > b->max_blocks_per_req * h->block_size)
+      return set_err(BULLET_EKV, "%s: request %d needs %d tokens > block table %d", nm, r, cx + q,
+                     b->max_blocks_per_req * h->block_size);
+    if (cx + q > h->cfg.max_position)
+      return set_err(BULLET_EINVAL, "%s: request %d position %d >= max_position", nm, r, cx + q - 1);
+    if (b->h_block_table) {
+      const int nb = (cx + q + h->block_size - 1) / h->block_size;
+      for (int i = 0; i < nb; ++i) {
+        const int blk = b->h_block_table[(size_t)r * b->max_blocks_per_req + i];
+        if (blk < 0 || blk >= h->n_blocks)
+          return set_err(BULLET_EKV, "%s: request %d block %d id %d out of [0,%d)", nm, r, i, blk, h->n_blocks);
+      }
+    }
+  }
+  return BULLET_OK;
+}
+
+int run_phase(Ctx& c, const bullet_batch* b) {
+  PhaseWS& P = c.h->ph[c.phase];
+  P.next_ctr = 0;
+  const bool tc_attn = c.h->cfg.dtype == BULLET_DTYPE_BF16 && c.h->cfg.head_dim == 128 && max_qlen(b) > 1;
+  PlanArgs pa{P.counters, P.n_counters, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ,
+              tc_attn ? P.tiles : nullptr, P.n_tiles};
+  CK(launch_plan(pa, c.st));
+  for (int l = b->layer_begin; l < b->layer_end; ++l) {
+    int rc = run_layer(c, b, l);
+    if (rc) return rc;
+  }
+  return BULLET_OK;
+}
+
+}  // namespace
+
+// ================================================================== C ABI
+extern "C" {
+
+const char* bullet_last_error(void) { return g_err.c_str(); }
+
+int bullet_nccl_unique_id(void* out128) {
+  if (!out128) return set_err(BULLET_EINVAL, "null");
+  if (!g_nccl.load()) return set_err(BULLET_ENCCL, "libnccl.so.2 not loadable: %s", dlerror());
+  ncclUniqueId id;
+  ncclResult_t r = g_nccl.getUniqueId(&id);
+  if (r != ncclSuccess) return set_err(BULLET_ENCCL, "ncclGetUniqueId: %s", g_nccl.errStr(r));
+  memcpy(out128, &id, sizeof id);
+  return BULLET_OK;
+}
+
+int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const void* nccl_uids,
+                  const char* perf_params_json, bullet_handle** out) {
+  if (!cfg || !pool || !out) return set_err(BULLET_EINVAL, "null argument");
+  *out = nullptr;
+  const bullet_model_cfg& c = *cfg;
+  if (c.n_layers <= 0 || c.d_model <= 0 || c.n_heads <= 0 || c.n_kv_heads <= 0 || c.head_dim <= 0 ||
+      c.d_ff <= 0 || c.n_heads % c.n_kv_heads || c.max_position <= 0 || c.tp_size <= 0 ||
+      c.tp_rank < 0 || c.tp_rank >= c.tp_size || c.max_prefill_tokens < 0 || c.max_decode_tokens < 0)
+    return set_err(BULLET_EINVAL, "invalid model cfg");
+  if (c.dtype != BULLET_DTYPE_BF16 && c.dtype != BULLET_DTYPE_FP32)
+    return set_err(BULLET_EINVAL, "dtype");
+  if (c.d_model % 64 || c.d_ff % 64 || (c.n_heads * c.head_dim) % 64 ||
+      ((c.n_heads + 2 * c.n_kv_heads) * c.head_dim) % 64)
+    return set_err(BULLET_EUNSUPPORTED, "dims must be multiples of 64");
+  if (c.head_dim != 128 && c.head_dim != 64) return set_err(BULLET_EUNSUPPORTED, "head_dim 64/128");
+  if (c.n_heads / c.n_kv_heads > 8) return set_err(BULLET_EUNSUPPORTED, "GQA group > 8");
+  if (pool->block_size != 16) return set_err(BULLET_EUNSUPPORTED, "block_size must be 16");
+  if (pool->n_blocks <= 0 || !pool->d_k || !pool->d_v) return set_err(BULLET_EINVAL, "kv pool");
+  if (c.tp_size > 1 && !nccl_uids) return set_err(BULLET_EINVAL, "tp_size > 1 needs nccl_uids");
+
+  int dev;
+  CK(cudaGetDevice(&dev));
+  cudaDeviceProp prop;
+  CK(cudaGetDeviceProperties(&prop, dev));
+  if (prop.major != 10) return set_err(BULLET_EUNSUPPORTED, "needs an sm_100 (Blackwell) GPU, got sm_%d%d", prop.major, prop.minor);
+  int rc = get_encode();
+  if (rc) return rc;
+
+  bullet_handle* h = new bullet_handle();
+  h->cfg = c;
+  h->dev = dev;
+  h->n_sms = prop.multiProcessorCount;
+  h->elt = c.dtype == BULLET_DTYPE_BF16 ? 2 : 4;
+  h->w.resize(c.n_layers);
+  h->w_set.assign(c.n_layers, 0);
+  h->n_blocks = pool->n_blocks;
+  h->block_size = pool->block_size;
+  for (int l = 0; l < c.n_layers; ++l) {
+    if (!pool->d_k[l] || !pool->d_v[l]) { delete h; return set_err(BULLET_EINVAL, "pool layer %d null", l); }
+    h->pk.push_back(pool->d_k[l]);
+    h->pv.push_back(pool->d_v[l]);
+  }
+  auto fail = [&](int code) { bullet_destroy(h); return code; };
+
+  // ---- SM probe (KI1): the live %smid set, sorted (TPC pairs adjacent)
+  {
+    const int n = h->n_sms * 16;
+    int* d_ids = nullptr;
+    if (cudaMalloc(&d_ids, n * sizeof(int)) != cudaSuccess) return fail(set_err(BULLET_ENOMEM, "probe"));
+    std::vector<int> ids(n);
+    cudaError_t e = launch_probe(d_ids, n, 0);
+    if (e == cudaSuccess) e = cudaMemcpy(ids.data(), d_ids, n * sizeof(int), cudaMemcpyDeviceToHost);
+    cudaFree(d_ids);
+    if (e != cudaSuccess) return fail(set_err(BULLET_ECUDA, "SM probe: %s", cudaGetErrorString(e)));
+    std::set<int> s(ids.begin(), ids.end());
+    h->sigma.assign(s.begin(), s.end());
+    if ((int)h->sigma.size() != h->n_sms || h->sigma.back() >= 256)
+      return fail(set_err(BULLET_ECUDA, "SM probe found %zu of %d SMs (max id %d)", h->sigma.size(),
+                          h->n_sms, h->sigma.empty() ? -1 : h->sigma.back()));
+  }
+
+  // ---- RoPE (cos, sin) table, computed in fp64 then stored fp32
+  {
+    const int half = c.head_dim / 2;
+    std::vector<double> inv(half);
+    for (int i = 0; i < half; ++i) {
+      double f = std::pow(c.rope_theta, -2.0 * i / c.head_dim);
+      if (c.rope_llama3) {  // llama3 band rescaling (public Llama-3.1 config)
+        const double L = c.rope_orig_max_pos, wl = 2.0 * M_PI / f;
+        const double hi_w = L / c.rope_high_freq, lo_w = L / c.rope_low_freq;
+        if (wl > lo_w) f /= c.rope_factor;
+        else if (wl >= hi_w) {
+          const double sm = (L / wl - c.rope_low_freq) / (c.rope_high_freq - c.rope_low_freq);
+          f = (1.0 - sm) * f / c.rope_factor + sm * f;
+        }
+      }
+      inv[i] = f;
+    }
+    std::vector<float2> cs((size_t)c.max_position * half);
+    for (int p = 0; p < c.max_position; ++p)
+      for (int i = 0; i < half; ++i) {
+        const double t = (double)p * inv[i];
+        cs[(size_t)p * half + i] = make_float2((float)std::cos(t), (float)std::sin(t));
+      }
+    if (cudaMalloc(&h->rope_cs, cs.size() * sizeof(float2)) != cudaSuccess ||
+        cudaMemcpy(h->rope_cs, cs.data(), cs.size() * sizeof(float2), cudaMemcpyHostToDevice) != cudaSuccess)
+      return fail(set_err(BULLET_ENOMEM, "rope table"));
+  }
+
+  // ---- per-phase workspace
+  const int nq = (c.n_heads + 2 * c.n_kv_heads) * c.head_dim;
+  for (int p = 0; p < 2; ++p) {
+    PhaseWS& P = h->ph[p];
+    P.max_tok = p == 0 ? c.max_prefill_tokens : c.max_decode_tokens;
+    const size_t T = std::max(1, P.max_tok);
+    P.n_counters = 8 * c.n_layers + 16;
+    P.partial_floats = (size_t)2 * h->n_sms * 128 * 256;
+    bool ok = cudaMalloc(&P.qkv, T * nq * sizeof(float)) == cudaSuccess &&
+              cudaMalloc(&P.q, T * c.n_heads * c.head_dim * h->elt) == cudaSuccess &&
+              cudaMalloc(&P.o, T * c.n_heads * c.head_dim * h->elt) == cudaSuccess &&
+              cudaMalloc(&P.h, T * c.d_model * h->elt) == cudaSuccess &&
+              cudaMalloc(&P.act, T * c.d_ff * h->elt) == cudaSuccess &&
+              cudaMalloc(&P.partials, P.partial_floats * sizeof(float)) == cudaSuccess &&
+              cudaMalloc(&P.tile_sems, N_TILE_SEMS * sizeof(int)) == cudaSuccess &&
+              cudaMalloc(&P.counters, P.n_counters * sizeof(int)) == cudaSuccess &&
+              cudaMalloc(&P.tiles, (T / ATTN_TC_BQ + 1024) * sizeof(int2)) == cudaSuccess &&
+              cudaMalloc(&P.n_tiles, sizeof(int)) == cudaSuccess;
+    if (!ok) return fail(set_err(BULLET_ENOMEM, "workspace allocation (phase %d)", p));
+    cudaMemset(P.tile_sems, 0, N_TILE_SEMS * sizeof(int));
+    cudaMemset(P.counters, 0, P.n_counters * sizeof(int));
+  }
+  if (cudaMalloc(&h->op_ctr, sizeof(int)) != cudaSuccess) return fail(set_err(BULLET_ENOMEM, "op ctr"));
+  if (cudaEventCreateWithFlags(&h->ev_ts, cudaEventDisableTiming) != cudaSuccess)
+    return fail(set_err(BULLET_ECUDA, "event"));
+  if (cudaDeviceSynchronize() != cudaSuccess) return fail(set_err(BULLET_ECUDA, "init sync"));
+
+  // ---- performance model parameters
+  h->perf.set_default(h->n_sms);
+  if (perf_params_json) {
+    std::string err;
+    if (!h->perf.parse(perf_params_json, &err)) return fail(set_err(BULLET_EINVAL, "%s", err.c_str()));
+  }
+
+  // ---- tensor parallelism: one communicator per phase (concurrent streams)
+  if (c.tp_size > 1) {
+    if (!g_nccl.load()) return fail(set_err(BULLET_ENCCL, "libnccl.so.2 not loadable"));
+    for (int p = 0; p < 2; ++p) {
+      ncclUniqueId id;
+      memcpy(&id, (const char*)nccl_uids + 128 * p, sizeof id);
+      ncclConfig_t conf = NCCL_CONFIG_INITIALIZER;
+      conf.maxCTAs = 16;  // NCCL kernels are not smid-gated: bound their footprint
+      ncclResult_t r = g_nccl.commInitRankConfig(&h->comm[p], c.tp_size, id, c.tp_rank, &conf);
+      if (r != ncclSuccess) return fail(set_err(BULLET_ENCCL, "ncclCommInitRankConfig: %s", g_nccl.errStr(r)));
+    }
+  }
+  *out = h;
+  return BULLET_OK;
+}
+
+int bullet_perf_create(const bullet_model_cfg* cfg, int n_sms, const char* json, bullet_handle** out) {
+  if (!cfg || !out || n_sms <= 0 || n_sms > 256) return set_err(BULLET_EINVAL, "bad argument");
+  if (cfg->n_heads <= 0 || cfg->n_kv_heads <= 0 || cfg->d_model <= 0 || cfg->head_dim <= 0 || cfg->d_ff <= 0)
+    return set_err(BULLET_EINVAL, "invalid model cfg");
+  bullet_handle* h = new bullet_handle();
+  h->cfg = *cfg;
+  h->host_only = true;
+  h->n_sms = n_sms;
+  h->elt = cfg->dtype == BULLET_DTYPE_BF16 ? 2 : 4;
+  for (int i = 0; i < n_sms; ++i) h->sigma.push_back(i);
+  h->perf.set_default(n_sms);
+  if (json) {
+    std::string err;
+    if (!h->perf.parse(json, &err)) { delete h; return set_err(BULLET_EINVAL, "%s", err.c_str()); }
+  }
+  *out = h;
+  return BULLET_OK;
+}
+
+int bullet_set_layer_weights(bullet_handle* h, int layer, const bullet_layer_weights* w) {
+  if (!h || !w) return set_err(BULLET_EINVAL, "null");
+  if (h->host_only) return set_err(BULLET_EUNSUPPORTED, "host-only handle");
+  if (layer < 0 || layer >= h->cfg.n_layers) return set_err(BULLET_EINVAL, "layer %d", layer);
+  if (!w->w_qkv || !w->w_o || !w->w_gate_up || !w->w_down || !w->g_attn || !w->g_mlp ||
+      (h->cfg.qkv_bias && !w->b_qkv))
+    return set_err(BULLET_EINVAL, "null weight pointer");
+  h->w[layer] = *w;
+  if (!h->cfg.qkv_bias) h->w[layer].b_qkv = nullptr;
+  h->w_set[layer] = 1;
+  return BULLET_OK;
+}
+
+int bullet_num_sms(const bullet_handle* h, int* n, int* g) {
+  if (!h) return set_err(BULLET_EINVAL, "null");
+  if (n) *n = h->n_sms;
+  if (g) *g = GRAN;
+  return BULLET_OK;
+}
+
+int bullet_sm_order(const bullet_handle* h, int32_t* out, int cap) {
+  if (!h || !out || cap < h->n_sms) return set_err(BULLET_EINVAL, "bad buffer");
+  for (int i = 0; i < h->n_sms; ++i) out[i] = h->sigma[i];
+  return BULLET_OK;
+}
+
+int bullet_set_smid_log(bullet_handle* h, int32_t* d_log, int capacity) {
+  if (!h) return set_err(BULLET_EINVAL, "null");
+  h->log = d_log;
+  h->log_cap = d_log ? capacity : 0;
+  return BULLET_OK;
+}
+
+int bullet_step(bullet_handle* h, const bullet_batch* pre, const bullet_batch* dec,
+                int prefill_sm_count, int flags, void* s_prefill, void* s_decode) {
+  if (!h) return set_err(BULLET_EINVAL, "null handle");
+  if (h->host_only) return set_err(BULLET_EUNSUPPORTED, "host-only handle");
+  const int N = h->n_sms, p = prefill_sm_count, mode = flags & 3;
+  if (mode == 3) return set_err(BULLET_EINVAL, "flags: TIMESLICED and UNGATED are exclusive");
+  if (p < 0 || p > N || (p % GRAN && p != N)) return set_err(BULLET_ESMRANGE, "prefill_sm_count %d not in [0,%d] step %d", p, N, GRAN);
+  const bool has_pre = pre && pre->n_tokens > 0, has_dec = dec && dec->n_tokens > 0;
+  int rc;
+  if (pre && (rc = validate_batch(h, pre, 0))) return rc;
+  if (dec && (rc = validate_batch(h, dec, 1))) return rc;
+  if (mode == BULLET_CORUN && has_pre && p == 0)
+    return set_err(BULLET_ESMRANGE, "prefill batch given with prefill_sm_count 0");
+  const bool run_dec = has_dec && !(mode == BULLET_CORUN && p == N);  // p = N: decode paused
+  if (h->log_cap == 0 && (flags & BULLET_SMID_LOG)) return set_err(BULLET_EINVAL, "SMID_LOG without a log buffer");
+  const bool log = (flags & BULLET_SMID_LOG) != 0;
+  cudaStream_t sp = (cudaStream_t)s_prefill, sd = (cudaStream_t)s_decode;
+  Ctx cp{h, 0, mode == BULLET_CORUN ? gate_of(h, 0, p) : gate_of(h, 0, N),
+         mode == BULLET_CORUN ? p : N, log, sp, false};
+  Ctx cd{h, 1, mode == BULLET_CORUN ? gate_of(h, p, N) : gate_of(h, 0, N),
+         mode == BULLET_CORUN ? N - p : N, log, sd, false};
+  if (has_pre && (rc = run_phase(cp, pre))) return rc;
+  if (run_dec) {
+    if (mode == BULLET_TIMESLICED && has_pre) {
+      CK(cudaEventRecord(h->ev_ts, sp));
+      CK(cudaStreamWaitEvent(sd, h->ev_ts, 0));
+    }
+    if ((rc = run_phase(cd, dec))) return rc;
+  }
+  return BULLET_OK;
+}
+
+static PhaseShape model_shape(const bullet_handle* h) {
+  PhaseShape s;
+  s.d = h->cfg.d_model; s.H = h->cfg.n_heads; s.Hkv = h->cfg.n_kv_heads; s.hd = h->cfg.head_dim;
+  s.I = h->cfg.d_ff; s.elt = h->elt;
+  return s;
+}
+
+int bullet_model_predict(const bullet_handle* h, const bullet_batch_shape* shape, int sm_count,
+                         int corun_sm_count, double* t_us) {
+  if (!h || !shape || !t_us || shape->n_reqs < 0) return set_err(BULLET_EINVAL, "null");
+  if (sm_count <= 0 || sm_count > h->n_sms || corun_sm_count < 0)
+    return set_err(BULLET_ESMRANGE, "sm_count %d", sm_count);
+  PhaseShape s = model_shape(h);
+  for (int i = 0; i < shape->n_reqs; ++i) {
+    s.q_lens.push_back(shape->q_lens[i]);
+    s.ctx_lens.push_back(shape->ctx_lens[i]);
+  }
+  *t_us = layer_time(s, h->perf, sm_count, corun_sm_count) * 1e6;
+  return BULLET_OK;
+}
+
+int bullet_choose_split(const bullet_handle* h, const bullet_sched_state* s, const bullet_slo* slo,
+                        int* prefill_sm_count, int* decode_layer_steps) {
+  if (!h || !s || !slo || !prefill_sm_count || !decode_layer_steps) return set_err(BULLET_EINVAL, "null");
+  if (slo->v_min < 1 || slo->v_min > h->n_sms || slo->percentile <= 0 || slo->percentile > 1)
+    return set_err(BULLET_EINVAL, "slo");
+  SchedState S;
+  S.layers_done = s->layers_done; S.total_layers = s->total_layers;
+  for (int i = 0; i < s->n_prefill; ++i) { S.prefill_lens.push_back(s->prefill_lens[i]); S.prefill_waited_ms.push_back(s->prefill_waited_ms[i]); }
+  for (int i = 0; i < s->n_pending; ++i) { S.pending_lens.push_back(s->pending_lens[i]); S.pending_waited_ms.push_back(s->pending_waited_ms[i]); }
+  for (int i = 0; i < s->n_decode; ++i) { S.decode_tokens.push_back(s->decode_tokens[i]); S.decode_elapsed_ms.push_back(s->decode_elapsed_ms[i]); }
+  S.decode_mean_ctx = s->decode_mean_ctx;
+  S.u_k = s->u_k; S.v_k = s->v_k;
+  Slo sl{slo->ttft_norm_ms_per_tok, slo->tpot_ms, slo->w_max, slo->v_min, slo->percentile};
+  PerfParams P = h->perf;
+  P.M = h->n_sms;
+  choose_split(P, model_shape(h), S, sl, GRAN, prefill_sm_count, decode_layer_steps);
+  return BULLET_OK;
+}
+
+int bullet_sync(bullet_handle* h) {
+  if (!h) return set_err(BULLET_EINVAL, "null");
+  if (h->host_only) return BULLET_OK;
+  CK(cudaDeviceSynchronize());
+  return BULLET_OK;
+}
+
+void bullet_destroy(bullet_handle* h) {
+  if (!h) return;
+  if (h->host_only) { delete h; return; }
+  cudaDeviceSynchronize();
+  for (int p = 0; p < 2; ++p) {
+    PhaseWS& P = h->ph[p];
+    cudaFree(P.qkv); cudaFree(P.q); cudaFree(P.o); cudaFree(P.h); cudaFree(P.act);
+    cudaFree(P.partials); cudaFree(P.tile_sems); cudaFree(P.counters); cudaFree(P.tiles);
+    cudaFree(P.n_tiles);
+    if (h->comm[p] && g_nccl.commDestroy) g_nccl.commDestroy(h->comm[p]);
+  }
+  cudaFree(h->rope_cs);
+  cudaFree(h->op_ctr);
+  if (h->ev_ts) cudaEventDestroy(h->ev_ts);
+  delete h;
+}
+
+// ---------------------------------------------------------- op-level entries
+static int op_ctx(bullet_handle* h, int lo, int hi, void* stream, Ctx* c) {
+  if (!h) return set_err(BULLET_EINVAL, "null handle");
+  if (h->host_only) return set_err(BULLET_EUNSUPPORTED, "host-only handle");
+  if (lo < 0 || hi > h->n_sms || lo >= hi) return set_err(BULLET_ESMRANGE, "range [%d,%d)", lo, hi);
+  *c = Ctx{h, 0, gate_of(h, lo, hi), hi - lo, h->log_cap > 0, (cudaStream_t)stream, true};
+  return BULLET_OK;
+}
+
+int bullet_op_gemm(bullet_handle* h, int epi, const void* A, int M, int K, const void* B, int N,
+                   int silu_half, const void* bias, const float* resid, void* out, int lo, int hi,
+                   void* stream) {
+  Ctx c;
+  int rc = op_ctx(h, lo, hi, stream, &c);
+  if (rc) return rc;
+  if (!A || !B || !out || M < 0 || K <= 0 || N <= 0 || epi < 0 || epi > 2) return set_err(BULLET_EINVAL, "gemm args");
+  if (epi == EPI_RESID && !resid) return set_err(BULLET_EINVAL, "resid null");
+  if (epi == EPI_SILU && (N % 2 || silu_half < N / 2)) return set_err(BULLET_EINVAL, "silu layout");
+  const int ldo = epi == EPI_SILU ? N / 2 : N;
+  return do_gemm(c, epi, A, M, K, B, N, silu_half, bias, resid, out, ldo);
+}
+
+int bullet_op_rmsnorm(bullet_handle* h, const float* x, int n, const void* g, void* out, int lo,
+                      int hi, void* stream) {
+  Ctx c;
+  int rc = op_ctx(h, lo, hi, stream, &c);
+  if (rc) return rc;
+  if (!x || !g || !out || n < 0) return set_err(BULLET_EINVAL, "rmsnorm args");
+  return do_rmsnorm(c, x, n, g, out);
+}
+
+int bullet_op_rope_kv(bullet_handle* h, const bullet_batch* b, int layer, const float* qkv, void* q,
+                      int lo, int hi, void* stream) {
+  Ctx c;
+  int rc = op_ctx(h, lo, hi, stream, &c);
+  if (rc) return rc;
+  if (!b || !qkv || !q || layer < 0 || layer >= h->cfg.n_layers) return set_err(BULLET_EINVAL, "rope args");
+  bullet_batch bb = *b;
+  bb.layer_begin = layer; bb.layer_end = layer;
+  if ((rc = validate_batch(h, &bb, 0))) return rc;
+  return do_rope(c, b, layer, qkv, q);
+}
+
+int bullet_op_attention(bullet_handle* h, const bullet_batch* b, int layer, const void* q, void* o,
+                        int kind, int lo, int hi, void* stream) {
+  Ctx c;
+  int rc = op_ctx(h, lo, hi, stream, &c);
+  if (rc) return rc;
+  if (!b || !q || !o || layer < 0 || layer >= h->cfg.n_layers || kind < 0 || kind > 2)
+    return set_err(BULLET_EINVAL, "attention args");
+  bullet_batch bb = *b;
+  bb.layer_begin = layer; bb.layer_end = layer;
+  if ((rc = validate_batch(h, &bb, 0))) return rc;
+  return do_attention(c, b, layer, q, o, kind);
+}
+
+}  // extern "C"

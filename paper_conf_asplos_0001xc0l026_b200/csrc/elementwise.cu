@@ -1,0 +1,227 @@
+// elementwise.cu — row-wise gated persistent kernels: RMSNorm (SURVEY §8a
+// S1/S6), RoPE + paged KV append (S3), the SIMT GEMM used for the fp32 model
+// (KI3), the per-step plan kernel and the SM probe.
+#include "kernels.h"
+
+namespace bl {
+
+// Warp-granular work claiming: lane 0 takes a unit, the warp shares it.
+__device__ __forceinline__ int warp_claim(const Launch& L) {
+  int u = 0;
+  if ((threadIdx.x & 31) == 0) u = atomicAdd(L.ctr, 1);
+  return __shfl_sync(0xffffffffu, u, 0);
+}
+
+// ------------------------------------------------------------------ RMSNorm
+// h = x / sqrt(mean(x^2) + eps) * g, one warp per row, fp32 math, rounded
+// once to the output type (oracle rounding point R1 / R4).
+template <typename T>
+__global__ void __launch_bounds__(256) k_rmsnorm(NormArgs a) {
+  if (!gate_ok(a.L.gate)) return;
+  const int lane = threadIdx.x & 31;
+  const T* g = reinterpret_cast<const T*>(a.g);
+  T* out = reinterpret_cast<T*>(a.out);
+  const int units = (a.n + ROWS_PER_UNIT - 1) / ROWS_PER_UNIT;
+  for (;;) {
+    const int u = warp_claim(a.L);
+    if (u >= units) break;
+    if (lane == 0) log_unit(a.L, u);
+    const int r1 = min(a.n, (u + 1) * ROWS_PER_UNIT);
+    for (int r = u * ROWS_PER_UNIT; r < r1; ++r) {
+      const float4* x4 = reinterpret_cast<const float4*>(a.x + (size_t)r * a.d);
+      float ss = 0.f;
+      for (int i = lane; i < a.d / 4; i += 32) {
+        float4 v = x4[i];
+        ss += v.x * v.x + v.y * v.y + v.z * v.z + v.w * v.w;
+      }
+      ss = warp_sum(ss);
+      const float inv = rsqrtf(ss / (float)a.d + a.eps);
+      T* o = out + (size_t)r * a.d;
+      for (int i = lane; i < a.d / 4; i += 32) {
+        float4 v = x4[i];
+        o[4 * i + 0] = Elt<T>::from_f(v.x * inv * Elt<T>::to_f(g[4 * i + 0]));
+        o[4 * i + 1] = Elt<T>::from_f(v.y * inv * Elt<T>::to_f(g[4 * i + 1]));
+        o[4 * i + 2] = Elt<T>::from_f(v.z * inv * Elt<T>::to_f(g[4 * i + 2]));
+        o[4 * i + 3] = Elt<T>::from_f(v.w * inv * Elt<T>::to_f(g[4 * i + 3]));
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------- RoPE + KV append
+// Token t of request r at position p = ctx[r] + (t - cu[r]).  Rotate-half
+// RoPE of q and k heads with the (cos, sin) table, round to the storage type
+// (point R2), q -> q_out[t], k / v -> pool slot bt[r][p / B] * B + p % B.
+template <typename T>
+__global__ void __launch_bounds__(256) k_rope_kv(RopeArgs a) {
+  if (!gate_ok(a.L.gate)) return;
+  const int lane = threadIdx.x & 31;
+  const int half = a.hd / 2;
+  T* q_out = reinterpret_cast<T*>(a.q_out);
+  T* pk = reinterpret_cast<T*>(a.pool_k);
+  T* pv = reinterpret_cast<T*>(a.pool_v);
+  const int nq = (a.H + 2 * a.Hkv) * a.hd;
+  const int units = (a.n_tok + ROWS_PER_UNIT - 1) / ROWS_PER_UNIT;
+  for (;;) {
+    const int u = warp_claim(a.L);
+    if (u >= units) break;
+    if (lane == 0) log_unit(a.L, u);
+    const int t1 = min(a.n_tok, (u + 1) * ROWS_PER_UNIT);
+    for (int t = u * ROWS_PER_UNIT; t < t1; ++t) {
+      const int r = find_req(a.cu, a.n_reqs, t);
+      const int pos = __ldg(a.ctx + r) + (t - __ldg(a.cu + r));
+      const int blk = __ldg(a.bt + (size_t)r * a.max_blocks + pos / a.B);
+      const int off = pos % a.B;
+      const float* src = a.qkv + (size_t)t * nq;
+      const float2* cs = a.cs + (size_t)pos * half;
+      for (int idx = lane; idx < (a.H + a.Hkv) * half; idx += 32) {
+        const int h = idx / half, i = idx % half;
+        const float x0 = src[h * a.hd + i], x1 = src[h * a.hd + i + half];
+        const float2 c = cs[i];
+        const float y0 = x0 * c.x - x1 * c.y, y1 = x1 * c.x + x0 * c.y;
+        T* dst;
+        if (h < a.H) dst = q_out + (size_t)t * a.H * a.hd + h * a.hd;
+        else dst = pk + (((size_t)blk * a.Hkv + (h - a.H)) * a.B + off) * a.hd;
+        dst[i] = Elt<T>::from_f(y0);
+        dst[i + half] = Elt<T>::from_f(y1);
+      }
+      const float* vs = src + (a.H + a.Hkv) * a.hd;
+      for (int idx = lane; idx < a.Hkv * a.hd; idx += 32) {
+        const int g = idx / a.hd, e = idx % a.hd;
+        pv[(((size_t)blk * a.Hkv + g) * a.B + off) * a.hd + e] = Elt<T>::from_f(vs[idx]);
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------ SIMT GEMM
+// Same contract and epilogues as the tcgen05 GEMM; used for the fp32 model
+// (tiny config, KI3).  64 x 64 output tiles, 4 x 4 per thread, fp32 FMA.
+template <typename T>
+__global__ void __launch_bounds__(256) k_gemm_simt(const T* __restrict__ A, const T* __restrict__ B,
+                                                   GemmArgs a) {
+  if (!gate_ok(a.L.gate)) return;
+  __shared__ float As[16][68], Bs[16][68], Us[16][68];
+  __shared__ int s_u;
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  const int NO = (a.epi == EPI_SILU) ? a.N / 2 : a.N;
+  const int mt = (a.M + 63) / 64, nt = (NO + 63) / 64, units = mt * nt;
+  for (;;) {
+    if (tid == 0) s_u = atomicAdd(a.L.ctr, 1);
+    __syncthreads();
+    const int u = s_u;
+    __syncthreads();
+    if (u >= units) break;
+    if (tid == 0) log_unit(a.L, u);
+    const int m0 = (u % mt) * 64, n0 = (u / mt) * 64;
+    float acc[4][4] = {}, acu[4][4] = {};
+    for (int k0 = 0; k0 < a.K; k0 += 16) {
+      for (int e = tid; e < 64 * 16; e += 256) {
+        const int rr = e / 16, kk = e % 16;
+        const int m = m0 + rr, n = n0 + rr;
+        As[kk][rr] = (m < a.M) ? Elt<T>::to_f(A[(size_t)m * a.K + k0 + kk]) : 0.f;
+        Bs[kk][rr] = (n < NO) ? Elt<T>::to_f(B[(size_t)n * a.K + k0 + kk]) : 0.f;
+        if (a.epi == EPI_SILU)
+          Us[kk][rr] = (n < NO) ? Elt<T>::to_f(B[(size_t)(a.silu_half + n) * a.K + k0 + kk]) : 0.f;
+      }
+      __syncthreads();
+#pragma unroll
+      for (int kk = 0; kk < 16; ++kk) {
+        float av[4], bv[4], uv[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) { av[i] = As[kk][ty * 4 + i]; bv[i] = Bs[kk][tx * 4 + i]; uv[i] = Us[kk][tx * 4 + i]; }
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
+            if (a.epi == EPI_SILU) acu[i][j] = fmaf(av[i], uv[j], acu[i][j]);
+          }
+      }
+      __syncthreads();
+    }
+    for (int i = 0; i < 4; ++i) {
+      const int m = m0 + ty * 4 + i;
+      if (m >= a.M) continue;
+      for (int j = 0; j < 4; ++j) {
+        const int n = n0 + tx * 4 + j;
+        if (n >= NO) continue;
+        const size_t o = (size_t)m * a.ldo + n;
+        if (a.epi == EPI_F32) {
+          float b = a.bias ? Elt<T>::to_f(reinterpret_cast<const T*>(a.bias)[n]) : 0.f;
+          a.out_f32[o] = acc[i][j] + b;
+        } else if (a.epi == EPI_RESID) {
+          a.out_f32[o] = a.resid[o] + acc[i][j];
+        } else {
+          const float z = acc[i][j];
+          reinterpret_cast<T*>(a.out_t)[o] = Elt<T>::from_f(z / (1.0f + expf(-z)) * acu[i][j]);
+        }
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------ plan
+// One thread: zero the phase's work counters and list the prefill attention
+// tiles (request, q-tile) longest-key-range first (LPT order).
+__global__ void k_plan(PlanArgs a) {
+  for (int i = threadIdx.x; i < a.n_counters; i += blockDim.x) a.counters[i] = 0;
+  if (threadIdx.x == 0 && a.tiles) {
+    int maxt = 0;
+    for (int r = 0; r < a.n_reqs; ++r) {
+      int len = a.cu[r + 1] - a.cu[r];
+      int nt = (len + a.bq - 1) / a.bq;
+      maxt = nt > maxt ? nt : maxt;
+    }
+    int n = 0;
+    for (int t = maxt - 1; t >= 0; --t)
+      for (int r = 0; r < a.n_reqs; ++r) {
+        int len = a.cu[r + 1] - a.cu[r];
+        if (t * a.bq < len) a.tiles[n++] = make_int2(r, t);
+      }
+    *a.n_tiles = n;
+  }
+}
+
+// SM probe (KI1): every CTA records its %smid; CTAs spin ~50 us so the
+// first wave spreads over every SM before any CTA retires.
+__global__ void k_probe(int* out, int n) {
+  const long long t0 = clock64();
+  while (clock64() - t0 < 100000) {
+  }
+  if (threadIdx.x == 0 && blockIdx.x < n) out[blockIdx.x] = (int)smid();
+}
+
+// ------------------------------------------------------------- launchers
+template <typename T>
+cudaError_t launch_gemm_simt(const T* A, const T* B, const GemmArgs& a, int grid, cudaStream_t st) {
+  k_gemm_simt<T><<<grid, 256, 0, st>>>(A, B, a);
+  return cudaGetLastError();
+}
+template <typename T>
+cudaError_t launch_rmsnorm(const NormArgs& a, int grid, cudaStream_t st) {
+  k_rmsnorm<T><<<grid, 256, 0, st>>>(a);
+  return cudaGetLastError();
+}
+template <typename T>
+cudaError_t launch_rope_kv(const RopeArgs& a, int grid, cudaStream_t st) {
+  k_rope_kv<T><<<grid, 256, 0, st>>>(a);
+  return cudaGetLastError();
+}
+cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st) {
+  k_plan<<<1, 256, 0, st>>>(a);
+  return cudaGetLastError();
+}
+cudaError_t launch_probe(int* out, int n, cudaStream_t st) {
+  k_probe<<<n, 32, 0, st>>>(out, n);
+  return cudaGetLastError();
+}
+
+template cudaError_t launch_gemm_simt<float>(const float*, const float*, const GemmArgs&, int, cudaStream_t);
+template cudaError_t launch_gemm_simt<__nv_bfloat16>(const __nv_bfloat16*, const __nv_bfloat16*, const GemmArgs&, int, cudaStream_t);
+template cudaError_t launch_rmsnorm<float>(const NormArgs&, int, cudaStream_t);
+template cudaError_t launch_rmsnorm<__nv_bfloat16>(const NormArgs&, int, cudaStream_t);
+template cudaError_t launch_rope_kv<float>(const RopeArgs&, int, cudaStream_t);
+template cudaError_t launch_rope_kv<__nv_bfloat16>(const RopeArgs&, int, cudaStream_t);
+
+}  // namespace bl

@@ -1,0 +1,336 @@
+// gemm_tc.cu — persistent, smid-gated tcgen05 GEMM for sm_100a.
+//
+// C[M x N] = A[M x K] . B[N x K]^T, bf16 operands (both K-major), fp32
+// accumulation in TMEM, fused epilogues (QKV store + bias, residual add,
+// SiLU(gate) * up).  Serves the QKV / O-proj / gate_up / down projections of
+// both phases (the paper's cuBLAS GEMMs P:L40).
+//
+// Structure (one CTA per SM, 256 threads):
+//   warp 0 lane 0  tile scheduler (atomic claim, gated) + TMA producer
+//   warp 1 lane 0  MMA issuer: tcgen05.mma.cta_group::1.kind::f16, M=128
+//   warp 2         TMEM allocator (512 columns = 2 accumulator stages)
+//   warps 4..7     epilogue: tcgen05.ld 32x32b -> registers -> global
+// Pipelines: smem stage ring (full/empty mbarriers, TMA complete_tx and
+// tcgen05.commit), accumulator ring (2 stages), work-unit queue (4 slots).
+// Operand tiles: A 128 x 64, B bn x 64 (bf16, 128-byte swizzle, TMA).
+// Split-K (decode-sized GEMMs): each unit writes an fp32 partial; the last
+// unit of a tile (atomic ticket) sums the partials in split order
+// (deterministic) and runs the epilogue.
+#include "kernels.h"
+
+namespace bl {
+
+namespace {
+
+constexpr int BM = 128, BK = 64, NT = 256;
+constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
+
+__device__ __forceinline__ uint64_t sw128_desc(uint32_t addr) {
+  // UMMA shared-memory descriptor, K-major, SWIZZLE_128B: start>>4 [0,14),
+  // LBO (unused for swizzled K-major) = 1 [16,30), SBO = 1024 B >> 4 [32,46),
+  // version 1 [46,48), layout SWIZZLE_128B = 2 [61,64).
+  return (uint64_t)((addr >> 4) & 0x3FFFu) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
+         ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
+}
+
+__device__ __forceinline__ void tc_fence_after() {
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_before() {
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_mma(uint32_t d_tmem, uint64_t ad, uint64_t bd, uint32_t idesc,
+                                       uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(ad), "l"(bd), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void tc_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                   smem_u32(bar))
+               : "memory");
+}
+
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
+  uint32_t r[32];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%"
+      "15,%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
+        "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]),
+        "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]), "=r"(r[25]),
+        "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+__device__ __forceinline__ float silu_f(float z) { return z / (1.0f + __expf(-z)); }
+
+// Epilogue for 32 consecutive output columns [col, col+32) of row m.
+__device__ __forceinline__ void epi_store(const GemmArgs& a, int m, int col, const float* v,
+                                          const float* u) {
+  const size_t o = (size_t)m * a.ldo + col;
+  if (a.epi == EPI_F32) {
+    float4* dst = reinterpret_cast<float4*>(a.out_f32 + o);
+    const __nv_bfloat16* b = reinterpret_cast<const __nv_bfloat16*>(a.bias);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      float4 w = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+      if (b) {
+        w.x += __bfloat162float(b[col + 4 * i]); w.y += __bfloat162float(b[col + 4 * i + 1]);
+        w.z += __bfloat162float(b[col + 4 * i + 2]); w.w += __bfloat162float(b[col + 4 * i + 3]);
+      }
+      dst[i] = w;
+    }
+  } else if (a.epi == EPI_RESID) {
+    const float4* r = reinterpret_cast<const float4*>(a.resid + o);
+    float4* dst = reinterpret_cast<float4*>(a.out_f32 + o);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      float4 w = r[i];
+      w.x += v[4 * i]; w.y += v[4 * i + 1]; w.z += v[4 * i + 2]; w.w += v[4 * i + 3];
+      dst[i] = w;
+    }
+  } else {  // EPI_SILU: out = silu(gate) * up, bf16
+    uint32_t p[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) {
+      __nv_bfloat162 h = __floats2bfloat162_rn(silu_f(v[2 * i]) * u[2 * i],
+                                              silu_f(v[2 * i + 1]) * u[2 * i + 1]);
+      p[i] = *reinterpret_cast<uint32_t*>(&h);
+    }
+    uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(a.out_t) + o);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) dst[i] = make_uint4(p[4 * i], p[4 * i + 1], p[4 * i + 2], p[4 * i + 3]);
+  }
+}
+
+}  // namespace
+
+int gemm_tc_stages(int bn) {
+  const int st = A_BYTES + bn * BK * 2;
+  int s = (192 * 1024) / st;
+  return s > 8 ? 8 : s;
+}
+size_t gemm_tc_smem_bytes(int bn) {
+  const int st = A_BYTES + bn * BK * 2;
+  return (size_t)gemm_tc_stages(bn) * st + 1024 /*align*/ + 512 /*barriers etc.*/;
+}
+
+__global__ void __launch_bounds__(NT, 1)
+    k_gemm_tc(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
+              GemmArgs a, int n_stages) {
+  if (!gate_ok(a.L.gate)) return;  // not this phase's SM: touch nothing
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~uintptr_t(1023));
+  const int bn = a.bn;
+  const uint32_t b_bytes = bn * BK * 2, st_bytes = A_BYTES + b_bytes;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + n_stages * st_bytes);
+  uint64_t* empty = full + n_stages;
+  uint64_t* accf = empty + n_stages;
+  uint64_t* acce = accf + 2;
+  uint64_t* tqf = acce + 2;
+  uint64_t* tqe = tqf + 4;
+  int* tile_q = reinterpret_cast<int*>(tqe + 4);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tile_q + 4);
+  int* s_last = reinterpret_cast<int*>(tmem_slot + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int m_tiles = (a.M + BM - 1) / BM;
+  const int n_tiles = a.N / bn;
+  const int units = m_tiles * n_tiles * a.splits;
+  const int k_blocks = a.K / BK;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < n_stages; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(accf + i, 1); mbar_init(acce + i, 4); }
+    for (int i = 0; i < 4; ++i) { mbar_init(tqf + i, 1); mbar_init(tqe + i, 5); }
+    mbar_fence_init();
+  }
+  if (warp == 0 && lane == 0) { tma_prefetch_desc(&mapA); tma_prefetch_desc(&mapB); }
+  if (warp == 2) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)),
+                 "r"(512));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {  // ---------------- scheduler + TMA producer
+      int it = 0, s = 0;
+      uint32_t ph = 0;
+      for (;;) {
+        const int slot = it & 3;
+        mbar_wait(tqe + slot, ((it >> 2) & 1) ^ 1);
+        int u = atomicAdd(a.L.ctr, 1);
+        if (u >= units) u = -1;
+        tile_q[slot] = u;
+        mbar_arrive(tqf + slot);
+        if (u < 0) break;
+        log_unit(a.L, u);
+        const int tile = u / a.splits, sp = u % a.splits;
+        const int m_blk = tile % m_tiles, n_blk = tile / m_tiles;
+        const int kb0 = sp * k_blocks / a.splits, kb1 = (sp + 1) * k_blocks / a.splits;
+        int r0, r1;
+        if (a.epi == EPI_SILU) { r0 = n_blk * (bn / 2); r1 = a.silu_half + r0; }
+        else { r0 = n_blk * bn; r1 = r0 + bn / 2; }
+        for (int kb = kb0; kb < kb1; ++kb) {
+          mbar_wait(empty + s, ph ^ 1);
+          uint8_t* sa = smem + s * st_bytes;
+          mbar_arrive_expect_tx(full + s, st_bytes);
+          tma_load_2d(sa, &mapA, full + s, kb * BK, m_blk * BM);
+          tma_load_2d(sa + A_BYTES, &mapB, full + s, kb * BK, r0);
+          tma_load_2d(sa + A_BYTES + b_bytes / 2, &mapB, full + s, kb * BK, r1);
+          if (++s == n_stages) { s = 0; ph ^= 1; }
+        }
+        ++it;
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {  // ---------------- MMA issuer
+      const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(bn >> 3) << 17) |
+                             ((uint32_t)(BM >> 4) << 24);
+      int it = 0, s = 0, as = 0;
+      uint32_t ph = 0, aph = 0;
+      for (;;) {
+        const int slot = it & 3;
+        mbar_wait(tqf + slot, (it >> 2) & 1);
+        const int u = tile_q[slot];
+        mbar_arrive(tqe + slot);
+        if (u < 0) break;
+        const int sp = u % a.splits;
+        const int kb0 = sp * k_blocks / a.splits, kb1 = (sp + 1) * k_blocks / a.splits;
+        mbar_wait(acce + as, aph ^ 1);
+        tc_fence_after();
+        const uint32_t d_tmem = tmem + as * 256;
+        for (int kb = kb0; kb < kb1; ++kb) {
+          mbar_wait(full + s, ph);
+          tc_fence_after();
+          const uint32_t a_addr = smem_u32(smem + s * st_bytes), b_addr = a_addr + A_BYTES;
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k)
+            tc_mma(d_tmem, sw128_desc(a_addr + k * 32), sw128_desc(b_addr + k * 32), idesc,
+                   (kb > kb0 || k > 0) ? 1u : 0u);
+          tc_commit(empty + s);
+          if (++s == n_stages) { s = 0; ph ^= 1; }
+        }
+        tc_commit(accf + as);
+        if (++as == 2) { as = 0; aph ^= 1; }
+        ++it;
+      }
+    }
+  } else if (warp >= 4) {  // ---------------- epilogue (warps 4..7 = TMEM lane quadrants 0..3)
+    const int et = threadIdx.x - 128, eq = warp & 3;
+    int it = 0, as = 0;
+    uint32_t aph = 0;
+    float v[32], w[32];
+    for (;;) {
+      const int slot = it & 3;
+      mbar_wait(tqf + slot, (it >> 2) & 1);
+      const int u = tile_q[slot];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(tqe + slot);
+      if (u < 0) break;
+      const int tile = u / a.splits;
+      const int m_blk = tile % m_tiles, n_blk = tile / m_tiles;
+      const int m = m_blk * BM + et;
+      const int col0 = (a.epi == EPI_SILU) ? n_blk * (bn / 2) : n_blk * bn;
+      const int out_chunks = (a.epi == EPI_SILU) ? bn / 64 : bn / 32;
+      mbar_wait(accf + as, aph);
+      tc_fence_after();
+      const uint32_t tb = tmem + ((uint32_t)(eq * 32) << 16) + as * 256;
+      if (a.splits == 1) {
+        for (int c = 0; c < out_chunks; ++c) {
+          tmem_ld32(tb + c * 32, v);
+          if (a.epi == EPI_SILU) tmem_ld32(tb + bn / 2 + c * 32, w);
+          if (m < a.M) epi_store(a, m, col0 + c * 32, v, w);
+        }
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(acce + as);
+      } else {
+        float* P = a.partials + ((size_t)u * BM + et) * bn;
+        for (int c = 0; c < bn / 32; ++c) {
+          tmem_ld32(tb + c * 32, v);
+          float4* d4 = reinterpret_cast<float4*>(P + c * 32);
+#pragma unroll
+          for (int i = 0; i < 8; ++i) d4[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+        }
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(acce + as);
+        __threadfence();
+        named_bar_sync(1, 128);
+        if (et == 0) {
+          const int old = atomicAdd(a.tile_sems + tile, 1);
+          const int last = (old == a.splits - 1);
+          if (last) a.tile_sems[tile] = 0;  // self-reset for the next launch
+          *s_last = last;
+        }
+        named_bar_sync(1, 128);
+        if (*s_last) {
+          __threadfence();
+          if (m < a.M) {
+            for (int c = 0; c < out_chunks; ++c) {
+#pragma unroll
+              for (int i = 0; i < 32; ++i) { v[i] = 0.f; w[i] = 0.f; }
+              for (int sp = 0; sp < a.splits; ++sp) {  // fixed split order: deterministic
+                const float* Q = a.partials + ((size_t)(tile * a.splits + sp) * BM + et) * bn;
+                const float4* q4 = reinterpret_cast<const float4*>(Q + c * 32);
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                  float4 t = __ldcg(q4 + i);
+                  v[4 * i] += t.x; v[4 * i + 1] += t.y; v[4 * i + 2] += t.z; v[4 * i + 3] += t.w;
+                }
+                if (a.epi == EPI_SILU) {
+                  const float4* g4 = reinterpret_cast<const float4*>(Q + bn / 2 + c * 32);
+#pragma unroll
+                  for (int i = 0; i < 8; ++i) {
+                    float4 t = __ldcg(g4 + i);
+                    w[4 * i] += t.x; w[4 * i + 1] += t.y; w[4 * i + 2] += t.z; w[4 * i + 3] += t.w;
+                  }
+                }
+              }
+              epi_store(a, m, col0 + c * 32, v, w);
+            }
+          }
+        }
+      }
+      if (++as == 2) { as = 0; aph ^= 1; }
+      ++it;
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
+  }
+}
+
+cudaError_t launch_gemm_tc(const CUtensorMap& mapA, const CUtensorMap& mapB, const GemmArgs& a,
+                           int grid, cudaStream_t st) {
+  const size_t smem = gemm_tc_smem_bytes(a.bn);
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(k_gemm_tc, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)gemm_tc_smem_bytes(64) > (int)gemm_tc_smem_bytes(256)
+                                             ? (int)gemm_tc_smem_bytes(64)
+                                             : (int)gemm_tc_smem_bytes(256));
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  k_gemm_tc<<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn));
+  return cudaGetLastError();
+}
+
+}  // namespace bl

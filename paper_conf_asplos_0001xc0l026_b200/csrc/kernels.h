@@ -1,0 +1,76 @@
+// kernels.h — argument structs and launchers of the Bullet sm_100a kernels.
+#pragma once
+#include "common.cuh"
+
+namespace bl {
+
+enum { EPI_F32 = 0, EPI_RESID = 1, EPI_SILU = 2 };
+
+// C[M x N] = A[M x K] . B[N x K]^T with a fused epilogue (all row-major).
+struct GemmArgs {
+  int M, N, K;        // N = B rows used (2 x output cols for EPI_SILU)
+  int bn;             // tile width in B rows (tcgen05: 64/128/256; SIMT: 64)
+  int splits;         // split-K factor (tcgen05 only)
+  int epi;
+  int silu_half;      // row offset of the "up" rows in B (EPI_SILU)
+  const void* bias;   // [N] of the element type, or null (EPI_F32)
+  const float* resid; // [M][ldo] (EPI_RESID; may alias out_f32)
+  float* out_f32;     // [M][ldo] (EPI_F32, EPI_RESID)
+  void* out_t;        // [M][ldo] of the element type (EPI_SILU)
+  int ldo;
+  float* partials;    // split-K: [units][128][bn]
+  int* tile_sems;     // split-K: [tiles], zero between launches (self-resetting)
+  Launch L;
+};
+
+struct NormArgs {
+  const float* x; const void* g; void* out;
+  int n, d; float eps;
+  Launch L;
+};
+
+struct RopeArgs {
+  const float* qkv; void* q_out; void* pool_k; void* pool_v;
+  const float2* cs;   // [max_pos][hd/2] (cos, sin)
+  const int32_t* cu; const int32_t* ctx; const int32_t* bt;
+  int n_reqs, max_blocks, n_tok, H, Hkv, hd, B, max_pos;
+  Launch L;
+};
+
+struct AttnArgs {
+  const void* q; void* o; const void* pool_k; const void* pool_v;
+  const int32_t* cu; const int32_t* ctx; const int32_t* bt;
+  int n_reqs, max_blocks, n_tok, H, Hkv, hd, B;
+  float scale;
+  const int2* tiles;      // prefill tensor-core kernel: (request, q-tile) list
+  const int* n_tiles;     // device count of `tiles`
+  Launch L;
+};
+
+struct PlanArgs {
+  int* counters; int n_counters;
+  const int32_t* cu; int n_reqs; int bq;
+  int2* tiles; int* n_tiles;
+};
+
+// launchers (return cudaError_t of the launch)
+cudaError_t launch_gemm_tc(const CUtensorMap& mapA, const CUtensorMap& mapB, const GemmArgs& a,
+                           int grid, cudaStream_t st);
+size_t gemm_tc_smem_bytes(int bn);
+int gemm_tc_stages(int bn);
+template <typename T>
+cudaError_t launch_gemm_simt(const T* A, const T* B, const GemmArgs& a, int grid, cudaStream_t st);
+template <typename T>
+cudaError_t launch_rmsnorm(const NormArgs& a, int grid, cudaStream_t st);
+template <typename T>
+cudaError_t launch_rope_kv(const RopeArgs& a, int grid, cudaStream_t st);
+template <typename T>
+cudaError_t launch_attn_simt(const AttnArgs& a, int grid, cudaStream_t st);
+cudaError_t launch_attn_prefill_tc(const AttnArgs& a, int grid, cudaStream_t st);
+cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);
+cudaError_t launch_probe(int* out_smid, int n, cudaStream_t st);
+
+constexpr int ATTN_TC_BQ = 64;    // query rows per tensor-core attention tile
+constexpr int ROWS_PER_UNIT = 8;  // rows per work unit of row-wise kernels
+
+}  // namespace bl

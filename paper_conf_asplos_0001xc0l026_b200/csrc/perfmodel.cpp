@@ -1,0 +1,290 @@
+// perfmodel.cpp — Bullet's performance estimator and SLO-aware split
+// decision, host C++ (product code; the test oracle restates the same
+// paper passages independently in oracle/perfmodel.py).
+//
+//   Eq. 1  s = 1 - g / (M ceil(g / M))
+//   Eq. 2  t_i = max(c_i/C M/(m d_c p_c), b_i/B M/(m d_b p_b)) / (1 - s_i)
+//   T_m = sum_i t_i
+//   Alg. 1 + decode-SM search + decode pause
+// Readings R-11..R-18 of DESIGN.md §3.
+#include "perfmodel.h"
+
+#include <algorithm>
+#include <cctype>
+#include <cmath>
+#include <cstdlib>
+#include <cstring>
+#include <limits>
+#include <map>
+#include <string>
+#include <vector>
+
+namespace bl {
+
+// ------------------------------------------------------------ tiny JSON
+namespace {
+struct JP {
+  const char* p;
+  std::map<std::string, std::vector<double>> out;
+  void ws() { while (*p && isspace((unsigned char)*p)) ++p; }
+  bool str(std::string& s) {
+    ws();
+    if (*p != '"') return false;
+    ++p;
+    s.clear();
+    while (*p && *p != '"') s += *p++;
+    if (*p != '"') return false;
+    ++p;
+    return true;
+  }
+  bool num(double& v) {
+    ws();
+    char* e = nullptr;
+    v = strtod(p, &e);
+    if (e == p) return false;
+    p = e;
+    return true;
+  }
+  // value at path `key` (dotted); objects recurse, arrays of numbers stored
+  bool value(const std::string& key) {
+    ws();
+    if (*p == '{') {
+      ++p;
+      ws();
+      if (*p == '}') { ++p; return true; }
+      for (;;) {
+        std::string k;
+        if (!str(k)) return false;
+        ws();
+        if (*p != ':') return false;
+        ++p;
+        if (!value(key.empty() ? k : key + "." + k)) return false;
+        ws();
+        if (*p == ',') { ++p; continue; }
+        if (*p == '}') { ++p; return true; }
+        return false;
+      }
+    }
+    if (*p == '[') {
+      ++p;
+      std::vector<double> v;
+      ws();
+      if (*p == ']') { ++p; out[key] = v; return true; }
+      for (;;) {
+        double d;
+        if (!num(d)) return false;
+        v.push_back(d);
+        ws();
+        if (*p == ',') { ++p; continue; }
+        if (*p == ']') { ++p; break; }
+        return false;
+      }
+      out[key] = v;
+      return true;
+    }
+    if (*p == '"') { std::string s; return str(s); }
+    double d;
+    if (!num(d)) return false;
+    out[key] = {d};
+    return true;
+  }
+};
+}  // namespace
+
+bool PerfParams::parse(const char* json, std::string* err) {
+  JP j{json, {}};
+  if (!j.value("")) { if (err) *err = "perf params: malformed JSON"; return false; }
+  auto get1 = [&](const char* k, double& dst) {
+    auto it = j.out.find(k);
+    if (it != j.out.end() && it->second.size() == 1) dst = it->second[0];
+  };
+  auto getv = [&](const char* k, std::vector<double>& dst) {
+    auto it = j.out.find(k);
+    if (it != j.out.end()) dst = it->second;
+  };
+  get1("M", M); get1("C_tflops", C_tflops); get1("B_gbs", B_gbs);
+  get1("p_c", p_c); get1("p_b", p_b);
+  getv("d_c.m", dc_m); getv("d_c.v", dc_v); getv("d_b.m", db_m); getv("d_b.v", db_v);
+  get1("tiles.gemm_bm", gemm_bm); get1("tiles.gemm_bn", gemm_bn); get1("tiles.gemm_bk", gemm_bk);
+  get1("tiles.min_k_blocks", min_k_blocks); get1("tiles.attn_bq", attn_bq);
+  get1("tiles.rows_per_unit", rows_per_unit);
+  get1("occ.gemm", occ_gemm); get1("occ.attn", occ_attn); get1("occ.elem", occ_elem);
+  if (dc_m.size() != dc_v.size() || db_m.size() != db_v.size() || dc_m.empty() || db_m.empty()) {
+    if (err) *err = "perf params: d_c / d_b tables malformed";
+    return false;
+  }
+  return true;
+}
+
+void PerfParams::set_default(int n_sms) {
+  M = n_sms;
+  C_tflops = 1649.5; B_gbs = 6549.4;   // MEASURED_PEAKS.json (burst GEMM, copy)
+  dc_m = {1.0, (double)n_sms}; dc_v = {1.0, 1.0};
+  db_m = {1.0, (double)n_sms}; db_v = {1.0, 1.0};
+  p_c = p_b = 1.0;
+}
+
+// Eq. 1
+double wave_idle(double g, double M) {
+  if (g <= 0 || M <= 0) return 0.0;
+  const double w = std::ceil(g / M);
+  return 1.0 - g / (M * w);
+}
+
+static double interp(const std::vector<double>& ms, const std::vector<double>& vs, double m) {
+  if (m <= ms[0]) return vs[0];
+  for (size_t i = 1; i < ms.size(); ++i)
+    if (m <= ms[i]) return vs[i - 1] + (m - ms[i - 1]) / (ms[i] - ms[i - 1]) * (vs[i] - vs[i - 1]);
+  return vs.back();
+}
+
+// Per-kernel (c_i, b_i, g_i, occupancy) of one layer of one phase.
+std::vector<KernelCost> layer_kernels(const PhaseShape& s, const PerfParams& P, int m) {
+  std::vector<KernelCost> ks;
+  double n = 0, pairs = 0, keys = 0;
+  int maxq = 0;
+  for (size_t i = 0; i < s.q_lens.size(); ++i) {
+    const double q = s.q_lens[i], c = s.ctx_lens[i];
+    n += q;
+    pairs += q * c + q * (q + 1) / 2;
+    keys += c + q;
+    maxq = std::max(maxq, s.q_lens[i]);
+  }
+  if (n == 0) return ks;
+  const double d = s.d, H = s.H, Hkv = s.Hkv, hd = s.hd, I = s.I, e = s.elt;
+  const double nq = (H + 2 * Hkv) * hd;
+  const double rows = P.rows_per_unit;
+  auto gemm = [&](const char* name, double K, double N, double extra) {
+    const double tiles = std::ceil(n / P.gemm_bm) * std::ceil(N / P.gemm_bn);
+    double splits = std::ceil(m * P.occ_gemm / tiles);
+    splits = std::max(1.0, std::min(splits, std::floor(K / (P.gemm_bk * P.min_k_blocks))));
+    ks.push_back({name, 2.0 * n * K * N, e * (K * N + n * K) + extra, tiles * splits, P.occ_gemm});
+  };
+  double attn_units = 0;
+  if (maxq > 1) {
+    for (int q : s.q_lens) attn_units += std::ceil(q / P.attn_bq);
+    attn_units *= H;
+  } else {
+    attn_units = (double)s.q_lens.size() * Hkv;
+  }
+  ks.push_back({"rmsnorm1", 4.0 * n * d, 4 * n * d + e * n * d + e * d, std::ceil(n / rows), P.occ_elem});
+  gemm("qkv", d, nq, 4 * n * nq);
+  ks.push_back({"rope_kv", 6.0 * n * (H + Hkv) * hd, 4 * n * nq + e * n * nq, std::ceil(n / rows), P.occ_elem});
+  ks.push_back({"attn", 4.0 * hd * H * pairs, 2 * e * Hkv * hd * keys + 2 * e * n * H * hd, attn_units, P.occ_attn});
+  gemm("o_proj", H * hd, d, 8 * n * d);
+  ks.push_back({"rmsnorm2", 4.0 * n * d, 4 * n * d + e * n * d + e * d, std::ceil(n / rows), P.occ_elem});
+  gemm("gate_up", d, 2 * I, e * n * I);
+  gemm("down", I, d, 8 * n * d);
+  return ks;
+}
+
+// T_m in seconds, Eq. 2 per kernel.
+double layer_time(const PhaseShape& s, const PerfParams& P, int m, int corun_m) {
+  if (m <= 0) return std::numeric_limits<double>::infinity();
+  const double C = P.C_tflops * 1e12, B = P.B_gbs * 1e9, M = P.M;
+  const double dc = interp(P.dc_m, P.dc_v, m), db = interp(P.db_m, P.db_v, m);
+  const double pc = corun_m > 0 ? P.p_c : 1.0, pb = corun_m > 0 ? P.p_b : 1.0;
+  double total = 0;
+  for (const auto& k : layer_kernels(s, P, m)) {
+    const double sidle = wave_idle(k.g, (double)m * k.occ);
+    const double tc = k.c / C * M / (m * dc * pc);
+    const double tb = k.b / B * M / (m * db * pb);
+    total += std::max(tc, tb) / (1.0 - sidle);
+  }
+  return total;
+}
+
+static double p90(std::vector<double> v, double pct) {
+  if (v.empty()) return 0.0;
+  std::sort(v.begin(), v.end());
+  long idx = (long)std::ceil(pct * (double)v.size()) - 1;
+  if (idx < 0) idx = 0;
+  return v[(size_t)idx];
+}
+
+struct Eval { double ttft, tpot, t_p; };
+
+static Eval evaluate(const PerfParams& P, const PhaseShape& model, const SchedState& S,
+                     const Slo& slo, int u, int v) {
+  const int N = (int)P.M, L = S.total_layers;
+  PhaseShape pre = model, dec = model;
+  pre.q_lens = S.prefill_lens; pre.ctx_lens.assign(S.prefill_lens.size(), 0);
+  const int mctx = (int)std::lround(S.decode_mean_ctx);
+  dec.q_lens.assign(S.decode_tokens.size(), 1); dec.ctx_lens.assign(S.decode_tokens.size(), mctx);
+  const double ms = 1e3;
+  const double t_p = S.prefill_lens.empty() ? 0.0 : layer_time(pre, P, u, v) * ms;
+  const double rem = t_p * (L - S.layers_done);                       // Alg. 1 l.3
+  std::vector<double> ttft, tpot;
+  for (size_t i = 0; i < S.prefill_lens.size(); ++i)                  // l.4-5
+    ttft.push_back((rem + S.prefill_waited_ms[i]) / (slo.ttft_norm * S.prefill_lens[i]));
+  for (size_t i = 0; i < S.pending_lens.size(); ++i) {                // l.6-7 (+ own prefill, R-15)
+    PhaseShape one = model;
+    one.q_lens = {S.pending_lens[i]}; one.ctx_lens = {0};
+    const double own = layer_time(one, P, u, v) * ms * L;
+    ttft.push_back((S.pending_waited_ms[i] + rem + own) / (slo.ttft_norm * S.pending_lens[i]));
+  }
+  if (!S.decode_tokens.empty()) {                                     // l.8-10 (R-14)
+    double t_iter;
+    if (v > 0) t_iter = layer_time(dec, P, v, u) * ms * L;
+    else t_iter = layer_time(pre, P, N, 0) * ms + layer_time(dec, P, S.v_k, 0) * ms * L;
+    for (size_t i = 0; i < S.decode_tokens.size(); ++i)
+      tpot.push_back(((S.decode_elapsed_ms[i] + t_iter) / (S.decode_tokens[i] + 1)) / slo.tpot_ms);
+  }
+  return {p90(ttft, slo.percentile), p90(tpot, slo.percentile), t_p};
+}
+
+void choose_split(const PerfParams& P, const PhaseShape& model, const SchedState& S,
+                  const Slo& slo, int gran, int* prefill_sms, int* decode_steps) {
+  const int N = (int)P.M, L = S.total_layers;
+  const bool has_pre = !S.prefill_lens.empty() || !S.pending_lens.empty();
+  if (S.decode_tokens.empty()) { *prefill_sms = N; *decode_steps = 0; return; }
+  if (!has_pre) { *prefill_sms = 0; *decode_steps = L; return; }
+  std::vector<int> cands;
+  for (int v = slo.v_min; v <= N - gran; ++v)
+    if (v % gran == 0 || v == slo.v_min) cands.push_back(v);
+  if (cands.empty()) { *prefill_sms = N; *decode_steps = 0; return; }
+  std::map<int, Eval> ev;
+  for (int v : cands) ev[v] = evaluate(P, model, S, slo, N - v, v);
+  int vk = cands[0];
+  for (int v : cands)
+    if (std::abs(v - S.v_k) < std::abs(vk - S.v_k)) vk = v;
+  const bool ok_t = ev[vk].ttft <= 1.0, ok_d = ev[vk].tpot <= 1.0;
+
+  auto reduce_decode = [&]() -> int {
+    for (int v : cands)   // ascending: first feasible = smallest decode SM count
+      if (v <= vk && ev[v].ttft <= 1.0 && ev[v].tpot <= 1.0) return v;
+    const Eval pz = evaluate(P, model, S, slo, N, 0);
+    if (pz.tpot <= 1.0) return 0;            // pause decode
+    return cands.front();                    // v_min
+  };
+  auto reduce_prefill = [&]() -> int {
+    for (int v : cands)
+      if (v >= vk && ev[v].tpot <= 1.0) return v;
+    int best = cands.front();
+    for (int v : cands)
+      if (ev[v].tpot < ev[best].tpot) best = v;
+    return best;
+  };
+  auto balanced = [&]() -> int {
+    int best = cands.front();
+    for (int v : cands)
+      if (std::max(ev[v].ttft, ev[v].tpot) < std::max(ev[best].ttft, ev[best].tpot)) best = v;
+    return best;
+  };
+  int v;
+  if (ok_t && ok_d) v = reduce_decode();
+  else if (!ok_t && !ok_d) v = balanced();
+  else if (ok_t && !ok_d && (int)S.pending_lens.size() <= slo.w_max) v = reduce_prefill();
+  else v = reduce_decode();
+  if (v == 0) { *prefill_sms = N; *decode_steps = 0; return; }
+  const int u = N - v;
+  PhaseShape dec = model;
+  const int mctx = (int)std::lround(S.decode_mean_ctx);
+  dec.q_lens.assign(S.decode_tokens.size(), 1); dec.ctx_lens.assign(S.decode_tokens.size(), mctx);
+  const double t_d = layer_time(dec, P, v, u) * 1e3;
+  const double t_p = ev[v].t_p;
+  *prefill_sms = u;
+  *decode_steps = t_d > 0 ? std::max(1, (int)std::floor(t_p / t_d + 0.5)) : 1;
+}
+
+}  // namespace bl

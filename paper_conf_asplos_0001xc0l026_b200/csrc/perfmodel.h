@@ -1,0 +1,50 @@
+// perfmodel.h — host-side performance estimator (Eq. 1, Eq. 2, T_m) and the
+// Alg. 1 split decision.  See perfmodel.cpp.
+#pragma once
+#include <string>
+#include <vector>
+
+namespace bl {
+
+struct PerfParams {
+  double M = 148, C_tflops = 1649.5, B_gbs = 6549.4;
+  std::vector<double> dc_m{1, 148}, dc_v{1, 1}, db_m{1, 148}, db_v{1, 1};
+  double p_c = 1, p_b = 1;
+  double gemm_bm = 128, gemm_bn = 256, gemm_bk = 64, min_k_blocks = 4, attn_bq = 64, rows_per_unit = 8;
+  double occ_gemm = 1, occ_attn = 1, occ_elem = 4;
+  bool parse(const char* json, std::string* err);
+  void set_default(int n_sms);
+};
+
+struct PhaseShape {
+  int d, H, Hkv, hd, I, elt;
+  std::vector<int> q_lens, ctx_lens;
+};
+
+struct KernelCost {
+  const char* name;
+  double c, b, g, occ;
+};
+
+struct SchedState {
+  int layers_done, total_layers;
+  std::vector<int> prefill_lens; std::vector<double> prefill_waited_ms;
+  std::vector<int> pending_lens; std::vector<double> pending_waited_ms;
+  std::vector<int> decode_tokens; std::vector<double> decode_elapsed_ms;
+  double decode_mean_ctx;
+  int u_k, v_k;
+};
+
+struct Slo {
+  double ttft_norm, tpot_ms;
+  int w_max, v_min;
+  double percentile;
+};
+
+double wave_idle(double g, double M);
+std::vector<KernelCost> layer_kernels(const PhaseShape& s, const PerfParams& P, int m);
+double layer_time(const PhaseShape& s, const PerfParams& P, int m, int corun_m);
+void choose_split(const PerfParams& P, const PhaseShape& model, const SchedState& S, const Slo& slo,
+                  int gran, int* prefill_sms, int* decode_steps);
+
+}  // namespace bl

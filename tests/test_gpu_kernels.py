@@ -1,0 +1,220 @@
+"""Per-kernel parity of the sm_100a kernels (through the C ABI op entry
+points) against the CPU oracle.  Needs a B200."""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+from workload import synth
+
+pytestmark = pytest.mark.gpu
+
+bf16 = torch.bfloat16
+
+
+@pytest.fixture(scope="module")
+def B():
+    import paper_conf_asplos_0001xc0l026_b200 as B
+    return B
+
+
+def _handle(B, m: synth.ModelShape, n_blocks=64, max_tok=8192, max_pos=8192, n_layers=1):
+    td = bf16 if m.dtype == "bf16" else torch.float32
+    pools = [(torch.zeros(n_blocks, m.n_kv_heads, 16, m.head_dim, dtype=td, device="cuda"),
+              torch.zeros(n_blocks, m.n_kv_heads, 16, m.head_dim, dtype=td, device="cuda"))
+             for _ in range(n_layers)]
+    return B.Bullet(B.Model.of(m), pools, max_tok, max_tok, max_pos), pools
+
+
+LLAMA = synth.MODELS["llama3.1-8b"]
+SMALL = synth.ModelShape("small-bf16", 1024, 8, 2, 128, 2816, 2)
+TINY = synth.MODELS["tiny"]
+
+
+def test_sm_probe(B):
+    bl, _ = _handle(B, SMALL)
+    props = torch.cuda.get_device_properties(0)
+    assert bl.n_sms == props.multi_processor_count
+    sig = bl.sm_order()
+    assert len(set(sig)) == bl.n_sms and sig == sorted(sig)
+
+
+def _int_operands(rng, M, K, N):
+    A = rng.integers(-2, 3, size=(M, K)).astype(np.float32)
+    W = rng.integers(-2, 3, size=(N, K)).astype(np.float32)
+    return A, W
+
+
+@pytest.mark.parametrize("M,N,K,lo,hi", [
+    (128, 6144, 4096, 0, None),     # decode-sized: bn 128 + split-K
+    (300, 1024, 1024, 0, None),     # ragged M tail
+    (4096, 6144, 4096, 0, None),    # prefill-sized: bn 256
+    (257, 4096, 4096, 10, 50),      # 40-SM gated range, split-K fixup
+    (64, 1280, 8192, 0, 16),        # 16 SMs, K = 8192
+])
+def test_gemm_f32_epilogue_bit_exact(B, M, N, K, lo, hi):
+    """Integer operands in {-2..2}: bf16 products and fp32 sums are exact, so
+    the tcgen05 GEMM must equal the exact product bit for bit."""
+    bl, _ = _handle(B, SMALL)
+    rng = np.random.default_rng(M + N)
+    A, W = _int_operands(rng, M, K, N)
+    bias = rng.integers(-3, 4, size=N).astype(np.float32)
+    out = torch.full((M, N), float("nan"), device="cuda")
+    bl.op_gemm(B.EPI_F32, torch.from_numpy(A).to("cuda", bf16), torch.from_numpy(W).to("cuda", bf16),
+               out, bias=torch.from_numpy(bias).to("cuda", bf16), lo=lo, hi=hi)
+    torch.cuda.synchronize()
+    ref = A.astype(np.int64) @ W.T.astype(np.int64) + bias.astype(np.int64)   # exact
+    assert np.array_equal(out.cpu().numpy(), ref.astype(np.float32))
+
+
+def test_gemm_matches_oracle_linear_small(B):
+    """Real-valued bf16 operands vs the oracle's fp64 linear (fp32-accumulate
+    error only)."""
+    bl, _ = _handle(B, SMALL)
+    rng = np.random.default_rng(5)
+    A = O.round_bf16(rng.standard_normal((200, 1024))).astype(np.float32)
+    W = O.round_bf16(rng.standard_normal((512, 1024)) * 1024 ** -0.5).astype(np.float32)
+    out = torch.zeros(200, 512, device="cuda")
+    bl.op_gemm(B.EPI_F32, torch.from_numpy(A).to("cuda", bf16), torch.from_numpy(W).to("cuda", bf16), out)
+    ref = O.linear(A.astype(np.float64), W)
+    assert np.abs(out.cpu().numpy() - ref).max() < 2e-4
+
+
+def test_gemm_resid_in_place_bit_exact(B):
+    bl, _ = _handle(B, SMALL)
+    rng = np.random.default_rng(7)
+    M, K, N = 333, 4096, 4096
+    A, W = _int_operands(rng, M, K, N)
+    R = rng.integers(-50, 50, size=(M, N)).astype(np.float32)
+    h = torch.from_numpy(R).cuda()
+    bl.op_gemm(B.EPI_RESID, torch.from_numpy(A).to("cuda", bf16), torch.from_numpy(W).to("cuda", bf16),
+               h, resid=h)
+    ref = R.astype(np.int64) + A.astype(np.int64) @ W.T.astype(np.int64)
+    assert np.array_equal(h.cpu().numpy(), ref.astype(np.float32))
+
+
+@pytest.mark.parametrize("M,lo,hi", [(128, 0, None), (1000, 0, None), (130, 100, 148)])
+def test_gemm_silu_mul(B, M, lo, hi):
+    """gate_up epilogue: a = silu(g) * u rounded to bf16 (point R5); integer
+    g, u exact, the silu/rounding within 1 bf16 ulp of the fp64 value."""
+    bl, _ = _handle(B, SMALL)
+    rng = np.random.default_rng(M)
+    K, I = 1024, 2816
+    A = rng.integers(-1, 2, size=(M, K)).astype(np.float32)
+    W = (rng.integers(-1, 2, size=(2 * I, K)) * 0.0625).astype(np.float32)
+    out = torch.zeros(M, I, dtype=bf16, device="cuda")
+    hi = bl.n_sms if hi is None else min(hi, bl.n_sms)
+    bl.op_gemm(B.EPI_SILU, torch.from_numpy(A).to("cuda", bf16), torch.from_numpy(W).to("cuda", bf16),
+               out, silu_half=I, lo=lo, hi=hi)
+    gu = A.astype(np.float64) @ W.T.astype(np.float64)
+    g, u = gu[:, :I], gu[:, I:]
+    ref = g / (1 + np.exp(-g)) * u
+    got = out.float().cpu().numpy()
+    ulp = np.maximum(np.abs(ref), 1e-30) * 2.0 ** -7
+    assert np.all(np.abs(got - ref) <= ulp + 1e-6)
+
+
+@pytest.mark.parametrize("m", [SMALL, TINY])
+def test_rmsnorm(B, m):
+    bl, _ = _handle(B, m)
+    rng = np.random.default_rng(3)
+    n, d = 77, m.d_model
+    x = rng.standard_normal((n, d)).astype(np.float32) * 3
+    g = synth.layer_weights(m, 0)["g_attn"]
+    td = bf16 if m.dtype == "bf16" else torch.float32
+    out = torch.zeros(n, d, dtype=td, device="cuda")
+    bl.op_rmsnorm(torch.from_numpy(x).cuda(), g.to("cuda", td), out)
+    ref = O.rmsnorm(x.astype(np.float64), g.numpy(), m.rms_eps)
+    got = out.float().cpu().numpy()
+    if m.dtype == "bf16":
+        rref = O.round_bf16(ref)
+        assert np.mean(got == rref) > 0.99                         # same rounding almost everywhere
+        assert np.all(np.abs(got - ref) <= np.abs(ref) * 2.0 ** -7 + 1e-30)   # never beyond 1 ulp
+    else:
+        assert np.abs(got - ref).max() < 1e-5
+
+
+def _batch(B, lay, rows, q, c, x):
+    return B.Batch(q, c, lay.block_table[rows], x)
+
+
+@pytest.mark.parametrize("m", [SMALL, TINY])
+def test_rope_kv_append(B, m):
+    """RoPE + paged KV append: q and the written pool slots vs the oracle's
+    rotate-half RoPE (R2 rounding, <= 1 ulp), every other slot untouched
+    (bit-exact sentinel)."""
+    q_lens, ctx = [37, 1, 1, 16], [0, 40, 15, 16]
+    lay = synth.paged_layout(q_lens, ctx, 16, seed_offset=3)
+    bl, pools = _handle(B, m, n_blocks=lay.n_blocks)
+    pools[0][0].fill_(-7.0); pools[0][1].fill_(-7.0)
+    rng = np.random.default_rng(9)
+    n = sum(q_lens)
+    nq = (m.n_heads + 2 * m.n_kv_heads) * m.head_dim
+    qkv = rng.standard_normal((n, nq)).astype(np.float32)
+    td = bf16 if m.dtype == "bf16" else torch.float32
+    qout = torch.zeros(n, m.n_heads * m.head_dim, dtype=td, device="cuda")
+    b = B.Batch(q_lens, ctx, lay.block_table, torch.zeros(n, m.d_model, device="cuda"))
+    bl.op_rope_kv(b, 0, torch.from_numpy(qkv).cuda(), qout)
+    torch.cuda.synchronize()
+    cfg = __import__("harness").oracle_cfg(m)
+    f = O.rope_inv_freq(cfg)
+    hd, H, Hkv = m.head_dim, m.n_heads, m.n_kv_heads
+    pk = pools[0][0].float().cpu().numpy(); pv = pools[0][1].float().cpu().numpy()
+    qg = qout.float().cpu().numpy()
+    written = np.zeros((lay.n_blocks, 16), bool)
+    row = 0
+    tol = (lambda r: np.abs(r) * 2.0 ** -7 + 1e-30) if m.dtype == "bf16" else (lambda r: 1e-5 + 1e-6 * np.abs(r))
+    for r, (ql, cl) in enumerate(zip(q_lens, ctx)):
+        for i in range(ql):
+            pos = cl + i
+            blk, off = lay.block_table[r][pos // 16], pos % 16
+            written[blk, off] = True
+            for h in range(H):
+                ref = O.rope_apply(qkv[row, h * hd:(h + 1) * hd], pos, f)
+                assert np.all(np.abs(qg[row, h * hd:(h + 1) * hd] - ref) <= tol(ref))
+            for g in range(Hkv):
+                ref = O.rope_apply(qkv[row, (H + g) * hd:(H + g + 1) * hd], pos, f)
+                assert np.all(np.abs(pk[blk, g, off] - ref) <= tol(ref))
+                vref = qkv[row, (H + Hkv + g) * hd:(H + Hkv + g + 1) * hd].astype(np.float64)
+                assert np.all(np.abs(pv[blk, g, off] - vref) <= tol(vref))
+            row += 1
+    assert np.all(pk[~written] == -7.0) and np.all(pv[~written] == -7.0)
+
+
+@pytest.mark.parametrize("m,kind", [(SMALL, 1), (SMALL, 2), (TINY, 1), (LLAMA, 2), (LLAMA, 1)])
+def test_attention_vs_oracle(B, m, kind):
+    """Paged attention (decode rows and causal prefill rows) vs the oracle's
+    plain softmax attention through the block table."""
+    q_lens, ctx = [150, 64, 1, 1, 1, 1], [0, 0, 0, 63, 200, 1000]
+    if kind == 2:
+        q_lens, ctx = [150, 64, 1, 77], [0, 0, 0, 0]
+    lay = synth.paged_layout(q_lens, ctx, 16, seed_offset=5)
+    bl, pools = _handle(B, m, n_blocks=lay.n_blocks)
+    pk_cpu, pv_cpu = synth.kv_pool(m, lay.n_blocks, 16, 0)
+    td = bf16 if m.dtype == "bf16" else torch.float32
+    pools[0][0].copy_(pk_cpu.to(td)); pools[0][1].copy_(pv_cpu.to(td))
+    n = sum(q_lens)
+    H, hd = m.n_heads, m.head_dim
+    rng = np.random.default_rng(11)
+    q = rng.standard_normal((n, H * hd))
+    if m.dtype == "bf16":
+        q = O.round_bf16(q)
+    o = torch.zeros(n, H * hd, dtype=td, device="cuda")
+    b = B.Batch(q_lens, ctx, lay.block_table, torch.zeros(n, m.d_model, device="cuda"))
+    bl.op_attention(b, 0, torch.from_numpy(q.astype(np.float32)).to("cuda", td), o, kind=kind)
+    got = o.float().cpu().numpy()
+    pk, pv = pk_cpu.numpy(), pv_cpu.numpy()
+    grp = H // m.n_kv_heads
+    row = 0
+    worst = 0.0
+    for r, (ql, cl) in enumerate(zip(q_lens, ctx)):
+        for i in range(ql):
+            if ql > 20 and i % 7 not in (0, 6) and i != ql - 1:
+                row += 1
+                continue            # sample prefill rows (keeps the test fast)
+            for h in range(H):
+                ref = O.attend_paged(q[row, h * hd:(h + 1) * hd], pk, pv, lay.block_table[r], 16,
+                                     h // grp, cl + i)
+                worst = max(worst, float(np.abs(got[row, h * hd:(h + 1) * hd] - ref).max()))
+            row += 1
+    assert worst < (1.6e-2 if m.dtype == "bf16" else 2e-5), worst

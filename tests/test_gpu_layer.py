@@ -1,0 +1,138 @@
+"""bullet_step parity (co-run prefill + decode layer step) vs the CPU oracle,
+SM-gating invariants from the smid log, and error paths.  Needs a B200."""
+import numpy as np
+import pytest
+import torch
+
+from workload import synth
+from harness import Setup, compare
+from oracle import perfmodel as PM
+
+pytestmark = pytest.mark.gpu
+
+
+def _run(S, p, flags):
+    B = S.B
+    pre, dec = S.batches()
+    sp, sd = torch.cuda.Stream(), torch.cuda.Stream()
+    S.bl.step(pre, dec, p, flags, sp, sd)
+    torch.cuda.synchronize()
+    return pre, dec
+
+
+@pytest.fixture(scope="module")
+def tiny():
+    """BASELINE config 1: tiny 2-layer fp32 model, 1 x 128 prefill + 4 decodes
+    with 64 cached tokens, paged KV block 16 (DESIGN R-6, R-7)."""
+    wl = synth.workload("tiny")
+    S = Setup(synth.MODELS["tiny"], wl.prefill_lens, wl.decode_ctx, n_layers=2)
+    return S, S.oracle()
+
+
+@pytest.mark.parametrize("mode", ["corun", "timesliced", "ungated"])
+def test_tiny_fp32_two_layers(tiny, mode):
+    S, ref = tiny
+    B = S.B
+    flags = {"corun": B.CORUN, "timesliced": B.TIMESLICED, "ungated": B.UNGATED}[mode]
+    pre, dec = _run(S, 74, flags)
+    for name, b in (("pre", pre), ("dec", dec)):
+        mx, mr = compare(b.hidden.cpu().numpy(), ref[name])
+        assert mx <= 1e-4 and mr <= 1e-5, (name, mx, mr)
+
+
+@pytest.fixture(scope="module")
+def small_bf16():
+    m = synth.ModelShape("small-bf16", 1024, 8, 2, 128, 2816, 2)
+    S = Setup(m, [300, 77, 1], [64, 1, 500, 31, 16, 1000], n_layers=2)
+    return S, S.oracle()
+
+
+@pytest.mark.parametrize("p", [2, 64, 146])
+def test_small_bf16_corun_splits(small_bf16, p):
+    """Reduced Llama-style bf16 model (hd 128, GQA 4), two layers, ragged
+    prefill lengths: co-run at edge and middle splits meets the bar."""
+    S, ref = small_bf16
+    pre, dec = _run(S, p, S.B.CORUN)
+    for name, b in (("pre", pre), ("dec", dec)):
+        mx, mr = compare(b.hidden.cpu().numpy(), ref[name])
+        assert mx <= 2e-2 and mr <= 1e-3, (name, p, mx, mr)
+
+
+def test_small_bf16_timesliced(small_bf16):
+    S, ref = small_bf16
+    pre, dec = _run(S, 148, S.B.TIMESLICED)
+    for name, b in (("pre", pre), ("dec", dec)):
+        mx, mr = compare(b.hidden.cpu().numpy(), ref[name])
+        assert mx <= 2e-2 and mr <= 1e-3, (name, mx, mr)
+
+
+def test_llama8b_config2_layer_sampled():
+    """BASELINE config 2 at full Llama-3.1-8B layer dims (8 ShareGPT-shaped
+    prefills summing to 4096 tokens + 128 decodes with 512-1536 cached
+    tokens), one layer, the launch configuration bench.py times (co-run at
+    the default split).  Oracle: all 128 decode rows and 64 sampled prefill
+    rows incl. the last row of every request."""
+    wl = synth.workload("sharegpt-8b")
+    S = Setup(synth.MODELS["llama3.1-8b"], wl.prefill_lens, wl.decode_ctx, n_layers=1)
+    n_p = sum(wl.prefill_lens)
+    rng = np.random.default_rng(0)
+    mask = np.zeros(n_p, np.uint8)
+    mask[rng.choice(n_p, 48, replace=False)] = 1
+    mask[np.cumsum(wl.prefill_lens) - 1] = 1
+    ref = S.oracle(row_mask_pre=mask)
+    pre, dec = _run(S, 104, S.B.CORUN)
+    mx, mr = compare(dec.hidden.cpu().numpy(), ref["dec"])
+    assert mx <= 2e-2 and mr <= 1e-3, ("dec", mx, mr)
+    got = pre.hidden.cpu().numpy()[mask == 1]
+    mx, mr = compare(got, ref["pre"][mask == 1])
+    assert mx <= 2e-2 and mr <= 1e-3, ("pre", mx, mr)
+
+
+@pytest.mark.parametrize("p", [2, 40, 146])
+def test_smid_gating_invariants(small_bf16, p):
+    """SM-range work assignment (§8a SG), bit-exact invariants: every work
+    unit of every launch ran exactly once, on an SM of its phase's range;
+    ranges = sigma[0:p) / sigma[p:N) (oracle range function)."""
+    S, _ = small_bf16
+    B = S.B
+    log = S.bl.set_smid_log(400000)
+    try:
+        _run(S, p, B.CORUN | B.SMID_LOG)
+        n = int(log[0].item())
+        assert 0 < n <= 400000
+        e = log[1:1 + 4 * n].view(n, 4).cpu().numpy()
+    finally:
+        S.bl.set_smid_log(None)
+    sigma = S.bl.sm_order()
+    pre_set, dec_set = map(set, PM.sm_ranges(p, sigma))
+    for launch in np.unique(e[:, 0]):
+        rows = e[e[:, 0] == launch]
+        phase = rows[0, 3]
+        assert np.all(rows[:, 3] == phase)
+        units = rows[:, 1]
+        assert len(np.unique(units)) == len(units), "unit executed twice"
+        assert units.min() == 0 and units.max() == len(units) - 1, "unit skipped"
+        allowed = pre_set if phase == 0 else dec_set
+        assert set(rows[:, 2].tolist()) <= allowed, (launch, phase)
+
+
+def test_decode_pause_and_errors(small_bf16):
+    S, _ = small_bf16
+    B = S.B
+    pre, dec = S.batches()
+    x0 = dec.hidden.clone()
+    S.bl.step(pre, dec, S.bl.n_sms, B.CORUN)          # p = N: decode paused
+    torch.cuda.synchronize()
+    assert torch.equal(dec.hidden, x0)
+    with pytest.raises(B.BulletError) as e:
+        S.bl.step(pre, dec, 0, B.CORUN)
+    assert e.value.code == -4
+    with pytest.raises(B.BulletError) as e:
+        S.bl.step(pre, dec, 3, B.CORUN)
+    assert e.value.code == -4
+    bad = S.lay.block_table[S.n_pre:].copy()
+    bad[0, 0] = S.lay.n_blocks + 5
+    dec_bad = B.Batch([1] * len(S.decode_ctx), S.decode_ctx, bad, dec.hidden)
+    with pytest.raises(B.BulletError) as e:
+        S.bl.step(None, dec_bad, 0, B.CORUN)
+    assert e.value.code == -5
