@@ -1,0 +1,432 @@
+#!/usr/bin/env python
+"""bench.py — Bullet co-run layer step on B200 (BASELINE.json metric:
+"co-run tokens/s/GPU vs time-sliced; decode HBM GB/s; prefill tensor-pipe util").
+
+A step = one pass of the whole hot path over one synthetic batch: the
+prefill batch through one layer on stream P, concurrently with the decode
+batch through k layer-steps on stream D, on disjoint SM ranges (bullet_step
+BULLET_CORUN).  tokens/s = (n_prefill_tokens * 1 + n_decode * k) / (L_model * T)
+(each token-layer counts 1/L_model of a token).  The same work
+is also timed time-sliced (BULLET_TIMESLICED: prefill then decode, all SMs).
+
+    python bench.py [--gpus N --steps K --warmup W] [--config sharegpt-8b]
+    python bench.py --impl reference      # the CPU oracle arm (rank 0 only)
+
+Prints ONE JSON line (rank 0).  Inputs: random-init weights of the named
+architecture, synthetic request mixes (workload/synth.py).  The per-step
+working set (weights + KV, GBs) is far larger than the 126 MB L2, so no L2
+flush is needed between steps.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from workload import synth  # noqa: E402
+
+PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d, "measured"
+    return PEAKS_FALLBACK, "fallback"
+
+
+# ---------------------------------------------------------------- dist utils
+def dist_init():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if ws > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    elif torch.cuda.is_available():
+        torch.cuda.set_device(0)
+    return ws, rank
+
+
+def barrier(ws):
+    if ws > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+def allreduce_max(x, ws):
+    if ws == 1:
+        return x
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+# ---------------------------------------------------------------- clocks
+class Clocks:
+    """nvidia-smi sampled every 200 ms during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, dev):
+        self.dev = dev
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.dev), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.p = None
+        return self
+
+    def __exit__(self, *a):
+        self.out = ""
+        if self.p:
+            time.sleep(0.25)
+            self.p.terminate()
+            try:
+                self.out, _ = self.p.communicate(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.p.kill()
+
+    def summary(self):
+        rows = [r.split(", ") for r in (self.out or "").strip().splitlines() if r.count(",") >= 5]
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(r[0]) for r in rows if r[0].strip().replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].strip().replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if "Active" == r[2 + i].strip()})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows)}
+
+
+# ---------------------------------------------------------------- workload
+class Step:
+    def __init__(self, config: str, k_max: int, device="cuda"):
+        import paper_conf_asplos_0001xc0l026_b200 as B
+        self.B = B
+        self.wl = synth.workload(config)
+        self.m = synth.MODELS[self.wl.model]
+        if self.wl.tp != 1:
+            raise SystemExit(f"config {config} needs tensor parallelism (tp={self.wl.tp}); "
+                             "bench.py runs it only under torchrun with WORLD_SIZE == tp")
+        m = self.m
+        self.k_max = k_max
+        n_layers = max(1, k_max)
+        q, c, self.n_pre = synth.combined_batch(self.wl)
+        self.lay = synth.paged_layout(q, c, 16)
+        self.n_p = sum(self.wl.prefill_lens)
+        self.n_d = len(self.wl.decode_ctx)
+        td = torch.bfloat16 if m.dtype == "bf16" else torch.float32
+        self.pools, self.weights = [], []
+        for l in range(n_layers):
+            w = synth.layer_weights(m, l, device=device)
+            self.weights.append({k: (None if v is None else v.to(td)) for k, v in w.items()})
+            del w
+            k_, v_ = synth.kv_pool(m, self.lay.n_blocks, 16, l, device=device)
+            self.pools.append((k_.to(td), v_.to(td)))
+            del k_, v_
+        torch.cuda.empty_cache()
+        maxpos = max(a + b for a, b in zip(q, c)) + 16
+        self.bl = B.Bullet(B.Model.of(m), self.pools, self.n_p, self.n_d, maxpos)
+        for l in range(n_layers):
+            self.bl.set_layer_weights(l, self.weights[l])
+        bt = self.lay.block_table
+        self.x_pre = synth.hidden(self.n_p, m.d_model, 0, device=device)
+        self.x_dec = synth.hidden(self.n_d, m.d_model, 1, device=device)
+        self.pre = B.Batch(self.wl.prefill_lens, [0] * self.n_pre, bt[:self.n_pre], self.x_pre, 0, 1)
+        self.dec = B.Batch([1] * self.n_d, self.wl.decode_ctx, bt[self.n_pre:], self.x_dec, 0, 1)
+        self.sp, self.sd = torch.cuda.Stream(), torch.cuda.Stream()
+        self.N = self.bl.n_sms
+
+    def enqueue(self, p, flags, pre=True, dec=True):
+        """One step: both streams start together and join at the end."""
+        ev = torch.cuda.Event()
+        ev.record(self.sp)
+        self.sd.wait_event(ev)
+        self.bl.step(self.pre if pre else None, self.dec if dec else None, p, flags, self.sp, self.sd)
+        ev2 = torch.cuda.Event()
+        ev2.record(self.sd)
+        self.sp.wait_event(ev2)
+
+    def time_steps(self, n, p, flags, pre=True, dec=True):
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(self.sp)
+        for _ in range(n):
+            self.enqueue(p, flags, pre, dec)
+        e1.record(self.sp)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / n
+
+    def tokens(self, k):
+        return (self.n_p * 1 + self.n_d * k) / self.m.n_layers
+
+    def tune(self, cands, reps=3):
+        """Isolated prefill layer on p SMs and decode layer-step on N-p SMs;
+        k = round(T_p / T_d); pick the p with the best predicted co-run
+        throughput (the model's (u_k, k) choice, measured instead of fitted)."""
+        B = self.B
+        self.dec.layer_end = 1
+        res = []
+        for p in cands:
+            self.time_steps(1, p, B.CORUN, dec=False)
+            tp = self.time_steps(reps, p, B.CORUN, dec=False)
+            self.time_steps(1, p, B.CORUN, pre=False)
+            td = self.time_steps(reps, p, B.CORUN, pre=False)
+            k = int(min(self.k_max, max(1, round(tp / td))))
+            est = self.tokens(k) / max(tp, k * td)
+            res.append({"p": p, "t_prefill_ms": tp, "t_decode_ms": td, "k": k, "est_tok_s": est * 1e3})
+        best = max(res, key=lambda r: r["est_tok_s"])
+        return best, res
+
+
+# ---------------------------------------------------------------- roofline
+def kernel_work(S: Step, kind: str, phase: int):
+    """Algorithmic flops (tensor) or bytes (hbm) of ONE launch."""
+    m = S.m
+    d, H, Hkv, hd, I = m.d_model, m.n_heads, m.n_kv_heads, m.head_dim, m.d_ff
+    nq = (H + 2 * Hkv) * hd
+    n = S.n_p if phase == 0 else S.n_d
+    if kind == "qkv":
+        return "tensor", 2.0 * n * d * nq
+    if kind == "o_proj":
+        return "tensor", 2.0 * n * H * hd * d
+    if kind == "gate_up":
+        return "tensor", 2.0 * n * d * 2 * I
+    if kind == "down":
+        return "tensor", 2.0 * n * I * d
+    if kind == "attn":
+        if phase == 0:
+            pairs = sum(s * (s + 1) // 2 for s in S.wl.prefill_lens)
+            return "tensor", 4.0 * hd * H * pairs
+        keys = sum(c + 1 for c in S.wl.decode_ctx)
+        return "hbm", 2.0 * 2 * Hkv * hd * keys + 2.0 * 2 * n * H * hd
+    if kind in ("rmsnorm1", "rmsnorm2"):
+        return "hbm", 4.0 * n * d + 2.0 * n * d
+    if kind == "rope_kv":
+        return "hbm", 4.0 * n * nq + 2.0 * n * nq
+    return "hbm", 0.0
+
+
+# ---------------------------------------------------------------- CPU oracle
+def oracle_sample(m: synth.ModelShape, wl: synth.Workload, n_pre_tok=64, n_dec=32):
+    """Bounded sample of the same workload for the CPU oracle: one prefill
+    request of n_pre_tok tokens + the first n_dec decode requests, one layer.
+    Returns (seconds, tokens) with tokens in the metric's unit."""
+    import oracle as O
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    from harness import oracle_cfg
+    q = [n_pre_tok] + [1] * n_dec
+    c = [0] + list(wl.decode_ctx[:n_dec])
+    lay = synth.paged_layout(q, c, 16)
+    w = {k: (None if v is None else v.numpy()) for k, v in synth.layer_weights(m, 0).items()}
+    pk, pv = synth.kv_pool(m, lay.n_blocks, 16, 0)
+    pk, pv = pk.numpy(), pv.numpy()
+    x = synth.hidden(sum(q), m.d_model).double().numpy()
+    t0 = time.perf_counter()
+    O.layer_forward(oracle_cfg(m), w, pk, pv, q, c, lay.block_table, x)
+    dt = time.perf_counter() - t0
+    return dt, (n_pre_tok + n_dec) / m.n_layers, f"1 layer: 1 prefill x {n_pre_tok} tok + {n_dec} decodes (ctx {min(c[1:])}-{max(c[1:])})"
+
+
+def run_reference(args, ws, rank):
+    if rank != 0:
+        return
+    wl = synth.workload(args.config)
+    m = synth.MODELS[wl.model]
+    for _ in range(args.warmup):
+        oracle_sample(m, wl)
+    ts, toks = [], 0.0
+    for _ in range(args.steps):
+        dt, tk, desc = oracle_sample(m, wl)
+        ts.append(dt)
+        toks = tk
+    T = sum(ts) / len(ts)
+    v = toks / T
+    cores = os.cpu_count()
+    print(json.dumps({
+        "impl": "reference", "metric": "co-run tokens/s/GPU vs time-sliced", "value": v,
+        "unit": "tokens/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": T * 1e3, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "f64", "data": "synthetic",
+        "config": {"workload": args.config, "model": wl.model, "sample": desc},
+        "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": cores, "kind": "oracle", "sample": desc},
+        "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}))
+
+
+# ---------------------------------------------------------------- main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="bullet", choices=["bullet", "reference"])
+    ap.add_argument("--config", default="sharegpt-8b")
+    ap.add_argument("--p", type=int, default=None, help="prefill SM count (default: tuned)")
+    ap.add_argument("--k", type=int, default=None, help="decode layer-steps per prefill layer")
+    ap.add_argument("--k-max", type=int, default=16)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--sweep", action="store_true", help="also print the p sweep (stderr)")
+    args = ap.parse_args()
+    ws, rank = dist_init()
+    if args.impl == "reference":
+        run_reference(args, ws, rank)
+        return
+    args.warmup = max(args.warmup, 3)
+    import paper_conf_asplos_0001xc0l026_b200 as B
+    S = Step(args.config, args.k_max)
+    N = S.N
+    # ---- choose the split (p, k)
+    if args.p is None or args.k is None:
+        cands = [args.p] if args.p else list(range(72, N - 15, 8))
+        best, table = S.tune(cands)
+        p = args.p or best["p"]
+        k = args.k or best["k"]
+        if args.sweep and rank == 0:
+            for r in table:
+                print(json.dumps(r), file=sys.stderr)
+    else:
+        p, k, table = args.p, args.k, []
+    S.dec.layer_end = k
+    # ---- alone-on-full-GPU references (per layer)
+    t_pre_full = S.time_steps(3, N, B.CORUN, dec=False)
+    S.dec.layer_end = 1
+    t_dec_full = S.time_steps(3, 0, B.CORUN, pre=False)
+    S.dec.layer_end = k
+    # ---- co-run (the method) and time-sliced, device-timed, max over ranks
+    for _ in range(args.warmup):
+        S.enqueue(p, B.CORUN)
+    barrier(ws)
+    torch.cuda.synchronize()
+    l0 = S.bl.launch_count()
+    with Clocks(torch.cuda.current_device()) as clk:
+        t_co = S.time_steps(args.steps, p, B.CORUN)
+    launches = S.bl.launch_count() - l0
+    barrier(ws)
+    t_co = allreduce_max(t_co, ws)
+    for _ in range(args.warmup):
+        S.enqueue(N, B.TIMESLICED)
+    barrier(ws)
+    t_ts = allreduce_max(S.time_steps(args.steps, N, B.TIMESLICED), ws)
+    # ---- profiled pass: per-kernel device times inside the co-run step
+    S.time_steps(2, p, B.CORUN | B.PROFILE)
+    prof = S.bl.profile_read()
+    by = {}
+    for kind, ph, layer, ms in prof:
+        by.setdefault((kind, ph), []).append(ms)
+    total = {key: sum(v) for key, v in by.items()}
+    dom = max(total, key=total.get)
+    bound, work = kernel_work(S, dom[0], dom[1])
+    avg_ms = float(np.mean(by[dom]))
+    P, src = peaks()
+    if bound == "tensor":
+        achieved = work / (avg_ms * 1e-3) / 1e12
+        peak, unit = P.get("bf16_tflops_sustained", P["bf16_tflops"]), "TFLOP/s"
+    else:
+        achieved = work / (avg_ms * 1e-3) / 1e9
+        peak, unit = P["hbm_gbs"], "GB/s"
+    # ---- e2e: host buffers through the C ABI, copies inside the timed region
+    h_pre = torch.empty_like(S.x_pre, device="cpu").pin_memory()
+    h_dec = torch.empty_like(S.x_dec, device="cpu").pin_memory()
+    h_pre.copy_(S.x_pre); h_dec.copy_(S.x_dec)
+    o_pre = torch.empty_like(h_pre).pin_memory(); o_dec = torch.empty_like(h_dec).pin_memory()
+    meta = [(torch.from_numpy(b.cu).pin_memory(), b.d_cu) for b in (S.pre, S.dec)] + \
+           [(torch.from_numpy(b.ctx_lens).pin_memory(), b.d_ctx) for b in (S.pre, S.dec)] + \
+           [(torch.from_numpy(b.block_table).pin_memory(), b.d_bt) for b in (S.pre, S.dec)]
+    h2d = h_pre.numel() * 4 + h_dec.numel() * 4 + sum(h.numel() * 4 for h, _ in meta)
+    d2h = o_pre.numel() * 4 + o_dec.numel() * 4
+
+    def e2e_step():
+        with torch.cuda.stream(S.sp):
+            S.x_pre.copy_(h_pre, non_blocking=True)
+            for h, d in meta:
+                d.copy_(h, non_blocking=True)
+        with torch.cuda.stream(S.sd):
+            S.x_dec.copy_(h_dec, non_blocking=True)
+        ev = torch.cuda.Event(); ev.record(S.sp); S.sd.wait_event(ev)
+        S.bl.step(S.pre, S.dec, p, B.CORUN, S.sp, S.sd)
+        with torch.cuda.stream(S.sp):
+            o_pre.copy_(S.x_pre, non_blocking=True)
+        with torch.cuda.stream(S.sd):
+            o_dec.copy_(S.x_dec, non_blocking=True)
+        ev2 = torch.cuda.Event(); ev2.record(S.sd); S.sp.wait_event(ev2)
+
+    for _ in range(args.warmup):
+        e2e_step()
+    barrier(ws)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(S.sp)
+    for _ in range(args.steps):
+        e2e_step()
+    e1.record(S.sp)
+    torch.cuda.synchronize()
+    t_e2e = allreduce_max(e0.elapsed_time(e1) / args.steps, ws)
+    # ---- report
+    tok = S.tokens(k)
+    value = ws * tok / (t_co * 1e-3)
+    ts_value = ws * tok / (t_ts * 1e-3)
+    m = S.m
+    nq = (m.n_heads + 2 * m.n_kv_heads) * m.head_dim
+    w_bytes = 2.0 * (nq * m.d_model + m.d_model * m.n_heads * m.head_dim + 3 * m.d_model * m.d_ff)
+    f_pre = 2.0 * S.n_p * w_bytes / 2 + kernel_work(S, "attn", 0)[1]
+    b_dec = k * (w_bytes + kernel_work(S, "attn", 1)[1])
+    out = {
+        "metric": "co-run tokens/s/GPU vs time-sliced; decode HBM GB/s; prefill tensor-pipe util",
+        "value": value, "unit": "tokens/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": t_co, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "bf16" if m.dtype == "bf16" else "fp32", "data": "synthetic (random-init weights, seeded request mix)",
+        "config": {"workload": args.config, "model": S.wl.model, "prefill_tokens": S.n_p,
+                   "prefill_reqs": S.n_pre, "decode_reqs": S.n_d,
+                   "decode_ctx_mean": float(np.mean(S.wl.decode_ctx)), "prefill_layers_per_step": 1,
+                   "decode_layer_steps": k, "prefill_sm_count": p, "n_sms": N,
+                   "parallelism": f"replicas x{ws}" if ws > 1 else "single GPU",
+                   "l2": "inputs larger than L2 (weights + KV per step >> 126 MB)"},
+        "timesliced": {"value": ts_value, "ms_per_step": t_ts},
+        "corun_speedup_vs_timesliced": t_ts / t_co,
+        "phase_alone_full_gpu_ms": {"prefill_layer": t_pre_full, "decode_layer": t_dec_full},
+        "phase_roofline_corun": {
+            "prefill_tensor_frac": f_pre / (t_co * 1e-3) / (P.get("bf16_tflops_sustained", 1395.1) * 1e12),
+            "decode_hbm_frac": b_dec / (t_co * 1e-3) / (P["hbm_gbs"] * 1e9),
+            "decode_hbm_gbs": b_dec / (t_co * 1e-3) / 1e9},
+        "roofline": {"bound": bound, "kernel": f"{dom[0]} ({'prefill' if dom[1] == 0 else 'decode'})",
+                     "achieved": achieved, "peak": peak, "unit": unit, "frac": achieved / peak,
+                     "peak_source": src, "avg_launch_ms": avg_ms, "traffic": None},
+        "kernel_ms": {f"{k_}/{'pre' if ph == 0 else 'dec'}": round(sum(v) / 2, 4) for (k_, ph), v in by.items()},
+        "e2e": {"value": ws * tok / (t_e2e * 1e-3), "unit": "tokens/s", "h2d_bytes_per_step": int(h2d),
+                "d2h_bytes_per_step": int(d2h), "ms_per_step": t_e2e},
+        "gpu_launches": int(launches),
+        "clocks": clk.summary(),
+        "tuning": table,
+    }
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        dt, tk, desc = oracle_sample(S.m, S.wl)
+        out["cpu_baseline"] = {"value": tk / dt, "unit": "tokens/s", "cores": os.cpu_count(),
+                               "kind": "oracle", "sample": desc}
+    if rank == 0:
+        print(json.dumps(out))
+    if ws > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -58,7 +58,15 @@ enum {
   BULLET_CORUN = 0,          /* phases concurrently on disjoint SM ranges (the method) */
   BULLET_TIMESLICED = 1,     /* same kernels on all SMs, prefill then decode (baseline) */
   BULLET_UNGATED = 2,        /* both phases concurrently on all SMs ("Naive") */
-  BULLET_SMID_LOG = 4        /* record (launch, tile, smid) of every work unit */
+  BULLET_SMID_LOG = 4,       /* record (launch, tile, smid) of every work unit */
+  BULLET_PROFILE = 8         /* CUDA events around every kernel (bullet_profile_read) */
+};
+
+/* Kernel kinds reported by bullet_profile_read. */
+enum {
+  BULLET_K_PLAN = 0, BULLET_K_RMSNORM1 = 1, BULLET_K_QKV = 2, BULLET_K_ROPE_KV = 3,
+  BULLET_K_ATTN = 4, BULLET_K_OPROJ = 5, BULLET_K_RMSNORM2 = 6, BULLET_K_GATE_UP = 7,
+  BULLET_K_DOWN = 8, BULLET_K_ALLREDUCE = 9
 };
 
 /* Model shape (per GPU under tensor parallelism: n_heads, n_kv_heads and
@@ -212,6 +220,17 @@ int bullet_choose_split(const bullet_handle *h, const bullet_sched_state *s, con
  * [1 + 4*capacity]; entry i = {launch_id, unit, smid, phase}; element 0 is
  * the entry counter (caller zeroes it).  NULL disables. */
 int bullet_set_smid_log(bullet_handle *h, int32_t *d_log, int capacity);
+
+/* Per-kernel device times of every launch made by bullet_step calls with
+ * BULLET_PROFILE since the last read (oldest first): kind (BULLET_K_*),
+ * phase (0 prefill, 1 decode), layer, milliseconds between CUDA events
+ * recorded on the launching stream around the kernel.  Synchronizes on the
+ * events; *n = number written (<= cap); the list is then cleared. */
+int bullet_profile_read(bullet_handle *h, int32_t *kind, int32_t *phase, int32_t *layer, float *ms,
+                        int cap, int *n);
+
+/* Total kernels this handle has launched (all entry points). */
+int bullet_launch_count(const bullet_handle *h, long long *n);
 
 /* Block until all work the handle enqueued has finished; surfaces
  * asynchronous CUDA / NCCL errors. */

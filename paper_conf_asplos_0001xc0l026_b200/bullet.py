@@ -17,7 +17,9 @@ c_int, c_double, c_float, c_void_p = ctypes.c_int, ctypes.c_double, ctypes.c_flo
 P_i32 = ctypes.POINTER(ctypes.c_int32)
 P_f64 = ctypes.POINTER(ctypes.c_double)
 
-CORUN, TIMESLICED, UNGATED, SMID_LOG = 0, 1, 2, 4
+CORUN, TIMESLICED, UNGATED, SMID_LOG, PROFILE = 0, 1, 2, 4, 8
+KERNEL_KINDS = ["plan", "rmsnorm1", "qkv", "rope_kv", "attn", "o_proj", "rmsnorm2", "gate_up",
+                "down", "allreduce"]
 DTYPE_FP32, DTYPE_BF16 = 0, 1
 EPI_F32, EPI_RESID, EPI_SILU = 0, 1, 2
 ERRORS = {0: "OK", -1: "EINVAL", -2: "ECUDA", -3: "ENCCL", -4: "ESMRANGE", -5: "EKV",
@@ -85,7 +87,8 @@ def lib():
         for name in ("bullet_create", "bullet_perf_create", "bullet_set_layer_weights", "bullet_num_sms", "bullet_sm_order",
                      "bullet_step", "bullet_model_predict", "bullet_choose_split",
                      "bullet_set_smid_log", "bullet_sync", "bullet_nccl_unique_id", "bullet_op_gemm",
-                     "bullet_op_rmsnorm", "bullet_op_rope_kv", "bullet_op_attention"):
+                     "bullet_op_rmsnorm", "bullet_op_rope_kv", "bullet_op_attention",
+                     "bullet_profile_read", "bullet_launch_count"):
             getattr(L, name).restype = c_int
         L.bullet_create.argtypes = [ctypes.POINTER(ModelCfg), ctypes.POINTER(KvPool), c_void_p,
                                     ctypes.c_char_p, ctypes.POINTER(c_void_p)]
@@ -101,6 +104,9 @@ def lib():
                                           ctypes.POINTER(c_int), ctypes.POINTER(c_int)]
         L.bullet_set_smid_log.argtypes = [c_void_p, c_void_p, c_int]
         L.bullet_sync.argtypes = [c_void_p]
+        L.bullet_profile_read.argtypes = [c_void_p, P_i32, P_i32, P_i32, ctypes.POINTER(c_float), c_int,
+                                          ctypes.POINTER(c_int)]
+        L.bullet_launch_count.argtypes = [c_void_p, ctypes.POINTER(ctypes.c_longlong)]
         L.bullet_nccl_unique_id.argtypes = [c_void_p]
         L.bullet_destroy.argtypes = [c_void_p]
         L.bullet_destroy.restype = None
@@ -274,6 +280,18 @@ class Bullet:
 
     def sync(self):
         _check(lib().bullet_sync(self.h))
+
+    def profile_read(self, cap=1 << 16):
+        """[(kind name, phase, layer, ms)] of launches made with PROFILE since the last read."""
+        k = (ctypes.c_int32 * cap)(); p = (ctypes.c_int32 * cap)(); l = (ctypes.c_int32 * cap)()
+        ms = (c_float * cap)(); n = c_int()
+        _check(lib().bullet_profile_read(self.h, k, p, l, ms, cap, ctypes.byref(n)))
+        return [(KERNEL_KINDS[k[i]], p[i], l[i], ms[i]) for i in range(n.value)]
+
+    def launch_count(self) -> int:
+        n = ctypes.c_longlong()
+        _check(lib().bullet_launch_count(self.h, ctypes.byref(n)))
+        return n.value
 
     def predict_us(self, q_lens, ctx_lens, sm_count, corun_sm_count=0) -> float:
         q = np.ascontiguousarray(q_lens, dtype=np.int32); c = np.ascontiguousarray(ctx_lens, dtype=np.int32)

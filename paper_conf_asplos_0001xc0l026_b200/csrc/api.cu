@@ -131,6 +131,12 @@ struct bullet_handle {
   ncclComm_t comm[2] = {nullptr, nullptr};
   cudaEvent_t ev_ts = nullptr;
   bool host_only = false;  // bullet_perf_create: perf model only
+  // BULLET_PROFILE: events around every launch
+  struct ProfRec { int kind, phase, layer; cudaEvent_t e0, e1; };
+  std::vector<ProfRec> prof_recs;
+  std::vector<cudaEvent_t> ev_pool;
+  size_t ev_used = 0;
+  long long n_launch = 0;
 };
 
 namespace {
@@ -153,9 +159,43 @@ struct Ctx {  // one phase's launch context within a call
   bool log;
   cudaStream_t st;
   bool op;     // op-level entry: counter = op_ctr, zeroed before each launch
+  bool prof = false;
+  int kind = 0, layer = -1;
 };
 
+constexpr size_t MAX_PROF = 1 << 16;
+
+cudaEvent_t take_event(bullet_handle* h) {
+  if (h->ev_used == h->ev_pool.size()) {
+    cudaEvent_t e;
+    if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+    h->ev_pool.push_back(e);
+  }
+  return h->ev_pool[h->ev_used++];
+}
+
+void prof_begin(Ctx& c) {
+  bullet_handle* h = c.h;
+  h->n_launch++;
+  if (!c.prof || h->prof_recs.size() >= MAX_PROF) return;
+  bullet_handle::ProfRec r{c.kind, c.phase, c.layer, take_event(h), take_event(h)};
+  if (!r.e0 || !r.e1) return;
+  cudaEventRecord(r.e0, c.st);
+  h->prof_recs.push_back(r);
+}
+
+void prof_end(Ctx& c) {
+  if (c.prof && !c.h->prof_recs.empty()) cudaEventRecord(c.h->prof_recs.back().e1, c.st);
+}
+
+#define LAUNCH(c, x)  \
+  do {                \
+    CK(x);            \
+    prof_end(c);      \
+  } while (0)
+
 int next_launch(Ctx& c, Launch* L) {
+  prof_begin(c);
   memset(L, 0, sizeof *L);
   L->gate = c.gate;
   L->log = c.log ? c.h->log : nullptr;
@@ -187,7 +227,7 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   if (h->cfg.dtype == BULLET_DTYPE_FP32) {
     if (K % 16) return set_err(BULLET_EUNSUPPORTED, "fp32 GEMM needs K %% 16 == 0");
     a.bn = 64; a.splits = 1;
-    CK(launch_gemm_simt<float>((const float*)A, (const float*)B, a, h->n_sms * 4, c.st));
+    LAUNCH(c, launch_gemm_simt<float>((const float*)A, (const float*)B, a, h->n_sms * 4, c.st));
     return BULLET_OK;
   }
   if (K % 64) return set_err(BULLET_EUNSUPPORTED, "GEMM needs K %% 64 == 0 (K=%d)", K);
@@ -215,7 +255,7 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   CUtensorMap ma, mb;
   if ((rc = make_map(&ma, A, M, K, 128))) return rc;
   if ((rc = make_map(&mb, B, N, K, bn / 2))) return rc;
-  CK(launch_gemm_tc(ma, mb, a, h->n_sms, c.st));
+  LAUNCH(c, launch_gemm_tc(ma, mb, a, h->n_sms, c.st));
   return BULLET_OK;
 }
 
@@ -225,8 +265,8 @@ int do_rmsnorm(Ctx& c, const float* x, int n, const void* g, void* out) {
   a.x = x; a.g = g; a.out = out; a.n = n; a.d = c.h->cfg.d_model; a.eps = c.h->cfg.rms_eps;
   int rc = next_launch(c, &a.L);
   if (rc) return rc;
-  if (c.h->cfg.dtype == BULLET_DTYPE_FP32) CK(launch_rmsnorm<float>(a, c.h->n_sms * 8, c.st));
-  else CK(launch_rmsnorm<__nv_bfloat16>(a, c.h->n_sms * 8, c.st));
+  if (c.h->cfg.dtype == BULLET_DTYPE_FP32) LAUNCH(c, launch_rmsnorm<float>(a, c.h->n_sms * 8, c.st));
+  else LAUNCH(c, launch_rmsnorm<__nv_bfloat16>(a, c.h->n_sms * 8, c.st));
   return BULLET_OK;
 }
 
@@ -241,8 +281,8 @@ int do_rope(Ctx& c, const bullet_batch* b, int layer, const float* qkv, void* q)
   a.max_pos = h->cfg.max_position;
   int rc = next_launch(c, &a.L);
   if (rc) return rc;
-  if (h->cfg.dtype == BULLET_DTYPE_FP32) CK(launch_rope_kv<float>(a, h->n_sms * 8, c.st));
-  else CK(launch_rope_kv<__nv_bfloat16>(a, h->n_sms * 8, c.st));
+  if (h->cfg.dtype == BULLET_DTYPE_FP32) LAUNCH(c, launch_rope_kv<float>(a, h->n_sms * 8, c.st));
+  else LAUNCH(c, launch_rope_kv<__nv_bfloat16>(a, h->n_sms * 8, c.st));
   return BULLET_OK;
 }
 
@@ -270,24 +310,27 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     a.tiles = P.tiles; a.n_tiles = P.n_tiles;
     if (c.op) {  // op-level: plan the tile list now
       PlanArgs pa{nullptr, 0, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ, P.tiles, P.n_tiles};
-      CK(launch_plan(pa, c.st));
+      prof_begin(c);
+      LAUNCH(c, launch_plan(pa, c.st));
     }
     int rc = next_launch(c, &a.L);
     if (rc) return rc;
-    CK(launch_attn_prefill_tc(a, h->n_sms * 2, c.st));
+    LAUNCH(c, launch_attn_prefill_tc(a, h->n_sms * 2, c.st));
     return BULLET_OK;
   }
   int rc = next_launch(c, &a.L);
   if (rc) return rc;
-  if (bf16) CK(launch_attn_simt<__nv_bfloat16>(a, h->n_sms * 4, c.st));
-  else CK(launch_attn_simt<float>(a, h->n_sms * 4, c.st));
+  if (bf16) LAUNCH(c, launch_attn_simt<__nv_bfloat16>(a, h->n_sms * 4, c.st));
+  else LAUNCH(c, launch_attn_simt<float>(a, h->n_sms * 4, c.st));
   return BULLET_OK;
 }
 
 int allreduce(Ctx& c, float* buf, size_t count) {
   bullet_handle* h = c.h;
+  prof_begin(c);
   ncclResult_t r = g_nccl.allReduce(buf, buf, count, ncclFloat32, ncclSum, h->comm[c.phase], c.st);
   if (r != ncclSuccess) return set_err(BULLET_ENCCL, "ncclAllReduce: %s", g_nccl.errStr(r));
+  prof_end(c);
   return BULLET_OK;
 }
 
@@ -301,19 +344,30 @@ int run_layer(Ctx& c, const bullet_batch* b, int layer) {
   const int I = cf.d_ff, nq = (H + 2 * Hkv) * hd;
   const bool tp = cf.tp_size > 1, lead = cf.tp_rank == 0;
   int rc;
+  c.layer = layer;
+  c.kind = BULLET_K_RMSNORM1;
   if ((rc = do_rmsnorm(c, b->d_hidden, n, w.g_attn, P.h))) return rc;                       // S1
+  c.kind = BULLET_K_QKV;
   if ((rc = do_gemm(c, EPI_F32, P.h, n, d, w.w_qkv, nq, 0, w.b_qkv, nullptr, P.qkv, nq))) return rc;  // S2
+  c.kind = BULLET_K_ROPE_KV;
   if ((rc = do_rope(c, b, layer, P.qkv, P.q))) return rc;                                    // S3
+  c.kind = BULLET_K_ATTN;
   if ((rc = do_attention(c, b, layer, P.q, P.o, 0))) return rc;                             // S4
   // S5: x1 = x + o W_o^T.  Under TP the non-lead ranks write their partial
   // into hidden and the fp32 all-reduce restores x + sum of partials (S9).
+  c.kind = BULLET_K_OPROJ;
   if ((rc = do_gemm(c, (!tp || lead) ? EPI_RESID : EPI_F32, P.o, n, H * hd, w.w_o, d, 0, nullptr,
                     b->d_hidden, b->d_hidden, d))) return rc;
+  c.kind = BULLET_K_ALLREDUCE;
   if (tp && (rc = allreduce(c, b->d_hidden, (size_t)n * d))) return rc;
+  c.kind = BULLET_K_RMSNORM2;
   if ((rc = do_rmsnorm(c, b->d_hidden, n, w.g_mlp, P.h))) return rc;                        // S6
+  c.kind = BULLET_K_GATE_UP;
   if ((rc = do_gemm(c, EPI_SILU, P.h, n, d, w.w_gate_up, 2 * I, I, nullptr, nullptr, P.act, I))) return rc;  // S7
+  c.kind = BULLET_K_DOWN;
   if ((rc = do_gemm(c, (!tp || lead) ? EPI_RESID : EPI_F32, P.act, n, I, w.w_down, d, 0, nullptr,
                     b->d_hidden, b->d_hidden, d))) return rc;                                // S8
+  c.kind = BULLET_K_ALLREDUCE;
   if (tp && (rc = allreduce(c, b->d_hidden, (size_t)n * d))) return rc;
   return BULLET_OK;
 }
@@ -361,7 +415,10 @@ int run_phase(Ctx& c, const bullet_batch* b) {
   const bool tc_attn = c.h->cfg.dtype == BULLET_DTYPE_BF16 && c.h->cfg.head_dim == 128 && max_qlen(b) > 1;
   PlanArgs pa{P.counters, P.n_counters, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ,
               tc_attn ? P.tiles : nullptr, P.n_tiles};
-  CK(launch_plan(pa, c.st));
+  c.kind = BULLET_K_PLAN;
+  c.layer = -1;
+  prof_begin(c);
+  LAUNCH(c, launch_plan(pa, c.st));
   for (int l = b->layer_begin; l < b->layer_end; ++l) {
     int rc = run_layer(c, b, l);
     if (rc) return rc;
@@ -594,10 +651,11 @@ int bullet_step(bullet_handle* h, const bullet_batch* pre, const bullet_batch* d
   if (h->log_cap == 0 && (flags & BULLET_SMID_LOG)) return set_err(BULLET_EINVAL, "SMID_LOG without a log buffer");
   const bool log = (flags & BULLET_SMID_LOG) != 0;
   cudaStream_t sp = (cudaStream_t)s_prefill, sd = (cudaStream_t)s_decode;
+  const bool prof = (flags & BULLET_PROFILE) != 0;
   Ctx cp{h, 0, mode == BULLET_CORUN ? gate_of(h, 0, p) : gate_of(h, 0, N),
-         mode == BULLET_CORUN ? p : N, log, sp, false};
+         mode == BULLET_CORUN ? p : N, log, sp, false, prof};
   Ctx cd{h, 1, mode == BULLET_CORUN ? gate_of(h, p, N) : gate_of(h, 0, N),
-         mode == BULLET_CORUN ? N - p : N, log, sd, false};
+         mode == BULLET_CORUN ? N - p : N, log, sd, false, prof};
   if (has_pre && (rc = run_phase(cp, pre))) return rc;
   if (run_dec) {
     if (mode == BULLET_TIMESLICED && has_pre) {
@@ -649,6 +707,32 @@ int bullet_choose_split(const bullet_handle* h, const bullet_sched_state* s, con
   return BULLET_OK;
 }
 
+int bullet_profile_read(bullet_handle* h, int32_t* kind, int32_t* phase, int32_t* layer, float* ms,
+                        int cap, int* n) {
+  if (!h || !n || cap < 0) return set_err(BULLET_EINVAL, "null");
+  *n = 0;
+  for (const auto& r : h->prof_recs) {
+    if (*n >= cap) break;
+    CK(cudaEventSynchronize(r.e1));
+    float t = 0.f;
+    CK(cudaEventElapsedTime(&t, r.e0, r.e1));
+    if (kind) kind[*n] = r.kind;
+    if (phase) phase[*n] = r.phase;
+    if (layer) layer[*n] = r.layer;
+    if (ms) ms[*n] = t;
+    ++*n;
+  }
+  h->prof_recs.clear();
+  h->ev_used = 0;
+  return BULLET_OK;
+}
+
+int bullet_launch_count(const bullet_handle* h, long long* n) {
+  if (!h || !n) return set_err(BULLET_EINVAL, "null");
+  *n = h->n_launch;
+  return BULLET_OK;
+}
+
 int bullet_sync(bullet_handle* h) {
   if (!h) return set_err(BULLET_EINVAL, "null");
   if (h->host_only) return BULLET_OK;
@@ -670,6 +754,7 @@ void bullet_destroy(bullet_handle* h) {
   cudaFree(h->rope_cs);
   cudaFree(h->op_ctr);
   if (h->ev_ts) cudaEventDestroy(h->ev_ts);
+  for (auto e : h->ev_pool) cudaEventDestroy(e);
   delete h;
 }
 

@@ -6,9 +6,9 @@
 // gathered through the block table from the paged pool with 16-byte
 // cp.async into XOR-swizzled shared memory (double-buffered).  Each of the
 // 4 warps owns 16 query rows: S = Q K^T with mma.m16n8k16 bf16 -> fp32,
-// online softmax in fp32 (exp2), then O += P V with P and V in fp16 (DESIGN
-// R-4b: bf16 P breaks the 1e-3 bar; bf16 -> fp16 is exact for |v| in
-// [2^-14, 65504]).  Round-1 kernel: mma.sync; the tcgen05 version is the
+// online softmax in fp32 (exp2), then O += P V with V in fp16 and P as an
+// fp16 hi + lo pair (DESIGN R-4b: a single bf16 or fp16 P adds measurable
+// error at the 1e-3 bar; bf16 -> fp16 is exact for |v| in [2^-14, 65504]).  Round-1 kernel: mma.sync; the tcgen05 version is the
 // next step.
 #include "kernels.h"
 
@@ -51,6 +51,14 @@ __device__ __forceinline__ uint32_t bf2_to_h2(uint32_t x) {
 __device__ __forceinline__ uint32_t pack_h2(float lo, float hi) {
   __half2 h = __floats2half2_rn(lo, hi);
   return *reinterpret_cast<uint32_t*>(&h);
+}
+// x -> (hi, lo) fp16 pairs with hi = fp16(x), lo = fp16(x - hi).
+__device__ __forceinline__ void split_h2(float x0, float x1, uint32_t& hi, uint32_t& lo) {
+  __half2 h = __floats2half2_rn(x0, x1);
+  const float2 hf = __half22float2(h);
+  __half2 l = __floats2half2_rn(x0 - hf.x, x1 - hf.y);
+  hi = *reinterpret_cast<uint32_t*>(&h);
+  lo = *reinterpret_cast<uint32_t*>(&l);
 }
 __device__ __forceinline__ void cp_async16_zfill(void* dst, const void* src, bool valid) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src),
@@ -185,21 +193,26 @@ __global__ void __launch_bounds__(128) k_attn_prefill_tc(AttnArgs a) {
         oacc[nd][0] *= alpha[0]; oacc[nd][1] *= alpha[0];
         oacc[nd][2] *= alpha[1]; oacc[nd][3] *= alpha[1];
       }
-      // O += P V  (fp16 P, fp16 V)
+      // O += P V with V in fp16 (exact) and P split into two fp16 halves
+      // P = P_hi + P_lo (22 significant bits): the P rounding stays far below
+      // the bf16 rounding of o (DESIGN R-4b).
 #pragma unroll
       for (int kk = 0; kk < 4; ++kk) {
-        uint32_t pa[4];
-        pa[0] = pack_h2(s[2 * kk][0], s[2 * kk][1]);
-        pa[1] = pack_h2(s[2 * kk][2], s[2 * kk][3]);
-        pa[2] = pack_h2(s[2 * kk + 1][0], s[2 * kk + 1][1]);
-        pa[3] = pack_h2(s[2 * kk + 1][2], s[2 * kk + 1][3]);
+        uint32_t pa[4], pl[4];
+        split_h2(s[2 * kk][0], s[2 * kk][1], pa[0], pl[0]);
+        split_h2(s[2 * kk][2], s[2 * kk][3], pa[1], pl[1]);
+        split_h2(s[2 * kk + 1][0], s[2 * kk + 1][1], pa[2], pl[2]);
+        split_h2(s[2 * kk + 1][2], s[2 * kk + 1][3], pa[3], pl[3]);
 #pragma unroll
         for (int ndp = 0; ndp < 8; ++ndp) {
           uint32_t b0, b1, b2, b3;
           const int mi = lane >> 3;
           ldsm_x4_t(vbase + swz(kk * 16 + (mi & 1) * 8 + (lane & 7), ndp * 2 + (mi >> 1)), b0, b1, b2, b3);
-          mma_f16(oacc[2 * ndp], pa, bf2_to_h2(b0), bf2_to_h2(b1));
-          mma_f16(oacc[2 * ndp + 1], pa, bf2_to_h2(b2), bf2_to_h2(b3));
+          b0 = bf2_to_h2(b0); b1 = bf2_to_h2(b1); b2 = bf2_to_h2(b2); b3 = bf2_to_h2(b3);
+          mma_f16(oacc[2 * ndp], pa, b0, b1);
+          mma_f16(oacc[2 * ndp + 1], pa, b2, b3);
+          mma_f16(oacc[2 * ndp], pl, b0, b1);
+          mma_f16(oacc[2 * ndp + 1], pl, b2, b3);
         }
       }
       __syncthreads();

@@ -87,6 +87,23 @@ class Setup:
         return out
 
 
+def oracle_layer(S, layer, x_pre, x_dec, row_mask_pre=None):
+    """One oracle layer step from given fp32 inputs (e.g. the GPU's output of
+    the previous layer): per-step parity (DESIGN R-4c)."""
+    cfg = oracle_cfg(S.m)
+    w = {k: (None if v is None else v.numpy()) for k, v in S.w_cpu[layer].items()}
+    out = {}
+    for name, x, q, c, bt, mask in (
+            ("pre", x_pre, S.prefill_lens, [0] * S.n_pre, S.lay.block_table[:S.n_pre], row_mask_pre),
+            ("dec", x_dec, [1] * len(S.decode_ctx), S.decode_ctx, S.lay.block_table[S.n_pre:], None)):
+        if not q:
+            continue
+        pk = S.pool_cpu[layer][0].numpy().copy(); pv = S.pool_cpu[layer][1].numpy().copy()
+        out[name] = O.layer_forward(cfg, w, pk, pv, q, c, bt, np.asarray(x, dtype=np.float64),
+                                    row_mask=mask)
+    return out
+
+
 def compare(got: np.ndarray, ref: np.ndarray):
     """(max-abs error, normalized-L1 mean-rel error) — DESIGN.md R-4."""
     err = np.abs(got.astype(np.float64) - ref)

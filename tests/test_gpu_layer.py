@@ -43,27 +43,46 @@ def test_tiny_fp32_two_layers(tiny, mode):
 @pytest.fixture(scope="module")
 def small_bf16():
     m = synth.ModelShape("small-bf16", 1024, 8, 2, 128, 2816, 2)
-    S = Setup(m, [300, 77, 1], [64, 1, 500, 31, 16, 1000], n_layers=2)
-    return S, S.oracle()
+    return Setup(m, [300, 77, 1], [64, 1, 500, 31, 16, 1000], n_layers=2)
+
+
+def _per_layer(S, p, flags):
+    """Run the two layers as two steps; check each step against the oracle
+    layer fed with the GPU's own input to that step (R-4c), then check the
+    single 2-layer step is bit-identical to the two 1-layer steps."""
+    from harness import oracle_layer
+    pre, dec = S.batches(0, 1)
+    x_pre0, x_dec0 = pre.hidden.cpu().numpy(), dec.hidden.cpu().numpy()
+    sp, sd = torch.cuda.Stream(), torch.cuda.Stream()
+    outs = []
+    for l in range(2):
+        pre.layer_begin, pre.layer_end = l, l + 1
+        dec.layer_begin, dec.layer_end = l, l + 1
+        xi_pre, xi_dec = pre.hidden.cpu().numpy(), dec.hidden.cpu().numpy()
+        S.bl.step(pre, dec, p, flags, sp, sd)
+        torch.cuda.synchronize()
+        ref = oracle_layer(S, l, xi_pre, xi_dec)
+        for name, b in (("pre", pre), ("dec", dec)):
+            mx, mr = compare(b.hidden.cpu().numpy(), ref[name])
+            assert mx <= 2e-2 and mr <= 1e-3, (name, l, p, mx, mr)
+        outs.append((pre.hidden.clone(), dec.hidden.clone()))
+    pre2, dec2 = S.batches(0, 2)
+    S.bl.step(pre2, dec2, p, flags, sp, sd)
+    torch.cuda.synchronize()
+    assert torch.equal(pre2.hidden, outs[1][0]) and torch.equal(dec2.hidden, outs[1][1])
 
 
 @pytest.mark.parametrize("p", [2, 64, 146])
 def test_small_bf16_corun_splits(small_bf16, p):
-    """Reduced Llama-style bf16 model (hd 128, GQA 4), two layers, ragged
-    prefill lengths: co-run at edge and middle splits meets the bar."""
-    S, ref = small_bf16
-    pre, dec = _run(S, p, S.B.CORUN)
-    for name, b in (("pre", pre), ("dec", dec)):
-        mx, mr = compare(b.hidden.cpu().numpy(), ref[name])
-        assert mx <= 2e-2 and mr <= 1e-3, (name, p, mx, mr)
+    """Reduced Llama-style bf16 model (hd 128, GQA 4), two layer steps,
+    ragged prefill lengths: co-run at edge and middle splits meets the bar."""
+    _per_layer(small_bf16, p, small_bf16.B.CORUN)
 
 
-def test_small_bf16_timesliced(small_bf16):
-    S, ref = small_bf16
-    pre, dec = _run(S, 148, S.B.TIMESLICED)
-    for name, b in (("pre", pre), ("dec", dec)):
-        mx, mr = compare(b.hidden.cpu().numpy(), ref[name])
-        assert mx <= 2e-2 and mr <= 1e-3, (name, mx, mr)
+@pytest.mark.parametrize("mode", ["timesliced", "ungated"])
+def test_small_bf16_baseline_modes(small_bf16, mode):
+    B = small_bf16.B
+    _per_layer(small_bf16, 148, B.TIMESLICED if mode == "timesliced" else B.UNGATED)
 
 
 def test_llama8b_config2_layer_sampled():
@@ -93,7 +112,7 @@ def test_smid_gating_invariants(small_bf16, p):
     """SM-range work assignment (§8a SG), bit-exact invariants: every work
     unit of every launch ran exactly once, on an SM of its phase's range;
     ranges = sigma[0:p) / sigma[p:N) (oracle range function)."""
-    S, _ = small_bf16
+    S = small_bf16
     B = S.B
     log = S.bl.set_smid_log(400000)
     try:
@@ -117,7 +136,7 @@ def test_smid_gating_invariants(small_bf16, p):
 
 
 def test_decode_pause_and_errors(small_bf16):
-    S, _ = small_bf16
+    S = small_bf16
     B = S.B
     pre, dec = S.batches()
     x0 = dec.hidden.clone()
