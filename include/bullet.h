@@ -258,6 +258,12 @@ int bullet_op_gemm(bullet_handle *h, int epi, const void *d_A, int M, int K, con
                    int N, int silu_half, const void *d_bias, const float *d_resid, void *d_out,
                    int lo, int hi, void *stream);
 
+/* KI2 microbenchmark: stream `bytes` (multiple of 64 KB) from d_src on the
+ * SMs sigma[lo:hi) and discard them; mode 0 LDG.128, 1 cp.async.bulk (TMA
+ * bulk copies), 2 cp.async 16 B.  Feeds the perf-model fit. */
+int bullet_op_stream(bullet_handle *h, const void *d_src, size_t bytes, int mode, int lo, int hi,
+                     void *stream);
+
 int bullet_op_rmsnorm(bullet_handle *h, const float *d_x, int n, const void *d_g, void *d_out,
                       int lo, int hi, void *stream);
 
@@ -269,7 +275,7 @@ int bullet_op_rope_kv(bullet_handle *h, const bullet_batch *batch, int layer, co
 /* Attention for `batch` rows reading K/V of `layer` through the block
  * table: q [n_tokens][H*hd] in, o [n_tokens][H*hd] out (dtype).
  * kind 0: automatic (what bullet_step uses), 1: SIMT kernel, 2: tensor-core
- * prefill kernel (bf16 only). */
+ * prefill kernel, 3: tensor-core decode kernel (2 and 3: bf16, head_dim 128). */
 int bullet_op_attention(bullet_handle *h, const bullet_batch *batch, int layer, const void *d_q,
                         void *d_o, int kind, int lo, int hi, void *stream);
 

@@ -233,22 +233,25 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   if (K % 64) return set_err(BULLET_EUNSUPPORTED, "GEMM needs K %% 64 == 0 (K=%d)", K);
   const int m_tiles = (M + 127) / 128;
   auto fits = [&](int bn) { return epi == EPI_SILU ? ((N / 2) % (bn / 2) == 0 && N % 2 == 0) : (N % bn == 0); };
-  int bn = 0;
-  if (fits(256) && m_tiles * (N / 256) >= c.m_sms) bn = 256;
-  else if (fits(128)) bn = 128;
-  else if (fits(64)) bn = 64;
-  else if (fits(256)) bn = 256;
-  if (!bn) return set_err(BULLET_EUNSUPPORTED, "GEMM N=%d not tileable", N);
-  const int tiles = m_tiles * (N / bn);
+  // Plan (bn, split-K) on the phase's m SMs: minimise waves x bytes per unit
+  // (A + B tile streams), plus the split-K partial round trip; ties prefer
+  // wider tiles (MMA efficiency).  Work units run one per CTA per wave.
   const int k_blocks = K / 64;
-  int splits = 1;
-  if (tiles < c.m_sms) {
-    splits = (c.m_sms + tiles - 1) / tiles;
-    splits = std::min(splits, std::max(1, k_blocks / 4));
-    while (splits > 1 && ((size_t)tiles * splits * 128 * bn > h->ph[c.phase].partial_floats ||
-                          tiles > N_TILE_SEMS))
-      --splits;
+  int bn = 0, splits = 1;
+  double best = 1e300;
+  for (int cand : {256, 128, 64}) {
+    if (!fits(cand)) continue;
+    const int tiles = m_tiles * (N / cand);
+    const int max_s = std::max(1, std::min(k_blocks / 4, N_TILE_SEMS / std::max(1, tiles)));
+    for (int s = 1; s <= max_s; ++s) {
+      if (s > 1 && (size_t)tiles * s * 128 * cand > h->ph[c.phase].partial_floats) break;
+      const double waves = std::ceil((double)tiles * s / c.m_sms);
+      const double cost = waves * ((double)k_blocks / s) * (128 + cand) * 128.0 +
+                          (s > 1 ? 3.0 * s * 128.0 * cand * 4.0 : 0.0) + waves * 64e3;
+      if (cost < best * 0.999) { best = cost; bn = cand; splits = s; }
+    }
   }
+  if (!bn) return set_err(BULLET_EUNSUPPORTED, "GEMM N=%d not tileable", N);
   a.bn = bn; a.splits = splits;
   a.partials = h->ph[c.phase].partials;
   a.tile_sems = h->ph[c.phase].tile_sems;
@@ -292,6 +295,13 @@ int max_qlen(const bullet_batch* b) {
   return mq;
 }
 
+int max_kv(const bullet_batch* b) {
+  int mk = 0;
+  for (int r = 0; r < b->n_reqs; ++r)
+    mk = std::max(mk, b->h_ctx_lens[r] + b->h_cu_seqlens[r + 1] - b->h_cu_seqlens[r]);
+  return mk;
+}
+
 int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* o, int kind) {
   bullet_handle* h = c.h;
   if (b->n_tokens == 0) return BULLET_OK;
@@ -302,8 +312,20 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
   a.n_reqs = b->n_reqs; a.max_blocks = b->max_blocks_per_req; a.n_tok = b->n_tokens;
   a.H = h->cfg.n_heads; a.Hkv = h->cfg.n_kv_heads; a.hd = h->cfg.head_dim; a.B = h->block_size;
   a.scale = (float)(1.0 / std::sqrt((double)a.hd));
+  static const int dbg = getenv("BULLET_DBG") ? atoi(getenv("BULLET_DBG")) : 0;
+  a.dbg = dbg;
   const bool bf16 = h->cfg.dtype == BULLET_DTYPE_BF16;
-  if (kind == 0) kind = (bf16 && a.hd == 128 && max_qlen(b) > 1) ? 2 : 1;
+  if (kind == 0) kind = (bf16 && a.hd == 128) ? (max_qlen(b) > 1 ? 2 : 3) : 1;
+  if (kind == 3 && max_kv(b) > attn_decode_max_blocks() * h->block_size) kind = c.op ? -1 : 1;
+  if (kind == -1) return set_err(BULLET_EUNSUPPORTED, "tensor-core decode attention: context too long");
+  if (kind == 3) {
+    if (!bf16 || a.hd != 128)
+      return set_err(BULLET_EUNSUPPORTED, "tensor-core decode attention: bf16, hd 128 only");
+    int rc = next_launch(c, &a.L);
+    if (rc) return rc;
+    LAUNCH(c, launch_attn_decode_tc(a, h->n_sms, c.st));
+    return BULLET_OK;
+  }
   if (kind == 2) {
     if (!bf16 || a.hd != 128) return set_err(BULLET_EUNSUPPORTED, "tensor-core attention: bf16, hd 128 only");
     PhaseWS& P = h->ph[c.phase];
@@ -780,6 +802,20 @@ int bullet_op_gemm(bullet_handle* h, int epi, const void* A, int M, int K, const
   return do_gemm(c, epi, A, M, K, B, N, silu_half, bias, resid, out, ldo);
 }
 
+int bullet_op_stream(bullet_handle* h, const void* src, size_t bytes, int mode, int lo, int hi,
+                     void* stream) {
+  Ctx c;
+  int rc = op_ctx(h, lo, hi, stream, &c);
+  if (rc) return rc;
+  if (!src || bytes == 0 || mode < 0 || mode > 2) return set_err(BULLET_EINVAL, "stream args");
+  StreamArgs a;
+  memset(&a, 0, sizeof a);
+  a.src = (const uint8_t*)src; a.bytes = bytes; a.mode = mode; a.sink = (uint32_t*)h->op_ctr;
+  if ((rc = next_launch(c, &a.L))) return rc;
+  LAUNCH(c, launch_stream(a, h->n_sms, c.st));
+  return BULLET_OK;
+}
+
 int bullet_op_rmsnorm(bullet_handle* h, const float* x, int n, const void* g, void* out, int lo,
                       int hi, void* stream) {
   Ctx c;
@@ -806,7 +842,7 @@ int bullet_op_attention(bullet_handle* h, const bullet_batch* b, int layer, cons
   Ctx c;
   int rc = op_ctx(h, lo, hi, stream, &c);
   if (rc) return rc;
-  if (!b || !q || !o || layer < 0 || layer >= h->cfg.n_layers || kind < 0 || kind > 2)
+  if (!b || !q || !o || layer < 0 || layer >= h->cfg.n_layers || kind < 0 || kind > 3)
     return set_err(BULLET_EINVAL, "attention args");
   bullet_batch bb = *b;
   bb.layer_begin = layer; bb.layer_end = layer;

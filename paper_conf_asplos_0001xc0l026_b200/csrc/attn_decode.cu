@@ -1,0 +1,337 @@
+// attn_decode.cu — paged decode attention on tensor cores, bf16, hd 128
+// (the paper's PagedAttention decode: "irregular
+// memory access" — here every (block, kv head) is one contiguous 4 KB chunk).
+//
+// Memory side: each of the 8 consumer warps streams its own blocks with
+// 16-byte cp.async (coalesced 4 KB chunks, XOR-swizzled into shared memory),
+// DEPTH blocks in flight per warp.  A claimer warp takes units from the
+// gated work counter and publishes each unit's block-table row and Q rows in
+// shared memory up to 4 units ahead, so no consumer waits on a dependent
+// global load; warps prefetch the next unit's first blocks before merging the
+// current one.  (A TMA version was capped near 27 GB/s per SM by the
+// per-operation cost of 2 KB paged boxes — DESIGN.md §5.)
+// Math side: swap-AB so the 16 keys of a block fill the MMA M dimension and
+// the GQA group (<= 8 query heads) fills N = 8:
+//   S^T[16 keys x 8 heads] = K[16 x 128] . Q^T[128 x 8]   (mma.m16n8k16 bf16)
+//   O^T[128 x 8]         += V^T[128 x 16] . P^T[16 x 8]  (P = hi + lo bf16)
+// P^T fragments come from the S^T accumulators by movmatrix (8x8 transpose).
+// Warps take blocks round-robin with private (max, sum, O^T) states, merged
+// through shared memory at the end of each unit.
+// Unit = (token, kv head); decode tokens are requests.
+#include "kernels.h"
+
+namespace bl {
+
+namespace {
+// DEPTH stages per warp: DEPTH - 1 blocks stay in flight while one is computed
+constexpr int KB = 16, HD = 128, NCW = 8, DEPTH = 3;
+constexpr int BLK_BYTES = KB * HD * 2;       // 4 KB: one (block, kv head) of K or V
+constexpr int STAGE_BYTES = 2 * BLK_BYTES;   // K + V
+constexpr int CMB_FLOATS = HD * 8 + 16;      // O^T[128][8] + m[8] + l[8] per warp (in a free stage)
+constexpr int THREADS = (NCW + 1) * 32;
+constexpr int QSLOT_BYTES = 8 * HD * 2;      // Q rows of up to 8 heads (bf16)
+constexpr int MAXNB = 512;                   // blocks per unit held in smem (8k tokens)
+static_assert(CMB_FLOATS * 4 <= STAGE_BYTES, "merge record must fit in one stage");
+
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void ldsm_x4(uint32_t addr, uint32_t* r) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]) : "r"(addr));
+}
+__device__ __forceinline__ void ldsm_x4_t(uint32_t addr, uint32_t* r) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]) : "r"(addr));
+}
+__device__ __forceinline__ void mma_bf16(float* c, const uint32_t* a, uint32_t b0, uint32_t b1) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+      "{%0,%1,%2,%3};"
+      : "+f"(c[0]), "+f"(c[1]), "+f"(c[2]), "+f"(c[3])
+      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+__device__ __forceinline__ uint32_t movtrans(uint32_t x) {
+  uint32_t y;
+  asm volatile("movmatrix.sync.aligned.m8n8.trans.b16 %0, %1;" : "=r"(y) : "r"(x));
+  return y;
+}
+__device__ __forceinline__ uint32_t pack_bf2(float a, float b) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+// x -> hi = bf16(x), lo = bf16(x - hi), packed pairwise.
+__device__ __forceinline__ void split_bf2(float a, float b, uint32_t& hi, uint32_t& lo) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  const float2 f = __bfloat1622float2(h);
+  hi = *reinterpret_cast<uint32_t*>(&h);
+  lo = pack_bf2(a - f.x, b - f.y);
+}
+// byte offset of 16-byte chunk c (0..15) of key row `row` in a [16][128] bf16
+// tile: rows of 256 B, chunk index XOR (row & 7) -> conflict-free ldmatrix
+__device__ __forceinline__ uint32_t tile_off(int row, int c) {
+  return row * 256 + ((c ^ (row & 7)) << 4);
+}
+
+struct Slot {  // one published unit
+  int u, t, pos, nb;
+};
+}  // namespace
+
+__global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
+  if (!gate_ok(a.L.gate)) return;
+  extern __shared__ __align__(128) uint8_t smem[];
+  uint8_t* stages = smem;                                                      // [NCW][DEPTH][STAGE]
+  uint8_t* qbuf = stages + NCW * DEPTH * STAGE_BYTES;                          // [4][QSLOT_BYTES]
+  int* btbuf = reinterpret_cast<int*>(qbuf + 4 * QSLOT_BYTES);                 // [4][MAXNB]
+  Slot* uq = reinterpret_cast<Slot*>(btbuf + 4 * MAXNB);
+  uint64_t* uqf = reinterpret_cast<uint64_t*>(uq + 4);
+  uint64_t* uqe = uqf + 4;
+  int* rec_stage = reinterpret_cast<int*>(uqe + 4);                            // [NCW]
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int grp = a.H / a.Hkv;
+  const int units = a.n_tok * a.Hkv;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < 4; ++i) { mbar_init(uqf + i, 1); mbar_init(uqe + i, NCW); }
+    mbar_fence_init();
+  }
+  __syncthreads();
+
+  if (warp == NCW) {  // ------------------------------------------ claimer
+    const __nv_bfloat16* qg = reinterpret_cast<const __nv_bfloat16*>(a.q);
+    for (int it = 0;; ++it) {
+      const int slot = it & 3;
+      // at most 2 units ahead of the consumers (load balance across CTAs)
+      if (lane == 0 && it >= 2) mbar_wait(uqe + ((it - 2) & 3), ((it - 2) >> 2) & 1);
+      __syncwarp();
+      int u = 0;
+      if (lane == 0) u = atomicAdd(a.L.ctr, 1);
+      u = __shfl_sync(0xffffffffu, u, 0);
+      if (u >= units) u = -1;
+      Slot sl{u, 0, 0, 0};
+      if (u >= 0) {
+        sl.t = u / a.Hkv;
+        const int r = find_req(a.cu, a.n_reqs, sl.t);
+        sl.pos = __ldg(a.ctx + r) + (sl.t - __ldg(a.cu + r));
+        sl.nb = sl.pos / KB + 1;
+        const int32_t* bt = a.bt + (size_t)r * a.max_blocks;
+        for (int b = lane; b < sl.nb; b += 32) btbuf[slot * MAXNB + b] = __ldg(bt + b);
+      }
+      __syncwarp();
+      if (lane == 0) {
+        uq[slot] = sl;
+        if (u >= 0) {  // Q rows of the unit ride on the slot's barrier
+          const int g = u % a.Hkv;
+          mbar_arrive_expect_tx(uqf + slot, grp * HD * 2);
+          bulk_g2s(qbuf + slot * QSLOT_BYTES, qg + (size_t)sl.t * a.H * HD + (size_t)g * grp * HD,
+                   grp * HD * 2, uqf + slot);
+          log_unit(a.L, u);
+        } else {
+          mbar_arrive(uqf + slot);
+        }
+      }
+      if (u < 0) break;
+    }
+    return;
+  }
+
+  // ------------------------------------------------------------ consumers
+  const int gq = lane >> 2, tq = lane & 3;
+  const float sl2 = a.scale * 1.4426950408889634f;
+  const __nv_bfloat16* pk = reinterpret_cast<const __nv_bfloat16*>(a.pool_k);
+  const __nv_bfloat16* pv = reinterpret_cast<const __nv_bfloat16*>(a.pool_v);
+  __nv_bfloat16* og = reinterpret_cast<__nv_bfloat16*>(a.o);
+  uint8_t* my = stages + warp * DEPTH * STAGE_BYTES;
+  const uint32_t my_s = smem_u32(my);
+  auto my_count = [&](int nb) { return nb > warp ? (nb - warp + NCW - 1) / NCW : 0; };
+  // per-lane swizzled offsets (loop invariant): cp.async destinations and
+  // ldmatrix sources for the QK (K, by k-step) and PV (V^T, by m-tile) MMAs
+  uint32_t cp_off[8], k_off[8], v_off[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    cp_off[i] = tile_off(2 * i + (lane >> 4), lane & 15);
+    k_off[i] = tile_off(lane & 15, i * 2 + (lane >> 4));
+    v_off[i] = BLK_BYTES + tile_off(((lane >> 3) >> 1) * 8 + (lane & 7), i * 2 + ((lane >> 3) & 1));
+  }
+
+  // issue cursor over this warp's block sequence (units in claim order,
+  // my blocks warp, warp + 8, ... of each), never beyond unit `limit`
+  int iu = 0, ij = 0, n_issued = 0, n_cons = 0;
+  int cur_nb = -1, cur_g = 0, cur_u = 0;   // cached slot of unit iu (-1: not read yet)
+  auto fill = [&](int limit, int cap) {
+    while (n_issued - n_cons < cap && iu <= limit) {
+      const int sl = iu & 3;
+      if (cur_nb < 0) {
+        mbar_wait(uqf + sl, (iu >> 2) & 1);
+        const Slot X = uq[sl];
+        cur_u = X.u; cur_nb = my_count(X.nb); cur_g = X.u >= 0 ? X.u % a.Hkv : 0;
+      }
+      if (cur_u < 0) return;
+      if (ij >= cur_nb) { ++iu; ij = 0; cur_nb = -1; continue; }
+      const int blk = btbuf[sl * MAXNB + warp + ij * NCW];
+      const uint8_t* ks = reinterpret_cast<const uint8_t*>(pk + ((size_t)blk * a.Hkv + cur_g) * KB * HD) + lane * 16;
+      const uint8_t* vs = reinterpret_cast<const uint8_t*>(pv + ((size_t)blk * a.Hkv + cur_g) * KB * HD) + lane * 16;
+      uint8_t* dk = my + (n_issued % DEPTH) * STAGE_BYTES;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        cp_async16(dk + cp_off[i], ks + 512 * i);
+        cp_async16(dk + BLK_BYTES + cp_off[i], vs + 512 * i);
+      }
+      cp_async_commit();
+      ++n_issued;
+      ++ij;
+    }
+  };
+
+  for (int it = 0;; ++it) {
+    const int slot = it & 3;
+    mbar_wait(uqf + slot, (it >> 2) & 1);
+    const Slot S = uq[slot];
+    if (S.u < 0) break;
+    const int g = S.u % a.Hkv;
+    // Q^T as the B operand: n = head gq (zero beyond the group), k = dims
+    uint32_t qb[8][2];
+    {
+      const bool ok = gq < grp;
+      const uint8_t* qh = qbuf + slot * QSLOT_BYTES + (ok ? gq : 0) * HD * 2;
+#pragma unroll
+      for (int ks = 0; ks < 8; ++ks) {
+        qb[ks][0] = ok ? *reinterpret_cast<const uint32_t*>(qh + (ks * 16 + 2 * tq) * 2) : 0u;
+        qb[ks][1] = ok ? *reinterpret_cast<const uint32_t*>(qh + (ks * 16 + 8 + 2 * tq) * 2) : 0u;
+      }
+    }
+    float m0 = -INFINITY, m1 = -INFINITY, l0 = 0.f, l1 = 0.f;   // heads 2tq, 2tq+1
+    float oacc[8][4];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) oacc[i][0] = oacc[i][1] = oacc[i][2] = oacc[i][3] = 0.f;
+
+    const int mine = my_count(S.nb);
+    for (int j = 0; j < mine; ++j) {
+      fill(it + 1, DEPTH);
+      const int pend = n_issued - n_cons;   // groups in flight; the oldest is block j
+      if (pend >= 3) cp_async_wait<2>(); else if (pend == 2) cp_async_wait<1>(); else cp_async_wait<0>();
+      __syncwarp();
+      const int b = warp + j * NCW;
+      const uint32_t kt = my_s + (n_cons % DEPTH) * STAGE_BYTES;
+      float s[4] = {0.f, 0.f, 0.f, 0.f}, s2[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+      for (int ks = 0; ks < 8; ks += 2) {   // two independent accumulation chains
+        uint32_t af[4], ag[4];
+        ldsm_x4(kt + k_off[ks], af);
+        ldsm_x4(kt + k_off[ks + 1], ag);
+        mma_bf16(s, af, qb[ks][0], qb[ks][1]);
+        mma_bf16(s2, ag, qb[ks + 1][0], qb[ks + 1][1]);
+      }
+      s[0] += s2[0]; s[1] += s2[1]; s[2] += s2[2]; s[3] += s2[3];
+      // s[0] (key gq, head 2tq), s[1] (gq, 2tq+1), s[2] (gq+8, 2tq), s[3] (gq+8, 2tq+1)
+      const int k0 = b * KB + gq, k1 = k0 + 8;
+      s[0] = k0 <= S.pos ? s[0] * sl2 : -INFINITY;
+      s[1] = k0 <= S.pos ? s[1] * sl2 : -INFINITY;
+      s[2] = k1 <= S.pos ? s[2] * sl2 : -INFINITY;
+      s[3] = k1 <= S.pos ? s[3] * sl2 : -INFINITY;
+      float bm0 = fmaxf(s[0], s[2]), bm1 = fmaxf(s[1], s[3]);
+#pragma unroll
+      for (int o = 4; o < 32; o <<= 1) {
+        bm0 = fmaxf(bm0, __shfl_xor_sync(0xffffffffu, bm0, o));
+        bm1 = fmaxf(bm1, __shfl_xor_sync(0xffffffffu, bm1, o));
+      }
+      const float mn0 = fmaxf(m0, bm0), mn1 = fmaxf(m1, bm1);
+      const float al0 = exp2f(m0 - mn0), al1 = exp2f(m1 - mn1);
+      m0 = mn0; m1 = mn1;
+      const float p00 = exp2f(s[0] - mn0), p01 = exp2f(s[1] - mn1);
+      const float p10 = exp2f(s[2] - mn0), p11 = exp2f(s[3] - mn1);
+      l0 = l0 * al0 + p00 + p10;
+      l1 = l1 * al1 + p01 + p11;
+      if (__any_sync(0xffffffffu, al0 != 1.f || al1 != 1.f)) {   // max moved: rescale O
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          oacc[i][0] *= al0; oacc[i][1] *= al1; oacc[i][2] *= al0; oacc[i][3] *= al1;
+        }
+      }
+      uint32_t h0, h1, lo0, lo1;
+      split_bf2(p00, p01, h0, lo0);
+      split_bf2(p10, p11, h1, lo1);
+      const uint32_t bh0 = movtrans(h0), bh1 = movtrans(h1);
+      const uint32_t bl0 = movtrans(lo0), bl1 = movtrans(lo1);
+      uint32_t vf[8][4];
+#pragma unroll
+      for (int mt = 0; mt < 8; ++mt) ldsm_x4_t(kt + v_off[mt], vf[mt]);
+#pragma unroll
+      for (int mt = 0; mt < 8; ++mt) mma_bf16(oacc[mt], vf[mt], bh0, bh1);
+#pragma unroll
+      for (int mt = 0; mt < 8; ++mt) mma_bf16(oacc[mt], vf[mt], bl0, bl1);
+      __syncwarp();
+      ++n_cons;
+    }
+    // the next unit's first DEPTH-1 blocks fly during the merge; the stage
+    // left free holds this warp's merge record
+    fill(it + 1, DEPTH - 1);
+    // full row sums over the 8 key lanes of each head
+#pragma unroll
+    for (int o = 4; o < 32; o <<= 1) {
+      l0 += __shfl_xor_sync(0xffffffffu, l0, o);
+      l1 += __shfl_xor_sync(0xffffffffu, l1, o);
+    }
+    const int fs = n_issued % DEPTH;
+    if (lane == 0) rec_stage[warp] = warp * DEPTH + fs;
+    float* rec = reinterpret_cast<float*>(my + fs * STAGE_BYTES);   // O^T[dim][head], m[8], l[8]
+#pragma unroll
+    for (int mt = 0; mt < 8; ++mt) {
+      rec[(mt * 16 + gq) * 8 + 2 * tq] = oacc[mt][0];
+      rec[(mt * 16 + gq) * 8 + 2 * tq + 1] = oacc[mt][1];
+      rec[(mt * 16 + gq + 8) * 8 + 2 * tq] = oacc[mt][2];
+      rec[(mt * 16 + gq + 8) * 8 + 2 * tq + 1] = oacc[mt][3];
+    }
+    if (gq == 0) {
+      rec[HD * 8 + 2 * tq] = m0; rec[HD * 8 + 2 * tq + 1] = m1;
+      rec[HD * 8 + 8 + 2 * tq] = l0; rec[HD * 8 + 8 + 2 * tq + 1] = l1;
+    }
+    named_bar_sync(1, NCW * 32);
+    const float* recs[NCW];
+#pragma unroll
+    for (int w = 0; w < NCW; ++w) recs[w] = reinterpret_cast<const float*>(stages + rec_stage[w] * STAGE_BYTES);
+    for (int e = threadIdx.x; e < grp * HD; e += NCW * 32) {
+      const int h = e / HD, d = e % HD;
+      float M = -INFINITY;
+      for (int w = 0; w < NCW; ++w) M = fmaxf(M, recs[w][HD * 8 + h]);
+      float L = 0.f, O = 0.f;
+      for (int w = 0; w < NCW; ++w) {
+        const float* rw = recs[w];
+        const float mw = rw[HD * 8 + h];
+        if (mw == -INFINITY) continue;
+        const float f = exp2f(mw - M);
+        L += rw[HD * 8 + 8 + h] * f;
+        O += rw[d * 8 + h] * f;
+      }
+      og[(size_t)S.t * a.H * HD + (size_t)(g * grp + h) * HD + d] = __float2bfloat16_rn(O / L);
+    }
+    named_bar_sync(1, NCW * 32);
+    if (lane == 0) mbar_arrive(uqe + slot);
+  }
+  cp_async_wait<0>();
+}
+
+size_t attn_decode_smem_bytes() {
+  return (size_t)NCW * DEPTH * STAGE_BYTES + 4 * QSLOT_BYTES + 4 * MAXNB * 4 + 4 * sizeof(Slot) +
+         8 * 8 + NCW * 4;
+}
+int attn_decode_max_blocks() { return MAXNB; }
+
+cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, cudaStream_t st) {
+  const size_t smem = attn_decode_smem_bytes();
+  static bool set = false;
+  if (!set) {
+    cudaError_t e = cudaFuncSetAttribute(k_attn_decode_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    set = true;
+  }
+  k_attn_decode_tc<<<grid, THREADS, smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+}  // namespace bl

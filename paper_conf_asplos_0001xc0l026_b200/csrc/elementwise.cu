@@ -12,39 +12,73 @@ __device__ __forceinline__ int warp_claim(const Launch& L) {
   return __shfl_sync(0xffffffffu, u, 0);
 }
 
+// 4-element vector load / store of the storage type.
+__device__ __forceinline__ float4 ld4(const float* p) { return *reinterpret_cast<const float4*>(p); }
+__device__ __forceinline__ float4 ld4(const __nv_bfloat16* p) {
+  const uint2 u = *reinterpret_cast<const uint2*>(p);
+  const float2 a = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&u.x));
+  const float2 b = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&u.y));
+  return make_float4(a.x, a.y, b.x, b.y);
+}
+__device__ __forceinline__ void st4(float* p, float4 v) { *reinterpret_cast<float4*>(p) = v; }
+__device__ __forceinline__ void st4(__nv_bfloat16* p, float4 v) {
+  __nv_bfloat162 a = __floats2bfloat162_rn(v.x, v.y), b = __floats2bfloat162_rn(v.z, v.w);
+  uint2 u;
+  u.x = *reinterpret_cast<uint32_t*>(&a);
+  u.y = *reinterpret_cast<uint32_t*>(&b);
+  *reinterpret_cast<uint2*>(p) = u;
+}
+__device__ __forceinline__ void st2(float* p, float a, float b) { *reinterpret_cast<float2*>(p) = make_float2(a, b); }
+__device__ __forceinline__ void st2(__nv_bfloat16* p, float a, float b) {
+  *reinterpret_cast<__nv_bfloat162*>(p) = __floats2bfloat162_rn(a, b);
+}
+
 // ------------------------------------------------------------------ RMSNorm
-// h = x / sqrt(mean(x^2) + eps) * g, one warp per row, fp32 math, rounded
-// once to the output type (oracle rounding point R1 / R4).
-template <typename T>
+// h = x / sqrt(mean(x^2) + eps) * g, one CTA (256 threads) per row with the
+// row held in registers (VPT float4 per thread), fp32 math, rounded once to
+// the output type (oracle rounding point R1 / R4).
+template <typename T, int VPT>
 __global__ void __launch_bounds__(256) k_rmsnorm(NormArgs a) {
   if (!gate_ok(a.L.gate)) return;
-  const int lane = threadIdx.x & 31;
+  __shared__ int s_u;
+  __shared__ float s_red[8];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const T* g = reinterpret_cast<const T*>(a.g);
   T* out = reinterpret_cast<T*>(a.out);
-  const int units = (a.n + ROWS_PER_UNIT - 1) / ROWS_PER_UNIT;
+  const int d4 = a.d / 4;
   for (;;) {
-    const int u = warp_claim(a.L);
-    if (u >= units) break;
-    if (lane == 0) log_unit(a.L, u);
-    const int r1 = min(a.n, (u + 1) * ROWS_PER_UNIT);
-    for (int r = u * ROWS_PER_UNIT; r < r1; ++r) {
-      const float4* x4 = reinterpret_cast<const float4*>(a.x + (size_t)r * a.d);
-      float ss = 0.f;
-      for (int i = lane; i < a.d / 4; i += 32) {
-        float4 v = x4[i];
-        ss += v.x * v.x + v.y * v.y + v.z * v.z + v.w * v.w;
-      }
-      ss = warp_sum(ss);
-      const float inv = rsqrtf(ss / (float)a.d + a.eps);
-      T* o = out + (size_t)r * a.d;
-      for (int i = lane; i < a.d / 4; i += 32) {
-        float4 v = x4[i];
-        o[4 * i + 0] = Elt<T>::from_f(v.x * inv * Elt<T>::to_f(g[4 * i + 0]));
-        o[4 * i + 1] = Elt<T>::from_f(v.y * inv * Elt<T>::to_f(g[4 * i + 1]));
-        o[4 * i + 2] = Elt<T>::from_f(v.z * inv * Elt<T>::to_f(g[4 * i + 2]));
-        o[4 * i + 3] = Elt<T>::from_f(v.w * inv * Elt<T>::to_f(g[4 * i + 3]));
+    if (tid == 0) s_u = atomicAdd(a.L.ctr, 1);
+    __syncthreads();
+    const int r = s_u;
+    if (r >= a.n) break;
+    if (tid == 0) log_unit(a.L, r);
+    const float* x = a.x + (size_t)r * a.d;
+    float4 v[VPT];
+    float ss = 0.f;
+#pragma unroll
+    for (int i = 0; i < VPT; ++i) {
+      const int idx = tid + i * 256;
+      v[i] = idx < d4 ? ld4(x + 4 * idx) : make_float4(0.f, 0.f, 0.f, 0.f);
+      ss += v[i].x * v[i].x + v[i].y * v[i].y + v[i].z * v[i].z + v[i].w * v[i].w;
+    }
+    ss = warp_sum(ss);
+    if (lane == 0) s_red[warp] = ss;
+    __syncthreads();
+    float tot = 0.f;
+#pragma unroll
+    for (int w = 0; w < 8; ++w) tot += s_red[w];
+    const float inv = rsqrtf(tot / (float)a.d + a.eps);
+    T* o = out + (size_t)r * a.d;
+#pragma unroll
+    for (int i = 0; i < VPT; ++i) {
+      const int idx = tid + i * 256;
+      if (idx < d4) {
+        const float4 gg = ld4(g + 4 * idx);
+        st4(o + 4 * idx, make_float4(v[i].x * inv * gg.x, v[i].y * inv * gg.y, v[i].z * inv * gg.z,
+                                     v[i].w * inv * gg.w));
       }
     }
+    __syncthreads();  // s_u / s_red reuse
   }
 }
 
@@ -52,44 +86,45 @@ __global__ void __launch_bounds__(256) k_rmsnorm(NormArgs a) {
 // Token t of request r at position p = ctx[r] + (t - cu[r]).  Rotate-half
 // RoPE of q and k heads with the (cos, sin) table, round to the storage type
 // (point R2), q -> q_out[t], k / v -> pool slot bt[r][p / B] * B + p % B.
+// One CTA (256 threads) per token; each thread rotates two adjacent pairs
+// (float2 loads, 2-element stores) and copies four v elements.
 template <typename T>
 __global__ void __launch_bounds__(256) k_rope_kv(RopeArgs a) {
   if (!gate_ok(a.L.gate)) return;
-  const int lane = threadIdx.x & 31;
-  const int half = a.hd / 2;
+  __shared__ int s_u;
+  const int tid = threadIdx.x;
+  const int half = a.hd / 2, hp = half / 2;  // pair-of-pairs per head
   T* q_out = reinterpret_cast<T*>(a.q_out);
   T* pk = reinterpret_cast<T*>(a.pool_k);
   T* pv = reinterpret_cast<T*>(a.pool_v);
   const int nq = (a.H + 2 * a.Hkv) * a.hd;
-  const int units = (a.n_tok + ROWS_PER_UNIT - 1) / ROWS_PER_UNIT;
   for (;;) {
-    const int u = warp_claim(a.L);
-    if (u >= units) break;
-    if (lane == 0) log_unit(a.L, u);
-    const int t1 = min(a.n_tok, (u + 1) * ROWS_PER_UNIT);
-    for (int t = u * ROWS_PER_UNIT; t < t1; ++t) {
-      const int r = find_req(a.cu, a.n_reqs, t);
-      const int pos = __ldg(a.ctx + r) + (t - __ldg(a.cu + r));
-      const int blk = __ldg(a.bt + (size_t)r * a.max_blocks + pos / a.B);
-      const int off = pos % a.B;
-      const float* src = a.qkv + (size_t)t * nq;
-      const float2* cs = a.cs + (size_t)pos * half;
-      for (int idx = lane; idx < (a.H + a.Hkv) * half; idx += 32) {
-        const int h = idx / half, i = idx % half;
-        const float x0 = src[h * a.hd + i], x1 = src[h * a.hd + i + half];
-        const float2 c = cs[i];
-        const float y0 = x0 * c.x - x1 * c.y, y1 = x1 * c.x + x0 * c.y;
-        T* dst;
-        if (h < a.H) dst = q_out + (size_t)t * a.H * a.hd + h * a.hd;
-        else dst = pk + (((size_t)blk * a.Hkv + (h - a.H)) * a.B + off) * a.hd;
-        dst[i] = Elt<T>::from_f(y0);
-        dst[i + half] = Elt<T>::from_f(y1);
-      }
-      const float* vs = src + (a.H + a.Hkv) * a.hd;
-      for (int idx = lane; idx < a.Hkv * a.hd; idx += 32) {
-        const int g = idx / a.hd, e = idx % a.hd;
-        pv[(((size_t)blk * a.Hkv + g) * a.B + off) * a.hd + e] = Elt<T>::from_f(vs[idx]);
-      }
+    if (tid == 0) s_u = atomicAdd(a.L.ctr, 1);
+    __syncthreads();
+    const int t = s_u;
+    __syncthreads();
+    if (t >= a.n_tok) break;
+    if (tid == 0) log_unit(a.L, t);
+    const int r = find_req(a.cu, a.n_reqs, t);
+    const int pos = __ldg(a.ctx + r) + (t - __ldg(a.cu + r));
+    const int blk = __ldg(a.bt + (size_t)r * a.max_blocks + pos / a.B);
+    const int off = pos % a.B;
+    const float* src = a.qkv + (size_t)t * nq;
+    const float2* cs = a.cs + (size_t)pos * half;
+    for (int idx = tid; idx < (a.H + a.Hkv) * hp; idx += 256) {
+      const int h = idx / hp, i = 2 * (idx % hp);
+      const float2 x0 = *reinterpret_cast<const float2*>(src + h * a.hd + i);
+      const float2 x1 = *reinterpret_cast<const float2*>(src + h * a.hd + i + half);
+      const float4 c = *reinterpret_cast<const float4*>(cs + i);   // (cos_i, sin_i, cos_i+1, sin_i+1)
+      T* dst = h < a.H ? q_out + (size_t)t * a.H * a.hd + h * a.hd
+                       : pk + (((size_t)blk * a.Hkv + (h - a.H)) * a.B + off) * a.hd;
+      st2(dst + i, x0.x * c.x - x1.x * c.y, x0.y * c.z - x1.y * c.w);
+      st2(dst + i + half, x1.x * c.x + x0.x * c.y, x1.y * c.z + x0.y * c.w);
+    }
+    const float* vs = src + (a.H + a.Hkv) * a.hd;
+    for (int idx = tid; idx < a.Hkv * a.hd / 4; idx += 256) {
+      const int g = (4 * idx) / a.hd, e = (4 * idx) % a.hd;
+      st4(pv + (((size_t)blk * a.Hkv + g) * a.B + off) * a.hd + e, ld4(vs + 4 * idx));
     }
   }
 }
@@ -200,7 +235,12 @@ cudaError_t launch_gemm_simt(const T* A, const T* B, const GemmArgs& a, int grid
 }
 template <typename T>
 cudaError_t launch_rmsnorm(const NormArgs& a, int grid, cudaStream_t st) {
-  k_rmsnorm<T><<<grid, 256, 0, st>>>(a);
+  const int v = (a.d / 4 + 255) / 256;
+  if (v <= 1) k_rmsnorm<T, 1><<<grid, 256, 0, st>>>(a);
+  else if (v <= 2) k_rmsnorm<T, 2><<<grid, 256, 0, st>>>(a);
+  else if (v <= 4) k_rmsnorm<T, 4><<<grid, 256, 0, st>>>(a);
+  else if (v <= 8) k_rmsnorm<T, 8><<<grid, 256, 0, st>>>(a);
+  else return cudaErrorInvalidValue;
   return cudaGetLastError();
 }
 template <typename T>

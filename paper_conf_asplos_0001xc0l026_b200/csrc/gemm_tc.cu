@@ -171,6 +171,9 @@ __global__ void __launch_bounds__(NT, 1)
       for (;;) {
         const int slot = it & 3;
         mbar_wait(tqe + slot, ((it >> 2) & 1) ^ 1);
+        // claim just in time: only once a smem stage is free to load into, so
+        // early CTAs cannot hoard units while others idle (load balance)
+        mbar_wait(empty + s, ph ^ 1);
         int u = atomicAdd(a.L.ctr, 1);
         if (u >= units) u = -1;
         tile_q[slot] = u;

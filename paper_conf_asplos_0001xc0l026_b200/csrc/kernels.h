@@ -44,6 +44,12 @@ struct AttnArgs {
   float scale;
   const int2* tiles;      // prefill tensor-core kernel: (request, q-tile) list
   const int* n_tiles;     // device count of `tiles`
+  int dbg;                // diagnostics (BULLET_DBG env): bit0 = decode consumers skip math
+  Launch L;
+};
+
+struct StreamArgs {   // KI2 streaming microbenchmark
+  const uint8_t* src; size_t bytes; int mode; uint32_t* sink;
   Launch L;
 };
 
@@ -67,7 +73,11 @@ cudaError_t launch_rope_kv(const RopeArgs& a, int grid, cudaStream_t st);
 template <typename T>
 cudaError_t launch_attn_simt(const AttnArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_attn_prefill_tc(const AttnArgs& a, int grid, cudaStream_t st);
+cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, cudaStream_t st);
+size_t attn_decode_smem_bytes();
+int attn_decode_max_blocks();
 cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);
+cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_probe(int* out_smid, int n, cudaStream_t st);
 
 constexpr int ATTN_TC_BQ = 64;    // query rows per tensor-core attention tile

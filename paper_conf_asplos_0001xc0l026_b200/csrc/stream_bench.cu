@@ -1,0 +1,107 @@
+// stream_bench.cu — KI2 microbenchmark: HBM read bandwidth reachable from m
+// SMs (the B200 analog of the paper's Fig. 7 partial-SM scaling, P:L139-145,
+// and the m_sat input of SURVEY §8d).  Gated persistent kernels stream a
+// buffer and fold it into a checksum (so no load is dead):
+//   mode 0  LDG.128: warps claim 8 KB units, 16 loads in flight per lane
+//           (16 warps -> 128 KB in flight per SM)
+//   mode 1  cp.async.bulk: one thread streams 32 KB bulk copies through a
+//           6 x 32 KB smem ring (192 KB in flight per SM)
+//   mode 2  cp.async 16 B (LDGSTS): 64 KB units, 3 in flight per CTA
+#include "kernels.h"
+
+namespace bl {
+
+namespace {
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+constexpr int BULK = 32768, NB = 6;
+}  // namespace
+
+__global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
+  if (!gate_ok(a.L.gate)) return;
+  extern __shared__ __align__(128) uint8_t sm[];
+  __shared__ int s_u;
+  __shared__ uint64_t bars[NB];
+  const int tid = threadIdx.x, lane = tid & 31;
+  uint32_t acc = 0;
+  if (a.mode == 0) {
+    const size_t units = a.bytes / 8192;
+    for (;;) {
+      int u = 0;
+      if (lane == 0) u = atomicAdd(a.L.ctr, 1);
+      u = __shfl_sync(0xffffffffu, u, 0);
+      if (u >= (int)units) break;
+      const uint4* p = reinterpret_cast<const uint4*>(a.src + (size_t)u * 8192) + lane;
+      uint4 v[16];
+#pragma unroll
+      for (int i = 0; i < 16; ++i) v[i] = __ldcs(p + 32 * i);
+#pragma unroll
+      for (int i = 0; i < 16; ++i) acc ^= v[i].x ^ v[i].y ^ v[i].z ^ v[i].w;
+    }
+  } else if (a.mode == 1) {
+    const size_t units = a.bytes / BULK;
+    if (tid == 0) {
+      for (int i = 0; i < NB; ++i) mbar_init(bars + i, 1);
+      mbar_fence_init();
+    }
+    __syncthreads();
+    if (tid == 0) {
+      uint32_t issued = 0, done = 0;
+      for (;;) {
+        if (issued - done == NB) {   // retire the oldest
+          mbar_wait(bars + (done % NB), (done / NB) & 1);
+          acc ^= *reinterpret_cast<const uint32_t*>(sm + (done % NB) * BULK);
+          ++done;
+        }
+        const int u = atomicAdd(a.L.ctr, 1);
+        if (u >= (int)units) break;
+        const int s = issued % NB;
+        mbar_arrive_expect_tx(bars + s, BULK);
+        bulk_g2s(sm + s * BULK, a.src + (size_t)u * BULK, BULK, bars + s);
+        ++issued;
+      }
+      while (done < issued) {
+        mbar_wait(bars + (done % NB), (done / NB) & 1);
+        acc ^= *reinterpret_cast<const uint32_t*>(sm + (done % NB) * BULK);
+        ++done;
+      }
+    }
+  } else {
+    const size_t units = a.bytes / 65536;
+    int n = 0;
+    for (;;) {
+      if (tid == 0) s_u = atomicAdd(a.L.ctr, 1);
+      __syncthreads();
+      const int u = s_u;
+      __syncthreads();
+      if (u >= (int)units) break;
+      const uint8_t* p = a.src + (size_t)u * 65536;
+      uint8_t* d = sm + (n % 3) * 65536;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) cp_async16(d + (tid + i * 512) * 16, p + (tid + i * 512) * 16);
+      cp_async_commit();
+      ++n;
+      if (n >= 3) {
+        cp_async_wait<2>();
+        acc ^= *reinterpret_cast<const uint32_t*>(sm + (n % 3) * 65536 + tid * 16);
+      }
+    }
+    cp_async_wait<0>();
+  }
+  if (acc == 0x12345678u) a.sink[0] = acc;   // keeps the loads alive
+}
+
+cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st) {
+  const int smem = a.mode == 1 ? NB * BULK : (a.mode == 2 ? 3 * 65536 : 0);
+  cudaError_t e = cudaFuncSetAttribute(k_stream, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return e;
+  k_stream<<<grid, 512, smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+}  // namespace bl
