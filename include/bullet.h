@@ -254,6 +254,9 @@ void bullet_destroy(bullet_handle *h);
  *               B rows [0, N/2) gate, [silu_half, silu_half + N/2) up;
  *               out of dtype                                    (gate_up)
  * N = number of B rows used (2 x output columns for SILU_MUL). */
+/* epi | BULLET_GEMM_PACKED: first repack B into the pre-swizzled tile layout
+ * that bullet_step uses for weights (kernels.h), then run the bulk-copy path. */
+enum { BULLET_GEMM_PACKED = 256 };
 int bullet_op_gemm(bullet_handle *h, int epi, const void *d_A, int M, int K, const void *d_B,
                    int N, int silu_half, const void *d_bias, const float *d_resid, void *d_out,
                    int lo, int hi, void *stream);

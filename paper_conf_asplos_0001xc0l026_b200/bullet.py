@@ -326,10 +326,12 @@ class Bullet:
         return p.value, k.value
 
     # ---- op-level entry points (per-kernel parity tests)
-    def op_gemm(self, epi, A, B, out, bias=None, resid=None, silu_half=0, lo=0, hi=None, stream=None):
+    def op_gemm(self, epi, A, B, out, bias=None, resid=None, silu_half=0, lo=0, hi=None, stream=None,
+                packed=False):
         M, K = A.shape
         N = B.shape[0] if epi != EPI_SILU else 2 * out.shape[1]
-        _check(lib().bullet_op_gemm(self.h, epi, _ptr(A), M, K, _ptr(B), N, silu_half, _ptr(bias),
+        _check(lib().bullet_op_gemm(self.h, epi | (256 if packed else 0), _ptr(A), M, K, _ptr(B), N,
+                                    silu_half, _ptr(bias),
                                     _ptr(resid), _ptr(out), lo, self.n_sms if hi is None else hi,
                                     _stream(stream)))
 

@@ -118,6 +118,10 @@ struct bullet_handle {
   int dev = 0, n_sms = 0, elt = 2;
   std::vector<int> sigma;
   std::vector<bullet_layer_weights> w;
+  struct Packed { uint8_t *base = nullptr, *qkv = nullptr, *o = nullptr, *gu = nullptr, *down = nullptr; };
+  std::vector<Packed> wp;            // bf16: pre-swizzled weight tiles (kernels.h)
+  uint8_t* op_pack = nullptr;        // scratch for bullet_op_gemm with BULLET_GEMM_PACKED
+  size_t op_pack_bytes = 0;
   std::vector<char> w_set;
   std::vector<void*> pk, pv;
   int n_blocks = 0, block_size = 0;
@@ -214,7 +218,7 @@ int next_launch(Ctx& c, Launch* L) {
 }
 
 int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, int silu_half,
-            const void* bias, const float* resid, void* out, int ldo) {
+            const void* bias, const float* resid, void* out, int ldo, const uint8_t* Bp = nullptr) {
   bullet_handle* h = c.h;
   if (M == 0) return BULLET_OK;
   GemmArgs a;
@@ -232,7 +236,11 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   }
   if (K % 64) return set_err(BULLET_EUNSUPPORTED, "GEMM needs K %% 64 == 0 (K=%d)", K);
   const int m_tiles = (M + 127) / 128;
-  auto fits = [&](int bn) { return epi == EPI_SILU ? ((N / 2) % (bn / 2) == 0 && N % 2 == 0) : (N % bn == 0); };
+  // packed B needs 64-row aligned halves: SiLU tiles of >= 128 rows
+  auto fits = [&](int bn) {
+    if (Bp && epi == EPI_SILU && bn < 128) return false;
+    return epi == EPI_SILU ? ((N / 2) % (bn / 2) == 0 && N % 2 == 0) : (N % bn == 0);
+  };
   // Plan (bn, split-K) on the phase's m SMs: minimise waves x bytes per unit
   // (A + B tile streams), plus the split-K partial round trip; ties prefer
   // wider tiles (MMA efficiency).  Work units run one per CTA per wave.
@@ -253,6 +261,8 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   }
   if (!bn) return set_err(BULLET_EUNSUPPORTED, "GEMM N=%d not tileable", N);
   a.bn = bn; a.splits = splits;
+  a.b_packed = Bp;
+  a.b_rows = N + (epi == EPI_SILU ? silu_half - N / 2 : 0);
   a.partials = h->ph[c.phase].partials;
   a.tile_sems = h->ph[c.phase].tile_sems;
   CUtensorMap ma, mb;
@@ -370,7 +380,9 @@ int run_layer(Ctx& c, const bullet_batch* b, int layer) {
   c.kind = BULLET_K_RMSNORM1;
   if ((rc = do_rmsnorm(c, b->d_hidden, n, w.g_attn, P.h))) return rc;                       // S1
   c.kind = BULLET_K_QKV;
-  if ((rc = do_gemm(c, EPI_F32, P.h, n, d, w.w_qkv, nq, 0, w.b_qkv, nullptr, P.qkv, nq))) return rc;  // S2
+  const bullet_handle::Packed* wp = h->wp.empty() ? nullptr : &h->wp[layer];
+  if ((rc = do_gemm(c, EPI_F32, P.h, n, d, w.w_qkv, nq, 0, w.b_qkv, nullptr, P.qkv, nq,
+                    wp ? wp->qkv : nullptr))) return rc;  // S2
   c.kind = BULLET_K_ROPE_KV;
   if ((rc = do_rope(c, b, layer, P.qkv, P.q))) return rc;                                    // S3
   c.kind = BULLET_K_ATTN;
@@ -379,16 +391,17 @@ int run_layer(Ctx& c, const bullet_batch* b, int layer) {
   // into hidden and the fp32 all-reduce restores x + sum of partials (S9).
   c.kind = BULLET_K_OPROJ;
   if ((rc = do_gemm(c, (!tp || lead) ? EPI_RESID : EPI_F32, P.o, n, H * hd, w.w_o, d, 0, nullptr,
-                    b->d_hidden, b->d_hidden, d))) return rc;
+                    b->d_hidden, b->d_hidden, d, wp ? wp->o : nullptr))) return rc;
   c.kind = BULLET_K_ALLREDUCE;
   if (tp && (rc = allreduce(c, b->d_hidden, (size_t)n * d))) return rc;
   c.kind = BULLET_K_RMSNORM2;
   if ((rc = do_rmsnorm(c, b->d_hidden, n, w.g_mlp, P.h))) return rc;                        // S6
   c.kind = BULLET_K_GATE_UP;
-  if ((rc = do_gemm(c, EPI_SILU, P.h, n, d, w.w_gate_up, 2 * I, I, nullptr, nullptr, P.act, I))) return rc;  // S7
+  if ((rc = do_gemm(c, EPI_SILU, P.h, n, d, w.w_gate_up, 2 * I, I, nullptr, nullptr, P.act, I,
+                    wp ? wp->gu : nullptr))) return rc;  // S7
   c.kind = BULLET_K_DOWN;
   if ((rc = do_gemm(c, (!tp || lead) ? EPI_RESID : EPI_F32, P.act, n, I, w.w_down, d, 0, nullptr,
-                    b->d_hidden, b->d_hidden, d))) return rc;                                // S8
+                    b->d_hidden, b->d_hidden, d, wp ? wp->down : nullptr))) return rc;       // S8
   c.kind = BULLET_K_ALLREDUCE;
   if (tp && (rc = allreduce(c, b->d_hidden, (size_t)n * d))) return rc;
   return BULLET_OK;
@@ -631,6 +644,22 @@ int bullet_set_layer_weights(bullet_handle* h, int layer, const bullet_layer_wei
       (h->cfg.qkv_bias && !w->b_qkv))
     return set_err(BULLET_EINVAL, "null weight pointer");
   h->w[layer] = *w;
+  if (h->cfg.dtype == BULLET_DTYPE_BF16) {   // pack the B operands once (kernels.h layout)
+    const bullet_model_cfg& c = h->cfg;
+    const size_t nq = (size_t)(c.n_heads + 2 * c.n_kv_heads) * c.head_dim, d = c.d_model;
+    const size_t hh = (size_t)c.n_heads * c.head_dim, I = c.d_ff;
+    const size_t sz[4] = {nq * d * 2, d * hh * 2, 2 * I * d * 2, d * I * 2};
+    if (h->wp.empty()) h->wp.resize(c.n_layers);
+    bullet_handle::Packed& P = h->wp[layer];
+    if (!P.base && cudaMalloc(&P.base, sz[0] + sz[1] + sz[2] + sz[3]) != cudaSuccess)
+      return set_err(BULLET_ENOMEM, "packed weights of layer %d", layer);
+    P.qkv = P.base; P.o = P.qkv + sz[0]; P.gu = P.o + sz[1]; P.down = P.gu + sz[2];
+    CK(launch_pack_weight((const __nv_bfloat16*)w->w_qkv, (int)nq, (int)d, P.qkv, 0));
+    CK(launch_pack_weight((const __nv_bfloat16*)w->w_o, (int)d, (int)hh, P.o, 0));
+    CK(launch_pack_weight((const __nv_bfloat16*)w->w_gate_up, (int)(2 * I), (int)d, P.gu, 0));
+    CK(launch_pack_weight((const __nv_bfloat16*)w->w_down, (int)d, (int)I, P.down, 0));
+    CK(cudaStreamSynchronize(0));
+  }
   if (!h->cfg.qkv_bias) h->w[layer].b_qkv = nullptr;
   h->w_set[layer] = 1;
   return BULLET_OK;
@@ -774,6 +803,8 @@ void bullet_destroy(bullet_handle* h) {
     if (h->comm[p] && g_nccl.commDestroy) g_nccl.commDestroy(h->comm[p]);
   }
   cudaFree(h->rope_cs);
+  for (auto& P : h->wp) cudaFree(P.base);
+  cudaFree(h->op_pack);
   cudaFree(h->op_ctr);
   if (h->ev_ts) cudaEventDestroy(h->ev_ts);
   for (auto e : h->ev_pool) cudaEventDestroy(e);
@@ -795,11 +826,27 @@ int bullet_op_gemm(bullet_handle* h, int epi, const void* A, int M, int K, const
   Ctx c;
   int rc = op_ctx(h, lo, hi, stream, &c);
   if (rc) return rc;
+  const bool packed = (epi & BULLET_GEMM_PACKED) != 0;
+  epi &= ~BULLET_GEMM_PACKED;
   if (!A || !B || !out || M < 0 || K <= 0 || N <= 0 || epi < 0 || epi > 2) return set_err(BULLET_EINVAL, "gemm args");
   if (epi == EPI_RESID && !resid) return set_err(BULLET_EINVAL, "resid null");
   if (epi == EPI_SILU && (N % 2 || silu_half < N / 2)) return set_err(BULLET_EINVAL, "silu layout");
   const int ldo = epi == EPI_SILU ? N / 2 : N;
-  return do_gemm(c, epi, A, M, K, B, N, silu_half, bias, resid, out, ldo);
+  const uint8_t* Bp = nullptr;
+  if (packed) {   // pack B into scratch first (the layout bullet_step uses)
+    if (h->cfg.dtype != BULLET_DTYPE_BF16) return set_err(BULLET_EUNSUPPORTED, "packed GEMM is bf16");
+    const int rows = epi == EPI_SILU ? silu_half + N / 2 : N;
+    const size_t need = (size_t)rows * K * 2;
+    if (need > h->op_pack_bytes) {
+      cudaFree(h->op_pack);
+      h->op_pack = nullptr; h->op_pack_bytes = 0;
+      if (cudaMalloc(&h->op_pack, need) != cudaSuccess) return set_err(BULLET_ENOMEM, "pack scratch");
+      h->op_pack_bytes = need;
+    }
+    CK(launch_pack_weight((const __nv_bfloat16*)B, rows, K, h->op_pack, c.st));
+    Bp = h->op_pack;
+  }
+  return do_gemm(c, epi, A, M, K, B, N, silu_half, bias, resid, out, ldo, Bp);
 }
 
 int bullet_op_stream(bullet_handle* h, const void* src, size_t bytes, int mode, int lo, int hi,

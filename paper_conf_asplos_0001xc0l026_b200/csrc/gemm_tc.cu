@@ -70,6 +70,15 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
 
 __device__ __forceinline__ float silu_f(float z) { return z / (1.0f + __expf(-z)); }
 
+// 1-D bulk copy global -> shared, completion on an mbarrier.
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
 // Epilogue for 32 consecutive output columns [col, col+32) of row m.
 __device__ __forceinline__ void epi_store(const GemmArgs& a, int m, int col, const float* v,
                                           const float* u) {
@@ -191,8 +200,18 @@ __global__ void __launch_bounds__(NT, 1)
           uint8_t* sa = smem + s * st_bytes;
           mbar_arrive_expect_tx(full + s, st_bytes);
           tma_load_2d(sa, &mapA, full + s, kb * BK, m_blk * BM);
-          tma_load_2d(sa + A_BYTES, &mapB, full + s, kb * BK, r0);
-          tma_load_2d(sa + A_BYTES + b_bytes / 2, &mapB, full + s, kb * BK, r1);
+          if (a.b_packed) {   // pre-swizzled tiles: contiguous bulk copies
+            const uint8_t* kbase = a.b_packed + (size_t)kb * (a.b_rows / 64) * 8192;
+            if (r1 == r0 + bn / 2) {
+              bulk_g2s(sa + A_BYTES, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s);
+            } else {
+              bulk_g2s(sa + A_BYTES, kbase + (size_t)(r0 / 64) * 8192, b_bytes / 2, full + s);
+              bulk_g2s(sa + A_BYTES + b_bytes / 2, kbase + (size_t)(r1 / 64) * 8192, b_bytes / 2, full + s);
+            }
+          } else {
+            tma_load_2d(sa + A_BYTES, &mapB, full + s, kb * BK, r0);
+            tma_load_2d(sa + A_BYTES + b_bytes / 2, &mapB, full + s, kb * BK, r1);
+          }
           if (++s == n_stages) { s = 0; ph ^= 1; }
         }
         ++it;
@@ -318,6 +337,28 @@ __global__ void __launch_bounds__(NT, 1)
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
   }
+}
+
+// One thread per 16-byte chunk of the packed image (see kernels.h).
+__global__ void k_pack_weight(const __nv_bfloat16* __restrict__ W, int R, int K, uint8_t* __restrict__ out) {
+  const size_t n_chunks = (size_t)R * K / 8;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n_chunks; i += (size_t)gridDim.x * blockDim.x) {
+    const int p = i & 7;                       // chunk position within the 128-byte row
+    const size_t row_lin = i >> 3;             // (kb, rb, r) linearised
+    const int r = row_lin & 63;
+    const size_t tile = row_lin >> 6;          // kb * (R/64) + rb
+    const int rb = tile % (R / 64);
+    const int kb = tile / (R / 64);
+    const int c = p ^ (r & 7);                 // logical k-chunk held at position p
+    const uint4 v = *reinterpret_cast<const uint4*>(W + (size_t)(rb * 64 + r) * K + kb * 64 + c * 8);
+    *reinterpret_cast<uint4*>(out + i * 16) = v;
+  }
+}
+
+cudaError_t launch_pack_weight(const __nv_bfloat16* W, int R, int K, uint8_t* out, cudaStream_t st) {
+  if (R % 64 || K % 64) return cudaErrorInvalidValue;
+  k_pack_weight<<<1184, 256, 0, st>>>(W, R, K, out);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_gemm_tc(const CUtensorMap& mapA, const CUtensorMap& mapB, const GemmArgs& a,

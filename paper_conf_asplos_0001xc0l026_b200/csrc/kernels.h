@@ -20,8 +20,17 @@ struct GemmArgs {
   int ldo;
   float* partials;    // split-K: [units][128][bn]
   int* tile_sems;     // split-K: [tiles], zero between launches (self-resetting)
+  const uint8_t* b_packed;  // B pre-packed by pack_weight (else B comes through mapB)
+  int b_rows;               // rows of B (packed layout stride)
   Launch L;
 };
+
+// Packed weight layout: W[R][K] bf16 -> [K/64][R/64] tiles of 64 rows x 64 k
+// (8 KB), each stored as the 128-byte-swizzled shared-memory image a TMA
+// SWIZZLE_128B load would produce (16-byte chunk c of row r at c ^ (r & 7)).
+// A B-operand stage of bn rows at k-block kb is then one or two contiguous
+// bulk copies.
+cudaError_t launch_pack_weight(const __nv_bfloat16* W, int R, int K, uint8_t* out, cudaStream_t st);
 
 struct NormArgs {
   const float* x; const void* g; void* out;

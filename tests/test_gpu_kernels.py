@@ -52,16 +52,18 @@ def _int_operands(rng, M, K, N):
     (257, 4096, 4096, 10, 50),      # 40-SM gated range, split-K fixup
     (64, 1280, 8192, 0, 16),        # 16 SMs, K = 8192
 ])
-def test_gemm_f32_epilogue_bit_exact(B, M, N, K, lo, hi):
+@pytest.mark.parametrize("packed", [False, True])
+def test_gemm_f32_epilogue_bit_exact(B, M, N, K, lo, hi, packed):
     """Integer operands in {-2..2}: bf16 products and fp32 sums are exact, so
-    the tcgen05 GEMM must equal the exact product bit for bit."""
+    the tcgen05 GEMM must equal the exact product bit for bit,
+    with B through TMA tiles or through the packed bulk-copy layout."""
     bl, _ = _handle(B, SMALL)
     rng = np.random.default_rng(M + N)
     A, W = _int_operands(rng, M, K, N)
     bias = rng.integers(-3, 4, size=N).astype(np.float32)
     out = torch.full((M, N), float("nan"), device="cuda")
     bl.op_gemm(B.EPI_F32, torch.from_numpy(A).to("cuda", bf16), torch.from_numpy(W).to("cuda", bf16),
-               out, bias=torch.from_numpy(bias).to("cuda", bf16), lo=lo, hi=hi)
+               out, bias=torch.from_numpy(bias).to("cuda", bf16), lo=lo, hi=hi, packed=packed)
     torch.cuda.synchronize()
     # fp64 BLAS is exact here: integer partial sums stay far below 2^53
     ref = (torch.from_numpy(A).double() @ torch.from_numpy(W).double().T).numpy() + bias
@@ -81,7 +83,8 @@ def test_gemm_matches_oracle_linear_small(B):
     assert np.abs(out.cpu().numpy() - ref).max() < 2e-4
 
 
-def test_gemm_resid_in_place_bit_exact(B):
+@pytest.mark.parametrize("packed", [False, True])
+def test_gemm_resid_in_place_bit_exact(B, packed):
     bl, _ = _handle(B, SMALL)
     rng = np.random.default_rng(7)
     M, K, N = 333, 4096, 4096
@@ -89,13 +92,14 @@ def test_gemm_resid_in_place_bit_exact(B):
     R = rng.integers(-50, 50, size=(M, N)).astype(np.float32)
     h = torch.from_numpy(R).cuda()
     bl.op_gemm(B.EPI_RESID, torch.from_numpy(A).to("cuda", bf16), torch.from_numpy(W).to("cuda", bf16),
-               h, resid=h)
+               h, resid=h, packed=packed)
     ref = R.astype(np.float64) + (torch.from_numpy(A).double() @ torch.from_numpy(W).double().T).numpy()
     assert np.array_equal(h.cpu().numpy(), ref.astype(np.float32))
 
 
+@pytest.mark.parametrize("packed", [False, True])
 @pytest.mark.parametrize("M,lo,hi", [(128, 0, None), (1000, 0, None), (130, 100, 148)])
-def test_gemm_silu_mul(B, M, lo, hi):
+def test_gemm_silu_mul(B, M, lo, hi, packed):
     """gate_up epilogue: a = silu(g) * u rounded to bf16 (point R5); integer
     g, u exact, the silu/rounding within 1 bf16 ulp of the fp64 value."""
     bl, _ = _handle(B, SMALL)
@@ -106,7 +110,7 @@ def test_gemm_silu_mul(B, M, lo, hi):
     out = torch.zeros(M, I, dtype=bf16, device="cuda")
     hi = bl.n_sms if hi is None else min(hi, bl.n_sms)
     bl.op_gemm(B.EPI_SILU, torch.from_numpy(A).to("cuda", bf16), torch.from_numpy(W).to("cuda", bf16),
-               out, silu_half=I, lo=lo, hi=hi)
+               out, silu_half=I, lo=lo, hi=hi, packed=packed)
     gu = A.astype(np.float64) @ W.T.astype(np.float64)
     g, u = gu[:, :I], gu[:, I:]
     ref = g / (1 + np.exp(-g)) * u
