@@ -325,7 +325,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
   static const int dbg = getenv("BULLET_DBG") ? atoi(getenv("BULLET_DBG")) : 0;
   a.dbg = dbg;
   const bool bf16 = h->cfg.dtype == BULLET_DTYPE_BF16;
-  if (kind == 0) kind = (bf16 && a.hd == 128) ? (max_qlen(b) > 1 ? 2 : 3) : 1;
+  if (kind == 0) kind = (bf16 && a.hd == 128) ? (max_qlen(b) > 1 ? 4 : 3) : 1;
   if (kind == 3 && max_kv(b) > attn_decode_max_blocks() * h->block_size) kind = c.op ? -1 : 1;
   if (kind == -1) return set_err(BULLET_EUNSUPPORTED, "tensor-core decode attention: context too long");
   if (kind == 3) {
@@ -336,7 +336,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     LAUNCH(c, launch_attn_decode_tc(a, h->n_sms, c.st));
     return BULLET_OK;
   }
-  if (kind == 2) {
+  if (kind == 2 || kind == 4) {
     if (!bf16 || a.hd != 128) return set_err(BULLET_EUNSUPPORTED, "tensor-core attention: bf16, hd 128 only");
     PhaseWS& P = h->ph[c.phase];
     a.tiles = P.tiles; a.n_tiles = P.n_tiles;
@@ -347,7 +347,8 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     }
     int rc = next_launch(c, &a.L);
     if (rc) return rc;
-    LAUNCH(c, launch_attn_prefill_tc(a, h->n_sms * 2, c.st));
+    if (kind == 4) LAUNCH(c, launch_attn_prefill5(a, h->n_sms * 2, c.st));
+    else LAUNCH(c, launch_attn_prefill_tc(a, h->n_sms * 2, c.st));
     return BULLET_OK;
   }
   int rc = next_launch(c, &a.L);
@@ -889,7 +890,7 @@ int bullet_op_attention(bullet_handle* h, const bullet_batch* b, int layer, cons
   Ctx c;
   int rc = op_ctx(h, lo, hi, stream, &c);
   if (rc) return rc;
-  if (!b || !q || !o || layer < 0 || layer >= h->cfg.n_layers || kind < 0 || kind > 3)
+  if (!b || !q || !o || layer < 0 || layer >= h->cfg.n_layers || kind < 0 || kind > 4)
     return set_err(BULLET_EINVAL, "attention args");
   bullet_batch bb = *b;
   bb.layer_begin = layer; bb.layer_end = layer;

@@ -15,7 +15,7 @@
 namespace bl {
 
 namespace {
-constexpr int BQ = ATTN_TC_BQ, BKV = 64, HDIM = 128, KB = 16;
+constexpr int BQ = 64, BKV = 64, HDIM = 128, KB = 16;
 constexpr int TILE_BYTES = 64 * HDIM * 2;  // 16 KB
 
 __device__ __forceinline__ uint32_t swz(int row, int chunk) {  // byte offset in a [64][128] bf16 tile
@@ -92,9 +92,10 @@ __global__ void __launch_bounds__(128) k_attn_prefill_tc(AttnArgs a) {
     if (u >= units) break;
     if (tid == 0) log_unit(a.L, u);
     const int2 rt = a.tiles[u / a.H];
-    const int h = u % a.H, g = h / grp, r = rt.x, q0 = rt.y * BQ;
+    const int h = u % a.H, g = h / grp, r = rt.x;
     const int tok0 = __ldg(a.cu + r);
     const int q_len = __ldg(a.cu + r + 1) - tok0;
+    for (int q0 = rt.y * ATTN_TC_BQ; q0 < min(q_len, (rt.y + 1) * ATTN_TC_BQ); q0 += BQ) {  // 64-row halves
     const int ctx = __ldg(a.ctx + r);
     const int kv_len = ctx + q_len;
     const int kmax = min(kv_len, ctx + q0 + BQ);
@@ -237,6 +238,7 @@ __global__ void __launch_bounds__(128) k_attn_prefill_tc(AttnArgs a) {
       }
     }
     __syncthreads();
+    }
   }
 }
 

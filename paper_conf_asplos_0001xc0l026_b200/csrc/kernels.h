@@ -82,6 +82,7 @@ cudaError_t launch_rope_kv(const RopeArgs& a, int grid, cudaStream_t st);
 template <typename T>
 cudaError_t launch_attn_simt(const AttnArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_attn_prefill_tc(const AttnArgs& a, int grid, cudaStream_t st);
+cudaError_t launch_attn_prefill5(const AttnArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, cudaStream_t st);
 size_t attn_decode_smem_bytes();
 int attn_decode_max_blocks();
@@ -89,7 +90,7 @@ cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);
 cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_probe(int* out_smid, int n, cudaStream_t st);
 
-constexpr int ATTN_TC_BQ = 64;    // query rows per tensor-core attention tile
+constexpr int ATTN_TC_BQ = 128;   // query rows per prefill attention tile (plan granularity)
 constexpr int ROWS_PER_UNIT = 8;  // rows per work unit of row-wise kernels
 
 }  // namespace bl

@@ -192,14 +192,15 @@ L70_TP8 = synth.MODELS["llama3.1-70b"].shard(8)       # GQA group 8
 
 
 @pytest.mark.parametrize("m,kind", [(SMALL, 1), (SMALL, 2), (TINY, 1), (LLAMA, 2), (LLAMA, 1),
+                                    (SMALL, 4), (LLAMA, 4), (QWEN_TP2, 4), (L70_TP8, 4),
                                     (SMALL, 3), (LLAMA, 3), (QWEN_TP2, 3), (L70_TP8, 3)])
 def test_attention_vs_oracle(B, m, kind):
     """Paged attention (decode rows and causal prefill rows) vs the oracle's
     plain softmax attention through the block table.  kind 1 SIMT, 2
     tensor-core prefill, 3 tensor-core decode (one query per request)."""
     q_lens, ctx = [150, 64, 1, 1, 1, 1], [0, 0, 0, 63, 200, 1000]
-    if kind == 2:
-        q_lens, ctx = [150, 64, 1, 77], [0, 0, 0, 0]
+    if kind in (2, 4):
+        q_lens, ctx = [150, 64, 1, 77, 300], [0, 0, 0, 0, 0]
     if kind == 3:
         q_lens, ctx = [1] * 7, [0, 15, 16, 63, 200, 1000, 2047]
     lay = synth.paged_layout(q_lens, ctx, 16, seed_offset=5)
