@@ -145,7 +145,10 @@ class Step:
             del k_, v_
         torch.cuda.empty_cache()
         maxpos = max(a + b for a, b in zip(q, c)) + 16
-        self.bl = B.Bullet(B.Model.of(m), self.pools, self.n_p, self.n_d, maxpos)
+        pp = os.path.join(ROOT, "profiles", "perf_params_b200.json")   # fitted by scripts/fit_perfmodel.py
+        self.perf_json = open(pp).read() if os.path.exists(pp) else None
+        self.bl = B.Bullet(B.Model.of(m), self.pools, self.n_p, self.n_d, maxpos,
+                           perf_params_json=self.perf_json)
         for l in range(n_layers):
             self.bl.set_layer_weights(l, self.weights[l])
         bt = self.lay.block_table
@@ -180,21 +183,30 @@ class Step:
         return (self.n_p * 1 + self.n_d * k) / self.m.n_layers
 
     def tune(self, cands, reps=3):
-        """Isolated prefill layer on p SMs and decode layer-step on N-p SMs;
-        k = round(T_p / T_d); pick the p with the best predicted co-run
-        throughput (the model's (u_k, k) choice, measured instead of fitted)."""
+        """For each candidate prefill SM count p: time the isolated prefill
+        layer on p SMs and decode layer-step on N-p SMs, set k = round(T_p/T_d)
+        (decode steps per prefill layer), then time the real co-run
+        step and the fitted model's prediction; pick the best measured co-run
+        tokens/s."""
         B = self.B
-        self.dec.layer_end = 1
         res = []
         for p in cands:
+            self.dec.layer_end = 1
             self.time_steps(1, p, B.CORUN, dec=False)
             tp = self.time_steps(reps, p, B.CORUN, dec=False)
             self.time_steps(1, p, B.CORUN, pre=False)
             td = self.time_steps(reps, p, B.CORUN, pre=False)
             k = int(min(self.k_max, max(1, round(tp / td))))
-            est = self.tokens(k) / max(tp, k * td)
-            res.append({"p": p, "t_prefill_ms": tp, "t_decode_ms": td, "k": k, "est_tok_s": est * 1e3})
-        best = max(res, key=lambda r: r["est_tok_s"])
+            self.dec.layer_end = k
+            self.time_steps(1, p, B.CORUN)
+            tco = self.time_steps(reps, p, B.CORUN)
+            q, c = self.pre.cu[1:] - self.pre.cu[:-1], self.pre.ctx_lens
+            mp = self.bl.predict_us(q, c, p, self.N - p) / 1e3
+            md = self.bl.predict_us([1] * self.n_d, self.dec.ctx_lens, self.N - p, p) / 1e3 * k
+            res.append({"p": p, "k": k, "t_prefill_ms": tp, "t_decode_ms": td, "t_corun_ms": tco,
+                        "tok_s": self.tokens(k) / tco * 1e3, "model_corun_ms": max(mp, md)})
+        best = max(res, key=lambda r: r["tok_s"])
+        self.dec.layer_end = 1
         return best, res
 
 
@@ -305,6 +317,14 @@ def main():
                 print(json.dumps(r), file=sys.stderr)
     else:
         p, k, table = args.p, args.k, []
+    # the paper's scheduler on this batch (Alg. 1 with the fitted model, Table 2
+    # ShareGPT SLOs: 3.0 ms/token normalized TTFT, 150 ms TPOT)
+    state = dict(layers_done=0, total_layers=S.m.n_layers, prefill_lens=list(S.wl.prefill_lens),
+                 prefill_waited_ms=[0.0] * S.n_pre, pending_lens=[], pending_waited_ms=[],
+                 decode_tokens=[64] * S.n_d, decode_elapsed_ms=[64 * 30.0] * S.n_d,
+                 decode_mean_ctx=float(np.mean(S.wl.decode_ctx)), u_k=p, v_k=N - p)
+    slo = {"ttft_norm_ms_per_tok": 3.0, "tpot_ms": 150.0, "w_max": 4, "v_min": 16, "percentile": 0.9}
+    model_split = S.bl.choose_split(state, slo)
     S.dec.layer_end = k
     # ---- alone-on-full-GPU references (per layer)
     t_pre_full = S.time_steps(3, N, B.CORUN, dec=False)
@@ -416,6 +436,8 @@ def main():
         "gpu_launches": int(launches),
         "clocks": clk.summary(),
         "tuning": table,
+        "alg1_split": {"prefill_sm_count": model_split[0], "decode_layer_steps": model_split[1],
+                       "perf_params": "profiles/perf_params_b200.json" if S.perf_json else "unfitted"},
     }
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
         dt, tk, desc = oracle_sample(S.m, S.wl)

@@ -114,3 +114,22 @@ def test_predict_rejects_bad_sm_count():
     assert e.value.code == -4
     with pytest.raises(B.BulletError):
         pm.predict_us([10], [0], 149)
+
+
+def test_fitted_perf_params_load_and_match_oracle():
+    """profiles/perf_params_b200.json (fitted on the B200 by
+    scripts/fit_perfmodel.py) parses in the C++ model and predicts exactly
+    what the oracle's Eq. 2 reading predicts with the same parameters."""
+    import os
+    path = os.path.join(os.path.dirname(os.path.dirname(__file__)), "profiles", "perf_params_b200.json")
+    if not os.path.exists(path):
+        pytest.skip("no fitted parameters yet")
+    P = json.load(open(path))
+    pm = _pm("llama8b", params=P)
+    shape = dict(MODELS["llama8b"])
+    for q, c in [([4096], [0]), ([1] * 128, [1024] * 128), ([512] * 8, [0] * 8)]:
+        for m, co in [(148, 0), (40, 108), (100, 48), (16, 0)]:
+            got = pm.predict_us(q, c, m, co)
+            ref = PM.layer_time(dict(shape, q_lens=q, ctx_lens=c), P, m, co) * 1e6
+            assert got == pytest.approx(ref, rel=1e-12)
+    assert P["fit"]["mre_heldout"] < 0.5
