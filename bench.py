@@ -357,6 +357,9 @@ def main():
     bound, work = kernel_work(S, dom[0], dom[1])
     avg_ms = float(np.mean(by[dom]))
     P, src = peaks()
+    tf = os.path.join(ROOT, "profiles", "r01_traffic.json")   # ncu --set full capture of the same kernel
+    dom_name = f"{dom[0]} ({'prefill' if dom[1] == 0 else 'decode'})"
+    traffic = json.load(open(tf))["bytes"].get(dom_name) if os.path.exists(tf) else None
     if bound == "tensor":
         achieved = work / (avg_ms * 1e-3) / 1e12
         peak, unit = P.get("bf16_tflops_sustained", P["bf16_tflops"]), "TFLOP/s"
@@ -427,9 +430,10 @@ def main():
             "prefill_tensor_frac": f_pre / (t_co * 1e-3) / (P.get("bf16_tflops_sustained", 1395.1) * 1e12),
             "decode_hbm_frac": b_dec / (t_co * 1e-3) / (P["hbm_gbs"] * 1e9),
             "decode_hbm_gbs": b_dec / (t_co * 1e-3) / 1e9},
-        "roofline": {"bound": bound, "kernel": f"{dom[0]} ({'prefill' if dom[1] == 0 else 'decode'})",
+        "roofline": {"bound": bound, "kernel": dom_name,
                      "achieved": achieved, "peak": peak, "unit": unit, "frac": achieved / peak,
-                     "peak_source": src, "avg_launch_ms": avg_ms, "traffic": None},
+                     "peak_source": src, "avg_launch_ms": avg_ms, "traffic": traffic,
+                     "algorithmic_" + ("flops" if bound == "tensor" else "bytes"): work},
         "kernel_ms": {f"{k_}/{'pre' if ph == 0 else 'dec'}": round(sum(v) / 2, 4) for (k_, ph), v in by.items()},
         "e2e": {"value": ws * tok / (t_e2e * 1e-3), "unit": "tokens/s", "h2d_bytes_per_step": int(h2d),
                 "d2h_bytes_per_step": int(d2h), "ms_per_step": t_e2e},

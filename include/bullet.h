@@ -263,7 +263,8 @@ int bullet_op_gemm(bullet_handle *h, int epi, const void *d_A, int M, int K, con
 
 /* KI2 microbenchmark: stream `bytes` (multiple of 64 KB) from d_src on the
  * SMs sigma[lo:hi) and discard them; mode 0 LDG.128, 1 cp.async.bulk (TMA
- * bulk copies), 2 cp.async 16 B.  Feeds the perf-model fit. */
+ * bulk copies), 2 cp.async 16 B; mode | (param << 8): LDG with `param` warps
+ * per SM, cp.async with `param` 64 KB units in flight.  KI2, DESIGN.md §5. */
 int bullet_op_stream(bullet_handle *h, const void *d_src, size_t bytes, int mode, int lo, int hi,
                      void *stream);
 

@@ -855,10 +855,11 @@ int bullet_op_stream(bullet_handle* h, const void* src, size_t bytes, int mode, 
   Ctx c;
   int rc = op_ctx(h, lo, hi, stream, &c);
   if (rc) return rc;
-  if (!src || bytes == 0 || mode < 0 || mode > 2) return set_err(BULLET_EINVAL, "stream args");
+  if (!src || bytes == 0 || (mode & 0xff) > 2 || mode < 0) return set_err(BULLET_EINVAL, "stream args");
   StreamArgs a;
   memset(&a, 0, sizeof a);
-  a.src = (const uint8_t*)src; a.bytes = bytes; a.mode = mode; a.sink = (uint32_t*)h->op_ctr;
+  a.src = (const uint8_t*)src; a.bytes = bytes; a.mode = mode & 0xff; a.param = mode >> 8;
+  a.sink = (uint32_t*)h->op_ctr;
   if ((rc = next_launch(c, &a.L))) return rc;
   LAUNCH(c, launch_stream(a, h->n_sms, c.st));
   return BULLET_OK;

@@ -58,7 +58,7 @@ struct AttnArgs {
 };
 
 struct StreamArgs {   // KI2 streaming microbenchmark
-  const uint8_t* src; size_t bytes; int mode; uint32_t* sink;
+  const uint8_t* src; size_t bytes; int mode; int param; uint32_t* sink;
   Launch L;
 };
 

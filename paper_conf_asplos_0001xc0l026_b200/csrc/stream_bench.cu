@@ -31,6 +31,7 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
   uint32_t acc = 0;
   if (a.mode == 0) {
     const size_t units = a.bytes / 8192;
+    if (a.param > 0 && tid >= a.param * 32) return;   // only `param` warps stream
     for (;;) {
       int u = 0;
       if (lane == 0) u = atomicAdd(a.L.ctr, 1);
@@ -86,7 +87,12 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
       for (int i = 0; i < 8; ++i) cp_async16(d + (tid + i * 512) * 16, p + (tid + i * 512) * 16);
       cp_async_commit();
       ++n;
-      if (n >= 3) {
+      if (a.param == 2) {            // 2 units (128 KB) in flight
+        if (n >= 2) {
+          cp_async_wait<1>();
+          acc ^= *reinterpret_cast<const uint32_t*>(sm + (n % 3) * 65536 + tid * 16);
+        }
+      } else if (n >= 3) {           // 3 units (192 KB) in flight
         cp_async_wait<2>();
         acc ^= *reinterpret_cast<const uint32_t*>(sm + (n % 3) * 65536 + tid * 16);
       }
