@@ -122,11 +122,16 @@ class Step:
     def __init__(self, config: str, k_max: int, device="cuda"):
         import paper_conf_asplos_0001xc0l026_b200 as B
         self.B = B
+        from paper_conf_asplos_0001xc0l026_b200 import parallel
         self.wl = synth.workload(config)
-        self.m = synth.MODELS[self.wl.model]
-        if self.wl.tp != 1:
-            raise SystemExit(f"config {config} needs tensor parallelism (tp={self.wl.tp}); "
-                             "bench.py runs it only under torchrun with WORLD_SIZE == tp")
+        self.m_full = synth.MODELS[self.wl.model]
+        self.tp = self.wl.tp
+        ws = int(os.environ.get("WORLD_SIZE", "1"))
+        self.rank = int(os.environ.get("RANK", "0"))
+        if self.tp != 1 and ws != self.tp:
+            raise SystemExit(f"config {config} is tensor-parallel (tp={self.tp}): run it under torchrun "
+                             f"with --nproc-per-node {self.tp}")
+        self.m = self.m_full.shard(self.tp) if self.tp > 1 else self.m_full
         m = self.m
         self.k_max = k_max
         n_layers = max(1, k_max)
@@ -137,8 +142,11 @@ class Step:
         td = torch.bfloat16 if m.dtype == "bf16" else torch.float32
         self.pools, self.weights = [], []
         for l in range(n_layers):
-            w = synth.layer_weights(m, l, device=device)
-            self.weights.append({k: (None if v is None else v.to(td)) for k, v in w.items()})
+            w = synth.layer_weights(self.m_full, l, device=device)   # same seeds on every rank
+            w = {k: (None if v is None else v.to(td)) for k, v in w.items()}
+            if self.tp > 1:   # Megatron shard of this rank (parallel.py)
+                w = parallel.shard_layer_weights(w, B.Model.of(self.m_full), self.tp, self.rank)
+            self.weights.append(w)
             del w
             k_, v_ = synth.kv_pool(m, self.lay.n_blocks, 16, l, device=device)
             self.pools.append((k_.to(td), v_.to(td)))
@@ -147,7 +155,9 @@ class Step:
         maxpos = max(a + b for a, b in zip(q, c)) + 16
         pp = os.path.join(ROOT, "profiles", "perf_params_b200.json")   # fitted by scripts/fit_perfmodel.py
         self.perf_json = open(pp).read() if os.path.exists(pp) else None
+        uids = parallel.nccl_uids() if self.tp > 1 else None
         self.bl = B.Bullet(B.Model.of(m), self.pools, self.n_p, self.n_d, maxpos,
+                           tp_size=self.tp, tp_rank=self.rank, nccl_uids=uids,
                            perf_params_json=self.perf_json)
         for l in range(n_layers):
             self.bl.set_layer_weights(l, self.weights[l])
@@ -405,8 +415,9 @@ def main():
     t_e2e = allreduce_max(e0.elapsed_time(e1) / args.steps, ws)
     # ---- report
     tok = S.tokens(k)
-    value = ws * tok / (t_co * 1e-3)
-    ts_value = ws * tok / (t_ts * 1e-3)
+    groups = ws // S.tp            # replicas (8B) or one TP group (configs 4-5)
+    value = groups * tok / (t_co * 1e-3)
+    ts_value = groups * tok / (t_ts * 1e-3)
     m = S.m
     nq = (m.n_heads + 2 * m.n_kv_heads) * m.head_dim
     w_bytes = 2.0 * (nq * m.d_model + m.d_model * m.n_heads * m.head_dim + 3 * m.d_model * m.d_ff)
@@ -421,7 +432,8 @@ def main():
                    "prefill_reqs": S.n_pre, "decode_reqs": S.n_d,
                    "decode_ctx_mean": float(np.mean(S.wl.decode_ctx)), "prefill_layers_per_step": 1,
                    "decode_layer_steps": k, "prefill_sm_count": p, "n_sms": N,
-                   "parallelism": f"replicas x{ws}" if ws > 1 else "single GPU",
+                   "parallelism": (f"tp{S.tp}" if S.tp > 1 else (f"replicas x{ws}" if ws > 1 else "single GPU")),
+                   "tokens_per_s_per_gpu": value / ws,
                    "l2": "inputs larger than L2 (weights + KV per step >> 126 MB)"},
         "timesliced": {"value": ts_value, "ms_per_step": t_ts},
         "corun_speedup_vs_timesliced": t_ts / t_co,
@@ -435,7 +447,7 @@ def main():
                      "peak_source": src, "avg_launch_ms": avg_ms, "traffic": traffic,
                      "algorithmic_" + ("flops" if bound == "tensor" else "bytes"): work},
         "kernel_ms": {f"{k_}/{'pre' if ph == 0 else 'dec'}": round(sum(v) / 2, 4) for (k_, ph), v in by.items()},
-        "e2e": {"value": ws * tok / (t_e2e * 1e-3), "unit": "tokens/s", "h2d_bytes_per_step": int(h2d),
+        "e2e": {"value": groups * tok / (t_e2e * 1e-3), "unit": "tokens/s", "h2d_bytes_per_step": int(h2d),
                 "d2h_bytes_per_step": int(d2h), "ms_per_step": t_e2e},
         "gpu_launches": int(launches),
         "clocks": clk.summary(),
