@@ -426,7 +426,8 @@ def main():
     out = {
         "metric": "co-run tokens/s/GPU vs time-sliced; decode HBM GB/s; prefill tensor-pipe util",
         "value": value, "unit": "tokens/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": t_co, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "ms_per_step": t_co, "higher_is_better": True, "scaling": "strong" if S.tp > 1 else "weak",
+        "vs_baseline": None,
         "dtype": "bf16" if m.dtype == "bf16" else "fp32", "data": "synthetic (random-init weights, seeded request mix)",
         "config": {"workload": args.config, "model": S.wl.model, "prefill_tokens": S.n_p,
                    "prefill_reqs": S.n_pre, "decode_reqs": S.n_d,
