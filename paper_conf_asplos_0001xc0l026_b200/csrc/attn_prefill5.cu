@@ -3,28 +3,35 @@
 // FlashAttention).
 //
 // Work unit = (request, 128-row query tile, query head), LPT order from the
-// plan kernel.  Two CTAs per SM (96 KB smem, 256 TMEM columns each) so one
-// CTA's softmax overlaps the other's MMAs.  Per 64-key KV tile:
-//   S  = Q K^T        tcgen05.mma M=128 (queries) N=64 (keys) -> TMEM fp32
-//   softmax          4 warps, thread t owns query row t = TMEM lane t:
-//                    tcgen05.ld, causal mask, exp2 against a lazily moved
-//                    reference max, P = hi + lo (two bf16 tiles, R-4b) -> smem
-//   O += P V         tcgen05.mma M=128 N=128 (dims), V used as an MN-major
-//                    operand straight from its [key][dim] tile; O stays in
-//                    TMEM, rescaled only when a row max grows by > 2^8
-// K/V rows are gathered through the block table with coalesced cp.async into
-// the 128-byte-swizzled layouts the UMMA descriptors describe; K(t+1) loads
-// during softmax(t), V(t+1) during S(t+1).
+// plan kernel.  Two CTAs per SM (96 KB smem, 256 TMEM columns each).  Per
+// 64-key KV tile t:
+//   S(t) = Q K(t)^T   tcgen05.mma M=128 (queries) N=64 (keys) -> TMEM fp32,
+//                     double-buffered so S(t+1) runs during softmax(t)
+//   softmax           4 warps, thread r owns query row r = TMEM lane r:
+//                     tcgen05.ld, causal mask, exp2 against a lazily moved
+//                     reference max, P = hi + lo (two bf16 halves, R-4b)
+//                     tcgen05.st'd over S(t) in TMEM
+//   O += P V          tcgen05.mma with A = P from TMEM, B = V(t) used as an
+//                     MN-major operand straight from its [key][dim] tile; O
+//                     stays in TMEM, rescaled only when a row max grows > 2^8
+// One __syncthreads per tile: after it one thread issues S(t+1) and PV(t)
+// back to back.  K/V rows are gathered through the block table with coalesced
+// cp.async into the 128-byte-swizzled layouts the UMMA descriptors describe,
+// two buffers each: K(t+2) loads from tile t on, V(t+1) during tile t.
 #include "kernels.h"
 
 namespace bl {
 
 namespace {
 constexpr int BQ = 128, BKV = 64, HD = 128, KB = 16, NT = 128;
-// smem: Q [2][128][128 B] | K [2][64][128 B] | V [2][64][128 B] | Phi, Plo [128][128 B]
-constexpr int OFF_Q = 0, OFF_K = 32768, OFF_V = 49152, OFF_PH = 65536, OFF_PL = 81920;
-constexpr int SMEM_BYTES = 98304 + 1024 + 64;
-constexpr uint32_t TMEM_COLS = 256;   // S: [0, 64), O: [128, 256)
+// smem: Q [2][128][128 B] | K[2 buffers] [2][64][128 B] | V[2 buffers] [2][64][128 B]
+// = 96 KB + barriers: two CTAs per SM.  The dynamic window must start
+// 1024-byte aligned (128-byte swizzle atoms); checked at entry.
+constexpr int OFF_Q = 0, OFF_K = 32768, OFF_V = 65536;
+constexpr int SMEM_BYTES = 98304 + 64;
+// TMEM: S/P double buffer in columns [0,64) and [64,128) (P = bf16 hi|lo
+// packed two per column, written over the S it came from), O in [128,256)
+constexpr uint32_t TMEM_COLS = 256;
 
 // 128-byte swizzled offset of 16-byte chunk c of `row` in a tile whose
 // 64-element halves are `half` bytes apart
@@ -44,6 +51,12 @@ __device__ __forceinline__ void tc_mma(uint32_t d, uint64_t ad, uint64_t bd, uin
       "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
       "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
       "l"(ad), "l"(bd), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void tc_mma_ts(uint32_t d, uint32_t a_tmem, uint64_t bd, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d),
+      "r"(a_tmem), "l"(bd), "r"(idesc), "r"(acc));
 }
 __device__ __forceinline__ void tc_commit(uint64_t* bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
@@ -86,6 +99,32 @@ __device__ __forceinline__ void cp_async16_zfill(void* dst, const void* src, boo
                "r"(valid ? 16 : 0)
                : "memory");
 }
+__device__ __forceinline__ float ex2(float x) {   // 2^x, MUFU only (ftz)
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+// Blackwell packed fp32 pairs (FFMA2 / FADD2)
+__device__ __forceinline__ float2 ffma2(float2 a, float b, float c) {
+  unsigned long long d;
+  const float2 bb = make_float2(b, b), cc = make_float2(c, c);
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d)
+      : "l"(*reinterpret_cast<const unsigned long long*>(&a)), "l"(*reinterpret_cast<const unsigned long long*>(&bb)),
+        "l"(*reinterpret_cast<const unsigned long long*>(&cc)));
+  return *reinterpret_cast<float2*>(&d);
+}
+__device__ __forceinline__ float2 fadd2(float2 a, float2 b) {
+  unsigned long long d;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d)
+      : "l"(*reinterpret_cast<const unsigned long long*>(&a)), "l"(*reinterpret_cast<const unsigned long long*>(&b)));
+  return *reinterpret_cast<float2*>(&d);
+}
+__device__ __forceinline__ float2 fsub2(float2 a, float2 b) {
+  unsigned long long d;
+  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d)
+      : "l"(*reinterpret_cast<const unsigned long long*>(&a)), "l"(*reinterpret_cast<const unsigned long long*>(&b)));
+  return *reinterpret_cast<float2*>(&d);
+}
 __device__ __forceinline__ uint32_t pack_bf2(float a, float b) {
   __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
   return *reinterpret_cast<uint32_t*>(&h);
@@ -94,8 +133,9 @@ __device__ __forceinline__ uint32_t pack_bf2(float a, float b) {
 
 __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
   if (!gate_ok(a.L.gate)) return;
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* sm = smem_raw;
+  if (smem_u32(sm) & 1023) __trap();   // swizzle atoms need 1024-byte alignment
   uint64_t* bar_s = reinterpret_cast<uint64_t*>(sm + 98304);
   uint64_t* bar_o = bar_s + 1;
   uint32_t* tslot = reinterpret_cast<uint32_t*>(bar_o + 1);
@@ -164,104 +204,119 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
                          pool + (((size_t)blk * a.Hkv + g) * KB + (ok ? kp % KB : 0)) * HD + c * 8, ok);
       }
     };
+    auto issue_s = [&](int kt) {       // S(kt) = Q K(kt)^T -> TMEM buffer kt&1
+      const uint32_t qa = sbase + OFF_Q, ka = sbase + OFF_K + (kt & 1) * 16384;
+#pragma unroll
+      for (int kk = 0; kk < HD / 16; ++kk)
+        tc_mma(t_s + (kt & 1) * 64, desc_k(qa + (kk >> 2) * 16384 + (kk & 3) * 32),
+               desc_k(ka + (kk >> 2) * 8192 + (kk & 3) * 32), id_s, kk > 0 ? 1u : 0u);
+      tc_commit(bar_s);
+    };
+    // cp.async groups, oldest first: {Q, K0, V0}, {K1}, then per tile t
+    // {K(t+2)}, {V(t+1)}; waiting for all but the newest two before tile
+    // t's MMAs leaves exactly K(t+2), V(t+1) in flight.
     load_kv(0, OFF_K, pk);
     load_kv(0, OFF_V, pv);
     cp_async_commit();
+    if (n_kt > 1) load_kv(1, OFF_K + 16384, pk);
+    cp_async_commit();
+    cp_async_wait<1>();
+    fence_async_smem();
+    tc_before();
+    __syncthreads();
+    tc_after();
+    if (tid == 0) issue_s(0);
 
     float m_ref = -INFINITY, l_run = 0.f;
     const int qpos = ctx + q0 + tid;
 
     for (int kt = 0; kt < n_kt; ++kt) {
-      cp_async_wait<0>();          // K(kt), V(kt) (and Q) landed
-      fence_async_smem();
-      tc_before();
-      __syncthreads();
-      tc_after();
-      // ---- S = Q K^T
-      if (tid == 0) {
-        const uint32_t qa = sbase + OFF_Q, ka = sbase + OFF_K;
-#pragma unroll
-        for (int kk = 0; kk < HD / 16; ++kk)
-          tc_mma(t_s, desc_k(qa + (kk >> 2) * 16384 + (kk & 3) * 32),
-                 desc_k(ka + (kk >> 2) * 8192 + (kk & 3) * 32), id_s, kk > 0 ? 1u : 0u);
-        tc_commit(bar_s);
-      }
-      mbar_wait(bar_s, ph_s);
+      const uint32_t t_sb = t_s + (kt & 1) * 64;
+      mbar_wait(bar_s, ph_s);        // S(kt) in TMEM
       ph_s ^= 1;
       tc_after();
-      if (kt + 1 < n_kt) load_kv(kt + 1, OFF_K, pk);   // K buffer free: S(kt) done
+      if (kt + 2 < n_kt) load_kv(kt + 2, OFF_K + (kt & 1) * 16384, pk);   // K buffer of S(kt) is free
       cp_async_commit();
-      // ---- softmax of row tid over the 64 keys of this tile
-      float v[2][32];
-      tmem_ld32(t_s + lane_off, v[0]);
-      tmem_ld32(t_s + lane_off + 32, v[1]);
-      float mx = -INFINITY;
+      // ---- softmax of row tid over the 64 keys of this tile; P -> TMEM in
+      //      place of S(kt) (hi in columns [0,32), lo in [32,64) of the buffer)
+      float v[64];
+      tmem_ld32(t_sb + lane_off, v);
+      tmem_ld32(t_sb + lane_off + 32, v + 32);
+      // only tiles crossing the causal diagonal or the end of the sequence
+      // need the per-element mask (CTA-uniform test)
+      if ((kt + 1) * BKV - 1 > ctx + q0 || (kt + 1) * BKV > kv_len) {
 #pragma unroll
-      for (int c = 0; c < 2; ++c)
-#pragma unroll
-        for (int i = 0; i < 32; ++i) {
-          const int kp = kt * BKV + c * 32 + i;
-          v[c][i] = (kp <= qpos && kp < kv_len) ? v[c][i] * sl2 : -INFINITY;
-          mx = fmaxf(mx, v[c][i]);
+        for (int i = 0; i < 64; ++i) {
+          const int kp = kt * BKV + i;
+          if (!(kp <= qpos && kp < kv_len)) v[i] = -INFINITY;
         }
-      const bool move = mx > m_ref + 8.f;          // includes m_ref = -inf (first tile)
-      const float m_new = move ? mx : m_ref;
-      if (kt > 0 && __any_sync(0xffffffffu, move)) {   // warp-uniform rescale of O in TMEM
-        const float alpha = move ? exp2f(m_ref - m_new) : 1.f;
-        float w[32];
-#pragma unroll
-        for (int c = 0; c < 4; ++c) {
-          tmem_ld32(t_o + lane_off + c * 32, w);
-#pragma unroll
-          for (int i = 0; i < 32; ++i) w[i] *= alpha;
-          tmem_st32(t_o + lane_off + c * 32, w);
-        }
-        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
-        l_run *= alpha;
       }
+      float mx = v[0];
+#pragma unroll
+      for (int i = 1; i < 64; ++i) mx = fmaxf(mx, v[i]);
+      const float mx_s = mx * sl2;                  // scale > 0 commutes with max
+      const bool move = mx_s > m_ref + 8.f;         // includes m_ref = -inf (first tile)
+      const float m_new = move ? mx_s : m_ref;
+      const float alpha = move ? ex2(m_ref - m_new) : 1.f;
+      float ls;
+      {
+        uint32_t hi[32], lo[32];
+        float2 acc = make_float2(0.f, 0.f);
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          const float2 t = ffma2(make_float2(v[2 * j], v[2 * j + 1]), sl2, -m_new);
+          const float2 pp = make_float2(ex2(t.x), ex2(t.y));
+          acc = fadd2(acc, pp);
+          const uint32_t h = pack_bf2(pp.x, pp.y);
+          const float2 l = fsub2(pp, make_float2(__uint_as_float(h << 16), __uint_as_float(h & 0xFFFF0000u)));
+          hi[j] = h;
+          lo[j] = pack_bf2(l.x, l.y);
+        }
+        ls = acc.x + acc.y;
+        tmem_st32(t_sb + lane_off, reinterpret_cast<const float*>(hi));
+        tmem_st32(t_sb + lane_off + 32, reinterpret_cast<const float*>(lo));
+      }
+      if (kt > 0) {                  // PV(kt-1) done: O may be rescaled, its V / P buffers reused
+        mbar_wait(bar_o, ph_o);
+        ph_o ^= 1;
+        tc_after();
+        if (__any_sync(0xffffffffu, move)) {   // warp-uniform lazy rescale of O (> 2^8 growth)
+          float w[32];
+#pragma unroll
+          for (int c = 0; c < 4; ++c) {
+            tmem_ld32(t_o + lane_off + c * 32, w);
+#pragma unroll
+            for (int i = 0; i < 32; ++i) w[i] *= alpha;
+            tmem_st32(t_o + lane_off + c * 32, w);
+          }
+        }
+      }
+      l_run = l_run * alpha + ls;
       m_ref = m_new;
-      float ls = 0.f;
-#pragma unroll
-      for (int c = 0; c < 2; ++c) {
-        uint32_t hi[16], lo[16];
-#pragma unroll
-        for (int i = 0; i < 32; i += 2) {
-          const float p0 = exp2f(v[c][i] - m_new), p1 = exp2f(v[c][i + 1] - m_new);
-          ls += p0 + p1;
-          const __nv_bfloat162 hh = __floats2bfloat162_rn(p0, p1);
-          const float2 hf = __bfloat1622float2(hh);
-          hi[i >> 1] = *reinterpret_cast<const uint32_t*>(&hh);
-          lo[i >> 1] = pack_bf2(p0 - hf.x, p1 - hf.y);
-        }
-#pragma unroll
-        for (int q = 0; q < 4; ++q) {
-          const uint32_t off = sw(tid, c * 4 + q, 0);
-          *reinterpret_cast<uint4*>(sm + OFF_PH + off) = make_uint4(hi[4 * q], hi[4 * q + 1], hi[4 * q + 2], hi[4 * q + 3]);
-          *reinterpret_cast<uint4*>(sm + OFF_PL + off) = make_uint4(lo[4 * q], lo[4 * q + 1], lo[4 * q + 2], lo[4 * q + 3]);
-        }
-      }
-      l_run += ls;
+      if (kt + 1 < n_kt) load_kv(kt + 1, OFF_V + ((kt + 1) & 1) * 16384, pv);
+      cp_async_commit();
+      cp_async_wait<2>();            // K(kt+1), V(kt) landed
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
       fence_async_smem();
       tc_before();
       __syncthreads();
       tc_after();
-      // ---- O += P V   (P = hi + lo)
       if (tid == 0) {
-        const uint32_t va = sbase + OFF_V;
+        if (kt + 1 < n_kt) issue_s(kt + 1);   // overwrites P(kt-1): PV(kt-1) is done
+        // ---- O += P V   (A = P from TMEM, B = V(kt) MN-major from smem)
+        const uint32_t va = sbase + OFF_V + (kt & 1) * 16384;
 #pragma unroll
         for (int kk = 0; kk < BKV / 16; ++kk)
-          tc_mma(t_o, desc_k(sbase + OFF_PH + kk * 32), desc_mn(va + kk * 2048), id_o, (kt > 0 || kk > 0) ? 1u : 0u);
+          tc_mma_ts(t_o, t_sb + kk * 8, desc_mn(va + kk * 2048), id_o, (kt > 0 || kk > 0) ? 1u : 0u);
 #pragma unroll
         for (int kk = 0; kk < BKV / 16; ++kk)
-          tc_mma(t_o, desc_k(sbase + OFF_PL + kk * 32), desc_mn(va + kk * 2048), id_o, 1u);
+          tc_mma_ts(t_o, t_sb + 32 + kk * 8, desc_mn(va + kk * 2048), id_o, 1u);
         tc_commit(bar_o);
       }
-      mbar_wait(bar_o, ph_o);
-      ph_o ^= 1;
-      tc_after();
-      if (kt + 1 < n_kt) load_kv(kt + 1, OFF_V, pv);   // V buffer free: PV(kt) done
-      cp_async_commit();
     }
+    mbar_wait(bar_o, ph_o);          // last PV
+    ph_o ^= 1;
+    tc_after();
     // ---- normalise and store row tid (bf16, point R3)
     {
       const float inv = 1.f / l_run;
