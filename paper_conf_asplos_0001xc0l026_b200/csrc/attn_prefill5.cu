@@ -23,12 +23,15 @@
 namespace bl {
 
 namespace {
-constexpr int BQ = 128, BKV = 64, HD = 128, KB = 16, NT = 128;
+constexpr int BQ = 128, BKV = 64, HD = 128, KB = 16;
+// warps 0-3 softmax + epilogue, 4 K/Q loader + unit claimer, 5 V loader, 6 MMA issuer
+constexpr int NT = 224, W_LOAD = 4, W_VLOAD = 5, W_MMA = 6;
 // smem: Q [2][128][128 B] | K[2 buffers] [2][64][128 B] | V[2 buffers] [2][64][128 B]
 // = 96 KB + barriers: two CTAs per SM.  The dynamic window must start
 // 1024-byte aligned (128-byte swizzle atoms); checked at entry.
-constexpr int OFF_Q = 0, OFF_K = 32768, OFF_V = 65536;
-constexpr int SMEM_BYTES = 98304 + 64;
+constexpr int NKB = 3;   // K buffers (K(g) may load once S(g-3) is done); V has 2
+constexpr int OFF_Q = 0, OFF_K = 32768, OFF_V = OFF_K + NKB * 16384, OFF_BAR = OFF_V + 2 * 16384;
+constexpr int SMEM_BYTES = OFF_BAR + 256;   // 20 mbarriers, TMEM slot, unit ring
 // TMEM: S/P double buffer in columns [0,64) and [64,128) (P = bf16 hi|lo
 // packed two per column, written over the S it came from), O in [128,256)
 constexpr uint32_t TMEM_COLS = 256;
@@ -94,6 +97,13 @@ __device__ __forceinline__ void tmem_st32(uint32_t taddr, const float* v) {
       "f"(v[30]), "f"(v[31])
       : "memory");
 }
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t* v) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]),
+      "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
+      : "memory");
+}
 __device__ __forceinline__ void cp_async16_zfill(void* dst, const void* src, bool valid) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src),
                "r"(valid ? 16 : 0)
@@ -129,6 +139,48 @@ __device__ __forceinline__ uint32_t pack_bf2(float a, float b) {
   __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
   return *reinterpret_cast<uint32_t*>(&h);
 }
+
+struct Unit {
+  int h, g, q0, tok0, q_len, ctx, kv_len, n_kt, r;
+};
+__device__ __forceinline__ Unit unit_of(const AttnArgs& a, int u) {
+  Unit U;
+  const int2 rt = a.tiles[u / a.H];
+  U.h = u % a.H;
+  U.g = U.h / (a.H / a.Hkv);
+  U.r = rt.x;
+  U.q0 = rt.y * BQ;
+  U.tok0 = __ldg(a.cu + U.r);
+  U.q_len = __ldg(a.cu + U.r + 1) - U.tok0;
+  U.ctx = __ldg(a.ctx + U.r);
+  U.kv_len = U.ctx + U.q_len;
+  U.n_kt = (min(U.kv_len, U.ctx + U.q0 + BQ) + BKV - 1) / BKV;
+  return U;
+}
+__device__ __forceinline__ void cp_async_arrive_noinc(uint64_t* bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+// One warp gathers KV tile kt (64 rows of head U.g through the block table)
+// into a 128-byte-swizzled [2][64][128 B] tile; `bar` completes when it lands.
+__device__ __forceinline__ void load_kv_tile(uint8_t* dst, const __nv_bfloat16* pool, const AttnArgs& a,
+                                             const Unit& U, int kt, int lane, uint64_t* bar) {
+  const int r0 = lane >> 4, c = lane & 15;   // this lane: rows r0 + 2j, 16-byte chunk c
+  const int32_t* bt = a.bt + (size_t)U.r * a.max_blocks;
+  const int kb = kt * BKV;
+  const bool full = kb + BKV <= U.kv_len;
+#pragma unroll
+  for (int b = 0; b < BKV / KB; ++b) {
+    const int blk = kb + b * KB < U.kv_len ? __ldg(bt + kt * (BKV / KB) + b) : 0;
+    const __nv_bfloat16* src = pool + (((size_t)blk * a.Hkv + U.g) * KB + r0) * HD + c * 8;
+#pragma unroll
+    for (int j = 0; j < KB / 2; ++j) {
+      const int row = b * KB + r0 + 2 * j;
+      const bool ok = full || kb + row < U.kv_len;
+      cp_async16_zfill(dst + sw(row, c, 8192), ok ? src + j * 2 * HD : pool, ok);
+    }
+  }
+  cp_async_arrive_noinc(bar);
+}
 }  // namespace
 
 __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
@@ -136,14 +188,33 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = smem_raw;
   if (smem_u32(sm) & 1023) __trap();   // swizzle atoms need 1024-byte alignment
-  uint64_t* bar_s = reinterpret_cast<uint64_t*>(sm + 98304);
-  uint64_t* bar_o = bar_s + 1;
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(bar_o + 1);
-  int* s_u = reinterpret_cast<int*>(tslot + 1);
-  const int tid = threadIdx.x, warp = tid >> 5;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + OFF_BAR);
+  uint64_t *vfull = bars, *sfull = bars + 2, *pfull = bars + 4, *pvdone = bars + 6;
+  uint64_t *qfull = bars + 8, *qempty = bars + 9, *oempty = bars + 10, *ufull = bars + 11, *uempty = bars + 13;
+  uint64_t *kfull = bars + 15, *kempty = bars + 18;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 21);
+  volatile int* ring = reinterpret_cast<volatile int*>(tslot + 1);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const uint32_t sbase = smem_u32(sm);
-  if (tid == 0) { mbar_init(bar_s, 1); mbar_init(bar_o, 1); mbar_fence_init(); }
-  if (warp == 0) {
+  if (tid == 0) {
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(vfull + i, 32);   // one cp.async-completion arrive per loader lane
+      mbar_init(sfull + i, 1);    // tcgen05.commit
+      mbar_init(pfull + i, 4);    // one arrive per softmax warp
+      mbar_init(pvdone + i, 1);
+      mbar_init(ufull + i, 1);
+      mbar_init(uempty + i, 6);   // MMA thread, V loader, 4 softmax warps
+    }
+    for (int i = 0; i < NKB; ++i) {
+      mbar_init(kfull + i, 32);
+      mbar_init(kempty + i, 1);
+    }
+    mbar_init(qfull, 32);
+    mbar_init(qempty, 1);
+    mbar_init(oempty, 4);
+    mbar_fence_init();
+  }
+  if (warp == W_MMA) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tslot)), "r"(TMEM_COLS));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
@@ -152,176 +223,211 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
   tc_after();
   const uint32_t tmem = *tslot;
   const uint32_t t_s = tmem, t_o = tmem + 128;
-  const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
-  // f32 accumulate, bf16 A/B; S: N = 64, B K-major; O: N = 128, B MN-major
-  const uint32_t id_s = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(BKV >> 3) << 17) | ((uint32_t)(BQ >> 4) << 24);
-  const uint32_t id_o = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(HD >> 3) << 17) |
-                        ((uint32_t)(BQ >> 4) << 24);
-  const int grp = a.H / a.Hkv;
-  const __nv_bfloat16* qg = reinterpret_cast<const __nv_bfloat16*>(a.q);
   const __nv_bfloat16* pk = reinterpret_cast<const __nv_bfloat16*>(a.pool_k);
   const __nv_bfloat16* pv = reinterpret_cast<const __nv_bfloat16*>(a.pool_v);
-  __nv_bfloat16* og = reinterpret_cast<__nv_bfloat16*>(a.o);
-  const float sl2 = a.scale * 1.4426950408889634f;
   const int units = (*a.n_tiles) * a.H;
-  uint32_t ph_s = 0, ph_o = 0;
 
-  for (;;) {
-    if (tid == 0) *s_u = atomicAdd(a.L.ctr, 1);
-    __syncthreads();
-    const int u = *s_u;
-    __syncthreads();
-    if (u >= units) break;
-    if (tid == 0) log_unit(a.L, u);
-    const int2 rt = a.tiles[u / a.H];
-    const int h = u % a.H, g = h / grp, r = rt.x, q0 = rt.y * BQ;
-    const int tok0 = __ldg(a.cu + r);
-    const int q_len = __ldg(a.cu + r + 1) - tok0;
-    const int ctx = __ldg(a.ctx + r);
-    const int kv_len = ctx + q_len;
-    const int kmax = min(kv_len, ctx + q0 + BQ);
-    const int n_kt = (kmax + BKV - 1) / BKV;
-    const int32_t* bt = a.bt + (size_t)r * a.max_blocks;
-
-    // coalesced gathers: 16 lanes per 256-byte row
-    {
-#pragma unroll
-      for (int i = 0; i < 16; ++i) {   // Q: 128 rows x 16 chunks
-        const int e = tid + NT * i, row = e >> 4, c = e & 15;
-        const bool ok = q0 + row < q_len;
-        cp_async16_zfill(sm + OFF_Q + sw(row, c, 16384),
-                         qg + (size_t)(tok0 + (ok ? q0 + row : 0)) * a.H * HD + h * HD + c * 8, ok);
+  if (warp == W_LOAD) {
+    // ---------------- K/Q loader: claims units, gathers Q and K(g) as soon as
+    // S(g-3) has released K buffer g % 3
+    const __nv_bfloat16* qg = reinterpret_cast<const __nv_bfloat16*>(a.q);
+    const int r0 = lane >> 4, c = lane & 15;   // this lane: rows r0 + 2j, 16-byte chunk c
+    uint32_t g = 0;
+    for (int n = 0;; ++n) {
+      int u = 0;
+      if (lane == 0) u = atomicAdd(a.L.ctr, 1);
+      u = __shfl_sync(0xffffffffu, u, 0);
+      const int slot = n & 1;
+      if (n >= 2) mbar_wait(uempty + slot, ((n - 2) >> 1) & 1);
+      if (lane == 0) {
+        ring[slot] = u < units ? u : -1;
+        mbar_arrive(ufull + slot);
+      }
+      if (u >= units) break;
+      if (lane == 0) log_unit(a.L, u);
+      const Unit U = unit_of(a, u);
+      for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
+        const int kb = g % NKB;
+        if (g >= NKB) mbar_wait(kempty + kb, (g / NKB - 1) & 1);
+        load_kv_tile(sm + OFF_K + kb * 16384, pk, a, U, kt, lane, kfull + kb);
+        if (kt == 0) {
+          if (n >= 1) mbar_wait(qempty, (n - 1) & 1);         // last S of the previous unit done
+#pragma unroll 8
+          for (int j = 0; j < BQ / 2; ++j) {
+            const int row = r0 + 2 * j;
+            const bool ok = U.q0 + row < U.q_len;
+            cp_async16_zfill(sm + OFF_Q + sw(row, c, 16384),
+                             qg + (size_t)(U.tok0 + (ok ? U.q0 + row : 0)) * a.H * HD + U.h * HD + c * 8, ok);
+          }
+          cp_async_arrive_noinc(qfull);
+        }
       }
     }
-    auto load_kv = [&](int kt, int off, const __nv_bfloat16* pool) {
-#pragma unroll
-      for (int i = 0; i < 8; ++i) {    // 64 rows x 16 chunks
-        const int e = tid + NT * i, row = e >> 4, c = e & 15;
-        const int kp = kt * BKV + row;
-        const bool ok = kp < kv_len;
-        const int blk = ok ? __ldg(bt + kp / KB) : 0;
-        cp_async16_zfill(sm + off + sw(row, c, 8192),
-                         pool + (((size_t)blk * a.Hkv + g) * KB + (ok ? kp % KB : 0)) * HD + c * 8, ok);
+  } else if (warp == W_VLOAD) {
+    // ---------------- V loader: V(g) as soon as PV(g-2) has released buffer g & 1
+    uint32_t g = 0;
+    for (int n = 0;; ++n) {
+      const int slot = n & 1;
+      mbar_wait(ufull + slot, (n >> 1) & 1);
+      const int u = ring[slot];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(uempty + slot);
+      if (u < 0) break;
+      const Unit U = unit_of(a, u);
+      for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
+        const int b = g & 1;
+        if (g >= 2) mbar_wait(pvdone + b, ((g - 2) >> 1) & 1);
+        load_kv_tile(sm + OFF_V + b * 16384, pv, a, U, kt, lane, vfull + b);
       }
-    };
-    auto issue_s = [&](int kt) {       // S(kt) = Q K(kt)^T -> TMEM buffer kt&1
-      const uint32_t qa = sbase + OFF_Q, ka = sbase + OFF_K + (kt & 1) * 16384;
-#pragma unroll
-      for (int kk = 0; kk < HD / 16; ++kk)
-        tc_mma(t_s + (kt & 1) * 64, desc_k(qa + (kk >> 2) * 16384 + (kk & 3) * 32),
-               desc_k(ka + (kk >> 2) * 8192 + (kk & 3) * 32), id_s, kk > 0 ? 1u : 0u);
-      tc_commit(bar_s);
-    };
-    // cp.async groups, oldest first: {Q, K0, V0}, {K1}, then per tile t
-    // {K(t+2)}, {V(t+1)}; waiting for all but the newest two before tile
-    // t's MMAs leaves exactly K(t+2), V(t+1) in flight.
-    load_kv(0, OFF_K, pk);
-    load_kv(0, OFF_V, pv);
-    cp_async_commit();
-    if (n_kt > 1) load_kv(1, OFF_K + 16384, pk);
-    cp_async_commit();
-    cp_async_wait<1>();
-    fence_async_smem();
-    tc_before();
-    __syncthreads();
-    tc_after();
-    if (tid == 0) issue_s(0);
-
-    float m_ref = -INFINITY, l_run = 0.f;
-    const int qpos = ctx + q0 + tid;
-
-    for (int kt = 0; kt < n_kt; ++kt) {
-      const uint32_t t_sb = t_s + (kt & 1) * 64;
-      mbar_wait(bar_s, ph_s);        // S(kt) in TMEM
-      ph_s ^= 1;
-      tc_after();
-      if (kt + 2 < n_kt) load_kv(kt + 2, OFF_K + (kt & 1) * 16384, pk);   // K buffer of S(kt) is free
-      cp_async_commit();
-      // ---- softmax of row tid over the 64 keys of this tile; P -> TMEM in
-      //      place of S(kt) (hi in columns [0,32), lo in [32,64) of the buffer)
-      float v[64];
-      tmem_ld32(t_sb + lane_off, v);
-      tmem_ld32(t_sb + lane_off + 32, v + 32);
-      // only tiles crossing the causal diagonal or the end of the sequence
-      // need the per-element mask (CTA-uniform test)
-      if ((kt + 1) * BKV - 1 > ctx + q0 || (kt + 1) * BKV > kv_len) {
-#pragma unroll
-        for (int i = 0; i < 64; ++i) {
-          const int kp = kt * BKV + i;
-          if (!(kp <= qpos && kp < kv_len)) v[i] = -INFINITY;
-        }
-      }
-      float mx = v[0];
-#pragma unroll
-      for (int i = 1; i < 64; ++i) mx = fmaxf(mx, v[i]);
-      const float mx_s = mx * sl2;                  // scale > 0 commutes with max
-      const bool move = mx_s > m_ref + 8.f;         // includes m_ref = -inf (first tile)
-      const float m_new = move ? mx_s : m_ref;
-      const float alpha = move ? ex2(m_ref - m_new) : 1.f;
-      float ls;
-      {
-        uint32_t hi[32], lo[32];
-        float2 acc = make_float2(0.f, 0.f);
-#pragma unroll
-        for (int j = 0; j < 32; ++j) {
-          const float2 t = ffma2(make_float2(v[2 * j], v[2 * j + 1]), sl2, -m_new);
-          const float2 pp = make_float2(ex2(t.x), ex2(t.y));
-          acc = fadd2(acc, pp);
-          const uint32_t h = pack_bf2(pp.x, pp.y);
-          const float2 l = fsub2(pp, make_float2(__uint_as_float(h << 16), __uint_as_float(h & 0xFFFF0000u)));
-          hi[j] = h;
-          lo[j] = pack_bf2(l.x, l.y);
-        }
-        ls = acc.x + acc.y;
-        tmem_st32(t_sb + lane_off, reinterpret_cast<const float*>(hi));
-        tmem_st32(t_sb + lane_off + 32, reinterpret_cast<const float*>(lo));
-      }
-      if (kt > 0) {                  // PV(kt-1) done: O may be rescaled, its V / P buffers reused
-        mbar_wait(bar_o, ph_o);
-        ph_o ^= 1;
+    }
+  } else if (warp == W_MMA) {
+    // ---------------- MMA issuer (one thread): S(g) then PV(g-1)
+    if (lane == 0) {
+      // f32 accumulate, bf16 A/B; S: N = 64, B K-major; O: N = 128, B MN-major
+      const uint32_t id_s = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(BKV >> 3) << 17) | ((uint32_t)(BQ >> 4) << 24);
+      const uint32_t id_o = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(HD >> 3) << 17) |
+                            ((uint32_t)(BQ >> 4) << 24);
+      uint32_t g = 0;
+      auto issue_pv = [&](uint32_t gp, bool first, int n) {
+        const int b = gp & 1;
+        mbar_wait(pfull + b, (gp >> 1) & 1);
+        mbar_wait(vfull + b, (gp >> 1) & 1);
+        if (first && n >= 1) mbar_wait(oempty, (n - 1) & 1);   // previous unit's O read out
         tc_after();
-        if (__any_sync(0xffffffffu, move)) {   // warp-uniform lazy rescale of O (> 2^8 growth)
-          float w[32];
+        fence_async_smem();
+        const uint32_t va = sbase + OFF_V + b * 16384, pa = t_s + b * 64;
+        // A = P from TMEM: keys 16kk..16kk+15 hi at column 32(kk/2) + 8(kk%2), lo 16 further
 #pragma unroll
+        for (int kk = 0; kk < BKV / 16; ++kk)
+          tc_mma_ts(t_o, pa + (kk >> 1) * 32 + (kk & 1) * 8, desc_mn(va + kk * 2048), id_o, (!first || kk > 0) ? 1u : 0u);
+#pragma unroll
+        for (int kk = 0; kk < BKV / 16; ++kk)
+          tc_mma_ts(t_o, pa + (kk >> 1) * 32 + 16 + (kk & 1) * 8, desc_mn(va + kk * 2048), id_o, 1u);
+        tc_commit(pvdone + b);
+      };
+      for (int n = 0;; ++n) {
+        const int slot = n & 1;
+        mbar_wait(ufull + slot, (n >> 1) & 1);
+        const int u = ring[slot];
+        mbar_arrive(uempty + slot);
+        if (u < 0) break;
+        const Unit U = unit_of(a, u);
+        mbar_wait(qfull, n & 1);
+        for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
+          const int b = g & 1, kb = g % NKB;
+          mbar_wait(kfull + kb, (g / NKB) & 1);
+          if (g >= 2) mbar_wait(pvdone + b, ((g - 2) >> 1) & 1);   // P(g-2) consumed: S buffer b free
+          tc_after();
+          fence_async_smem();
+          const uint32_t qa = sbase + OFF_Q, ka = sbase + OFF_K + kb * 16384;
+#pragma unroll
+          for (int kk = 0; kk < HD / 16; ++kk)
+            tc_mma(t_s + b * 64, desc_k(qa + (kk >> 2) * 16384 + (kk & 3) * 32),
+                   desc_k(ka + (kk >> 2) * 8192 + (kk & 3) * 32), id_s, kk > 0 ? 1u : 0u);
+          tc_commit(sfull + b);
+          tc_commit(kempty + kb);
+          if (kt == U.n_kt - 1) tc_commit(qempty);
+          if (kt > 0) issue_pv(g - 1, kt == 1, n);
+        }
+        issue_pv(g - 1, U.n_kt == 1, n);
+      }
+    }
+  } else {
+    // ---------------- softmax + epilogue: thread tid owns query row tid (TMEM lane tid)
+    __nv_bfloat16* og = reinterpret_cast<__nv_bfloat16*>(a.o);
+    const float sl2 = a.scale * 1.4426950408889634f;
+    const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
+    uint32_t g = 0;
+    for (int n = 0;; ++n) {
+      const int slot = n & 1;
+      mbar_wait(ufull + slot, (n >> 1) & 1);
+      const int u = ring[slot];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(uempty + slot);
+      if (u < 0) break;
+      const Unit U = unit_of(a, u);
+      const int qpos = U.ctx + U.q0 + tid;
+      float m_ref = -INFINITY, l_run = 0.f;
+      for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
+        const int b = g & 1;
+        const uint32_t t_sb = t_s + b * 64 + lane_off;
+        mbar_wait(sfull + b, (g >> 1) & 1);
+        tc_after();
+        // two passes over S in TMEM (32 columns at a time) keep ~32 scores live:
+        // pass 1 row max, pass 2 P.  Only tiles crossing the causal diagonal or
+        // the end of the sequence need the per-element mask (warp-uniform test).
+        const bool edge = (kt + 1) * BKV - 1 > U.ctx + U.q0 || (kt + 1) * BKV > U.kv_len;
+        const int lim = min(qpos + 1, U.kv_len) - kt * BKV;   // keys [0, lim) of this tile are visible
+        float mx = -INFINITY;
+#pragma unroll
+        for (int half = 0; half < 2; ++half) {
+          float v[32];
+          tmem_ld32(t_sb + half * 32, v);
+          if (edge) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i)
+              if (half * 32 + i >= lim) v[i] = -INFINITY;
+          }
+#pragma unroll
+          for (int i = 0; i < 32; ++i) mx = fmaxf(mx, v[i]);
+        }
+        const float mx_s = mx * sl2;                  // scale > 0 commutes with max
+        const bool move = mx_s > m_ref + 8.f;         // includes m_ref = -inf (first tile)
+        const float m_new = move ? mx_s : m_ref;
+        const float alpha = move ? ex2(m_ref - m_new) : 1.f;
+        if (kt > 0 && __any_sync(0xffffffffu, move)) {   // lazy rescale of O: PV(g-1) must be done
+          mbar_wait(pvdone + ((g - 1) & 1), ((g - 1) >> 1) & 1);
+          tc_after();
+#pragma unroll 1
           for (int c = 0; c < 4; ++c) {
+            float w[32];
             tmem_ld32(t_o + lane_off + c * 32, w);
 #pragma unroll
             for (int i = 0; i < 32; ++i) w[i] *= alpha;
             tmem_st32(t_o + lane_off + c * 32, w);
           }
         }
+        // P = 2^(s*scale*log2e - m) as bf16 hi + lo, written over S(g): keys
+        // 32h..32h+31 go to columns [32h, 32h+16) (hi) and [32h+16, 32h+32) (lo),
+        // exactly the columns their scores came from, so half 1's scores are
+        // still intact when half 0's P is stored.
+        float2 acc = make_float2(0.f, 0.f);
+#pragma unroll
+        for (int half = 0; half < 2; ++half) {
+          float v[32];
+          tmem_ld32(t_sb + half * 32, v);
+          if (edge) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i)
+              if (half * 32 + i >= lim) v[i] = -INFINITY;
+          }
+          uint32_t hi[16], lo[16];
+#pragma unroll
+          for (int j = 0; j < 16; ++j) {
+            const float2 t = ffma2(make_float2(v[2 * j], v[2 * j + 1]), sl2, -m_new);
+            const float2 pp = make_float2(ex2(t.x), ex2(t.y));
+            acc = fadd2(acc, pp);
+            const uint32_t h = pack_bf2(pp.x, pp.y);
+            const float2 l = fsub2(pp, make_float2(__uint_as_float(h << 16), __uint_as_float(h & 0xFFFF0000u)));
+            hi[j] = h;
+            lo[j] = pack_bf2(l.x, l.y);
+          }
+          tmem_st16(t_sb + half * 32, hi);
+          tmem_st16(t_sb + half * 32 + 16, lo);
+        }
+        l_run = l_run * alpha + (acc.x + acc.y);
+        m_ref = m_new;
+        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        tc_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(pfull + b);
       }
-      l_run = l_run * alpha + ls;
-      m_ref = m_new;
-      if (kt + 1 < n_kt) load_kv(kt + 1, OFF_V + ((kt + 1) & 1) * 16384, pv);
-      cp_async_commit();
-      cp_async_wait<2>();            // K(kt+1), V(kt) landed
-      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
-      fence_async_smem();
-      tc_before();
-      __syncthreads();
+      // ---- normalise and store row tid (bf16, point R3) once the last PV is done
+      mbar_wait(pvdone + ((g - 1) & 1), ((g - 1) >> 1) & 1);
       tc_after();
-      if (tid == 0) {
-        if (kt + 1 < n_kt) issue_s(kt + 1);   // overwrites P(kt-1): PV(kt-1) is done
-        // ---- O += P V   (A = P from TMEM, B = V(kt) MN-major from smem)
-        const uint32_t va = sbase + OFF_V + (kt & 1) * 16384;
-#pragma unroll
-        for (int kk = 0; kk < BKV / 16; ++kk)
-          tc_mma_ts(t_o, t_sb + kk * 8, desc_mn(va + kk * 2048), id_o, (kt > 0 || kk > 0) ? 1u : 0u);
-#pragma unroll
-        for (int kk = 0; kk < BKV / 16; ++kk)
-          tc_mma_ts(t_o, t_sb + 32 + kk * 8, desc_mn(va + kk * 2048), id_o, 1u);
-        tc_commit(bar_o);
-      }
-    }
-    mbar_wait(bar_o, ph_o);          // last PV
-    ph_o ^= 1;
-    tc_after();
-    // ---- normalise and store row tid (bf16, point R3)
-    {
       const float inv = 1.f / l_run;
-      const bool ok = q0 + tid < q_len;
-      __nv_bfloat16* dst = og + (size_t)(tok0 + q0 + (ok ? tid : 0)) * a.H * HD + h * HD;
+      const bool ok = U.q0 + tid < U.q_len;
+      __nv_bfloat16* dst = og + (size_t)(U.tok0 + U.q0 + (ok ? tid : 0)) * a.H * HD + U.h * HD;
 #pragma unroll
       for (int c = 0; c < 4; ++c) {
         float w[32];
@@ -334,12 +440,14 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
                            pack_bf2(w[8 * q + 4] * inv, w[8 * q + 5] * inv), pack_bf2(w[8 * q + 6] * inv, w[8 * q + 7] * inv));
         }
       }
+      tc_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(oempty);
     }
-    tc_before();
-    __syncthreads();
-    tc_after();
   }
-  if (warp == 0) {
+  tc_before();
+  __syncthreads();
+  if (warp == W_MMA) {
     tc_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS));
   }
