@@ -160,17 +160,43 @@ __device__ __forceinline__ Unit unit_of(const AttnArgs& a, int u) {
 __device__ __forceinline__ void cp_async_arrive_noinc(uint64_t* bar) {
   asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
+// Suspending wait (the warp sleeps until the phase completes instead of
+// spinning and taking issue slots from the softmax warps).
+__device__ __forceinline__ void wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, 0x989680;\n\t"
+      "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+// Block-table window of a loader warp: lane l holds entry 32w + l of the
+// unit's block-table row for the current window w (8 KV tiles) and prefetches
+// the next window, so no tile waits on a block-table load.
+struct BtWin {
+  int cur, nxt;
+  __device__ __forceinline__ void start(const int32_t* bt, int n_blk, int lane) {
+    cur = lane < n_blk ? __ldg(bt + lane) : 0;
+    nxt = 32 + lane < n_blk ? __ldg(bt + 32 + lane) : 0;
+  }
+  // call at tile kt (kt % 8 == 0, kt > 0): window kt / 8 becomes current
+  __device__ __forceinline__ void advance(const int32_t* bt, int n_blk, int kt, int lane) {
+    cur = nxt;
+    const int e = (kt / 8 + 1) * 32 + lane;
+    nxt = e < n_blk ? __ldg(bt + e) : 0;
+  }
+};
 // One warp gathers KV tile kt (64 rows of head U.g through the block table)
 // into a 128-byte-swizzled [2][64][128 B] tile; `bar` completes when it lands.
 __device__ __forceinline__ void load_kv_tile(uint8_t* dst, const __nv_bfloat16* pool, const AttnArgs& a,
-                                             const Unit& U, int kt, int lane, uint64_t* bar) {
+                                             const Unit& U, int kt, int lane, uint64_t* bar, const BtWin& w) {
   const int r0 = lane >> 4, c = lane & 15;   // this lane: rows r0 + 2j, 16-byte chunk c
-  const int32_t* bt = a.bt + (size_t)U.r * a.max_blocks;
   const int kb = kt * BKV;
   const bool full = kb + BKV <= U.kv_len;
 #pragma unroll
   for (int b = 0; b < BKV / KB; ++b) {
-    const int blk = kb + b * KB < U.kv_len ? __ldg(bt + kt * (BKV / KB) + b) : 0;
+    const int blk = __shfl_sync(0xffffffffu, w.cur, (kt % 8) * (BKV / KB) + b);
     const __nv_bfloat16* src = pool + (((size_t)blk * a.Hkv + U.g) * KB + r0) * HD + c * 8;
 #pragma unroll
     for (int j = 0; j < KB / 2; ++j) {
@@ -238,7 +264,7 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
       if (lane == 0) u = atomicAdd(a.L.ctr, 1);
       u = __shfl_sync(0xffffffffu, u, 0);
       const int slot = n & 1;
-      if (n >= 2) mbar_wait(uempty + slot, ((n - 2) >> 1) & 1);
+      if (n >= 2) wait(uempty + slot, ((n - 2) >> 1) & 1);
       if (lane == 0) {
         ring[slot] = u < units ? u : -1;
         mbar_arrive(ufull + slot);
@@ -246,12 +272,17 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
       if (u >= units) break;
       if (lane == 0) log_unit(a.L, u);
       const Unit U = unit_of(a, u);
+      const int32_t* bt = a.bt + (size_t)U.r * a.max_blocks;
+      const int n_blk = (U.kv_len + KB - 1) / KB;   // blocks this sequence owns
+      BtWin w;
+      w.start(bt, n_blk, lane);
       for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
         const int kb = g % NKB;
-        if (g >= NKB) mbar_wait(kempty + kb, (g / NKB - 1) & 1);
-        load_kv_tile(sm + OFF_K + kb * 16384, pk, a, U, kt, lane, kfull + kb);
+        if (kt > 0 && kt % 8 == 0) w.advance(bt, n_blk, kt, lane);
+        if (g >= NKB) wait(kempty + kb, (g / NKB - 1) & 1);
+        load_kv_tile(sm + OFF_K + kb * 16384, pk, a, U, kt, lane, kfull + kb, w);
         if (kt == 0) {
-          if (n >= 1) mbar_wait(qempty, (n - 1) & 1);         // last S of the previous unit done
+          if (n >= 1) wait(qempty, (n - 1) & 1);         // last S of the previous unit done
 #pragma unroll 8
           for (int j = 0; j < BQ / 2; ++j) {
             const int row = r0 + 2 * j;
@@ -268,16 +299,21 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
     uint32_t g = 0;
     for (int n = 0;; ++n) {
       const int slot = n & 1;
-      mbar_wait(ufull + slot, (n >> 1) & 1);
+      wait(ufull + slot, (n >> 1) & 1);
       const int u = ring[slot];
       __syncwarp();
       if (lane == 0) mbar_arrive(uempty + slot);
       if (u < 0) break;
       const Unit U = unit_of(a, u);
+      const int32_t* bt = a.bt + (size_t)U.r * a.max_blocks;
+      const int n_blk = (U.kv_len + KB - 1) / KB;   // blocks this sequence owns
+      BtWin w;
+      w.start(bt, n_blk, lane);
       for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
         const int b = g & 1;
-        if (g >= 2) mbar_wait(pvdone + b, ((g - 2) >> 1) & 1);
-        load_kv_tile(sm + OFF_V + b * 16384, pv, a, U, kt, lane, vfull + b);
+        if (kt > 0 && kt % 8 == 0) w.advance(bt, n_blk, kt, lane);
+        if (g >= 2) wait(pvdone + b, ((g - 2) >> 1) & 1);
+        load_kv_tile(sm + OFF_V + b * 16384, pv, a, U, kt, lane, vfull + b, w);
       }
     }
   } else if (warp == W_MMA) {
@@ -290,9 +326,9 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
       uint32_t g = 0;
       auto issue_pv = [&](uint32_t gp, bool first, int n) {
         const int b = gp & 1;
-        mbar_wait(pfull + b, (gp >> 1) & 1);
-        mbar_wait(vfull + b, (gp >> 1) & 1);
-        if (first && n >= 1) mbar_wait(oempty, (n - 1) & 1);   // previous unit's O read out
+        wait(pfull + b, (gp >> 1) & 1);
+        wait(vfull + b, (gp >> 1) & 1);
+        if (first && n >= 1) wait(oempty, (n - 1) & 1);   // previous unit's O read out
         tc_after();
         fence_async_smem();
         const uint32_t va = sbase + OFF_V + b * 16384, pa = t_s + b * 64;
@@ -307,16 +343,16 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
       };
       for (int n = 0;; ++n) {
         const int slot = n & 1;
-        mbar_wait(ufull + slot, (n >> 1) & 1);
+        wait(ufull + slot, (n >> 1) & 1);
         const int u = ring[slot];
         mbar_arrive(uempty + slot);
         if (u < 0) break;
         const Unit U = unit_of(a, u);
-        mbar_wait(qfull, n & 1);
+        wait(qfull, n & 1);
         for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
           const int b = g & 1, kb = g % NKB;
-          mbar_wait(kfull + kb, (g / NKB) & 1);
-          if (g >= 2) mbar_wait(pvdone + b, ((g - 2) >> 1) & 1);   // P(g-2) consumed: S buffer b free
+          wait(kfull + kb, (g / NKB) & 1);
+          if (g >= 2) wait(pvdone + b, ((g - 2) >> 1) & 1);   // P(g-2) consumed: S buffer b free
           tc_after();
           fence_async_smem();
           const uint32_t qa = sbase + OFF_Q, ka = sbase + OFF_K + kb * 16384;
@@ -340,7 +376,7 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
     uint32_t g = 0;
     for (int n = 0;; ++n) {
       const int slot = n & 1;
-      mbar_wait(ufull + slot, (n >> 1) & 1);
+      wait(ufull + slot, (n >> 1) & 1);
       const int u = ring[slot];
       __syncwarp();
       if (lane == 0) mbar_arrive(uempty + slot);
@@ -351,7 +387,7 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
       for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
         const int b = g & 1;
         const uint32_t t_sb = t_s + b * 64 + lane_off;
-        mbar_wait(sfull + b, (g >> 1) & 1);
+        wait(sfull + b, (g >> 1) & 1);
         tc_after();
         // two passes over S in TMEM (32 columns at a time) keep ~32 scores live:
         // pass 1 row max, pass 2 P.  Only tiles crossing the causal diagonal or
@@ -376,7 +412,7 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
         const float m_new = move ? mx_s : m_ref;
         const float alpha = move ? ex2(m_ref - m_new) : 1.f;
         if (kt > 0 && __any_sync(0xffffffffu, move)) {   // lazy rescale of O: PV(g-1) must be done
-          mbar_wait(pvdone + ((g - 1) & 1), ((g - 1) >> 1) & 1);
+          wait(pvdone + ((g - 1) & 1), ((g - 1) >> 1) & 1);
           tc_after();
 #pragma unroll 1
           for (int c = 0; c < 4; ++c) {
@@ -423,7 +459,7 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
         if (lane == 0) mbar_arrive(pfull + b);
       }
       // ---- normalise and store row tid (bf16, point R3) once the last PV is done
-      mbar_wait(pvdone + ((g - 1) & 1), ((g - 1) >> 1) & 1);
+      wait(pvdone + ((g - 1) & 1), ((g - 1) >> 1) & 1);
       tc_after();
       const float inv = 1.f / l_run;
       const bool ok = U.q0 + tid < U.q_len;
