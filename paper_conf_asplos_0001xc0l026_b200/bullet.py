@@ -81,7 +81,7 @@ def lib():
     """Load (building first if missing or stale) the in-tree libbullet.so."""
     global _lib
     if _lib is None:
-        path = _build.build() if _build.stale() else _build.OUT
+        path = os.environ.get("BULLET_LIB") or (_build.build() if _build.stale() else _build.OUT)   # override: A/B experiments
         L = ctypes.CDLL(path, mode=ctypes.RTLD_GLOBAL)
         L.bullet_last_error.restype = ctypes.c_char_p
         for name in ("bullet_create", "bullet_perf_create", "bullet_set_layer_weights", "bullet_num_sms", "bullet_sm_order",

@@ -230,43 +230,75 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   if (rc) return rc;
   if (h->cfg.dtype == BULLET_DTYPE_FP32) {
     if (K % 16) return set_err(BULLET_EUNSUPPORTED, "fp32 GEMM needs K %% 16 == 0");
-    a.bn = 64; a.splits = 1;
+    a.bn = 64; a.mh = 1; a.splits = 1; a.n_full = 0;
     LAUNCH(c, launch_gemm_simt<float>((const float*)A, (const float*)B, a, h->n_sms * 4, c.st));
     return BULLET_OK;
   }
   if (K % 64) return set_err(BULLET_EUNSUPPORTED, "GEMM needs K %% 64 == 0 (K=%d)", K);
-  const int m_tiles = (M + 127) / 128;
   // packed B needs 64-row aligned halves: SiLU tiles of >= 128 rows
   auto fits = [&](int bn) {
     if (Bp && epi == EPI_SILU && bn < 128) return false;
     return epi == EPI_SILU ? ((N / 2) % (bn / 2) == 0 && N % 2 == 0) : (N % bn == 0);
   };
-  // Plan (bn, split-K) on the phase's m SMs: minimise waves x bytes per unit
-  // (A + B tile streams), plus the split-K partial round trip; ties prefer
-  // wider tiles (MMA efficiency).  Work units run one per CTA per wave.
+  // Plan (mh, bn, tail split) on the phase's m SMs.  A tile costs
+  // max(bytes streamed / per-SM copy bandwidth, MMA flops / per-SM tensor
+  // rate) plus a fixed pipeline fill (at M >= 256 decode GEMMs are
+  // compute-bound per SM; at M <= 128 the weight stream binds).  Tiles fill
+  // full waves of m SMs; the ragged remainder may be split `ts` ways over K,
+  // paying an fp32 partial round trip (the fixup is latency-bound: priced at
+  // 8 GB/s per SM).  A single accumulator stage
+  // (mh * bn > 256 columns) exposes the epilogue.  mh = 2 only for
+  // decode-sized M.  Rates: KI2.
+  constexpr double BW_SM = 90e9, FL_SM = 10.5e12, EPI_BW = 100e9, FIX_BW = 8e9, T0 = 0.6e-6;
   const int k_blocks = K / 64;
-  int bn = 0, splits = 1;
+  int mh = 1, bn = 0, ts = 1, n_full = 0;
   double best = 1e300;
-  for (int cand : {256, 128, 64}) {
-    if (!fits(cand)) continue;
-    const int tiles = m_tiles * (N / cand);
-    const int max_s = std::max(1, std::min(k_blocks / 4, N_TILE_SEMS / std::max(1, tiles)));
-    for (int s = 1; s <= max_s; ++s) {
-      if (s > 1 && (size_t)tiles * s * 128 * cand > h->ph[c.phase].partial_floats) break;
-      const double waves = std::ceil((double)tiles * s / c.m_sms);
-      const double cost = waves * ((double)k_blocks / s) * (128 + cand) * 128.0 +
-                          (s > 1 ? 3.0 * s * 128.0 * cand * 4.0 : 0.0) + waves * 64e3;
-      if (cost < best * 0.999) { best = cost; bn = cand; splits = s; }
+  for (int cmh = (M > 128 && M <= 512) ? 2 : 1; cmh >= 1; --cmh) {
+    const int m_tiles = (M + 128 * cmh - 1) / (128 * cmh);
+    for (int cand : {256, 128, 64}) {
+      if (!fits(cand)) continue;
+      const int tiles = m_tiles * (N / cand);
+      const double out_b = 128.0 * cmh * cand * 4.0;
+      const double t_tile = std::max((double)k_blocks * (cmh * 16384.0 + cand * 128.0) / BW_SM,
+                                     2.0 * 128 * cmh * cand * K / FL_SM) +
+                            (2 * cmh * cand > 512 ? out_b / EPI_BW : 0.0) + T0;
+      const int full_waves = tiles / c.m_sms, rem = tiles % c.m_sms;
+      const int max_ts = rem ? std::max(1, std::min(16, k_blocks / 4)) : 1;
+      for (int cts = 1; cts <= max_ts; ++cts) {
+        if (cts > 1 && ((size_t)rem * cts * 128 * cmh * cand > h->ph[c.phase].partial_floats || rem > N_TILE_SEMS))
+          break;
+        const double tail = rem == 0 ? 0.0
+                            : cts == 1 ? t_tile
+                                       : std::ceil((double)rem * cts / c.m_sms) *
+                                             ((t_tile - T0) / cts + T0 + (cts + 2) * out_b / FIX_BW);
+        const double cost = full_waves * t_tile + tail;
+        if (cost < best * 0.999) {
+          best = cost; mh = cmh; bn = cand; ts = cts;
+          n_full = cts > 1 ? tiles - rem : tiles;
+        }
+      }
     }
   }
   if (!bn) return set_err(BULLET_EUNSUPPORTED, "GEMM N=%d not tileable", N);
-  a.bn = bn; a.splits = splits;
+  if (const char* ov = getenv("BULLET_GEMM_PLAN")) {   // experiments: "mh,bn,ts"
+    int omh = 0, obn = 0, ots = 0;
+    if (sscanf(ov, "%d,%d,%d", &omh, &obn, &ots) == 3 && fits(obn) && omh >= 1 && omh <= 2 && ots >= 1) {
+      const int tiles = ((M + 128 * omh - 1) / (128 * omh)) * (N / obn), rem = tiles % c.m_sms;
+      if (ots == 1 || (rem && (size_t)rem * ots * 128 * omh * obn <= h->ph[c.phase].partial_floats)) {
+        mh = omh; bn = obn; ts = ots; n_full = (ts > 1) ? tiles - rem : tiles;
+      }
+    }
+  }
+  if (getenv("BULLET_GEMM_DEBUG"))
+    fprintf(stderr, "gemm M=%d N=%d K=%d m_sms=%d -> mh=%d bn=%d n_full=%d ts=%d\n", M, N, K, c.m_sms, mh, bn,
+            n_full, ts);
+  a.bn = bn; a.mh = mh; a.splits = ts; a.n_full = n_full;
   a.b_packed = Bp;
   a.b_rows = N + (epi == EPI_SILU ? silu_half - N / 2 : 0);
   a.partials = h->ph[c.phase].partials;
   a.tile_sems = h->ph[c.phase].tile_sems;
   CUtensorMap ma, mb;
-  if ((rc = make_map(&ma, A, M, K, 128))) return rc;
+  if ((rc = make_map(&ma, A, M, K, 128))) return rc;   // one 128-row half per TMA box
   if ((rc = make_map(&mb, B, N, K, bn / 2))) return rc;
   LAUNCH(c, launch_gemm_tc(ma, mb, a, h->n_sms, c.st));
   return BULLET_OK;

@@ -12,10 +12,15 @@
 //   warps 4..7     epilogue: tcgen05.ld 32x32b -> registers -> global
 // Pipelines: smem stage ring (full/empty mbarriers, TMA complete_tx and
 // tcgen05.commit), accumulator ring (2 stages), work-unit queue (4 slots).
-// Operand tiles: A 128 x 64, B bn x 64 (bf16, 128-byte swizzle, TMA).
-// Split-K (decode-sized GEMMs): each unit writes an fp32 partial; the last
-// unit of a tile (atomic ticket) sums the partials in split order
-// (deterministic) and runs the epilogue.
+// Operand tiles: A mh x (128 x 64), B bn x 64 (bf16, 128-byte swizzle, TMA).
+// mh = 2 (decode-sized M <= 512): a unit covers 256 rows with two M=128
+// accumulators that share every B stage, so weights stream through an SM
+// once per 256 rows instead of once per 128.
+// Tail split: units [0, n_full) are whole tiles; each remaining tile (the
+// ragged last wave) is split `splits` ways over K so that wave fills the
+// partition.  A split unit writes an fp32 partial; the last unit of its tile
+// (atomic ticket) sums the partials in split order (deterministic) and runs
+// the epilogue.
 #include "kernels.h"
 
 namespace bl {
@@ -23,7 +28,21 @@ namespace bl {
 namespace {
 
 constexpr int BM = 128, BK = 64, NT = 256;
-constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
+constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB per 128-row half
+
+struct UnitInfo {
+  int tile, sp, ns, tail;   // tail: index among split units (partials slot), -1 for whole tiles
+};
+__device__ __forceinline__ UnitInfo unit_info(const GemmArgs& a, int u) {
+  UnitInfo r;
+  if (u < a.n_full) {
+    r.tile = u; r.sp = 0; r.ns = 1; r.tail = -1;
+  } else {
+    const int t = u - a.n_full;
+    r.tile = a.n_full + t / a.splits; r.sp = t % a.splits; r.ns = a.splits; r.tail = t;
+  }
+  return r;
+}
 
 __device__ __forceinline__ uint64_t sw128_desc(uint32_t addr) {
   // UMMA shared-memory descriptor, K-major, SWIZZLE_128B: start>>4 [0,14),
@@ -120,16 +139,17 @@ __device__ __forceinline__ void epi_store(const GemmArgs& a, int m, int col, con
 
 }  // namespace
 
-int gemm_tc_stages(int bn) {
-  const int st = A_BYTES + bn * BK * 2;
+int gemm_tc_stages(int bn, int mh) {
+  const int st = mh * A_BYTES + bn * BK * 2;
   int s = (192 * 1024) / st;
   return s > 8 ? 8 : s;
 }
-size_t gemm_tc_smem_bytes(int bn) {
-  const int st = A_BYTES + bn * BK * 2;
-  return (size_t)gemm_tc_stages(bn) * st + 1024 /*align*/ + 512 /*barriers etc.*/;
+size_t gemm_tc_smem_bytes(int bn, int mh) {
+  const int st = mh * A_BYTES + bn * BK * 2;
+  return (size_t)gemm_tc_stages(bn, mh) * st + 1024 /*align*/ + 512 /*barriers etc.*/;
 }
 
+template <int mh>
 __global__ void __launch_bounds__(NT, 1)
     k_gemm_tc(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
               GemmArgs a, int n_stages) {
@@ -138,7 +158,10 @@ __global__ void __launch_bounds__(NT, 1)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~uintptr_t(1023));
   const int bn = a.bn;
-  const uint32_t b_bytes = bn * BK * 2, st_bytes = A_BYTES + b_bytes;
+  const uint32_t a_bytes = mh * A_BYTES, b_bytes = bn * BK * 2, st_bytes = a_bytes + b_bytes;
+  // accumulator ring: mh * bn TMEM columns per stage, two stages when they fit
+  const uint32_t acc_cols = mh * bn;
+  const int n_acc = 2 * acc_cols <= 512 ? 2 : 1;
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + n_stages * st_bytes);
   uint64_t* empty = full + n_stages;
   uint64_t* accf = empty + n_stages;
@@ -150,9 +173,9 @@ __global__ void __launch_bounds__(NT, 1)
   int* s_last = reinterpret_cast<int*>(tmem_slot + 1);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int m_tiles = (a.M + BM - 1) / BM;
+  const int m_tiles = (a.M + BM * mh - 1) / (BM * mh);
   const int n_tiles = a.N / bn;
-  const int units = m_tiles * n_tiles * a.splits;
+  const int units = a.n_full + (m_tiles * n_tiles - a.n_full) * a.splits;
   const int k_blocks = a.K / BK;
 
   if (threadIdx.x == 0) {
@@ -189,9 +212,9 @@ __global__ void __launch_bounds__(NT, 1)
         mbar_arrive(tqf + slot);
         if (u < 0) break;
         log_unit(a.L, u);
-        const int tile = u / a.splits, sp = u % a.splits;
-        const int m_blk = tile % m_tiles, n_blk = tile / m_tiles;
-        const int kb0 = sp * k_blocks / a.splits, kb1 = (sp + 1) * k_blocks / a.splits;
+        const UnitInfo ui = unit_info(a, u);
+        const int m_blk = ui.tile % m_tiles, n_blk = ui.tile / m_tiles;
+        const int kb0 = ui.sp * k_blocks / ui.ns, kb1 = (ui.sp + 1) * k_blocks / ui.ns;
         int r0, r1;
         if (a.epi == EPI_SILU) { r0 = n_blk * (bn / 2); r1 = a.silu_half + r0; }
         else { r0 = n_blk * bn; r1 = r0 + bn / 2; }
@@ -199,18 +222,21 @@ __global__ void __launch_bounds__(NT, 1)
           mbar_wait(empty + s, ph ^ 1);
           uint8_t* sa = smem + s * st_bytes;
           mbar_arrive_expect_tx(full + s, st_bytes);
-          tma_load_2d(sa, &mapA, full + s, kb * BK, m_blk * BM);
+#pragma unroll
+          for (int hh = 0; hh < mh; ++hh)   // rows past M are zero-filled by TMA
+            tma_load_2d(sa + hh * A_BYTES, &mapA, full + s, kb * BK, (m_blk * mh + hh) * BM);
+          uint8_t* sb = sa + a_bytes;
           if (a.b_packed) {   // pre-swizzled tiles: contiguous bulk copies
             const uint8_t* kbase = a.b_packed + (size_t)kb * (a.b_rows / 64) * 8192;
             if (r1 == r0 + bn / 2) {
-              bulk_g2s(sa + A_BYTES, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s);
+              bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s);
             } else {
-              bulk_g2s(sa + A_BYTES, kbase + (size_t)(r0 / 64) * 8192, b_bytes / 2, full + s);
-              bulk_g2s(sa + A_BYTES + b_bytes / 2, kbase + (size_t)(r1 / 64) * 8192, b_bytes / 2, full + s);
+              bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes / 2, full + s);
+              bulk_g2s(sb + b_bytes / 2, kbase + (size_t)(r1 / 64) * 8192, b_bytes / 2, full + s);
             }
           } else {
-            tma_load_2d(sa + A_BYTES, &mapB, full + s, kb * BK, r0);
-            tma_load_2d(sa + A_BYTES + b_bytes / 2, &mapB, full + s, kb * BK, r1);
+            tma_load_2d(sb, &mapB, full + s, kb * BK, r0);
+            tma_load_2d(sb + b_bytes / 2, &mapB, full + s, kb * BK, r1);
           }
           if (++s == n_stages) { s = 0; ph ^= 1; }
         }
@@ -229,24 +255,26 @@ __global__ void __launch_bounds__(NT, 1)
         const int u = tile_q[slot];
         mbar_arrive(tqe + slot);
         if (u < 0) break;
-        const int sp = u % a.splits;
-        const int kb0 = sp * k_blocks / a.splits, kb1 = (sp + 1) * k_blocks / a.splits;
+        const UnitInfo ui = unit_info(a, u);
+        const int kb0 = ui.sp * k_blocks / ui.ns, kb1 = (ui.sp + 1) * k_blocks / ui.ns;
         mbar_wait(acce + as, aph ^ 1);
         tc_fence_after();
-        const uint32_t d_tmem = tmem + as * 256;
+        const uint32_t d_tmem = tmem + as * acc_cols;
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(full + s, ph);
           tc_fence_after();
-          const uint32_t a_addr = smem_u32(smem + s * st_bytes), b_addr = a_addr + A_BYTES;
+          const uint32_t a_addr = smem_u32(smem + s * st_bytes), b_addr = a_addr + a_bytes;
 #pragma unroll
           for (int k = 0; k < BK / 16; ++k)
-            tc_mma(d_tmem, sw128_desc(a_addr + k * 32), sw128_desc(b_addr + k * 32), idesc,
-                   (kb > kb0 || k > 0) ? 1u : 0u);
+#pragma unroll
+            for (int hh = 0; hh < mh; ++hh)
+              tc_mma(d_tmem + hh * bn, sw128_desc(a_addr + hh * A_BYTES + k * 32), sw128_desc(b_addr + k * 32),
+                     idesc, (kb > kb0 || k > 0) ? 1u : 0u);
           tc_commit(empty + s);
           if (++s == n_stages) { s = 0; ph ^= 1; }
         }
         tc_commit(accf + as);
-        if (++as == 2) { as = 0; aph ^= 1; }
+        if (++as == n_acc) { as = 0; aph ^= 1; }
         ++it;
       }
     }
@@ -262,64 +290,66 @@ __global__ void __launch_bounds__(NT, 1)
       __syncwarp();
       if (lane == 0) mbar_arrive(tqe + slot);
       if (u < 0) break;
-      const int tile = u / a.splits;
-      const int m_blk = tile % m_tiles, n_blk = tile / m_tiles;
-      const int m = m_blk * BM + et;
+      const UnitInfo ui = unit_info(a, u);
+      const int m_blk = ui.tile % m_tiles, n_blk = ui.tile / m_tiles;
       const int col0 = (a.epi == EPI_SILU) ? n_blk * (bn / 2) : n_blk * bn;
       const int out_chunks = (a.epi == EPI_SILU) ? bn / 64 : bn / 32;
       mbar_wait(accf + as, aph);
       tc_fence_after();
-      const uint32_t tb = tmem + ((uint32_t)(eq * 32) << 16) + as * 256;
-      if (a.splits == 1) {
-        for (int c = 0; c < out_chunks; ++c) {
-          tmem_ld32(tb + c * 32, v);
-          if (a.epi == EPI_SILU) tmem_ld32(tb + bn / 2 + c * 32, w);
-          if (m < a.M) epi_store(a, m, col0 + c * 32, v, w);
+      const uint32_t tb = tmem + ((uint32_t)(eq * 32) << 16) + as * acc_cols;
+      if (ui.ns == 1) {
+        for (int hh = 0; hh < mh; ++hh) {
+          const int m = (m_blk * mh + hh) * BM + et;
+          for (int c = 0; c < out_chunks; ++c) {
+            tmem_ld32(tb + hh * bn + c * 32, v);
+            if (a.epi == EPI_SILU) tmem_ld32(tb + hh * bn + bn / 2 + c * 32, w);
+            if (m < a.M) epi_store(a, m, col0 + c * 32, v, w);
+          }
         }
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(acce + as);
       } else {
-        float* P = a.partials + ((size_t)u * BM + et) * bn;
-        for (int c = 0; c < bn / 32; ++c) {
-          tmem_ld32(tb + c * 32, v);
-          float4* d4 = reinterpret_cast<float4*>(P + c * 32);
+        // partial tile stored column-major per half ([hh][col][row]): a warp's
+        // 32 rows of one column are 128 contiguous bytes, so the stores and
+        // the fixup's loads are fully coalesced
+        const size_t tile_floats = (size_t)mh * BM * bn;
+        float* P = a.partials + (size_t)ui.tail * tile_floats + et;
+        for (int hh = 0; hh < mh; ++hh)
+          for (int c = 0; c < bn / 32; ++c) {
+            tmem_ld32(tb + hh * bn + c * 32, v);
 #pragma unroll
-          for (int i = 0; i < 8; ++i) d4[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
-        }
+            for (int i = 0; i < 32; ++i) __stcg(P + (size_t)hh * BM * bn + (size_t)(c * 32 + i) * BM, v[i]);
+          }
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(acce + as);
         __threadfence();
         named_bar_sync(1, 128);
+        const int sem = ui.tile - a.n_full;
         if (et == 0) {
-          const int old = atomicAdd(a.tile_sems + tile, 1);
-          const int last = (old == a.splits - 1);
-          if (last) a.tile_sems[tile] = 0;  // self-reset for the next launch
+          const int old = atomicAdd(a.tile_sems + sem, 1);
+          const int last = (old == ui.ns - 1);
+          if (last) a.tile_sems[sem] = 0;  // self-reset for the next launch
           *s_last = last;
         }
         named_bar_sync(1, 128);
         if (*s_last) {
           __threadfence();
-          if (m < a.M) {
+          const float* T0 = a.partials + (size_t)(ui.tail - ui.sp) * tile_floats + et;   // split 0 of this tile
+          for (int hh = 0; hh < mh; ++hh) {
+            const int m = (m_blk * mh + hh) * BM + et;
+            if (m >= a.M) continue;
             for (int c = 0; c < out_chunks; ++c) {
 #pragma unroll
               for (int i = 0; i < 32; ++i) { v[i] = 0.f; w[i] = 0.f; }
-              for (int sp = 0; sp < a.splits; ++sp) {  // fixed split order: deterministic
-                const float* Q = a.partials + ((size_t)(tile * a.splits + sp) * BM + et) * bn;
-                const float4* q4 = reinterpret_cast<const float4*>(Q + c * 32);
+              for (int sp = 0; sp < ui.ns; ++sp) {  // fixed split order: deterministic
+                const float* Q = T0 + (size_t)sp * tile_floats + (size_t)hh * BM * bn;
 #pragma unroll
-                for (int i = 0; i < 8; ++i) {
-                  float4 t = __ldcg(q4 + i);
-                  v[4 * i] += t.x; v[4 * i + 1] += t.y; v[4 * i + 2] += t.z; v[4 * i + 3] += t.w;
-                }
+                for (int i = 0; i < 32; ++i) v[i] += __ldcg(Q + (size_t)(c * 32 + i) * BM);
                 if (a.epi == EPI_SILU) {
-                  const float4* g4 = reinterpret_cast<const float4*>(Q + bn / 2 + c * 32);
 #pragma unroll
-                  for (int i = 0; i < 8; ++i) {
-                    float4 t = __ldcg(g4 + i);
-                    w[4 * i] += t.x; w[4 * i + 1] += t.y; w[4 * i + 2] += t.z; w[4 * i + 3] += t.w;
-                  }
+                  for (int i = 0; i < 32; ++i) w[i] += __ldcg(Q + (size_t)(bn / 2 + c * 32 + i) * BM);
                 }
               }
               epi_store(a, m, col0 + c * 32, v, w);
@@ -327,7 +357,7 @@ __global__ void __launch_bounds__(NT, 1)
           }
         }
       }
-      if (++as == 2) { as = 0; aph ^= 1; }
+      if (++as == n_acc) { as = 0; aph ^= 1; }
       ++it;
     }
   }
@@ -363,17 +393,20 @@ cudaError_t launch_pack_weight(const __nv_bfloat16* W, int R, int K, uint8_t* ou
 
 cudaError_t launch_gemm_tc(const CUtensorMap& mapA, const CUtensorMap& mapB, const GemmArgs& a,
                            int grid, cudaStream_t st) {
-  const size_t smem = gemm_tc_smem_bytes(a.bn);
+  const size_t smem = gemm_tc_smem_bytes(a.bn, a.mh);
   static bool attr_set = false;
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_gemm_tc, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)gemm_tc_smem_bytes(64) > (int)gemm_tc_smem_bytes(256)
-                                             ? (int)gemm_tc_smem_bytes(64)
-                                             : (int)gemm_tc_smem_bytes(256));
+    size_t mx = 0;
+    for (int mh = 1; mh <= 2; ++mh)
+      for (int bn = 64; bn <= 256; bn *= 2) mx = std::max(mx, gemm_tc_smem_bytes(bn, mh));
+    cudaError_t e = cudaFuncSetAttribute(k_gemm_tc<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)mx);
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(k_gemm_tc<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)mx);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  k_gemm_tc<<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn));
+  if (a.mh < 1 || a.mh > 2 || a.splits < 1) return cudaErrorInvalidValue;
+  if (a.mh == 2) k_gemm_tc<2><<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn, 2));
+  else k_gemm_tc<1><<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn, 1));
   return cudaGetLastError();
 }
 

@@ -10,7 +10,9 @@ enum { EPI_F32 = 0, EPI_RESID = 1, EPI_SILU = 2 };
 struct GemmArgs {
   int M, N, K;        // N = B rows used (2 x output cols for EPI_SILU)
   int bn;             // tile width in B rows (tcgen05: 64/128/256; SIMT: 64)
-  int splits;         // split-K factor (tcgen05 only)
+  int mh;             // tcgen05: 128-row halves per unit (1, or 2 = 256 rows sharing each B stage)
+  int n_full;         // tcgen05: units [0, n_full) are whole tiles over all of K ...
+  int splits;         // ... the remaining tiles are split `splits` ways over K (tail split)
   int epi;
   int silu_half;      // row offset of the "up" rows in B (EPI_SILU)
   const void* bias;   // [N] of the element type, or null (EPI_F32)
@@ -18,8 +20,8 @@ struct GemmArgs {
   float* out_f32;     // [M][ldo] (EPI_F32, EPI_RESID)
   void* out_t;        // [M][ldo] of the element type (EPI_SILU)
   int ldo;
-  float* partials;    // split-K: [units][128][bn]
-  int* tile_sems;     // split-K: [tiles], zero between launches (self-resetting)
+  float* partials;    // tail split: [tail units][mh][bn][128] (column-major per half)
+  int* tile_sems;     // tail split: [tail tiles], zero between launches (self-resetting)
   const uint8_t* b_packed;  // B pre-packed by pack_weight (else B comes through mapB)
   int b_rows;               // rows of B (packed layout stride)
   Launch L;
@@ -71,8 +73,8 @@ struct PlanArgs {
 // launchers (return cudaError_t of the launch)
 cudaError_t launch_gemm_tc(const CUtensorMap& mapA, const CUtensorMap& mapB, const GemmArgs& a,
                            int grid, cudaStream_t st);
-size_t gemm_tc_smem_bytes(int bn);
-int gemm_tc_stages(int bn);
+size_t gemm_tc_smem_bytes(int bn, int mh);
+int gemm_tc_stages(int bn, int mh);
 template <typename T>
 cudaError_t launch_gemm_simt(const T* A, const T* B, const GemmArgs& a, int grid, cudaStream_t st);
 template <typename T>

@@ -46,10 +46,10 @@ def _int_operands(rng, M, K, N):
 
 
 @pytest.mark.parametrize("M,N,K,lo,hi", [
-    (128, 6144, 4096, 0, None),     # decode-sized: bn 128 + split-K
+    (128, 6144, 4096, 0, None),     # decode-sized
     (300, 1024, 1024, 0, None),     # ragged M tail
     (4096, 6144, 4096, 0, None),    # prefill-sized: bn 256
-    (257, 4096, 4096, 10, 50),      # 40-SM gated range, split-K fixup
+    (257, 4096, 4096, 10, 50),      # 40-SM gated range: mh=2 units, tail split
     (64, 1280, 8192, 0, 16),        # 16 SMs, K = 8192
 ])
 @pytest.mark.parametrize("packed", [False, True])
@@ -68,6 +68,41 @@ def test_gemm_f32_epilogue_bit_exact(B, M, N, K, lo, hi, packed):
     # fp64 BLAS is exact here: integer partial sums stay far below 2^53
     ref = (torch.from_numpy(A).double() @ torch.from_numpy(W).double().T).numpy() + bias
     assert np.array_equal(out.cpu().numpy(), ref.astype(np.float32))
+
+
+# Every plan shape of the tcgen05 GEMM, forced through BULLET_GEMM_PLAN
+# ("mh,bn,ts"): 256-row units (mh=2) with a ragged second half, tail splits
+# of the last wave on a 20-SM partition, both combined, every epilogue.
+@pytest.mark.parametrize("plan", ["1,256,1", "2,256,1", "2,128,1", "1,128,5", "2,128,3", "2,64,7", "2,256,2"])
+@pytest.mark.parametrize("epi", ["f32", "resid", "silu"])
+def test_gemm_plans_bit_exact(B, plan, epi, monkeypatch):
+    monkeypatch.setenv("BULLET_GEMM_PLAN", plan)
+    bl, _ = _handle(B, SMALL)
+    rng = np.random.default_rng(11)
+    M, K, N = 200, 2048, 1536
+    A, W = _int_operands(rng, M, K, N)
+    if epi == "silu":
+        W = W * 0.0625
+    At, Wt = torch.from_numpy(A).to("cuda", bf16), torch.from_numpy(W).to("cuda", bf16)
+    gu = (torch.from_numpy(A).double() @ torch.from_numpy(W).double().T).numpy()
+    lo, hi = 100, 120
+    if epi == "f32":
+        out = torch.full((M, N), float("nan"), device="cuda")
+        bl.op_gemm(B.EPI_F32, At, Wt, out, lo=lo, hi=hi)
+        assert np.array_equal(out.cpu().numpy(), gu.astype(np.float32))
+    elif epi == "resid":
+        R = rng.integers(-50, 50, size=(M, N)).astype(np.float32)
+        h = torch.from_numpy(R).cuda()
+        bl.op_gemm(B.EPI_RESID, At, Wt, h, resid=h, lo=lo, hi=hi)
+        assert np.array_equal(h.cpu().numpy(), (R + gu).astype(np.float32))
+    else:
+        I = N // 2
+        out = torch.zeros(M, I, dtype=bf16, device="cuda")
+        bl.op_gemm(B.EPI_SILU, At, Wt, out, silu_half=I, lo=lo, hi=hi)
+        g, u = gu[:, :I], gu[:, I:]
+        ref = g / (1 + np.exp(-g)) * u
+        got = out.float().cpu().numpy()
+        assert np.all(np.abs(got - ref) <= np.maximum(np.abs(ref), 1e-30) * 2.0 ** -7 + 1e-6)
 
 
 def test_gemm_matches_oracle_linear_small(B):
