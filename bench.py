@@ -192,12 +192,13 @@ class Step:
     def tokens(self, k):
         return (self.n_p * 1 + self.n_d * k) / self.m.n_layers
 
-    def tune(self, cands, reps=3):
+    def tune(self, cands, t_pre_full, t_dec_full, reps=3):
         """For each candidate prefill SM count p: time the isolated prefill
-        layer on p SMs and decode layer-step on N-p SMs, set k = round(T_p/T_d)
-        (decode steps per prefill layer), then time the real co-run
-        step and the fitted model's prediction; pick the best measured co-run
-        tokens/s."""
+        layer on p SMs and decode layer-step on N-p SMs; around the balance
+        point k0 = round(T_p/T_d) (decode steps per prefill layer) try
+        k0-1 .. k0+2, timing the real co-run step and the fitted model's
+        prediction.  Pick the (p, k) with the best co-run speedup over running
+        the same batch time-sliced on the full GPU (BASELINE's target)."""
         B = self.B
         res = []
         for p in cands:
@@ -206,16 +207,20 @@ class Step:
             tp = self.time_steps(reps, p, B.CORUN, dec=False)
             self.time_steps(1, p, B.CORUN, pre=False)
             td = self.time_steps(reps, p, B.CORUN, pre=False)
-            k = int(min(self.k_max, max(1, round(tp / td))))
-            self.dec.layer_end = k
-            self.time_steps(1, p, B.CORUN)
-            tco = self.time_steps(reps, p, B.CORUN)
+            k0 = int(max(1, round(tp / td)))
             q, c = self.pre.cu[1:] - self.pre.cu[:-1], self.pre.ctx_lens
             mp = self.bl.predict_us(q, c, p, self.N - p) / 1e3
-            md = self.bl.predict_us([1] * self.n_d, self.dec.ctx_lens, self.N - p, p) / 1e3 * k
-            res.append({"p": p, "k": k, "t_prefill_ms": tp, "t_decode_ms": td, "t_corun_ms": tco,
-                        "tok_s": self.tokens(k) / tco * 1e3, "model_corun_ms": max(mp, md)})
-        best = max(res, key=lambda r: r["tok_s"])
+            md1 = self.bl.predict_us([1] * self.n_d, self.dec.ctx_lens, self.N - p, p) / 1e3
+            for k in sorted({max(1, k0 - 1), k0, k0 + 1, k0 + 2}):
+                if k > self.k_max:
+                    continue
+                self.dec.layer_end = k
+                self.time_steps(1, p, B.CORUN)
+                tco = self.time_steps(reps, p, B.CORUN)
+                res.append({"p": p, "k": k, "t_prefill_ms": tp, "t_decode_ms": td, "t_corun_ms": tco,
+                            "tok_s": self.tokens(k) / tco * 1e3, "model_corun_ms": max(mp, md1 * k),
+                            "speedup_vs_timesliced_est": (t_pre_full + k * t_dec_full) / tco})
+        best = max(res, key=lambda r: r["speedup_vs_timesliced_est"])
         self.dec.layer_end = 1
         return best, res
 
@@ -316,10 +321,16 @@ def main():
     import paper_conf_asplos_0001xc0l026_b200 as B
     S = Step(args.config, args.k_max)
     N = S.N
+    # ---- alone-on-full-GPU references (per layer)
+    S.dec.layer_end = 1
+    S.time_steps(1, N, B.CORUN, dec=False)
+    t_pre_full = S.time_steps(3, N, B.CORUN, dec=False)
+    S.time_steps(1, 0, B.CORUN, pre=False)
+    t_dec_full = S.time_steps(3, 0, B.CORUN, pre=False)
     # ---- choose the split (p, k)
     if args.p is None or args.k is None:
         cands = [args.p] if args.p else list(range(72, N - 15, 8))
-        best, table = S.tune(cands)
+        best, table = S.tune(cands, t_pre_full, t_dec_full)
         p = args.p or best["p"]
         k = args.k or best["k"]
         if args.sweep and rank == 0:
@@ -335,11 +346,6 @@ def main():
                  decode_mean_ctx=float(np.mean(S.wl.decode_ctx)), u_k=p, v_k=N - p)
     slo = {"ttft_norm_ms_per_tok": 3.0, "tpot_ms": 150.0, "w_max": 4, "v_min": 16, "percentile": 0.9}
     model_split = S.bl.choose_split(state, slo)
-    S.dec.layer_end = k
-    # ---- alone-on-full-GPU references (per layer)
-    t_pre_full = S.time_steps(3, N, B.CORUN, dec=False)
-    S.dec.layer_end = 1
-    t_dec_full = S.time_steps(3, 0, B.CORUN, pre=False)
     S.dec.layer_end = k
     # ---- co-run (the method) and time-sliced, device-timed, max over ranks
     for _ in range(args.warmup):
@@ -369,7 +375,8 @@ def main():
     P, src = peaks()
     tf = os.path.join(ROOT, "profiles", "r01_traffic.json")   # ncu --set full capture of the same kernel
     dom_name = f"{dom[0]} ({'prefill' if dom[1] == 0 else 'decode'})"
-    traffic = json.load(open(tf))["bytes"].get(dom_name) if os.path.exists(tf) else None
+    traffic = (json.load(open(tf))["bytes"].get(args.config, {}).get(dom_name)
+               if os.path.exists(tf) else None)
     if bound == "tensor":
         achieved = work / (avg_ms * 1e-3) / 1e12
         peak, unit = P.get("bf16_tflops_sustained", P["bf16_tflops"]), "TFLOP/s"

@@ -245,11 +245,12 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   // rate) plus a fixed pipeline fill (at M >= 256 decode GEMMs are
   // compute-bound per SM; at M <= 128 the weight stream binds).  Tiles fill
   // full waves of m SMs; the ragged remainder may be split `ts` ways over K,
-  // paying an fp32 partial round trip (the fixup is latency-bound: priced at
-  // 8 GB/s per SM).  A single accumulator stage
+  // paying an fp32 partial round trip: the writes, then the last unit's
+  // latency-bound sum (one ~1.3 us round trip per 2 splits x 32 columns).
+  // A single accumulator stage
   // (mh * bn > 256 columns) exposes the epilogue.  mh = 2 only for
   // decode-sized M.  Rates: KI2.
-  constexpr double BW_SM = 90e9, FL_SM = 10.5e12, EPI_BW = 100e9, FIX_BW = 8e9, T0 = 0.6e-6;
+  constexpr double BW_SM = 90e9, FL_SM = 10.5e12, EPI_BW = 100e9, RTT = 1.3e-6, T0 = 0.6e-6;
   const int k_blocks = K / 64;
   int mh = 1, bn = 0, ts = 1, n_full = 0;
   double best = 1e300;
@@ -270,7 +271,8 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
         const double tail = rem == 0 ? 0.0
                             : cts == 1 ? t_tile
                                        : std::ceil((double)rem * cts / c.m_sms) *
-                                             ((t_tile - T0) / cts + T0 + (cts + 2) * out_b / FIX_BW);
+                                                 ((t_tile - T0) / cts + T0 + out_b / EPI_BW) +
+                                             std::ceil(cts / 2.0) * (cmh * cand / 32) * RTT;
         const double cost = full_waves * t_tile + tail;
         if (cost < best * 0.999) {
           best = cost; mh = cmh; bn = cand; ts = cts;

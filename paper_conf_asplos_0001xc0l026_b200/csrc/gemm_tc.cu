@@ -310,16 +310,19 @@ __global__ void __launch_bounds__(NT, 1)
         __syncwarp();
         if (lane == 0) mbar_arrive(acce + as);
       } else {
-        // partial tile stored column-major per half ([hh][col][row]): a warp's
-        // 32 rows of one column are 128 contiguous bytes, so the stores and
-        // the fixup's loads are fully coalesced
-        const size_t tile_floats = (size_t)mh * BM * bn;
-        float* P = a.partials + (size_t)ui.tail * tile_floats + et;
+        // partial tile stored as float4 groups interleaved by row per half
+        // ([hh][col/4][row][4]): a thread's 4 consecutive columns are one
+        // float4 and a warp's 32 rows are 512 contiguous bytes, so stores
+        // and the fixup's loads are vectorised and coalesced
+        const size_t tile_f4 = (size_t)mh * BM * bn / 4;
+        float4* P = reinterpret_cast<float4*>(a.partials) + (size_t)ui.tail * tile_f4 + et;
         for (int hh = 0; hh < mh; ++hh)
           for (int c = 0; c < bn / 32; ++c) {
             tmem_ld32(tb + hh * bn + c * 32, v);
 #pragma unroll
-            for (int i = 0; i < 32; ++i) __stcg(P + (size_t)hh * BM * bn + (size_t)(c * 32 + i) * BM, v[i]);
+            for (int i = 0; i < 8; ++i)
+              __stcg(P + (size_t)hh * BM * bn / 4 + (size_t)(c * 8 + i) * BM,
+                     make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]));
           }
         tc_fence_before();
         __syncwarp();
@@ -336,22 +339,34 @@ __global__ void __launch_bounds__(NT, 1)
         named_bar_sync(1, 128);
         if (*s_last) {
           __threadfence();
-          const float* T0 = a.partials + (size_t)(ui.tail - ui.sp) * tile_floats + et;   // split 0 of this tile
+          const float4* T0 = reinterpret_cast<const float4*>(a.partials) + (size_t)(ui.tail - ui.sp) * tile_f4 + et;
+          // sum 32 columns of all splits (fixed split order: deterministic),
+          // two splits per batch so 16 float4 loads are in flight per thread
+          auto sum32 = [&](const float4* base, float* acc) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i) acc[i] = 0.f;
+            for (int sp = 0; sp < ui.ns; sp += 2) {
+              float4 x[8], y[8];
+              const bool two = sp + 1 < ui.ns;
+#pragma unroll
+              for (int i = 0; i < 8; ++i) {
+                x[i] = __ldcg(base + (size_t)sp * tile_f4 + (size_t)i * BM);
+                y[i] = two ? __ldcg(base + (size_t)(sp + 1) * tile_f4 + (size_t)i * BM) : make_float4(0.f, 0.f, 0.f, 0.f);
+              }
+#pragma unroll
+              for (int i = 0; i < 8; ++i) {   // split sp first, then sp + 1
+                acc[4 * i] += x[i].x; acc[4 * i + 1] += x[i].y; acc[4 * i + 2] += x[i].z; acc[4 * i + 3] += x[i].w;
+                acc[4 * i] += y[i].x; acc[4 * i + 1] += y[i].y; acc[4 * i + 2] += y[i].z; acc[4 * i + 3] += y[i].w;
+              }
+            }
+          };
           for (int hh = 0; hh < mh; ++hh) {
             const int m = (m_blk * mh + hh) * BM + et;
             if (m >= a.M) continue;
+            const float4* H = T0 + (size_t)hh * BM * bn / 4;
             for (int c = 0; c < out_chunks; ++c) {
-#pragma unroll
-              for (int i = 0; i < 32; ++i) { v[i] = 0.f; w[i] = 0.f; }
-              for (int sp = 0; sp < ui.ns; ++sp) {  // fixed split order: deterministic
-                const float* Q = T0 + (size_t)sp * tile_floats + (size_t)hh * BM * bn;
-#pragma unroll
-                for (int i = 0; i < 32; ++i) v[i] += __ldcg(Q + (size_t)(c * 32 + i) * BM);
-                if (a.epi == EPI_SILU) {
-#pragma unroll
-                  for (int i = 0; i < 32; ++i) w[i] += __ldcg(Q + (size_t)(bn / 2 + c * 32 + i) * BM);
-                }
-              }
+              sum32(H + (size_t)(c * 8) * BM, v);
+              if (a.epi == EPI_SILU) sum32(H + (size_t)(bn / 8 + c * 8) * BM, w);
               epi_store(a, m, col0 + c * 32, v, w);
             }
           }

@@ -20,7 +20,7 @@ struct GemmArgs {
   float* out_f32;     // [M][ldo] (EPI_F32, EPI_RESID)
   void* out_t;        // [M][ldo] of the element type (EPI_SILU)
   int ldo;
-  float* partials;    // tail split: [tail units][mh][bn][128] (column-major per half)
+  float* partials;    // tail split: [tail units][mh][bn/4][128][4] (float4 groups interleaved by row)
   int* tile_sems;     // tail split: [tail tiles], zero between launches (self-resetting)
   const uint8_t* b_packed;  // B pre-packed by pack_weight (else B comes through mapB)
   int b_rows;               // rows of B (packed layout stride)
