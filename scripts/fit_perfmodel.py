@@ -105,7 +105,7 @@ def base_params(N):
             "p_c": 1.0, "p_b": 1.0,
             "tiles": {"gemm_bm": 128, "gemm_bn": 256, "gemm_bk": 64, "min_k_blocks": 4, "attn_bq": 128,
                       "rows_per_unit": 8},
-            "occ": {"gemm": 1, "attn": 1, "elem": 4}}
+            "occ": {"gemm": 1, "attn": 2, "elem": 4}}
 
 
 def predictor(m_shape, P, N):
