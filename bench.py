@@ -274,6 +274,16 @@ def oracle_sample(m: synth.ModelShape, wl: synth.Workload, n_pre_tok=64, n_dec=3
     return dt, (n_pre_tok + n_dec) / m.n_layers, f"1 layer: 1 prefill x {n_pre_tok} tok + {n_dec} decodes (ctx {min(c[1:])}-{max(c[1:])})"
 
 
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
 def run_reference(args, ws, rank):
     if rank != 0:
         return
@@ -295,7 +305,8 @@ def run_reference(args, ws, rank):
         "ms_per_step": T * 1e3, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "f64", "data": "synthetic",
         "config": {"workload": args.config, "model": wl.model, "sample": desc},
-        "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": cores, "kind": "oracle", "sample": desc},
+        "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": cores, "kind": "oracle", "sample": desc,
+                         "cpu_model": cpu_model()},
         "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}))
 
 
@@ -362,6 +373,21 @@ def main():
         S.enqueue(N, B.TIMESLICED)
     barrier(ws)
     t_ts = allreduce_max(S.time_steps(args.steps, N, B.TIMESLICED), ws)
+    # the paper's "Naive": both phases on all SMs at once, no gating
+    for _ in range(args.warmup):
+        S.enqueue(p, B.UNGATED)
+    barrier(ws)
+    t_ung = allreduce_max(S.time_steps(args.steps, p, B.UNGATED), ws)
+    # model-predict and split-decision latency (host, Table 3 analog)
+    qd, cd = S.pre.cu[1:] - S.pre.cu[:-1], S.pre.ctx_lens
+    t0 = time.perf_counter()
+    for _ in range(200):
+        S.bl.predict_us(qd, cd, p, N - p)
+    us_predict = (time.perf_counter() - t0) / 200 * 1e6
+    t0 = time.perf_counter()
+    for _ in range(20):
+        S.bl.choose_split(state, slo)
+    us_decide = (time.perf_counter() - t0) / 20 * 1e6
     # ---- profiled pass: per-kernel device times inside the co-run step
     S.time_steps(2, p, B.CORUN | B.PROFILE)
     prof = S.bl.profile_read()
@@ -428,8 +454,9 @@ def main():
     m = S.m
     nq = (m.n_heads + 2 * m.n_kv_heads) * m.head_dim
     w_bytes = 2.0 * (nq * m.d_model + m.d_model * m.n_heads * m.head_dim + 3 * m.d_model * m.d_ff)
-    f_pre = 2.0 * S.n_p * w_bytes / 2 + kernel_work(S, "attn", 0)[1]
-    b_dec = k * (w_bytes + kernel_work(S, "attn", 1)[1])
+    f_pre1 = 2.0 * S.n_p * w_bytes / 2 + kernel_work(S, "attn", 0)[1]   # one prefill layer
+    b_dec1 = w_bytes + kernel_work(S, "attn", 1)[1]                      # one decode layer-step
+    f_pre, b_dec = f_pre1, k * b_dec1
     out = {
         "metric": "co-run tokens/s/GPU vs time-sliced; decode HBM GB/s; prefill tensor-pipe util",
         "value": value, "unit": "tokens/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
@@ -445,6 +472,21 @@ def main():
                    "l2": "inputs larger than L2 (weights + KV per step >> 126 MB)"},
         "timesliced": {"value": ts_value, "ms_per_step": t_ts},
         "corun_speedup_vs_timesliced": t_ts / t_co,
+        "ungated": {"value": groups * tok / (t_ung * 1e-3), "ms_per_step": t_ung,
+                    "note": "both phases on all SMs concurrently (the paper's Naive, P:L304)"},
+        "tokens_per_s_by_phase": {"prefill": groups * S.n_p / S.m.n_layers / (t_co * 1e-3),
+                                  "decode": groups * S.n_d * k / S.m.n_layers / (t_co * 1e-3)},
+        "roofline_fractions": {
+            "prefill_alone": {"tflops": f_pre1 / (t_pre_full * 1e-3) / 1e12,
+                              "frac_nominal_2250": f_pre1 / (t_pre_full * 1e-3) / 2250e12,
+                              "frac_measured": f_pre1 / (t_pre_full * 1e-3) / (P["bf16_tflops"] * 1e12)},
+            "decode_alone": {"gbs": b_dec1 / (t_dec_full * 1e-3) / 1e9,
+                             "frac_nominal_8000": b_dec1 / (t_dec_full * 1e-3) / 8000e9,
+                             "frac_measured": b_dec1 / (t_dec_full * 1e-3) / (P["hbm_gbs"] * 1e9)},
+            "corun_sum_measured": f_pre / (t_co * 1e-3) / (P["bf16_tflops"] * 1e12) +
+                                  b_dec / (t_co * 1e-3) / (P["hbm_gbs"] * 1e9),
+            "note": "prefill F_p = 2 P n_p + causal attention flops; decode B_d = weights + KV + activations (SURVEY 8d)"},
+        "model_latency_us": {"predict": us_predict, "choose_split": us_decide},
         "phase_alone_full_gpu_ms": {"prefill_layer": t_pre_full, "decode_layer": t_dec_full},
         "phase_roofline_corun": {
             "prefill_tensor_frac": f_pre / (t_co * 1e-3) / (P.get("bf16_tflops_sustained", 1395.1) * 1e12),
@@ -464,9 +506,14 @@ def main():
                        "perf_params": "profiles/perf_params_b200.json" if S.perf_json else "unfitted"},
     }
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        import oracle as O
         dt, tk, desc = oracle_sample(S.m, S.wl)
+        O.set_threads(1)
+        dt1, tk1, desc1 = oracle_sample(S.m, S.wl, n_pre_tok=16, n_dec=8)
+        O.set_threads(0)
         out["cpu_baseline"] = {"value": tk / dt, "unit": "tokens/s", "cores": os.cpu_count(),
-                               "kind": "oracle", "sample": desc}
+                               "kind": "oracle", "sample": desc, "cpu_model": cpu_model(),
+                               "one_core": {"value": tk1 / dt1, "cores": 1, "sample": desc1}}
     if rank == 0:
         print(json.dumps(out))
     if ws > 1:

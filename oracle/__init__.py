@@ -63,6 +63,8 @@ def lib():
     global _lib
     if _lib is None:
         _lib = ctypes.CDLL(build())
+        _lib.orc_set_threads.restype = ctypes.c_int
+        _lib.orc_set_threads.argtypes = [ctypes.c_int]
         _lib.orc_round_bf16.restype = ctypes.c_double
         _lib.orc_round_bf16.argtypes = [ctypes.c_double]
         _lib.orc_rmsnorm_row.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int,
@@ -130,6 +132,12 @@ def _p(a):
 
 
 # ----------------------------------------------------------------- primitives
+
+def set_threads(n: int) -> int:
+    """OpenMP threads for the oracle's loops (timing only; n <= 0: all cores).
+    Returns the thread count now in effect."""
+    return lib().orc_set_threads(int(n))
+
 
 def round_bf16(x):
     """Round each value to the nearest bf16, ties to even (DESIGN R-3)."""

@@ -283,3 +283,19 @@ int orc_layer_forward(const orc_cfg *c, const orc_weights *w,
   free(row_req); free(row_pos); free(inv_freq); free(q_all);
   return 0;
 }
+
+/* Thread count for the OpenMP loops above (timing only: the 1-core run of
+ * the CPU baseline, SURVEY §8d "Oracle timing"); n <= 0 restores all cores.
+ * Results do not depend on it: every parallel loop writes disjoint rows. */
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+int orc_set_threads(int n) {
+#ifdef _OPENMP
+  omp_set_num_threads(n > 0 ? n : omp_get_num_procs());
+  return omp_get_max_threads();
+#else
+  (void)n;
+  return 1;
+#endif
+}
