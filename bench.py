@@ -167,6 +167,8 @@ class Step:
         self.pre = B.Batch(self.wl.prefill_lens, [0] * self.n_pre, bt[:self.n_pre], self.x_pre, 0, 1)
         self.dec = B.Batch([1] * self.n_d, self.wl.decode_ctx, bt[self.n_pre:], self.x_dec, 0, 1)
         self.sp, self.sd = torch.cuda.Stream(), torch.cuda.Stream()
+        self.sp.wait_stream(torch.cuda.current_stream())   # inputs were made on the current stream
+        self.sd.wait_stream(torch.cuda.current_stream())
         self.N = self.bl.n_sms
 
     def enqueue(self, p, flags, pre=True, dec=True):

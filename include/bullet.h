@@ -198,6 +198,10 @@ int bullet_sm_order(const bullet_handle *h, int32_t *h_sigma, int cap);
  * (smid-gated persistent kernels; replaces libsmctrl masks over MPS,
  * P:L212).  prefill_sm_count = N pauses decode; 0 requires an empty
  * prefill.  Either batch may be NULL.  Asynchronous: enqueue only.
+ * Ordering is the caller's: everything the step reads (hidden, tables,
+ * pools, weights) must already be complete or ordered before s_prefill /
+ * s_decode (e.g. cudaStreamWaitEvent); the step orders only its own kernels
+ * (back to back on each stream, programmatic dependent launches).
  * Errors: EINVAL (shapes), ESMRANGE (split), EKV (block table), ENOMEM
  * (batch larger than cfg max_*). */
 int bullet_step(bullet_handle *h, const bullet_batch *prefill, const bullet_batch *decode,

@@ -54,6 +54,7 @@ class Rig:
             bt[i, :n] = np.arange(pos, pos + n)
             pos += n
         x = torch.randn(sum(q_lens), self.m.d_model, device="cuda")
+        torch.cuda.synchronize()   # x is read on the phase streams
         return B.Batch(q_lens, ctx_lens, bt, x, 0, 1), pos
 
     def time(self, pre, dec, p, reps=5):

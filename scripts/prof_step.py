@@ -25,6 +25,7 @@ def main():
     ap.add_argument("--k", type=int, default=1)
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--quiet", action="store_true")
+    ap.add_argument("--time", type=int, default=0, help="also time this many steps without PROFILE")
     a = ap.parse_args()
     torch.cuda.set_device(0)
     S = bench.Step(a.config, max(1, a.k))
@@ -37,6 +38,8 @@ def main():
     for _ in range(a.reps - 1):
         S.enqueue(p, flags, pre, dec)
     torch.cuda.synchronize()
+    if a.time:
+        print(f"timed {S.time_steps(a.time, p, flags, pre, dec):.4f} ms/step over {a.time} steps")
     ms = S.time_steps(1, p, flags | B.PROFILE, pre, dec)
     if not a.quiet:
         print(f"step {ms:.4f} ms")

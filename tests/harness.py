@@ -18,6 +18,17 @@ def oracle_cfg(m: synth.ModelShape) -> O.OracleCfg:
                        bf16_mirror=1 if m.dtype == "bf16" else 0)
 
 
+def phase_streams():
+    """Two fresh streams for bullet_step, ordered after everything already
+    enqueued on the current stream (the inputs' host->device copies): the
+    library orders nothing the caller enqueued elsewhere (include/bullet.h)."""
+    cur = torch.cuda.current_stream()
+    sp, sd = torch.cuda.Stream(), torch.cuda.Stream()
+    sp.wait_stream(cur)
+    sd.wait_stream(cur)
+    return sp, sd
+
+
 class Setup:
     """Model weights + KV pools + one co-run step's batches, on CPU (oracle)
     and on the GPU (product)."""

@@ -5,7 +5,7 @@ import pytest
 import torch
 
 from workload import synth
-from harness import Setup, compare
+from harness import Setup, compare, phase_streams
 from oracle import perfmodel as PM
 
 pytestmark = pytest.mark.gpu
@@ -14,7 +14,7 @@ pytestmark = pytest.mark.gpu
 def _run(S, p, flags):
     B = S.B
     pre, dec = S.batches()
-    sp, sd = torch.cuda.Stream(), torch.cuda.Stream()
+    sp, sd = phase_streams()
     S.bl.step(pre, dec, p, flags, sp, sd)
     torch.cuda.synchronize()
     return pre, dec
@@ -53,7 +53,7 @@ def _per_layer(S, p, flags):
     from harness import oracle_layer
     pre, dec = S.batches(0, 1)
     x_pre0, x_dec0 = pre.hidden.cpu().numpy(), dec.hidden.cpu().numpy()
-    sp, sd = torch.cuda.Stream(), torch.cuda.Stream()
+    sp, sd = phase_streams()
     outs = []
     for l in range(2):
         pre.layer_begin, pre.layer_end = l, l + 1
