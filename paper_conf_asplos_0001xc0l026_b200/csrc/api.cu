@@ -306,14 +306,23 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   return BULLET_OK;
 }
 
+// Grid of the row-per-CTA kernels: all SMs (gated-out CTAs exit at once), at
+// most 8 CTAs per SM and no more per SM than the partition has rows for —
+// small decode batches would otherwise spend the kernel churning through
+// CTAs that find no row left to claim.
+int row_grid(const Ctx& c, int rows) {
+  const int per_sm = std::max(1, std::min(8, (rows + c.m_sms - 1) / std::max(1, c.m_sms)));
+  return c.h->n_sms * per_sm;
+}
+
 int do_rmsnorm(Ctx& c, const float* x, int n, const void* g, void* out) {
   if (n == 0) return BULLET_OK;
   NormArgs a;
   a.x = x; a.g = g; a.out = out; a.n = n; a.d = c.h->cfg.d_model; a.eps = c.h->cfg.rms_eps;
   int rc = next_launch(c, &a.L);
   if (rc) return rc;
-  if (c.h->cfg.dtype == BULLET_DTYPE_FP32) LAUNCH(c, launch_rmsnorm<float>(a, c.h->n_sms * 8, c.st));
-  else LAUNCH(c, launch_rmsnorm<__nv_bfloat16>(a, c.h->n_sms * 8, c.st));
+  if (c.h->cfg.dtype == BULLET_DTYPE_FP32) LAUNCH(c, launch_rmsnorm<float>(a, row_grid(c, n), c.st));
+  else LAUNCH(c, launch_rmsnorm<__nv_bfloat16>(a, row_grid(c, n), c.st));
   return BULLET_OK;
 }
 
@@ -328,8 +337,8 @@ int do_rope(Ctx& c, const bullet_batch* b, int layer, const float* qkv, void* q)
   a.max_pos = h->cfg.max_position;
   int rc = next_launch(c, &a.L);
   if (rc) return rc;
-  if (h->cfg.dtype == BULLET_DTYPE_FP32) LAUNCH(c, launch_rope_kv<float>(a, h->n_sms * 8, c.st));
-  else LAUNCH(c, launch_rope_kv<__nv_bfloat16>(a, h->n_sms * 8, c.st));
+  if (h->cfg.dtype == BULLET_DTYPE_FP32) LAUNCH(c, launch_rope_kv<float>(a, row_grid(c, b->n_tokens), c.st));
+  else LAUNCH(c, launch_rope_kv<__nv_bfloat16>(a, row_grid(c, b->n_tokens), c.st));
   return BULLET_OK;
 }
 
