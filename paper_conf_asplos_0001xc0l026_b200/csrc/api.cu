@@ -230,7 +230,7 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   if (rc) return rc;
   if (h->cfg.dtype == BULLET_DTYPE_FP32) {
     if (K % 16) return set_err(BULLET_EUNSUPPORTED, "fp32 GEMM needs K %% 16 == 0");
-    a.bn = 64; a.mh = 1; a.splits = 1; a.n_full = 0;
+    a.bn = 64; a.mh = 1; a.splits = 1; a.n_full = 0; a.band = 1;
     LAUNCH(c, launch_gemm_simt<float>((const float*)A, (const float*)B, a, h->n_sms * 4, c.st));
     return BULLET_OK;
   }
@@ -295,6 +295,13 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
     fprintf(stderr, "gemm M=%d N=%d K=%d m_sms=%d -> mh=%d bn=%d n_full=%d ts=%d\n", M, N, K, c.m_sms, mh, bn,
             n_full, ts);
   a.bn = bn; a.mh = mh; a.splits = ts; a.n_full = n_full;
+  {  // rasterisation band: activations of a band <= 32 MB (L2-resident)
+    const int m_tiles = (M + 128 * mh - 1) / (128 * mh);
+    const double a_tile = 128.0 * mh * K * 2;
+    int band = 1;
+    while (band * 2 <= m_tiles && band * 2 * a_tile <= 32e6) band *= 2;
+    a.band = std::max(1, std::min(band, m_tiles));
+  }
   a.b_packed = Bp;
   a.b_rows = N + (epi == EPI_SILU ? silu_half - N / 2 : 0);
   a.partials = h->ph[c.phase].partials;

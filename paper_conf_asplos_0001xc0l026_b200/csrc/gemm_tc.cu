@@ -30,6 +30,18 @@ namespace {
 constexpr int BM = 128, BK = 64, NT = 256;
 constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB per 128-row half
 
+// Tile order: bands of `band` M tiles; inside a band the M tile varies
+// fastest, then N.  A band's activations (<= ~32 MB) stay L2-resident while
+// every weight tile streams past them once per band, instead of the whole
+// activation block being re-read from DRAM for every N tile.
+__device__ __forceinline__ void tile_coords(int tile, int m_tiles, int n_tiles, int band, int& m_blk,
+                                            int& n_blk) {
+  const int per_band = band * n_tiles;            // tiles in a full band
+  const int b = tile / per_band, r = tile % per_band;
+  const int rows = min(band, m_tiles - b * band);  // the last band may be short
+  m_blk = b * band + r % rows;
+  n_blk = r / rows;
+}
 struct UnitInfo {
   int tile, sp, ns, tail;   // tail: index among split units (partials slot), -1 for whole tiles
 };
@@ -213,7 +225,8 @@ __global__ void __launch_bounds__(NT, 1)
         if (u < 0) break;
         log_unit(a.L, u);
         const UnitInfo ui = unit_info(a, u);
-        const int m_blk = ui.tile % m_tiles, n_blk = ui.tile / m_tiles;
+        int m_blk, n_blk;
+        tile_coords(ui.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
         const int kb0 = ui.sp * k_blocks / ui.ns, kb1 = (ui.sp + 1) * k_blocks / ui.ns;
         int r0, r1;
         if (a.epi == EPI_SILU) { r0 = n_blk * (bn / 2); r1 = a.silu_half + r0; }
@@ -291,7 +304,8 @@ __global__ void __launch_bounds__(NT, 1)
       if (lane == 0) mbar_arrive(tqe + slot);
       if (u < 0) break;
       const UnitInfo ui = unit_info(a, u);
-      const int m_blk = ui.tile % m_tiles, n_blk = ui.tile / m_tiles;
+      int m_blk, n_blk;
+      tile_coords(ui.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
       const int col0 = (a.epi == EPI_SILU) ? n_blk * (bn / 2) : n_blk * bn;
       const int out_chunks = (a.epi == EPI_SILU) ? bn / 64 : bn / 32;
       mbar_wait(accf + as, aph);

@@ -13,6 +13,7 @@ struct GemmArgs {
   int mh;             // tcgen05: 128-row halves per unit (1, or 2 = 256 rows sharing each B stage)
   int n_full;         // tcgen05: units [0, n_full) are whole tiles over all of K ...
   int splits;         // ... the remaining tiles are split `splits` ways over K (tail split)
+  int band;           // tcgen05: M tiles per rasterisation band (see tile_coords)
   int epi;
   int silu_half;      // row offset of the "up" rows in B (EPI_SILU)
   const void* bias;   // [N] of the element type, or null (EPI_F32)

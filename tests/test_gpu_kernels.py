@@ -51,6 +51,7 @@ def _int_operands(rng, M, K, N):
     (4096, 6144, 4096, 0, None),    # prefill-sized: bn 256
     (257, 4096, 4096, 10, 50),      # 40-SM gated range: mh=2 units, tail split
     (64, 1280, 8192, 0, 16),        # 16 SMs, K = 8192
+    (1700, 1024, 16384, 0, None),   # rasterisation bands of 4 M tiles, short last band
 ])
 @pytest.mark.parametrize("packed", [False, True])
 def test_gemm_f32_epilogue_bit_exact(B, M, N, K, lo, hi, packed):
