@@ -217,6 +217,21 @@ int next_launch(Ctx& c, Launch* L) {
   return BULLET_OK;
 }
 
+// Grid of the one-CTA-per-SM persistent kernels.  CTAs that land on the
+// other phase's SMs (free for a moment between its kernels) exit at once;
+// with exactly one CTA per SM each such CTA would leave an SM of this phase
+// without a worker for the whole kernel.  Spare CTAs (BULLET_GRID_MULT > 1)
+// would take their place; measured: no gain (co-run 3.01-3.03 ms at x1 vs
+// 3.09-3.24 at x2/x3, config 2), so the default is one CTA per SM.
+int persist_grid(const Ctx& c, int per_sm) {
+  static const int mult = [] {
+    const char* e = getenv("BULLET_GRID_MULT");
+    const int v = e ? atoi(e) : 1;
+    return v >= 1 && v <= 8 ? v : 1;
+  }();
+  return c.h->n_sms * per_sm * (c.m_sms < c.h->n_sms ? mult : 1);
+}
+
 int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, int silu_half,
             const void* bias, const float* resid, void* out, int ldo, const uint8_t* Bp = nullptr) {
   bullet_handle* h = c.h;
@@ -309,7 +324,7 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   CUtensorMap ma, mb;
   if ((rc = make_map(&ma, A, M, K, 128))) return rc;   // one 128-row half per TMA box
   if ((rc = make_map(&mb, B, N, K, bn / 2))) return rc;
-  LAUNCH(c, launch_gemm_tc(ma, mb, a, h->n_sms, c.st));
+  LAUNCH(c, launch_gemm_tc(ma, mb, a, persist_grid(c, 1), c.st));
   return BULLET_OK;
 }
 
@@ -383,7 +398,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
       return set_err(BULLET_EUNSUPPORTED, "tensor-core decode attention: bf16, hd 128 only");
     int rc = next_launch(c, &a.L);
     if (rc) return rc;
-    LAUNCH(c, launch_attn_decode_tc(a, h->n_sms, c.st));
+    LAUNCH(c, launch_attn_decode_tc(a, persist_grid(c, 1), c.st));
     return BULLET_OK;
   }
   if (kind == 2 || kind == 4) {
@@ -397,8 +412,8 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     }
     int rc = next_launch(c, &a.L);
     if (rc) return rc;
-    if (kind == 4) LAUNCH(c, launch_attn_prefill5(a, h->n_sms * 2, c.st));
-    else LAUNCH(c, launch_attn_prefill_tc(a, h->n_sms * 2, c.st));
+    if (kind == 4) LAUNCH(c, launch_attn_prefill5(a, persist_grid(c, 2), c.st));
+    else LAUNCH(c, launch_attn_prefill_tc(a, persist_grid(c, 2), c.st));
     return BULLET_OK;
   }
   int rc = next_launch(c, &a.L);
