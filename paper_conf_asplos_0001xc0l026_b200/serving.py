@@ -1,0 +1,257 @@
+"""Multi-step serving loop over bullet_step.
+
+PAPER.md §3.3: every scheduling cycle the prefill batch
+advances by a group of layers while the decode batch advances by k layer
+steps on the other SMs; Alg. 1 re-decides (prefill SM count, k) each cycle
+from the live request state (readings R-14..R-19); a request
+that finishes prefill joins the decode batch copy-free (its KV blocks and
+block-table row are kept).  Requests arrive by a seeded Poisson
+process with ShareGPT-like prompt and output lengths (synthetic: the paper's
+traces are out of scope).
+
+This module is host orchestration only: request bookkeeping, a paged-block
+allocator, the cycle state machine and the SLO metrics (TTFT, normalized
+TTFT, TPOT, goodput).  All compute happens in the injected `step` callable —
+on the GPU that is one bullet_step (scripts/serve.py); tests drive the same
+loop with the host-only performance model.  Time is virtual: the clock
+advances by each cycle's measured (or predicted) device time, so different
+policies see the same arrival process.
+
+Policies:
+  bullet      co-run, (p, k) from Alg. 1 (bullet_choose_split)
+  timesliced  same cycle structure, both phases on all SMs one after the
+              other (BULLET_TIMESLICED), k from the model's full-GPU balance
+  prefill_first  vLLM-style: while a prefill batch exists decode is paused
+              (p = N); otherwise decode runs whole iterations on all SMs
+"""
+from __future__ import annotations
+
+import math
+from dataclasses import dataclass, field
+
+import numpy as np
+
+
+@dataclass
+class Request:
+    rid: int
+    arrival_ms: float
+    prompt: int
+    out_len: int                      # tokens to generate (first one comes from prefill)
+    blocks: list = field(default_factory=list)
+    first_token_ms: float | None = None
+    finish_ms: float | None = None
+    tokens: int = 0                   # tokens generated so far
+
+    @property
+    def ctx(self) -> int:
+        """Cached positions before the token being decoded now."""
+        return self.prompt + self.tokens - 1
+
+
+def poisson_trace(rate_per_s: float, duration_s: float, seed: int = 0, prompt_mu=math.log(400),
+                  prompt_sigma=0.8, prompt_clip=(32, 2048), out_mu=math.log(128), out_sigma=0.7,
+                  out_clip=(8, 512)) -> list[Request]:
+    """Seeded Poisson arrivals; prompt / output lengths lognormal, clipped
+    (ShareGPT-like shapes)."""
+    rng = np.random.default_rng(seed)
+    t, reqs = 0.0, []
+    while True:
+        t += rng.exponential(1000.0 / rate_per_s)
+        if t > duration_s * 1000.0:
+            return reqs
+        p = int(np.clip(round(rng.lognormal(prompt_mu, prompt_sigma)), *prompt_clip))
+        o = int(np.clip(round(rng.lognormal(out_mu, out_sigma)), *out_clip))
+        reqs.append(Request(len(reqs), t, p, o))
+
+
+class BlockAllocator:
+    """Free list of KV blocks (block ids index every layer's pool alike)."""
+
+    def __init__(self, n_blocks: int, block_size: int = 16):
+        self.free = list(range(n_blocks - 1, -1, -1))
+        self.n_blocks, self.block_size = n_blocks, block_size
+
+    def alloc(self, n_tokens: int):
+        n = -(-n_tokens // self.block_size)
+        if n > len(self.free):
+            return None
+        return [self.free.pop() for _ in range(n)]
+
+    def release(self, blocks):
+        self.free.extend(reversed(blocks))
+
+
+@dataclass
+class PhaseWork:
+    """What one phase runs this cycle (consumed by the step callable)."""
+    reqs: list
+    q_lens: list
+    ctx_lens: list
+    layer_begin: int
+    layer_end: int
+    batch_id: int                     # changes when the batch membership changes
+
+
+@dataclass
+class Slo:
+    ttft_norm_ms_per_tok: float = 3.0  # Table 2 ShareGPT row
+    tpot_ms: float = 150.0
+    w_max: int = 4
+    v_min: int = 16
+    percentile: float = 0.9
+
+    def as_dict(self):
+        return dict(ttft_norm_ms_per_tok=self.ttft_norm_ms_per_tok, tpot_ms=self.tpot_ms,
+                    w_max=self.w_max, v_min=self.v_min, percentile=self.percentile)
+
+
+class ServingLoop:
+    """step(prefill: PhaseWork|None, decode: PhaseWork|None, p, flags_mode) -> device ms;
+    choose(state dict, slo dict) -> (p, k)  [Alg. 1, used by the bullet policy];
+    k_full: decode layer-steps per cycle for the time-sliced policy."""
+
+    def __init__(self, n_layers: int, n_sms: int, step, choose, policy: str, allocator: BlockAllocator,
+                 slo: Slo = Slo(), prefill_layers_per_cycle: int = 1, max_prefill_tokens: int = 8192,
+                 max_decodes: int = 256, k_full: int = 4):
+        assert policy in ("bullet", "timesliced", "prefill_first")
+        self.L, self.N = n_layers, n_sms
+        self.step, self.choose, self.policy = step, choose, policy
+        self.alloc, self.slo = allocator, slo
+        self.lp = prefill_layers_per_cycle
+        self.max_prefill_tokens, self.max_decodes, self.k_full = max_prefill_tokens, max_decodes, k_full
+        self.split = (n_sms // 2, n_sms - n_sms // 2)
+        self.log = []                 # per cycle: (now, p, k, prefill tokens, decodes, ms)
+
+    # ------------------------------------------------------------ helpers
+    def _alg1_state(self, now, prefill, layers_done, pending, members):
+        return dict(layers_done=layers_done if prefill else 0, total_layers=self.L,
+                    prefill_lens=[r.prompt for r in prefill] if prefill else [],
+                    prefill_waited_ms=[now - r.arrival_ms for r in prefill] if prefill else [],
+                    pending_lens=[r.prompt for r in pending],
+                    pending_waited_ms=[now - r.arrival_ms for r in pending],
+                    decode_tokens=[r.tokens for r in members],
+                    decode_elapsed_ms=[now - r.first_token_ms for r in members],
+                    decode_mean_ctx=float(np.mean([r.ctx for r in members])) if members else 0.0,
+                    u_k=self.split[0], v_k=self.split[1])
+
+    # ------------------------------------------------------------ loop
+    def run(self, trace: list[Request], horizon_ms: float | None = None, max_cycles: int = 10 ** 7):
+        trace = sorted(trace, key=lambda r: r.arrival_ms)
+        horizon = horizon_ms if horizon_ms is not None else float("inf")
+        now, nxt = 0.0, 0
+        pending, ready, members = [], [], []
+        prefill, layers_done, pre_id, dec_id = None, 0, 0, 0
+        d_layer = 0                   # next decode layer of the current iteration
+        done = []
+        for _ in range(max_cycles):
+            while nxt < len(trace) and trace[nxt].arrival_ms <= now:
+                pending.append(trace[nxt]); nxt += 1
+            # new prefill batch (FCFS while tokens and KV blocks last)
+            if prefill is None and pending:
+                batch, toks = [], 0
+                while pending and toks + pending[0].prompt <= self.max_prefill_tokens:
+                    r = pending[0]
+                    blk = self.alloc.alloc(r.prompt + r.out_len)
+                    if blk is None:
+                        break
+                    r.blocks = blk
+                    batch.append(pending.pop(0)); toks += r.prompt
+                if batch:
+                    prefill, layers_done, pre_id = batch, 0, pre_id + 1
+            # decode membership changes only between iterations
+            if d_layer == 0:
+                room = self.max_decodes - len(members)
+                members += ready[:room]
+                del ready[:room]
+                dec_id += 1
+            if prefill is None and not members:
+                if nxt >= len(trace) and not pending and not ready:
+                    break
+                if nxt < len(trace):           # idle until the next arrival
+                    now = max(now, trace[nxt].arrival_ms)
+                    continue
+            if now >= horizon:
+                break
+            # ---- split decision
+            if self.policy == "bullet":
+                if prefill and members:
+                    p, k = self.choose(self._alg1_state(now, prefill, layers_done, pending, members),
+                                       self.slo.as_dict())
+                elif prefill:
+                    p, k = self.N, 0
+                else:
+                    p, k = 0, self.k_full
+                mode = "corun"
+            elif self.policy == "timesliced":
+                p, k, mode = self.N, (self.k_full if members else 0), "timesliced"
+            else:  # prefill_first
+                p, k, mode = (self.N, 0, "corun") if prefill else (0, self.L, "corun")
+            if p >= self.N:
+                k = 0 if mode == "corun" else k   # decode paused
+            if not members:
+                k = 0
+            pw = None
+            if prefill and (p > 0 or mode == "timesliced"):
+                le = min(layers_done + self.lp, self.L)
+                pw = PhaseWork(prefill, [r.prompt for r in prefill], [0] * len(prefill), layers_done, le, pre_id)
+            dw = None
+            if k > 0:
+                de = min(d_layer + k, self.L)
+                dw = PhaseWork(members, [1] * len(members), [r.ctx for r in members], d_layer, de, dec_id)
+            if pw is None and dw is None:     # e.g. p = 0 chosen while decode is empty
+                p, k = self.N, 0
+                le = min(layers_done + self.lp, self.L)
+                pw = PhaseWork(prefill, [r.prompt for r in prefill], [0] * len(prefill), layers_done, le, pre_id)
+            if mode == "corun" and pw is None:
+                p = 0
+            self.split = (p, self.N - p)
+            ms = self.step(pw, dw, p, mode)
+            self.log.append((now, p, k, sum(pw.q_lens) if pw else 0, len(members) if dw else 0, ms))
+            now += ms
+            # ---- advance the prefill batch
+            if pw is not None:
+                layers_done = pw.layer_end
+                if layers_done >= self.L:
+                    for r in prefill:
+                        r.first_token_ms, r.tokens = now, 1
+                        if r.out_len <= 1:
+                            r.finish_ms = now
+                            self.alloc.release(r.blocks)
+                            done.append(r)
+                        else:
+                            ready.append(r)
+                    prefill, layers_done = None, 0
+            # ---- advance the decode iteration
+            if dw is not None:
+                d_layer = dw.layer_end
+                if d_layer >= self.L:
+                    d_layer = 0
+                    still = []
+                    for r in members:
+                        r.tokens += 1
+                        if r.tokens >= r.out_len:
+                            r.finish_ms = now
+                            self.alloc.release(r.blocks)
+                            done.append(r)
+                        else:
+                            still.append(r)
+                    members = still
+        return self.metrics(done, trace, now)
+
+    def metrics(self, done, trace, now):
+        s = self.slo
+        ttft = np.array([r.first_token_ms - r.arrival_ms for r in done]) if done else np.zeros(0)
+        nttft = np.array([(r.first_token_ms - r.arrival_ms) / r.prompt for r in done]) if done else np.zeros(0)
+        tpot = np.array([(r.finish_ms - r.first_token_ms) / (r.out_len - 1) for r in done if r.out_len > 1])
+        ok = [((r.first_token_ms - r.arrival_ms) / r.prompt <= s.ttft_norm_ms_per_tok and
+               (r.out_len <= 1 or (r.finish_ms - r.first_token_ms) / (r.out_len - 1) <= s.tpot_ms))
+              for r in done]
+        pct = lambda a, q: float(np.percentile(a, q)) if len(a) else None  # noqa: E731
+        dur_s = max(now, 1e-9) / 1000.0
+        return {"policy": self.policy, "requests": len(trace), "finished": len(done), "sim_ms": now,
+                "cycles": len(self.log), "slo_attainment": float(np.mean(ok)) if ok else 0.0,
+                "goodput_req_s": sum(ok) / dur_s, "throughput_tok_s": sum(r.prompt + r.out_len for r in done) / dur_s,
+                "ttft_ms_p50": pct(ttft, 50), "ttft_ms_p90": pct(ttft, 90),
+                "norm_ttft_ms_per_tok_p90": pct(nttft, 90), "tpot_ms_p50": pct(tpot, 50),
+                "tpot_ms_p90": pct(tpot, 90), "slo": s.as_dict()}
