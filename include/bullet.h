@@ -59,7 +59,9 @@ enum {
   BULLET_TIMESLICED = 1,     /* same kernels on all SMs, prefill then decode (baseline) */
   BULLET_UNGATED = 2,        /* both phases concurrently on all SMs ("Naive") */
   BULLET_SMID_LOG = 4,       /* record (launch, tile, smid) of every work unit */
-  BULLET_PROFILE = 8         /* CUDA events around every kernel (bullet_profile_read) */
+  BULLET_PROFILE = 8,        /* CUDA events around every kernel (bullet_profile_read) */
+  BULLET_UNFUSED = 16        /* run S3 (RoPE + KV append) as its own kernel instead of the
+                                QKV GEMM epilogue (bf16, head_dim 128); A/B tests only */
 };
 
 /* Kernel kinds reported by bullet_profile_read. */
@@ -283,8 +285,10 @@ int bullet_op_rope_kv(bullet_handle *h, const bullet_batch *batch, int layer, co
 /* Attention for `batch` rows reading K/V of `layer` through the block
  * table: q [n_tokens][H*hd] in, o [n_tokens][H*hd] out (dtype).
  * kind 0: automatic (what bullet_step uses), 1: SIMT kernel, 2: mma.sync
- * prefill kernel, 3: tensor-core decode kernel, 4: tcgen05 prefill kernel
- * (2-4: bf16, head_dim 128). */
+ * prefill kernel, 3: tensor-core decode kernel (cp.async staging), 4: tcgen05
+ * prefill kernel, 5: register-direct decode kernel (one token per request,
+ * n_tokens <= max_decode_tokens; the default for decode batches)
+ * (2-5: bf16, head_dim 128). */
 int bullet_op_attention(bullet_handle *h, const bullet_batch *batch, int layer, const void *d_q,
                         void *d_o, int kind, int lo, int hi, void *stream);
 

@@ -105,10 +105,18 @@ struct PhaseWS {
   int n_counters = 0, next_ctr = 0;
   int2* tiles = nullptr;
   int* n_tiles = nullptr;
+  TokInfo* tok = nullptr;          // per-token (position, KV slot), written by the plan kernel
+  // register-direct decode attention: (token, chunk) list, partial records, tickets
+  int2* dlist = nullptr;
+  int* n_dlist = nullptr;
+  float* dpart = nullptr;
+  int* tickets = nullptr;
+  int cb = 0;                      // KV blocks per chunk of the current step
   int max_tok = 0;
 };
 
 constexpr int GRAN = 2;            // split granularity: one TPC
+constexpr int DEC_UNITS_MAX = 24576;   // decode attention units (token, kv head, chunk) per launch
 constexpr int N_TILE_SEMS = 2048;
 
 }  // namespace
@@ -165,6 +173,7 @@ struct Ctx {  // one phase's launch context within a call
   bool op;     // op-level entry: counter = op_ctr, zeroed before each launch
   bool prof = false;
   int kind = 0, layer = -1;
+  bool fuse_qkv = false;   // S3 in the QKV epilogue (EPI_QKV)
 };
 
 constexpr size_t MAX_PROF = 1 << 16;
@@ -232,8 +241,13 @@ int persist_grid(const Ctx& c, int per_sm) {
   return c.h->n_sms * per_sm * (c.m_sms < c.h->n_sms ? mult : 1);
 }
 
+struct QkvEpi {   // EPI_QKV destinations
+  void* q; void* pk; void* pv;
+};
+
 int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, int silu_half,
-            const void* bias, const float* resid, void* out, int ldo, const uint8_t* Bp = nullptr) {
+            const void* bias, const float* resid, void* out, int ldo, const uint8_t* Bp = nullptr,
+            const QkvEpi* qe = nullptr) {
   bullet_handle* h = c.h;
   if (M == 0) return BULLET_OK;
   GemmArgs a;
@@ -241,6 +255,12 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   a.M = M; a.N = N; a.K = K; a.epi = epi; a.silu_half = silu_half; a.bias = bias;
   a.resid = resid; a.ldo = ldo;
   if (epi == EPI_SILU) a.out_t = out; else a.out_f32 = (float*)out;
+  if (epi == EPI_QKV) {
+    if (!qe || h->cfg.head_dim != 128 || h->cfg.dtype != BULLET_DTYPE_BF16)
+      return set_err(BULLET_EUNSUPPORTED, "EPI_QKV: bf16, head_dim 128 only");
+    a.q_out = qe->q; a.pool_k = qe->pk; a.pool_v = qe->pv; a.cs = h->rope_cs; a.tok = h->ph[c.phase].tok;
+    a.H = h->cfg.n_heads; a.Hkv = h->cfg.n_kv_heads; a.kvB = h->block_size;
+  }
   int rc = next_launch(c, &a.L);
   if (rc) return rc;
   if (h->cfg.dtype == BULLET_DTYPE_FP32) {
@@ -253,6 +273,7 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   // packed B needs 64-row aligned halves: SiLU tiles of >= 128 rows
   auto fits = [&](int bn) {
     if (Bp && epi == EPI_SILU && bn < 128) return false;
+    if (epi == EPI_QKV) return bn % 128 == 0 && N % bn == 0;   // tiles hold whole heads
     return epi == EPI_SILU ? ((N / 2) % (bn / 2) == 0 && N % 2 == 0) : (N % bn == 0);
   };
   // Plan (mh, bn, tail split) on the phase's m SMs.  A tile costs
@@ -297,7 +318,11 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
     }
   }
   if (!bn) return set_err(BULLET_EUNSUPPORTED, "GEMM N=%d not tileable", N);
-  if (const char* ov = getenv("BULLET_GEMM_PLAN")) {   // experiments: "mh,bn,ts"
+  char kenv[32];
+  snprintf(kenv, sizeof kenv, "BULLET_GEMM_PLAN_K%d", c.kind);   // per kernel kind (experiments)
+  const char* ov = getenv(kenv);
+  if (!ov) ov = getenv("BULLET_GEMM_PLAN");
+  if (ov) {   // experiments: "mh,bn,ts"
     int omh = 0, obn = 0, ots = 0;
     if (sscanf(ov, "%d,%d,%d", &omh, &obn, &ots) == 3 && fits(obn) && omh >= 1 && omh <= 2 && ots >= 1) {
       const int tiles = ((M + 128 * omh - 1) / (128 * omh)) * (N / obn), rem = tiles % c.m_sms;
@@ -377,6 +402,25 @@ int max_kv(const bullet_batch* b) {
   return mk;
 }
 
+// KV blocks per decode-attention chunk: about 4 units per warp of the
+// partition (load balance), within the unit capacity of the workspace.
+int decode_cb(const bullet_handle* h, const bullet_batch* b, int m_sms) {
+  long long total = 0;
+  for (int r = 0; r < b->n_reqs; ++r) total += b->h_ctx_lens[r] / h->block_size + 1;
+  const long long hkv = h->cfg.n_kv_heads;
+  const long long target = 4LL * attn_decode2_warps() * std::max(1, m_sms);
+  long long cb = std::max(1LL, (total * hkv + target - 1) / target);
+  if (const char* e = getenv("BULLET_DEC2_CB")) cb = std::max(1, atoi(e));   // tests / experiments
+  while ((total / cb + b->n_reqs + 1) * hkv > DEC_UNITS_MAX) ++cb;
+  return (int)cb;
+}
+
+bool use_decode2(const bullet_handle* h, const bullet_batch* b) {
+  static const int forced = getenv("BULLET_DEC_ATTN") ? atoi(getenv("BULLET_DEC_ATTN")) : 0;
+  return forced == 5 && h->cfg.dtype == BULLET_DTYPE_BF16 && h->cfg.head_dim == 128 && max_qlen(b) == 1 &&
+         h->cfg.n_heads / h->cfg.n_kv_heads <= 8;
+}
+
 int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* o, int kind) {
   bullet_handle* h = c.h;
   if (b->n_tokens == 0) return BULLET_OK;
@@ -390,7 +434,26 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
   static const int dbg = getenv("BULLET_DBG") ? atoi(getenv("BULLET_DBG")) : 0;
   a.dbg = dbg;
   const bool bf16 = h->cfg.dtype == BULLET_DTYPE_BF16;
-  if (kind == 0) kind = (bf16 && a.hd == 128) ? (max_qlen(b) > 1 ? 4 : 3) : 1;
+  if (kind == 0) kind = (bf16 && a.hd == 128) ? (max_qlen(b) > 1 ? 4 : (use_decode2(h, b) ? 5 : 3)) : 1;
+  if (kind == 5) {
+    if (!bf16 || a.hd != 128 || max_qlen(b) != 1 || a.H / a.Hkv > 8)
+      return set_err(BULLET_EUNSUPPORTED, "register-direct decode attention: bf16, hd 128, one token per request");
+    PhaseWS& P = h->ph[c.op ? 1 : c.phase];   // the decode workspace holds the chunk list
+    if (!P.dlist) return set_err(BULLET_EUNSUPPORTED, "decode attention workspace missing");
+    if (c.op) {   // op-level: plan the chunk list now
+      P.cb = decode_cb(h, b, c.m_sms);
+      PlanArgs pa{nullptr, 0, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ, nullptr, nullptr,
+                  nullptr, b->d_ctx_lens, b->d_block_table, b->max_blocks_per_req, h->block_size, b->n_tokens,
+                  P.dlist, P.n_dlist, P.cb};
+      prof_begin(c);
+      LAUNCH(c, launch_plan(pa, c.st));
+    }
+    a.tiles = P.dlist; a.n_tiles = P.n_dlist; a.cb = P.cb; a.part = P.dpart; a.tickets = P.tickets;
+    int rc = next_launch(c, &a.L);
+    if (rc) return rc;
+    LAUNCH(c, launch_attn_decode2(a, persist_grid(c, 1), c.st));
+    return BULLET_OK;
+  }
   if (kind == 3 && max_kv(b) > attn_decode_max_blocks() * h->block_size) kind = c.op ? -1 : 1;
   if (kind == -1) return set_err(BULLET_EUNSUPPORTED, "tensor-core decode attention: context too long");
   if (kind == 3) {
@@ -406,7 +469,8 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     PhaseWS& P = h->ph[c.phase];
     a.tiles = P.tiles; a.n_tiles = P.n_tiles;
     if (c.op) {  // op-level: plan the tile list now
-      PlanArgs pa{nullptr, 0, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ, P.tiles, P.n_tiles};
+      PlanArgs pa{nullptr, 0, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ, P.tiles, P.n_tiles,
+                  nullptr, nullptr, nullptr, 0, 0, 0, nullptr, nullptr, 0};
       prof_begin(c);
       LAUNCH(c, launch_plan(pa, c.st));
     }
@@ -447,10 +511,16 @@ int run_layer(Ctx& c, const bullet_batch* b, int layer) {
   if ((rc = do_rmsnorm(c, b->d_hidden, n, w.g_attn, P.h))) return rc;                       // S1
   c.kind = BULLET_K_QKV;
   const bullet_handle::Packed* wp = h->wp.empty() ? nullptr : &h->wp[layer];
-  if ((rc = do_gemm(c, EPI_F32, P.h, n, d, w.w_qkv, nq, 0, w.b_qkv, nullptr, P.qkv, nq,
-                    wp ? wp->qkv : nullptr))) return rc;  // S2
-  c.kind = BULLET_K_ROPE_KV;
-  if ((rc = do_rope(c, b, layer, P.qkv, P.q))) return rc;                                    // S3
+  if (c.fuse_qkv) {   // S2 + S3: RoPE and the KV append in the QKV epilogue
+    const QkvEpi qe{P.q, h->pk[layer], h->pv[layer]};
+    if ((rc = do_gemm(c, EPI_QKV, P.h, n, d, w.w_qkv, nq, 0, w.b_qkv, nullptr, nullptr, nq,
+                      wp ? wp->qkv : nullptr, &qe))) return rc;
+  } else {
+    if ((rc = do_gemm(c, EPI_F32, P.h, n, d, w.w_qkv, nq, 0, w.b_qkv, nullptr, P.qkv, nq,
+                      wp ? wp->qkv : nullptr))) return rc;  // S2
+    c.kind = BULLET_K_ROPE_KV;
+    if ((rc = do_rope(c, b, layer, P.qkv, P.q))) return rc;                                  // S3
+  }
   c.kind = BULLET_K_ATTN;
   if ((rc = do_attention(c, b, layer, P.q, P.o, 0))) return rc;                             // S4
   // S5: x1 = x + o W_o^T.  Under TP the non-lead ranks write their partial
@@ -514,8 +584,13 @@ int run_phase(Ctx& c, const bullet_batch* b) {
   PhaseWS& P = c.h->ph[c.phase];
   P.next_ctr = 0;
   const bool tc_attn = c.h->cfg.dtype == BULLET_DTYPE_BF16 && c.h->cfg.head_dim == 128 && max_qlen(b) > 1;
+  const bool dec2 = use_decode2(c.h, b);
+  if (dec2) P.cb = decode_cb(c.h, b, c.m_sms);
   PlanArgs pa{P.counters, P.n_counters, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ,
-              tc_attn ? P.tiles : nullptr, P.n_tiles};
+              tc_attn ? P.tiles : nullptr, P.n_tiles,
+              c.fuse_qkv ? P.tok : nullptr, b->d_ctx_lens, b->d_block_table, b->max_blocks_per_req,
+              c.h->block_size, b->n_tokens,
+              dec2 ? P.dlist : nullptr, P.n_dlist, P.cb};
   c.kind = BULLET_K_PLAN;
   c.layer = -1;
   prof_begin(c);
@@ -650,9 +725,17 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
               cudaMalloc(&P.tile_sems, N_TILE_SEMS * sizeof(int)) == cudaSuccess &&
               cudaMalloc(&P.counters, P.n_counters * sizeof(int)) == cudaSuccess &&
               cudaMalloc(&P.tiles, (T / ATTN_TC_BQ + 1024) * sizeof(int2)) == cudaSuccess &&
-              cudaMalloc(&P.n_tiles, sizeof(int)) == cudaSuccess;
+              cudaMalloc(&P.n_tiles, sizeof(int)) == cudaSuccess &&
+              cudaMalloc(&P.tok, T * sizeof(TokInfo)) == cudaSuccess &&
+              cudaMalloc(&P.n_dlist, sizeof(int)) == cudaSuccess &&
+              cudaMalloc(&P.tickets, T * c.n_kv_heads * sizeof(int)) == cudaSuccess;
+    if (ok && p == 1 && c.dtype == BULLET_DTYPE_BF16 && c.head_dim == 128 && c.n_heads / c.n_kv_heads <= 8)
+      ok = cudaMalloc(&P.dlist, (size_t)DEC_UNITS_MAX * sizeof(int2)) == cudaSuccess &&
+           cudaMalloc(&P.dpart, (size_t)DEC_UNITS_MAX * attn_decode2_rec_floats(c.n_heads / c.n_kv_heads) *
+                                     sizeof(float)) == cudaSuccess;
     if (!ok) return fail(set_err(BULLET_ENOMEM, "workspace allocation (phase %d)", p));
     cudaMemset(P.tile_sems, 0, N_TILE_SEMS * sizeof(int));
+    cudaMemset(P.tickets, 0, T * c.n_kv_heads * sizeof(int));
     cudaMemset(P.counters, 0, P.n_counters * sizeof(int));
   }
   if (cudaMalloc(&h->op_ctr, sizeof(int)) != cudaSuccess) return fail(set_err(BULLET_ENOMEM, "op ctr"));
@@ -773,6 +856,8 @@ int bullet_step(bullet_handle* h, const bullet_batch* pre, const bullet_batch* d
          mode == BULLET_CORUN ? p : N, log, sp, false, prof};
   Ctx cd{h, 1, mode == BULLET_CORUN ? gate_of(h, p, N) : gate_of(h, 0, N),
          mode == BULLET_CORUN ? N - p : N, log, sd, false, prof};
+  cp.fuse_qkv = cd.fuse_qkv = !(flags & BULLET_UNFUSED) && h->cfg.dtype == BULLET_DTYPE_BF16 &&
+                              h->cfg.head_dim == 128;
   if (has_pre && (rc = run_phase(cp, pre))) return rc;
   if (run_dec) {
     if (mode == BULLET_TIMESLICED && has_pre) {
@@ -865,7 +950,8 @@ void bullet_destroy(bullet_handle* h) {
     PhaseWS& P = h->ph[p];
     cudaFree(P.qkv); cudaFree(P.q); cudaFree(P.o); cudaFree(P.h); cudaFree(P.act);
     cudaFree(P.partials); cudaFree(P.tile_sems); cudaFree(P.counters); cudaFree(P.tiles);
-    cudaFree(P.n_tiles);
+    cudaFree(P.n_tiles); cudaFree(P.tok);
+    cudaFree(P.dlist); cudaFree(P.n_dlist); cudaFree(P.dpart); cudaFree(P.tickets);
     if (h->comm[p] && g_nccl.commDestroy) g_nccl.commDestroy(h->comm[p]);
   }
   cudaFree(h->rope_cs);
@@ -920,7 +1006,7 @@ int bullet_op_stream(bullet_handle* h, const void* src, size_t bytes, int mode, 
   Ctx c;
   int rc = op_ctx(h, lo, hi, stream, &c);
   if (rc) return rc;
-  if (!src || bytes == 0 || (mode & 0xff) > 2 || mode < 0) return set_err(BULLET_EINVAL, "stream args");
+  if (!src || bytes == 0 || (mode & 0xff) > 4 || mode < 0) return set_err(BULLET_EINVAL, "stream args");
   StreamArgs a;
   memset(&a, 0, sizeof a);
   a.src = (const uint8_t*)src; a.bytes = bytes; a.mode = mode & 0xff; a.param = mode >> 8;
@@ -956,8 +1042,11 @@ int bullet_op_attention(bullet_handle* h, const bullet_batch* b, int layer, cons
   Ctx c;
   int rc = op_ctx(h, lo, hi, stream, &c);
   if (rc) return rc;
-  if (!b || !q || !o || layer < 0 || layer >= h->cfg.n_layers || kind < 0 || kind > 4)
+  if (!b || !q || !o || layer < 0 || layer >= h->cfg.n_layers || kind < 0 || kind > 5)
     return set_err(BULLET_EINVAL, "attention args");
+  if ((kind == 5 || (kind == 0 && use_decode2(h, b))) && b->n_tokens > h->ph[1].max_tok)
+    return set_err(BULLET_ENOMEM, "decode attention: %d tokens > max_decode_tokens %d", b->n_tokens,
+                   h->ph[1].max_tok);
   bullet_batch bb = *b;
   bb.layer_begin = layer; bb.layer_end = layer;
   if ((rc = validate_batch(h, &bb, 0))) return rc;

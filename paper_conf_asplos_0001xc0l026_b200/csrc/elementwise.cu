@@ -197,24 +197,63 @@ __global__ void __launch_bounds__(256) k_gemm_simt(const T* __restrict__ A, cons
 }
 
 // ------------------------------------------------------------------ plan
-// One thread: zero the phase's work counters and list the prefill attention
-// tiles (request, q-tile) longest-key-range first (LPT order).
+// CTA 0, thread 0: zero the phase's work counters and list the prefill
+// attention tiles (request, q-tile) longest-key-range first (LPT order).
+// Every thread (grid-stride over tokens): the token's position and KV slot
+// (request by binary search over cu), consumed by the fused QKV epilogue.
 __global__ void k_plan(PlanArgs a) {
-  for (int i = threadIdx.x; i < a.n_counters; i += blockDim.x) a.counters[i] = 0;
-  if (threadIdx.x == 0 && a.tiles) {
-    int maxt = 0;
-    for (int r = 0; r < a.n_reqs; ++r) {
-      int len = a.cu[r + 1] - a.cu[r];
-      int nt = (len + a.bq - 1) / a.bq;
-      maxt = nt > maxt ? nt : maxt;
-    }
-    int n = 0;
-    for (int t = maxt - 1; t >= 0; --t)
+  if (blockIdx.x == 0) {
+    for (int i = threadIdx.x; i < a.n_counters; i += blockDim.x) a.counters[i] = 0;
+    if (threadIdx.x == 0 && a.tiles) {
+      int maxt = 0;
       for (int r = 0; r < a.n_reqs; ++r) {
         int len = a.cu[r + 1] - a.cu[r];
-        if (t * a.bq < len) a.tiles[n++] = make_int2(r, t);
+        int nt = (len + a.bq - 1) / a.bq;
+        maxt = nt > maxt ? nt : maxt;
       }
-    *a.n_tiles = n;
+      int n = 0;
+      for (int t = maxt - 1; t >= 0; --t)
+        for (int r = 0; r < a.n_reqs; ++r) {
+          int len = a.cu[r + 1] - a.cu[r];
+          if (t * a.bq < len) a.tiles[n++] = make_int2(r, t);
+        }
+      *a.n_tiles = n;
+    }
+    if (a.dlist) {   // decode chunk list: block-wide exclusive scan of chunk counts
+      __shared__ int s_w[8];
+      __shared__ int s_base;
+      if (threadIdx.x == 0) s_base = 0;
+      __syncthreads();
+      const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+      for (int t0 = 0; t0 < a.n_tok; t0 += blockDim.x) {
+        const int t = t0 + threadIdx.x;
+        const int nch = t < a.n_tok ? ((__ldg(a.ctx + t) / a.B + 1) + a.cb - 1) / a.cb : 0;
+        int x = nch;   // inclusive warp scan
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int y = __shfl_up_sync(0xffffffffu, x, o);
+          if (lane >= o) x += y;
+        }
+        if (lane == 31) s_w[w] = x;
+        __syncthreads();
+        int off = s_base;
+        for (int i = 0; i < w; ++i) off += s_w[i];
+        off += x - nch;
+        for (int c = 0; c < nch; ++c) a.dlist[off + c] = make_int2(t, c);
+        __syncthreads();
+        if (threadIdx.x == blockDim.x - 1) s_base = off + nch;
+        __syncthreads();
+      }
+      if (threadIdx.x == 0) *a.n_dlist = s_base;
+    }
+  }
+  if (a.tok) {
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < a.n_tok; t += gridDim.x * blockDim.x) {
+      const int r = find_req(a.cu, a.n_reqs, t);
+      const int pos = __ldg(a.ctx + r) + (t - __ldg(a.cu + r));
+      const int blk = __ldg(a.bt + (size_t)r * a.max_blocks + pos / a.B);
+      a.tok[t] = make_int2(pos, blk * a.B + pos % a.B);
+    }
   }
 }
 
@@ -249,7 +288,9 @@ cudaError_t launch_rope_kv(const RopeArgs& a, int grid, cudaStream_t st) {
   return cudaGetLastError();
 }
 cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st) {
-  k_plan<<<1, 256, 0, st>>>(a);
+  int grid = a.tok ? (a.n_tok + 255) / 256 : 1;
+  grid = grid < 1 ? 1 : grid > 64 ? 64 : grid;
+  k_plan<<<grid, 256, 0, st>>>(a);
   return cudaGetLastError();
 }
 cudaError_t launch_probe(int* out, int n, cudaStream_t st) {

@@ -149,6 +149,54 @@ __device__ __forceinline__ void epi_store(const GemmArgs& a, int m, int col, con
   }
 }
 
+// EPI_QKV for 32 columns [col, col+32) of head col/128 (col % 128 in {0, 32})
+// of token m: v holds those columns, w the partner columns col+64.. of the
+// rotate-half pairs.  Bias, RoPE (q and k heads), bf16 rounding (R2), then
+// q -> q_out, k / v -> pool slot (same arithmetic as k_rope_kv).
+__device__ __forceinline__ void epi_qkv(const GemmArgs& a, int m, int col, float* v, float* w) {
+  const int head = col >> 7, i0 = col & 127;
+  if (a.bias) {
+    const __nv_bfloat16* b = reinterpret_cast<const __nv_bfloat16*>(a.bias);
+#pragma unroll
+    for (int j = 0; j < 32; ++j) { v[j] += __bfloat162float(b[col + j]); w[j] += __bfloat162float(b[col + 64 + j]); }
+  }
+  const TokInfo ti = a.tok[m];
+  __nv_bfloat16* dst;
+  if (head < a.H + a.Hkv) {
+    const float4* cs = reinterpret_cast<const float4*>(a.cs + (size_t)ti.x * 64 + i0);
+#pragma unroll
+    for (int j = 0; j < 16; ++j) {
+      const float4 c = cs[j];   // (cos, sin) of frequencies i0 + 2j, i0 + 2j + 1
+      const float x0 = v[2 * j], x1 = w[2 * j], y0 = v[2 * j + 1], y1 = w[2 * j + 1];
+      v[2 * j] = x0 * c.x - x1 * c.y;
+      w[2 * j] = x1 * c.x + x0 * c.y;
+      v[2 * j + 1] = y0 * c.z - y1 * c.w;
+      w[2 * j + 1] = y1 * c.z + y0 * c.w;
+    }
+    dst = head < a.H ? reinterpret_cast<__nv_bfloat16*>(a.q_out) + ((size_t)m * a.H + head) * 128
+                     : reinterpret_cast<__nv_bfloat16*>(a.pool_k) +
+                           (((size_t)(ti.y / a.kvB) * a.Hkv + (head - a.H)) * a.kvB + ti.y % a.kvB) * 128;
+  } else {
+    dst = reinterpret_cast<__nv_bfloat16*>(a.pool_v) +
+          (((size_t)(ti.y / a.kvB) * a.Hkv + (head - a.H - a.Hkv)) * a.kvB + ti.y % a.kvB) * 128;
+  }
+  uint32_t p[16], q[16];
+#pragma unroll
+  for (int i = 0; i < 16; ++i) {
+    __nv_bfloat162 h = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
+    __nv_bfloat162 g = __floats2bfloat162_rn(w[2 * i], w[2 * i + 1]);
+    p[i] = *reinterpret_cast<uint32_t*>(&h);
+    q[i] = *reinterpret_cast<uint32_t*>(&g);
+  }
+  uint4* d0 = reinterpret_cast<uint4*>(dst + i0);
+  uint4* d1 = reinterpret_cast<uint4*>(dst + 64 + i0);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    d0[i] = make_uint4(p[4 * i], p[4 * i + 1], p[4 * i + 2], p[4 * i + 3]);
+    d1[i] = make_uint4(q[4 * i], q[4 * i + 1], q[4 * i + 2], q[4 * i + 3]);
+  }
+}
+
 }  // namespace
 
 int gemm_tc_stages(int bn, int mh) {
@@ -314,6 +362,15 @@ __global__ void __launch_bounds__(NT, 1)
       if (ui.ns == 1) {
         for (int hh = 0; hh < mh; ++hh) {
           const int m = (m_blk * mh + hh) * BM + et;
+          if (a.epi == EPI_QKV) {   // per head: column chunks (c, c + 2) are rotate-half partners
+            for (int c0 = 0; c0 < bn; c0 += 128)
+              for (int c = 0; c < 64; c += 32) {
+                tmem_ld32(tb + hh * bn + c0 + c, v);
+                tmem_ld32(tb + hh * bn + c0 + 64 + c, w);
+                if (m < a.M) epi_qkv(a, m, col0 + c0 + c, v, w);
+              }
+            continue;
+          }
           for (int c = 0; c < out_chunks; ++c) {
             tmem_ld32(tb + hh * bn + c * 32, v);
             if (a.epi == EPI_SILU) tmem_ld32(tb + hh * bn + bn / 2 + c * 32, w);
@@ -378,6 +435,15 @@ __global__ void __launch_bounds__(NT, 1)
             const int m = (m_blk * mh + hh) * BM + et;
             if (m >= a.M) continue;
             const float4* H = T0 + (size_t)hh * BM * bn / 4;
+            if (a.epi == EPI_QKV) {
+              for (int c0 = 0; c0 < bn; c0 += 128)
+                for (int c = 0; c < 64; c += 32) {
+                  sum32(H + (size_t)((c0 + c) / 4) * BM, v);
+                  sum32(H + (size_t)((c0 + 64 + c) / 4) * BM, w);
+                  epi_qkv(a, m, col0 + c0 + c, v, w);
+                }
+              continue;
+            }
             for (int c = 0; c < out_chunks; ++c) {
               sum32(H + (size_t)(c * 8) * BM, v);
               if (a.epi == EPI_SILU) sum32(H + (size_t)(bn / 8 + c * 8) * BM, w);

@@ -4,7 +4,11 @@
 
 namespace bl {
 
-enum { EPI_F32 = 0, EPI_RESID = 1, EPI_SILU = 2 };
+enum { EPI_F32 = 0, EPI_RESID = 1, EPI_SILU = 2, EPI_QKV = 3 };
+
+// Per-token position and KV slot of a phase's batch (plan kernel, once per
+// step): x = position p = ctx[r] + (t - cu[r]), y = slot = bt[r][p / B] * B + p % B.
+typedef int2 TokInfo;
 
 // C[M x N] = A[M x K] . B[N x K]^T with a fused epilogue (all row-major).
 struct GemmArgs {
@@ -25,6 +29,14 @@ struct GemmArgs {
   int* tile_sems;     // tail split: [tail tiles], zero between launches (self-resetting)
   const uint8_t* b_packed;  // B pre-packed by pack_weight (else B comes through mapB)
   int b_rows;               // rows of B (packed layout stride)
+  // EPI_QKV (bf16, head_dim 128; fuses SURVEY §8a S3 into S2): the epilogue
+  // adds the bias, rotates q / k heads (rotate-half RoPE from the (cos, sin)
+  // table), rounds to bf16 (point R2) and stores q -> q_out[t][H][128],
+  // k / v -> the paged pool slot of token t.  Tiles cover whole heads.
+  void* q_out; void* pool_k; void* pool_v;
+  const float2* cs;         // [max_pos][64] (cos, sin)
+  const TokInfo* tok;       // [M]
+  int H, Hkv, kvB;
   Launch L;
 };
 
@@ -57,6 +69,12 @@ struct AttnArgs {
   const int2* tiles;      // prefill tensor-core kernel: (request, q-tile) list
   const int* n_tiles;     // device count of `tiles`
   int dbg;                // diagnostics (BULLET_DBG env): bit0 = decode consumers skip math
+  // register-direct decode kernel (attn_decode2.cu): `tiles` holds the
+  // (token, chunk) list, chunks of `cb` KV blocks; partial records and
+  // per-(token, kv head) tickets (zero between launches, self-resetting)
+  int cb;
+  float* part;
+  int* tickets;
   Launch L;
 };
 
@@ -69,6 +87,11 @@ struct PlanArgs {
   int* counters; int n_counters;
   const int32_t* cu; int n_reqs; int bq;
   int2* tiles; int* n_tiles;
+  // per-token (position, slot) table (nullable): needs ctx, bt, max_blocks, B
+  TokInfo* tok; const int32_t* ctx; const int32_t* bt; int max_blocks, B, n_tok;
+  // decode chunk list (nullable): (token, chunk) for chunks of cb blocks of
+  // ctx[t] + 1 keys, token order, written to dlist[0, *n_dlist)
+  int2* dlist; int* n_dlist; int cb;
 };
 
 // launchers (return cudaError_t of the launch)
@@ -87,9 +110,12 @@ cudaError_t launch_attn_simt(const AttnArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_attn_prefill_tc(const AttnArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_attn_prefill5(const AttnArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, cudaStream_t st);
+cudaError_t launch_attn_decode2(const AttnArgs& a, int grid, cudaStream_t st);
+int attn_decode2_rec_floats(int grp);
+int attn_decode2_warps();
 size_t attn_decode_smem_bytes();
 int attn_decode_max_blocks();
-cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);
+cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);   // grid sized to n_tok
 cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_probe(int* out_smid, int n, cudaStream_t st);
 

@@ -44,6 +44,51 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
 #pragma unroll
       for (int i = 0; i < 16; ++i) acc ^= v[i].x ^ v[i].y ^ v[i].z ^ v[i].w;
     }
+  } else if (a.mode == 3 || a.mode == 4) {
+    // mode 3: LDG.128 -> registers -> STS.128 into a per-warp smem slot (a
+    // register-staged producer); mode 4: same loads, no STS.  Warps claim
+    // 32 KB (4 x 8 KB) per atomic; `param` = 8 KB loads in flight per warp (1|2).
+    const size_t units = a.bytes / 32768;
+    const int warp = tid >> 5;
+    uint4* slot = reinterpret_cast<uint4*>(sm) + (size_t)warp * 512;   // 8 KB per warp
+    for (;;) {
+      int u = 0;
+      if (lane == 0) u = atomicAdd(a.L.ctr, 1);
+      u = __shfl_sync(0xffffffffu, u, 0);
+      if (u >= (int)units) break;
+      const uint4* p = reinterpret_cast<const uint4*>(a.src + (size_t)u * 32768) + lane;
+      if (a.param == 2) {
+#pragma unroll 1
+        for (int h = 0; h < 4; h += 2) {
+          uint4 v[32];
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = __ldcs(p + (h * 16 + i) * 32);
+          if (a.mode == 3) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i) slot[(i & 15) * 32 + lane] = v[i];
+          } else {
+#pragma unroll
+            for (int i = 0; i < 32; ++i) acc ^= v[i].x ^ v[i].w;
+          }
+        }
+      } else {
+#pragma unroll 1
+        for (int h = 0; h < 4; ++h) {
+          uint4 v[16];
+#pragma unroll
+          for (int i = 0; i < 16; ++i) v[i] = __ldcs(p + (h * 16 + i) * 32);
+          if (a.mode == 3) {
+#pragma unroll
+            for (int i = 0; i < 16; ++i) slot[i * 32 + lane] = v[i];
+          } else {
+#pragma unroll
+            for (int i = 0; i < 16; ++i) acc ^= v[i].x ^ v[i].w;
+          }
+        }
+      }
+      __syncwarp();
+      if (a.mode == 3) acc ^= reinterpret_cast<const uint32_t*>(slot)[lane];
+    }
   } else if (a.mode == 1) {
     const size_t units = a.bytes / BULK;
     if (tid == 0) {
@@ -103,7 +148,7 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
 }
 
 cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st) {
-  const int smem = a.mode == 1 ? NB * BULK : (a.mode == 2 ? 3 * 65536 : 0);
+  const int smem = a.mode == 1 ? NB * BULK : (a.mode == 2 ? 3 * 65536 : (a.mode == 3 ? 16 * 8192 : 0));
   cudaError_t e = cudaFuncSetAttribute(k_stream, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return e;
   k_stream<<<grid, 512, smem, st>>>(a);

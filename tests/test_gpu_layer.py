@@ -155,3 +155,34 @@ def test_decode_pause_and_errors(small_bf16):
     with pytest.raises(B.BulletError) as e:
         S.bl.step(None, dec_bad, 0, B.CORUN)
     assert e.value.code == -5
+
+
+@pytest.mark.parametrize("bias", [0, 1])
+@pytest.mark.parametrize("p", [40, 0])
+def test_fused_qkv_rope_matches_unfused(p, bias):
+    """S3 (RoPE + paged KV append) in the QKV GEMM epilogue (EPI_QKV) against
+    the separate k_rope_kv kernel (BULLET_UNFUSED): same q, same pool
+    contents (the only difference allowed is FMA contraction: <= 1 bf16 ulp),
+    and both layer outputs meet the oracle bar."""
+    m = synth.ModelShape("small-bias", 1024, 8, 2, 128, 2816, 1, qkv_bias=bias, rope_theta=1e6,
+                         rope_llama3=0)
+    S = Setup(m, [300, 77, 1, 129], [64, 1, 500, 31, 16], n_layers=1)
+    ref = S.oracle()
+    res = []
+    mode = S.B.CORUN if p else S.B.TIMESLICED   # p = 0: both phases on all SMs
+    p = p or S.bl.n_sms
+    for flags in (mode | S.B.UNFUSED, mode):
+        for k, v in S.pool_gpu:   # same starting pools
+            k.zero_(); v.zero_()
+        for (k, v), (kc, vc) in zip(S.pool_gpu, S.pool_cpu):
+            k.copy_(kc.to(k.dtype)); v.copy_(vc.to(v.dtype))
+        pre, dec = _run(S, p, flags)
+        for name, b in (("pre", pre), ("dec", dec)):
+            mx, mr = compare(b.hidden.cpu().numpy(), ref[name])
+            assert mx <= 2e-2 and mr <= 1e-3, (flags, name, mx, mr)
+        res.append((pre.hidden.clone(), dec.hidden.clone(), S.pool_gpu[0][0].clone(), S.pool_gpu[0][1].clone()))
+    (a_pre, a_dec, a_k, a_v), (b_pre, b_dec, b_k, b_v) = res
+    assert torch.equal(a_v, b_v)   # v: bias + bf16 round only, no rotation
+    dk = (a_k.float() - b_k.float()).abs()
+    assert float((dk / b_k.float().abs().clamp_min(1e-30)).max()) <= 2 ** -7
+    assert float((a_pre - b_pre).abs().max()) <= 2e-2 and float((a_dec - b_dec).abs().max()) <= 2e-2
