@@ -368,7 +368,14 @@ def main():
     slo = {"ttft_norm_ms_per_tok": 3.0, "tpot_ms": 150.0, "w_max": 4, "v_min": 16, "percentile": 0.9}
     model_split = S.bl.choose_split(state, slo)
     S.dec.layer_end = k
-    # ---- co-run (the method) and time-sliced, device-timed, max over ranks
+    # ---- co-run (the method) and time-sliced, device-timed, max over ranks.
+    # The time-sliced baseline is timed right before AND right after the
+    # co-run region (K steps each) and averaged, so a power / clock drift
+    # during the run (the co-run step sits at sw_power_cap) biases neither.
+    for _ in range(args.warmup):
+        S.enqueue(N, B.TIMESLICED)
+    barrier(ws)
+    t_ts0 = allreduce_max(S.time_steps(args.steps, N, B.TIMESLICED), ws)
     for _ in range(args.warmup):
         S.enqueue(p, B.CORUN)
     barrier(ws)
@@ -379,10 +386,9 @@ def main():
     launches = S.bl.launch_count() - l0
     barrier(ws)
     t_co = allreduce_max(t_co, ws)
-    for _ in range(args.warmup):
-        S.enqueue(N, B.TIMESLICED)
     barrier(ws)
-    t_ts = allreduce_max(S.time_steps(args.steps, N, B.TIMESLICED), ws)
+    t_ts1 = allreduce_max(S.time_steps(args.steps, N, B.TIMESLICED), ws)
+    t_ts = 0.5 * (t_ts0 + t_ts1)
     # the paper's "Naive": both phases on all SMs at once, no gating
     for _ in range(args.warmup):
         S.enqueue(p, B.UNGATED)
@@ -480,7 +486,9 @@ def main():
                    "parallelism": (f"tp{S.tp}" if S.tp > 1 else (f"replicas x{ws}" if ws > 1 else "single GPU")),
                    "tokens_per_s_per_gpu": value / ws,
                    "l2": "inputs larger than L2 (weights + KV per step >> 126 MB)"},
-        "timesliced": {"value": ts_value, "ms_per_step": t_ts},
+        "timesliced": {"value": ts_value, "ms_per_step": t_ts, "ms_per_step_before": t_ts0,
+                       "ms_per_step_after": t_ts1,
+                       "note": "same batch, same kernels on all SMs, prefill then decode; timed before and after the co-run region"},
         "corun_speedup_vs_timesliced": t_ts / t_co,
         "ungated": {"value": groups * tok / (t_ung * 1e-3), "ms_per_step": t_ung,
                     "note": "both phases on all SMs concurrently (the paper's Naive, P:L304)"},
@@ -504,6 +512,8 @@ def main():
             "decode_hbm_gbs": b_dec / (t_co * 1e-3) / 1e9},
         "roofline": {"bound": bound, "kernel": dom_name,
                      "achieved": achieved, "peak": peak, "unit": unit, "frac": achieved / peak,
+                     "sms": p if dom[1] == 0 else N - p,
+                     "frac_of_partition": achieved / (peak * (p if dom[1] == 0 else N - p) / N),
                      "peak_source": src, "avg_launch_ms": avg_ms, "traffic": traffic,
                      "algorithmic_" + ("flops" if bound == "tensor" else "bytes"): work},
         "kernel_ms": {f"{k_}/{'pre' if ph == 0 else 'dec'}": round(sum(v) / 2, 4) for (k_, ph), v in by.items()},

@@ -285,10 +285,8 @@ int bullet_op_rope_kv(bullet_handle *h, const bullet_batch *batch, int layer, co
 /* Attention for `batch` rows reading K/V of `layer` through the block
  * table: q [n_tokens][H*hd] in, o [n_tokens][H*hd] out (dtype).
  * kind 0: automatic (what bullet_step uses), 1: SIMT kernel, 2: mma.sync
- * prefill kernel, 3: tensor-core decode kernel (cp.async staging), 4: tcgen05
- * prefill kernel, 5: register-direct decode kernel (one token per request,
- * n_tokens <= max_decode_tokens; the default for decode batches)
- * (2-5: bf16, head_dim 128). */
+ * prefill kernel, 3: tensor-core decode kernel, 4: tcgen05 prefill kernel
+ * (2-4: bf16, head_dim 128). */
 int bullet_op_attention(bullet_handle *h, const bullet_batch *batch, int layer, const void *d_q,
                         void *d_o, int kind, int lo, int hi, void *stream);
 

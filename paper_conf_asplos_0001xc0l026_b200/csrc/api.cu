@@ -106,17 +106,10 @@ struct PhaseWS {
   int2* tiles = nullptr;
   int* n_tiles = nullptr;
   TokInfo* tok = nullptr;          // per-token (position, KV slot), written by the plan kernel
-  // register-direct decode attention: (token, chunk) list, partial records, tickets
-  int2* dlist = nullptr;
-  int* n_dlist = nullptr;
-  float* dpart = nullptr;
-  int* tickets = nullptr;
-  int cb = 0;                      // KV blocks per chunk of the current step
   int max_tok = 0;
 };
 
 constexpr int GRAN = 2;            // split granularity: one TPC
-constexpr int DEC_UNITS_MAX = 24576;   // decode attention units (token, kv head, chunk) per launch
 constexpr int N_TILE_SEMS = 2048;
 
 }  // namespace
@@ -402,25 +395,6 @@ int max_kv(const bullet_batch* b) {
   return mk;
 }
 
-// KV blocks per decode-attention chunk: about 4 units per warp of the
-// partition (load balance), within the unit capacity of the workspace.
-int decode_cb(const bullet_handle* h, const bullet_batch* b, int m_sms) {
-  long long total = 0;
-  for (int r = 0; r < b->n_reqs; ++r) total += b->h_ctx_lens[r] / h->block_size + 1;
-  const long long hkv = h->cfg.n_kv_heads;
-  const long long target = 4LL * attn_decode2_warps() * std::max(1, m_sms);
-  long long cb = std::max(1LL, (total * hkv + target - 1) / target);
-  if (const char* e = getenv("BULLET_DEC2_CB")) cb = std::max(1, atoi(e));   // tests / experiments
-  while ((total / cb + b->n_reqs + 1) * hkv > DEC_UNITS_MAX) ++cb;
-  return (int)cb;
-}
-
-bool use_decode2(const bullet_handle* h, const bullet_batch* b) {
-  static const int forced = getenv("BULLET_DEC_ATTN") ? atoi(getenv("BULLET_DEC_ATTN")) : 0;
-  return forced == 5 && h->cfg.dtype == BULLET_DTYPE_BF16 && h->cfg.head_dim == 128 && max_qlen(b) == 1 &&
-         h->cfg.n_heads / h->cfg.n_kv_heads <= 8;
-}
-
 int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* o, int kind) {
   bullet_handle* h = c.h;
   if (b->n_tokens == 0) return BULLET_OK;
@@ -434,26 +408,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
   static const int dbg = getenv("BULLET_DBG") ? atoi(getenv("BULLET_DBG")) : 0;
   a.dbg = dbg;
   const bool bf16 = h->cfg.dtype == BULLET_DTYPE_BF16;
-  if (kind == 0) kind = (bf16 && a.hd == 128) ? (max_qlen(b) > 1 ? 4 : (use_decode2(h, b) ? 5 : 3)) : 1;
-  if (kind == 5) {
-    if (!bf16 || a.hd != 128 || max_qlen(b) != 1 || a.H / a.Hkv > 8)
-      return set_err(BULLET_EUNSUPPORTED, "register-direct decode attention: bf16, hd 128, one token per request");
-    PhaseWS& P = h->ph[c.op ? 1 : c.phase];   // the decode workspace holds the chunk list
-    if (!P.dlist) return set_err(BULLET_EUNSUPPORTED, "decode attention workspace missing");
-    if (c.op) {   // op-level: plan the chunk list now
-      P.cb = decode_cb(h, b, c.m_sms);
-      PlanArgs pa{nullptr, 0, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ, nullptr, nullptr,
-                  nullptr, b->d_ctx_lens, b->d_block_table, b->max_blocks_per_req, h->block_size, b->n_tokens,
-                  P.dlist, P.n_dlist, P.cb};
-      prof_begin(c);
-      LAUNCH(c, launch_plan(pa, c.st));
-    }
-    a.tiles = P.dlist; a.n_tiles = P.n_dlist; a.cb = P.cb; a.part = P.dpart; a.tickets = P.tickets;
-    int rc = next_launch(c, &a.L);
-    if (rc) return rc;
-    LAUNCH(c, launch_attn_decode2(a, persist_grid(c, 1), c.st));
-    return BULLET_OK;
-  }
+  if (kind == 0) kind = (bf16 && a.hd == 128) ? (max_qlen(b) > 1 ? 4 : 3) : 1;
   if (kind == 3 && max_kv(b) > attn_decode_max_blocks() * h->block_size) kind = c.op ? -1 : 1;
   if (kind == -1) return set_err(BULLET_EUNSUPPORTED, "tensor-core decode attention: context too long");
   if (kind == 3) {
@@ -461,7 +416,10 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
       return set_err(BULLET_EUNSUPPORTED, "tensor-core decode attention: bf16, hd 128 only");
     int rc = next_launch(c, &a.L);
     if (rc) return rc;
-    LAUNCH(c, launch_attn_decode_tc(a, persist_grid(c, 1), c.st));
+    // two consumer groups per SM on partitions (per-unit merge over twice the
+    // blocks: 146 -> 133 us on 68 SMs, ShareGPT), one on the full GPU (tail
+    // balance: 96 vs 101 us) — scripts/attn_dec_bench.py, DESIGN.md §5
+    LAUNCH(c, launch_attn_decode_tc(a, persist_grid(c, 1), c.m_sms <= 100 ? 2 : 1, c.st));
     return BULLET_OK;
   }
   if (kind == 2 || kind == 4) {
@@ -470,7 +428,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     a.tiles = P.tiles; a.n_tiles = P.n_tiles;
     if (c.op) {  // op-level: plan the tile list now
       PlanArgs pa{nullptr, 0, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ, P.tiles, P.n_tiles,
-                  nullptr, nullptr, nullptr, 0, 0, 0, nullptr, nullptr, 0};
+                  nullptr, nullptr, nullptr, 0, 0, 0};
       prof_begin(c);
       LAUNCH(c, launch_plan(pa, c.st));
     }
@@ -584,13 +542,10 @@ int run_phase(Ctx& c, const bullet_batch* b) {
   PhaseWS& P = c.h->ph[c.phase];
   P.next_ctr = 0;
   const bool tc_attn = c.h->cfg.dtype == BULLET_DTYPE_BF16 && c.h->cfg.head_dim == 128 && max_qlen(b) > 1;
-  const bool dec2 = use_decode2(c.h, b);
-  if (dec2) P.cb = decode_cb(c.h, b, c.m_sms);
   PlanArgs pa{P.counters, P.n_counters, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ,
               tc_attn ? P.tiles : nullptr, P.n_tiles,
               c.fuse_qkv ? P.tok : nullptr, b->d_ctx_lens, b->d_block_table, b->max_blocks_per_req,
-              c.h->block_size, b->n_tokens,
-              dec2 ? P.dlist : nullptr, P.n_dlist, P.cb};
+              c.h->block_size, b->n_tokens};
   c.kind = BULLET_K_PLAN;
   c.layer = -1;
   prof_begin(c);
@@ -726,16 +681,9 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
               cudaMalloc(&P.counters, P.n_counters * sizeof(int)) == cudaSuccess &&
               cudaMalloc(&P.tiles, (T / ATTN_TC_BQ + 1024) * sizeof(int2)) == cudaSuccess &&
               cudaMalloc(&P.n_tiles, sizeof(int)) == cudaSuccess &&
-              cudaMalloc(&P.tok, T * sizeof(TokInfo)) == cudaSuccess &&
-              cudaMalloc(&P.n_dlist, sizeof(int)) == cudaSuccess &&
-              cudaMalloc(&P.tickets, T * c.n_kv_heads * sizeof(int)) == cudaSuccess;
-    if (ok && p == 1 && c.dtype == BULLET_DTYPE_BF16 && c.head_dim == 128 && c.n_heads / c.n_kv_heads <= 8)
-      ok = cudaMalloc(&P.dlist, (size_t)DEC_UNITS_MAX * sizeof(int2)) == cudaSuccess &&
-           cudaMalloc(&P.dpart, (size_t)DEC_UNITS_MAX * attn_decode2_rec_floats(c.n_heads / c.n_kv_heads) *
-                                     sizeof(float)) == cudaSuccess;
+              cudaMalloc(&P.tok, T * sizeof(TokInfo)) == cudaSuccess;
     if (!ok) return fail(set_err(BULLET_ENOMEM, "workspace allocation (phase %d)", p));
     cudaMemset(P.tile_sems, 0, N_TILE_SEMS * sizeof(int));
-    cudaMemset(P.tickets, 0, T * c.n_kv_heads * sizeof(int));
     cudaMemset(P.counters, 0, P.n_counters * sizeof(int));
   }
   if (cudaMalloc(&h->op_ctr, sizeof(int)) != cudaSuccess) return fail(set_err(BULLET_ENOMEM, "op ctr"));
@@ -951,7 +899,6 @@ void bullet_destroy(bullet_handle* h) {
     cudaFree(P.qkv); cudaFree(P.q); cudaFree(P.o); cudaFree(P.h); cudaFree(P.act);
     cudaFree(P.partials); cudaFree(P.tile_sems); cudaFree(P.counters); cudaFree(P.tiles);
     cudaFree(P.n_tiles); cudaFree(P.tok);
-    cudaFree(P.dlist); cudaFree(P.n_dlist); cudaFree(P.dpart); cudaFree(P.tickets);
     if (h->comm[p] && g_nccl.commDestroy) g_nccl.commDestroy(h->comm[p]);
   }
   cudaFree(h->rope_cs);
@@ -1006,7 +953,7 @@ int bullet_op_stream(bullet_handle* h, const void* src, size_t bytes, int mode, 
   Ctx c;
   int rc = op_ctx(h, lo, hi, stream, &c);
   if (rc) return rc;
-  if (!src || bytes == 0 || (mode & 0xff) > 4 || mode < 0) return set_err(BULLET_EINVAL, "stream args");
+  if (!src || bytes == 0 || (mode & 0xff) > 5 || mode < 0) return set_err(BULLET_EINVAL, "stream args");
   StreamArgs a;
   memset(&a, 0, sizeof a);
   a.src = (const uint8_t*)src; a.bytes = bytes; a.mode = mode & 0xff; a.param = mode >> 8;
@@ -1042,11 +989,8 @@ int bullet_op_attention(bullet_handle* h, const bullet_batch* b, int layer, cons
   Ctx c;
   int rc = op_ctx(h, lo, hi, stream, &c);
   if (rc) return rc;
-  if (!b || !q || !o || layer < 0 || layer >= h->cfg.n_layers || kind < 0 || kind > 5)
+  if (!b || !q || !o || layer < 0 || layer >= h->cfg.n_layers || kind < 0 || kind > 4)
     return set_err(BULLET_EINVAL, "attention args");
-  if ((kind == 5 || (kind == 0 && use_decode2(h, b))) && b->n_tokens > h->ph[1].max_tok)
-    return set_err(BULLET_ENOMEM, "decode attention: %d tokens > max_decode_tokens %d", b->n_tokens,
-                   h->ph[1].max_tok);
   bullet_batch bb = *b;
   bb.layer_begin = layer; bb.layer_end = layer;
   if ((rc = validate_batch(h, &bb, 0))) return rc;

@@ -18,6 +18,8 @@
 // Warps take blocks round-robin with private (max, sum, O^T) states, merged
 // through shared memory at the end of each unit.
 // Unit = (token, kv head); decode tokens are requests.
+#include <stdlib.h>
+
 #include "kernels.h"
 
 namespace bl {
@@ -82,7 +84,12 @@ struct Slot {  // one published unit
 };
 }  // namespace
 
+// NG consumer groups of NCW / NG warps: group gw takes the units it = gw,
+// gw + NG, ... (units alternate between groups), so a unit's blocks are
+// split over fewer warps and the per-unit merge is paid over more blocks.
+template <int NG>
 __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
+  constexpr int GW = NCW / NG;
   if (!gate_ok(a.L.gate)) return;
   extern __shared__ __align__(128) uint8_t smem[];
   uint8_t* stages = smem;                                                      // [NCW][DEPTH][STAGE]
@@ -97,20 +104,23 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
   const int grp = a.H / a.Hkv;
   const int units = a.n_tok * a.Hkv;
   if (threadIdx.x == 0) {
-    for (int i = 0; i < 4; ++i) { mbar_init(uqf + i, 1); mbar_init(uqe + i, NCW); }
+    for (int i = 0; i < 4; ++i) { mbar_init(uqf + i, 1); mbar_init(uqe + i, GW); }
     mbar_fence_init();
   }
   __syncthreads();
 
   if (warp == NCW) {  // ------------------------------------------ claimer
     const __nv_bfloat16* qg = reinterpret_cast<const __nv_bfloat16*>(a.q);
+    int n_end = 0;
     for (int it = 0;; ++it) {
       const int slot = it & 3;
-      // at most 2 units ahead of the consumers (load balance across CTAs)
-      if (lane == 0 && it >= 2) mbar_wait(uqe + ((it - 2) & 3), ((it - 2) >> 2) & 1);
+      // a group holds at most 2 units (current + next, so its warps can
+      // prefetch across the boundary): unit it waits for unit it - 2 NG of
+      // the same group (load balance across CTAs; 4 slots = 2 NG)
+      if (lane == 0 && it >= 2 * NG) mbar_wait(uqe + ((it - 2 * NG) & 3), ((it - 2 * NG) >> 2) & 1);
       __syncwarp();
       int u = 0;
-      if (lane == 0) u = atomicAdd(a.L.ctr, 1);
+      if (lane == 0) u = n_end ? units : atomicAdd(a.L.ctr, 1);
       u = __shfl_sync(0xffffffffu, u, 0);
       if (u >= units) u = -1;
       Slot sl{u, 0, 0, 0};
@@ -135,7 +145,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
           mbar_arrive(uqf + slot);
         }
       }
-      if (u < 0) break;
+      if (u < 0 && ++n_end == NG) break;   // one terminator per group
     }
     return;
   }
@@ -148,7 +158,8 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
   __nv_bfloat16* og = reinterpret_cast<__nv_bfloat16*>(a.o);
   uint8_t* my = stages + warp * DEPTH * STAGE_BYTES;
   const uint32_t my_s = smem_u32(my);
-  auto my_count = [&](int nb) { return nb > warp ? (nb - warp + NCW - 1) / NCW : 0; };
+  const int gw = warp / GW, wl = warp % GW;   // group, index in the group
+  auto my_count = [&](int nb) { return nb > wl ? (nb - wl + GW - 1) / GW : 0; };
   // per-lane swizzled offsets (loop invariant): cp.async destinations and
   // ldmatrix sources for the QK (K, by k-step) and PV (V^T, by m-tile) MMAs
   uint32_t cp_off[8], k_off[8], v_off[8];
@@ -161,7 +172,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
 
   // issue cursor over this warp's block sequence (units in claim order,
   // my blocks warp, warp + 8, ... of each), never beyond unit `limit`
-  int iu = 0, ij = 0, n_issued = 0, n_cons = 0;
+  int iu = gw, ij = 0, n_issued = 0, n_cons = 0;
   int cur_nb = -1, cur_g = 0, cur_u = 0;   // cached slot of unit iu (-1: not read yet)
   auto fill = [&](int limit, int cap) {
     while (n_issued - n_cons < cap && iu <= limit) {
@@ -172,8 +183,8 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
         cur_u = X.u; cur_nb = my_count(X.nb); cur_g = X.u >= 0 ? X.u % a.Hkv : 0;
       }
       if (cur_u < 0) return;
-      if (ij >= cur_nb) { ++iu; ij = 0; cur_nb = -1; continue; }
-      const int blk = btbuf[sl * MAXNB + warp + ij * NCW];
+      if (ij >= cur_nb) { iu += NG; ij = 0; cur_nb = -1; continue; }
+      const int blk = btbuf[sl * MAXNB + wl + ij * GW];
       const uint8_t* ks = reinterpret_cast<const uint8_t*>(pk + ((size_t)blk * a.Hkv + cur_g) * KB * HD) + lane * 16;
       const uint8_t* vs = reinterpret_cast<const uint8_t*>(pv + ((size_t)blk * a.Hkv + cur_g) * KB * HD) + lane * 16;
       uint8_t* dk = my + (n_issued % DEPTH) * STAGE_BYTES;
@@ -188,7 +199,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
     }
   };
 
-  for (int it = 0;; ++it) {
+  for (int it = gw;; it += NG) {
     const int slot = it & 3;
     mbar_wait(uqf + slot, (it >> 2) & 1);
     const Slot S = uq[slot];
@@ -212,11 +223,11 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
 
     const int mine = my_count(S.nb);
     for (int j = 0; j < mine; ++j) {
-      fill(it + 1, DEPTH);
+      fill(it + NG, DEPTH);
       const int pend = n_issued - n_cons;   // groups in flight; the oldest is block j
       if (pend >= 3) cp_async_wait<2>(); else if (pend == 2) cp_async_wait<1>(); else cp_async_wait<0>();
       __syncwarp();
-      const int b = warp + j * NCW;
+      const int b = wl + j * GW;
       const uint32_t kt = my_s + (n_cons % DEPTH) * STAGE_BYTES;
       float s[4] = {0.f, 0.f, 0.f, 0.f}, s2[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
@@ -270,7 +281,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
     }
     // the next unit's first DEPTH-1 blocks fly during the merge; the stage
     // left free holds this warp's merge record
-    fill(it + 1, DEPTH - 1);
+    fill(it + NG, DEPTH - 1);
     // full row sums over the 8 key lanes of each head
 #pragma unroll
     for (int o = 4; o < 32; o <<= 1) {
@@ -291,16 +302,16 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
       rec[HD * 8 + 2 * tq] = m0; rec[HD * 8 + 2 * tq + 1] = m1;
       rec[HD * 8 + 8 + 2 * tq] = l0; rec[HD * 8 + 8 + 2 * tq + 1] = l1;
     }
-    named_bar_sync(1, NCW * 32);
-    const float* recs[NCW];
+    named_bar_sync(1 + gw, GW * 32);
+    const float* recs[GW];
 #pragma unroll
-    for (int w = 0; w < NCW; ++w) recs[w] = reinterpret_cast<const float*>(stages + rec_stage[w] * STAGE_BYTES);
-    for (int e = threadIdx.x; e < grp * HD; e += NCW * 32) {
+    for (int w = 0; w < GW; ++w) recs[w] = reinterpret_cast<const float*>(stages + rec_stage[gw * GW + w] * STAGE_BYTES);
+    for (int e = threadIdx.x - gw * GW * 32; e < grp * HD; e += GW * 32) {
       const int h = e / HD, d = e % HD;
       float M = -INFINITY;
-      for (int w = 0; w < NCW; ++w) M = fmaxf(M, recs[w][HD * 8 + h]);
+      for (int w = 0; w < GW; ++w) M = fmaxf(M, recs[w][HD * 8 + h]);
       float L = 0.f, O = 0.f;
-      for (int w = 0; w < NCW; ++w) {
+      for (int w = 0; w < GW; ++w) {
         const float* rw = recs[w];
         const float mw = rw[HD * 8 + h];
         if (mw == -INFINITY) continue;
@@ -310,7 +321,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
       }
       og[(size_t)S.t * a.H * HD + (size_t)(g * grp + h) * HD + d] = __float2bfloat16_rn(O / L);
     }
-    named_bar_sync(1, NCW * 32);
+    named_bar_sync(1 + gw, GW * 32);
     if (lane == 0) mbar_arrive(uqe + slot);
   }
   cp_async_wait<0>();
@@ -322,15 +333,21 @@ size_t attn_decode_smem_bytes() {
 }
 int attn_decode_max_blocks() { return MAXNB; }
 
-cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, cudaStream_t st) {
+// `ng` consumer groups per CTA (1 or 2; BULLET_DEC_GROUPS overrides).
+cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStream_t st) {
   const size_t smem = attn_decode_smem_bytes();
+  static const int forced = getenv("BULLET_DEC_GROUPS") ? atoi(getenv("BULLET_DEC_GROUPS")) : 0;
+  if (forced == 1 || forced == 2) ng = forced;
   static bool set = false;
   if (!set) {
-    cudaError_t e = cudaFuncSetAttribute(k_attn_decode_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(k_attn_decode_tc<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(k_attn_decode_tc<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     set = true;
   }
-  k_attn_decode_tc<<<grid, THREADS, smem, st>>>(a);
+  if (ng == 1) k_attn_decode_tc<1><<<grid, THREADS, smem, st>>>(a);
+  else k_attn_decode_tc<2><<<grid, THREADS, smem, st>>>(a);
   return cudaGetLastError();
 }
 

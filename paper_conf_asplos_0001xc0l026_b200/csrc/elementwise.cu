@@ -219,33 +219,6 @@ __global__ void k_plan(PlanArgs a) {
         }
       *a.n_tiles = n;
     }
-    if (a.dlist) {   // decode chunk list: block-wide exclusive scan of chunk counts
-      __shared__ int s_w[8];
-      __shared__ int s_base;
-      if (threadIdx.x == 0) s_base = 0;
-      __syncthreads();
-      const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-      for (int t0 = 0; t0 < a.n_tok; t0 += blockDim.x) {
-        const int t = t0 + threadIdx.x;
-        const int nch = t < a.n_tok ? ((__ldg(a.ctx + t) / a.B + 1) + a.cb - 1) / a.cb : 0;
-        int x = nch;   // inclusive warp scan
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const int y = __shfl_up_sync(0xffffffffu, x, o);
-          if (lane >= o) x += y;
-        }
-        if (lane == 31) s_w[w] = x;
-        __syncthreads();
-        int off = s_base;
-        for (int i = 0; i < w; ++i) off += s_w[i];
-        off += x - nch;
-        for (int c = 0; c < nch; ++c) a.dlist[off + c] = make_int2(t, c);
-        __syncthreads();
-        if (threadIdx.x == blockDim.x - 1) s_base = off + nch;
-        __syncthreads();
-      }
-      if (threadIdx.x == 0) *a.n_dlist = s_base;
-    }
   }
   if (a.tok) {
     for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < a.n_tok; t += gridDim.x * blockDim.x) {

@@ -69,12 +69,6 @@ struct AttnArgs {
   const int2* tiles;      // prefill tensor-core kernel: (request, q-tile) list
   const int* n_tiles;     // device count of `tiles`
   int dbg;                // diagnostics (BULLET_DBG env): bit0 = decode consumers skip math
-  // register-direct decode kernel (attn_decode2.cu): `tiles` holds the
-  // (token, chunk) list, chunks of `cb` KV blocks; partial records and
-  // per-(token, kv head) tickets (zero between launches, self-resetting)
-  int cb;
-  float* part;
-  int* tickets;
   Launch L;
 };
 
@@ -89,9 +83,6 @@ struct PlanArgs {
   int2* tiles; int* n_tiles;
   // per-token (position, slot) table (nullable): needs ctx, bt, max_blocks, B
   TokInfo* tok; const int32_t* ctx; const int32_t* bt; int max_blocks, B, n_tok;
-  // decode chunk list (nullable): (token, chunk) for chunks of cb blocks of
-  // ctx[t] + 1 keys, token order, written to dlist[0, *n_dlist)
-  int2* dlist; int* n_dlist; int cb;
 };
 
 // launchers (return cudaError_t of the launch)
@@ -109,10 +100,7 @@ template <typename T>
 cudaError_t launch_attn_simt(const AttnArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_attn_prefill_tc(const AttnArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_attn_prefill5(const AttnArgs& a, int grid, cudaStream_t st);
-cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, cudaStream_t st);
-cudaError_t launch_attn_decode2(const AttnArgs& a, int grid, cudaStream_t st);
-int attn_decode2_rec_floats(int grp);
-int attn_decode2_warps();
+cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStream_t st);
 size_t attn_decode_smem_bytes();
 int attn_decode_max_blocks();
 cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);   // grid sized to n_tok

@@ -44,7 +44,7 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
 #pragma unroll
       for (int i = 0; i < 16; ++i) acc ^= v[i].x ^ v[i].y ^ v[i].z ^ v[i].w;
     }
-  } else if (a.mode == 3 || a.mode == 4) {
+  } else if ((a.mode == 3 || a.mode == 4) || (a.mode == 5 && tid >= 32)) {
     // mode 3: LDG.128 -> registers -> STS.128 into a per-warp smem slot (a
     // register-staged producer); mode 4: same loads, no STS.  Warps claim
     // 32 KB (4 x 8 KB) per atomic; `param` = 8 KB loads in flight per warp (1|2).
@@ -89,13 +89,14 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
       __syncwarp();
       if (a.mode == 3) acc ^= reinterpret_cast<const uint32_t*>(slot)[lane];
     }
-  } else if (a.mode == 1) {
+  } else if (a.mode == 1 || a.mode == 5) {
+    // mode 5 (warp 0 only here): bulk copies concurrently with LDG warps 1..15
     const size_t units = a.bytes / BULK;
     if (tid == 0) {
       for (int i = 0; i < NB; ++i) mbar_init(bars + i, 1);
       mbar_fence_init();
     }
-    __syncthreads();
+    if (a.mode == 1) __syncthreads(); else __syncwarp();
     if (tid == 0) {
       uint32_t issued = 0, done = 0;
       for (;;) {
@@ -148,7 +149,7 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
 }
 
 cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st) {
-  const int smem = a.mode == 1 ? NB * BULK : (a.mode == 2 ? 3 * 65536 : (a.mode == 3 ? 16 * 8192 : 0));
+  const int smem = a.mode == 1 ? NB * BULK : (a.mode == 2 ? 3 * 65536 : (a.mode == 3 ? 16 * 8192 : (a.mode == 5 ? NB * BULK : 0)));
   cudaError_t e = cudaFuncSetAttribute(k_stream, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return e;
   k_stream<<<grid, 512, smem, st>>>(a);

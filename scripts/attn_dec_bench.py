@@ -1,9 +1,9 @@
 """Decode-attention microbenchmark: bullet_op_attention on the bench
 workload's decode batch (random KV, the bench's block tables) on the last
-m SMs; prints KV GB/s and GB/s per SM.  Env: BULLET_DBG (kernel variants),
-BULLET_DEC2_WARPS, BULLET_DEC2_CB.
+m SMs; prints KV GB/s and GB/s per SM.  Env:
+BULLET_DEC_GROUPS (consumer groups per SM).
 
-  python scripts/attn_dec_bench.py --config arxiv-8b --kind 5 --sms 60 148
+  python scripts/attn_dec_bench.py --config arxiv-8b --kind 3 --sms 60 148
 """
 import argparse
 import json
@@ -35,7 +35,7 @@ def main():
     lay = synth.paged_layout([1] * n, ctx, 16)
     pk = torch.randn(lay.n_blocks, m.n_kv_heads, 16, m.head_dim, device="cuda").to(torch.bfloat16)
     pv = torch.randn_like(pk)
-    bl = B.Bullet(B.Model.of(m), [(pk, pv)], 16, n, max(ctx) + 32)
+    bl = B.Bullet(B.Model.of(m), [(pk, pv)], n, n, max(ctx) + 32)
     q = torch.randn(n, m.n_heads * m.head_dim, device="cuda").to(torch.bfloat16)
     o = torch.empty_like(q)
     b = B.Batch([1] * n, ctx, lay.block_table, torch.zeros(n, m.d_model, device="cuda"))

@@ -20,7 +20,8 @@ def main():
     bl = B.Bullet(B.Model.of(m), pools, 16, 16, 64)
     buf = torch.empty(2 << 30, dtype=torch.uint8, device="cuda")
     for mode, param, name in ((3, 1, "ldg+sts 8KB/warp"), (3, 2, "ldg+sts 16KB/warp"), (4, 1, "ldg 8KB/warp"),
-                              (4, 2, "ldg 16KB/warp"), (2, 0, "cp.async 192KB"), (1, 0, "bulk 192KB")):
+                              (4, 2, "ldg 16KB/warp"), (2, 0, "cp.async 192KB"), (1, 0, "bulk 192KB"),
+                              (5, 1, "bulk 192KB + ldg 15 warps x 8KB")):
         for msm in (20, 40, 68, 100, 148):
             lo = bl.n_sms - msm
             code = mode | (param << 8)

@@ -229,8 +229,7 @@ L70_TP8 = synth.MODELS["llama3.1-70b"].shard(8)       # GQA group 8
 
 @pytest.mark.parametrize("m,kind", [(SMALL, 1), (SMALL, 2), (TINY, 1), (LLAMA, 2), (LLAMA, 1),
                                     (SMALL, 4), (LLAMA, 4), (QWEN_TP2, 4), (L70_TP8, 4),
-                                    (SMALL, 3), (LLAMA, 3), (QWEN_TP2, 3), (L70_TP8, 3),
-                                    (SMALL, 5), (LLAMA, 5), (QWEN_TP2, 5), (L70_TP8, 5)])
+                                    (SMALL, 3), (LLAMA, 3), (QWEN_TP2, 3), (L70_TP8, 3)])
 def test_attention_vs_oracle(B, m, kind):
     """Paged attention (decode rows and causal prefill rows) vs the oracle's
     plain softmax attention through the block table.  kind 1 SIMT, 2
@@ -240,8 +239,6 @@ def test_attention_vs_oracle(B, m, kind):
         q_lens, ctx = [150, 64, 1, 77, 300], [0, 0, 0, 0, 0]
     if kind == 3:
         q_lens, ctx = [1] * 7, [0, 15, 16, 63, 200, 1000, 2047]
-    if kind == 5:
-        q_lens, ctx = [1] * 8, [0, 15, 16, 63, 200, 1000, 2047, 5000]
     lay = synth.paged_layout(q_lens, ctx, 16, seed_offset=5)
     bl, pools = _handle(B, m, n_blocks=lay.n_blocks)
     pk_cpu, pv_cpu = synth.kv_pool(m, lay.n_blocks, 16, 0)
@@ -273,34 +270,3 @@ def test_attention_vs_oracle(B, m, kind):
             row += 1
     assert worst < (1.6e-2 if m.dtype == "bf16" else 2e-5), worst
 
-
-@pytest.mark.parametrize("cb,lo", [(None, 0), (None, 140), (1, 0), (7, 100), (40, 0), (400, 146)])
-def test_decode2_chunking(B, cb, lo, monkeypatch):
-    """Register-direct decode attention (kind 5) at forced chunk sizes and SM
-    ranges: single-chunk rows (direct write), many-chunk rows (partials +
-    ticket merge), chunks longer than 32 blocks (block-id register refill)."""
-    if cb is not None:
-        monkeypatch.setenv("BULLET_DEC2_CB", str(cb))
-    m = LLAMA
-    q_lens, ctx = [1] * 9, [0, 15, 16, 511, 512, 1000, 2047, 3000, 6000]
-    lay = synth.paged_layout(q_lens, ctx, 16, seed_offset=9)
-    bl, pools = _handle(B, m, n_blocks=lay.n_blocks)
-    pk_cpu, pv_cpu = synth.kv_pool(m, lay.n_blocks, 16, 0)
-    pools[0][0].copy_(pk_cpu.to(bf16)); pools[0][1].copy_(pv_cpu.to(bf16))
-    n, H, hd = len(q_lens), m.n_heads, m.head_dim
-    q = O.round_bf16(np.random.default_rng(3).standard_normal((n, H * hd)))
-    b = B.Batch(q_lens, ctx, lay.block_table, torch.zeros(n, m.d_model, device="cuda"))
-    outs = []
-    for _ in range(2):   # second launch: the tickets reset themselves
-        o = torch.zeros(n, H * hd, dtype=bf16, device="cuda")
-        bl.op_attention(b, 0, torch.from_numpy(q.astype(np.float32)).to("cuda", bf16), o, kind=5, lo=lo)
-        torch.cuda.synchronize()
-        outs.append(o.float().cpu().numpy())
-    assert np.array_equal(outs[0], outs[1])   # deterministic merge order
-    pk, pv = pk_cpu.numpy(), pv_cpu.numpy()
-    worst = 0.0
-    for r in range(n):
-        for h in range(H):
-            ref = O.attend_paged(q[r, h * hd:(h + 1) * hd], pk, pv, lay.block_table[r], 16, h // 4, ctx[r])
-            worst = max(worst, float(np.abs(outs[0][r, h * hd:(h + 1) * hd] - ref).max()))
-    assert worst < 1.6e-2, worst
