@@ -956,7 +956,8 @@ int bullet_op_stream(bullet_handle* h, const void* src, size_t bytes, int mode, 
   if (!src || bytes == 0 || (mode & 0xff) > 5 || mode < 0) return set_err(BULLET_EINVAL, "stream args");
   StreamArgs a;
   memset(&a, 0, sizeof a);
-  a.src = (const uint8_t*)src; a.bytes = bytes; a.mode = mode & 0xff; a.param = mode >> 8;
+  a.src = (const uint8_t*)src; a.bytes = bytes; a.mode = mode & 0xff; a.param = (mode >> 8) & 0xff;
+  a.wrap = (mode >> 16) ? ((size_t)1 << (mode >> 16)) - 1 : ~(size_t)0;   // window 2^(mode >> 16) bytes
   a.sink = (uint32_t*)h->op_ctr;
   if ((rc = next_launch(c, &a.L))) return rc;
   LAUNCH(c, launch_stream(a, h->n_sms, c.st));

@@ -74,6 +74,7 @@ struct AttnArgs {
 
 struct StreamArgs {   // KI2 streaming microbenchmark
   const uint8_t* src; size_t bytes; int mode; int param; uint32_t* sink;
+  size_t wrap;        // offsets masked by wrap (window - 1): re-read an L2-resident window
   Launch L;
 };
 

@@ -37,7 +37,7 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
       if (lane == 0) u = atomicAdd(a.L.ctr, 1);
       u = __shfl_sync(0xffffffffu, u, 0);
       if (u >= (int)units) break;
-      const uint4* p = reinterpret_cast<const uint4*>(a.src + (size_t)u * 8192) + lane;
+      const uint4* p = reinterpret_cast<const uint4*>(a.src + (((size_t)u * 8192) & a.wrap)) + lane;
       uint4 v[16];
 #pragma unroll
       for (int i = 0; i < 16; ++i) v[i] = __ldcs(p + 32 * i);
@@ -56,7 +56,7 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
       if (lane == 0) u = atomicAdd(a.L.ctr, 1);
       u = __shfl_sync(0xffffffffu, u, 0);
       if (u >= (int)units) break;
-      const uint4* p = reinterpret_cast<const uint4*>(a.src + (size_t)u * 32768) + lane;
+      const uint4* p = reinterpret_cast<const uint4*>(a.src + (((size_t)u * 32768) & a.wrap)) + lane;
       if (a.param == 2) {
 #pragma unroll 1
         for (int h = 0; h < 4; h += 2) {
@@ -109,7 +109,7 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
         if (u >= (int)units) break;
         const int s = issued % NB;
         mbar_arrive_expect_tx(bars + s, BULK);
-        bulk_g2s(sm + s * BULK, a.src + (size_t)u * BULK, BULK, bars + s);
+        bulk_g2s(sm + s * BULK, a.src + (((size_t)u * BULK) & a.wrap), BULK, bars + s);
         ++issued;
       }
       while (done < issued) {
@@ -127,7 +127,7 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
       const int u = s_u;
       __syncthreads();
       if (u >= (int)units) break;
-      const uint8_t* p = a.src + (size_t)u * 65536;
+      const uint8_t* p = a.src + (((size_t)u * 65536) & a.wrap);
       uint8_t* d = sm + (n % 3) * 65536;
 #pragma unroll
       for (int i = 0; i < 8; ++i) cp_async16(d + (tid + i * 512) * 16, p + (tid + i * 512) * 16);
