@@ -156,7 +156,7 @@ class Step:
         pp = os.path.join(ROOT, "profiles", "perf_params_b200.json")   # fitted by scripts/fit_perfmodel.py
         self.perf_json = open(pp).read() if os.path.exists(pp) else None
         uids = parallel.nccl_uids() if self.tp > 1 else None
-        self.bl = B.Bullet(B.Model.of(m), self.pools, self.n_p, self.n_d, maxpos,
+        self.bl = B.Bullet(B.Model.of(m), self.pools, self.n_p + self.n_d, self.n_d, maxpos,
                            tp_size=self.tp, tp_rank=self.rank, nccl_uids=uids,
                            perf_params_json=self.perf_json)
         for l in range(n_layers):
@@ -190,6 +190,55 @@ class Step:
         e1.record(self.sp)
         torch.cuda.synchronize()
         return e0.elapsed_time(e1) / n
+
+    # ---- chunked-prefill hybrid baseline
+    def build_hybrid(self, k):
+        """The same work as one co-run step (prefill batch through one layer,
+        decode batch through k layer-steps) as k hybrid layer-steps on all
+        SMs: step c carries chunk c of every prompt (ctx = the chunks before
+        it, attended through the block table) plus every decode, at layer c."""
+        B = self.B
+        lens = list(self.wl.prefill_lens)
+        bt = self.lay.block_table
+        self.hyb = []
+        for c in range(k):
+            q, ctx, rows = [], [], []
+            for r, L in enumerate(lens):
+                a, b = c * L // k, (c + 1) * L // k
+                if b > a:
+                    q.append(b - a); ctx.append(a); rows.append(r)
+            q += [1] * self.n_d
+            ctx += list(self.wl.decode_ctx)
+            table = np.concatenate([bt[rows], bt[self.n_pre:]], axis=0)
+            x = synth.hidden(sum(q), self.m.d_model, 5 + c, device="cuda")
+            self.hyb.append(B.Batch(q, ctx, table, x, c, c + 1))
+
+    def enqueue_hybrid(self):
+        for hb in self.hyb:
+            self.bl.step(hb, None, self.N, self.B.TIMESLICED, self.sp, self.sd)
+
+    def time_hybrid(self, n):
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(self.sp)
+        for _ in range(n):
+            self.enqueue_hybrid()
+        e1.record(self.sp)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / n
+
+    def ab_vs_hybrid(self, p, blocks=6, per=5):
+        """Co-run vs the chunked-prefill hybrid on the same work, alternating blocks."""
+        ratios, th = [], []
+        for b in range(blocks):
+            if b % 2 == 0:
+                c = self.time_steps(per, p, self.B.CORUN)
+                h = self.time_hybrid(per)
+            else:
+                h = self.time_hybrid(per)
+                c = self.time_steps(per, p, self.B.CORUN)
+            ratios.append(h / c); th.append(h)
+        return float(np.median(ratios)), float(np.mean(th))
 
     def ab_speedup(self, p, blocks=6, per=5):
         """Co-run vs time-sliced on the same batch, measured in alternating
@@ -251,6 +300,10 @@ class Step:
         best = max(top, key=lambda r: r["speedup_ab"])
         self.dec.layer_end = 1
         return best, res
+
+
+def groups_tok(S, k, ws):
+    return (ws // S.tp) * S.tokens(k)
 
 
 # ---------------------------------------------------------------- roofline
@@ -410,6 +463,18 @@ def main():
     # drift-robust comparison: alternating co-run / time-sliced blocks
     ab, ab_co, ab_ts = S.ab_speedup(p, blocks=8, per=5)
     ab = allreduce_max(ab, ws)
+    # chunked-prefill hybrid baseline on the same work (k hybrid layer-steps)
+    hyb = None
+    if S.tp == 1:
+        S.build_hybrid(k)
+        for _ in range(args.warmup):
+            S.enqueue_hybrid()
+        t_hyb = S.time_hybrid(args.steps)
+        hab, hab_t = S.ab_vs_hybrid(p, blocks=8, per=5)
+        hyb = {"value": groups_tok(S, k, ws) / (t_hyb * 1e-3), "ms_per_step": t_hyb,
+               "corun_speedup_vs_hybrid": hab, "interleaved_hybrid_ms": hab_t,
+               "note": f"chunked prefill (SARATHI-style): {k} hybrid layer-steps on all SMs, each with chunk c "
+                       f"of every prompt (attending to the earlier chunks) + all {S.n_d} decodes"}
     # the paper's "Naive": both phases on all SMs at once, no gating
     for _ in range(args.warmup):
         S.enqueue(p, B.UNGATED)
@@ -516,6 +581,7 @@ def main():
             "bracketed": t_ts / t_co,
             "method": "median over 8 alternating blocks of 5 co-run and 5 time-sliced steps (order flipped "
                       "every block); 'bracketed' = time-sliced K steps before and after the K timed co-run steps"},
+        "hybrid_chunked_prefill": hyb,
         "ungated": {"value": groups * tok / (t_ung * 1e-3), "ms_per_step": t_ung,
                     "note": "both phases on all SMs concurrently (the paper's Naive, P:L304)"},
         "tokens_per_s_by_phase": {"prefill": groups * S.n_p / S.m.n_layers / (t_co * 1e-3),

@@ -119,7 +119,12 @@ typedef struct {
  * ctx_lens[r] .. ctx_lens[r] + q_len_r - 1.  Prefill: ctx 0 (any ctx works);
  * decode: q_len 1.  `hidden` rows are the new tokens, request-major; it is
  * read as x and overwritten with the layer output (fp32 residual stream).
- * The batch runs layers [layer_begin, layer_end) in order. */
+ * The batch runs layers [layer_begin, layer_end) in order.
+ * Hybrid (chunked-prefill) batches: requests with q_len > 1 first (prefill
+ * chunks, any ctx), then requests with q_len 1 (decodes); attention then runs
+ * the prefill kernel over the chunks and the decode kernel over the rest
+ * (the SARATHI-style baseline of SURVEY §8(f) NEXT-3: pass it as the
+ * prefill batch with mode TIMESLICED and no decode batch). */
 typedef struct {
   int n_reqs, n_tokens, max_blocks_per_req;
   const int32_t *d_cu_seqlens;   /* device [n_reqs+1] */
@@ -203,11 +208,22 @@ int bullet_sm_order(const bullet_handle *h, int32_t *h_sigma, int cap);
  * Ordering is the caller's: everything the step reads (hidden, tables,
  * pools, weights) must already be complete or ordered before s_prefill /
  * s_decode (e.g. cudaStreamWaitEvent); the step orders only its own kernels
- * (back to back on each stream, programmatic dependent launches).
+ * (back to back on each stream).
  * Errors: EINVAL (shapes), ESMRANGE (split), EKV (block table), ENOMEM
  * (batch larger than cfg max_*). */
 int bullet_step(bullet_handle *h, const bullet_batch *prefill, const bullet_batch *decode,
                 int prefill_sm_count, int flags, void *s_prefill, void *s_decode);
+
+/* bullet_step (BULLET_CORUN only) with explicit SM ranges of sigma: the
+ * prefill phase claims work on sigma[pre_lo, pre_hi), decode on
+ * sigma[dec_lo, dec_hi).  The ranges may overlap (non-strict partition,
+ * SURVEY §8(f) NEXT-4): an SM in both ranges runs whichever
+ * phase's CTA it receives, so a phase that finishes its kernels early leaves
+ * the shared band to the other.  Bounds on the TPC granularity within [0, N];
+ * a non-empty batch needs a non-empty range.  Errors as bullet_step. */
+int bullet_step_ranges(bullet_handle *h, const bullet_batch *prefill, const bullet_batch *decode,
+                       int pre_lo, int pre_hi, int dec_lo, int dec_hi, int flags, void *s_prefill,
+                       void *s_decode);
 
 /* Eq. 2 / T_m: predicted time (microseconds) of one layer of the given
  * batch on sm_count SMs; corun_sm_count > 0 applies the co-location factors

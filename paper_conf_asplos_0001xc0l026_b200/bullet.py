@@ -85,7 +85,7 @@ def lib():
         L = ctypes.CDLL(path, mode=ctypes.RTLD_GLOBAL)
         L.bullet_last_error.restype = ctypes.c_char_p
         for name in ("bullet_create", "bullet_perf_create", "bullet_set_layer_weights", "bullet_num_sms", "bullet_sm_order",
-                     "bullet_step", "bullet_model_predict", "bullet_choose_split",
+                     "bullet_step", "bullet_step_ranges", "bullet_model_predict", "bullet_choose_split",
                      "bullet_set_smid_log", "bullet_sync", "bullet_nccl_unique_id", "bullet_op_gemm",
                      "bullet_op_rmsnorm", "bullet_op_rope_kv", "bullet_op_attention",
                      "bullet_profile_read", "bullet_launch_count"):
@@ -99,6 +99,8 @@ def lib():
         L.bullet_sm_order.argtypes = [c_void_p, P_i32, c_int]
         L.bullet_step.argtypes = [c_void_p, ctypes.POINTER(CBatch), ctypes.POINTER(CBatch), c_int, c_int,
                                   c_void_p, c_void_p]
+        L.bullet_step_ranges.argtypes = [c_void_p, ctypes.POINTER(CBatch), ctypes.POINTER(CBatch), c_int, c_int,
+                                         c_int, c_int, c_int, c_void_p, c_void_p]
         L.bullet_model_predict.argtypes = [c_void_p, ctypes.POINTER(BatchShape), c_int, c_int, P_f64]
         L.bullet_choose_split.argtypes = [c_void_p, ctypes.POINTER(SchedState), ctypes.POINTER(Slo),
                                           ctypes.POINTER(c_int), ctypes.POINTER(c_int)]
@@ -279,6 +281,16 @@ class Bullet:
         _check(lib().bullet_step(self.h, ctypes.byref(pb) if pb else None,
                                  ctypes.byref(db) if db else None, int(prefill_sm_count), int(flags),
                                  _stream(s_prefill), _stream(s_decode)))
+
+    def step_ranges(self, prefill: Batch | None, decode: Batch | None, pre_range, dec_range, flags: int = CORUN,
+                    s_prefill=None, s_decode=None):
+        """Co-run step on explicit (possibly overlapping) SM ranges of sigma."""
+        pb = prefill.c() if prefill else None
+        db = decode.c() if decode else None
+        _check(lib().bullet_step_ranges(self.h, ctypes.byref(pb) if pb else None,
+                                        ctypes.byref(db) if db else None, int(pre_range[0]), int(pre_range[1]),
+                                        int(dec_range[0]), int(dec_range[1]), int(flags),
+                                        _stream(s_prefill), _stream(s_decode)))
 
     def sync(self):
         _check(lib().bullet_sync(self.h))

@@ -395,6 +395,19 @@ int max_kv(const bullet_batch* b) {
   return mk;
 }
 
+// Mixed (chunked-prefill hybrid) batch: leading requests with q > 1, then
+// only requests with q <= 1.  Returns the number of leading requests (0 when
+// the batch is not mixed) and their token count in *t0.
+int mixed_split(const bullet_batch* b, int* t0) {
+  int r0 = 0;
+  while (r0 < b->n_reqs && b->h_cu_seqlens[r0 + 1] - b->h_cu_seqlens[r0] > 1) ++r0;
+  if (r0 == 0 || r0 == b->n_reqs) return 0;
+  for (int r = r0; r < b->n_reqs; ++r)
+    if (b->h_cu_seqlens[r + 1] - b->h_cu_seqlens[r] > 1) return 0;
+  *t0 = b->h_cu_seqlens[r0];
+  return *t0 < b->n_tokens ? r0 : 0;
+}
+
 int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* o, int kind) {
   bullet_handle* h = c.h;
   if (b->n_tokens == 0) return BULLET_OK;
@@ -408,6 +421,23 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
   static const int dbg = getenv("BULLET_DBG") ? atoi(getenv("BULLET_DBG")) : 0;
   a.dbg = dbg;
   const bool bf16 = h->cfg.dtype == BULLET_DTYPE_BF16;
+  int t0 = 0;
+  const int r0 = (kind == 0 && !c.op && bf16 && a.hd == 128) ? mixed_split(b, &t0) : 0;
+  if (r0) {   // hybrid batch: tcgen05 FA over the prefill chunks, decode kernel over the rest
+    for (int r = r0; r < b->n_reqs; ++r)
+      if (b->h_ctx_lens[r] + 1 > attn_decode_max_blocks() * h->block_size)
+        return set_err(BULLET_EUNSUPPORTED, "hybrid batch: decode context too long");
+    PhaseWS& P = h->ph[c.phase];
+    a.tiles = P.tiles; a.n_tiles = P.n_tiles;   // the plan listed tiles of requests [0, r0) only
+    int rc = next_launch(c, &a.L);
+    if (rc) return rc;
+    LAUNCH(c, launch_attn_prefill5(a, persist_grid(c, 2), c.st));
+    AttnArgs d = a;
+    d.tok_base = t0;
+    if ((rc = next_launch(c, &d.L))) return rc;
+    LAUNCH(c, launch_attn_decode_tc(d, persist_grid(c, 1), c.m_sms <= 100 ? 2 : 1, c.st));
+    return BULLET_OK;
+  }
   if (kind == 0) kind = (bf16 && a.hd == 128) ? (max_qlen(b) > 1 ? 4 : 3) : 1;
   if (kind == 3 && max_kv(b) > attn_decode_max_blocks() * h->block_size) kind = c.op ? -1 : 1;
   if (kind == -1) return set_err(BULLET_EUNSUPPORTED, "tensor-core decode attention: context too long");
@@ -427,7 +457,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     PhaseWS& P = h->ph[c.phase];
     a.tiles = P.tiles; a.n_tiles = P.n_tiles;
     if (c.op) {  // op-level: plan the tile list now
-      PlanArgs pa{nullptr, 0, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ, P.tiles, P.n_tiles,
+      PlanArgs pa{nullptr, 0, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ, b->n_reqs, P.tiles, P.n_tiles,
                   nullptr, nullptr, nullptr, 0, 0, 0};
       prof_begin(c);
       LAUNCH(c, launch_plan(pa, c.st));
@@ -542,7 +572,9 @@ int run_phase(Ctx& c, const bullet_batch* b) {
   PhaseWS& P = c.h->ph[c.phase];
   P.next_ctr = 0;
   const bool tc_attn = c.h->cfg.dtype == BULLET_DTYPE_BF16 && c.h->cfg.head_dim == 128 && max_qlen(b) > 1;
-  PlanArgs pa{P.counters, P.n_counters, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ,
+  int t0 = 0;
+  const int r0 = tc_attn ? mixed_split(b, &t0) : 0;
+  PlanArgs pa{P.counters, P.n_counters, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ, r0 ? r0 : b->n_reqs,
               tc_attn ? P.tiles : nullptr, P.n_tiles,
               c.fuse_qkv ? P.tok : nullptr, b->d_ctx_lens, b->d_block_table, b->max_blocks_per_req,
               c.h->block_size, b->n_tokens};
@@ -782,28 +814,28 @@ int bullet_set_smid_log(bullet_handle* h, int32_t* d_log, int capacity) {
   return BULLET_OK;
 }
 
-int bullet_step(bullet_handle* h, const bullet_batch* pre, const bullet_batch* dec,
-                int prefill_sm_count, int flags, void* s_prefill, void* s_decode) {
-  if (!h) return set_err(BULLET_EINVAL, "null handle");
-  if (h->host_only) return set_err(BULLET_EUNSUPPORTED, "host-only handle");
-  const int N = h->n_sms, p = prefill_sm_count, mode = flags & 3;
-  if (mode == 3) return set_err(BULLET_EINVAL, "flags: TIMESLICED and UNGATED are exclusive");
-  if (p < 0 || p > N || (p % GRAN && p != N)) return set_err(BULLET_ESMRANGE, "prefill_sm_count %d not in [0,%d] step %d", p, N, GRAN);
+// Shared body of bullet_step / bullet_step_ranges: prefill claims work on
+// sigma[plo, phi), decode on sigma[dlo, dhi) (mode CORUN), else on all SMs.
+static int step_impl(bullet_handle* h, const bullet_batch* pre, const bullet_batch* dec, int plo, int phi,
+                     int dlo, int dhi, bool dec_paused, int flags, void* s_prefill, void* s_decode) {
+  const int N = h->n_sms, mode = flags & 3;
   const bool has_pre = pre && pre->n_tokens > 0, has_dec = dec && dec->n_tokens > 0;
   int rc;
   if (pre && (rc = validate_batch(h, pre, 0))) return rc;
   if (dec && (rc = validate_batch(h, dec, 1))) return rc;
-  if (mode == BULLET_CORUN && has_pre && p == 0)
-    return set_err(BULLET_ESMRANGE, "prefill batch given with prefill_sm_count 0");
-  const bool run_dec = has_dec && !(mode == BULLET_CORUN && p == N);  // p = N: decode paused
+  if (mode == BULLET_CORUN && has_pre && phi <= plo)
+    return set_err(BULLET_ESMRANGE, "prefill batch given with an empty prefill SM range");
+  const bool run_dec = has_dec && !(mode == BULLET_CORUN && dec_paused);
+  if (mode == BULLET_CORUN && run_dec && dhi <= dlo)
+    return set_err(BULLET_ESMRANGE, "decode batch given with an empty decode SM range");
   if (h->log_cap == 0 && (flags & BULLET_SMID_LOG)) return set_err(BULLET_EINVAL, "SMID_LOG without a log buffer");
   const bool log = (flags & BULLET_SMID_LOG) != 0;
   cudaStream_t sp = (cudaStream_t)s_prefill, sd = (cudaStream_t)s_decode;
   const bool prof = (flags & BULLET_PROFILE) != 0;
-  Ctx cp{h, 0, mode == BULLET_CORUN ? gate_of(h, 0, p) : gate_of(h, 0, N),
-         mode == BULLET_CORUN ? p : N, log, sp, false, prof};
-  Ctx cd{h, 1, mode == BULLET_CORUN ? gate_of(h, p, N) : gate_of(h, 0, N),
-         mode == BULLET_CORUN ? N - p : N, log, sd, false, prof};
+  Ctx cp{h, 0, mode == BULLET_CORUN ? gate_of(h, plo, phi) : gate_of(h, 0, N),
+         mode == BULLET_CORUN ? phi - plo : N, log, sp, false, prof};
+  Ctx cd{h, 1, mode == BULLET_CORUN ? gate_of(h, dlo, dhi) : gate_of(h, 0, N),
+         mode == BULLET_CORUN ? dhi - dlo : N, log, sd, false, prof};
   cp.fuse_qkv = cd.fuse_qkv = !(flags & BULLET_UNFUSED) && h->cfg.dtype == BULLET_DTYPE_BF16 &&
                               h->cfg.head_dim == 128;
   if (has_pre && (rc = run_phase(cp, pre))) return rc;
@@ -815,6 +847,31 @@ int bullet_step(bullet_handle* h, const bullet_batch* pre, const bullet_batch* d
     if ((rc = run_phase(cd, dec))) return rc;
   }
   return BULLET_OK;
+}
+
+int bullet_step(bullet_handle* h, const bullet_batch* pre, const bullet_batch* dec,
+                int prefill_sm_count, int flags, void* s_prefill, void* s_decode) {
+  if (!h) return set_err(BULLET_EINVAL, "null handle");
+  if (h->host_only) return set_err(BULLET_EUNSUPPORTED, "host-only handle");
+  const int N = h->n_sms, p = prefill_sm_count, mode = flags & 3;
+  if (mode == 3) return set_err(BULLET_EINVAL, "flags: TIMESLICED and UNGATED are exclusive");
+  if (p < 0 || p > N || (p % GRAN && p != N)) return set_err(BULLET_ESMRANGE, "prefill_sm_count %d not in [0,%d] step %d", p, N, GRAN);
+  if (mode == BULLET_CORUN && pre && pre->n_tokens > 0 && p == 0)
+    return set_err(BULLET_ESMRANGE, "prefill batch given with prefill_sm_count 0");
+  return step_impl(h, pre, dec, 0, p, p, N, p == N, flags, s_prefill, s_decode);   // p = N: decode paused
+}
+
+int bullet_step_ranges(bullet_handle* h, const bullet_batch* pre, const bullet_batch* dec, int pre_lo, int pre_hi,
+                       int dec_lo, int dec_hi, int flags, void* s_prefill, void* s_decode) {
+  if (!h) return set_err(BULLET_EINVAL, "null handle");
+  if (h->host_only) return set_err(BULLET_EUNSUPPORTED, "host-only handle");
+  const int N = h->n_sms, mode = flags & 3;
+  if (mode != BULLET_CORUN) return set_err(BULLET_EINVAL, "bullet_step_ranges: CORUN only");
+  auto ok = [&](int x) { return x >= 0 && x <= N && (x % GRAN == 0 || x == N); };
+  if (!ok(pre_lo) || !ok(pre_hi) || !ok(dec_lo) || !ok(dec_hi) || pre_lo > pre_hi || dec_lo > dec_hi)
+    return set_err(BULLET_ESMRANGE, "ranges [%d,%d) [%d,%d) not within [0,%d] on step %d", pre_lo, pre_hi,
+                   dec_lo, dec_hi, N, GRAN);
+  return step_impl(h, pre, dec, pre_lo, pre_hi, dec_lo, dec_hi, false, flags, s_prefill, s_decode);
 }
 
 static PhaseShape model_shape(const bullet_handle* h) {

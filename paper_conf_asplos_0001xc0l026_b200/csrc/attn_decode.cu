@@ -102,7 +102,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int grp = a.H / a.Hkv;
-  const int units = a.n_tok * a.Hkv;
+  const int units = (a.n_tok - a.tok_base) * a.Hkv;   // decode rows are tokens [tok_base, n_tok)
   if (threadIdx.x == 0) {
     for (int i = 0; i < 4; ++i) { mbar_init(uqf + i, 1); mbar_init(uqe + i, GW); }
     mbar_fence_init();
@@ -125,7 +125,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
       if (u >= units) u = -1;
       Slot sl{u, 0, 0, 0};
       if (u >= 0) {
-        sl.t = u / a.Hkv;
+        sl.t = a.tok_base + u / a.Hkv;
         const int r = find_req(a.cu, a.n_reqs, sl.t);
         sl.pos = __ldg(a.ctx + r) + (sl.t - __ldg(a.cu + r));
         sl.nb = sl.pos / KB + 1;

@@ -206,14 +206,14 @@ __global__ void k_plan(PlanArgs a) {
     for (int i = threadIdx.x; i < a.n_counters; i += blockDim.x) a.counters[i] = 0;
     if (threadIdx.x == 0 && a.tiles) {
       int maxt = 0;
-      for (int r = 0; r < a.n_reqs; ++r) {
+      for (int r = 0; r < a.n_tile_reqs; ++r) {
         int len = a.cu[r + 1] - a.cu[r];
         int nt = (len + a.bq - 1) / a.bq;
         maxt = nt > maxt ? nt : maxt;
       }
       int n = 0;
       for (int t = maxt - 1; t >= 0; --t)
-        for (int r = 0; r < a.n_reqs; ++r) {
+        for (int r = 0; r < a.n_tile_reqs; ++r) {
           int len = a.cu[r + 1] - a.cu[r];
           if (t * a.bq < len) a.tiles[n++] = make_int2(r, t);
         }

@@ -69,6 +69,7 @@ struct AttnArgs {
   const int2* tiles;      // prefill tensor-core kernel: (request, q-tile) list
   const int* n_tiles;     // device count of `tiles`
   int dbg;                // diagnostics (BULLET_DBG env): bit0 = decode consumers skip math
+  int tok_base;           // decode kernel: its rows are tokens [tok_base, n_tok) (mixed batches)
   Launch L;
 };
 
@@ -81,6 +82,7 @@ struct StreamArgs {   // KI2 streaming microbenchmark
 struct PlanArgs {
   int* counters; int n_counters;
   const int32_t* cu; int n_reqs; int bq;
+  int n_tile_reqs;    // prefill attention tiles cover requests [0, n_tile_reqs)
   int2* tiles; int* n_tiles;
   // per-token (position, slot) table (nullable): needs ctx, bt, max_blocks, B
   TokInfo* tok; const int32_t* ctx; const int32_t* bt; int max_blocks, B, n_tok;

@@ -237,6 +237,8 @@ def test_attention_vs_oracle(B, m, kind):
     q_lens, ctx = [150, 64, 1, 1, 1, 1], [0, 0, 0, 63, 200, 1000]
     if kind in (2, 4):
         q_lens, ctx = [150, 64, 1, 77, 300], [0, 0, 0, 0, 0]
+    if kind == 4 and m is LLAMA:   # chunked prefill: chunks attend to cached context
+        q_lens, ctx = [150, 64, 1, 77, 300], [512, 0, 33, 1000, 129]
     if kind == 3:
         q_lens, ctx = [1] * 7, [0, 15, 16, 63, 200, 1000, 2047]
     lay = synth.paged_layout(q_lens, ctx, 16, seed_offset=5)

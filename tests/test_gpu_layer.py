@@ -186,3 +186,71 @@ def test_fused_qkv_rope_matches_unfused(p, bias):
     dk = (a_k.float() - b_k.float()).abs()
     assert float((dk / b_k.float().abs().clamp_min(1e-30)).max()) <= 2 ** -7
     assert float((a_pre - b_pre).abs().max()) <= 2e-2 and float((a_dec - b_dec).abs().max()) <= 2e-2
+
+
+@pytest.mark.parametrize("mode", ["timesliced", "corun"])
+def test_hybrid_chunked_prefill_batch(mode):
+    """Chunked-prefill hybrid batch: prefill chunks
+    with cached context (ctx > 0, attention over the earlier chunks through the
+    block table) followed by decode requests, as ONE batch through one layer:
+    tcgen05 prefill attention over the chunks, decode kernel over the rest.
+    Checked against the oracle layer on the same mixed batch."""
+    from harness import oracle_cfg
+    import oracle as O
+    m = synth.ModelShape("small-bf16", 1024, 8, 2, 128, 2816, 1)
+    q = [256, 130, 64, 1, 1, 1, 1, 1]
+    c = [512, 77, 0, 63, 500, 16, 1000, 1]
+    lay = synth.paged_layout(q, c, 16)
+    w_cpu = synth.layer_weights(m, 0)
+    pk_cpu, pv_cpu = synth.kv_pool(m, lay.n_blocks, 16, 0)
+    x = synth.hidden(sum(q), m.d_model, seed_offset=0)
+    import paper_conf_asplos_0001xc0l026_b200 as B
+    pools = [(pk_cpu.to("cuda", torch.bfloat16).contiguous(), pv_cpu.to("cuda", torch.bfloat16).contiguous())]
+    bl = B.Bullet(B.Model.of(m), pools, sum(q), 16, max(a + b for a, b in zip(q, c)) + 16)
+    bl.set_layer_weights(0, {k: (None if v is None else v.to("cuda", torch.bfloat16)) for k, v in w_cpu.items()})
+    b = B.Batch(q, c, lay.block_table, x.cuda().contiguous(), 0, 1)
+    sp, sd = phase_streams()
+    flags = B.TIMESLICED if mode == "timesliced" else B.CORUN
+    bl.step(b, None, bl.n_sms if mode == "timesliced" else 64, flags, sp, sd)
+    torch.cuda.synchronize()
+    w = {k: (None if v is None else v.numpy()) for k, v in w_cpu.items()}
+    ref = O.layer_forward(oracle_cfg(m), w, pk_cpu.numpy().copy(), pv_cpu.numpy().copy(), q, c,
+                          lay.block_table, x.double().numpy())
+    mx, mr = compare(b.hidden.cpu().numpy(), ref)
+    assert mx <= 2e-2 and mr <= 1e-3, (mx, mr)
+    n_pre = sum(q[:3])
+    mx, mr = compare(b.hidden.cpu().numpy()[n_pre:], ref[n_pre:])   # the decode rows alone
+    assert mx <= 2e-2 and mr <= 1e-3, ("decode rows", mx, mr)
+
+
+@pytest.mark.parametrize("ranges", [((0, 80), (60, 148)), ((0, 148), (0, 148)), ((20, 100), (0, 40))])
+def test_step_ranges_overlapping(small_bf16, ranges):
+    """bullet_step_ranges (NEXT-4: non-strict partitions): with overlapping
+    SM ranges both phases still meet the oracle bar, every unit runs exactly
+    once, and each phase's units ran only inside its own range."""
+    S = small_bf16
+    B = S.B
+    (plo, phi), (dlo, dhi) = ranges
+    ref = S.oracle(layers=1)
+    pre, dec = S.batches(0, 1)
+    log = S.bl.set_smid_log(400000)
+    try:
+        sp, sd = phase_streams()
+        S.bl.step_ranges(pre, dec, (plo, phi), (dlo, dhi), B.CORUN | B.SMID_LOG, sp, sd)
+        torch.cuda.synchronize()
+        n = int(log[0].item())
+        e = log[1:1 + 4 * n].view(n, 4).cpu().numpy()
+    finally:
+        S.bl.set_smid_log(None)
+    for name, b in (("pre", pre), ("dec", dec)):
+        mx, mr = compare(b.hidden.cpu().numpy(), ref[name])
+        assert mx <= 2e-2 and mr <= 1e-3, (name, mx, mr)
+    sigma = list(S.bl.sm_order())
+    allowed = {0: set(sigma[plo:phi]), 1: set(sigma[dlo:dhi])}
+    for launch in np.unique(e[:, 0]):
+        rows = e[e[:, 0] == launch]
+        units = rows[:, 1]
+        assert len(np.unique(units)) == len(units) and units.max() == len(units) - 1
+        assert set(rows[:, 2].tolist()) <= allowed[int(rows[0, 3])]
+    with pytest.raises(B.BulletError):
+        S.bl.step_ranges(pre, dec, (0, 0), (0, 148), B.CORUN)   # non-empty batch, empty range
