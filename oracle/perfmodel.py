@@ -78,10 +78,15 @@ def layer_kernels(shape: dict, P: dict, m: int) -> list:
         attn_units = sum(math.ceil(q / T["attn_bq"]) for q in q_lens) * H
     else:                   # decode: one unit per (request, kv head)
         attn_units = len(q_lens) * Hkv
+    if e == 2 and hd == 128:   # bf16: RoPE + KV append fused into the QKV GEMM epilogue
+        name, c, b, g, occ = gemm("qkv", d, nq, e * n * nq)
+        qkv = [(name, c + 6.0 * n * (H + Hkv) * hd, b, g, occ)]
+    else:
+        qkv = [gemm("qkv", d, nq, 4 * n * nq),
+               ("rope_kv", 6.0 * n * (H + Hkv) * hd, 4 * n * nq + e * n * nq, math.ceil(n / rows), occ_e)]
     ks = [
         ("rmsnorm1", 4.0 * n * d, 4 * n * d + e * n * d + e * d, math.ceil(n / rows), occ_e),
-        gemm("qkv", d, nq, 4 * n * nq),
-        ("rope_kv", 6.0 * n * (H + Hkv) * hd, 4 * n * nq + e * n * nq, math.ceil(n / rows), occ_e),
+        *qkv,
         ("attn", 4.0 * hd * H * pairs, 2 * e * Hkv * hd * keys + 2 * e * n * H * hd, attn_units, occ_a),
         gemm("o_proj", H * hd, d, 8 * n * d),
         ("rmsnorm2", 4.0 * n * d, 4 * n * d + e * n * d + e * d, math.ceil(n / rows), occ_e),

@@ -168,8 +168,13 @@ std::vector<KernelCost> layer_kernels(const PhaseShape& s, const PerfParams& P, 
     attn_units = (double)s.q_lens.size() * Hkv;
   }
   ks.push_back({"rmsnorm1", 4.0 * n * d, 4 * n * d + e * n * d + e * d, std::ceil(n / rows), P.occ_elem});
-  gemm("qkv", d, nq, 4 * n * nq);
-  ks.push_back({"rope_kv", 6.0 * n * (H + Hkv) * hd, 4 * n * nq + e * n * nq, std::ceil(n / rows), P.occ_elem});
+  if (e == 2 && hd == 128) {   // bf16: RoPE + KV append fused into the QKV epilogue (bf16 q / k / v out)
+    gemm("qkv", d, nq, e * n * nq);
+    ks.back().c += 6.0 * n * (H + Hkv) * hd;
+  } else {
+    gemm("qkv", d, nq, 4 * n * nq);
+    ks.push_back({"rope_kv", 6.0 * n * (H + Hkv) * hd, 4 * n * nq + e * n * nq, std::ceil(n / rows), P.occ_elem});
+  }
   ks.push_back({"attn", 4.0 * hd * H * pairs, 2 * e * Hkv * hd * keys + 2 * e * n * H * hd, attn_units, P.occ_attn});
   gemm("o_proj", H * hd, d, 8 * n * d);
   ks.push_back({"rmsnorm2", 4.0 * n * d, 4 * n * d + e * n * d + e * d, std::ceil(n / rows), P.occ_elem});

@@ -254,3 +254,35 @@ def test_step_ranges_overlapping(small_bf16, ranges):
         assert set(rows[:, 2].tolist()) <= allowed[int(rows[0, 3])]
     with pytest.raises(B.BulletError):
         S.bl.step_ranges(pre, dec, (0, 0), (0, 148), B.CORUN)   # non-empty batch, empty range
+
+
+def test_cuda_graph_replay_matches_stream_launch(small_bf16):
+    """NEXT-4: a co-run step captured into a CUDA graph (both phase streams
+    forked from the capture stream) replays to the same bits as the direct
+    launch: the per-step plan kernel re-zeroes the work counters and the split-K
+    semaphores reset themselves, so replays are self-contained."""
+    S = small_bf16
+    B = S.B
+    pre, dec = S.batches(0, 2)
+    x_pre, x_dec = pre.hidden.clone(), dec.hidden.clone()
+    sp, sd = phase_streams()
+
+    def enqueue():
+        ev = torch.cuda.Event(); ev.record(sp); sd.wait_event(ev)
+        S.bl.step(pre, dec, 64, B.CORUN, sp, sd)
+        ev2 = torch.cuda.Event(); ev2.record(sd); sp.wait_event(ev2)
+
+    enqueue()
+    torch.cuda.synchronize()
+    want = (pre.hidden.clone(), dec.hidden.clone())
+    g = torch.cuda.CUDAGraph()
+    pre.hidden.copy_(x_pre); dec.hidden.copy_(x_dec)
+    torch.cuda.synchronize()
+    with torch.cuda.graph(g, stream=sp):
+        enqueue()
+    for _ in range(2):   # capture does not execute; every replay restarts from the inputs
+        pre.hidden.copy_(x_pre); dec.hidden.copy_(x_dec)
+        torch.cuda.synchronize()
+        g.replay()
+        torch.cuda.synchronize()
+        assert torch.equal(pre.hidden, want[0]) and torch.equal(dec.hidden, want[1])

@@ -67,7 +67,12 @@ def test_layer_kernel_inventory_flops():
     shape = dict(d=4096, H=32, Hkv=8, hd=128, I=14336, elt=2, q_lens=[512, 100], ctx_lens=[0, 0])
     ks = {k[0]: k for k in PM.layer_kernels(shape, P, 148)}
     n = 612
-    assert ks["qkv"][1] == 2.0 * n * 4096 * 6144
+    # bf16 / hd 128: RoPE (6 flops per rotated pair element) rides in the QKV epilogue, no rope_kv kernel
+    assert ks["qkv"][1] == 2.0 * n * 4096 * 6144 + 6.0 * n * (32 + 8) * 128
+    assert ks["qkv"][2] == 2 * (4096 * 6144 + n * 4096) + 2 * n * 6144   # weights + A + bf16 q/k/v out
+    assert "rope_kv" not in ks
+    f32 = {k[0]: k for k in PM.layer_kernels(dict(shape, elt=4), P, 148)}
+    assert f32["qkv"][1] == 2.0 * n * 4096 * 6144 and f32["rope_kv"][1] == 6.0 * n * (32 + 8) * 128
     assert ks["o_proj"][1] == 2.0 * n * 4096 * 4096
     assert ks["gate_up"][1] == 2.0 * n * 4096 * 2 * 14336
     assert ks["down"][1] == 2.0 * n * 14336 * 4096
