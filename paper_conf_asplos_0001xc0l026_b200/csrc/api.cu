@@ -361,8 +361,16 @@ int do_rmsnorm(Ctx& c, const float* x, int n, const void* g, void* out) {
   a.x = x; a.g = g; a.out = out; a.n = n; a.d = c.h->cfg.d_model; a.eps = c.h->cfg.rms_eps;
   int rc = next_launch(c, &a.L);
   if (rc) return rc;
-  if (c.h->cfg.dtype == BULLET_DTYPE_FP32) LAUNCH(c, launch_rmsnorm<float>(a, row_grid(c, n), c.st));
-  else LAUNCH(c, launch_rmsnorm<__nv_bfloat16>(a, row_grid(c, n), c.st));
+  // warp per row (BULLET_NORM=cta: one CTA per row, the first version)
+  static const bool cta = getenv("BULLET_NORM") && !strcmp(getenv("BULLET_NORM"), "cta");
+  if (cta) {
+    if (c.h->cfg.dtype == BULLET_DTYPE_FP32) LAUNCH(c, launch_rmsnorm<float>(a, row_grid(c, n), c.st));
+    else LAUNCH(c, launch_rmsnorm<__nv_bfloat16>(a, row_grid(c, n), c.st));
+    return BULLET_OK;
+  }
+  const int per_sm = std::max(1, std::min(8, (n + 8 * c.m_sms - 1) / (8 * std::max(1, c.m_sms))));
+  if (c.h->cfg.dtype == BULLET_DTYPE_FP32) LAUNCH(c, launch_rmsnorm_warp<float>(a, c.h->n_sms * per_sm, c.st));
+  else LAUNCH(c, launch_rmsnorm_warp<__nv_bfloat16>(a, c.h->n_sms * per_sm, c.st));
   return BULLET_OK;
 }
 

@@ -82,6 +82,43 @@ __global__ void __launch_bounds__(256) k_rmsnorm(NormArgs a) {
   }
 }
 
+// Warp-per-row RMSNorm (same contract as k_rmsnorm): each warp claims a row,
+// sums x^2 over the row with shuffles only (no CTA barrier), then re-reads the
+// row (L1 hit) and writes x * inv * g.  Decode batches have few rows: one
+// claim round per warp instead of per-row CTA barriers.
+template <typename T>
+__global__ void __launch_bounds__(256) k_rmsnorm_warp(NormArgs a) {
+  if (!gate_ok(a.L.gate)) return;
+  const int lane = threadIdx.x & 31;
+  const T* g = reinterpret_cast<const T*>(a.g);
+  T* out = reinterpret_cast<T*>(a.out);
+  const int d4 = a.d / 4;
+  for (;;) {
+    int r = 0;
+    if (lane == 0) r = atomicAdd(a.L.ctr, 1);
+    r = __shfl_sync(0xffffffffu, r, 0);
+    if (r >= a.n) break;
+    if (lane == 0) log_unit(a.L, r);
+    const float4* x = reinterpret_cast<const float4*>(a.x + (size_t)r * a.d);
+    float s0 = 0.f, s1 = 0.f;
+    int i = lane;
+#pragma unroll 4
+    for (; i + 32 < d4; i += 64) {
+      const float4 u = x[i], v = x[i + 32];
+      s0 += u.x * u.x + u.y * u.y + u.z * u.z + u.w * u.w;
+      s1 += v.x * v.x + v.y * v.y + v.z * v.z + v.w * v.w;
+    }
+    if (i < d4) { const float4 u = x[i]; s0 += u.x * u.x + u.y * u.y + u.z * u.z + u.w * u.w; }
+    const float inv = rsqrtf(warp_sum(s0 + s1) / (float)a.d + a.eps);
+    T* o = out + (size_t)r * a.d;
+#pragma unroll 4
+    for (int j = lane; j < d4; j += 32) {
+      const float4 u = x[j], gg = ld4(g + 4 * j);
+      st4(o + 4 * j, make_float4(u.x * inv * gg.x, u.y * inv * gg.y, u.z * inv * gg.z, u.w * inv * gg.w));
+    }
+  }
+}
+
 // ------------------------------------------------------- RoPE + KV append
 // Token t of request r at position p = ctx[r] + (t - cu[r]).  Rotate-half
 // RoPE of q and k heads with the (cos, sin) table, round to the storage type
@@ -246,6 +283,12 @@ cudaError_t launch_gemm_simt(const T* A, const T* B, const GemmArgs& a, int grid
   return cudaGetLastError();
 }
 template <typename T>
+cudaError_t launch_rmsnorm_warp(const NormArgs& a, int grid, cudaStream_t st) {
+  if (a.d % 4) return cudaErrorInvalidValue;
+  k_rmsnorm_warp<T><<<grid, 256, 0, st>>>(a);
+  return cudaGetLastError();
+}
+template <typename T>
 cudaError_t launch_rmsnorm(const NormArgs& a, int grid, cudaStream_t st) {
   const int v = (a.d / 4 + 255) / 256;
   if (v <= 1) k_rmsnorm<T, 1><<<grid, 256, 0, st>>>(a);
@@ -274,6 +317,8 @@ cudaError_t launch_probe(int* out, int n, cudaStream_t st) {
 template cudaError_t launch_gemm_simt<float>(const float*, const float*, const GemmArgs&, int, cudaStream_t);
 template cudaError_t launch_gemm_simt<__nv_bfloat16>(const __nv_bfloat16*, const __nv_bfloat16*, const GemmArgs&, int, cudaStream_t);
 template cudaError_t launch_rmsnorm<float>(const NormArgs&, int, cudaStream_t);
+template cudaError_t launch_rmsnorm_warp<float>(const NormArgs&, int, cudaStream_t);
+template cudaError_t launch_rmsnorm_warp<__nv_bfloat16>(const NormArgs&, int, cudaStream_t);
 template cudaError_t launch_rmsnorm<__nv_bfloat16>(const NormArgs&, int, cudaStream_t);
 template cudaError_t launch_rope_kv<float>(const RopeArgs&, int, cudaStream_t);
 template cudaError_t launch_rope_kv<__nv_bfloat16>(const RopeArgs&, int, cudaStream_t);

@@ -98,6 +98,8 @@ cudaError_t launch_gemm_simt(const T* A, const T* B, const GemmArgs& a, int grid
 template <typename T>
 cudaError_t launch_rmsnorm(const NormArgs& a, int grid, cudaStream_t st);
 template <typename T>
+cudaError_t launch_rmsnorm_warp(const NormArgs& a, int grid, cudaStream_t st);
+template <typename T>
 cudaError_t launch_rope_kv(const RopeArgs& a, int grid, cudaStream_t st);
 template <typename T>
 cudaError_t launch_attn_simt(const AttnArgs& a, int grid, cudaStream_t st);
