@@ -79,6 +79,14 @@ __device__ __forceinline__ uint32_t tile_off(int row, int c) {
   return row * 256 + ((c ^ (row & 7)) << 4);
 }
 
+// KV is streamed once per launch: evict-first keeps it from displacing the
+// other phase's L2-resident activation tiles.
+__device__ __forceinline__ void cp_async16_ef(void* dst, const void* src, uint64_t pol) {
+  asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src),
+               "l"(pol)
+               : "memory");
+}
+
 struct Slot {  // one published unit
   int u, t, pos, nb;
 };
@@ -157,6 +165,8 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
   const __nv_bfloat16* pv = reinterpret_cast<const __nv_bfloat16*>(a.pool_v);
   __nv_bfloat16* og = reinterpret_cast<__nv_bfloat16*>(a.o);
   uint8_t* my = stages + warp * DEPTH * STAGE_BYTES;
+  uint64_t pol_kv;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_kv));
   const uint32_t my_s = smem_u32(my);
   const int gw = warp / GW, wl = warp % GW;   // group, index in the group
   auto my_count = [&](int nb) { return nb > wl ? (nb - wl + GW - 1) / GW : 0; };
@@ -190,8 +200,8 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
       uint8_t* dk = my + (n_issued % DEPTH) * STAGE_BYTES;
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
-        cp_async16(dk + cp_off[i], ks + 512 * i);
-        cp_async16(dk + BLK_BYTES + cp_off[i], vs + 512 * i);
+        cp_async16_ef(dk + cp_off[i], ks + 512 * i, pol_kv);
+        cp_async16_ef(dk + BLK_BYTES + cp_off[i], vs + 512 * i, pol_kv);
       }
       cp_async_commit();
       ++n_issued;

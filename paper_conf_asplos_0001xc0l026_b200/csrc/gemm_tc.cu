@@ -101,12 +101,34 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
 
 __device__ __forceinline__ float silu_f(float z) { return z / (1.0f + __expf(-z)); }
 
-// 1-D bulk copy global -> shared, completion on an mbarrier.
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+// L2 cache policies: weights stream through once per launch (evict first),
+// activation tiles are re-read by every N tile (evict last) — keeps the
+// activation band L2-resident against the weight stream.
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+// 1-D bulk copy global -> shared, completion on an mbarrier, L2 cache hint.
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint64_t pol) {
   asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
           smem_u32(dst)),
-      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+      : "memory");
+}
+// TMA 2D tile load with an L2 cache hint.
+__device__ __forceinline__ void tma_load_2d_hint(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
+                                                 uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1, {%3, %4}], [%2], %5;" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "l"(pol)
       : "memory");
 }
 
@@ -258,6 +280,7 @@ __global__ void __launch_bounds__(NT, 1)
 
   if (warp == 0) {
     if (lane == 0) {  // ---------------- scheduler + TMA producer
+      const uint64_t pol_a = policy_evict_last(), pol_b = policy_evict_first();
       int it = 0, s = 0;
       uint32_t ph = 0;
       for (;;) {
@@ -285,19 +308,19 @@ __global__ void __launch_bounds__(NT, 1)
           mbar_arrive_expect_tx(full + s, st_bytes);
 #pragma unroll
           for (int hh = 0; hh < mh; ++hh)   // rows past M are zero-filled by TMA
-            tma_load_2d(sa + hh * A_BYTES, &mapA, full + s, kb * BK, (m_blk * mh + hh) * BM);
+            tma_load_2d_hint(sa + hh * A_BYTES, &mapA, full + s, kb * BK, (m_blk * mh + hh) * BM, pol_a);
           uint8_t* sb = sa + a_bytes;
           if (a.b_packed) {   // pre-swizzled tiles: contiguous bulk copies
             const uint8_t* kbase = a.b_packed + (size_t)kb * (a.b_rows / 64) * 8192;
             if (r1 == r0 + bn / 2) {
-              bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s);
+              bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s, pol_b);
             } else {
-              bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes / 2, full + s);
-              bulk_g2s(sb + b_bytes / 2, kbase + (size_t)(r1 / 64) * 8192, b_bytes / 2, full + s);
+              bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes / 2, full + s, pol_b);
+              bulk_g2s(sb + b_bytes / 2, kbase + (size_t)(r1 / 64) * 8192, b_bytes / 2, full + s, pol_b);
             }
           } else {
-            tma_load_2d(sb, &mapB, full + s, kb * BK, r0);
-            tma_load_2d(sb + b_bytes / 2, &mapB, full + s, kb * BK, r1);
+            tma_load_2d_hint(sb, &mapB, full + s, kb * BK, r0, pol_b);
+            tma_load_2d_hint(sb + b_bytes / 2, &mapB, full + s, kb * BK, r1, pol_b);
           }
           if (++s == n_stages) { s = 0; ph ^= 1; }
         }

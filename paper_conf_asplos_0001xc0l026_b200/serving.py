@@ -23,6 +23,13 @@ Policies:
               other (BULLET_TIMESLICED), k from the model's full-GPU balance
   prefill_first  vLLM-style: while a prefill batch exists decode is paused
               (p = N); otherwise decode runs whole iterations on all SMs
+  chunked     SARATHI / SGLang chunked prefill (the paper's comparison axis,
+              P:L82-86): every iteration is ONE hybrid batch on
+              all SMs — the decode members plus a chunk of the waiting
+              prompts (token budget `chunk_tokens`, each chunk attending to
+              the prompt's earlier chunks through the block table) — advanced
+              k_full layers per cycle; a prompt's first token comes when its
+              last chunk leaves the last layer
 """
 from __future__ import annotations
 
@@ -113,14 +120,15 @@ class ServingLoop:
 
     def __init__(self, n_layers: int, n_sms: int, step, choose, policy: str, allocator: BlockAllocator,
                  slo: Slo = Slo(), prefill_layers_per_cycle: int = 1, max_prefill_tokens: int = 8192,
-                 max_decodes: int = 256, k_full: int = 4):
-        assert policy in ("bullet", "timesliced", "prefill_first")
+                 max_decodes: int = 256, k_full: int = 4, chunk_tokens: int = 2048):
+        assert policy in ("bullet", "timesliced", "prefill_first", "chunked")
         self.L, self.N = n_layers, n_sms
         self.step, self.choose, self.policy = step, choose, policy
         self.alloc, self.slo = allocator, slo
         self.lp = prefill_layers_per_cycle
         self.max_prefill_tokens, self.max_decodes, self.k_full = max_prefill_tokens, max_decodes, k_full
         self.split = (n_sms // 2, n_sms - n_sms // 2)
+        self.chunk_tokens = chunk_tokens
         self.log = []                 # per cycle: (now, p, k, prefill tokens, decodes, ms)
 
     # ------------------------------------------------------------ helpers
@@ -135,10 +143,82 @@ class ServingLoop:
                     decode_mean_ctx=float(np.mean([r.ctx for r in members])) if members else 0.0,
                     u_k=self.split[0], v_k=self.split[1])
 
+    # ------------------------------------------------------------ chunked prefill (baseline)
+    def _run_chunked(self, trace, horizon, max_cycles):
+        now, nxt = 0.0, 0
+        pending, members, done = [], [], []
+        filling = []                  # admitted prompts with tokens still to prefill: [req, tokens done]
+        d_layer, it_id, hyb = 0, 0, None
+        for _ in range(max_cycles):
+            while nxt < len(trace) and trace[nxt].arrival_ms <= now:
+                pending.append(trace[nxt]); nxt += 1
+            if d_layer == 0:          # new iteration: admit prompts, cut this iteration's chunks
+                while pending and len(members) + len(filling) < self.max_decodes:
+                    blk = self.alloc.alloc(pending[0].prompt + pending[0].out_len)
+                    if blk is None:
+                        break
+                    r = pending.pop(0); r.blocks = blk
+                    filling.append([r, 0])
+                budget = max(0, self.chunk_tokens - len(members))
+                chunks = []
+                for f in filling:
+                    if budget <= 0:
+                        break
+                    c = min(budget, f[0].prompt - f[1])
+                    if c > 0:
+                        chunks.append((f, c)); budget -= c
+                if not chunks and not members:
+                    if nxt >= len(trace) and not pending and not filling:
+                        break
+                    if nxt < len(trace):
+                        now = max(now, trace[nxt].arrival_ms)
+                        continue
+                it_id += 1
+                # prefill chunks (q > 1 first), then the decodes: one hybrid batch
+                order = sorted(chunks, key=lambda fc: fc[1] == 1)
+                reqs = [f[0] for f, _ in order] + members
+                q = [c for _, c in order] + [1] * len(members)
+                ctx = [f[1] for f, _ in order] + [r.ctx for r in members]
+                hyb = (order, list(members), reqs, q, ctx)
+            if now >= horizon:
+                break
+            order, mem, reqs, q, ctx = hyb
+            le = min(d_layer + self.k_full, self.L)
+            pw = PhaseWork(reqs, q, ctx, d_layer, le, it_id)
+            self.split = (self.N, 0)
+            ms = self.step(pw, None, self.N, "timesliced")
+            self.log.append((now, self.N, le - d_layer, sum(q) - len(mem), len(mem), ms))
+            now += ms
+            d_layer = le
+            if d_layer < self.L:
+                continue
+            d_layer = 0               # iteration complete: chunks advance, decodes emit a token
+            for f, c in order:
+                f[1] += c
+                if f[1] >= f[0].prompt:
+                    r = f[0]
+                    filling.remove(f)
+                    r.first_token_ms, r.tokens = now, 1
+                    if r.out_len <= 1:
+                        r.finish_ms = now; self.alloc.release(r.blocks); done.append(r)
+                    else:
+                        members.append(r)
+            still = []
+            for r in mem:
+                r.tokens += 1
+                if r.tokens >= r.out_len:
+                    r.finish_ms = now; self.alloc.release(r.blocks); done.append(r)
+                else:
+                    still.append(r)
+            members = still + [r for r in members if r not in mem]
+        return self.metrics(done, trace, now)
+
     # ------------------------------------------------------------ loop
     def run(self, trace: list[Request], horizon_ms: float | None = None, max_cycles: int = 10 ** 7):
         trace = sorted(trace, key=lambda r: r.arrival_ms)
         horizon = horizon_ms if horizon_ms is not None else float("inf")
+        if self.policy == "chunked":
+            return self._run_chunked(trace, horizon, max_cycles)
         now, nxt = 0.0, 0
         pending, ready, members = [], [], []
         prefill, layers_done, pre_id, dec_id = None, 0, 0, 0

@@ -7,7 +7,7 @@ trace is served under each policy and one JSON line per policy is printed:
 TTFT / normalized TTFT / TPOT percentiles, SLO attainment (Table 2 ShareGPT
 SLOs) and goodput, on virtual time = summed device time.
 
-  python scripts/serve.py --rate 60 --duration 10 --policies bullet timesliced prefill_first
+  python scripts/serve.py --rate 60 --duration 10 --policies bullet timesliced prefill_first chunked
 """
 import argparse
 import json
@@ -91,7 +91,8 @@ def main():
     ap.add_argument("--rate", type=float, default=60.0, help="requests / s (Poisson)")
     ap.add_argument("--duration", type=float, default=10.0, help="seconds of arrivals")
     ap.add_argument("--layers", type=int, default=32)
-    ap.add_argument("--policies", nargs="+", default=["bullet", "timesliced", "prefill_first"])
+    ap.add_argument("--policies", nargs="+", default=["bullet", "timesliced", "prefill_first", "chunked"])
+    ap.add_argument("--chunk-tokens", type=int, default=2048, help="chunked policy: token budget per iteration")
     ap.add_argument("--max-decodes", type=int, default=256)
     ap.add_argument("--max-prefill", type=int, default=8192)
     ap.add_argument("--blocks", type=int, default=24000)
@@ -110,7 +111,8 @@ def main():
     for pol in a.policies:
         trace = SV.poisson_trace(a.rate, a.duration, seed=a.seed)
         loop = SV.ServingLoop(a.layers, g.N, g, g.bl.choose_split, pol, SV.BlockAllocator(a.blocks),
-                              max_prefill_tokens=a.max_prefill, max_decodes=a.max_decodes, k_full=k_ts)
+                              max_prefill_tokens=a.max_prefill, max_decodes=a.max_decodes, k_full=k_ts,
+                              chunk_tokens=a.chunk_tokens)
         t0 = time.perf_counter()
         res = loop.run(trace)
         res.update(rate_req_s=a.rate, arrivals_s=a.duration, layers=a.layers, k_timesliced=k_ts,

@@ -54,7 +54,7 @@ def _run(pm, policy, rate=40.0, dur=1.0):
     return trace, rec, alloc, loop, res
 
 
-@pytest.mark.parametrize("policy", ["bullet", "timesliced", "prefill_first"])
+@pytest.mark.parametrize("policy", ["bullet", "timesliced", "prefill_first", "chunked"])
 def test_every_request_completes_and_blocks_return(pm, policy):
     trace, rec, alloc, loop, res = _run(pm, policy)
     assert res["finished"] == len(trace) > 10
@@ -64,7 +64,7 @@ def test_every_request_completes_and_blocks_return(pm, policy):
     json.dumps(res)   # serialisable metrics
 
 
-@pytest.mark.parametrize("policy", ["bullet", "timesliced", "prefill_first"])
+@pytest.mark.parametrize("policy", ["bullet", "timesliced", "prefill_first", "chunked"])
 def test_layer_progress_and_decode_membership(pm, policy):
     trace, rec, alloc, loop, res = _run(pm, policy)
     pre, dec = {}, {}
@@ -92,6 +92,39 @@ def test_policy_rules(pm):
     both = [(p, dw) for pw, dw, p, mode, *_ in rec.calls if pw is not None and dw is not None]
     assert both and all(0 < p < N for p, _ in both)                           # a real split
     assert all(p % 2 == 0 for pw, dw, p, mode, *_ in rec.calls)              # TPC granularity
+
+
+def test_chunked_policy_batches():
+    """Chunked prefill: every cycle is one hybrid batch on all SMs (prefill
+    chunks with q > 1 first, then q = 1 rows), within the token budget; a
+    prompt's chunks cover it exactly once, in order (ctx = tokens before)."""
+    trace = SV.poisson_trace(40.0, 1.0, seed=3)
+    rec = Recorder(pm_fixture_cache())
+    loop = SV.ServingLoop(L, N, rec, None, "chunked", SV.BlockAllocator(8000), max_decodes=128, k_full=4,
+                          chunk_tokens=512)
+    loop.run(trace)
+    covered = {}
+    for pw, dw, p, mode, pinfo, _ in rec.calls:
+        assert dw is None and mode == "timesliced" and p == N
+        assert sum(pw.q_lens) <= max(512, sum(1 for q in pw.q_lens if q == 1))
+        ones = [q == 1 for q in pw.q_lens]
+        assert ones == sorted(ones)                     # q > 1 rows first
+        if pw.layer_begin == 0:
+            for r, q, c in zip(pw.reqs, pw.q_lens, pw.ctx_lens):
+                if c < r.prompt:                        # a prefill chunk of r
+                    assert covered.get(r.rid, 0) == c
+                    covered[r.rid] = c + q
+    assert all(covered[r.rid] == r.prompt for r in trace)
+
+
+_PM = []
+
+
+def pm_fixture_cache():
+    if not _PM:
+        pj = os.path.join(ROOT, "profiles", "perf_params_b200.json")
+        _PM.append(PerfModel(Model.of(synth.MODELS["llama3.1-8b"]), N, open(pj).read() if os.path.exists(pj) else None))
+    return _PM[0]
 
 
 def test_trace_is_seeded_and_shaped():
