@@ -33,6 +33,7 @@ constexpr int CMB_FLOATS = HD * 8 + 16;      // O^T[128][8] + m[8] + l[8] per wa
 constexpr int THREADS = (NCW + 1) * 32;
 constexpr int QSLOT_BYTES = 8 * HD * 2;      // Q rows of up to 8 heads (bf16)
 constexpr int MAXNB = 512;                   // blocks per unit held in smem (8k tokens)
+constexpr int NS_MAX = 8;                    // unit slots (2 per consumer group, up to 4 groups)
 static_assert(CMB_FLOATS * 4 <= STAGE_BYTES, "merge record must fit in one stage");
 
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
@@ -98,21 +99,22 @@ struct Slot {  // one published unit
 template <int NG>
 __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
   constexpr int GW = NCW / NG;
+  constexpr int NS = 2 * NG;   // unit slots: each group holds <= 2 units (current + next)
   if (!gate_ok(a.L.gate)) return;
   extern __shared__ __align__(128) uint8_t smem[];
   uint8_t* stages = smem;                                                      // [NCW][DEPTH][STAGE]
-  uint8_t* qbuf = stages + NCW * DEPTH * STAGE_BYTES;                          // [4][QSLOT_BYTES]
-  int* btbuf = reinterpret_cast<int*>(qbuf + 4 * QSLOT_BYTES);                 // [4][MAXNB]
-  Slot* uq = reinterpret_cast<Slot*>(btbuf + 4 * MAXNB);
-  uint64_t* uqf = reinterpret_cast<uint64_t*>(uq + 4);
-  uint64_t* uqe = uqf + 4;
-  int* rec_stage = reinterpret_cast<int*>(uqe + 4);                            // [NCW]
+  uint8_t* qbuf = stages + NCW * DEPTH * STAGE_BYTES;                          // [NS_MAX][QSLOT_BYTES]
+  int* btbuf = reinterpret_cast<int*>(qbuf + NS_MAX * QSLOT_BYTES);            // [NS_MAX][MAXNB]
+  Slot* uq = reinterpret_cast<Slot*>(btbuf + NS_MAX * MAXNB);
+  uint64_t* uqf = reinterpret_cast<uint64_t*>(uq + NS_MAX);
+  uint64_t* uqe = uqf + NS_MAX;
+  int* rec_stage = reinterpret_cast<int*>(uqe + NS_MAX);                       // [NCW]
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int grp = a.H / a.Hkv;
   const int units = (a.n_tok - a.tok_base) * a.Hkv;   // decode rows are tokens [tok_base, n_tok)
   if (threadIdx.x == 0) {
-    for (int i = 0; i < 4; ++i) { mbar_init(uqf + i, 1); mbar_init(uqe + i, GW); }
+    for (int i = 0; i < NS; ++i) { mbar_init(uqf + i, 1); mbar_init(uqe + i, GW); }
     mbar_fence_init();
   }
   __syncthreads();
@@ -121,11 +123,11 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
     const __nv_bfloat16* qg = reinterpret_cast<const __nv_bfloat16*>(a.q);
     int n_end = 0;
     for (int it = 0;; ++it) {
-      const int slot = it & 3;
+      const int slot = it % NS;
       // a group holds at most 2 units (current + next, so its warps can
       // prefetch across the boundary): unit it waits for unit it - 2 NG of
       // the same group (load balance across CTAs; 4 slots = 2 NG)
-      if (lane == 0 && it >= 2 * NG) mbar_wait(uqe + ((it - 2 * NG) & 3), ((it - 2 * NG) >> 2) & 1);
+      if (lane == 0 && it >= NS) mbar_wait(uqe + ((it - NS) % NS), ((it - NS) / NS) & 1);
       __syncwarp();
       int u = 0;
       if (lane == 0) u = n_end ? units : atomicAdd(a.L.ctr, 1);
@@ -186,9 +188,9 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
   int cur_nb = -1, cur_g = 0, cur_u = 0;   // cached slot of unit iu (-1: not read yet)
   auto fill = [&](int limit, int cap) {
     while (n_issued - n_cons < cap && iu <= limit) {
-      const int sl = iu & 3;
+      const int sl = iu % NS;
       if (cur_nb < 0) {
-        mbar_wait(uqf + sl, (iu >> 2) & 1);
+        mbar_wait(uqf + sl, (iu / NS) & 1);
         const Slot X = uq[sl];
         cur_u = X.u; cur_nb = my_count(X.nb); cur_g = X.u >= 0 ? X.u % a.Hkv : 0;
       }
@@ -210,8 +212,8 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
   };
 
   for (int it = gw;; it += NG) {
-    const int slot = it & 3;
-    mbar_wait(uqf + slot, (it >> 2) & 1);
+    const int slot = it % NS;
+    mbar_wait(uqf + slot, (it / NS) & 1);
     const Slot S = uq[slot];
     if (S.u < 0) break;
     const int g = S.u % a.Hkv;
@@ -338,25 +340,28 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
 }
 
 size_t attn_decode_smem_bytes() {
-  return (size_t)NCW * DEPTH * STAGE_BYTES + 4 * QSLOT_BYTES + 4 * MAXNB * 4 + 4 * sizeof(Slot) +
-         8 * 8 + NCW * 4;
+  return (size_t)NCW * DEPTH * STAGE_BYTES + NS_MAX * QSLOT_BYTES + NS_MAX * MAXNB * 4 + NS_MAX * sizeof(Slot) +
+         2 * NS_MAX * 8 + NCW * 4;
 }
 int attn_decode_max_blocks() { return MAXNB; }
 
-// `ng` consumer groups per CTA (1 or 2; BULLET_DEC_GROUPS overrides).
+// `ng` consumer groups per CTA (1, 2 or 4; BULLET_DEC_GROUPS overrides).
 cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStream_t st) {
   const size_t smem = attn_decode_smem_bytes();
   static const int forced = getenv("BULLET_DEC_GROUPS") ? atoi(getenv("BULLET_DEC_GROUPS")) : 0;
-  if (forced == 1 || forced == 2) ng = forced;
+  if (forced == 1 || forced == 2 || forced == 4) ng = forced;
   static bool set = false;
   if (!set) {
     cudaError_t e = cudaFuncSetAttribute(k_attn_decode_tc<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(k_attn_decode_tc<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(k_attn_decode_tc<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     set = true;
   }
   if (ng == 1) k_attn_decode_tc<1><<<grid, THREADS, smem, st>>>(a);
+  else if (ng == 4) k_attn_decode_tc<4><<<grid, THREADS, smem, st>>>(a);
   else k_attn_decode_tc<2><<<grid, THREADS, smem, st>>>(a);
   return cudaGetLastError();
 }

@@ -101,12 +101,17 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
 
 __device__ __forceinline__ float silu_f(float z) { return z / (1.0f + __expf(-z)); }
 
-// L2 cache policies: weights stream through once per launch (evict first),
-// activation tiles are re-read by every N tile (evict last) — keeps the
-// activation band L2-resident against the weight stream.
+// L2 cache policies: activation tiles are re-read by every N tile (evict
+// last); decode-sized GEMMs (one M tile) stream each weight tile once (evict
+// first), prefill GEMMs re-read it for every M tile of the band (normal).
 __device__ __forceinline__ uint64_t policy_evict_first() {
   uint64_t p;
   asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_normal() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
   return p;
 }
 __device__ __forceinline__ uint64_t policy_evict_last() {
@@ -280,7 +285,7 @@ __global__ void __launch_bounds__(NT, 1)
 
   if (warp == 0) {
     if (lane == 0) {  // ---------------- scheduler + TMA producer
-      const uint64_t pol_a = policy_evict_last(), pol_b = policy_evict_first();
+      const uint64_t pol_a = policy_evict_last(), pol_b = a.b_evict_first ? policy_evict_first() : policy_evict_normal();
       int it = 0, s = 0;
       uint32_t ph = 0;
       for (;;) {

@@ -28,6 +28,7 @@ struct GemmArgs {
   float* partials;    // tail split: [tail units][mh][bn/4][128][4] (float4 groups interleaved by row)
   int* tile_sems;     // tail split: [tail tiles], zero between launches (self-resetting)
   const uint8_t* b_packed;  // B pre-packed by pack_weight (else B comes through mapB)
+  int b_evict_first;        // one M tile: the weight stream is used once (L2 evict-first)
   int b_rows;               // rows of B (packed layout stride)
   // EPI_QKV (bf16, head_dim 128; fuses SURVEY §8a S3 into S2): the epilogue
   // adds the bias, rotates q / k heads (rotate-half RoPE from the (cos, sin)
