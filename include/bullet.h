@@ -172,7 +172,8 @@ typedef struct {
 /* Create a handle on the current CUDA device.  Probes the live SM ids
  * (%smid) and orders them (sigma).  `nccl_uids`: for tp_size > 1, 2 x 128
  * bytes (ncclUniqueId of the prefill and the decode communicator, same on
- * every rank), else NULL.  `perf_params_json`: fitted perf-model
+ * every rank) for the NCCL all-reduce, or NULL for the fused peer-memory
+ * all-reduce (PEER mode, bullet_tp_connect below); NULL if tp_size = 1.  `perf_params_json`: fitted perf-model
  * parameters, or NULL for the unfitted roofline (d = p = 1).
  * Unsupported shapes (BULLET_EUNSUPPORTED): bf16 with d_model, H*hd or d_ff
  * not multiples of 64; (H+2Hkv)*hd, d_model or d_ff not multiples of 64;
@@ -255,11 +256,54 @@ int bullet_profile_read(bullet_handle *h, int32_t *kind, int32_t *phase, int32_t
 int bullet_launch_count(const bullet_handle *h, long long *n);
 
 /* Block until all work the handle enqueued has finished; surfaces
- * asynchronous CUDA / NCCL errors. */
+ * asynchronous CUDA / NCCL errors and peer all-reduce timeouts (ENCCL). */
 int bullet_sync(bullet_handle *h);
 
 /* ncclGetUniqueId into out (128 bytes), for tensor-parallel setup. */
 int bullet_nccl_unique_id(void *out128);
+
+/* ---- Fused tensor-parallel all-reduce over peer memory (
+ * north_star (4): "an NCCL all-reduce over NVLink after the attention-out and
+ * MLP-down projections", here fused into those GEMMs and smid-gated).
+ * A handle created with tp_size > 1 and nccl_uids == NULL is in PEER mode:
+ * bullet_create allocates one symmetric device region (same layout on every
+ * rank: per phase two fp32 partial buffers [max_tokens][d_model], the fp32
+ * residual stream `hidden` [max_tokens][d_model], ready / done counters).
+ * Before the first step every rank connects to all ranks' regions (its own
+ * included) with bullet_tp_connect (device addresses valid in this process:
+ * same-process ranks, e.g. ranks simulated on SM partitions of one GPU) or
+ * bullet_tp_connect_ipc (cudaIpcMemHandle_t of every rank, one process per
+ * GPU; rank order).  In a step, the O-proj and down GEMMs of rank r write
+ * fp32 partials into r's region and the same kernels then reduce rank r's
+ * column slab [r d/n, (r+1) d/n) of every 16-row chunk as soon as all ranks'
+ * partials of its 128-row block are ready (x + partial_0 + ... +
+ * partial_{n-1}, fixed rank order: deterministic), store it into every
+ * rank's hidden and return once all slabs have arrived.
+ * Every batch passed to bullet_step must use the phase's symmetric hidden
+ * (bullet_tp_hidden) as its `d_hidden` (else EINVAL); all ranks must make the
+ * same sequence of steps with the same batch shapes (as with NCCL).  bf16
+ * only.  A peer that never arrives makes the waiting kernels give up after
+ * 20 s; bullet_sync then returns BULLET_ENCCL. */
+
+/* Device address of this handle's symmetric region (PEER mode). */
+int bullet_tp_base(const bullet_handle *h, void **d_base);
+
+/* cudaIpcMemHandle_t (64 bytes) of this handle's symmetric region. */
+int bullet_tp_ipc_handle(const bullet_handle *h, void *out64);
+
+/* Connect to the tp_size regions `d_bases` (rank order; d_bases[tp_rank]
+ * must be this handle's own).  Errors: EINVAL (not PEER mode, wrong own
+ * base, null), EUNSUPPORTED (tp_size > 8). */
+int bullet_tp_connect(bullet_handle *h, void *const *d_bases);
+
+/* Open the other ranks' regions from tp_size x 64 bytes of IPC handles (rank
+ * order, as gathered from every rank's bullet_tp_ipc_handle) and connect.
+ * The handle closes them in bullet_destroy.  Errors: ECUDA (open failed). */
+int bullet_tp_connect_ipc(bullet_handle *h, const void *handles);
+
+/* The phase's (0 prefill, 1 decode) symmetric residual stream, fp32
+ * [cfg max tokens of the phase][d_model]: the `d_hidden` of PEER-mode steps. */
+int bullet_tp_hidden(const bullet_handle *h, int phase, float **d_hidden);
 
 const char *bullet_last_error(void);
 void bullet_destroy(bullet_handle *h);

@@ -88,7 +88,8 @@ def lib():
                      "bullet_step", "bullet_step_ranges", "bullet_model_predict", "bullet_choose_split",
                      "bullet_set_smid_log", "bullet_sync", "bullet_nccl_unique_id", "bullet_op_gemm",
                      "bullet_op_rmsnorm", "bullet_op_rope_kv", "bullet_op_attention",
-                     "bullet_profile_read", "bullet_launch_count"):
+                     "bullet_profile_read", "bullet_launch_count", "bullet_tp_base", "bullet_tp_ipc_handle",
+                     "bullet_tp_connect", "bullet_tp_connect_ipc", "bullet_tp_hidden"):
             getattr(L, name).restype = c_int
         L.bullet_create.argtypes = [ctypes.POINTER(ModelCfg), ctypes.POINTER(KvPool), c_void_p,
                                     ctypes.c_char_p, ctypes.POINTER(c_void_p)]
@@ -110,6 +111,11 @@ def lib():
                                           ctypes.POINTER(c_int)]
         L.bullet_launch_count.argtypes = [c_void_p, ctypes.POINTER(ctypes.c_longlong)]
         L.bullet_nccl_unique_id.argtypes = [c_void_p]
+        L.bullet_tp_base.argtypes = [c_void_p, ctypes.POINTER(c_void_p)]
+        L.bullet_tp_ipc_handle.argtypes = [c_void_p, c_void_p]
+        L.bullet_tp_connect.argtypes = [c_void_p, ctypes.POINTER(c_void_p)]
+        L.bullet_tp_connect_ipc.argtypes = [c_void_p, c_void_p]
+        L.bullet_tp_hidden.argtypes = [c_void_p, c_int, ctypes.POINTER(c_void_p)]
         L.bullet_destroy.argtypes = [c_void_p]
         L.bullet_destroy.restype = None
         L.bullet_op_gemm.argtypes = [c_void_p, c_int, c_void_p, c_int, c_int, c_void_p, c_int, c_int,
@@ -144,6 +150,15 @@ def nccl_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(128)
     _check(lib().bullet_nccl_unique_id(buf))
     return buf.raw
+
+
+class _DeviceArray:
+    """__cuda_array_interface__ view of library-owned device memory (the
+    PEER-mode symmetric hidden), so torch.as_tensor can alias it."""
+
+    def __init__(self, ptr: int, shape, typestr="<f4"):
+        self.__cuda_array_interface__ = {"data": (ptr, False), "shape": tuple(shape), "typestr": typestr,
+                                         "version": 3, "strides": None}
 
 
 class Batch:
@@ -294,6 +309,32 @@ class Bullet:
 
     def sync(self):
         _check(lib().bullet_sync(self.h))
+
+    # ---- fused tensor-parallel all-reduce over peer memory (PEER mode: tp_size > 1, no nccl_uids)
+    def tp_base(self) -> int:
+        p = c_void_p()
+        _check(lib().bullet_tp_base(self.h, ctypes.byref(p)))
+        return p.value
+
+    def tp_ipc_handle(self) -> bytes:
+        buf = ctypes.create_string_buffer(64)
+        _check(lib().bullet_tp_ipc_handle(self.h, buf))
+        return buf.raw
+
+    def tp_connect(self, bases):
+        arr = (c_void_p * len(bases))(*bases)
+        _check(lib().bullet_tp_connect(self.h, arr))
+
+    def tp_connect_ipc(self, handles: bytes):
+        buf = ctypes.create_string_buffer(handles, len(handles))
+        _check(lib().bullet_tp_connect_ipc(self.h, buf))
+
+    def tp_hidden(self, phase: int, n_tokens: int) -> torch.Tensor:
+        """The phase's symmetric fp32 residual stream [n_tokens][d_model] (a
+        view of library memory): PEER-mode batches must use it as `hidden`."""
+        p = c_void_p()
+        _check(lib().bullet_tp_hidden(self.h, int(phase), ctypes.byref(p)))
+        return torch.as_tensor(_DeviceArray(p.value, (n_tokens, self.model.d_model)), device="cuda")
 
     def profile_read(self, cap=1 << 16):
         """[(kind name, phase, layer, ms)] of launches made with PROFILE since the last read."""

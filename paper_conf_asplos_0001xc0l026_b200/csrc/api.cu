@@ -110,6 +110,32 @@ struct PhaseWS {
 };
 
 constexpr int GRAN = 2;            // split granularity: one TPC
+
+// Symmetric region of the fused peer all-reduce (PEER mode, include/bullet.h):
+// per phase two fp32 partial buffers, the fp32 hidden, ready counters
+// [tp][max_rb], done counters [max_rb], expected-value bases [2][max_rb], an
+// error word.  Offsets depend only on the model cfg: identical on every rank.
+struct SymLayout {
+  size_t part[2], hid, ready, done, base, err, end;
+  int max_rb;
+};
+inline size_t al256(size_t x) { return (x + 255) & ~size_t(255); }
+SymLayout sym_layout(const bullet_model_cfg& c, int phase) {
+  SymLayout L{};
+  size_t off = 0;
+  for (int p = 0; p <= phase; ++p) {
+    const size_t T = std::max(1, p == 0 ? c.max_prefill_tokens : c.max_decode_tokens);
+    const size_t f = al256(T * c.d_model * sizeof(float));
+    L.max_rb = (int)((T + 127) / 128);
+    L.part[0] = off; L.part[1] = off + f; L.hid = off + 2 * f; L.ready = off + 3 * f;
+    L.done = L.ready + al256((size_t)c.tp_size * L.max_rb * 8);
+    L.base = L.done + al256((size_t)L.max_rb * 8);
+    L.err = L.base + al256((size_t)2 * L.max_rb * 8);
+    off = L.err + 256;
+  }
+  L.end = off;
+  return L;
+}
 constexpr int N_TILE_SEMS = 2048;
 
 }  // namespace
@@ -134,6 +160,12 @@ struct bullet_handle {
   int launch_seq = 0;
   PerfParams perf;
   ncclComm_t comm[2] = {nullptr, nullptr};
+  // fused peer all-reduce (PEER mode): own symmetric region, every rank's base
+  bool peer_mode = false, peer_connected = false;
+  uint8_t* sym = nullptr;
+  size_t sym_bytes = 0;
+  std::vector<uint8_t*> peer_base;
+  std::vector<void*> ipc_opened;
   cudaEvent_t ev_ts = nullptr;
   bool host_only = false;  // bullet_perf_create: perf model only
   // BULLET_PROFILE: events around every launch
@@ -240,7 +272,7 @@ struct QkvEpi {   // EPI_QKV destinations
 
 int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, int silu_half,
             const void* bias, const float* resid, void* out, int ldo, const uint8_t* Bp = nullptr,
-            const QkvEpi* qe = nullptr) {
+            const QkvEpi* qe = nullptr, const ArArgs* ar = nullptr) {
   bullet_handle* h = c.h;
   if (M == 0) return BULLET_OK;
   GemmArgs a;
@@ -256,6 +288,13 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   }
   int rc = next_launch(c, &a.L);
   if (rc) return rc;
+  if (ar) {   // fused peer all-reduce (bf16 only, checked at create): its own unit counter
+    PhaseWS& P = h->ph[c.phase];
+    if (c.op || epi != EPI_F32) return set_err(BULLET_EINVAL, "fused all-reduce: step GEMMs with EPI_F32 only");
+    if (P.next_ctr >= P.n_counters) return set_err(BULLET_ENOMEM, "work counters exhausted");
+    a.ar = *ar;
+    a.ar.ctr = P.counters + P.next_ctr++;
+  }
   if (h->cfg.dtype == BULLET_DTYPE_FP32) {
     if (K % 16) return set_err(BULLET_EUNSUPPORTED, "fp32 GEMM needs K %% 16 == 0");
     a.bn = 64; a.mh = 1; a.splits = 1; a.n_full = 0; a.band = 1;
@@ -494,6 +533,25 @@ int allreduce(Ctx& c, float* buf, size_t count) {
   return BULLET_OK;
 }
 
+// All-reduce arguments of a phase's row-parallel GEMM: every rank's partial
+// buffer `buf`, hidden and counters (PEER mode, connected).
+ArArgs make_ar(const bullet_handle* h, int phase, int buf) {
+  ArArgs r;
+  memset(&r, 0, sizeof r);
+  const SymLayout L = sym_layout(h->cfg, phase);
+  r.n = h->cfg.tp_size; r.rank = h->cfg.tp_rank; r.max_rb = L.max_rb;
+  for (int s = 0; s < r.n; ++s) {
+    uint8_t* b = h->peer_base[s];
+    r.part[s] = reinterpret_cast<float*>(b + L.part[buf]);
+    r.hid[s] = reinterpret_cast<float*>(b + L.hid);
+    r.ready[s] = reinterpret_cast<unsigned long long*>(b + L.ready);
+    r.done[s] = reinterpret_cast<unsigned long long*>(b + L.done);
+  }
+  r.base = reinterpret_cast<unsigned long long*>(h->sym + L.base);
+  r.err = reinterpret_cast<int*>(h->sym + L.err);
+  return r;
+}
+
 // One decoder layer of one phase (DESIGN.md §2 steps S1-S9).
 int run_layer(Ctx& c, const bullet_batch* b, int layer) {
   bullet_handle* h = c.h;
@@ -521,19 +579,32 @@ int run_layer(Ctx& c, const bullet_batch* b, int layer) {
   }
   c.kind = BULLET_K_ATTN;
   if ((rc = do_attention(c, b, layer, P.q, P.o, 0))) return rc;                             // S4
-  // S5: x1 = x + o W_o^T.  Under TP the non-lead ranks write their partial
-  // into hidden and the fp32 all-reduce restores x + sum of partials (S9).
+  // S5: x1 = x + o W_o^T.  Under TP (NCCL) the non-lead ranks write their
+  // partial into hidden and the fp32 all-reduce restores x + sum of partials
+  // (S9); in PEER mode the GEMM writes its partial to the symmetric buffer
+  // and reduces in the same kernel (NEXT-2).
   c.kind = BULLET_K_OPROJ;
-  if ((rc = do_gemm(c, (!tp || lead) ? EPI_RESID : EPI_F32, P.o, n, H * hd, w.w_o, d, 0, nullptr,
-                    b->d_hidden, b->d_hidden, d, wp ? wp->o : nullptr))) return rc;
-  c.kind = BULLET_K_ALLREDUCE;
-  if (tp && (rc = allreduce(c, b->d_hidden, (size_t)n * d))) return rc;
+  if (h->peer_mode) {
+    const ArArgs ar = make_ar(h, c.phase, 0);
+    if ((rc = do_gemm(c, EPI_F32, P.o, n, H * hd, w.w_o, d, 0, nullptr, nullptr, ar.part[ar.rank], d,
+                      wp ? wp->o : nullptr, nullptr, &ar))) return rc;
+  } else {
+    if ((rc = do_gemm(c, (!tp || lead) ? EPI_RESID : EPI_F32, P.o, n, H * hd, w.w_o, d, 0, nullptr,
+                      b->d_hidden, b->d_hidden, d, wp ? wp->o : nullptr))) return rc;
+    c.kind = BULLET_K_ALLREDUCE;
+    if (tp && (rc = allreduce(c, b->d_hidden, (size_t)n * d))) return rc;
+  }
   c.kind = BULLET_K_RMSNORM2;
   if ((rc = do_rmsnorm(c, b->d_hidden, n, w.g_mlp, P.h))) return rc;                        // S6
   c.kind = BULLET_K_GATE_UP;
   if ((rc = do_gemm(c, EPI_SILU, P.h, n, d, w.w_gate_up, 2 * I, I, nullptr, nullptr, P.act, I,
                     wp ? wp->gu : nullptr))) return rc;  // S7
   c.kind = BULLET_K_DOWN;
+  if (h->peer_mode) {   // S8 + S9 fused (partial buffer 1: consecutive all-reduces alternate)
+    const ArArgs ar = make_ar(h, c.phase, 1);
+    return do_gemm(c, EPI_F32, P.act, n, I, w.w_down, d, 0, nullptr, nullptr, ar.part[ar.rank], d,
+                   wp ? wp->down : nullptr, nullptr, &ar);
+  }
   if ((rc = do_gemm(c, (!tp || lead) ? EPI_RESID : EPI_F32, P.act, n, I, w.w_down, d, 0, nullptr,
                     b->d_hidden, b->d_hidden, d, wp ? wp->down : nullptr))) return rc;       // S8
   c.kind = BULLET_K_ALLREDUCE;
@@ -552,6 +623,11 @@ int validate_batch(const bullet_handle* h, const bullet_batch* b, int phase) {
     return set_err(BULLET_EINVAL, "%s: cu_seqlens must run 0..n_tokens", nm);
   if (b->n_tokens > h->ph[phase].max_tok)
     return set_err(BULLET_ENOMEM, "%s: %d tokens > max %d", nm, b->n_tokens, h->ph[phase].max_tok);
+  if (h->peer_mode) {
+    if (!h->peer_connected) return set_err(BULLET_EINVAL, "PEER mode: bullet_tp_connect first");
+    if ((const uint8_t*)b->d_hidden != h->sym + sym_layout(h->cfg, phase).hid)
+      return set_err(BULLET_EINVAL, "%s: PEER mode needs the symmetric hidden (bullet_tp_hidden)", nm);
+  }
   if (b->layer_begin < 0 || b->layer_end > h->cfg.n_layers || b->layer_begin > b->layer_end)
     return set_err(BULLET_EINVAL, "%s: layer range [%d,%d)", nm, b->layer_begin, b->layer_end);
   for (int l = b->layer_begin; l < b->layer_end; ++l)
@@ -634,7 +710,11 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
   if (c.n_heads / c.n_kv_heads > 8) return set_err(BULLET_EUNSUPPORTED, "GQA group > 8");
   if (pool->block_size != 16) return set_err(BULLET_EUNSUPPORTED, "block_size must be 16");
   if (pool->n_blocks <= 0 || !pool->d_k || !pool->d_v) return set_err(BULLET_EINVAL, "kv pool");
-  if (c.tp_size > 1 && !nccl_uids) return set_err(BULLET_EINVAL, "tp_size > 1 needs nccl_uids");
+  if (c.tp_size > 1 && !nccl_uids) {   // PEER mode: fused all-reduce over peer memory
+    if (c.dtype != BULLET_DTYPE_BF16) return set_err(BULLET_EUNSUPPORTED, "fused all-reduce: bf16 only");
+    if (c.tp_size > AR_MAX_RANKS) return set_err(BULLET_EUNSUPPORTED, "fused all-reduce: tp_size <= %d", AR_MAX_RANKS);
+    if (c.d_model % (4 * c.tp_size)) return set_err(BULLET_EUNSUPPORTED, "fused all-reduce: d_model %% (4 tp) != 0");
+  }
 
   int dev;
   CK(cudaGetDevice(&dev));
@@ -711,7 +791,7 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
     PhaseWS& P = h->ph[p];
     P.max_tok = p == 0 ? c.max_prefill_tokens : c.max_decode_tokens;
     const size_t T = std::max(1, P.max_tok);
-    P.n_counters = 8 * c.n_layers + 16;
+    P.n_counters = 10 * c.n_layers + 16;
     P.partial_floats = (size_t)2 * h->n_sms * 128 * 256;
     bool ok = cudaMalloc(&P.qkv, T * nq * sizeof(float)) == cudaSuccess &&
               cudaMalloc(&P.q, T * c.n_heads * c.head_dim * h->elt) == cudaSuccess &&
@@ -740,8 +820,16 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
     if (!h->perf.parse(perf_params_json, &err)) return fail(set_err(BULLET_EINVAL, "%s", err.c_str()));
   }
 
+  // ---- fused peer all-reduce: the symmetric region (zeroed counters)
+  if (c.tp_size > 1 && !nccl_uids) {
+    h->peer_mode = true;
+    h->sym_bytes = sym_layout(c, 1).end;
+    if (cudaMalloc(&h->sym, h->sym_bytes) != cudaSuccess) return fail(set_err(BULLET_ENOMEM, "symmetric region"));
+    if (cudaMemset(h->sym, 0, h->sym_bytes) != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess)
+      return fail(set_err(BULLET_ECUDA, "symmetric region init"));
+  }
   // ---- tensor parallelism: one communicator per phase (concurrent streams)
-  if (c.tp_size > 1) {
+  if (c.tp_size > 1 && nccl_uids) {
     if (!g_nccl.load()) return fail(set_err(BULLET_ENCCL, "libnccl.so.2 not loadable"));
     for (int p = 0; p < 2; ++p) {
       ncclUniqueId id;
@@ -954,6 +1042,12 @@ int bullet_sync(bullet_handle* h) {
   if (!h) return set_err(BULLET_EINVAL, "null");
   if (h->host_only) return BULLET_OK;
   CK(cudaDeviceSynchronize());
+  if (h->peer_mode)
+    for (int p = 0; p < 2; ++p) {
+      int e = 0;
+      CK(cudaMemcpy(&e, h->sym + sym_layout(h->cfg, p).err, sizeof e, cudaMemcpyDeviceToHost));
+      if (e) return set_err(BULLET_ENCCL, "fused all-reduce (phase %d): a peer did not arrive within 20 s", p);
+    }
   return BULLET_OK;
 }
 
@@ -968,6 +1062,8 @@ void bullet_destroy(bullet_handle* h) {
     cudaFree(P.n_tiles); cudaFree(P.tok);
     if (h->comm[p] && g_nccl.commDestroy) g_nccl.commDestroy(h->comm[p]);
   }
+  for (void* p : h->ipc_opened) cudaIpcCloseMemHandle(p);
+  cudaFree(h->sym);
   cudaFree(h->rope_cs);
   for (auto& P : h->wp) cudaFree(P.base);
   cudaFree(h->op_pack);
@@ -975,6 +1071,62 @@ void bullet_destroy(bullet_handle* h) {
   if (h->ev_ts) cudaEventDestroy(h->ev_ts);
   for (auto e : h->ev_pool) cudaEventDestroy(e);
   delete h;
+}
+
+// ------------------------------------------------ fused peer all-reduce setup
+int bullet_tp_base(const bullet_handle* h, void** base) {
+  if (!h || !base) return set_err(BULLET_EINVAL, "null");
+  if (!h->peer_mode) return set_err(BULLET_EINVAL, "not in PEER mode (tp_size > 1, nccl_uids NULL)");
+  *base = h->sym;
+  return BULLET_OK;
+}
+
+int bullet_tp_ipc_handle(const bullet_handle* h, void* out64) {
+  if (!h || !out64) return set_err(BULLET_EINVAL, "null");
+  if (!h->peer_mode) return set_err(BULLET_EINVAL, "not in PEER mode");
+  cudaIpcMemHandle_t m;
+  CK(cudaIpcGetMemHandle(&m, h->sym));
+  static_assert(sizeof m == 64, "cudaIpcMemHandle_t is 64 bytes");
+  memcpy(out64, &m, sizeof m);
+  return BULLET_OK;
+}
+
+int bullet_tp_connect(bullet_handle* h, void* const* bases) {
+  if (!h || !bases) return set_err(BULLET_EINVAL, "null");
+  if (!h->peer_mode) return set_err(BULLET_EINVAL, "not in PEER mode");
+  const int n = h->cfg.tp_size;
+  if (bases[h->cfg.tp_rank] != h->sym) return set_err(BULLET_EINVAL, "bases[tp_rank] is not this handle's region");
+  for (int s = 0; s < n; ++s)
+    if (!bases[s]) return set_err(BULLET_EINVAL, "null base of rank %d", s);
+  h->peer_base.assign(n, nullptr);
+  for (int s = 0; s < n; ++s) h->peer_base[s] = (uint8_t*)bases[s];
+  h->peer_connected = true;
+  return BULLET_OK;
+}
+
+int bullet_tp_connect_ipc(bullet_handle* h, const void* handles) {
+  if (!h || !handles) return set_err(BULLET_EINVAL, "null");
+  if (!h->peer_mode) return set_err(BULLET_EINVAL, "not in PEER mode");
+  const int n = h->cfg.tp_size;
+  std::vector<void*> bases(n, nullptr);
+  for (int s = 0; s < n; ++s) {
+    if (s == h->cfg.tp_rank) { bases[s] = h->sym; continue; }
+    cudaIpcMemHandle_t m;
+    memcpy(&m, (const char*)handles + 64 * s, sizeof m);
+    void* p = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&p, m, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) return set_err(BULLET_ECUDA, "cudaIpcOpenMemHandle (rank %d): %s", s, cudaGetErrorString(e));
+    h->ipc_opened.push_back(p);
+    bases[s] = p;
+  }
+  return bullet_tp_connect(h, bases.data());
+}
+
+int bullet_tp_hidden(const bullet_handle* h, int phase, float** hidden) {
+  if (!h || !hidden || phase < 0 || phase > 1) return set_err(BULLET_EINVAL, "bad argument");
+  if (!h->peer_mode) return set_err(BULLET_EINVAL, "not in PEER mode");
+  *hidden = reinterpret_cast<float*>(h->sym + sym_layout(h->cfg, phase).hid);
+  return BULLET_OK;
 }
 
 // ---------------------------------------------------------- op-level entries

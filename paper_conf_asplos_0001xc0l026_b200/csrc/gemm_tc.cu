@@ -224,6 +224,92 @@ __device__ __forceinline__ void epi_qkv(const GemmArgs& a, int m, int col, float
   }
 }
 
+// ---------------------------------------------------------------- fused all-reduce (kernels.h ArArgs)
+__device__ __forceinline__ void red_release_sys_add(unsigned long long* p, unsigned long long v) {
+  asm volatile("red.release.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void fence_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// Spin until *p >= target.  Bounded: after 20 s (a dead or absent peer) the
+// error word is set and the wait gives up, so a broken peer set cannot hang
+// the GPU; bullet_sync reports it.
+__device__ __forceinline__ void wait_ge(const unsigned long long* p, unsigned long long target, int* err) {
+  if (ld_acquire_sys(p) >= target) return;
+  const uint64_t t0 = globaltimer_ns();
+  while (ld_acquire_sys(p) < target) {
+    __nanosleep(100);
+    if (*reinterpret_cast<volatile int*>(err)) return;
+    if (globaltimer_ns() - t0 > 20000000000ull) { atomicExch(err, 1); return; }
+  }
+}
+// Called by the 128 epilogue threads once the tile's rows are stored: count
+// the tile's columns in ready[rank][rb] of every rank for each 128-row block.
+__device__ __forceinline__ void ar_signal(const GemmArgs& a, int m_blk, int mh, int et) {
+  fence_sys();               // this thread's partial stores, before the counts
+  named_bar_sync(1, 128);
+  if (et < a.ar.n) {
+    for (int hh = 0; hh < mh; ++hh) {
+      const int rb = m_blk * mh + hh;
+      if (rb * BM >= a.M) break;
+      red_release_sys_add(a.ar.ready[et] + (size_t)a.ar.rank * a.ar.max_rb + rb, (unsigned long long)a.bn);
+    }
+  }
+}
+// After the CTA's GEMM units: reduce units, then wait units (kernels.h).
+__device__ __forceinline__ void ar_phase(const GemmArgs& a, int* s_u) {
+  const ArArgs& r = a.ar;
+  const int n = r.n, M = a.M, N4 = a.N / 4, slab4 = N4 / n, c4 = r.rank * slab4;
+  constexpr int CPB = BM / AR_ROWS;   // chunks per 128-row block
+  const int n_chunks = (M + AR_ROWS - 1) / AR_ROWS, n_rb = (M + BM - 1) / BM;
+  for (;;) {
+    if (threadIdx.x == 0) *s_u = atomicAdd(r.ctr, 1);
+    __syncthreads();
+    const int u = *s_u;
+    __syncthreads();
+    if (u >= n_chunks + n_rb) break;
+    if (u < n_chunks) {
+      const int rb = u / CPB;
+      if ((int)threadIdx.x < n)   // every rank's partial of block rb is complete
+        wait_ge(r.ready[r.rank] + (size_t)threadIdx.x * r.max_rb + rb, __ldcg(r.base + rb) + (unsigned long long)a.N,
+                r.err);
+      __syncthreads();
+      const int row0 = u * AR_ROWS, items = min(AR_ROWS, M - row0) * slab4;
+      for (int i = threadIdx.x; i < items; i += NT) {
+        const size_t off = (size_t)(row0 + i / slab4) * N4 + c4 + i % slab4;
+        float4 p[AR_MAX_RANKS];
+#pragma unroll
+        for (int s = 0; s < AR_MAX_RANKS; ++s)
+          if (s < n) p[s] = __ldcg(reinterpret_cast<const float4*>(r.part[s]) + off);
+        float4 acc = __ldcg(reinterpret_cast<const float4*>(r.hid[r.rank]) + off);   // x
+#pragma unroll
+        for (int s = 0; s < AR_MAX_RANKS; ++s)   // x + partial_0 + ... in rank order
+          if (s < n) { acc.x += p[s].x; acc.y += p[s].y; acc.z += p[s].z; acc.w += p[s].w; }
+#pragma unroll
+        for (int s = 0; s < AR_MAX_RANKS; ++s)
+          if (s < n) __stcg(reinterpret_cast<float4*>(r.hid[s]) + off, acc);
+      }
+      fence_sys();
+      __syncthreads();
+      if ((int)threadIdx.x < n) red_release_sys_add(r.done[threadIdx.x] + rb, 1ull);
+    } else if (threadIdx.x == 0) {   // wait unit: all n slabs of block rb are here
+      const int rb = u - n_chunks, chunks = min(CPB, n_chunks - rb * CPB);
+      const unsigned long long t = __ldcg(r.base + r.max_rb + rb) + (unsigned long long)n * chunks;
+      wait_ge(r.done[r.rank] + rb, t, r.err);
+      __stcg(r.base + r.max_rb + rb, t);
+      __stcg(r.base + rb, __ldcg(r.base + rb) + (unsigned long long)a.N);
+    }
+  }
+}
+
 }  // namespace
 
 int gemm_tc_stages(int bn, int mh) {
@@ -408,6 +494,7 @@ __global__ void __launch_bounds__(NT, 1)
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(acce + as);
+        if (a.ar.n) ar_signal(a, m_blk, mh, et);
       } else {
         // partial tile stored as float4 groups interleaved by row per half
         // ([hh][col/4][row][4]): a thread's 4 consecutive columns are one
@@ -436,7 +523,8 @@ __global__ void __launch_bounds__(NT, 1)
           *s_last = last;
         }
         named_bar_sync(1, 128);
-        if (*s_last) {
+        const bool last = *s_last;
+        if (last) {
           __threadfence();
           const float4* T0 = reinterpret_cast<const float4*>(a.partials) + (size_t)(ui.tail - ui.sp) * tile_f4 + et;
           // sum 32 columns of all splits (fixed split order: deterministic),
@@ -478,11 +566,16 @@ __global__ void __launch_bounds__(NT, 1)
               epi_store(a, m, col0 + c * 32, v, w);
             }
           }
+          if (a.ar.n) ar_signal(a, m_blk, mh, et);
         }
       }
       if (++as == n_acc) { as = 0; aph ^= 1; }
       ++it;
     }
+  }
+  if (a.ar.n) {   // fused all-reduce: this CTA's GEMM units are done
+    __syncthreads();
+    ar_phase(a, s_last + 1);
   }
   tc_fence_before();
   __syncthreads();

@@ -10,6 +10,31 @@ enum { EPI_F32 = 0, EPI_RESID = 1, EPI_SILU = 2, EPI_QKV = 3 };
 // step): x = position p = ctx[r] + (t - cu[r]), y = slot = bt[r][p / B] * B + p % B.
 typedef int2 TokInfo;
 
+// Fused tensor-parallel all-reduce over peer memory (SURVEY §8f NEXT-2,
+// DESIGN.md §8).  A row-parallel GEMM (O-proj, down) of rank `rank` writes its
+// fp32 partial into its symmetric partial buffer and, per finished 128-row
+// block, adds the block's column count to ready[rank][rb] on every rank.
+// When its own tiles run out, each CTA turns to reduce units: 16 rows of
+// this rank's column slab [rank N/n, (rank+1) N/n) — wait until every rank's
+// partial of the block is ready, sum x + partial_0 + ... + partial_{n-1} in
+// rank order (deterministic), store the result into every rank's hidden and
+// count the chunk in done[rb] on every rank — then to wait units (one per
+// row block) that return once all n slabs of the block have landed here.  The
+// kernel ends with hidden = x + sum of partials on every rank.  Counters only
+// grow; `base` holds the values expected before this all-reduce
+// ([0, max_rb): ready, [max_rb, 2 max_rb): done), advanced by the wait units.
+constexpr int AR_MAX_RANKS = 8, AR_ROWS = 16;
+struct ArArgs {
+  int n, rank, max_rb;                              // n = 0: off
+  float* part[AR_MAX_RANKS];                        // rank s's partial buffer [M][N] (this all-reduce's parity)
+  float* hid[AR_MAX_RANKS];                         // rank s's hidden [M][N]
+  unsigned long long* ready[AR_MAX_RANKS];          // rank s's ready counters [n][max_rb]
+  unsigned long long* done[AR_MAX_RANKS];           // rank s's done counters [max_rb]
+  unsigned long long* base;                         // local [2][max_rb]
+  int* ctr;                                         // reduce / wait unit counter (zero at launch)
+  int* err;                                         // set on a peer timeout
+};
+
 // C[M x N] = A[M x K] . B[N x K]^T with a fused epilogue (all row-major).
 struct GemmArgs {
   int M, N, K;        // N = B rows used (2 x output cols for EPI_SILU)
@@ -38,6 +63,7 @@ struct GemmArgs {
   const float2* cs;         // [max_pos][64] (cos, sin)
   const TokInfo* tok;       // [M]
   int H, Hkv, kvB;
+  ArArgs ar;                // EPI_F32 into ar.part[ar.rank] + the fused all-reduce (ar.n > 1)
   Launch L;
 };
 

@@ -6,9 +6,12 @@ QKV and gate/up are column-parallel (rank r owns query heads
 O-proj and down are row-parallel (the matching input columns).  Inside
 `bullet_step` the non-lead ranks write their fp32 partial products into the
 residual stream and an in-place ncclAllReduce(float32, sum) after S5 and S8
-restores x + sum of partials.  KV pools shard by kv head; block
-tables are replicated.  torch.distributed is used only to launch ranks and to
-broadcast the two ncclUniqueIds (one communicator per phase)."""
+restores x + sum of partials.  In PEER mode (no ncclUniqueIds)
+the O-proj / down GEMMs reduce over the ranks' symmetric buffers themselves
+(fused, smid-gated); `connect_peers` exchanges the
+cudaIpcMemHandles.  KV pools shard by kv head; block tables are replicated.
+torch.distributed is used only to launch ranks and to exchange these few
+bytes."""
 from __future__ import annotations
 
 import torch
@@ -59,3 +62,19 @@ def nccl_uids(group=None, make=nccl_unique_id) -> bytes:
     obj = [make() + make() if rank == 0 else None]
     dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group else 0, group=group)
     return obj[0]
+
+
+def gather_bytes(blob: bytes, group=None) -> bytes:
+    """Every rank's `blob` (equal lengths), concatenated in rank order."""
+    import torch.distributed as dist
+    out = [None] * dist.get_world_size(group)
+    dist.all_gather_object(out, blob, group=group)
+    if len({len(b) for b in out}) != 1:
+        raise ValueError("ranks sent blobs of different lengths")
+    return b"".join(out)
+
+
+def connect_peers(bl, group=None):
+    """PEER mode, one process per GPU: exchange the symmetric regions'
+    cudaIpcMemHandles and connect (bullet_tp_connect_ipc)."""
+    bl.tp_connect_ipc(gather_bytes(bl.tp_ipc_handle(), group))

@@ -77,7 +77,9 @@ def _worker(rank, tp, port, q):
         out_tp = _rank_partials(rank, tp, q_lens, ctx, lay, x, w, pk, pv)
         ref = O.layer_forward(_cfg(M), w, pk.copy(), pv.copy(), q_lens, ctx, lay.block_table, x)
         uids = parallel.nccl_uids(make=lambda: bytes([7]) * 128)
-        q.put((rank, float(np.abs(out_tp - ref).max()), len(uids), uids[:4]))
+        # PEER mode bootstrap: every rank's 64-byte IPC handle, in rank order
+        handles = parallel.gather_bytes(bytes([rank + 1]) * 64)
+        q.put((rank, float(np.abs(out_tp - ref).max()), len(uids), uids[:4], handles))
     finally:
         dist.destroy_process_group()
 
@@ -94,9 +96,10 @@ def test_tp2_sharded_layer_equals_unsharded_oracle():
     for p in ps:
         p.join(60)
         assert p.exitcode == 0
-    for rank, err, n, head in res:
+    for rank, err, n, head, handles in res:
         assert err < 1e-9, (rank, err)      # same bf16 rounding points, fp64 sums
         assert n == 256 and head == bytes([7]) * 4
+        assert handles == b"".join(bytes([r + 1]) * 64 for r in range(tp))
 
 
 def test_shard_shapes_all_tp_configs():
