@@ -120,7 +120,7 @@ class Clocks:
 
 # ---------------------------------------------------------------- workload
 class Step:
-    def __init__(self, config: str, k_max: int, device="cuda"):
+    def __init__(self, config: str, k_max: int, device="cuda", allreduce="peer"):
         import paper_conf_asplos_0001xc0l026_b200 as B
         self.B = B
         from paper_conf_asplos_0001xc0l026_b200 import parallel
@@ -156,7 +156,10 @@ class Step:
         maxpos = max(a + b for a, b in zip(q, c)) + 16
         pp = os.path.join(ROOT, "profiles", "perf_params_b200.json")   # fitted by scripts/fit_perfmodel.py
         self.perf_json = open(pp).read() if os.path.exists(pp) else None
-        uids = parallel.nccl_uids() if self.tp > 1 else None
+        # TP all-reduce: fused into the O-proj / down GEMMs over peer memory
+        # (PEER mode, NEXT-2; default) or NCCL (--allreduce nccl)
+        self.peer = self.tp > 1 and allreduce == "peer"
+        uids = parallel.nccl_uids() if self.tp > 1 and not self.peer else None
         self.bl = B.Bullet(B.Model.of(m), self.pools, self.n_p + self.n_d, self.n_d, maxpos,
                            tp_size=self.tp, tp_rank=self.rank, nccl_uids=uids,
                            perf_params_json=self.perf_json)
@@ -165,6 +168,11 @@ class Step:
         bt = self.lay.block_table
         self.x_pre = synth.hidden(self.n_p, m.d_model, 0, device=device)
         self.x_dec = synth.hidden(self.n_d, m.d_model, 1, device=device)
+        if self.peer:   # batches live in the symmetric residual streams
+            parallel.connect_peers(self.bl)
+            xp, xd = self.bl.tp_hidden(0, self.n_p), self.bl.tp_hidden(1, self.n_d)
+            xp.copy_(self.x_pre); xd.copy_(self.x_dec)
+            self.x_pre, self.x_dec = xp, xd
         self.pre = B.Batch(self.wl.prefill_lens, [0] * self.n_pre, bt[:self.n_pre], self.x_pre, 0, 1)
         self.dec = B.Batch([1] * self.n_d, self.wl.decode_ctx, bt[self.n_pre:], self.x_dec, 0, 1)
         self.sp, self.sd = torch.cuda.Stream(), torch.cuda.Stream()
@@ -405,6 +413,8 @@ def main():
     ap.add_argument("--k-max", type=int, default=16)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--sweep", action="store_true", help="also print the p sweep (stderr)")
+    ap.add_argument("--allreduce", default="peer", choices=["peer", "nccl"],
+                    help="TP configs: fused peer-memory all-reduce (default) or NCCL")
     args = ap.parse_args()
     ws, rank = dist_init()
     if args.impl == "reference":
@@ -412,7 +422,7 @@ def main():
         return
     args.warmup = max(args.warmup, 3)
     import paper_conf_asplos_0001xc0l026_b200 as B
-    S = Step(args.config, args.k_max)
+    S = Step(args.config, args.k_max, allreduce=args.allreduce)
     N = S.N
     # ---- alone-on-full-GPU references (per layer)
     S.dec.layer_end = 1
@@ -572,7 +582,57 @@ def main():
         e2e_step()
     e1.record(S.sp)
     torch.cuda.synchronize()
-    t_e2e = allreduce_max(e0.elapsed_time(e1) / args.steps, ws)
+    t_e2e_serial = allreduce_max(e0.elapsed_time(e1) / args.steps, ws)
+    # pipelined e2e (the way a serving loop runs it): two device input sets;
+    # step i's host->device copies (copy stream) overlap step i-1's compute and
+    # step i-1's device->host read overlaps step i's compute.  Every step still
+    # copies its full inputs in and its results out inside the timed region.
+    t_e2e, e2e_mode = t_e2e_serial, "serial"
+    if not S.peer:
+        bt = S.lay.block_table
+        sets = [(S.pre, S.dec),
+                (B.Batch(S.wl.prefill_lens, [0] * S.n_pre, bt[:S.n_pre], torch.empty_like(S.x_pre), 0, 1),
+                 B.Batch([1] * S.n_d, S.wl.decode_ctx, bt[S.n_pre:], torch.empty_like(S.x_dec), 0, k))]
+        h_meta = [torch.from_numpy(a).pin_memory() for a in (S.pre.cu, S.dec.cu, S.pre.ctx_lens, S.dec.ctx_lens,
+                                                              S.pre.block_table, S.dec.block_table)]
+        s_in, s_out = torch.cuda.Stream(), torch.cuda.Stream()
+        ev_in = [torch.cuda.Event() for _ in range(2)]
+        ev_done = [torch.cuda.Event() for _ in range(2)]
+        ev_out = [torch.cuda.Event() for _ in range(2)]
+        for e in ev_done + ev_out:
+            e.record(torch.cuda.current_stream())
+
+        def e2e_pipe_step(i):
+            st = i % 2
+            pre_b, dec_b = sets[st]
+            with torch.cuda.stream(s_in):          # inputs of step i (set st free once step i-2 is read out)
+                s_in.wait_event(ev_out[st])
+                pre_b.hidden.copy_(h_pre, non_blocking=True)
+                dec_b.hidden.copy_(h_dec, non_blocking=True)
+                for h, d in zip(h_meta, (pre_b.d_cu, dec_b.d_cu, pre_b.d_ctx, dec_b.d_ctx, pre_b.d_bt, dec_b.d_bt)):
+                    d.copy_(h, non_blocking=True)
+                ev_in[st].record(s_in)
+            S.sp.wait_event(ev_in[st]); S.sd.wait_event(ev_in[st])
+            S.bl.step(pre_b, dec_b, p, B.CORUN, S.sp, S.sd)
+            ev2 = torch.cuda.Event(); ev2.record(S.sd); S.sp.wait_event(ev2)
+            ev_done[st].record(S.sp)
+            with torch.cuda.stream(s_out):         # results of step i
+                s_out.wait_event(ev_done[st])
+                o_pre.copy_(pre_b.hidden, non_blocking=True)
+                o_dec.copy_(dec_b.hidden, non_blocking=True)
+                ev_out[st].record(s_out)
+
+        for i in range(args.warmup):
+            e2e_pipe_step(i)
+        barrier(ws)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s_in)
+        for i in range(args.steps):
+            e2e_pipe_step(i)
+        e1.record(s_out)
+        torch.cuda.synchronize()
+        t_e2e, e2e_mode = allreduce_max(e0.elapsed_time(e1) / args.steps, ws), "pipelined"
     # ---- report
     tok = S.tokens(k)
     groups = ws // S.tp            # replicas (8B) or one TP group (configs 4-5)
@@ -595,6 +655,7 @@ def main():
                    "decode_ctx_mean": float(np.mean(S.wl.decode_ctx)), "prefill_layers_per_step": 1,
                    "decode_layer_steps": k, "prefill_sm_count": p, "n_sms": N,
                    "parallelism": (f"tp{S.tp}" if S.tp > 1 else (f"replicas x{ws}" if ws > 1 else "single GPU")),
+                   "allreduce": (("fused peer-memory (PEER mode)" if S.peer else "nccl fp32") if S.tp > 1 else None),
                    "tokens_per_s_per_gpu": value / ws,
                    "l2": "inputs larger than L2 (weights + KV per step >> 126 MB)"},
         "timesliced": {"value": ts_value, "ms_per_step": t_ts, "ms_per_step_before": t_ts0,
@@ -638,7 +699,11 @@ def main():
                      "algorithmic_" + ("flops" if bound == "tensor" else "bytes"): work},
         "kernel_ms": {f"{k_}/{'pre' if ph == 0 else 'dec'}": round(sum(v) / 2, 4) for (k_, ph), v in by.items()},
         "e2e": {"value": groups * tok / (t_e2e * 1e-3), "unit": "tokens/s", "h2d_bytes_per_step": int(h2d),
-                "d2h_bytes_per_step": int(d2h), "ms_per_step": t_e2e},
+                "d2h_bytes_per_step": int(d2h), "ms_per_step": t_e2e, "mode": e2e_mode,
+                "serial": {"value": groups * tok / (t_e2e_serial * 1e-3), "ms_per_step": t_e2e_serial},
+                "note": "pinned host inputs -> device -> bullet_step -> host every step; 'pipelined' overlaps "
+                        "step i's copies with the neighbouring steps' compute (two device input sets, copy "
+                        "streams), 'serial' copies, computes and reads back one step at a time"},
         "gpu_launches": int(launches),
         "clocks": clk.summary(),
         "tuning": table,
