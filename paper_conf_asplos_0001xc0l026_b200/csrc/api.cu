@@ -241,12 +241,14 @@ int next_launch(Ctx& c, Launch* L) {
   L->launch_id = c.h->launch_seq++;
   L->phase = c.phase;
   if (c.op) {
-    CK(cudaMemsetAsync(c.h->op_ctr, 0, sizeof(int), c.st));
+    CK(cudaMemsetAsync(c.h->op_ctr, 0, 2 * sizeof(int), c.st));
     L->ctr = c.h->op_ctr;
+    L->burn = c.h->op_ctr + 1;
   } else {
     PhaseWS& P = c.h->ph[c.phase];
-    if (P.next_ctr >= P.n_counters) return set_err(BULLET_ENOMEM, "work counters exhausted");
+    if (P.next_ctr + 2 > P.n_counters) return set_err(BULLET_ENOMEM, "work counters exhausted");
     L->ctr = P.counters + P.next_ctr++;
+    L->burn = P.counters + P.next_ctr++;
   }
   return BULLET_OK;
 }
@@ -723,6 +725,11 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
   if (prop.major != 10) return set_err(BULLET_EUNSUPPORTED, "needs an sm_100 (Blackwell) GPU, got sm_%d%d", prop.major, prop.minor);
   int rc = get_encode();
   if (rc) return rc;
+  for (auto pre : {preload_attn_decode, preload_attn_prefill5, preload_attn_tc, preload_attn_simt,
+                   preload_elementwise, preload_gemm_tc, preload_stream}) {
+    cudaError_t e = pre();
+    if (e != cudaSuccess) return set_err(BULLET_ECUDA, "kernel preload: %s", cudaGetErrorString(e));
+  }
 
   bullet_handle* h = new bullet_handle();
   h->cfg = c;
@@ -791,7 +798,7 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
     PhaseWS& P = h->ph[p];
     P.max_tok = p == 0 ? c.max_prefill_tokens : c.max_decode_tokens;
     const size_t T = std::max(1, P.max_tok);
-    P.n_counters = 10 * c.n_layers + 16;
+    P.n_counters = 20 * c.n_layers + 32;
     P.partial_floats = (size_t)2 * h->n_sms * 128 * 256;
     bool ok = cudaMalloc(&P.qkv, T * nq * sizeof(float)) == cudaSuccess &&
               cudaMalloc(&P.q, T * c.n_heads * c.head_dim * h->elt) == cudaSuccess &&
@@ -808,7 +815,7 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
     cudaMemset(P.tile_sems, 0, N_TILE_SEMS * sizeof(int));
     cudaMemset(P.counters, 0, P.n_counters * sizeof(int));
   }
-  if (cudaMalloc(&h->op_ctr, sizeof(int)) != cudaSuccess) return fail(set_err(BULLET_ENOMEM, "op ctr"));
+  if (cudaMalloc(&h->op_ctr, 2 * sizeof(int)) != cudaSuccess) return fail(set_err(BULLET_ENOMEM, "op ctr"));
   if (cudaEventCreateWithFlags(&h->ev_ts, cudaEventDisableTiming) != cudaSuccess)
     return fail(set_err(BULLET_ECUDA, "event"));
   if (cudaDeviceSynchronize() != cudaSuccess) return fail(set_err(BULLET_ECUDA, "init sync"));

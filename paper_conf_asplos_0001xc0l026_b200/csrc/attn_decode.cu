@@ -100,7 +100,7 @@ template <int NG>
 __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
   constexpr int GW = NCW / NG;
   constexpr int NS = 2 * NG;   // unit slots: each group holds <= 2 units (current + next)
-  if (!gate_ok(a.L.gate)) return;
+  if (!gate_enter(a.L)) return;
   extern __shared__ __align__(128) uint8_t smem[];
   uint8_t* stages = smem;                                                      // [NCW][DEPTH][STAGE]
   uint8_t* qbuf = stages + NCW * DEPTH * STAGE_BYTES;                          // [NS_MAX][QSLOT_BYTES]
@@ -364,6 +364,14 @@ cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStrea
   else if (ng == 4) k_attn_decode_tc<4><<<grid, THREADS, smem, st>>>(a);
   else k_attn_decode_tc<2><<<grid, THREADS, smem, st>>>(a);
   return cudaGetLastError();
+}
+
+cudaError_t preload_attn_decode() {
+  cudaFuncAttributes f;
+  cudaError_t e = cudaFuncGetAttributes(&f, k_attn_decode_tc<1>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_attn_decode_tc<2>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_attn_decode_tc<4>);
+  return e;
 }
 
 }  // namespace bl

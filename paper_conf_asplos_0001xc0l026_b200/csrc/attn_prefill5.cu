@@ -210,7 +210,7 @@ __device__ __forceinline__ void load_kv_tile(uint8_t* dst, const __nv_bfloat16* 
 }  // namespace
 
 __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
-  if (!gate_ok(a.L.gate)) return;
+  if (!gate_enter(a.L)) return;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = smem_raw;
   if (smem_u32(sm) & 1023) __trap();   // swizzle atoms need 1024-byte alignment
@@ -498,6 +498,11 @@ cudaError_t launch_attn_prefill5(const AttnArgs& a, int grid, cudaStream_t st) {
   }
   k_attn_prefill5<<<grid, NT, SMEM_BYTES, st>>>(a);
   return cudaGetLastError();
+}
+
+cudaError_t preload_attn_prefill5() {
+  cudaFuncAttributes f;
+  return cudaFuncGetAttributes(&f, k_attn_prefill5);
 }
 
 }  // namespace bl

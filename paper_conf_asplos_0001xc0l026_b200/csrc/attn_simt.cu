@@ -19,7 +19,7 @@ constexpr int WARPS = 4;
 
 template <typename T, int HD, int HH>
 __global__ void __launch_bounds__(128) k_attn_simt(AttnArgs a) {
-  if (!gate_ok(a.L.gate)) return;
+  if (!gate_enter(a.L)) return;
   constexpr int EPC = 16 / sizeof(T);           // elements per 16-byte chunk
   constexpr int CPR = HD / EPC;                 // chunks per key row
   constexpr int SWZ = (CPR < 16 ? CPR : 16) - 1;
@@ -234,6 +234,24 @@ cudaError_t launch_attn_simt(const AttnArgs& a, int grid, cudaStream_t st) {
     if (hh == 4) return launch_one<T, 64, 4>(a, grid, st);
   }
   return cudaErrorInvalidValue;
+}
+
+template <typename T>
+static cudaError_t preload_simt_t() {
+  cudaFuncAttributes f;
+  const void* k[] = {(const void*)k_attn_simt<T, 128, 1>, (const void*)k_attn_simt<T, 128, 2>,
+                     (const void*)k_attn_simt<T, 128, 3>, (const void*)k_attn_simt<T, 128, 4>,
+                     (const void*)k_attn_simt<T, 64, 1>, (const void*)k_attn_simt<T, 64, 2>,
+                     (const void*)k_attn_simt<T, 64, 3>, (const void*)k_attn_simt<T, 64, 4>};
+  for (const void* p : k) {
+    cudaError_t e = cudaFuncGetAttributes(&f, p);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+cudaError_t preload_attn_simt() {
+  cudaError_t e = preload_simt_t<float>();
+  return e == cudaSuccess ? preload_simt_t<__nv_bfloat16>() : e;
 }
 
 template cudaError_t launch_attn_simt<float>(const AttnArgs&, int, cudaStream_t);

@@ -68,7 +68,7 @@ __device__ __forceinline__ void cp_async16_zfill(void* dst, const void* src, boo
 }  // namespace
 
 __global__ void __launch_bounds__(128) k_attn_prefill_tc(AttnArgs a) {
-  if (!gate_ok(a.L.gate)) return;
+  if (!gate_enter(a.L)) return;
   extern __shared__ __align__(128) uint8_t sm[];
   uint8_t* Qs = sm;
   uint8_t* Ks = sm + TILE_BYTES;          // [2][64][128]
@@ -252,6 +252,11 @@ cudaError_t launch_attn_prefill_tc(const AttnArgs& a, int grid, cudaStream_t st)
   }
   k_attn_prefill_tc<<<grid, 128, smem, st>>>(a);
   return cudaGetLastError();
+}
+
+cudaError_t preload_attn_tc() {
+  cudaFuncAttributes f;
+  return cudaFuncGetAttributes(&f, k_attn_prefill_tc);
 }
 
 }  // namespace bl

@@ -22,6 +22,7 @@ struct Gate {
 struct Launch {
   Gate gate;
   int* ctr;        // work counter, zero at launch
+  int* burn;       // CTAs that left out of range (zero at launch; nullable)
   int32_t* log;    // smid log (nullable): [0] = count, then {launch, unit, smid, phase}
   int log_cap;
   int launch_id;
@@ -37,6 +38,19 @@ __device__ __forceinline__ uint32_t smid() {
 __device__ __forceinline__ bool gate_ok(const Gate& g) {
   uint32_t s = smid();
   return s < 256 && ((g.m[s >> 5] >> (s & 31)) & 1u);
+}
+
+// Kernel entry: a CTA on one of the phase's SMs works; one elsewhere leaves
+// at once — unless every other CTA of the grid already left that way (they
+// all landed outside the range, e.g. on SMs another phase or rank freed for
+// a moment): then this last CTA works where it is, so a launch can never end
+// with its units unprocessed (correctness never depends on CTA placement).
+__device__ __forceinline__ bool gate_enter(const Launch& L) {
+  if (gate_ok(L.gate)) return true;
+  if (!L.burn) return false;
+  int last = 0;   // (no shared memory: kernels align their dynamic smem base)
+  if (threadIdx.x == 0) last = atomicAdd(L.burn, 1) == (int)(gridDim.x * gridDim.y * gridDim.z) - 1;
+  return __syncthreads_or(last) != 0;
 }
 
 __device__ __forceinline__ void log_unit(const Launch& L, int unit) {

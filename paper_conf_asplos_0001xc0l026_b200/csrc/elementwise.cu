@@ -39,7 +39,7 @@ __device__ __forceinline__ void st2(__nv_bfloat16* p, float a, float b) {
 // the output type (oracle rounding point R1 / R4).
 template <typename T, int VPT>
 __global__ void __launch_bounds__(256) k_rmsnorm(NormArgs a) {
-  if (!gate_ok(a.L.gate)) return;
+  if (!gate_enter(a.L)) return;
   __shared__ int s_u;
   __shared__ float s_red[8];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -88,7 +88,7 @@ __global__ void __launch_bounds__(256) k_rmsnorm(NormArgs a) {
 // claim round per warp instead of per-row CTA barriers.
 template <typename T>
 __global__ void __launch_bounds__(256) k_rmsnorm_warp(NormArgs a) {
-  if (!gate_ok(a.L.gate)) return;
+  if (!gate_enter(a.L)) return;
   const int lane = threadIdx.x & 31;
   const T* g = reinterpret_cast<const T*>(a.g);
   T* out = reinterpret_cast<T*>(a.out);
@@ -127,7 +127,7 @@ __global__ void __launch_bounds__(256) k_rmsnorm_warp(NormArgs a) {
 // (float2 loads, 2-element stores) and copies four v elements.
 template <typename T>
 __global__ void __launch_bounds__(256) k_rope_kv(RopeArgs a) {
-  if (!gate_ok(a.L.gate)) return;
+  if (!gate_enter(a.L)) return;
   __shared__ int s_u;
   const int tid = threadIdx.x;
   const int half = a.hd / 2, hp = half / 2;  // pair-of-pairs per head
@@ -172,7 +172,7 @@ __global__ void __launch_bounds__(256) k_rope_kv(RopeArgs a) {
 template <typename T>
 __global__ void __launch_bounds__(256) k_gemm_simt(const T* __restrict__ A, const T* __restrict__ B,
                                                    GemmArgs a) {
-  if (!gate_ok(a.L.gate)) return;
+  if (!gate_enter(a.L)) return;
   __shared__ float As[16][68], Bs[16][68], Us[16][68];
   __shared__ int s_u;
   const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
@@ -312,6 +312,27 @@ cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st) {
 cudaError_t launch_probe(int* out, int n, cudaStream_t st) {
   k_probe<<<n, 32, 0, st>>>(out, n);
   return cudaGetLastError();
+}
+
+template <typename T>
+static cudaError_t preload_elt_t() {
+  cudaFuncAttributes f;
+  const void* k[] = {(const void*)k_gemm_simt<T>, (const void*)k_rmsnorm_warp<T>, (const void*)k_rope_kv<T>,
+                     (const void*)k_rmsnorm<T, 1>, (const void*)k_rmsnorm<T, 2>, (const void*)k_rmsnorm<T, 4>,
+                     (const void*)k_rmsnorm<T, 8>};
+  for (const void* p : k) {
+    cudaError_t e = cudaFuncGetAttributes(&f, p);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+cudaError_t preload_elementwise() {
+  cudaFuncAttributes f;
+  cudaError_t e = cudaFuncGetAttributes(&f, k_plan);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_probe);
+  if (e == cudaSuccess) e = preload_elt_t<float>();
+  if (e == cudaSuccess) e = preload_elt_t<__nv_bfloat16>();
+  return e;
 }
 
 template cudaError_t launch_gemm_simt<float>(const float*, const float*, const GemmArgs&, int, cudaStream_t);

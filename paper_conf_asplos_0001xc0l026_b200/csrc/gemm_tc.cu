@@ -326,7 +326,7 @@ template <int mh>
 __global__ void __launch_bounds__(NT, 1)
     k_gemm_tc(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
               GemmArgs a, int n_stages) {
-  if (!gate_ok(a.L.gate)) return;  // not this phase's SM: touch nothing
+  if (!gate_enter(a.L)) return;  // not this phase's SM: touch nothing
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~uintptr_t(1023));
@@ -624,6 +624,14 @@ cudaError_t launch_gemm_tc(const CUtensorMap& mapA, const CUtensorMap& mapB, con
   if (a.mh == 2) k_gemm_tc<2><<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn, 2));
   else k_gemm_tc<1><<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn, 1));
   return cudaGetLastError();
+}
+
+cudaError_t preload_gemm_tc() {
+  cudaFuncAttributes f;
+  cudaError_t e = cudaFuncGetAttributes(&f, k_gemm_tc<1>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_gemm_tc<2>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_pack_weight);
+  return e;
 }
 
 }  // namespace bl

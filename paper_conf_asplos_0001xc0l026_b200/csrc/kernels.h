@@ -139,6 +139,18 @@ cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);   // grid sized to 
 cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_probe(int* out_smid, int n, cudaStream_t st);
 
+// Lazy module loading (CUDA default) loads a kernel at its first launch
+// with a device-wide synchronisation, which can deadlock kernels that wait
+// on kernels of another stream (the fused all-reduce): load every kernel at
+// bullet_create instead.
+cudaError_t preload_attn_decode();
+cudaError_t preload_attn_prefill5();
+cudaError_t preload_attn_tc();
+cudaError_t preload_attn_simt();
+cudaError_t preload_elementwise();
+cudaError_t preload_gemm_tc();
+cudaError_t preload_stream();
+
 constexpr int ATTN_TC_BQ = 128;   // query rows per prefill attention tile (plan granularity)
 constexpr int ROWS_PER_UNIT = 8;  // rows per work unit of row-wise kernels
 

@@ -23,7 +23,7 @@ constexpr int BULK = 32768, NB = 6;
 }  // namespace
 
 __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
-  if (!gate_ok(a.L.gate)) return;
+  if (!gate_enter(a.L)) return;
   extern __shared__ __align__(128) uint8_t sm[];
   __shared__ int s_u;
   __shared__ uint64_t bars[NB];
@@ -154,6 +154,11 @@ cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st) {
   if (e != cudaSuccess) return e;
   k_stream<<<grid, 512, smem, st>>>(a);
   return cudaGetLastError();
+}
+
+cudaError_t preload_stream() {
+  cudaFuncAttributes f;
+  return cudaFuncGetAttributes(&f, k_stream);
 }
 
 }  // namespace bl

@@ -26,7 +26,7 @@ bl = B.Bullet(B.Model.of(m), pools, 8192, 8192, 8192)
 wg = {k: (None if v is None else v.to("cuda", bf)) for k, v in w.items()}
 n, d, H, hd, I = a[4], m.d_model, m.n_heads, 128, m.d_ff
 nq = (H + 2 * m.n_kv_heads) * hd
-for kind in (1, 2):
+for kind in (1, 2, 4):
     pools[0][0].copy_(pk.to(bf)); pools[0][1].copy_(pv.to(bf))
     xg = x.cuda().contiguous()
     b = B.Batch(q_lens, ctx, lay.block_table, xg)
@@ -35,6 +35,14 @@ for kind in (1, 2):
     act = torch.zeros(n, I, dtype=bf, device="cuda")
     bl.op_rmsnorm(xg, wg["g_attn"], h)
     bl.op_gemm(B.EPI_F32, h, wg["w_qkv"], qkv)
+    if kind == 1:   # stage isolation: RMSNorm rounding flips, QKV GEMM accumulation error
+        torch.cuda.synchronize()
+        h_ref = O.round_bf16(O.rmsnorm(x.double().numpy(), w["g_attn"].double().numpy(), m.rms_eps))
+        hg = h.float().cpu().numpy()
+        ex = O.linear(hg.astype(np.float64), w["w_qkv"].double().numpy())
+        f32 = torch.nn.functional.linear(torch.from_numpy(hg), w["w_qkv"].float()).numpy()
+        gq = qkv.cpu().numpy()
+        print(f"h flips {np.mean(hg != h_ref):.4f}   qkv GEMM vs fp64 (same h): gpu {compare(gq, ex)}  cpu-fp32 {compare(f32, ex)}")
     bl.op_rope_kv(b, 0, qkv, q)
     bl.op_attention(b, 0, q, o, kind=kind)
     bl.op_gemm(B.EPI_RESID, o, wg["w_o"], xg, resid=xg)

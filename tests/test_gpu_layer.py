@@ -107,6 +107,27 @@ def test_llama8b_config2_layer_sampled():
     assert mx <= 2e-2 and mr <= 1e-3, ("pre", mx, mr)
 
 
+def test_llama8b_config3_layer_sampled():
+    """BASELINE config 3 at full size (one 8192-token arXiv-shaped prefill +
+    256 decodes with 2048-6144 cached tokens, 5.4 GB of paged KV per layer),
+    one layer at the split bench.py uses for it (p = 88).  Oracle: all 256
+    decode rows and 49 sampled prefill rows incl. the last."""
+    wl = synth.workload("arxiv-8b")
+    S = Setup(synth.MODELS["llama3.1-8b"], wl.prefill_lens, wl.decode_ctx, n_layers=1)
+    n_p = sum(wl.prefill_lens)
+    rng = np.random.default_rng(1)
+    mask = np.zeros(n_p, np.uint8)
+    mask[rng.choice(n_p, 48, replace=False)] = 1
+    mask[np.cumsum(wl.prefill_lens) - 1] = 1
+    ref = S.oracle(row_mask_pre=mask)
+    pre, dec = _run(S, 88, S.B.CORUN)
+    mx, mr = compare(dec.hidden.cpu().numpy(), ref["dec"])
+    assert mx <= 2e-2 and mr <= 1e-3, ("dec", mx, mr)
+    got = pre.hidden.cpu().numpy()[mask == 1]
+    mx, mr = compare(got, ref["pre"][mask == 1])
+    assert mx <= 2e-2 and mr <= 1e-3, ("pre", mx, mr)
+
+
 @pytest.mark.parametrize("p", [2, 40, 146])
 def test_smid_gating_invariants(small_bf16, p):
     """SM-range work assignment (§8a SG), bit-exact invariants: every work
