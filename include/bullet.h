@@ -334,6 +334,13 @@ int bullet_op_gemm(bullet_handle *h, int epi, const void *d_A, int M, int K, con
 int bullet_op_stream(bullet_handle *h, const void *d_src, size_t bytes, int mode, int lo, int hi,
                      void *stream);
 
+/* KI3 microbenchmark (not gated; n_ctas CTAs in clusters of 2, one per SM):
+ * stream `bytes` (multiple of 32 KB) into shared memory in 32 KB stages; mc = 1:
+ * each CTA fetches half of every stage with a .multicast::cluster bulk copy
+ * into both CTAs, mc = 0: each CTA fetches the whole stage.  Measures whether
+ * multicast lifts the per-SM async-copy ceiling. */
+int bullet_op_stream_mc(bullet_handle *h, const void *d_src, size_t bytes, int mc, int n_ctas, void *stream);
+
 int bullet_op_rmsnorm(bullet_handle *h, const float *d_x, int n, const void *d_g, void *d_out,
                       int lo, int hi, void *stream);
 

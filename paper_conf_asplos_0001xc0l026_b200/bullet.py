@@ -121,6 +121,8 @@ def lib():
         L.bullet_op_gemm.argtypes = [c_void_p, c_int, c_void_p, c_int, c_int, c_void_p, c_int, c_int,
                                      c_void_p, c_void_p, c_void_p, c_int, c_int, c_void_p]
         L.bullet_op_stream.restype = c_int
+        L.bullet_op_stream_mc.restype = c_int
+        L.bullet_op_stream_mc.argtypes = [c_void_p, c_void_p, ctypes.c_size_t, c_int, c_int, c_void_p]
         L.bullet_op_stream.argtypes = [c_void_p, c_void_p, ctypes.c_size_t, c_int, c_int, c_int, c_void_p]
         L.bullet_op_rmsnorm.argtypes = [c_void_p, c_void_p, c_int, c_void_p, c_void_p, c_int, c_int, c_void_p]
         L.bullet_op_rope_kv.argtypes = [c_void_p, ctypes.POINTER(CBatch), c_int, c_void_p, c_void_p,
@@ -391,6 +393,10 @@ class Bullet:
     def op_stream(self, src, mode=0, lo=0, hi=None, stream=None):
         _check(lib().bullet_op_stream(self.h, _ptr(src), src.numel() * src.element_size(), mode, lo,
                                       self.n_sms if hi is None else hi, _stream(stream)))
+
+    def op_stream_mc(self, src, mc, n_ctas, stream=None):
+        _check(lib().bullet_op_stream_mc(self.h, _ptr(src), src.numel() * src.element_size(), int(mc), int(n_ctas),
+                                         _stream(stream)))
 
     def op_rmsnorm(self, x, g, out, lo=0, hi=None, stream=None):
         _check(lib().bullet_op_rmsnorm(self.h, _ptr(x), x.shape[0], _ptr(g), _ptr(out), lo,

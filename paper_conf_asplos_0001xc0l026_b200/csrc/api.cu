@@ -1190,6 +1190,13 @@ int bullet_op_stream(bullet_handle* h, const void* src, size_t bytes, int mode, 
   return BULLET_OK;
 }
 
+int bullet_op_stream_mc(bullet_handle* h, const void* src, size_t bytes, int mc, int n_ctas, void* stream) {
+  if (!h || !src || n_ctas < 2 || bytes == 0) return set_err(BULLET_EINVAL, "stream_mc args");
+  if (h->host_only) return set_err(BULLET_EUNSUPPORTED, "host-only handle");
+  CK(launch_stream_mc((const uint8_t*)src, bytes, mc, n_ctas, (uint32_t*)h->op_ctr, (cudaStream_t)stream));
+  return BULLET_OK;
+}
+
 int bullet_op_rmsnorm(bullet_handle* h, const float* x, int n, const void* g, void* out, int lo,
                       int hi, void* stream) {
   Ctx c;

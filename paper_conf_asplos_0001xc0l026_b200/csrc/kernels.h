@@ -137,6 +137,7 @@ size_t attn_decode_smem_bytes();
 int attn_decode_max_blocks();
 cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);   // grid sized to n_tok
 cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st);
+cudaError_t launch_stream_mc(const uint8_t* src, size_t bytes, int mc, int grid, uint32_t* sink, cudaStream_t st);
 cudaError_t launch_probe(int* out_smid, int n, cudaStream_t st);
 
 // Lazy module loading (CUDA default) loads a kernel at its first launch

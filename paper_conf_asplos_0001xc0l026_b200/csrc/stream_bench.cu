@@ -20,6 +20,7 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       : "memory");
 }
 constexpr int BULK = 32768, NB = 6;
+constexpr int NB_MC = 7;   // k_stream_mc ring (7 x 32 KB)
 }  // namespace
 
 __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
@@ -153,6 +154,80 @@ cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st) {
   cudaError_t e = cudaFuncSetAttribute(k_stream, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return e;
   k_stream<<<grid, 512, smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+// KI3: does TMA multicast lift the per-SM async-copy ceiling?  Clusters of
+// two CTAs stream 32 KB stages; mc = 1: each CTA bulk-copies its 16 KB half
+// with .multicast::cluster into both CTAs' stage (each SM requests half of
+// what it receives); mc = 0: each CTA copies all 32 KB itself.  Same bytes
+// delivered into every SM either way; units are assigned statically by
+// cluster (no gating: a standalone microbenchmark, not a hot-path kernel).
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ uint32_t mapa_u32(uint32_t addr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
+  return r;
+}
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(128, 1)
+    k_stream_mc(const uint8_t* src, size_t bytes, int mc, uint32_t* sink) {
+  extern __shared__ __align__(128) uint8_t sm[];
+  __shared__ uint64_t full[NB_MC], empty[NB_MC];
+  const uint32_t cr = cluster_rank();
+  const int n_cl = gridDim.x / 2, cl = blockIdx.x / 2;
+  const size_t units = bytes / BULK;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < NB_MC; ++i) { mbar_init(full + i, 1); mbar_init(empty + i, 2); }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  cluster_sync_all();
+  uint32_t acc = 0;
+  if (threadIdx.x == 0) {
+    const int n_it = units > (size_t)cl ? (int)((units - cl + n_cl - 1) / n_cl) : 0;
+    constexpr int LAG = NB_MC - 3;   // stages in flight; a stage is released 3 issues before its reuse
+    for (int it = 0; it < n_it + LAG; ++it) {
+      if (it < n_it) {   // issue stage `it`
+        const int s = it % NB_MC;
+        if (it >= NB_MC) mbar_wait(empty + s, ((it / NB_MC) & 1) ^ 1);   // both CTAs released it
+        mbar_arrive_expect_tx(full + s, BULK);
+        const uint8_t* g = src + ((size_t)cl + (size_t)it * n_cl) * BULK;
+        if (mc) {
+          const uint32_t half = BULK / 2;
+          asm volatile(
+              "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1], %2, [%3], %4;" ::"r"(
+                  smem_u32(sm + s * BULK + cr * half)),
+              "l"(g + cr * half), "r"(half), "r"(smem_u32(full + s)), "h"((uint16_t)3)
+              : "memory");
+        } else {
+          bulk_g2s(sm + s * BULK, g, BULK, full + s);
+        }
+      }
+      const int j = it - LAG;
+      if (j >= 0) {      // consume stage j, release it in both CTAs
+        const int s = j % NB_MC;
+        mbar_wait(full + s, (j / NB_MC) & 1);
+        acc ^= *reinterpret_cast<const uint32_t*>(sm + s * BULK + (j & 1023) * 16);
+        const uint32_t b = smem_u32(empty + s);
+        for (uint32_t r = 0; r < 2; ++r)
+          asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(mapa_u32(b, r)) : "memory");
+      }
+    }
+  }
+  cluster_sync_all();   // no multicast / arrive may target an exited CTA
+  if (acc == 0x12345678u) sink[0] = acc;
+}
+
+cudaError_t launch_stream_mc(const uint8_t* src, size_t bytes, int mc, int grid, uint32_t* sink, cudaStream_t st) {
+  cudaError_t e = cudaFuncSetAttribute(k_stream_mc, cudaFuncAttributeMaxDynamicSharedMemorySize, NB_MC * BULK);
+  if (e != cudaSuccess) return e;
+  k_stream_mc<<<grid & ~1, 128, NB_MC * BULK, st>>>(src, bytes, mc, sink);
   return cudaGetLastError();
 }
 
