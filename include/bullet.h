@@ -60,8 +60,10 @@ enum {
   BULLET_UNGATED = 2,        /* both phases concurrently on all SMs ("Naive") */
   BULLET_SMID_LOG = 4,       /* record (launch, tile, smid) of every work unit */
   BULLET_PROFILE = 8,        /* CUDA events around every kernel (bullet_profile_read) */
-  BULLET_UNFUSED = 16        /* run S3 (RoPE + KV append) as its own kernel instead of the
+  BULLET_UNFUSED = 16,       /* run S3 (RoPE + KV append) as its own kernel instead of the
                                 QKV GEMM epilogue (bf16, head_dim 128); A/B tests only */
+  BULLET_UNFUSED_NORM = 32   /* run S6 / the next layer's S1 (RMSNorm) as their own kernels
+                                instead of the tail of the O-proj / down GEMM; A/B tests only */
 };
 
 /* Kernel kinds reported by bullet_profile_read. */

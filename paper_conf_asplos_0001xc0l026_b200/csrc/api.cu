@@ -107,6 +107,8 @@ struct PhaseWS {
   int* n_tiles = nullptr;
   TokInfo* tok = nullptr;          // per-token (position, KV slot), written by the plan kernel
   int max_tok = 0;
+  int* rbc = nullptr;              // fused-norm row-block counters [n_rbc_slices][max_rb], zeroed per step
+  int max_rb = 0, n_rbc_slices = 0, next_rbc = 0;
 };
 
 constexpr int GRAN = 2;            // split granularity: one TPC
@@ -199,6 +201,7 @@ struct Ctx {  // one phase's launch context within a call
   bool prof = false;
   int kind = 0, layer = -1;
   bool fuse_qkv = false;   // S3 in the QKV epilogue (EPI_QKV)
+  bool fuse_norm = false;  // S6 / next S1 in the tail of the O-proj / down GEMM (NormFuse)
 };
 
 constexpr size_t MAX_PROF = 1 << 16;
@@ -274,7 +277,8 @@ struct QkvEpi {   // EPI_QKV destinations
 
 int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, int silu_half,
             const void* bias, const float* resid, void* out, int ldo, const uint8_t* Bp = nullptr,
-            const QkvEpi* qe = nullptr, const ArArgs* ar = nullptr) {
+            const QkvEpi* qe = nullptr, const ArArgs* ar = nullptr, const void* norm_g = nullptr,
+            void* norm_out = nullptr) {
   bullet_handle* h = c.h;
   if (M == 0) return BULLET_OK;
   GemmArgs a;
@@ -290,6 +294,20 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   }
   int rc = next_launch(c, &a.L);
   if (rc) return rc;
+  if (norm_out) {   // fused RMSNorm in the GEMM tail: row-block counters + a row counter
+    PhaseWS& P = h->ph[c.phase];
+    if (c.op || epi != EPI_RESID || h->cfg.dtype != BULLET_DTYPE_BF16)
+      return set_err(BULLET_EINVAL, "fused norm: bf16 step GEMMs with EPI_RESID only");
+    if (P.next_ctr >= P.n_counters || P.next_rbc >= P.n_rbc_slices)
+      return set_err(BULLET_ENOMEM, "work counters exhausted");
+    a.nf.g = norm_g; a.nf.out = norm_out; a.nf.eps = h->cfg.rms_eps;
+    {   // rows per claim: about one claim per SM of the partition, at most 4
+      const int per = (M + c.m_sms - 1) / std::max(1, c.m_sms);
+      a.nf.rows = per >= 4 ? 4 : per >= 2 ? 2 : 1;
+    }
+    a.nf.unit_ctr = P.counters + P.next_ctr++;
+    a.nf.rb_ctr = P.rbc + (size_t)P.next_rbc++ * P.max_rb;
+  }
   if (ar) {   // fused peer all-reduce (bf16 only, checked at create): its own unit counter
     PhaseWS& P = h->ph[c.phase];
     if (c.op || epi != EPI_F32) return set_err(BULLET_EINVAL, "fused all-reduce: step GEMMs with EPI_F32 only");
@@ -566,7 +584,9 @@ int run_layer(Ctx& c, const bullet_batch* b, int layer) {
   int rc;
   c.layer = layer;
   c.kind = BULLET_K_RMSNORM1;
-  if ((rc = do_rmsnorm(c, b->d_hidden, n, w.g_attn, P.h))) return rc;                       // S1
+  // S1 — already done by the previous layer's down GEMM when the norm is fused
+  if (!(c.fuse_norm && layer > b->layer_begin) && (rc = do_rmsnorm(c, b->d_hidden, n, w.g_attn, P.h)))
+    return rc;
   c.kind = BULLET_K_QKV;
   const bullet_handle::Packed* wp = h->wp.empty() ? nullptr : &h->wp[layer];
   if (c.fuse_qkv) {   // S2 + S3: RoPE and the KV append in the QKV epilogue
@@ -591,13 +611,16 @@ int run_layer(Ctx& c, const bullet_batch* b, int layer) {
     if ((rc = do_gemm(c, EPI_F32, P.o, n, H * hd, w.w_o, d, 0, nullptr, nullptr, ar.part[ar.rank], d,
                       wp ? wp->o : nullptr, nullptr, &ar))) return rc;
   } else {
+    const bool fn = c.fuse_norm && !tp;   // S5 + S6: RMSNorm in the O-proj GEMM's tail
     if ((rc = do_gemm(c, (!tp || lead) ? EPI_RESID : EPI_F32, P.o, n, H * hd, w.w_o, d, 0, nullptr,
-                      b->d_hidden, b->d_hidden, d, wp ? wp->o : nullptr))) return rc;
+                      b->d_hidden, b->d_hidden, d, wp ? wp->o : nullptr, nullptr, nullptr,
+                      fn ? w.g_mlp : nullptr, fn ? P.h : nullptr))) return rc;
     c.kind = BULLET_K_ALLREDUCE;
     if (tp && (rc = allreduce(c, b->d_hidden, (size_t)n * d))) return rc;
   }
   c.kind = BULLET_K_RMSNORM2;
-  if ((rc = do_rmsnorm(c, b->d_hidden, n, w.g_mlp, P.h))) return rc;                        // S6
+  if (!(c.fuse_norm && !tp && !h->peer_mode) && (rc = do_rmsnorm(c, b->d_hidden, n, w.g_mlp, P.h)))
+    return rc;                                                                                // S6
   c.kind = BULLET_K_GATE_UP;
   if ((rc = do_gemm(c, EPI_SILU, P.h, n, d, w.w_gate_up, 2 * I, I, nullptr, nullptr, P.act, I,
                     wp ? wp->gu : nullptr))) return rc;  // S7
@@ -607,8 +630,11 @@ int run_layer(Ctx& c, const bullet_batch* b, int layer) {
     return do_gemm(c, EPI_F32, P.act, n, I, w.w_down, d, 0, nullptr, nullptr, ar.part[ar.rank], d,
                    wp ? wp->down : nullptr, nullptr, &ar);
   }
+  // S8 (+ the next layer's S1 in the GEMM tail when the norm is fused)
+  const bool fn = c.fuse_norm && !tp && layer + 1 < b->layer_end;
   if ((rc = do_gemm(c, (!tp || lead) ? EPI_RESID : EPI_F32, P.act, n, I, w.w_down, d, 0, nullptr,
-                    b->d_hidden, b->d_hidden, d, wp ? wp->down : nullptr))) return rc;       // S8
+                    b->d_hidden, b->d_hidden, d, wp ? wp->down : nullptr, nullptr, nullptr,
+                    fn ? h->w[layer + 1].g_attn : nullptr, fn ? P.h : nullptr))) return rc;
   c.kind = BULLET_K_ALLREDUCE;
   if (tp && (rc = allreduce(c, b->d_hidden, (size_t)n * d))) return rc;
   return BULLET_OK;
@@ -659,13 +685,14 @@ int validate_batch(const bullet_handle* h, const bullet_batch* b, int phase) {
 int run_phase(Ctx& c, const bullet_batch* b) {
   PhaseWS& P = c.h->ph[c.phase];
   P.next_ctr = 0;
+  P.next_rbc = 0;
   const bool tc_attn = c.h->cfg.dtype == BULLET_DTYPE_BF16 && c.h->cfg.head_dim == 128 && max_qlen(b) > 1;
   int t0 = 0;
   const int r0 = tc_attn ? mixed_split(b, &t0) : 0;
   PlanArgs pa{P.counters, P.n_counters, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ, r0 ? r0 : b->n_reqs,
               tc_attn ? P.tiles : nullptr, P.n_tiles,
               c.fuse_qkv ? P.tok : nullptr, b->d_ctx_lens, b->d_block_table, b->max_blocks_per_req,
-              c.h->block_size, b->n_tokens};
+              c.h->block_size, b->n_tokens, P.rbc, P.n_rbc_slices * P.max_rb};
   c.kind = BULLET_K_PLAN;
   c.layer = -1;
   prof_begin(c);
@@ -810,7 +837,10 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
               cudaMalloc(&P.counters, P.n_counters * sizeof(int)) == cudaSuccess &&
               cudaMalloc(&P.tiles, (T / ATTN_TC_BQ + 1024) * sizeof(int2)) == cudaSuccess &&
               cudaMalloc(&P.n_tiles, sizeof(int)) == cudaSuccess &&
-              cudaMalloc(&P.tok, T * sizeof(TokInfo)) == cudaSuccess;
+              cudaMalloc(&P.tok, T * sizeof(TokInfo)) == cudaSuccess &&
+              cudaMalloc(&P.rbc, (size_t)(2 * c.n_layers + 2) * ((T + 127) / 128) * sizeof(int)) == cudaSuccess;
+    P.max_rb = (int)((T + 127) / 128);
+    P.n_rbc_slices = 2 * c.n_layers + 2;
     if (!ok) return fail(set_err(BULLET_ENOMEM, "workspace allocation (phase %d)", p));
     cudaMemset(P.tile_sems, 0, N_TILE_SEMS * sizeof(int));
     cudaMemset(P.counters, 0, P.n_counters * sizeof(int));
@@ -943,6 +973,14 @@ static int step_impl(bullet_handle* h, const bullet_batch* pre, const bullet_bat
          mode == BULLET_CORUN ? dhi - dlo : N, log, sd, false, prof};
   cp.fuse_qkv = cd.fuse_qkv = !(flags & BULLET_UNFUSED) && h->cfg.dtype == BULLET_DTYPE_BF16 &&
                               h->cfg.head_dim == 128;
+  // fused norm pays for decode-sized batches (the standalone kernel's launch
+  // and drain dominate there: decode layer-step -1.6 % on 76 SMs); a prefill
+  // GEMM's tail runs it with one CTA per SM where the standalone kernel packs
+  // several (+0.7 % on a prefill layer) — so only up to 1024 rows
+  const bool fn_ok = !(flags & BULLET_UNFUSED_NORM) && h->cfg.dtype == BULLET_DTYPE_BF16 && !h->peer_mode &&
+                     h->cfg.d_model <= 8192;
+  cp.fuse_norm = fn_ok && pre && pre->n_tokens <= 1024;
+  cd.fuse_norm = fn_ok && dec && dec->n_tokens <= 1024;
   if (has_pre && (rc = run_phase(cp, pre))) return rc;
   if (run_dec) {
     if (mode == BULLET_TIMESLICED && has_pre) {
@@ -1066,7 +1104,7 @@ void bullet_destroy(bullet_handle* h) {
     PhaseWS& P = h->ph[p];
     cudaFree(P.qkv); cudaFree(P.q); cudaFree(P.o); cudaFree(P.h); cudaFree(P.act);
     cudaFree(P.partials); cudaFree(P.tile_sems); cudaFree(P.counters); cudaFree(P.tiles);
-    cudaFree(P.n_tiles); cudaFree(P.tok);
+    cudaFree(P.n_tiles); cudaFree(P.tok); cudaFree(P.rbc);
     if (h->comm[p] && g_nccl.commDestroy) g_nccl.commDestroy(h->comm[p]);
   }
   for (void* p : h->ipc_opened) cudaIpcCloseMemHandle(p);

@@ -241,6 +241,7 @@ __global__ void __launch_bounds__(256) k_gemm_simt(const T* __restrict__ A, cons
 __global__ void k_plan(PlanArgs a) {
   if (blockIdx.x == 0) {
     for (int i = threadIdx.x; i < a.n_counters; i += blockDim.x) a.counters[i] = 0;
+    for (int i = threadIdx.x; i < a.n_zero2; i += blockDim.x) a.zero2[i] = 0;
     if (threadIdx.x == 0 && a.tiles) {
       int maxt = 0;
       for (int r = 0; r < a.n_tile_reqs; ++r) {

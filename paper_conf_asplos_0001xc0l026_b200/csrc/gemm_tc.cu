@@ -310,6 +310,96 @@ __device__ __forceinline__ void ar_phase(const GemmArgs& a, int* s_u) {
   }
 }
 
+// ---------------------------------------------------------------- fused RMSNorm (kernels.h NormFuse)
+// Called by the 128 epilogue threads once the tile's rows are stored.
+__device__ __forceinline__ void norm_signal(const GemmArgs& a, int m_blk, int mh, int et) {
+  __threadfence();
+  named_bar_sync(1, 128);
+  if (et == 0)
+    for (int hh = 0; hh < mh; ++hh) {
+      const int rb = m_blk * mh + hh;
+      if (rb * BM >= a.M) break;
+      asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(a.nf.rb_ctr + rb), "r"(a.bn) : "memory");
+    }
+}
+__device__ __forceinline__ int ld_acquire_gpu(const int* p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+// After the CTA's GEMM units (all 256 threads): R rows per claim (their
+// loads in flight together), each row with the arithmetic of
+// k_rmsnorm<bf16, VPT> (elementwise.cu) in the same order: bit-identical.
+template <int VPT, int R>
+__device__ __forceinline__ void norm_phase(const GemmArgs& a, int* s_u, float* s_red) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, d = a.N, d4 = d / 4;
+  const __nv_bfloat16* g = reinterpret_cast<const __nv_bfloat16*>(a.nf.g);
+  __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(a.nf.out);
+  const int units = (a.M + R - 1) / R;
+  for (;;) {
+    if (tid == 0) {
+      const int u = atomicAdd(a.nf.unit_ctr, 1);
+      if (u < units) {   // the row blocks of rows [u R, u R + R) are complete
+        const int r0 = u * R, r1 = min(a.M, r0 + R) - 1;
+        for (int rb = r0 / BM; rb <= r1 / BM; ++rb)
+          while (ld_acquire_gpu(a.nf.rb_ctr + rb) < d) __nanosleep(64);
+      }
+      *s_u = u;
+    }
+    __syncthreads();
+    const int u = *s_u;
+    if (u >= units) break;
+    float4 v[R][VPT];
+    float ss[R];
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      const int r = min(u * R + j, a.M - 1);   // rows past M: recomputed, not stored
+      const float4* x = reinterpret_cast<const float4*>(a.out_f32 + (size_t)r * a.ldo);
+#pragma unroll
+      for (int i = 0; i < VPT; ++i) {
+        const int idx = tid + i * 256;
+        v[j][i] = idx < d4 ? __ldcg(x + idx) : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      ss[j] = 0.f;
+#pragma unroll
+      for (int i = 0; i < VPT; ++i)
+        ss[j] += v[j][i].x * v[j][i].x + v[j][i].y * v[j][i].y + v[j][i].z * v[j][i].z + v[j][i].w * v[j][i].w;
+      ss[j] = warp_sum(ss[j]);
+      if (lane == 0) s_red[j * 8 + warp] = ss[j];
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      const int r = u * R + j;
+      if (r >= a.M) break;
+      float tot = 0.f;
+#pragma unroll
+      for (int w = 0; w < 8; ++w) tot += s_red[j * 8 + w];
+      const float inv = rsqrtf(tot / (float)d + a.nf.eps);
+      __nv_bfloat16* o = out + (size_t)r * d;
+#pragma unroll
+      for (int i = 0; i < VPT; ++i) {
+        const int idx = tid + i * 256;
+        if (idx < d4) {
+          const uint2 gu = *reinterpret_cast<const uint2*>(g + 4 * idx);
+          const float2 g0 = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&gu.x));
+          const float2 g1 = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&gu.y));
+          __nv_bfloat162 p0 = __floats2bfloat162_rn(v[j][i].x * inv * g0.x, v[j][i].y * inv * g0.y);
+          __nv_bfloat162 p1 = __floats2bfloat162_rn(v[j][i].z * inv * g1.x, v[j][i].w * inv * g1.y);
+          uint2 w2;
+          w2.x = *reinterpret_cast<uint32_t*>(&p0);
+          w2.y = *reinterpret_cast<uint32_t*>(&p1);
+          *reinterpret_cast<uint2*>(o + 4 * idx) = w2;
+        }
+      }
+    }
+    __syncthreads();   // s_u / s_red reuse
+  }
+}
+
 }  // namespace
 
 int gemm_tc_stages(int bn, int mh) {
@@ -495,6 +585,7 @@ __global__ void __launch_bounds__(NT, 1)
         __syncwarp();
         if (lane == 0) mbar_arrive(acce + as);
         if (a.ar.n) ar_signal(a, m_blk, mh, et);
+        if (a.nf.out) norm_signal(a, m_blk, mh, et);
       } else {
         // partial tile stored as float4 groups interleaved by row per half
         // ([hh][col/4][row][4]): a thread's 4 consecutive columns are one
@@ -567,6 +658,7 @@ __global__ void __launch_bounds__(NT, 1)
             }
           }
           if (a.ar.n) ar_signal(a, m_blk, mh, et);
+          if (a.nf.out) norm_signal(a, m_blk, mh, et);
         }
       }
       if (++as == n_acc) { as = 0; aph ^= 1; }
@@ -576,6 +668,19 @@ __global__ void __launch_bounds__(NT, 1)
   if (a.ar.n) {   // fused all-reduce: this CTA's GEMM units are done
     __syncthreads();
     ar_phase(a, s_last + 1);
+  }
+  if (a.nf.out) {   // fused RMSNorm of the rows this GEMM finished
+    __syncthreads();
+    float* s_red = reinterpret_cast<float*>(smem);   // the stage ring is idle now
+    const int vpt = (a.N / 4 + 255) / 256;
+    if (vpt <= 4) {
+      if (a.nf.rows >= 4) norm_phase<4, 4>(a, s_last + 1, s_red);
+      else if (a.nf.rows == 2) norm_phase<4, 2>(a, s_last + 1, s_red);
+      else norm_phase<4, 1>(a, s_last + 1, s_red);
+    } else {
+      if (a.nf.rows >= 2) norm_phase<8, 2>(a, s_last + 1, s_red);
+      else norm_phase<8, 1>(a, s_last + 1, s_red);
+    }
   }
   tc_fence_before();
   __syncthreads();

@@ -35,6 +35,20 @@ struct ArArgs {
   int* err;                                         // set on a peer timeout
 };
 
+// RMSNorm fused into the tail of a residual GEMM (EPI_RESID; S6 after the
+// O-proj, the next layer's S1 after down): every finished tile adds its
+// column count to rb_ctr[128-row block]; once a CTA's GEMM units run out it
+// claims rows from unit_ctr, waits until the row's block holds all N columns
+// and normalises the row exactly as k_rmsnorm does (same reduction order:
+// bit-identical), out = bf16(x * rsqrt(mean x^2 + eps) * g).
+struct NormFuse {
+  const void* g; void* out;   // out == nullptr: off
+  float eps;
+  int* rb_ctr;                // [ceil(M / 128)], zero at launch
+  int* unit_ctr;              // zero at launch
+  int rows;                   // rows per claim (1, 2, 4): several rows' loads in flight per CTA
+};
+
 // C[M x N] = A[M x K] . B[N x K]^T with a fused epilogue (all row-major).
 struct GemmArgs {
   int M, N, K;        // N = B rows used (2 x output cols for EPI_SILU)
@@ -64,6 +78,7 @@ struct GemmArgs {
   const TokInfo* tok;       // [M]
   int H, Hkv, kvB;
   ArArgs ar;                // EPI_F32 into ar.part[ar.rank] + the fused all-reduce (ar.n > 1)
+  NormFuse nf;              // EPI_RESID + RMSNorm of the finished rows (nf.out != nullptr)
   Launch L;
 };
 
@@ -113,6 +128,7 @@ struct PlanArgs {
   int2* tiles; int* n_tiles;
   // per-token (position, slot) table (nullable): needs ctx, bt, max_blocks, B
   TokInfo* tok; const int32_t* ctx; const int32_t* bt; int max_blocks, B, n_tok;
+  int* zero2; int n_zero2;   // second array zeroed per step (fused-norm row-block counters)
 };
 
 // launchers (return cudaError_t of the launch)

@@ -26,12 +26,13 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--quiet", action="store_true")
     ap.add_argument("--time", type=int, default=0, help="also time this many steps without PROFILE")
+    ap.add_argument("--extra-flags", type=int, default=0, help="OR'ed into the step flags (e.g. 32 = UNFUSED_NORM)")
     a = ap.parse_args()
     torch.cuda.set_device(0)
     S = bench.Step(a.config, max(1, a.k))
     B = S.B
     S.dec.layer_end = a.k
-    flags = B.TIMESLICED if a.mode == "timesliced" else B.CORUN
+    flags = (B.TIMESLICED if a.mode == "timesliced" else B.CORUN) | a.extra_flags
     pre = a.mode in ("pre", "corun", "timesliced")
     dec = a.mode in ("dec", "corun", "timesliced")
     p = a.p if a.mode != "timesliced" else S.N

@@ -128,6 +128,28 @@ def test_llama8b_config3_layer_sampled():
     assert mx <= 2e-2 and mr <= 1e-3, ("pre", mx, mr)
 
 
+@pytest.mark.parametrize("p", [64, 146])
+def test_fused_norm_bit_identical_to_rmsnorm_kernel(small_bf16, p):
+    """RMSNorm in the O-proj / down GEMM tails (S6 and the next layer's S1)
+    reproduces the standalone k_rmsnorm bit for bit (same reduction order)
+    over a 2-layer step with ragged prefill rows, and launches 2 kernels
+    fewer per layer after the first."""
+    S = small_bf16
+    B = S.B
+    outs, launches = [], []
+    for flags in (B.CORUN, B.CORUN | B.UNFUSED_NORM):
+        pre, dec = S.batches(0, 2)
+        sp, sd = phase_streams()
+        n0 = S.bl.launch_count()
+        S.bl.step(pre, dec, p, flags, sp, sd)
+        torch.cuda.synchronize()
+        launches.append(S.bl.launch_count() - n0)
+        outs.append((pre.hidden.clone(), dec.hidden.clone()))
+    assert torch.equal(outs[0][0], outs[1][0]) and torch.equal(outs[0][1], outs[1][1])
+    # both batches have <= 1024 rows: 2 phases x (S6 x 2 layers + S1 of layer 1)
+    assert launches[1] - launches[0] == 2 * (2 * 2 - 1)
+
+
 @pytest.mark.parametrize("p", [2, 40, 146])
 def test_smid_gating_invariants(small_bf16, p):
     """SM-range work assignment (§8a SG), bit-exact invariants: every work
