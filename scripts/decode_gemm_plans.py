@@ -18,8 +18,8 @@ import bench  # noqa: E402
 
 KINDS = {"qkv": 2, "o_proj": 5, "gate_up": 7, "down": 8}
 PLANS = {
-    "qkv": ["", "1,128,1", "1,256,1", "1,256,2", "1,256,3", "1,128,2", "1,256,4"],
-    "o_proj": ["", "1,64,1", "1,128,2", "1,256,4", "1,256,3", "1,128,3", "1,256,6", "1,256,8"],
+    "qkv": ["", "1,128,1", "1,64,1", "1,64,2", "1,128,2", "1,128,3", "1,256,2", "1,256,3", "1,256,4"],
+    "o_proj": ["", "1,64,1", "1,64,2", "1,128,1", "1,128,2", "1,256,4", "1,256,3", "1,128,3", "1,256,6"],
     "gate_up": ["", "1,256,1", "1,128,1", "1,256,2"],
     "down": ["", "1,128,2", "1,256,4", "1,256,3", "1,128,3", "1,256,6", "1,256,8", "1,64,1"],
 }
