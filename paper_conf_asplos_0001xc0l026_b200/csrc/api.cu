@@ -109,6 +109,8 @@ struct PhaseWS {
   int max_tok = 0;
   int* rbc = nullptr;              // fused-norm row-block counters [n_rbc_slices][max_rb], zeroed per step
   int max_rb = 0, n_rbc_slices = 0, next_rbc = 0;
+  int* order = nullptr;            // decode rows in LPT order (plan kernel), valid this step if order_ok
+  bool order_ok = false;
 };
 
 constexpr int GRAN = 2;            // split granularity: one TPC
@@ -503,6 +505,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     LAUNCH(c, launch_attn_prefill5(a, persist_grid(c, 2), c.st));
     AttnArgs d = a;
     d.tok_base = t0;
+    d.order = P.order_ok ? P.order : nullptr;
     if ((rc = next_launch(c, &d.L))) return rc;
     LAUNCH(c, launch_attn_decode_tc(d, persist_grid(c, 1), c.m_sms <= 100 ? 2 : 1, c.st));
     return BULLET_OK;
@@ -518,6 +521,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     // two consumer groups per SM on partitions (per-unit merge over twice the
     // blocks: 146 -> 133 us on 68 SMs, ShareGPT), one on the full GPU (tail
     // balance: 96 vs 101 us) — scripts/attn_dec_bench.py, DESIGN.md §5
+    if (!c.op && h->ph[c.phase].order_ok) a.order = h->ph[c.phase].order;
     LAUNCH(c, launch_attn_decode_tc(a, persist_grid(c, 1), c.m_sms <= 100 ? 2 : 1, c.st));
     return BULLET_OK;
   }
@@ -692,7 +696,12 @@ int run_phase(Ctx& c, const bullet_batch* b) {
   PlanArgs pa{P.counters, P.n_counters, b->d_cu_seqlens, b->n_reqs, ATTN_TC_BQ, r0 ? r0 : b->n_reqs,
               tc_attn ? P.tiles : nullptr, P.n_tiles,
               c.fuse_qkv ? P.tok : nullptr, b->d_ctx_lens, b->d_block_table, b->max_blocks_per_req,
-              c.h->block_size, b->n_tokens, P.rbc, P.n_rbc_slices * P.max_rb};
+              c.h->block_size, b->n_tokens, P.rbc, P.n_rbc_slices * P.max_rb, nullptr, 0};
+  // LPT order of the decode rows (pure decode batch, or the decode tail of a hybrid one)
+  static const bool no_order = getenv("BULLET_DEC_ORDER") && !strcmp(getenv("BULLET_DEC_ORDER"), "0");
+  P.order_ok = !no_order && c.h->cfg.dtype == BULLET_DTYPE_BF16 && c.h->cfg.head_dim == 128 &&
+               (r0 > 0 || max_qlen(b) == 1) && b->n_tokens > 0;
+  if (P.order_ok) { pa.order = P.order; pa.order_base = r0 ? t0 : 0; }
   c.kind = BULLET_K_PLAN;
   c.layer = -1;
   prof_begin(c);
@@ -838,6 +847,7 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
               cudaMalloc(&P.tiles, (T / ATTN_TC_BQ + 1024) * sizeof(int2)) == cudaSuccess &&
               cudaMalloc(&P.n_tiles, sizeof(int)) == cudaSuccess &&
               cudaMalloc(&P.tok, T * sizeof(TokInfo)) == cudaSuccess &&
+              cudaMalloc(&P.order, T * sizeof(int)) == cudaSuccess &&
               cudaMalloc(&P.rbc, (size_t)(2 * c.n_layers + 2) * ((T + 127) / 128) * sizeof(int)) == cudaSuccess;
     P.max_rb = (int)((T + 127) / 128);
     P.n_rbc_slices = 2 * c.n_layers + 2;
@@ -1104,7 +1114,7 @@ void bullet_destroy(bullet_handle* h) {
     PhaseWS& P = h->ph[p];
     cudaFree(P.qkv); cudaFree(P.q); cudaFree(P.o); cudaFree(P.h); cudaFree(P.act);
     cudaFree(P.partials); cudaFree(P.tile_sems); cudaFree(P.counters); cudaFree(P.tiles);
-    cudaFree(P.n_tiles); cudaFree(P.tok); cudaFree(P.rbc);
+    cudaFree(P.n_tiles); cudaFree(P.tok); cudaFree(P.rbc); cudaFree(P.order);
     if (h->comm[p] && g_nccl.commDestroy) g_nccl.commDestroy(h->comm[p]);
   }
   for (void* p : h->ipc_opened) cudaIpcCloseMemHandle(p);

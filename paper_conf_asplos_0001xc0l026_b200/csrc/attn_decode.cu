@@ -135,7 +135,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
       if (u >= units) u = -1;
       Slot sl{u, 0, 0, 0};
       if (u >= 0) {
-        sl.t = a.tok_base + u / a.Hkv;
+        sl.t = a.tok_base + (a.order ? __ldg(a.order + u / a.Hkv) : u / a.Hkv);
         const int r = find_req(a.cu, a.n_reqs, sl.t);
         sl.pos = __ldg(a.ctx + r) + (sl.t - __ldg(a.cu + r));
         sl.nb = sl.pos / KB + 1;

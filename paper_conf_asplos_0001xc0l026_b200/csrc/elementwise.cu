@@ -242,6 +242,26 @@ __global__ void k_plan(PlanArgs a) {
   if (blockIdx.x == 0) {
     for (int i = threadIdx.x; i < a.n_counters; i += blockDim.x) a.counters[i] = 0;
     for (int i = threadIdx.x; i < a.n_zero2; i += blockDim.x) a.zero2[i] = 0;
+    if (a.order) {   // counting sort of the decode rows by block count, descending (LPT)
+      __shared__ int hist[DEC_ORDER_BUCKETS + 1];
+      const int n = a.n_tok - a.order_base;
+      auto nb_of = [&](int i) {
+        const int t = a.order_base + i;
+        const int r = find_req(a.cu, a.n_reqs, t);
+        const int nb = (__ldg(a.ctx + r) + (t - __ldg(a.cu + r))) / a.B + 1;
+        return nb < DEC_ORDER_BUCKETS ? nb : DEC_ORDER_BUCKETS;
+      };
+      for (int i = threadIdx.x; i <= DEC_ORDER_BUCKETS; i += blockDim.x) hist[i] = 0;
+      __syncthreads();
+      for (int i = threadIdx.x; i < n; i += blockDim.x) atomicAdd(hist + nb_of(i), 1);
+      __syncthreads();
+      if (threadIdx.x == 0) {   // bucket starts, longest first
+        int run = 0;
+        for (int b = DEC_ORDER_BUCKETS; b >= 0; --b) { const int c = hist[b]; hist[b] = run; run += c; }
+      }
+      __syncthreads();
+      for (int i = threadIdx.x; i < n; i += blockDim.x) a.order[atomicAdd(hist + nb_of(i), 1)] = i;
+    }
     if (threadIdx.x == 0 && a.tiles) {
       int maxt = 0;
       for (int r = 0; r < a.n_tile_reqs; ++r) {

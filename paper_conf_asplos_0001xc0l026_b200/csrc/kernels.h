@@ -112,6 +112,7 @@ struct AttnArgs {
   const int* n_tiles;     // device count of `tiles`
   int dbg;                // diagnostics (BULLET_DBG env): bit0 = decode consumers skip math
   int tok_base;           // decode kernel: its rows are tokens [tok_base, n_tok) (mixed batches)
+  const int* order;       // decode kernel (nullable): unit token i -> tok_base + order[i], longest context first
   Launch L;
 };
 
@@ -129,6 +130,9 @@ struct PlanArgs {
   // per-token (position, slot) table (nullable): needs ctx, bt, max_blocks, B
   TokInfo* tok; const int32_t* ctx; const int32_t* bt; int max_blocks, B, n_tok;
   int* zero2; int n_zero2;   // second array zeroed per step (fused-norm row-block counters)
+  // decode rows [order_base, n_tok) in descending context length (nullable): LPT order of the
+  // decode attention's units (the longest rows start first, the tail is short)
+  int* order; int order_base;
 };
 
 // launchers (return cudaError_t of the launch)
@@ -168,7 +172,8 @@ cudaError_t preload_elementwise();
 cudaError_t preload_gemm_tc();
 cudaError_t preload_stream();
 
-constexpr int ATTN_TC_BQ = 128;   // query rows per prefill attention tile (plan granularity)
+constexpr int ATTN_TC_BQ = 128;
+constexpr int DEC_ORDER_BUCKETS = 512;   // LPT sort buckets (block counts; longer rows share the last)   // query rows per prefill attention tile (plan granularity)
 constexpr int ROWS_PER_UNIT = 8;  // rows per work unit of row-wise kernels
 
 }  // namespace bl
