@@ -119,6 +119,24 @@ def test_gemm_matches_oracle_linear_small(B):
     assert np.abs(out.cpu().numpy() - ref).max() < 2e-4
 
 
+@pytest.mark.parametrize("M,K,N", [(57, 4096, 6144), (512, 14336, 4096)])
+def test_gemm_accumulation_precision(B, M, K, N):
+    """DESIGN.md R-4e: the tcgen05 fp32 accumulation error at Llama-3.1-8B
+    QKV / down shapes, against an fp64 product of the same bf16 operands.
+    Measured 4.3e-6 normalised L1 at (57, 4096, 6144), ~30x IEEE fp32 on the
+    CPU (1.5e-7): the readings' bar analysis depends on it staying there."""
+    bl, _ = _handle(B, SMALL)
+    rng = np.random.default_rng(9)
+    A = O.round_bf16(rng.standard_normal((M, K))).astype(np.float32)
+    W = O.round_bf16(rng.standard_normal((N, K)) * K ** -0.5).astype(np.float32)
+    out = torch.zeros(M, N, device="cuda")
+    bl.op_gemm(B.EPI_F32, torch.from_numpy(A).to("cuda", bf16), torch.from_numpy(W).to("cuda", bf16), out)
+    ref = A.astype(np.float64) @ W.astype(np.float64).T
+    err = np.abs(out.cpu().numpy() - ref)
+    rel = err.sum() / np.abs(ref).sum()
+    assert rel < 1e-5, rel
+
+
 @pytest.mark.parametrize("packed", [False, True])
 def test_gemm_resid_in_place_bit_exact(B, packed):
     bl, _ = _handle(B, SMALL)

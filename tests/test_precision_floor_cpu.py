@@ -4,7 +4,7 @@ mirrored, exact fp32 softmax) against the fp64 oracle, one Llama-3.1-8B
 layer on a 57-token batch.  It pins the readings' claim that the bar
 (mean-rel 1e-3) leaves ~35 % headroom over IEEE fp32 at these dims — the
 tensor-core GEMM accumulation (4.3e-6 relative per GEMM, measured on the
-B200 by scripts/diag_layer.py) spends most of it.  Test-only code."""
+B200 by tests/tools/diag_layer.py and test_gpu_kernels.py::test_gemm_accumulation_precision) spends most of it.  Test-only code."""
 import numpy as np
 import torch
 

@@ -1,8 +1,9 @@
 """Per-stage error diagnosis of one bf16 layer (op entry points vs oracle
-diagnostics).  Usage: python scripts/diag_layer.py [d H Hkv I prefill_len]"""
+diagnostics; test infrastructure, lives under tests/ with the other oracle
+users).  Usage: python tests/tools/diag_layer.py [d H Hkv I prefill_len]"""
 import sys, os
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
+_T = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path[:0] = [os.path.dirname(_T), _T]
 import numpy as np, torch
 import oracle as O
 from workload import synth
