@@ -62,8 +62,13 @@ enum {
   BULLET_PROFILE = 8,        /* CUDA events around every kernel (bullet_profile_read) */
   BULLET_UNFUSED = 16,       /* run S3 (RoPE + KV append) as its own kernel instead of the
                                 QKV GEMM epilogue (bf16, head_dim 128); A/B tests only */
-  BULLET_UNFUSED_NORM = 32   /* run S6 / the next layer's S1 (RMSNorm) as their own kernels
+  BULLET_UNFUSED_NORM = 32,  /* run S6 / the next layer's S1 (RMSNorm) as their own kernels
                                 instead of the tail of the O-proj / down GEMM; A/B tests only */
+  BULLET_DEVICE_SPLIT = 64   /* CORUN: kernels read the phases' SM sets from device memory
+                                (bullet_set_split) instead of kernel arguments, so one CUDA
+                                graph captured from the step follows any later split
+                                (SURVEY §8f NEXT-4); prefill_sm_count / the ranges still size
+                                the GEMM plans */
 };
 
 /* Kernel kinds reported by bullet_profile_read. */
@@ -227,6 +232,17 @@ int bullet_step(bullet_handle *h, const bullet_batch *prefill, const bullet_batc
 int bullet_step_ranges(bullet_handle *h, const bullet_batch *prefill, const bullet_batch *decode,
                        int pre_lo, int pre_hi, int dec_lo, int dec_hi, int flags, void *s_prefill,
                        void *s_decode);
+
+/* BULLET_DEVICE_SPLIT: enqueue on `stream` the write of the device-resident
+ * SM sets — prefill on sigma[pre_lo, pre_hi), decode on sigma[dec_lo, dec_hi)
+ * (granularity and bounds as bullet_step_ranges; the ranges may overlap).
+ * Steps (or replays of graphs captured from steps) with BULLET_DEVICE_SPLIT
+ * that are ordered after it on the device use these sets.  Not captured into
+ * a graph by itself: call it outside capture, before each replay that needs
+ * a new split.  Initially every SM belongs to both phases.  A phase whose
+ * set holds none of its CTAs still completes (the grid's last CTA works
+ * wherever it landed — correct, slow).  Errors: ESMRANGE. */
+int bullet_set_split(bullet_handle *h, int pre_lo, int pre_hi, int dec_lo, int dec_hi, void *stream);
 
 /* Eq. 2 / T_m: predicted time (microseconds) of one layer of the given
  * batch on sm_count SMs; corun_sm_count > 0 applies the co-location factors

@@ -17,7 +17,7 @@ c_int, c_double, c_float, c_void_p = ctypes.c_int, ctypes.c_double, ctypes.c_flo
 P_i32 = ctypes.POINTER(ctypes.c_int32)
 P_f64 = ctypes.POINTER(ctypes.c_double)
 
-CORUN, TIMESLICED, UNGATED, SMID_LOG, PROFILE, UNFUSED, UNFUSED_NORM = 0, 1, 2, 4, 8, 16, 32
+CORUN, TIMESLICED, UNGATED, SMID_LOG, PROFILE, UNFUSED, UNFUSED_NORM, DEVICE_SPLIT = 0, 1, 2, 4, 8, 16, 32, 64
 KERNEL_KINDS = ["plan", "rmsnorm1", "qkv", "rope_kv", "attn", "o_proj", "rmsnorm2", "gate_up",
                 "down", "allreduce"]
 DTYPE_FP32, DTYPE_BF16 = 0, 1
@@ -89,7 +89,7 @@ def lib():
                      "bullet_set_smid_log", "bullet_sync", "bullet_nccl_unique_id", "bullet_op_gemm",
                      "bullet_op_rmsnorm", "bullet_op_rope_kv", "bullet_op_attention",
                      "bullet_profile_read", "bullet_launch_count", "bullet_tp_base", "bullet_tp_ipc_handle",
-                     "bullet_tp_connect", "bullet_tp_connect_ipc", "bullet_tp_hidden"):
+                     "bullet_tp_connect", "bullet_tp_connect_ipc", "bullet_tp_hidden", "bullet_set_split"):
             getattr(L, name).restype = c_int
         L.bullet_create.argtypes = [ctypes.POINTER(ModelCfg), ctypes.POINTER(KvPool), c_void_p,
                                     ctypes.c_char_p, ctypes.POINTER(c_void_p)]
@@ -112,6 +112,7 @@ def lib():
         L.bullet_launch_count.argtypes = [c_void_p, ctypes.POINTER(ctypes.c_longlong)]
         L.bullet_nccl_unique_id.argtypes = [c_void_p]
         L.bullet_tp_base.argtypes = [c_void_p, ctypes.POINTER(c_void_p)]
+        L.bullet_set_split.argtypes = [c_void_p, c_int, c_int, c_int, c_int, c_void_p]
         L.bullet_tp_ipc_handle.argtypes = [c_void_p, c_void_p]
         L.bullet_tp_connect.argtypes = [c_void_p, ctypes.POINTER(c_void_p)]
         L.bullet_tp_connect_ipc.argtypes = [c_void_p, c_void_p]
@@ -311,6 +312,11 @@ class Bullet:
 
     def sync(self):
         _check(lib().bullet_sync(self.h))
+
+    def set_split(self, pre_range, dec_range, stream=None):
+        """Device-resident SM sets for steps / graph replays with DEVICE_SPLIT."""
+        _check(lib().bullet_set_split(self.h, int(pre_range[0]), int(pre_range[1]), int(dec_range[0]),
+                                      int(dec_range[1]), _stream(stream)))
 
     # ---- fused tensor-parallel all-reduce over peer memory (PEER mode: tp_size > 1, no nccl_uids)
     def tp_base(self) -> int:

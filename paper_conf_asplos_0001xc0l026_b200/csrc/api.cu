@@ -159,6 +159,7 @@ struct bullet_handle {
   float2* rope_cs = nullptr;
   PhaseWS ph[2];
   int* op_ctr = nullptr;
+  Gate* d_gates = nullptr;           // BULLET_DEVICE_SPLIT: [2] (prefill, decode), written by bullet_set_split
   int32_t* log = nullptr;
   int log_cap = 0;
   int launch_seq = 0;
@@ -204,6 +205,7 @@ struct Ctx {  // one phase's launch context within a call
   int kind = 0, layer = -1;
   bool fuse_qkv = false;   // S3 in the QKV epilogue (EPI_QKV)
   bool fuse_norm = false;  // S6 / next S1 in the tail of the O-proj / down GEMM (NormFuse)
+  const Gate* gdev = nullptr;   // BULLET_DEVICE_SPLIT: the phase's gate in device memory
 };
 
 constexpr size_t MAX_PROF = 1 << 16;
@@ -241,6 +243,7 @@ int next_launch(Ctx& c, Launch* L) {
   prof_begin(c);
   memset(L, 0, sizeof *L);
   L->gate = c.gate;
+  L->gdev = c.gdev;
   L->log = c.log ? c.h->log : nullptr;
   L->log_cap = c.h->log_cap;
   L->launch_id = c.h->launch_seq++;
@@ -856,6 +859,13 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
     cudaMemset(P.counters, 0, P.n_counters * sizeof(int));
   }
   if (cudaMalloc(&h->op_ctr, 2 * sizeof(int)) != cudaSuccess) return fail(set_err(BULLET_ENOMEM, "op ctr"));
+  if (cudaMalloc(&h->d_gates, 2 * sizeof(Gate)) != cudaSuccess) return fail(set_err(BULLET_ENOMEM, "gates"));
+  {   // default device split: everything to decode (bullet_set_split overwrites)
+    const Gate all = gate_of(h, 0, h->n_sms);
+    if (cudaMemcpy(h->d_gates, &all, sizeof all, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemcpy(h->d_gates + 1, &all, sizeof all, cudaMemcpyHostToDevice) != cudaSuccess)
+      return fail(set_err(BULLET_ECUDA, "gates init"));
+  }
   if (cudaEventCreateWithFlags(&h->ev_ts, cudaEventDisableTiming) != cudaSuccess)
     return fail(set_err(BULLET_ECUDA, "event"));
   if (cudaDeviceSynchronize() != cudaSuccess) return fail(set_err(BULLET_ECUDA, "init sync"));
@@ -981,6 +991,11 @@ static int step_impl(bullet_handle* h, const bullet_batch* pre, const bullet_bat
          mode == BULLET_CORUN ? phi - plo : N, log, sp, false, prof};
   Ctx cd{h, 1, mode == BULLET_CORUN ? gate_of(h, dlo, dhi) : gate_of(h, 0, N),
          mode == BULLET_CORUN ? dhi - dlo : N, log, sd, false, prof};
+  if (flags & BULLET_DEVICE_SPLIT) {   // SM sets from bullet_set_split (graph replay follows it)
+    if (mode != BULLET_CORUN) return set_err(BULLET_EINVAL, "BULLET_DEVICE_SPLIT: CORUN only");
+    cp.gdev = h->d_gates;
+    cd.gdev = h->d_gates + 1;
+  }
   cp.fuse_qkv = cd.fuse_qkv = !(flags & BULLET_UNFUSED) && h->cfg.dtype == BULLET_DTYPE_BF16 &&
                               h->cfg.head_dim == 128;
   // fused norm pays for decode-sized batches (the standalone kernel's launch
@@ -1123,9 +1138,22 @@ void bullet_destroy(bullet_handle* h) {
   for (auto& P : h->wp) cudaFree(P.base);
   cudaFree(h->op_pack);
   cudaFree(h->op_ctr);
+  cudaFree(h->d_gates);
   if (h->ev_ts) cudaEventDestroy(h->ev_ts);
   for (auto e : h->ev_pool) cudaEventDestroy(e);
   delete h;
+}
+
+int bullet_set_split(bullet_handle* h, int pre_lo, int pre_hi, int dec_lo, int dec_hi, void* stream) {
+  if (!h) return set_err(BULLET_EINVAL, "null handle");
+  if (h->host_only) return set_err(BULLET_EUNSUPPORTED, "host-only handle");
+  const int N = h->n_sms;
+  auto ok = [&](int x) { return x >= 0 && x <= N && (x % GRAN == 0 || x == N); };
+  if (!ok(pre_lo) || !ok(pre_hi) || !ok(dec_lo) || !ok(dec_hi) || pre_lo > pre_hi || dec_lo > dec_hi)
+    return set_err(BULLET_ESMRANGE, "ranges [%d,%d) [%d,%d) not within [0,%d] on step %d", pre_lo, pre_hi,
+                   dec_lo, dec_hi, N, GRAN);
+  CK(launch_set_gates(h->d_gates, gate_of(h, pre_lo, pre_hi), gate_of(h, dec_lo, dec_hi), (cudaStream_t)stream));
+  return BULLET_OK;
 }
 
 // ------------------------------------------------ fused peer all-reduce setup

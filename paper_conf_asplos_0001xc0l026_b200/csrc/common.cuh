@@ -21,6 +21,8 @@ struct Gate {
 // Per-launch context passed by value to every kernel.
 struct Launch {
   Gate gate;
+  const Gate* gdev;  // non-null: the phase's SM set lives in device memory (BULLET_DEVICE_SPLIT) —
+                     // a captured graph then follows bullet_set_split at replay
   int* ctr;        // work counter, zero at launch
   int* burn;       // CTAs that left out of range (zero at launch; nullable)
   int32_t* log;    // smid log (nullable): [0] = count, then {launch, unit, smid, phase}
@@ -46,7 +48,7 @@ __device__ __forceinline__ bool gate_ok(const Gate& g) {
 // a moment): then this last CTA works where it is, so a launch can never end
 // with its units unprocessed (correctness never depends on CTA placement).
 __device__ __forceinline__ bool gate_enter(const Launch& L) {
-  if (gate_ok(L.gate)) return true;
+  if (L.gdev ? gate_ok(*L.gdev) : gate_ok(L.gate)) return true;
   if (!L.burn) return false;
   int last = 0;   // (no shared memory: kernels align their dynamic smem base)
   if (threadIdx.x == 0) last = atomicAdd(L.burn, 1) == (int)(gridDim.x * gridDim.y * gridDim.z) - 1;

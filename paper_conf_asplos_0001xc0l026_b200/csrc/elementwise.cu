@@ -330,6 +330,15 @@ cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st) {
   k_plan<<<grid, 256, 0, st>>>(a);
   return cudaGetLastError();
 }
+// BULLET_DEVICE_SPLIT: write both phases' SM sets (one warp, stream-ordered).
+__global__ void k_set_gates(Gate* d, Gate pre, Gate dec) {
+  if (threadIdx.x < 8) { d[0].m[threadIdx.x] = pre.m[threadIdx.x]; d[1].m[threadIdx.x] = dec.m[threadIdx.x]; }
+}
+cudaError_t launch_set_gates(Gate* d_gates, const Gate& pre, const Gate& dec, cudaStream_t st) {
+  k_set_gates<<<1, 32, 0, st>>>(d_gates, pre, dec);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_probe(int* out, int n, cudaStream_t st) {
   k_probe<<<n, 32, 0, st>>>(out, n);
   return cudaGetLastError();
@@ -350,6 +359,7 @@ static cudaError_t preload_elt_t() {
 cudaError_t preload_elementwise() {
   cudaFuncAttributes f;
   cudaError_t e = cudaFuncGetAttributes(&f, k_plan);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_set_gates);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_probe);
   if (e == cudaSuccess) e = preload_elt_t<float>();
   if (e == cudaSuccess) e = preload_elt_t<__nv_bfloat16>();

@@ -329,3 +329,58 @@ def test_cuda_graph_replay_matches_stream_launch(small_bf16):
         g.replay()
         torch.cuda.synchronize()
         assert torch.equal(pre.hidden, want[0]) and torch.equal(dec.hidden, want[1])
+
+
+def test_device_split_graph_follows_set_split(small_bf16):
+    """NEXT-4 with the split in device memory: one graph captured from a
+    BULLET_DEVICE_SPLIT step at p = 64 replays at p = 100 after
+    bullet_set_split — every unit runs inside the NEW ranges (smid log), and
+    the bits equal the p = 64 replay (the captured GEMM plans fix the
+    arithmetic; the split only moves where units run)."""
+    S = small_bf16
+    B = S.B
+    pre, dec = S.batches(0, 2)
+    x_pre, x_dec = pre.hidden.clone(), dec.hidden.clone()
+    sp, sd = phase_streams()
+    log = S.bl.set_smid_log(400000)
+    sigma = list(S.bl.sm_order())
+
+    def enqueue():
+        ev = torch.cuda.Event(); ev.record(sp); sd.wait_event(ev)
+        S.bl.step(pre, dec, 64, B.CORUN | B.DEVICE_SPLIT | B.SMID_LOG, sp, sd)
+        ev2 = torch.cuda.Event(); ev2.record(sd); sp.wait_event(ev2)
+
+    try:
+        # direct DEVICE_SPLIT step == plain step at the same split
+        S.bl.set_split((0, 64), (64, 148), sp)
+        enqueue()
+        torch.cuda.synchronize()
+        direct = (pre.hidden.clone(), dec.hidden.clone())
+        pre.hidden.copy_(x_pre); dec.hidden.copy_(x_dec)
+        torch.cuda.synchronize()
+        S.bl.step(pre, dec, 64, B.CORUN, sp, sd)
+        torch.cuda.synchronize()
+        assert torch.equal(pre.hidden, direct[0]) and torch.equal(dec.hidden, direct[1])
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=sp):
+            enqueue()
+        outs = []
+        for p in (64, 100):
+            pre.hidden.copy_(x_pre); dec.hidden.copy_(x_dec)
+            S.bl.set_split((0, p), (p, 148), sp)
+            log.zero_()
+            torch.cuda.synchronize()
+            g.replay()
+            torch.cuda.synchronize()
+            outs.append((pre.hidden.clone(), dec.hidden.clone()))
+            n = int(log[0].item())
+            e = log[1:1 + 4 * n].view(n, 4).cpu().numpy()
+            allowed = {0: set(sigma[0:p]), 1: set(sigma[p:148])}
+            assert n > 0
+            for ph in (0, 1):
+                rows = e[e[:, 3] == ph]
+                assert set(rows[:, 2].tolist()) <= allowed[ph], (p, ph)
+        assert torch.equal(outs[0][0], outs[1][0]) and torch.equal(outs[0][1], outs[1][1])
+        assert torch.equal(outs[0][0], direct[0]) and torch.equal(outs[0][1], direct[1])
+    finally:
+        S.bl.set_smid_log(None)
