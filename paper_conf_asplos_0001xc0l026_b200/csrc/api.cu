@@ -109,7 +109,7 @@ struct PhaseWS {
   int max_tok = 0;
   int* rbc = nullptr;              // fused-norm row-block counters [n_rbc_slices][max_rb], zeroed per step
   int max_rb = 0, n_rbc_slices = 0, next_rbc = 0;
-  int* order = nullptr;            // decode rows in LPT order (plan kernel), valid this step if order_ok
+  int4* order = nullptr;           // decode rows in LPT order (plan kernel), valid this step if order_ok
   bool order_ok = false;
 };
 
@@ -850,7 +850,7 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
               cudaMalloc(&P.tiles, (T / ATTN_TC_BQ + 1024) * sizeof(int2)) == cudaSuccess &&
               cudaMalloc(&P.n_tiles, sizeof(int)) == cudaSuccess &&
               cudaMalloc(&P.tok, T * sizeof(TokInfo)) == cudaSuccess &&
-              cudaMalloc(&P.order, T * sizeof(int)) == cudaSuccess &&
+              cudaMalloc(&P.order, T * sizeof(int4)) == cudaSuccess &&
               cudaMalloc(&P.rbc, (size_t)(2 * c.n_layers + 2) * ((T + 127) / 128) * sizeof(int)) == cudaSuccess;
     P.max_rb = (int)((T + 127) / 128);
     P.n_rbc_slices = 2 * c.n_layers + 2;

@@ -135,9 +135,15 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
       if (u >= units) u = -1;
       Slot sl{u, 0, 0, 0};
       if (u >= 0) {
-        sl.t = a.tok_base + (a.order ? __ldg(a.order + u / a.Hkv) : u / a.Hkv);
-        const int r = find_req(a.cu, a.n_reqs, sl.t);
-        sl.pos = __ldg(a.ctx + r) + (sl.t - __ldg(a.cu + r));
+        int r;
+        if (a.order) {   // (row, request, position) from the plan kernel: one load
+          const int4 od = __ldg(a.order + u / a.Hkv);
+          sl.t = a.tok_base + od.x; r = od.y; sl.pos = od.z;
+        } else {
+          sl.t = a.tok_base + u / a.Hkv;
+          r = find_req(a.cu, a.n_reqs, sl.t);
+          sl.pos = __ldg(a.ctx + r) + (sl.t - __ldg(a.cu + r));
+        }
         sl.nb = sl.pos / KB + 1;
         const int32_t* bt = a.bt + (size_t)r * a.max_blocks;
         for (int b = lane; b < sl.nb; b += 32) btbuf[slot * MAXNB + b] = __ldg(bt + b);
@@ -241,6 +247,11 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
       __syncwarp();
       const int b = wl + j * GW;
       const uint32_t kt = my_s + (n_cons % DEPTH) * STAGE_BYTES;
+      if (a.dbg & 1) {   // diagnostics (BULLET_DBG): stream only, no math
+        __syncwarp();
+        ++n_cons;
+        continue;
+      }
       float s[4] = {0.f, 0.f, 0.f, 0.f}, s2[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
       for (int ks = 0; ks < 8; ks += 2) {   // two independent accumulation chains
@@ -294,6 +305,11 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
     // the next unit's first DEPTH-1 blocks fly during the merge; the stage
     // left free holds this warp's merge record
     fill(it + NG, DEPTH - 1);
+    if (a.dbg & 2) {   // diagnostics (BULLET_DBG): skip the merge and the output
+      __syncwarp();
+      if (lane == 0) mbar_arrive(uqe + slot);
+      continue;
+    }
     // full row sums over the 8 key lanes of each head
 #pragma unroll
     for (int o = 4; o < 32; o <<= 1) {

@@ -260,7 +260,12 @@ __global__ void k_plan(PlanArgs a) {
         for (int b = DEC_ORDER_BUCKETS; b >= 0; --b) { const int c = hist[b]; hist[b] = run; run += c; }
       }
       __syncthreads();
-      for (int i = threadIdx.x; i < n; i += blockDim.x) a.order[atomicAdd(hist + nb_of(i), 1)] = i;
+      for (int i = threadIdx.x; i < n; i += blockDim.x) {
+        const int t = a.order_base + i;
+        const int r = find_req(a.cu, a.n_reqs, t);
+        const int pos = __ldg(a.ctx + r) + (t - __ldg(a.cu + r));
+        a.order[atomicAdd(hist + nb_of(i), 1)] = make_int4(i, r, pos, 0);
+      }
     }
     if (threadIdx.x == 0 && a.tiles) {
       int maxt = 0;

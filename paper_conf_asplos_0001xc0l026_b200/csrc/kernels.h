@@ -112,7 +112,8 @@ struct AttnArgs {
   const int* n_tiles;     // device count of `tiles`
   int dbg;                // diagnostics (BULLET_DBG env): bit0 = decode consumers skip math
   int tok_base;           // decode kernel: its rows are tokens [tok_base, n_tok) (mixed batches)
-  const int* order;       // decode kernel (nullable): unit token i -> tok_base + order[i], longest context first
+  const int4* order;      // decode kernel (nullable): unit row i -> (token - tok_base, request, position, -),
+                          // longest context first; saves the claimer its per-unit request search
   Launch L;
 };
 
@@ -132,7 +133,7 @@ struct PlanArgs {
   int* zero2; int n_zero2;   // second array zeroed per step (fused-norm row-block counters)
   // decode rows [order_base, n_tok) in descending context length (nullable): LPT order of the
   // decode attention's units (the longest rows start first, the tail is short)
-  int* order; int order_base;
+  int4* order; int order_base;
 };
 
 // launchers (return cudaError_t of the launch)

@@ -26,11 +26,17 @@ def main():
     ap.add_argument("--sms", type=int, nargs="+", default=[60, 68, 148])
     ap.add_argument("--reps", type=int, default=10)
     ap.add_argument("--tag", default="")
+    ap.add_argument("--uniform", type=int, nargs="*", default=None,
+                    help="uniform contexts instead of the workload's: ctx values, n = 512K tokens / ctx")
     a = ap.parse_args()
     torch.cuda.set_device(0)
     wl = synth.workload(a.config)
     m = synth.MODELS[wl.model]
-    ctx = list(wl.decode_ctx)
+    for ctx in ([list(wl.decode_ctx)] if a.uniform is None else [[c] * max(1, (1 << 19) // c) for c in a.uniform]):
+        run(a, m, ctx)
+
+
+def run(a, m, ctx):
     n = len(ctx)
     lay = synth.paged_layout([1] * n, ctx, 16)
     pk = torch.randn(lay.n_blocks, m.n_kv_heads, 16, m.head_dim, device="cuda").to(torch.bfloat16)
@@ -53,7 +59,8 @@ def main():
         torch.cuda.synchronize()
         us = e0.elapsed_time(e1) / a.reps * 1e3
         gbs = kv_bytes / us / 1e3
-        print(json.dumps({"config": a.config, "kind": a.kind, "tag": a.tag, "sms": msm, "us": round(us, 1),
+        print(json.dumps({"config": a.config, "kind": a.kind, "tag": a.tag, "ctx": ctx[0] if a.uniform else "mix",
+                          "n": n, "units": n * m.n_kv_heads, "sms": msm, "us": round(us, 1),
                           "gbs": round(gbs), "gbs_per_sm": round(gbs / msm, 1)}), flush=True)
 
 
