@@ -151,11 +151,53 @@ def fit(N, pts, m_shape):
         return float(np.mean([abs(pm.predict_us(p["q"], p["c"], p["m"], p["co"]) / 1e3 - p["ms"]) / p["ms"] for p in ps]))
     P["fit"] = {"n_points": len(pts), "n_train": len(train), "n_heldout": len(test),
                 "mre_train": mre(train), "mre_heldout": mre(test), "paper_mre": 0.191,
+                "slo_accuracy_heldout": slo_accuracy(pm, test), "paper_slo_accuracy": 0.88,
                 "source": "scripts/fit_perfmodel.py on B200"}
     return P
 
 
+def split_heldout(pts):
+    rng = np.random.default_rng(0)     # the same split fit() uses
+    idx = rng.permutation(len(pts))
+    held = set(idx[: len(pts) // 5].tolist())
+    return [p for i, p in enumerate(pts) if i not in held], [p for i, p in enumerate(pts) if i in held]
+
+
+def slo_accuracy(pm, pts, quantiles=(0.25, 0.5, 0.75)):
+    """P:L311's second number: how often the model classifies a layer step
+    the same way as the measurement with respect to a latency target ("meets"
+    = time <= target).  Reading: targets at the 25 / 50 / 75 % quantiles of
+    the measured times of each kind (prefill / decode layer steps), i.e. the
+    decisions the scheduler takes near its SLO boundaries; mean over kinds
+    and quantiles."""
+    acc = []
+    for kind in sorted({p["kind"] for p in pts}):
+        ps = [p for p in pts if p["kind"] == kind]
+        meas = np.array([p["ms"] for p in ps])
+        pred = np.array([pm.predict_us(p["q"], p["c"], p["m"], p["co"]) / 1e3 for p in ps])
+        for qn in quantiles:
+            thr = float(np.quantile(meas, qn))
+            acc.append(float(np.mean((pred <= thr) == (meas <= thr))))
+    return float(np.mean(acc))
+
+
+def evaluate(params_path, points_path):
+    """Held-out MRE and SLO-classification accuracy of committed parameters
+    (host-only model: no GPU)."""
+    P = json.load(open(params_path))
+    pts = json.load(open(points_path))
+    _, test = split_heldout(pts)
+    pm = predictor(synth.MODELS["llama3.1-8b"], P, P["M"])
+    mre = float(np.mean([abs(pm.predict_us(p["q"], p["c"], p["m"], p["co"]) / 1e3 - p["ms"]) / p["ms"] for p in test]))
+    return {"n_heldout": len(test), "mre_heldout": mre, "slo_accuracy_heldout": slo_accuracy(pm, test),
+            "slo_accuracy_all": slo_accuracy(pm, pts), "paper": {"mre": 0.191, "slo_accuracy": 0.88}}
+
+
 def main():
+    if len(sys.argv) > 1 and sys.argv[1] == "--evaluate":
+        pp = os.path.join(ROOT, "profiles", "perf_params_b200.json")
+        print(json.dumps(evaluate(pp, pp.replace(".json", "_points.json"))))
+        return
     out = sys.argv[1] if len(sys.argv) > 1 else os.path.join(ROOT, "profiles", "perf_params_b200.json")
     t0 = time.time()
     N, pts = measure()

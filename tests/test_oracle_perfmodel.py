@@ -185,3 +185,22 @@ def test_degenerate_states():
     P = PM.default_params()
     assert PM.choose_split(P, MODEL, _state(decode_tokens=[], decode_elapsed_ms=[]), SLO) == (148, 0)
     assert PM.choose_split(P, MODEL, _state(prefill_lens=[], prefill_waited_ms=[]), SLO) == (0, 32)
+
+
+def test_fitted_model_heldout_report_reproduces():
+    """The reported fit quality (profiles/r01c_perfmodel_eval.json: held-out
+    MRE and SLO-classification accuracy) is what the committed
+    parameters give on the committed B200 measurements with the host-only
+    model of the product (bullet_perf_create) — no GPU needed."""
+    import json
+    import os
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, os.path.join(root, "scripts"))
+    import fit_perfmodel as F
+    pp = os.path.join(root, "profiles", "perf_params_b200.json")
+    got = F.evaluate(pp, pp.replace(".json", "_points.json"))
+    want = json.load(open(os.path.join(root, "profiles", "r01c_perfmodel_eval.json")))
+    assert abs(got["mre_heldout"] - want["mre_heldout"]) < 1e-9
+    assert abs(got["slo_accuracy_heldout"] - want["slo_accuracy_heldout"]) < 1e-9
+    assert got["mre_heldout"] < 0.191 and got["slo_accuracy_heldout"] > 0.88   # paper's numbers, context
