@@ -174,6 +174,9 @@ typedef struct {
   int w_max;                     /* W_max, Alg. 1 l.18 */
   int v_min;                     /* minimum decode SMs when co-running */
   double percentile;             /* 0.9 (Alg. 1 "P90") */
+  int objective;                 /* 0: Alg. 1 as read (DESIGN R-14..R-17); 1: when both SLOs hold,
+                                    the split with the most predicted tokens/s among the SLO-feasible
+                                    ones instead of the fewest decode SMs (R-21) */
 } bullet_slo;
 
 /* Create a handle on the current CUDA device.  Probes the live SM ids

@@ -196,7 +196,28 @@ def choose_split(P, model, state, slo, gran=2):
     def balanced():
         return min(cands, key=lambda v: (max(ev[v][0], ev[v][1]), v))   # R-16, tie -> larger u
 
-    if ok_t and ok_d:
+    def max_throughput():
+        # R-21 (objective 1, "meet stringent SLO requirements while
+        # maximizing throughput"): among the SLO-feasible splits, the most
+        # predicted tokens per ms; ties to the larger prefill share
+        dec = _phase_shape(model, [1] * len(state["decode_tokens"]),
+                           [int(math.floor(state["decode_mean_ctx"] + 0.5))] * len(state["decode_tokens"]))
+        n_pre = float(sum(state["prefill_lens"]))
+        best, best_t = None, -1.0
+        for v in cands:
+            if ev[v][0] > 1.0 or ev[v][1] > 1.0:
+                continue
+            t_p, t_d = ev[v][2], layer_time(dec, P, v, N - v) * 1e3
+            k = max(1, int(math.floor(t_p / t_d + 0.5))) if t_d > 0 else 1
+            cyc = max(t_p, k * t_d)
+            tput = (n_pre + len(state["decode_tokens"]) * k) / cyc if cyc > 0 else 0.0
+            if tput > best_t:
+                best, best_t = v, tput
+        return best
+
+    if ok_t and ok_d and slo.get("objective", 0) == 1 and max_throughput() is not None:
+        v = max_throughput()                           # R-21
+    elif ok_t and ok_d:
         v = reduce_decode()                            # line 12-13
     elif not ok_t and not ok_d:
         v = balanced()                                 # line 15-16 (R-14: follow the algorithm)

@@ -71,7 +71,7 @@ class SchedState(ctypes.Structure):
 
 class Slo(ctypes.Structure):
     _fields_ = [("ttft_norm_ms_per_tok", c_double), ("tpot_ms", c_double), ("w_max", c_int),
-                ("v_min", c_int), ("percentile", c_double)]
+                ("v_min", c_int), ("percentile", c_double), ("objective", c_int)]
 
 
 _lib = None
@@ -380,7 +380,7 @@ class Bullet:
                        i32("decode_tokens"), f64("decode_elapsed_ms"), state["decode_mean_ctx"],
                        state["u_k"], state["v_k"])
         sl = Slo(slo["ttft_norm_ms_per_tok"], slo["tpot_ms"], slo["w_max"], slo["v_min"],
-                 slo.get("percentile", 0.9))
+                 slo.get("percentile", 0.9), int(slo.get("objective", 0)))
         p, k = c_int(), c_int()
         _check(lib().bullet_choose_split(self.h, ctypes.byref(s), ctypes.byref(sl), ctypes.byref(p),
                                          ctypes.byref(k)))

@@ -1075,7 +1075,8 @@ int bullet_choose_split(const bullet_handle* h, const bullet_sched_state* s, con
   for (int i = 0; i < s->n_decode; ++i) { S.decode_tokens.push_back(s->decode_tokens[i]); S.decode_elapsed_ms.push_back(s->decode_elapsed_ms[i]); }
   S.decode_mean_ctx = s->decode_mean_ctx;
   S.u_k = s->u_k; S.v_k = s->v_k;
-  Slo sl{slo->ttft_norm_ms_per_tok, slo->tpot_ms, slo->w_max, slo->v_min, slo->percentile};
+  if (slo->objective < 0 || slo->objective > 1) return set_err(BULLET_EINVAL, "slo objective");
+  Slo sl{slo->ttft_norm_ms_per_tok, slo->tpot_ms, slo->w_max, slo->v_min, slo->percentile, slo->objective};
   PerfParams P = h->perf;
   P.M = h->n_sms;
   choose_split(P, model_shape(h), S, sl, GRAN, prefill_sm_count, decode_layer_steps);

@@ -276,8 +276,32 @@ void choose_split(const PerfParams& P, const PhaseShape& model, const SchedState
       if (std::max(ev[v].ttft, ev[v].tpot) < std::max(ev[best].ttft, ev[best].tpot)) best = v;
     return best;
   };
+  // R-21 (objective 1): "meet stringent SLO requirements while maximizing
+  // throughput" — among the splits that keep both SLOs, the one with
+  // the most predicted tokens per ms: (prefill tokens + decode tokens x k) /
+  // max(t_p, k t_d), k = round(t_p / t_d) >= 1; ties to the larger prefill
+  // share.  None feasible: Alg. 1's rule.
+  auto max_throughput = [&]() -> int {
+    PhaseShape dec = model;
+    const int mctx = (int)std::lround(S.decode_mean_ctx);
+    dec.q_lens.assign(S.decode_tokens.size(), 1); dec.ctx_lens.assign(S.decode_tokens.size(), mctx);
+    double n_pre = 0.0;
+    for (int q : S.prefill_lens) n_pre += q;
+    int best = -1;
+    double best_t = -1.0;
+    for (int v : cands) {
+      if (ev[v].ttft > 1.0 || ev[v].tpot > 1.0) continue;
+      const double t_p = ev[v].t_p, t_d = layer_time(dec, P, v, N - v) * 1e3;
+      const int k = t_d > 0 ? std::max(1, (int)std::floor(t_p / t_d + 0.5)) : 1;
+      const double cyc = std::max(t_p, k * t_d);
+      const double tput = cyc > 0 ? (n_pre + (double)S.decode_tokens.size() * k) / cyc : 0.0;
+      if (tput > best_t) { best_t = tput; best = v; }
+    }
+    return best;
+  };
   int v;
-  if (ok_t && ok_d) v = reduce_decode();
+  if (ok_t && ok_d && slo.objective == 1 && max_throughput() >= 0) v = max_throughput();
+  else if (ok_t && ok_d) v = reduce_decode();
   else if (!ok_t && !ok_d) v = balanced();
   else if (ok_t && !ok_d && (int)S.pending_lens.size() <= slo.w_max) v = reduce_prefill();
   else v = reduce_decode();

@@ -39,6 +39,7 @@ struct Slo {
   double ttft_norm, tpot_ms;
   int w_max, v_min;
   double percentile;
+  int objective;   // 0: Alg. 1 as read (R-14..R-17); 1: + throughput among SLO-feasible splits (R-21)
 };
 
 double wave_idle(double g, double M);

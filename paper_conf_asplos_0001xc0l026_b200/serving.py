@@ -19,6 +19,8 @@ policies see the same arrival process.
 
 Policies:
   bullet      co-run, (p, k) from Alg. 1 (bullet_choose_split)
+  bullet_tput the same with objective 1: when both SLOs hold, the split with
+              the most predicted tokens/s among the SLO-feasible ones (R-21)
   timesliced  same cycle structure, both phases on all SMs one after the
               other (BULLET_TIMESLICED), k from the model's full-GPU balance
   prefill_first  vLLM-style: while a prefill batch exists decode is paused
@@ -107,10 +109,11 @@ class Slo:
     w_max: int = 4
     v_min: int = 16
     percentile: float = 0.9
+    objective: int = 0                 # 1: throughput among SLO-feasible splits (R-21, policy bullet_tput)
 
     def as_dict(self):
         return dict(ttft_norm_ms_per_tok=self.ttft_norm_ms_per_tok, tpot_ms=self.tpot_ms,
-                    w_max=self.w_max, v_min=self.v_min, percentile=self.percentile)
+                    w_max=self.w_max, v_min=self.v_min, percentile=self.percentile, objective=self.objective)
 
 
 class ServingLoop:
@@ -121,7 +124,10 @@ class ServingLoop:
     def __init__(self, n_layers: int, n_sms: int, step, choose, policy: str, allocator: BlockAllocator,
                  slo: Slo = Slo(), prefill_layers_per_cycle: int = 1, max_prefill_tokens: int = 8192,
                  max_decodes: int = 256, k_full: int = 4, chunk_tokens: int = 2048):
-        assert policy in ("bullet", "timesliced", "prefill_first", "chunked")
+        assert policy in ("bullet", "bullet_tput", "timesliced", "prefill_first", "chunked")
+        if policy == "bullet_tput":   # Alg. 1 with the throughput objective among feasible splits (R-21)
+            policy = "bullet"
+            slo = Slo(**{**slo.__dict__, "objective": 1})
         self.L, self.N = n_layers, n_sms
         self.step, self.choose, self.policy = step, choose, policy
         self.alloc, self.slo = allocator, slo

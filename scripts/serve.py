@@ -91,7 +91,8 @@ def main():
     ap.add_argument("--rate", type=float, default=60.0, help="requests / s (Poisson)")
     ap.add_argument("--duration", type=float, default=10.0, help="seconds of arrivals")
     ap.add_argument("--layers", type=int, default=32)
-    ap.add_argument("--policies", nargs="+", default=["bullet", "timesliced", "prefill_first", "chunked"])
+    ap.add_argument("--policies", nargs="+", default=["bullet", "bullet_tput", "timesliced", "prefill_first",
+                                                       "chunked"])
     ap.add_argument("--chunk-tokens", type=int, default=2048, help="chunked policy: token budget per iteration")
     ap.add_argument("--max-decodes", type=int, default=256)
     ap.add_argument("--max-prefill", type=int, default=8192)
@@ -115,6 +116,7 @@ def main():
                               chunk_tokens=a.chunk_tokens)
         t0 = time.perf_counter()
         res = loop.run(trace)
+        res["policy"] = pol
         res.update(rate_req_s=a.rate, arrivals_s=a.duration, layers=a.layers, k_timesliced=k_ts,
                    wall_s=time.perf_counter() - t0, model="llama3.1-8b", data="synthetic Poisson trace")
         ps = [c[1] for c in loop.log if 0 < c[1] < g.N]

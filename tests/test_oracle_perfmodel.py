@@ -145,6 +145,29 @@ def test_case_both_ok_reduces_decode_to_minimal_feasible():
     assert k >= 1
 
 
+def test_objective_throughput_picks_feasible_split_with_most_tokens_per_ms():
+    """R-21 (objective 1): both SLOs met -> among the SLO-feasible
+    splits the one with the highest predicted (prefill tokens + decode tokens
+    x k) / cycle, checked by brute force over every candidate; objective 0
+    keeps Alg. 1's ReduceDecodeSM."""
+    P = PM.default_params()
+    st = _state()
+    slo1 = dict(SLO, objective=1)
+    ev = _eval_all(P, st, slo1)
+    dec = PM._phase_shape(MODEL, [1] * 64, [1024] * 64)
+
+    def tput(v):
+        t_p, t_d = ev[v][2], PM.layer_time(dec, P, v, P["M"] - v) * 1e3
+        k = max(1, int(math.floor(t_p / t_d + 0.5)))
+        return (2048 + 64 * k) / max(t_p, k * t_d), k
+    feas = [v for v in ev if ev[v][0] <= 1 and ev[v][1] <= 1]
+    u, k = PM.choose_split(P, MODEL, st, slo1)
+    v = P["M"] - u
+    assert v in feas and tput(v)[0] == max(tput(w)[0] for w in feas) and k == tput(v)[1]
+    u0, _ = PM.choose_split(P, MODEL, st, SLO)          # objective 0 unchanged: fewest decode SMs
+    assert P["M"] - u0 == min(feas) and tput(P["M"] - u0)[0] <= tput(v)[0]
+
+
 def test_case_both_violated_sets_balanced():
     """Alg. 1 l.15-16 (R-14): both violated -> argmin of max ratio."""
     P = PM.default_params()
