@@ -253,6 +253,15 @@ int bullet_set_split(bullet_handle *h, int pre_lo, int pre_hi, int dec_lo, int d
 int bullet_model_predict(const bullet_handle *h, const bullet_batch_shape *shape, int sm_count,
                          int corun_sm_count, double *t_layer_us);
 
+/* Online estimator feedback ("correlating deviations between
+ * predicted latency and observed execution times across scheduling cycles,
+ * using the inter-cycle duration t_{k+1} - t_k as dynamic feedback"): read /
+ * replace the co-location factors p_c, p_b of Eq. 2 that every co-run
+ * prediction (corun_sm_count > 0) and bullet_choose_split use.  Errors:
+ * EINVAL (non-positive factors). */
+int bullet_get_colocation(const bullet_handle *h, double *p_c, double *p_b);
+int bullet_set_colocation(bullet_handle *h, double p_c, double p_b);
+
 /* Alg. 1 and the §3.3.3 search under the readings
  * of DESIGN.md §3 (R-14..R-17): returns the prefill SM count for the next
  * cycle (N = decode paused) and the number of decode layer-steps to co-run

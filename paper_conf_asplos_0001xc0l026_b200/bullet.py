@@ -89,7 +89,8 @@ def lib():
                      "bullet_set_smid_log", "bullet_sync", "bullet_nccl_unique_id", "bullet_op_gemm",
                      "bullet_op_rmsnorm", "bullet_op_rope_kv", "bullet_op_attention",
                      "bullet_profile_read", "bullet_launch_count", "bullet_tp_base", "bullet_tp_ipc_handle",
-                     "bullet_tp_connect", "bullet_tp_connect_ipc", "bullet_tp_hidden", "bullet_set_split"):
+                     "bullet_tp_connect", "bullet_tp_connect_ipc", "bullet_tp_hidden", "bullet_set_split",
+                     "bullet_get_colocation", "bullet_set_colocation"):
             getattr(L, name).restype = c_int
         L.bullet_create.argtypes = [ctypes.POINTER(ModelCfg), ctypes.POINTER(KvPool), c_void_p,
                                     ctypes.c_char_p, ctypes.POINTER(c_void_p)]
@@ -113,6 +114,8 @@ def lib():
         L.bullet_nccl_unique_id.argtypes = [c_void_p]
         L.bullet_tp_base.argtypes = [c_void_p, ctypes.POINTER(c_void_p)]
         L.bullet_set_split.argtypes = [c_void_p, c_int, c_int, c_int, c_int, c_void_p]
+        L.bullet_get_colocation.argtypes = [c_void_p, P_f64, P_f64]
+        L.bullet_set_colocation.argtypes = [c_void_p, c_double, c_double]
         L.bullet_tp_ipc_handle.argtypes = [c_void_p, c_void_p]
         L.bullet_tp_connect.argtypes = [c_void_p, ctypes.POINTER(c_void_p)]
         L.bullet_tp_connect_ipc.argtypes = [c_void_p, c_void_p]
@@ -355,6 +358,14 @@ class Bullet:
         n = ctypes.c_longlong()
         _check(lib().bullet_launch_count(self.h, ctypes.byref(n)))
         return n.value
+
+    def colocation(self):
+        a, b = c_double(), c_double()
+        _check(lib().bullet_get_colocation(self.h, ctypes.byref(a), ctypes.byref(b)))
+        return a.value, b.value
+
+    def set_colocation(self, p_c: float, p_b: float):
+        _check(lib().bullet_set_colocation(self.h, float(p_c), float(p_b)))
 
     def predict_us(self, q_lens, ctx_lens, sm_count, corun_sm_count=0) -> float:
         q = np.ascontiguousarray(q_lens, dtype=np.int32); c = np.ascontiguousarray(ctx_lens, dtype=np.int32)

@@ -1083,6 +1083,18 @@ int bullet_choose_split(const bullet_handle* h, const bullet_sched_state* s, con
   return BULLET_OK;
 }
 
+int bullet_get_colocation(const bullet_handle* h, double* p_c, double* p_b) {
+  if (!h || !p_c || !p_b) return set_err(BULLET_EINVAL, "null");
+  *p_c = h->perf.p_c; *p_b = h->perf.p_b;
+  return BULLET_OK;
+}
+
+int bullet_set_colocation(bullet_handle* h, double p_c, double p_b) {
+  if (!h || !(p_c > 0.0) || !(p_b > 0.0)) return set_err(BULLET_EINVAL, "co-location factors must be > 0");
+  h->perf.p_c = p_c; h->perf.p_b = p_b;
+  return BULLET_OK;
+}
+
 int bullet_profile_read(bullet_handle* h, int32_t* kind, int32_t* phase, int32_t* layer, float* ms,
                         int cap, int* n) {
   if (!h || !n || cap < 0) return set_err(BULLET_EINVAL, "null");

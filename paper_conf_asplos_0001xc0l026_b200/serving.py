@@ -123,7 +123,8 @@ class ServingLoop:
 
     def __init__(self, n_layers: int, n_sms: int, step, choose, policy: str, allocator: BlockAllocator,
                  slo: Slo = Slo(), prefill_layers_per_cycle: int = 1, max_prefill_tokens: int = 8192,
-                 max_decodes: int = 256, k_full: int = 4, chunk_tokens: int = 2048):
+                 max_decodes: int = 256, k_full: int = 4, chunk_tokens: int = 2048, feedback_model=None,
+                 feedback_alpha: float = 0.2):
         assert policy in ("bullet", "bullet_tput", "timesliced", "prefill_first", "chunked")
         if policy == "bullet_tput":   # Alg. 1 with the throughput objective among feasible splits (R-21)
             policy = "bullet"
@@ -136,8 +137,28 @@ class ServingLoop:
         self.split = (n_sms // 2, n_sms - n_sms // 2)
         self.chunk_tokens = chunk_tokens
         self.log = []                 # per cycle: (now, p, k, prefill tokens, decodes, ms)
+        # online estimator feedback: after every co-run cycle the
+        # ratio measured / predicted cycle time updates an EMA that rescales
+        # the model's co-location factors p_c, p_b (bullet_set_colocation),
+        # so the next decisions see the contention actually observed
+        self.fb = feedback_model
+        self.fb_alpha, self.fb_ratio = feedback_alpha, 1.0
+        self.fb_base = feedback_model.colocation() if feedback_model is not None else None
 
     # ------------------------------------------------------------ helpers
+    def _feedback(self, pw, dw, p, ms):
+        """correlate the observed cycle time with the prediction."""
+        n_pl, k = pw.layer_end - pw.layer_begin, dw.layer_end - dw.layer_begin
+        t_p = self.fb.predict_us(pw.q_lens, pw.ctx_lens, p, self.N - p) / 1e3 * n_pl
+        t_d = self.fb.predict_us(dw.q_lens, dw.ctx_lens, self.N - p, p) / 1e3 * k
+        pred = max(t_p, t_d)
+        if pred <= 0:
+            return
+        r = ms / pred * self.fb_ratio        # ratio to the uncorrected model
+        r = min(2.0, max(0.5, r))
+        self.fb_ratio = (1 - self.fb_alpha) * self.fb_ratio + self.fb_alpha * r
+        self.fb.set_colocation(self.fb_base[0] / self.fb_ratio, self.fb_base[1] / self.fb_ratio)
+
     def _alg1_state(self, now, prefill, layers_done, pending, members):
         return dict(layers_done=layers_done if prefill else 0, total_layers=self.L,
                     prefill_lens=[r.prompt for r in prefill] if prefill else [],
@@ -294,6 +315,8 @@ class ServingLoop:
             self.split = (p, self.N - p)
             ms = self.step(pw, dw, p, mode)
             self.log.append((now, p, k, sum(pw.q_lens) if pw else 0, len(members) if dw else 0, ms))
+            if self.fb is not None and mode == "corun" and pw is not None and dw is not None and 0 < p < self.N:
+                self._feedback(pw, dw, p, ms)
             now += ms
             # ---- advance the prefill batch
             if pw is not None:

@@ -27,8 +27,9 @@ from workload import synth  # noqa: E402
 M_GRID = [16, 32, 48, 64, 80, 96, 112, 128, 148]
 PRE_SHAPES = [[512], [1024], [2048], [4096], [8192], synth.workload("sharegpt-8b").prefill_lens]
 DEC_SHAPES = [(bs, cl) for bs in (32, 64, 128, 256) for cl in (512, 1024, 2048, 4096)]
-CORUN = [(pre, dec, p) for pre in ([2048], synth.workload("sharegpt-8b").prefill_lens)
-         for dec in ((128, 1024), (256, 2048)) for p in (48, 72, 96, 120)]
+L_CO = 16
+CORUN = [(pre, dec, p) for pre in ([2048], synth.workload("sharegpt-8b").prefill_lens, [8192])
+         for dec in ((128, 1024), (256, 2048), (256, 512)) for p in (48, 72, 96, 120, 132)]
 
 
 class Rig:
@@ -41,8 +42,12 @@ class Rig:
         k, v = synth.kv_pool(self.m, self.n_blocks, 16, 0, device="cuda")
         self.pool = [(k.bfloat16(), v.bfloat16())]
         del k, v
-        self.bl = B.Bullet(B.Model.of(self.m), self.pool, 8192, 256, 8192 + 32)
-        self.bl.set_layer_weights(0, self.w)
+        # L_CO layers sharing one weight set and one KV pool: a co-run point
+        # runs k decode layer-steps against one prefill layer so the phases
+        # overlap for the whole step (as in bullet_step), not just its start
+        self.bl = B.Bullet(B.Model.of(self.m), self.pool * L_CO, 8192, 256, 8192 + 32)
+        for l in range(L_CO):
+            self.bl.set_layer_weights(l, self.w)
         self.N = self.bl.n_sms
         self.sp, self.sd = torch.cuda.Stream(), torch.cuda.Stream()
 
@@ -92,9 +97,13 @@ def measure():
     for lens, (bs, cl), p in CORUN:
         pre, used = R.batch(lens, [0] * len(lens))
         dec, _ = R.batch([1] * bs, [cl] * bs, used)
+        tp0, _ = R.time(pre, None, p)                 # alone on the same SMs: the balance k
+        _, td0 = R.time(None, dec, p)
+        k = int(min(L_CO, max(1, round(tp0 / max(td0, 1e-6)))))
+        dec.layer_end = k
         tp, td = R.time(pre, dec, p)
-        pts.append({"kind": "pre", "q": lens, "c": [0] * len(lens), "m": p, "co": R.N - p, "ms": tp})
-        pts.append({"kind": "dec", "q": [1] * bs, "c": [cl] * bs, "m": R.N - p, "co": p, "ms": td})
+        pts.append({"kind": "pre", "q": lens, "c": [0] * len(lens), "m": p, "co": R.N - p, "ms": tp, "k": k})
+        pts.append({"kind": "dec", "q": [1] * bs, "c": [cl] * bs, "m": R.N - p, "co": p, "ms": td / k, "k": k})
     return R.N, pts
 
 

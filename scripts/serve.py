@@ -45,6 +45,7 @@ class GpuStep:
         self.sp, self.sd = torch.cuda.Stream(), torch.cuda.Stream()
         self.pre_id = self.dec_id = -1
         self.pre = self.dec = None
+        self.rec = []   # per cycle (for --log-cycles): split, shapes, device ms
 
     @staticmethod
     def _table(reqs):
@@ -83,7 +84,12 @@ class GpuStep:
         e1.record(self.sp)
         cur.wait_stream(self.sp)
         e1.synchronize()
-        return e0.elapsed_time(e1)
+        ms = e0.elapsed_time(e1)
+        self.rec.append({"p": p, "mode": mode, "q": list(pw.q_lens) if pw is not None else [],
+                         "pl": (pw.layer_end - pw.layer_begin) if pw is not None else 0,
+                         "k": (dw.layer_end - dw.layer_begin) if dw is not None else 0,
+                         "ctx": list(dw.ctx_lens) if dw is not None else [], "ms": ms})
+        return ms
 
 
 def main():
@@ -97,6 +103,8 @@ def main():
     ap.add_argument("--max-decodes", type=int, default=256)
     ap.add_argument("--max-prefill", type=int, default=8192)
     ap.add_argument("--blocks", type=int, default=24000)
+    ap.add_argument("--no-feedback", action="store_true", help="bullet policies: no online estimator feedback")
+    ap.add_argument("--log-cycles", default=None, help="write every cycle (split, shapes, ms) as JSON lines here")
     ap.add_argument("--k-ts", type=int, default=0, help="decode layer-steps per cycle when time-sliced (0: model)")
     ap.add_argument("--seed", type=int, default=0)
     a = ap.parse_args()
@@ -109,14 +117,19 @@ def main():
     # typical batch against one decode layer-step of a typical decode batch
     k_ts = a.k_ts or max(1, round(g.bl.predict_us([400] * 8, [0] * 8, g.N) /
                                   g.bl.predict_us([1] * 128, [600] * 128, g.N)))
+    base = g.bl.colocation()
     for pol in a.policies:
         trace = SV.poisson_trace(a.rate, a.duration, seed=a.seed)
+        g.bl.set_colocation(*base)   # every policy starts from the fitted factors
+        fb = g.bl if (pol.startswith("bullet") and not a.no_feedback) else None
         loop = SV.ServingLoop(a.layers, g.N, g, g.bl.choose_split, pol, SV.BlockAllocator(a.blocks),
                               max_prefill_tokens=a.max_prefill, max_decodes=a.max_decodes, k_full=k_ts,
-                              chunk_tokens=a.chunk_tokens)
+                              chunk_tokens=a.chunk_tokens, feedback_model=fb)
         t0 = time.perf_counter()
         res = loop.run(trace)
         res["policy"] = pol
+        res["estimator_feedback"] = None if fb is None else {"corun_ratio": loop.fb_ratio,
+                                                             "p_c_p_b": list(g.bl.colocation())}
         res.update(rate_req_s=a.rate, arrivals_s=a.duration, layers=a.layers, k_timesliced=k_ts,
                    wall_s=time.perf_counter() - t0, model="llama3.1-8b", data="synthetic Poisson trace")
         ps = [c[1] for c in loop.log if 0 < c[1] < g.N]
@@ -124,6 +137,11 @@ def main():
         ks = [c[2] for c in loop.log if c[2] > 0]
         res["mean_decode_steps_per_cycle"] = float(np.mean(ks)) if ks else None
         print(json.dumps(res), flush=True)
+        if a.log_cycles:
+            with open(f"{a.log_cycles}.{pol}.jsonl", "w") as f:
+                for r in g.rec:
+                    f.write(json.dumps(r) + "\n")
+        g.rec = []
 
 
 if __name__ == "__main__":

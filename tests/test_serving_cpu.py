@@ -132,3 +132,37 @@ def test_trace_is_seeded_and_shaped():
     assert [(r.arrival_ms, r.prompt, r.out_len) for r in a] == [(r.arrival_ms, r.prompt, r.out_len) for r in b]
     assert 60 < len(a) < 140                                                 # ~100 arrivals
     assert all(32 <= r.prompt <= 2048 and 8 <= r.out_len <= 512 for r in a)
+
+
+def test_online_feedback_learns_observed_contention():
+    """P:L195 online estimator feedback: when every co-run cycle takes 1.3x
+    what the model predicts (a fixed, uncorrected contention), the loop's EMA
+    converges to that ratio and the model's co-location factors are rescaled
+    by 1/1.3 — later co-run predictions match the observations; non-co-run
+    predictions are untouched.  The factors are restored afterwards."""
+    pj = os.path.join(ROOT, "profiles", "perf_params_b200.json")
+    truth = PerfModel(Model.of(synth.MODELS["llama3.1-8b"]), N, open(pj).read())   # uncorrected
+    est = PerfModel(Model.of(synth.MODELS["llama3.1-8b"]), N, open(pj).read())     # corrected online
+    base = est.colocation()
+
+    class Slow(Recorder):
+        def __call__(self, pw, dw, p, mode):
+            ms = super().__call__(pw, dw, p, mode)
+            return ms * 1.3 if (pw is not None and dw is not None and mode == "corun" and 0 < p < N) else ms
+
+    trace = SV.poisson_trace(60.0, 1.0, seed=5)
+    loop = SV.ServingLoop(L, N, Slow(truth), est.choose_split, "bullet", SV.BlockAllocator(8000),
+                          max_decodes=128, k_full=4, feedback_model=est)
+    res = loop.run(trace)
+    assert res["finished"] == len(trace)
+    n_co = sum(1 for c in loop.log if 0 < c[1] < N and c[2] > 0 and c[3] > 0)
+    assert n_co > 20
+    assert abs(loop.fb_ratio - 1.3) < 0.02, loop.fb_ratio
+    pc, pb = est.colocation()
+    assert abs(pc - base[0] / loop.fb_ratio) < 1e-12 and abs(pb - base[1] / loop.fb_ratio) < 1e-12
+    q, c = [512, 300], [0, 0]
+    assert est.predict_us(q, c, 100, 48) == pytest.approx(truth.predict_us(q, c, 100, 48) * loop.fb_ratio, rel=1e-9)
+    assert est.predict_us(q, c, 148, 0) == truth.predict_us(q, c, 148, 0)   # alone: no co-location factor
+    est.set_colocation(*base)
+    with pytest.raises(Exception):
+        est.set_colocation(0.0, 1.0)
