@@ -266,10 +266,21 @@ class Step:
             ratios.append(t / c); tc.append(c); tt.append(t)
         return float(np.median(ratios)), float(np.mean(tc)), float(np.mean(tt))
 
+    def _tune_points(self, cands, refine):
+        """Coarse candidates, then the neighbours (+-refine SMs) of the best
+        coarse estimate — the speedup surface is smooth on this scale."""
+        for p in cands:
+            yield p
+        if refine and self._tune_res:
+            best = max(self._tune_res, key=lambda r: r["speedup_vs_timesliced_est"])["p"]
+            for p in (best - refine, best + refine):
+                if 2 <= p <= self.N - 2 and p not in cands:
+                    yield p
+
     def tokens(self, k):
         return (self.n_p * 1 + self.n_d * k) / self.m.n_layers
 
-    def tune(self, cands, t_pre_full, t_dec_full, reps=3):
+    def tune(self, cands, t_pre_full, t_dec_full, reps=3, refine=4):
         """For each candidate prefill SM count p: time the isolated prefill
         layer on p SMs and decode layer-step on N-p SMs; around the balance
         point k0 = round(T_p/T_d) (decode steps per prefill layer) try
@@ -278,7 +289,9 @@ class Step:
         the same batch time-sliced on the full GPU (BASELINE's target)."""
         B = self.B
         res = []
-        for p in cands:
+        cands = list(cands)
+        self._tune_res = res
+        for p in self._tune_points(cands, refine):
             self.dec.layer_end = 1
             self.time_steps(1, p, B.CORUN, dec=False)
             tp = self.time_steps(reps, p, B.CORUN, dec=False)
