@@ -1004,8 +1004,9 @@ static int step_impl(bullet_handle* h, const bullet_batch* pre, const bullet_bat
   // several (+0.7 % on a prefill layer) — so only up to 1024 rows
   const bool fn_ok = !(flags & BULLET_UNFUSED_NORM) && h->cfg.dtype == BULLET_DTYPE_BF16 && !h->peer_mode &&
                      h->cfg.d_model <= 8192;
-  cp.fuse_norm = fn_ok && pre && pre->n_tokens <= 1024;
-  cd.fuse_norm = fn_ok && dec && dec->n_tokens <= 1024;
+  static const int fn_rows = getenv("BULLET_FUSED_NORM_MAX_ROWS") ? atoi(getenv("BULLET_FUSED_NORM_MAX_ROWS")) : 1024;
+  cp.fuse_norm = fn_ok && pre && pre->n_tokens <= fn_rows;
+  cd.fuse_norm = fn_ok && dec && dec->n_tokens <= fn_rows;
   if (has_pre && (rc = run_phase(cp, pre))) return rc;
   if (run_dec) {
     if (mode == BULLET_TIMESLICED && has_pre) {
