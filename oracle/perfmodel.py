@@ -196,7 +196,7 @@ def choose_split(P, model, state, slo, gran=2):
     def balanced():
         return min(cands, key=lambda v: (max(ev[v][0], ev[v][1]), v))   # R-16, tie -> larger u
 
-    def max_throughput():
+    def max_throughput_t():
         # R-21 (objective 1, "meet stringent SLO requirements while
         # maximizing throughput"): among the SLO-feasible splits, the most
         # predicted tokens per ms; ties to the larger prefill share
@@ -213,10 +213,41 @@ def choose_split(P, model, state, slo, gran=2):
             tput = (n_pre + len(state["decode_tokens"]) * k) / cyc if cyc > 0 else 0.0
             if tput > best_t:
                 best, best_t = v, tput
-        return best
+        return best, best_t
 
-    if ok_t and ok_d and slo.get("objective", 0) == 1 and max_throughput() is not None:
-        v = max_throughput()                           # R-21
+    def timesliced():
+        # R-22: one prefill layer then k_ts decode layer-steps, both alone on
+        # all N SMs, k_ts = round(t_p / t_d); Alg. 1 l.3-10 on the cycle time;
+        # returns (k_ts, tokens per ms), k_ts = 0 when an SLO is missed
+        pre = _phase_shape(model, list(state["prefill_lens"]), [0] * len(state["prefill_lens"]))
+        dec = _phase_shape(model, [1] * len(state["decode_tokens"]),
+                           [int(math.floor(state["decode_mean_ctx"] + 0.5))] * len(state["decode_tokens"]))
+        tp = layer_time(pre, P, N, 0) * 1e3 if state["prefill_lens"] else 0.0
+        td = layer_time(dec, P, N, 0) * 1e3
+        if tp <= 0.0 or td <= 0.0:
+            return 0, -1.0
+        k = max(1, int(math.floor(tp / td + 0.5)))
+        cyc = tp + k * td
+        rem = cyc * (L - state["layers_done"])
+        ttft = [(rem + q) / (slo["ttft_norm_ms_per_tok"] * ln)
+                for ln, q in zip(state["prefill_lens"], state["prefill_waited_ms"])]
+        for ln, q in zip(state["pending_lens"], state["pending_waited_ms"]):
+            own = layer_time(_phase_shape(model, [ln], [0]), P, N, 0) * 1e3 * L
+            ttft.append((q + rem + own) / (slo["ttft_norm_ms_per_tok"] * ln))
+        it = cyc * L / k
+        tpot = [((dlat + it) / (o + 1)) / slo["tpot_ms"]
+                for o, dlat in zip(state["decode_tokens"], state["decode_elapsed_ms"])]
+        pct = slo.get("percentile", 0.9)
+        if p90(ttft, pct) > 1.0 or p90(tpot, pct) > 1.0:
+            return 0, -1.0
+        return k, (float(sum(state["prefill_lens"])) + len(state["decode_tokens"]) * k) / cyc
+
+    if ok_t and ok_d and slo.get("objective", 0) == 1:
+        vb, t_co = max_throughput_t()                  # R-21
+        k_ts, t_ts = timesliced()                      # R-22
+        if k_ts > 0 and t_ts > t_co:
+            return N, k_ts                             # time-sliced cycle (p = N, k > 0)
+        v = vb if vb is not None else reduce_decode()
     elif ok_t and ok_d:
         v = reduce_decode()                            # line 12-13
     elif not ok_t and not ok_d:

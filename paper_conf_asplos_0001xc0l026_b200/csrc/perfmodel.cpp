@@ -281,7 +281,7 @@ void choose_split(const PerfParams& P, const PhaseShape& model, const SchedState
   // the most predicted tokens per ms: (prefill tokens + decode tokens x k) /
   // max(t_p, k t_d), k = round(t_p / t_d) >= 1; ties to the larger prefill
   // share.  None feasible: Alg. 1's rule.
-  auto max_throughput = [&]() -> int {
+  auto max_throughput = [&](double* best_tput) -> int {
     PhaseShape dec = model;
     const int mctx = (int)std::lround(S.decode_mean_ctx);
     dec.q_lens.assign(S.decode_tokens.size(), 1); dec.ctx_lens.assign(S.decode_tokens.size(), mctx);
@@ -297,10 +297,51 @@ void choose_split(const PerfParams& P, const PhaseShape& model, const SchedState
       const double tput = cyc > 0 ? (n_pre + (double)S.decode_tokens.size() * k) / cyc : 0.0;
       if (tput > best_t) { best_t = tput; best = v; }
     }
+    if (best_tput) *best_tput = best_t;
     return best;
   };
+  // R-22 (objective 1): the time-sliced cycle — one prefill layer, then k_ts
+  // decode layer-steps, both alone on all N SMs, k_ts = round(t_p / t_d) —
+  // is a candidate too, with its own TTFT / TPOT estimate (Alg. 1 l.3-10 on
+  // the cycle time t_p + k_ts t_d); returns k_ts, or 0 when it misses an SLO
+  auto timesliced = [&](double* tput) -> int {
+    PhaseShape pre = model, dec = model;
+    pre.q_lens = S.prefill_lens; pre.ctx_lens.assign(S.prefill_lens.size(), 0);
+    const int mctx = (int)std::lround(S.decode_mean_ctx);
+    dec.q_lens.assign(S.decode_tokens.size(), 1); dec.ctx_lens.assign(S.decode_tokens.size(), mctx);
+    const double tp = S.prefill_lens.empty() ? 0.0 : layer_time(pre, P, N, 0) * 1e3;
+    const double td = layer_time(dec, P, N, 0) * 1e3;
+    if (tp <= 0.0 || td <= 0.0) return 0;
+    const int k = std::max(1, (int)std::floor(tp / td + 0.5));
+    const double cyc = tp + k * td, rem = cyc * (L - S.layers_done);
+    std::vector<double> ttft, tpot;
+    for (size_t i = 0; i < S.prefill_lens.size(); ++i)
+      ttft.push_back((rem + S.prefill_waited_ms[i]) / (slo.ttft_norm * S.prefill_lens[i]));
+    for (size_t i = 0; i < S.pending_lens.size(); ++i) {
+      PhaseShape one = model;
+      one.q_lens = {S.pending_lens[i]}; one.ctx_lens = {0};
+      const double own = layer_time(one, P, N, 0) * 1e3 * L;
+      ttft.push_back((S.pending_waited_ms[i] + rem + own) / (slo.ttft_norm * S.pending_lens[i]));
+    }
+    const double iter = cyc * L / k;
+    for (size_t i = 0; i < S.decode_tokens.size(); ++i)
+      tpot.push_back(((S.decode_elapsed_ms[i] + iter) / (S.decode_tokens[i] + 1)) / slo.tpot_ms);
+    if (p90(ttft, slo.percentile) > 1.0 || p90(tpot, slo.percentile) > 1.0) return 0;
+    double n_pre = 0.0;
+    for (int q : S.prefill_lens) n_pre += q;
+    *tput = (n_pre + (double)S.decode_tokens.size() * k) / cyc;
+    return k;
+  };
   int v;
-  if (ok_t && ok_d && slo.objective == 1 && max_throughput() >= 0) v = max_throughput();
+  if (ok_t && ok_d && slo.objective == 1) {
+    double t_co = -1.0, t_ts = -1.0;
+    const int vb = max_throughput(&t_co);
+    const int k_ts = timesliced(&t_ts);
+    if (k_ts > 0 && t_ts > t_co) {   // time-sliced cycle: prefill_sms = N with k > 0
+      *prefill_sms = N; *decode_steps = k_ts; return;
+    }
+    v = vb >= 0 ? vb : reduce_decode();
+  }
   else if (ok_t && ok_d) v = reduce_decode();
   else if (!ok_t && !ok_d) v = balanced();
   else if (ok_t && !ok_d && (int)S.pending_lens.size() <= slo.w_max) v = reduce_prefill();

@@ -282,14 +282,16 @@ class ServingLoop:
                 break
             # ---- split decision
             if self.policy == "bullet":
+                mode = "corun"
                 if prefill and members:
                     p, k = self.choose(self._alg1_state(now, prefill, layers_done, pending, members),
                                        self.slo.as_dict())
+                    if p >= self.N and k > 0:   # R-22: a time-sliced cycle (objective 1)
+                        mode = "timesliced"
                 elif prefill:
                     p, k = self.N, 0
                 else:
                     p, k = 0, self.k_full
-                mode = "corun"
             elif self.policy == "timesliced":
                 p, k, mode = self.N, (self.k_full if members else 0), "timesliced"
             else:  # prefill_first

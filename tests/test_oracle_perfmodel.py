@@ -168,6 +168,34 @@ def test_objective_throughput_picks_feasible_split_with_most_tokens_per_ms():
     assert P["M"] - u0 == min(feas) and tput(P["M"] - u0)[0] <= tput(v)[0]
 
 
+def test_objective_throughput_takes_timesliced_cycle_when_corun_costs_more():
+    """R-22: with both SLOs met and co-location made expensive (p_c = p_b =
+    0.3: every co-run kernel 3.3x slower), the time-sliced cycle (prefill layer
+    then k_ts = round(t_p / t_d) decode layer-steps, all SMs each) has more
+    predicted tokens/ms than any co-run split, so objective 1 returns it as
+    (N, k_ts); with the fitted-free default factors co-running wins."""
+    P = dict(PM.default_params(), p_c=0.3, p_b=0.3)
+    st = _state()
+    slo1 = dict(SLO, objective=1)
+    N = P["M"]
+    pre = PM._phase_shape(MODEL, [2048], [0])
+    dec = PM._phase_shape(MODEL, [1] * 64, [1024] * 64)
+    tp, td = PM.layer_time(pre, P, N, 0) * 1e3, PM.layer_time(dec, P, N, 0) * 1e3
+    k_ts = max(1, int(math.floor(tp / td + 0.5)))
+    t_ts = (2048 + 64 * k_ts) / (tp + k_ts * td)
+    ev = _eval_all(P, st, slo1)
+    t_co = 0.0
+    for v, (a, b, t_p) in ev.items():
+        if a <= 1 and b <= 1:
+            t_d = PM.layer_time(dec, P, v, N - v) * 1e3
+            k = max(1, int(math.floor(t_p / t_d + 0.5)))
+            t_co = max(t_co, (2048 + 64 * k) / max(t_p, k * t_d))
+    assert t_ts > t_co
+    assert PM.choose_split(P, MODEL, st, slo1) == (N, k_ts)
+    u, k = PM.choose_split(PM.default_params(), MODEL, st, slo1)
+    assert u < N   # default factors: a co-run split
+
+
 def test_case_both_violated_sets_balanced():
     """Alg. 1 l.15-16 (R-14): both violated -> argmin of max ratio."""
     P = PM.default_params()
