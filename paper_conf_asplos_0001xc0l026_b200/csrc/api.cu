@@ -510,7 +510,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     d.tok_base = t0;
     d.order = P.order_ok ? P.order : nullptr;
     if ((rc = next_launch(c, &d.L))) return rc;
-    LAUNCH(c, launch_attn_decode_tc(d, persist_grid(c, 1), c.m_sms <= 100 ? 2 : 1, c.st));
+    LAUNCH(c, launch_attn_decode_tc(d, persist_grid(c, 1), c.m_sms <= 100 ? 4 : 1, c.st));
     return BULLET_OK;
   }
   if (kind == 0) kind = (bf16 && a.hd == 128) ? (max_qlen(b) > 1 ? 4 : 3) : 1;
@@ -521,11 +521,11 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
       return set_err(BULLET_EUNSUPPORTED, "tensor-core decode attention: bf16, hd 128 only");
     int rc = next_launch(c, &a.L);
     if (rc) return rc;
-    // two consumer groups per SM on partitions (per-unit merge over twice the
-    // blocks: 146 -> 133 us on 68 SMs, ShareGPT), one on the full GPU (tail
-    // balance: 96 vs 101 us) — scripts/attn_dec_bench.py, DESIGN.md §5
+    // four consumer groups of 3 warps per SM on partitions (68 SMs: 78.6 vs
+    // 72.3 GB/s/SM with two groups at 1k contexts), one on the full GPU (tail
+    // balance) — scripts/attn_dec_bench.py, DESIGN.md §5
     if (!c.op && h->ph[c.phase].order_ok) a.order = h->ph[c.phase].order;
-    LAUNCH(c, launch_attn_decode_tc(a, persist_grid(c, 1), c.m_sms <= 100 ? 2 : 1, c.st));
+    LAUNCH(c, launch_attn_decode_tc(a, persist_grid(c, 1), c.m_sms <= 100 ? 4 : 1, c.st));
     return BULLET_OK;
   }
   if (kind == 2 || kind == 4) {

@@ -26,7 +26,17 @@ namespace bl {
 
 namespace {
 // DEPTH stages per warp: DEPTH - 1 blocks stay in flight while one is computed
-constexpr int KB = 16, HD = 128, NCW = 8, DEPTH = 3;
+// 12 consumer warps x 2 stages (8 x 3 before): the kernel is bound by the
+// per-warp latency of its block math, so more warps beat deeper per-warp
+// pipelines — 68 SMs, 1k / 4k contexts: 62 -> 72-79 / 71 -> 84-86 GB/s/SM;
+// 148 SMs: 6.8 TB/s (the HBM roofline); 6 x 4 and 4 x 5 were slower
+// (scripts/attn_dec_bench.py)
+#ifndef DEC_NCW
+#define DEC_NCW 12
+#define DEC_DEPTH 2
+#endif
+constexpr int KB = 16, HD = 128, NCW = DEC_NCW, DEPTH = DEC_DEPTH;
+static_assert(DEPTH <= 5, "cp.async wait ladder covers DEPTH <= 5");
 constexpr int BLK_BYTES = KB * HD * 2;       // 4 KB: one (block, kv head) of K or V
 constexpr int STAGE_BYTES = 2 * BLK_BYTES;   // K + V
 constexpr int CMB_FLOATS = HD * 8 + 16;      // O^T[128][8] + m[8] + l[8] per warp (in a free stage)
@@ -243,7 +253,8 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
     for (int j = 0; j < mine; ++j) {
       fill(it + NG, DEPTH);
       const int pend = n_issued - n_cons;   // groups in flight; the oldest is block j
-      if (pend >= 3) cp_async_wait<2>(); else if (pend == 2) cp_async_wait<1>(); else cp_async_wait<0>();
+      if (pend >= 5) cp_async_wait<4>(); else if (pend == 4) cp_async_wait<3>();
+      else if (pend == 3) cp_async_wait<2>(); else if (pend == 2) cp_async_wait<1>(); else cp_async_wait<0>();
       __syncwarp();
       const int b = wl + j * GW;
       const uint32_t kt = my_s + (n_cons % DEPTH) * STAGE_BYTES;
@@ -377,7 +388,7 @@ cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStrea
     set = true;
   }
   if (ng == 1) k_attn_decode_tc<1><<<grid, THREADS, smem, st>>>(a);
-  else if (ng == 4) k_attn_decode_tc<4><<<grid, THREADS, smem, st>>>(a);
+  else if (ng == 4 && NCW % 4 == 0) k_attn_decode_tc<4><<<grid, THREADS, smem, st>>>(a);
   else k_attn_decode_tc<2><<<grid, THREADS, smem, st>>>(a);
   return cudaGetLastError();
 }
