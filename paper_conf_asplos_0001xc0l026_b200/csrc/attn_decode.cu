@@ -376,7 +376,7 @@ int attn_decode_max_blocks() { return MAXNB; }
 cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStream_t st) {
   const size_t smem = attn_decode_smem_bytes();
   static const int forced = getenv("BULLET_DEC_GROUPS") ? atoi(getenv("BULLET_DEC_GROUPS")) : 0;
-  if (forced == 1 || forced == 2 || forced == 4) ng = forced;
+  if (forced >= 1 && forced <= 4) ng = forced;
   static bool set = false;
   if (!set) {
     cudaError_t e = cudaFuncSetAttribute(k_attn_decode_tc<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -384,11 +384,14 @@ cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStrea
       e = cudaFuncSetAttribute(k_attn_decode_tc<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(k_attn_decode_tc<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(k_attn_decode_tc<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     set = true;
   }
   if (ng == 1) k_attn_decode_tc<1><<<grid, THREADS, smem, st>>>(a);
   else if (ng == 4 && NCW % 4 == 0) k_attn_decode_tc<4><<<grid, THREADS, smem, st>>>(a);
+  else if (ng == 3 && NCW % 3 == 0) k_attn_decode_tc<3><<<grid, THREADS, smem, st>>>(a);
   else k_attn_decode_tc<2><<<grid, THREADS, smem, st>>>(a);
   return cudaGetLastError();
 }
@@ -398,6 +401,7 @@ cudaError_t preload_attn_decode() {
   cudaError_t e = cudaFuncGetAttributes(&f, k_attn_decode_tc<1>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_attn_decode_tc<2>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_attn_decode_tc<4>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_attn_decode_tc<3>);
   return e;
 }
 
