@@ -443,10 +443,15 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
             const float2 t = ffma2(make_float2(v[2 * j], v[2 * j + 1]), sl2, -m_new);
             const float2 pp = make_float2(ex2(t.x), ex2(t.y));
             acc = fadd2(acc, pp);
-            const uint32_t h = pack_bf2(pp.x, pp.y);
-            const float2 l = fsub2(pp, make_float2(__uint_as_float(h << 16), __uint_as_float(h & 0xFFFF0000u)));
-            hi[j] = h;
-            lo[j] = pack_bf2(l.x, l.y);
+            // P = hi + lo with both parts truncated to bf16 by byte permutes
+            // (ALU) instead of two cvt.rn.bf16x2 (conversion pipe, shared with
+            // nothing the MMA needs but slow): x - trunc(x) is exact, so the
+            // only error is lo's truncation, < 2^-15 |P| (R-4b asks for better
+            // than bf16's 2^-9)
+            const uint32_t ux = __float_as_uint(pp.x), uy = __float_as_uint(pp.y);
+            const float2 l = fsub2(pp, make_float2(__uint_as_float(ux & 0xFFFF0000u), __uint_as_float(uy & 0xFFFF0000u)));
+            hi[j] = __byte_perm(ux, uy, 0x7632);
+            lo[j] = __byte_perm(__float_as_uint(l.x), __float_as_uint(l.y), 0x7632);
           }
           tmem_st16(t_sb + half * 32, hi);
           tmem_st16(t_sb + half * 32 + 16, lo);
