@@ -32,6 +32,7 @@
 #ifndef BULLET_H
 #define BULLET_H
 
+#include <stddef.h>
 #include <stdint.h>
 
 #ifdef __cplusplus

@@ -4,6 +4,8 @@ decision (C++) equal the oracle's plain reading (oracle/perfmodel.py)."""
 import json
 
 import numpy as np
+import os
+
 import pytest
 
 import paper_conf_asplos_0001xc0l026_b200 as B
@@ -133,3 +135,19 @@ def test_fitted_perf_params_load_and_match_oracle():
             ref = PM.layer_time(dict(shape, q_lens=q, ctx_lens=c), P, m, co) * 1e6
             assert got == pytest.approx(ref, rel=1e-12)
     assert P["fit"]["mre_heldout"] < 0.5
+
+
+def test_header_is_plain_c99(tmp_path):
+    """include/bullet.h is a C ABI: it must compile as strict C99 on its own
+    (no C++ or torch types cross the boundary)."""
+    import shutil
+    import subprocess
+    gcc = shutil.which("gcc")
+    if gcc is None:
+        pytest.skip("no gcc")
+    src = tmp_path / "t.c"
+    src.write_text('#include "bullet.h"\nint main(void) { bullet_handle *h = 0; (void)h; return 0; }\n')
+    inc = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "include")
+    r = subprocess.run([gcc, "-std=c99", "-Wall", "-Wextra", "-pedantic", "-Werror", "-fsyntax-only", "-I", inc, str(src)],
+                       capture_output=True, text=True)
+    assert r.returncode == 0, r.stderr
