@@ -65,6 +65,9 @@ enum {
                                 QKV GEMM epilogue (bf16, head_dim 128); A/B tests only */
   BULLET_UNFUSED_NORM = 32,  /* run S6 / the next layer's S1 (RMSNorm) as their own kernels
                                 instead of the tail of the O-proj / down GEMM; A/B tests only */
+  BULLET_CHECK_KV = 128,     /* validation (host, before enqueue): EKV if a KV block used by a
+                                prefill request is also used by a decode request (the
+                                phases run concurrently: shared blocks would race) */
   BULLET_DEVICE_SPLIT = 64   /* CORUN: kernels read the phases' SM sets from device memory
                                 (bullet_set_split) instead of kernel arguments, so one CUDA
                                 graph captured from the step follows any later split

@@ -17,7 +17,7 @@ c_int, c_double, c_float, c_void_p = ctypes.c_int, ctypes.c_double, ctypes.c_flo
 P_i32 = ctypes.POINTER(ctypes.c_int32)
 P_f64 = ctypes.POINTER(ctypes.c_double)
 
-CORUN, TIMESLICED, UNGATED, SMID_LOG, PROFILE, UNFUSED, UNFUSED_NORM, DEVICE_SPLIT = 0, 1, 2, 4, 8, 16, 32, 64
+CORUN, TIMESLICED, UNGATED, SMID_LOG, PROFILE, UNFUSED, UNFUSED_NORM, DEVICE_SPLIT, CHECK_KV = 0, 1, 2, 4, 8, 16, 32, 64, 128
 KERNEL_KINDS = ["plan", "rmsnorm1", "qkv", "rope_kv", "attn", "o_proj", "rmsnorm2", "gate_up",
                 "down", "allreduce"]
 DTYPE_FP32, DTYPE_BF16 = 0, 1

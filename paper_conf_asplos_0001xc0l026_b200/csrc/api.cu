@@ -984,6 +984,27 @@ static int step_impl(bullet_handle* h, const bullet_batch* pre, const bullet_bat
   if (mode == BULLET_CORUN && run_dec && dhi <= dlo)
     return set_err(BULLET_ESMRANGE, "decode batch given with an empty decode SM range");
   if (h->log_cap == 0 && (flags & BULLET_SMID_LOG)) return set_err(BULLET_EINVAL, "SMID_LOG without a log buffer");
+  if ((flags & BULLET_CHECK_KV) && has_pre && has_dec) {   // disjoint block sets
+    if (!pre->h_block_table || !dec->h_block_table)
+      return set_err(BULLET_EINVAL, "BULLET_CHECK_KV needs host block tables");
+    std::vector<char> used(h->n_blocks, 0);
+    auto mark = [&](const bullet_batch* b, bool check) -> int {
+      for (int r = 0; r < b->n_reqs; ++r) {
+        const int q = b->h_cu_seqlens[r + 1] - b->h_cu_seqlens[r];
+        if (q == 0) continue;
+        const int nb = (b->h_ctx_lens[r] + q + h->block_size - 1) / h->block_size;
+        for (int i = 0; i < nb; ++i) {
+          const int blk = b->h_block_table[(size_t)r * b->max_blocks_per_req + i];
+          if (check && used[blk]) return blk;
+          if (!check) used[blk] = 1;
+        }
+      }
+      return -1;
+    };
+    mark(pre, false);
+    const int clash = mark(dec, true);
+    if (clash >= 0) return set_err(BULLET_EKV, "KV block %d is used by both a prefill and a decode request", clash);
+  }
   const bool log = (flags & BULLET_SMID_LOG) != 0;
   cudaStream_t sp = (cudaStream_t)s_prefill, sd = (cudaStream_t)s_decode;
   const bool prof = (flags & BULLET_PROFILE) != 0;

@@ -198,6 +198,16 @@ def test_decode_pause_and_errors(small_bf16):
     with pytest.raises(B.BulletError) as e:
         S.bl.step(None, dec_bad, 0, B.CORUN)
     assert e.value.code == -5
+    # BULLET_CHECK_KV: disjoint prefill / decode block sets pass,
+    # a decode request pointing at a prefill request's block is rejected
+    S.bl.step(pre, dec, 64, B.CORUN | B.CHECK_KV)
+    torch.cuda.synchronize()
+    shared = S.lay.block_table[S.n_pre:].copy()
+    shared[0, 0] = S.lay.block_table[0, 0]
+    dec_sh = B.Batch([1] * len(S.decode_ctx), S.decode_ctx, shared, dec.hidden)
+    with pytest.raises(B.BulletError) as e:
+        S.bl.step(pre, dec_sh, 64, B.CORUN | B.CHECK_KV)
+    assert e.value.code == -5
 
 
 @pytest.mark.parametrize("bias", [0, 1])
