@@ -19,6 +19,8 @@ policies see the same arrival process.
 
 Policies:
   bullet      co-run, (p, k) from Alg. 1 (bullet_choose_split)
+  static      co-run at one fixed (prefill SMs, k) every cycle — the bench's
+              tuned split; a diagnostic of the decision layer, not a policy
   bullet_tput the same with objective 1: when both SLOs hold, the split with
               the most predicted tokens/s among the SLO-feasible ones (R-21)
   timesliced  same cycle structure, both phases on all SMs one after the
@@ -124,8 +126,9 @@ class ServingLoop:
     def __init__(self, n_layers: int, n_sms: int, step, choose, policy: str, allocator: BlockAllocator,
                  slo: Slo = Slo(), prefill_layers_per_cycle: int = 1, max_prefill_tokens: int = 8192,
                  max_decodes: int = 256, k_full: int = 4, chunk_tokens: int = 2048, feedback_model=None,
-                 feedback_alpha: float = 0.2):
-        assert policy in ("bullet", "bullet_tput", "timesliced", "prefill_first", "chunked")
+                 feedback_alpha: float = 0.2, static_split=(88, 6)):
+        assert policy in ("bullet", "bullet_tput", "static", "timesliced", "prefill_first", "chunked")
+        self.static_split = static_split   # policy "static": fixed (prefill SMs, decode layer-steps) co-run
         if policy == "bullet_tput":   # Alg. 1 with the throughput objective among feasible splits (R-21)
             policy = "bullet"
             slo = Slo(**{**slo.__dict__, "objective": 1})
@@ -292,6 +295,9 @@ class ServingLoop:
                     p, k = self.N, 0
                 else:
                     p, k = 0, self.k_full
+            elif self.policy == "static":      # the bench-tuned split every cycle (diagnostic)
+                p, k = self.static_split if (prefill and members) else ((self.N, 0) if prefill else (0, self.k_full))
+                mode = "corun"
             elif self.policy == "timesliced":
                 p, k, mode = self.N, (self.k_full if members else 0), "timesliced"
             else:  # prefill_first

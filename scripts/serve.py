@@ -103,6 +103,7 @@ def main():
     ap.add_argument("--max-decodes", type=int, default=256)
     ap.add_argument("--max-prefill", type=int, default=8192)
     ap.add_argument("--blocks", type=int, default=24000)
+    ap.add_argument("--static", type=int, nargs=2, default=[88, 6], help="policy static: prefill SMs, decode steps")
     ap.add_argument("--no-feedback", action="store_true", help="bullet policies: no online estimator feedback")
     ap.add_argument("--log-cycles", default=None, help="write every cycle (split, shapes, ms) as JSON lines here")
     ap.add_argument("--k-ts", type=int, default=0, help="decode layer-steps per cycle when time-sliced (0: model)")
@@ -124,7 +125,7 @@ def main():
         fb = g.bl if (pol.startswith("bullet") and not a.no_feedback) else None
         loop = SV.ServingLoop(a.layers, g.N, g, g.bl.choose_split, pol, SV.BlockAllocator(a.blocks),
                               max_prefill_tokens=a.max_prefill, max_decodes=a.max_decodes, k_full=k_ts,
-                              chunk_tokens=a.chunk_tokens, feedback_model=fb)
+                              chunk_tokens=a.chunk_tokens, feedback_model=fb, static_split=tuple(a.static))
         t0 = time.perf_counter()
         res = loop.run(trace)
         res["policy"] = pol
