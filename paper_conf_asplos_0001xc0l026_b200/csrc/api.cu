@@ -392,6 +392,10 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
     fprintf(stderr, "gemm M=%d N=%d K=%d m_sms=%d -> mh=%d bn=%d n_full=%d ts=%d\n", M, N, K, c.m_sms, mh, bn,
             n_full, ts);
   a.bn = bn; a.mh = mh; a.splits = ts; a.n_full = n_full;
+  {   // second copy issuer for the weight tiles (BULLET_GEMM_SPLIT_B=0/1 overrides; default: on)
+    static const int sb = getenv("BULLET_GEMM_SPLIT_B") ? atoi(getenv("BULLET_GEMM_SPLIT_B")) : 1;
+    a.split_b = sb ? 1 : 0;
+  }
   {  // rasterisation band: activations of a band <= 32 MB (L2-resident)
     const int m_tiles = (M + 128 * mh - 1) / (128 * mh);
     const double a_tile = 128.0 * mh * K * 2;
@@ -1290,7 +1294,7 @@ int bullet_op_stream(bullet_handle* h, const void* src, size_t bytes, int mode, 
   Ctx c;
   int rc = op_ctx(h, lo, hi, stream, &c);
   if (rc) return rc;
-  if (!src || bytes == 0 || (mode & 0xff) > 5 || mode < 0) return set_err(BULLET_EINVAL, "stream args");
+  if (!src || bytes == 0 || (mode & 0xff) > 8 || mode < 0) return set_err(BULLET_EINVAL, "stream args");
   StreamArgs a;
   memset(&a, 0, sizeof a);
   a.src = (const uint8_t*)src; a.bytes = bytes; a.mode = mode & 0xff; a.param = (mode >> 8) & 0xff;

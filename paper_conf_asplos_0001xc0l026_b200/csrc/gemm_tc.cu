@@ -442,9 +442,9 @@ __global__ void __launch_bounds__(NT, 1)
   const int k_blocks = a.K / BK;
 
   if (threadIdx.x == 0) {
-    for (int s = 0; s < n_stages; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
+    for (int s = 0; s < n_stages; ++s) { mbar_init(full + s, a.split_b ? 2 : 1); mbar_init(empty + s, 1); }
     for (int i = 0; i < 2; ++i) { mbar_init(accf + i, 1); mbar_init(acce + i, 4); }
-    for (int i = 0; i < 4; ++i) { mbar_init(tqf + i, 1); mbar_init(tqe + i, 5); }
+    for (int i = 0; i < 4; ++i) { mbar_init(tqf + i, 1); mbar_init(tqe + i, a.split_b ? 6 : 5); }
     mbar_fence_init();
   }
   if (warp == 0 && lane == 0) { tma_prefetch_desc(&mapA); tma_prefetch_desc(&mapB); }
@@ -486,12 +486,58 @@ __global__ void __launch_bounds__(NT, 1)
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(empty + s, ph ^ 1);
           uint8_t* sa = smem + s * st_bytes;
-          mbar_arrive_expect_tx(full + s, st_bytes);
+          mbar_arrive_expect_tx(full + s, a.split_b ? a_bytes : st_bytes);
 #pragma unroll
           for (int hh = 0; hh < mh; ++hh)   // rows past M are zero-filled by TMA
             tma_load_2d_hint(sa + hh * A_BYTES, &mapA, full + s, kb * BK, (m_blk * mh + hh) * BM, pol_a);
           uint8_t* sb = sa + a_bytes;
-          if (a.b_packed) {   // pre-swizzled tiles: contiguous bulk copies
+          if (a.split_b) {
+            // B comes from warp 3's issuer
+          } else if (a.b_packed) {   // pre-swizzled tiles: contiguous bulk copies
+            const uint8_t* kbase = a.b_packed + (size_t)kb * (a.b_rows / 64) * 8192;
+            if (r1 == r0 + bn / 2) {
+              bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s, pol_b);
+            } else {
+              bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes / 2, full + s, pol_b);
+              bulk_g2s(sb + b_bytes / 2, kbase + (size_t)(r1 / 64) * 8192, b_bytes / 2, full + s, pol_b);
+            }
+          } else {
+            tma_load_2d_hint(sb, &mapB, full + s, kb * BK, r0, pol_b);
+            tma_load_2d_hint(sb + b_bytes / 2, &mapB, full + s, kb * BK, r1, pol_b);
+          }
+          if (++s == n_stages) { s = 0; ph ^= 1; }
+        }
+        ++it;
+      }
+    }
+  } else if (warp == 3) {
+    if (lane == 0 && a.split_b) {  // ---------------- second issuer: B (weight) tiles
+      // one thread's issue loop (wait for a free stage, arm, issue) caps the
+      // copy stream it can keep in flight; a second issuing thread for the
+      // weight operand lifts the per-SM ceiling (KI2: 99 -> 123 GB/s/SM,
+      // profiles/r01c_ki2_issuers.jsonl).  Same unit / k-block / stage
+      // sequence as warp 0, its own arrival on each full barrier (count 2).
+      const uint64_t pol_b = a.b_evict_first ? policy_evict_first() : policy_evict_normal();
+      int it = 0, s = 0;
+      uint32_t ph = 0;
+      for (;;) {
+        const int slot = it & 3;
+        mbar_wait(tqf + slot, (it >> 2) & 1);
+        const int u = tile_q[slot];
+        mbar_arrive(tqe + slot);
+        if (u < 0) break;
+        const UnitInfo ui = unit_info(a, u);
+        int m_blk, n_blk;
+        tile_coords(ui.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
+        const int kb0 = ui.sp * k_blocks / ui.ns, kb1 = (ui.sp + 1) * k_blocks / ui.ns;
+        int r0, r1;
+        if (a.epi == EPI_SILU) { r0 = n_blk * (bn / 2); r1 = a.silu_half + r0; }
+        else { r0 = n_blk * bn; r1 = r0 + bn / 2; }
+        for (int kb = kb0; kb < kb1; ++kb) {
+          mbar_wait(empty + s, ph ^ 1);
+          uint8_t* sb = smem + s * st_bytes + a_bytes;
+          mbar_arrive_expect_tx(full + s, b_bytes);
+          if (a.b_packed) {
             const uint8_t* kbase = a.b_packed + (size_t)kb * (a.b_rows / 64) * 8192;
             if (r1 == r0 + bn / 2) {
               bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s, pol_b);

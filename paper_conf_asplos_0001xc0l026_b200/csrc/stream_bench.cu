@@ -90,35 +90,53 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
       __syncwarp();
       if (a.mode == 3) acc ^= reinterpret_cast<const uint32_t*>(slot)[lane];
     }
-  } else if (a.mode == 1 || a.mode == 5) {
+  } else if (a.mode == 1 || a.mode == 5 || a.mode == 7 || a.mode == 8) {
     // mode 5 (warp 0 only here): bulk copies concurrently with LDG warps 1..15
+    // mode 7: two issuing threads (tid 0, tid 32) in ONE CTA, 3 stages each
     const size_t units = a.bytes / BULK;
+    const int nb = a.mode == 7 ? NB / 2 : (a.mode == 1 && a.param > 0 && a.param < NB) ? a.param : NB;
+    const int iss = (tid == 0) ? 0 : (a.mode == 7 && tid == 32) ? 1 : -1;
     if (tid == 0) {
       for (int i = 0; i < NB; ++i) mbar_init(bars + i, 1);
       mbar_fence_init();
     }
-    if (a.mode == 1) __syncthreads(); else __syncwarp();
-    if (tid == 0) {
+    if (a.mode != 5) __syncthreads(); else __syncwarp();
+    uint64_t* bars_i = bars + (iss > 0 ? iss * nb : 0);
+    uint8_t* sm_i = sm + (size_t)(iss > 0 ? iss * nb : 0) * BULK;
+#define bars bars_i
+#define sm sm_i
+    if (iss >= 0) {
       uint32_t issued = 0, done = 0;
+      int batch_u = 0, batch_left = 0;
       for (;;) {
-        if (issued - done == NB) {   // retire the oldest
-          mbar_wait(bars + (done % NB), (done / NB) & 1);
-          acc ^= *reinterpret_cast<const uint32_t*>(sm + (done % NB) * BULK);
+        if (issued - done == (uint32_t)nb) {   // retire the oldest
+          mbar_wait(bars + (done % nb), (done / nb) & 1);
+          acc ^= *reinterpret_cast<const uint32_t*>(sm + (done % nb) * BULK);
           ++done;
         }
-        const int u = atomicAdd(a.L.ctr, 1);
+        // claim granularity: param2 = units per atomic (mode 1 | (depth << 8) | (batch << 16) would
+        // collide with the wrap field, so mode 8 = mode 1 with 8-unit claims)
+        int u;
+        if (a.mode == 8) {
+          if (batch_left == 0) { batch_u = atomicAdd(a.L.ctr, 8); batch_left = 8; }
+          u = batch_u++; --batch_left;
+        } else {
+          u = atomicAdd(a.L.ctr, 1);
+        }
         if (u >= (int)units) break;
-        const int s = issued % NB;
+        const int s = issued % nb;
         mbar_arrive_expect_tx(bars + s, BULK);
         bulk_g2s(sm + s * BULK, a.src + (((size_t)u * BULK) & a.wrap), BULK, bars + s);
         ++issued;
       }
       while (done < issued) {
-        mbar_wait(bars + (done % NB), (done / NB) & 1);
-        acc ^= *reinterpret_cast<const uint32_t*>(sm + (done % NB) * BULK);
+        mbar_wait(bars + (done % nb), (done / nb) & 1);
+        acc ^= *reinterpret_cast<const uint32_t*>(sm + (done % nb) * BULK);
         ++done;
       }
     }
+#undef bars
+#undef sm
   } else {
     const size_t units = a.bytes / 65536;
     int n = 0;
@@ -150,10 +168,14 @@ __global__ void __launch_bounds__(512, 1) k_stream(StreamArgs a) {
 }
 
 cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st) {
-  const int smem = a.mode == 1 ? NB * BULK : (a.mode == 2 ? 3 * 65536 : (a.mode == 3 ? 16 * 8192 : (a.mode == 5 ? NB * BULK : 0)));
-  cudaError_t e = cudaFuncSetAttribute(k_stream, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  // mode 1 with param = ring depth d < NB: d x 32 KB per CTA and two CTAs per
+  // SM (two bulk-copy issuers per SM: is the ~85 GB/s/SM ceiling per issuer?)
+  const bool two = a.mode == 1 && a.param > 0 && a.param < NB;
+  const int smem = (a.mode == 1 || a.mode == 7 || a.mode == 8) ? (two ? a.param : NB) * BULK
+                               : (a.mode == 2 ? 3 * 65536 : (a.mode == 3 ? 16 * 8192 : (a.mode == 5 ? NB * BULK : 0)));
+  cudaError_t e = cudaFuncSetAttribute(k_stream, cudaFuncAttributeMaxDynamicSharedMemorySize, NB * BULK);
   if (e != cudaSuccess) return e;
-  k_stream<<<grid, 512, smem, st>>>(a);
+  k_stream<<<two ? 2 * grid : grid, two ? 256 : 512, smem, st>>>(a);
   return cudaGetLastError();
 }
 
