@@ -78,44 +78,104 @@ def allreduce_max(x, ws):
 
 # ---------------------------------------------------------------- clocks
 class Clocks:
-    """nvidia-smi sampled every 200 ms during the timed region."""
-    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
-         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap")
+    """SM clock and throttle reasons sampled DURING the timed region: an NVML
+    thread polls every 5 ms (the timed region is ~0.1 s, too short for
+    `nvidia-smi -lms`, whose first row arrives after it ended), plus one
+    sample at entry and one at exit; nvidia-smi is the fallback when NVML is
+    unavailable."""
+    NAMES = ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap")
 
     def __init__(self, dev):
         self.dev = dev
+        self.rows = []            # (sm_mhz, max_mhz, set of reason names)
+        self.nvml = None
         self.p = None
 
-    def __enter__(self):
+    def _nvml_handle(self):
+        import pynvml as N
+        N.nvmlInit()
+        # match the CUDA device by UUID (nvmlDeviceGetHandleByPciBusId
+        # segfaults in this image's pynvml); else CUDA_VISIBLE_DEVICES / index
         try:
-            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.dev), f"--query-gpu={self.Q}",
-                                       "--format=csv,noheader,nounits", "-lms", "200"],
-                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-        except OSError:
-            self.p = None
+            uid = str(torch.cuda.get_device_properties(self.dev).uuid).lower()
+            for i in range(N.nvmlDeviceGetCount()):
+                h = N.nvmlDeviceGetHandleByIndex(i)
+                u = N.nvmlDeviceGetUUID(h)
+                u = (u.decode() if isinstance(u, bytes) else u).lower()
+                if u.endswith(uid) or uid.endswith(u.replace("gpu-", "")):
+                    return N, h
+        except Exception:
+            pass
+        vis = os.environ.get("CUDA_VISIBLE_DEVICES", "")
+        idx = int(vis.split(",")[self.dev]) if vis and vis.split(",")[0].isdigit() else self.dev
+        return N, N.nvmlDeviceGetHandleByIndex(idx)
+
+    def _sample(self):
+        N, h = self.nvml
+        bits = N.nvmlDeviceGetCurrentClocksEventReasons(h)
+        masks = (N.nvmlClocksEventReasonHwSlowdown, N.nvmlClocksEventReasonHwThermalSlowdown,
+                 N.nvmlClocksEventReasonSwThermalSlowdown, N.nvmlClocksEventReasonSwPowerCap)
+        self.rows.append((float(N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_SM)),
+                          float(N.nvmlDeviceGetMaxClockInfo(h, N.NVML_CLOCK_SM)),
+                          {n for n, m in zip(self.NAMES, masks) if bits & m}))
+
+    def _poll(self):
+        while not self.stop.wait(0.005):
+            try:
+                self._sample()
+            except Exception:
+                return
+
+    def __enter__(self):
+        import threading
+        try:
+            self.nvml = self._nvml_handle()
+            self._sample()
+            self.stop = threading.Event()
+            self.th = threading.Thread(target=self._poll, daemon=True)
+            self.th.start()
+        except Exception:
+            self.nvml = None
+            try:
+                q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+                     "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+                     "clocks_event_reasons.sw_power_cap")
+                self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.dev), f"--query-gpu={q}",
+                                           "--format=csv,noheader,nounits", "-lms", "100"],
+                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            except OSError:
+                self.p = None
         return self
 
     def __exit__(self, *a):
-        self.out = ""
-        if self.p:
+        if self.nvml:
+            self.stop.set()
+            self.th.join()
+            try:
+                self._sample()
+            except Exception:
+                pass
+        elif self.p:
             time.sleep(0.25)
             self.p.terminate()
             try:
-                self.out, _ = self.p.communicate(timeout=5)
+                out, _ = self.p.communicate(timeout=5)
             except subprocess.TimeoutExpired:
                 self.p.kill()
+                out = ""
+            for r in (out or "").strip().splitlines():
+                r = r.split(", ")
+                if len(r) >= 6 and r[0].strip().replace(".", "").isdigit():
+                    self.rows.append((float(r[0]), float(r[1]),
+                                      {n for n, x in zip(self.NAMES, r[2:6]) if x.strip() == "Active"}))
 
     def summary(self):
-        rows = [r.split(", ") for r in (self.out or "").strip().splitlines() if r.count(",") >= 5]
-        if not rows:
+        if not self.rows:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
-        sm = [float(r[0]) for r in rows if r[0].strip().replace(".", "").isdigit()]
-        mx = [float(r[1]) for r in rows if r[1].strip().replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in rows for i in range(4) if "Active" == r[2 + i].strip()})
-        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(rows)}
+        return {"sm_mhz": float(np.median([r[0] for r in self.rows])),
+                "sm_max_mhz": max(r[1] for r in self.rows),
+                "reasons": sorted(set().union(*(r[2] for r in self.rows))),
+                "samples": len(self.rows), "source": "nvml" if self.nvml else "nvidia-smi"}
 
 
 # ---------------------------------------------------------------- workload

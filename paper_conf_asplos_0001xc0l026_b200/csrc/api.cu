@@ -388,6 +388,19 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
       }
     }
   }
+  {   // experiments (R-4e): two-level accumulation — every tile split over K
+      // into chunks of <= kc, each accumulated in TMEM, the chunks summed in
+      // IEEE fp32 by the split-K fixup (fixed order)
+    static const int kc = getenv("BULLET_GEMM_KCHUNK") ? atoi(getenv("BULLET_GEMM_KCHUNK")) : 0;
+    if (kc >= 64 && K > kc) {
+      const int tiles = ((M + 128 * mh - 1) / (128 * mh)) * (N / bn);
+      const size_t per = (size_t)tiles * 128 * mh * bn;
+      int want = (K + kc - 1) / kc;
+      want = std::min(want, k_blocks);
+      const int cap = (int)std::min<size_t>(want, h->ph[c.phase].partial_floats / per);
+      if (cap >= 2 && tiles <= N_TILE_SEMS) { ts = cap; n_full = 0; }
+    }
+  }
   if (getenv("BULLET_GEMM_DEBUG"))
     fprintf(stderr, "gemm M=%d N=%d K=%d m_sms=%d -> mh=%d bn=%d n_full=%d ts=%d\n", M, N, K, c.m_sms, mh, bn,
             n_full, ts);

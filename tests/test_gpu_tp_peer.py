@@ -78,7 +78,7 @@ def _step_all(S, ranks, x_pre, x_dec, lb, le):
 
 
 @pytest.mark.parametrize("name,tp", [("qwen2.5-14b", 2), ("qwen2.5-14b", 4)])
-def test_peer_allreduce_full_model_dims(name, tp):
+def test_peer_allreduce_full_model_dims(name, tp, bar=1.5e-3):
     """BASELINE configs 4 (Qwen2.5-14B TP2 / TP4, QKV bias) and 5
     (Llama-3.1-70B TP8) at full layer dims, few tokens (the oracle is fp64
     C): one layer step of every simulated rank (TP8 = 16 partitions of 8 SMs)
@@ -109,7 +109,7 @@ def test_peer_allreduce_full_model_dims(name, tp):
         for i, nm in enumerate(("pre", "dec")):
             t = got[0][i].cpu().numpy()
             mx, mr = compare(t, ref[nm])
-            assert mx <= 2e-2 and mr <= 1.5e-3, (name, tp, nm, mx, mr)
+            assert mx <= 2e-2 and mr <= bar, (name, tp, nm, mx, mr)
             mx, mr = compare(t, single[i].astype(np.float64))
             assert mx <= 2e-2 and mr <= 5e-4, (name, tp, nm, "vs single-GPU", mx, mr)
         for bl in ranks:
@@ -182,3 +182,22 @@ def test_peer_allreduce_tp8_llama70b_subprocess():
             "T.test_peer_allreduce_full_model_dims('llama3.1-70b', 8); print('TP8-OK')" % (here, os.path.dirname(here)))
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=900)
     assert r.returncode == 0 and "TP8-OK" in r.stdout, (r.stdout[-2000:], r.stderr[-4000:])
+
+
+@pytest.mark.parametrize("kc", [1024, 512])
+def test_peer_allreduce_qwen14b_kchunk_meets_1e3(kc):
+    """DESIGN.md R-4e, two-level accumulation: with BULLET_GEMM_KCHUNK=kc
+    every long-K GEMM is split over K into chunks of <= kc (TMEM per chunk,
+    IEEE fp32 across chunks, fixed order), which brings the Qwen2.5-14B TP2
+    layer under the north-star bar (mean-rel 1e-3) against the oracle.  The
+    knob is read once per process: fresh process."""
+    import os
+    import subprocess
+    import sys
+    env = dict(os.environ, BULLET_GEMM_KCHUNK=str(kc))
+    here = os.path.dirname(os.path.abspath(__file__))
+    code = ("import sys; sys.path[:0] = [%r, %r]; import test_gpu_tp_peer as T; "
+            "T.test_peer_allreduce_full_model_dims('qwen2.5-14b', 2, bar=1e-3); print('KC-OK')"
+            % (here, os.path.dirname(here)))
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0 and "KC-OK" in r.stdout, (r.stdout[-2000:], r.stderr[-4000:])
