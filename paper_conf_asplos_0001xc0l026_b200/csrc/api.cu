@@ -388,23 +388,33 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
       }
     }
   }
-  {   // experiments (R-4e): two-level accumulation — every tile split over K
-      // into chunks of <= kc, each accumulated in TMEM, the chunks summed in
-      // IEEE fp32 by the split-K fixup (fixed order)
+  int kcb = 0;
+  {   // two-level accumulation (DESIGN R-4e), K chunks of <= kc accumulated
+      // in TMEM and summed in fp32 in a fixed order.  BULLET_GEMM_KCHUNK=kc
+      // (0 = off).  Default ("onchip"): the epilogue sums the chunks in
+      // registers (tile 128 x 128, whole tiles).  BULLET_GEMM_KCHUNK_MODE=
+      // splitk: every tile split over K, chunks summed by the split-K fixup
+      // through global memory (the first measurement; costly).
     static const int kc = getenv("BULLET_GEMM_KCHUNK") ? atoi(getenv("BULLET_GEMM_KCHUNK")) : 0;
+    static const bool splitk = getenv("BULLET_GEMM_KCHUNK_MODE") && !strcmp(getenv("BULLET_GEMM_KCHUNK_MODE"), "splitk");
     if (kc >= 64 && K > kc) {
-      const int tiles = ((M + 128 * mh - 1) / (128 * mh)) * (N / bn);
-      const size_t per = (size_t)tiles * 128 * mh * bn;
-      int want = (K + kc - 1) / kc;
-      want = std::min(want, k_blocks);
-      const int cap = (int)std::min<size_t>(want, h->ph[c.phase].partial_floats / per);
-      if (cap >= 2 && tiles <= N_TILE_SEMS) { ts = cap; n_full = 0; }
+      if (splitk) {
+        const int tiles = ((M + 128 * mh - 1) / (128 * mh)) * (N / bn);
+        const size_t per = (size_t)tiles * 128 * mh * bn;
+        const int want = std::min((K + kc - 1) / kc, k_blocks);
+        const int cap = (int)std::min<size_t>(want, h->ph[c.phase].partial_floats / per);
+        if (cap >= 2 && tiles <= N_TILE_SEMS) { ts = cap; n_full = 0; }
+      } else if (fits(128)) {
+        mh = 1; bn = 128; ts = 1;
+        n_full = ((M + 127) / 128) * (N / 128);
+        kcb = kc / 64;
+      }
     }
   }
   if (getenv("BULLET_GEMM_DEBUG"))
-    fprintf(stderr, "gemm M=%d N=%d K=%d m_sms=%d -> mh=%d bn=%d n_full=%d ts=%d\n", M, N, K, c.m_sms, mh, bn,
-            n_full, ts);
-  a.bn = bn; a.mh = mh; a.splits = ts; a.n_full = n_full;
+    fprintf(stderr, "gemm M=%d N=%d K=%d m_sms=%d -> mh=%d bn=%d n_full=%d kcb=%d ts=%d\n", M, N, K, c.m_sms, mh, bn,
+            n_full, kcb, ts);
+  a.bn = bn; a.mh = mh; a.splits = ts; a.n_full = n_full; a.kcb = kcb;
   {   // second copy issuer for the weight tiles (BULLET_GEMM_SPLIT_B=0/1 overrides; default: on)
     static const int sb = getenv("BULLET_GEMM_SPLIT_B") ? atoi(getenv("BULLET_GEMM_SPLIT_B")) : 1;
     a.split_b = sb ? 1 : 0;

@@ -412,7 +412,7 @@ size_t gemm_tc_smem_bytes(int bn, int mh) {
   return (size_t)gemm_tc_stages(bn, mh) * st + 1024 /*align*/ + 512 /*barriers etc.*/;
 }
 
-template <int mh>
+template <int mh, bool KC = false>
 __global__ void __launch_bounds__(NT, 1)
     k_gemm_tc(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
               GemmArgs a, int n_stages) {
@@ -571,7 +571,20 @@ __global__ void __launch_bounds__(NT, 1)
         mbar_wait(acce + as, aph ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tmem + as * acc_cols;
+        uint32_t d_tmem_c = d_tmem;
+        int kc0 = kb0;   // first k-block of the current accumulation chunk
         for (int kb = kb0; kb < kb1; ++kb) {
+          if (KC && kb > kb0 && (kb - kb0) % a.kcb == 0) {
+            // two-level accumulation: hand the finished chunk to the epilogue
+            // (it adds it to its fp32 registers) and start the next chunk in
+            // the other accumulator stage
+            tc_commit(accf + as);
+            if (++as == n_acc) { as = 0; aph ^= 1; }
+            mbar_wait(acce + as, aph ^ 1);
+            tc_fence_after();
+            d_tmem_c = tmem + as * acc_cols;
+            kc0 = kb;
+          }
           mbar_wait(full + s, ph);
           tc_fence_after();
           const uint32_t a_addr = smem_u32(smem + s * st_bytes), b_addr = a_addr + a_bytes;
@@ -579,8 +592,8 @@ __global__ void __launch_bounds__(NT, 1)
           for (int k = 0; k < BK / 16; ++k)
 #pragma unroll
             for (int hh = 0; hh < mh; ++hh)
-              tc_mma(d_tmem + hh * bn, sw128_desc(a_addr + hh * A_BYTES + k * 32), sw128_desc(b_addr + k * 32),
-                     idesc, (kb > kb0 || k > 0) ? 1u : 0u);
+              tc_mma(d_tmem_c + hh * bn, sw128_desc(a_addr + hh * A_BYTES + k * 32), sw128_desc(b_addr + k * 32),
+                     idesc, (kb > kc0 || k > 0) ? 1u : 0u);
           tc_commit(empty + s);
           if (++s == n_stages) { s = 0; ph ^= 1; }
         }
@@ -606,6 +619,42 @@ __global__ void __launch_bounds__(NT, 1)
       tile_coords(ui.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
       const int col0 = (a.epi == EPI_SILU) ? n_blk * (bn / 2) : n_blk * bn;
       const int out_chunks = (a.epi == EPI_SILU) ? bn / 64 : bn / 32;
+      if constexpr (KC) {   // mh == 1, bn == 128, whole tiles (plan guarantees)
+        const int n_ch = (k_blocks + a.kcb - 1) / a.kcb;
+        float R[128];
+        for (int ch = 0; ch < n_ch; ++ch) {
+          mbar_wait(accf + as, aph);
+          tc_fence_after();
+          const uint32_t tb = tmem + ((uint32_t)(eq * 32) << 16) + as * acc_cols;
+#pragma unroll
+          for (int c = 0; c < 4; ++c) {
+            tmem_ld32(tb + c * 32, v);
+#pragma unroll
+            for (int i = 0; i < 32; ++i) R[c * 32 + i] = ch ? R[c * 32 + i] + v[i] : v[i];   // chunk order: fixed
+          }
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(acce + as);
+          if (++as == n_acc) { as = 0; aph ^= 1; }
+        }
+        const int m = m_blk * BM + et;
+        if (m < a.M) {
+          if (a.epi == EPI_QKV) {
+            epi_qkv(a, m, col0, R, R + 64);
+            epi_qkv(a, m, col0 + 32, R + 32, R + 96);
+          } else if (a.epi == EPI_SILU) {
+            epi_store(a, m, col0, R, R + 64);
+            epi_store(a, m, col0 + 32, R + 32, R + 96);
+          } else {
+#pragma unroll
+            for (int c = 0; c < 4; ++c) epi_store(a, m, col0 + c * 32, R + c * 32, nullptr);
+          }
+        }
+        if (a.ar.n) ar_signal(a, m_blk, mh, et);
+        if (a.nf.out) norm_signal(a, m_blk, mh, et);
+        ++it;
+        continue;
+      }
       mbar_wait(accf + as, aph);
       tc_fence_after();
       const uint32_t tb = tmem + ((uint32_t)(eq * 32) << 16) + as * acc_cols;
@@ -768,11 +817,16 @@ cudaError_t launch_gemm_tc(const CUtensorMap& mapA, const CUtensorMap& mapB, con
       for (int bn = 64; bn <= 256; bn *= 2) mx = std::max(mx, gemm_tc_smem_bytes(bn, mh));
     cudaError_t e = cudaFuncSetAttribute(k_gemm_tc<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)mx);
     if (e == cudaSuccess) e = cudaFuncSetAttribute(k_gemm_tc<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)mx);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(k_gemm_tc<1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)mx);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
   if (a.mh < 1 || a.mh > 2 || a.splits < 1) return cudaErrorInvalidValue;
-  if (a.mh == 2) k_gemm_tc<2><<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn, 2));
+  if (a.kcb) {
+    if (a.mh != 1 || a.bn != 128 || a.n_full != (a.M + BM - 1) / BM * (a.N / 128)) return cudaErrorInvalidValue;
+    k_gemm_tc<1, true><<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn, 1));
+  } else if (a.mh == 2) k_gemm_tc<2><<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn, 2));
   else k_gemm_tc<1><<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn, 1));
   return cudaGetLastError();
 }
@@ -781,6 +835,7 @@ cudaError_t preload_gemm_tc() {
   cudaFuncAttributes f;
   cudaError_t e = cudaFuncGetAttributes(&f, k_gemm_tc<1>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_gemm_tc<2>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_gemm_tc<1, true>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_pack_weight);
   return e;
 }

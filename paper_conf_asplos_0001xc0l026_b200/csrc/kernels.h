@@ -70,6 +70,9 @@ struct GemmArgs {
   int b_evict_first;        // one M tile: the weight stream is used once (L2 evict-first)
   int b_rows;               // rows of B (packed layout stride)
   int split_b;              // 1: warp 3 issues the B tiles (second copy issuer), warp 0 the A tiles
+  int kcb;                  // two-level accumulation (DESIGN R-4e): K chunk in k-blocks (0 = off);
+                            // each chunk accumulates in TMEM, the chunks are summed in fp32
+                            // registers by the epilogue (requires mh == 1, bn == 128, splits == 1)
   // EPI_QKV (bf16, head_dim 128; fuses SURVEY §8a S3 into S2): the epilogue
   // adds the bias, rotates q / k heads (rotate-half RoPE from the (cos, sin)
   // table), rounds to bf16 (point R2) and stores q -> q_out[t][H][128],
