@@ -397,10 +397,14 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
       // through global memory (the first measurement; costly).
     static const int kc = getenv("BULLET_GEMM_KCHUNK") ? atoi(getenv("BULLET_GEMM_KCHUNK")) : 0;
     static const bool splitk = getenv("BULLET_GEMM_KCHUNK_MODE") && !strcmp(getenv("BULLET_GEMM_KCHUNK_MODE"), "splitk");
-    // BULLET_GEMM_KCHUNK_ONLY=silu: chunk only the gate_up GEMM (its R5
-    // rounding flips dominate the layer error, R-4e)
-    static const bool only_silu = getenv("BULLET_GEMM_KCHUNK_ONLY") && !strcmp(getenv("BULLET_GEMM_KCHUNK_ONLY"), "silu");
-    if (kc >= 64 && K > kc && (!only_silu || epi == EPI_SILU)) {
+    // BULLET_GEMM_KCHUNK_ONLY=silu: only the gate_up GEMM; =attn: only the
+    // GEMMs whose outputs are rounded or normalised inside the layer (QKV ->
+    // R2, O-proj -> RMSNorm -> R4); the down GEMM's fp32 output is the layer's
+    // own (R-4e)
+    static const char* only = getenv("BULLET_GEMM_KCHUNK_ONLY");
+    const bool sel = !only || (!strcmp(only, "silu") && epi == EPI_SILU) ||
+                     (!strcmp(only, "attn") && (epi == EPI_QKV || epi == EPI_F32 || (epi == EPI_RESID && K <= N)));
+    if (kc >= 64 && K > kc && sel) {
       if (splitk) {
         const int tiles = ((M + 128 * mh - 1) / (128 * mh)) * (N / bn);
         const size_t per = (size_t)tiles * 128 * mh * bn;
