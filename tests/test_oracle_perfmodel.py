@@ -255,3 +255,93 @@ def test_fitted_model_heldout_report_reproduces():
     assert abs(got["mre_heldout"] - want["mre_heldout"]) < 1e-9
     assert abs(got["slo_accuracy_heldout"] - want["slo_accuracy_heldout"]) < 1e-9
     assert got["mre_heldout"] < 0.191 and got["slo_accuracy_heldout"] > 0.88   # paper's numbers, context
+
+
+# ------------------------------------------- Alg. 1 l.3-10, hand-derived pins
+# evaluate_split and the R-21 / R-22 candidates are pinned here against values
+# worked out by hand from Alg. 1 with a stub layer time, so a
+# slip in rem_time, the queueing term, the TPOT update or the cycle / k
+# arithmetic fails independently of the kernel inventory.  Stub (ms): prefill
+# layer of n new tokens on m SMs = n / 3 / m, decode layer = 10 / m, both x f
+# when a co-runner holds SMs (f = 1.25), and M = 100 SMs.
+
+def _stub_layer_time(f):
+    def lt(shape, P, m, corun_m):
+        if m <= 0:
+            return math.inf
+        g = f if corun_m > 0 else 1.0
+        q = shape["q_lens"]
+        ms = 10.0 / m * g if all(x == 1 for x in q) else sum(q) / 3.0 / m * g
+        return ms / 1e3
+    return lt
+
+
+HAND = dict(layers_done=4, total_layers=32, prefill_lens=[100, 200], prefill_waited_ms=[10.0, 20.0],
+            pending_lens=[50], pending_waited_ms=[5.0], decode_tokens=[9, 19, 4],
+            decode_elapsed_ms=[90.0, 380.0, 40.0], decode_mean_ctx=1000, u_k=50, v_k=50)
+HAND_SLO = dict(ttft_norm_ms_per_tok=0.5, tpot_ms=20.0, w_max=4, v_min=16, percentile=0.9)
+
+
+def test_evaluate_split_hand_derived(monkeypatch):
+    """Split (u, v) = (50, 50), co-run factor 1.25, L = 32, l_k = 4:
+    t_p = 300/3/50 x 1.25 = 2.5 ms; rem = 2.5 x 28 = 70 ms (l.3).
+    TTFT/SLO (l.4-7, R-18: SLO = 0.5 ms x input length):
+      (70 + 10) / 50 = 1.6;  (70 + 20) / 100 = 0.9;
+      pending 50 tok: own = 50/3/50 x 1.25 x 32 = 13.333 ms -> (5 + 70 + 13.333) / 25 = 3.5333.
+    TPOT/SLO (l.8-10, R-14): iteration = 10/50 x 1.25 x 32 = 8 ms;
+      (90 + 8)/10/20 = 0.49, (380 + 8)/20/20 = 0.97, (40 + 8)/5/20 = 0.48.
+    Nearest-rank P90 of 3 = the largest; P50 = the 2nd smallest."""
+    monkeypatch.setattr(PM, "layer_time", _stub_layer_time(1.25))
+    P = PM.default_params(M=100)
+    ttft, tpot, t_p = PM.evaluate_split(P, MODEL, dict(HAND), HAND_SLO, 50, 50)
+    assert math.isclose(t_p, 2.5) and math.isclose(ttft, 3.5333333333333333) and math.isclose(tpot, 0.97)
+    ttft, tpot, _ = PM.evaluate_split(P, MODEL, dict(HAND), dict(HAND_SLO, percentile=0.5), 50, 50)
+    assert math.isclose(ttft, 1.6) and math.isclose(tpot, 0.49)
+
+
+def test_evaluate_split_decode_pause_hand_derived(monkeypatch):
+    """Decode pause (u, v) = (100, 0), v_k = 40: no co-runner, so
+    t_p = 300/3/100 = 1 ms, rem = 28 ms; TTFT/SLO = 38/50 = 0.76, 48/100 = 0.48,
+    pending (5 + 28 + 50/3/100 x 32) / 25 = 1.5333; the decodes wait one
+    prefill layer and then run an iteration alone on v_k SMs:
+    1 + 10/40 x 32 = 9 ms -> (90 + 9)/10/20 = 0.495, (380 + 9)/20/20 = 0.9725,
+    (40 + 9)/5/20 = 0.49."""
+    monkeypatch.setattr(PM, "layer_time", _stub_layer_time(1.25))
+    P = PM.default_params(M=100)
+    ttft, tpot, t_p = PM.evaluate_split(P, MODEL, dict(HAND, u_k=60, v_k=40), HAND_SLO, 100, 0)
+    assert math.isclose(t_p, 1.0) and math.isclose(ttft, 1.5333333333333333) and math.isclose(tpot, 0.9725)
+
+
+def _hand_state():
+    return dict(HAND, pending_lens=[], pending_waited_ms=[])
+
+
+HAND_SLO_LOOSE = dict(HAND_SLO, ttft_norm_ms_per_tok=100.0, tpot_ms=1e4)
+
+
+def test_reduce_decode_hand_derived(monkeypatch):
+    """Objective 0, both SLOs met everywhere: ReduceDecodeSM -> v = v_min = 16,
+    u = 84; k = round(t_p / t_d) = round((100/84 x 1.25) / (10/16 x 1.25))
+    = round(1.905) = 2."""
+    monkeypatch.setattr(PM, "layer_time", _stub_layer_time(1.25))
+    assert PM.choose_split(PM.default_params(M=100), MODEL, _hand_state(), HAND_SLO_LOOSE) == (84, 2)
+
+
+def test_max_throughput_and_timesliced_hand_derived(monkeypatch):
+    """Objective 1 (R-21 / R-22), n_pre = 300 tokens, 3 decodes.
+    Time-sliced cycle: t_p = 1 ms, t_d = 0.1 ms alone on 100 SMs, k_ts = 10,
+    cycle 2 ms -> (300 + 30) / 2 = 165 tokens/ms.
+    Co-run, f = 1.25: t_p = 125/(100 - v), t_d = 12.5/v, k = round(t_p/t_d):
+      v = 16: 1.488 / 0.781 -> k 2, cycle 1.5625, 306/1.5625 = 195.8
+      v = 18: 1.524 / 0.694 -> k 2, cycle 1.5244, 306/1.5244 = 200.7  (best)
+      v = 20: 1.5625 / 0.625 -> k 3, cycle 1.875, 309/1.875 = 164.8
+      v = 22: 1.603 / 0.568 -> k 3, cycle 1.705, 181.3;  v = 24: k 3, 1.645, 187.9
+    and t_p grows with v from there (v = 50: k 10, 330/2.5 = 132) -> (82, 2),
+    since 200.7 > 165.  With f = 2 every co-run time doubles (v = 18:
+    306/3.049 = 100.4 < 165) -> the time-sliced cycle (100, 10)."""
+    P = PM.default_params(M=100)
+    slo = dict(HAND_SLO_LOOSE, objective=1)
+    monkeypatch.setattr(PM, "layer_time", _stub_layer_time(1.25))
+    assert PM.choose_split(P, MODEL, _hand_state(), slo) == (82, 2)
+    monkeypatch.setattr(PM, "layer_time", _stub_layer_time(2.0))
+    assert PM.choose_split(P, MODEL, _hand_state(), slo) == (100, 10)
