@@ -276,6 +276,45 @@ int persist_grid(const Ctx& c, int per_sm) {
   return c.h->n_sms * per_sm * (c.m_sms < c.h->n_sms ? mult : 1);
 }
 
+// Two-level accumulation policy (DESIGN R-4e).  Default: K chunks of
+// KC_DEFAULT on the QKV and O-proj GEMMs when d_model >= 5120 — the GEMMs
+// whose outputs are rounded (R2) or normalised and rounded (R4) inside the
+// layer, where accumulation error turns into bf16 rounding flips that the
+// rest of the layer amplifies.  Overrides (read once per process):
+//   BULLET_GEMM_KCHUNK=kc (0 = off), BULLET_GEMM_KCHUNK_ONLY=list of
+//   qkv,oproj,gate_up,down | all | attn (= qkv,oproj) | silu (= gate_up),
+//   BULLET_GEMM_KCHUNK_MODE=splitk.
+constexpr int KC_DEFAULT = 256;
+constexpr unsigned KC_ALL = (1u << BULLET_K_QKV) | (1u << BULLET_K_OPROJ) | (1u << BULLET_K_GATE_UP) |
+                            (1u << BULLET_K_DOWN);
+struct KcPolicy { int kc_override; unsigned mask; bool splitk; };
+const KcPolicy& kc_policy() {
+  static const KcPolicy p = [] {
+    KcPolicy r{-1, (1u << BULLET_K_QKV) | (1u << BULLET_K_OPROJ), false};
+    if (const char* e = getenv("BULLET_GEMM_KCHUNK")) r.kc_override = atoi(e);
+    if (const char* e = getenv("BULLET_GEMM_KCHUNK_MODE")) r.splitk = !strcmp(e, "splitk");
+    if (const char* e = getenv("BULLET_GEMM_KCHUNK_ONLY")) {
+      r.mask = 0;
+      std::string s(e);
+      size_t a = 0;
+      while (a <= s.size()) {
+        size_t b = s.find(',', a);
+        if (b == std::string::npos) b = s.size();
+        const std::string t = s.substr(a, b - a);
+        if (t == "qkv") r.mask |= 1u << BULLET_K_QKV;
+        else if (t == "oproj") r.mask |= 1u << BULLET_K_OPROJ;
+        else if (t == "gate_up" || t == "silu") r.mask |= 1u << BULLET_K_GATE_UP;
+        else if (t == "down") r.mask |= 1u << BULLET_K_DOWN;
+        else if (t == "attn") r.mask |= (1u << BULLET_K_QKV) | (1u << BULLET_K_OPROJ);
+        else if (t == "all") r.mask |= KC_ALL;
+        a = b + 1;
+      }
+    }
+    return r;
+  }();
+  return p;
+}
+
 struct QkvEpi {   // EPI_QKV destinations
   void* q; void* pk; void* pv;
 };
@@ -389,32 +428,35 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
     }
   }
   int kcb = 0;
-  {   // two-level accumulation (DESIGN R-4e), K chunks of <= kc accumulated
-      // in TMEM and summed in fp32 in a fixed order.  BULLET_GEMM_KCHUNK=kc
-      // (0 = off).  Default ("onchip"): the epilogue sums the chunks in
-      // registers (tile 128 x 128, whole tiles).  BULLET_GEMM_KCHUNK_MODE=
-      // splitk: every tile split over K, chunks summed by the split-K fixup
-      // through global memory (the first measurement; costly).
-    static const int kc = getenv("BULLET_GEMM_KCHUNK") ? atoi(getenv("BULLET_GEMM_KCHUNK")) : 0;
-    static const bool splitk = getenv("BULLET_GEMM_KCHUNK_MODE") && !strcmp(getenv("BULLET_GEMM_KCHUNK_MODE"), "splitk");
-    // BULLET_GEMM_KCHUNK_ONLY=silu: only the gate_up GEMM; =attn: only the
-    // GEMMs whose outputs are rounded or normalised inside the layer (QKV ->
-    // R2, O-proj -> RMSNorm -> R4); the down GEMM's fp32 output is the layer's
-    // own (R-4e)
-    static const char* only = getenv("BULLET_GEMM_KCHUNK_ONLY");
-    const bool sel = !only || (!strcmp(only, "silu") && epi == EPI_SILU) ||
-                     (!strcmp(only, "attn") && (epi == EPI_QKV || epi == EPI_F32 || (epi == EPI_RESID && K <= N)));
+  {   // two-level accumulation (DESIGN R-4e): every tile's K range in chunks
+      // of <= kc, each accumulated in TMEM, the chunks summed in IEEE fp32 in
+      // a fixed order.  It brings the tcgen05 accumulation error (truncating,
+      // 4.3e-6 relative per long-K GEMM) near IEEE fp32, which the layer needs
+      // to stay under the north-star bar at d_model >= 5120 (R-4e).  Applied
+      // by GEMM kind (kc_policy); on-chip (the epilogue sums the chunks in
+      // registers, tile 128 x 128) unless BULLET_GEMM_KCHUNK_MODE=splitk
+      // (chunks summed by the split-K fixup through global memory).
+    const KcPolicy& kp = kc_policy();
+    const int kc = kp.kc_override >= 0 ? kp.kc_override : (h->cfg.d_model >= 5120 ? KC_DEFAULT : 0);
+    int kind = c.kind;
+    if (c.op) kind = epi == EPI_QKV ? BULLET_K_QKV : epi == EPI_SILU ? BULLET_K_GATE_UP : -1;
+    const bool sel = kind >= 0 ? ((kp.mask >> kind) & 1u) != 0 : kp.mask == KC_ALL;
     if (kc >= 64 && K > kc && sel) {
-      if (splitk) {
+      bool done = false;
+      if (kp.splitk) {
         const int tiles = ((M + 128 * mh - 1) / (128 * mh)) * (N / bn);
         const size_t per = (size_t)tiles * 128 * mh * bn;
         const int want = std::min((K + kc - 1) / kc, k_blocks);
-        const int cap = (int)std::min<size_t>(want, h->ph[c.phase].partial_floats / per);
-        if (cap >= 2 && tiles <= N_TILE_SEMS) { ts = cap; n_full = 0; }
-      } else if (fits(128)) {
+        const size_t cap = h->ph[c.phase].partial_floats / per;
+        // every chunk must get its own split: when the partials do not fit
+        // (prefill-sized M) fall through to the on-chip mode instead of
+        // silently running fewer, longer chunks
+        if ((size_t)want <= cap && tiles <= N_TILE_SEMS) { ts = want; n_full = 0; done = true; }
+      }
+      if (!done && fits(128)) {
         mh = 1; bn = 128; ts = 1;
         n_full = ((M + 127) / 128) * (N / 128);
-        kcb = kc / 64;
+        kcb = std::max(1, kc / 64);
       }
     }
   }
@@ -881,7 +923,7 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
               cudaMalloc(&P.partials, P.partial_floats * sizeof(float)) == cudaSuccess &&
               cudaMalloc(&P.tile_sems, N_TILE_SEMS * sizeof(int)) == cudaSuccess &&
               cudaMalloc(&P.counters, P.n_counters * sizeof(int)) == cudaSuccess &&
-              cudaMalloc(&P.tiles, (T / ATTN_TC_BQ + 1024) * sizeof(int2)) == cudaSuccess &&
+              cudaMalloc(&P.tiles, (T / ATTN_TC_BQ + T + 1) * sizeof(int2)) == cudaSuccess &&
               cudaMalloc(&P.n_tiles, sizeof(int)) == cudaSuccess &&
               cudaMalloc(&P.tok, T * sizeof(TokInfo)) == cudaSuccess &&
               cudaMalloc(&P.order, T * sizeof(int4)) == cudaSuccess &&
@@ -1057,7 +1099,10 @@ static int step_impl(bullet_handle* h, const bullet_batch* pre, const bullet_bat
   // and drain dominate there: decode layer-step -1.6 % on 76 SMs); a prefill
   // GEMM's tail runs it with one CTA per SM where the standalone kernel packs
   // several (+0.7 % on a prefill layer) — so only up to 1024 rows
-  const bool fn_ok = !(flags & BULLET_UNFUSED_NORM) && h->cfg.dtype == BULLET_DTYPE_BF16 && !h->peer_mode &&
+  // never under tensor parallelism: the row-parallel GEMMs' outputs are
+  // partials until the all-reduce, so a norm in their tail would read them
+  // (and S1 of the next layer would be skipped with nothing replacing it)
+  const bool fn_ok = !(flags & BULLET_UNFUSED_NORM) && h->cfg.dtype == BULLET_DTYPE_BF16 && h->cfg.tp_size == 1 &&
                      h->cfg.d_model <= 8192;
   static const int fn_rows = getenv("BULLET_FUSED_NORM_MAX_ROWS") ? atoi(getenv("BULLET_FUSED_NORM_MAX_ROWS")) : 1024;
   cp.fuse_norm = fn_ok && pre && pre->n_tokens <= fn_rows;

@@ -140,6 +140,7 @@ class ServingLoop:
         self.split = (n_sms // 2, n_sms - n_sms // 2)
         self.chunk_tokens = chunk_tokens
         self.log = []                 # per cycle: (now, p, k, prefill tokens, decodes, ms)
+        self.unservable = []          # requests that can never be admitted (reported, loop ends)
         # online estimator feedback: after every co-run cycle the
         # ratio measured / predicted cycle time updates an EMA that rescales
         # the model's co-location factors p_c, p_b (bullet_set_colocation),
@@ -281,6 +282,9 @@ class ServingLoop:
                 if nxt < len(trace):           # idle until the next arrival
                     now = max(now, trace[nxt].arrival_ms)
                     continue
+                if not ready:                  # pending requests that can never be admitted
+                    self.unservable = list(pending)   # (prompt > max_prefill_tokens or KV pool too small)
+                    break
             if now >= horizon:
                 break
             # ---- split decision
@@ -315,6 +319,9 @@ class ServingLoop:
                 de = min(d_layer + k, self.L)
                 dw = PhaseWork(members, [1] * len(members), [r.ctx for r in members], d_layer, de, dec_id)
             if pw is None and dw is None:     # e.g. p = 0 chosen while decode is empty
+                if prefill is None:           # nothing runnable this cycle: stop, never build an empty batch
+                    self.unservable = list(pending)
+                    break
                 p, k = self.N, 0
                 le = min(layers_done + self.lp, self.L)
                 pw = PhaseWork(prefill, [r.prompt for r in prefill], [0] * len(prefill), layers_done, le, pre_id)
@@ -371,4 +378,4 @@ class ServingLoop:
                 "goodput_req_s": sum(ok) / dur_s, "throughput_tok_s": sum(r.prompt + r.out_len for r in done) / dur_s,
                 "ttft_ms_p50": pct(ttft, 50), "ttft_ms_p90": pct(ttft, 90),
                 "norm_ttft_ms_per_tok_p90": pct(nttft, 90), "tpot_ms_p50": pct(tpot, 50),
-                "tpot_ms_p90": pct(tpot, 90), "slo": s.as_dict()}
+                "tpot_ms_p90": pct(tpot, 90), "unservable": len(self.unservable), "slo": s.as_dict()}

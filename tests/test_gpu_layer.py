@@ -241,6 +241,56 @@ def test_fused_qkv_rope_matches_unfused(p, bias):
     assert float((a_pre - b_pre).abs().max()) <= 2e-2 and float((a_dec - b_dec).abs().max()) <= 2e-2
 
 
+@pytest.mark.parametrize("bias", [0, 1])
+def test_fused_qkv_pool_vs_oracle(bias):
+    """S3 in the QKV GEMM epilogue (EPI_QKV, the default bf16 path) against
+    the oracle directly: after one co-run layer step the pool holds the
+    oracle's k / v at exactly the slots the definition names
+    (block_table[r][p / 16] * 16 + p % 16 for every new position p of every
+    request; a sentinel planted there must be gone), every other slot of the
+    pool is bit-for-bit what it was, and the written values equal the
+    oracle's R2-rounded k / v except for rare one-step rounding flips."""
+    m = synth.ModelShape("qkvpool", 1024, 8, 2, 128, 2816, 1, qkv_bias=bias, rope_theta=1e6, rope_llama3=0)
+    pre_lens, dec_ctx = [300, 77, 1, 129], [64, 1, 500, 31, 16, 0]
+    S = Setup(m, pre_lens, dec_ctx, n_layers=1)
+    q = pre_lens + [1] * len(dec_ctx)
+    c = [0] * len(pre_lens) + dec_ctx
+    slots = set()
+    for r, (ql, cl) in enumerate(zip(q, c)):
+        for i in range(ql):
+            pos = cl + i
+            slots.add((int(S.lay.block_table[r][pos // 16]), pos % 16))
+    SENT = -3.0
+    for k, v in S.pool_cpu:                       # sentinel at every slot the step must write
+        for blk, off in slots:
+            k[blk, :, off, :] = SENT; v[blk, :, off, :] = SENT
+    for (k, v), (kc, vc) in zip(S.pool_gpu, S.pool_cpu):
+        k.copy_(kc.to(k.dtype)); v.copy_(vc.to(v.dtype))
+    before_k, before_v = S.pool_cpu[0][0].clone(), S.pool_cpu[0][1].clone()
+    # oracle: one layer on copies of the same pool (it writes k / v in place)
+    import oracle as O
+    from harness import oracle_cfg
+    cfg = oracle_cfg(m)
+    w = {kk: (None if vv is None else vv.numpy()) for kk, vv in S.w_cpu[0].items()}
+    pk, pv = before_k.numpy().astype(np.float32).copy(), before_v.numpy().astype(np.float32).copy()
+    O.layer_forward(cfg, w, pk, pv, pre_lens, [0] * len(pre_lens), S.lay.block_table[:S.n_pre],
+                    S.x_pre.double().numpy())
+    O.layer_forward(cfg, w, pk, pv, [1] * len(dec_ctx), dec_ctx, S.lay.block_table[S.n_pre:],
+                    S.x_dec.double().numpy())
+    _run(S, 64, S.B.CORUN)
+    gk, gv = S.pool_gpu[0][0].float().cpu().numpy(), S.pool_gpu[0][1].float().cpu().numpy()
+    mask = np.zeros((S.lay.n_blocks, 16), bool)
+    for blk, off in slots:
+        mask[blk, off] = True
+    for got, ref, old in ((gk, pk, before_k.numpy()), (gv, pv, before_v.numpy())):
+        g_s, r_s, o_s = (a.transpose(0, 2, 1, 3) for a in (got, ref, old))   # [blk][slot][Hkv][hd]
+        assert np.array_equal(g_s[~mask], o_s[~mask])          # untouched slots: bit-identical
+        assert not np.any(g_s[mask] == SENT)                  # every named slot written
+        gw, rw = g_s[mask].astype(np.float64), r_s[mask].astype(np.float64)   # oracle: already R2-rounded
+        assert np.all(np.abs(gw - rw) <= np.abs(rw) * 2.0 ** -7)   # equal, or one bf16 step apart (a flip)
+        assert np.mean(gw == rw) > 0.99
+
+
 @pytest.mark.parametrize("mode", ["timesliced", "corun"])
 def test_hybrid_chunked_prefill_batch(mode):
     """Chunked-prefill hybrid batch: prefill chunks

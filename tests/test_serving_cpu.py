@@ -166,3 +166,17 @@ def test_online_feedback_learns_observed_contention():
     est.set_colocation(*base)
     with pytest.raises(Exception):
         est.set_colocation(0.0, 1.0)
+
+
+@pytest.mark.parametrize("policy", ["bullet", "timesliced", "prefill_first"])
+def test_unservable_request_ends_the_loop(pm, policy):
+    """A request whose prompt exceeds max_prefill_tokens can never be admitted:
+    once the rest of the trace is served the loop stops and reports it (it
+    never builds a prefill batch out of nothing)."""
+    trace = SV.poisson_trace(40.0, 0.3, seed=3)
+    big = SV.Request(rid=10 ** 6, arrival_ms=trace[-1].arrival_ms + 1.0, prompt=9000, out_len=4)
+    rec = Recorder(pm)
+    loop = SV.ServingLoop(L, N, rec, pm.choose_split, policy, SV.BlockAllocator(8000), max_decodes=128,
+                          k_full=4, max_prefill_tokens=8192)
+    res = loop.run(trace + [big])
+    assert res["finished"] == len(trace) and res["unservable"] == 1 and loop.unservable[0].rid == 10 ** 6
