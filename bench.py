@@ -49,13 +49,20 @@ def peaks():
 
 # ---------------------------------------------------------------- dist utils
 def dist_init():
+    """One process per GPU (torchrun env).  When there are fewer GPUs than
+    ranks (a multi-rank check on a 1-GPU lease) ranks share devices and the
+    process group runs on gloo — NCCL refuses two ranks on one device."""
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if ws > 1:
         import torch.distributed as dist
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        n_dev = torch.cuda.device_count()
+        torch.cuda.set_device(local % n_dev)
+        if n_dev >= ws:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group("gloo")
     elif torch.cuda.is_available():
         torch.cuda.set_device(0)
     return ws, rank
@@ -68,12 +75,27 @@ def barrier(ws):
 
 
 def allreduce_max(x, ws):
+    """Max over ranks (device timings: the slowest rank defines the job)."""
     if ws == 1:
         return x
     import torch.distributed as dist
-    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
+
+
+def broadcast_obj(x, ws):
+    """Rank 0's value of x on every rank."""
+    if ws == 1:
+        return x
+    import torch.distributed as dist
+    o = [x]
+    dist.broadcast_object_list(o, src=0)
+    return o[0]
+
+
+DEFAULT_CONFIG = {1: "arxiv-8b", 2: "qwen14b-tp2", 4: "qwen14b-tp4", 8: "llama70b-tp8"}
 
 
 # ---------------------------------------------------------------- clocks
@@ -188,6 +210,7 @@ class Step:
         self.m_full = synth.MODELS[self.wl.model]
         self.tp = self.wl.tp
         ws = int(os.environ.get("WORLD_SIZE", "1"))
+        self.ws = ws
         self.rank = int(os.environ.get("RANK", "0"))
         if self.tp != 1 and ws != self.tp:
             raise SystemExit(f"config {config} is tensor-parallel (tp={self.tp}): run it under torchrun "
@@ -251,6 +274,9 @@ class Step:
         self.sp.wait_event(ev2)
 
     def time_steps(self, n, p, flags, pre=True, dec=True):
+        """Device time per step (ms), max over ranks: every rank gets the same
+        number, so decisions taken from timings agree across ranks and every
+        rank enqueues the identical step sequence (TP collectives pair up)."""
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(self.sp)
@@ -258,7 +284,7 @@ class Step:
             self.enqueue(p, flags, pre, dec)
         e1.record(self.sp)
         torch.cuda.synchronize()
-        return e0.elapsed_time(e1) / n
+        return allreduce_max(e0.elapsed_time(e1) / n, self.ws)
 
     # ---- chunked-prefill hybrid baseline
     def build_hybrid(self, k):
@@ -294,7 +320,7 @@ class Step:
             self.enqueue_hybrid()
         e1.record(self.sp)
         torch.cuda.synchronize()
-        return e0.elapsed_time(e1) / n
+        return allreduce_max(e0.elapsed_time(e1) / n, self.ws)
 
     def ab_vs_hybrid(self, p, blocks=6, per=5):
         """Co-run vs the chunked-prefill hybrid on the same work, alternating blocks."""
@@ -420,24 +446,72 @@ def kernel_work(S: Step, kind: str, phase: int):
 
 
 # ---------------------------------------------------------------- CPU oracle
-def oracle_sample(m: synth.ModelShape, wl: synth.Workload, n_pre_tok=64, n_dec=32):
-    """Bounded sample of the same workload for the CPU oracle: one prefill
-    request of n_pre_tok tokens + the first n_dec decode requests, one layer.
-    Returns (seconds, tokens) with tokens in the metric's unit."""
+def oracle_rowsampled(m: synth.ModelShape, wl: synth.Workload, k: int, pre_rows=256, dec_rows=64, kv_limit=None):
+    """The CPU oracle timed on a row sample of the config's OWN step (SURVEY
+    §8c "How the oracle runs at scale"), extrapolated to the whole step —
+    the extrapolation is labelled in the returned description.
+
+    Prefill: every request at its full length; the layer's RMSNorm + QKV +
+    RoPE + KV write for every token (the keys are needed) is timed alone
+    (empty row mask: T_kv), then the whole layer for `pre_rows` sampled query
+    rows (always the last row of every request): T_s.  Decode: `dec_rows` of
+    the decode requests (seeded sample), each with its full context: T_d.
+    Extrapolation: T_pre = T_kv + (T_s - T_kv) * n_p / pre_rows,
+    T_dec = T_d * n_d / dec_rows, step = one prefill layer + k decode
+    layer-steps, tokens = (n_p + n_d k) / L (the GPU line's unit).
+    `kv_limit` (reference arm): time the prefill on its first kv_limit tokens
+    of each request instead, scaled by n_p / kv_limit rows (also labelled)."""
     import oracle as O
     sys.path.insert(0, os.path.join(ROOT, "tests"))
     from harness import oracle_cfg
-    q = [n_pre_tok] + [1] * n_dec
-    c = [0] + list(wl.decode_ctx[:n_dec])
-    lay = synth.paged_layout(q, c, 16)
-    w = {k: (None if v is None else v.numpy()) for k, v in synth.layer_weights(m, 0).items()}
+    cfg = oracle_cfg(m)
+    w = {kk: (None if v is None else v.numpy()) for kk, v in synth.layer_weights(m, 0).items()}
+    rng = np.random.default_rng(11)
+    pre = [min(x, kv_limit) for x in wl.prefill_lens] if kv_limit else list(wl.prefill_lens)
+    n_p_run = sum(pre)
+    # ---- prefill
+    lay = synth.paged_layout(pre, [0] * len(pre), 16)
     pk, pv = synth.kv_pool(m, lay.n_blocks, 16, 0)
     pk, pv = pk.numpy(), pv.numpy()
-    x = synth.hidden(sum(q), m.d_model).double().numpy()
+    x = synth.hidden(n_p_run, m.d_model).double().numpy()
+    rows = min(pre_rows, n_p_run)
+    mask = np.zeros(n_p_run, dtype=np.uint8)
+    last = np.cumsum(pre) - 1
+    mask[last] = 1
+    extra = rows - int(mask.sum())
+    if extra > 0:
+        mask[rng.choice(np.flatnonzero(mask == 0), extra, replace=False)] = 1
+    rows = int(mask.sum())
     t0 = time.perf_counter()
-    O.layer_forward(oracle_cfg(m), w, pk, pv, q, c, lay.block_table, x)
-    dt = time.perf_counter() - t0
-    return dt, (n_pre_tok + n_dec) / m.n_layers, f"1 layer: 1 prefill x {n_pre_tok} tok + {n_dec} decodes (ctx {min(c[1:])}-{max(c[1:])})"
+    O.layer_forward(cfg, w, pk.copy(), pv.copy(), pre, [0] * len(pre), lay.block_table, x,
+                    row_mask=np.zeros(n_p_run, dtype=np.uint8))
+    t_kv = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    O.layer_forward(cfg, w, pk, pv, pre, [0] * len(pre), lay.block_table, x, row_mask=mask)
+    t_s = time.perf_counter() - t0
+    n_p = sum(wl.prefill_lens)
+    scale_kv = n_p / n_p_run
+    t_pre = (t_kv + max(0.0, t_s - t_kv) * n_p_run / rows) * scale_kv
+    # ---- decode
+    n_d = len(wl.decode_ctx)
+    di = np.sort(rng.choice(n_d, min(dec_rows, n_d), replace=False))
+    ctx = [wl.decode_ctx[i] for i in di]
+    lay_d = synth.paged_layout([1] * len(ctx), ctx, 16, seed_offset=1)
+    dk, dv = synth.kv_pool(m, lay_d.n_blocks, 16, 0)
+    xd = synth.hidden(len(ctx), m.d_model, 1).double().numpy()
+    t0 = time.perf_counter()
+    O.layer_forward(cfg, w, dk.numpy(), dv.numpy(), [1] * len(ctx), ctx, lay_d.block_table, xd)
+    t_d = (time.perf_counter() - t0) * n_d / len(ctx)
+    t_step = t_pre + k * t_d
+    tokens = (n_p + n_d * k) / m.n_layers
+    desc = (f"{wl.name} step (1 prefill layer + {k} decode layer-steps, {m.name}), extrapolated from a row "
+            f"sample: prefill {len(pre)} reqs / {n_p_run} tok with K/V of every token "
+            f"({t_kv:.1f} s) + full layer on {rows} sampled rows ({t_s:.1f} s), x{n_p_run / rows:.0f} rows"
+            + (f", x{scale_kv:.1f} for the untimed prompt tail (prompts capped at {kv_limit})" if kv_limit else "")
+            + f"; decode {len(ctx)} of {n_d} requests with full contexts ({t_d * len(ctx) / n_d:.1f} s), "
+            f"x{n_d / len(ctx):.0f}")
+    return {"seconds_per_step": t_step, "tokens_per_step": tokens, "value": tokens / t_step, "sample": desc,
+            "t_prefill_layer_s": t_pre, "t_decode_layer_s": t_d, "timed_s": t_kv + t_s + t_d * len(ctx) / n_d}
 
 
 def cpu_model() -> str:
@@ -451,28 +525,33 @@ def cpu_model() -> str:
 
 
 def run_reference(args, ws, rank):
+    """The oracle arm (`--impl reference`): there is no reference code (the
+    reference is PAPER.md only), so the CPU oracle, as it stands, is timed on
+    the box's host cores for the same config / metric / unit.  Each step is
+    a bounded row sample of the config's step (prompts capped at 512 tokens,
+    32 sampled prefill rows, 8 decode requests), extrapolated to the whole
+    step (labelled).  Rank 0 only."""
     if rank != 0:
         return
     wl = synth.workload(args.config)
     m = synth.MODELS[wl.model]
+    k = args.k or 4
     for _ in range(args.warmup):
-        oracle_sample(m, wl)
-    ts, toks = [], 0.0
-    for _ in range(args.steps):
-        dt, tk, desc = oracle_sample(m, wl)
-        ts.append(dt)
-        toks = tk
-    T = sum(ts) / len(ts)
-    v = toks / T
-    cores = os.cpu_count()
+        oracle_rowsampled(m, wl, k, pre_rows=32, dec_rows=8, kv_limit=512)
+    res = [oracle_rowsampled(m, wl, k, pre_rows=32, dec_rows=8, kv_limit=512) for _ in range(args.steps)]
+    T = float(np.mean([r["seconds_per_step"] for r in res]))
+    v = res[0]["tokens_per_step"] / T
+    import oracle as O
+    cores = O.set_threads(0)
     print(json.dumps({
         "impl": "reference", "metric": METRIC, "value": v,
         "unit": "tokens/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": T * 1e3, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "f64", "data": "synthetic",
-        "config": {"workload": args.config, "model": wl.model, "sample": desc},
-        "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": cores, "kind": "oracle", "sample": desc,
-                         "cpu_model": cpu_model()},
+        "config": {"workload": args.config, "model": wl.model, "decode_layer_steps": k},
+        "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": cores, "kind": "oracle",
+                         "sample": res[0]["sample"], "cpu_model": cpu_model(),
+                         "timed_s_per_step": float(np.mean([r["timed_s"] for r in res]))},
         "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}))
 
 
@@ -483,7 +562,8 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="bullet", choices=["bullet", "reference"])
-    ap.add_argument("--config", default="sharegpt-8b")
+    ap.add_argument("--config", default=None,
+                    help="workload (default by --gpus: 1 arxiv-8b (BASELINE config 3), 2/4 qwen14b-tp2/4, 8 llama70b-tp8)")
     ap.add_argument("--p", type=int, default=None, help="prefill SM count (default: tuned)")
     ap.add_argument("--k", type=int, default=None, help="decode layer-steps per prefill layer")
     ap.add_argument("--k-max", type=int, default=16)
@@ -493,6 +573,8 @@ def main():
                     help="TP configs: fused peer-memory all-reduce (default) or NCCL")
     args = ap.parse_args()
     ws, rank = dist_init()
+    if args.config is None:
+        args.config = DEFAULT_CONFIG.get(args.gpus, "arxiv-8b")
     if args.impl == "reference":
         run_reference(args, ws, rank)
         return
@@ -788,13 +870,11 @@ def main():
     }
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
         import oracle as O
-        dt, tk, desc = oracle_sample(S.m, S.wl)
-        O.set_threads(1)
-        dt1, tk1, desc1 = oracle_sample(S.m, S.wl, n_pre_tok=16, n_dec=8)
-        O.set_threads(0)
-        out["cpu_baseline"] = {"value": tk / dt, "unit": "tokens/s", "cores": os.cpu_count(),
-                               "kind": "oracle", "sample": desc, "cpu_model": cpu_model(),
-                               "one_core": {"value": tk1 / dt1, "cores": 1, "sample": desc1}}
+        cores = O.set_threads(0)
+        cb = oracle_rowsampled(S.m, S.wl, k, pre_rows=256, dec_rows=len(S.wl.decode_ctx))
+        out["cpu_baseline"] = {"value": cb["value"], "unit": "tokens/s", "cores": cores, "kind": "oracle",
+                               "sample": cb["sample"], "cpu_model": cpu_model(), "timed_s": cb["timed_s"],
+                               "seconds_per_step_extrapolated": cb["seconds_per_step"]}
     if rank == 0:
         print(json.dumps(out))
     if ws > 1:

@@ -90,7 +90,8 @@ def lib():
                      "bullet_op_rmsnorm", "bullet_op_rope_kv", "bullet_op_attention",
                      "bullet_profile_read", "bullet_launch_count", "bullet_tp_base", "bullet_tp_ipc_handle",
                      "bullet_tp_connect", "bullet_tp_connect_ipc", "bullet_tp_hidden", "bullet_set_split",
-                     "bullet_get_colocation", "bullet_set_colocation"):
+                     "bullet_get_colocation", "bullet_set_colocation", "bullet_trace_enable",
+                     "bullet_trace_read"):
             getattr(L, name).restype = c_int
         L.bullet_create.argtypes = [ctypes.POINTER(ModelCfg), ctypes.POINTER(KvPool), c_void_p,
                                     ctypes.c_char_p, ctypes.POINTER(c_void_p)]
@@ -111,6 +112,8 @@ def lib():
         L.bullet_profile_read.argtypes = [c_void_p, P_i32, P_i32, P_i32, ctypes.POINTER(c_float), c_int,
                                           ctypes.POINTER(c_int)]
         L.bullet_launch_count.argtypes = [c_void_p, ctypes.POINTER(ctypes.c_longlong)]
+        L.bullet_trace_enable.argtypes = [c_void_p, c_int]
+        L.bullet_trace_read.argtypes = [c_void_p, c_void_p, c_void_p, c_int, ctypes.POINTER(c_int)]
         L.bullet_nccl_unique_id.argtypes = [c_void_p]
         L.bullet_tp_base.argtypes = [c_void_p, ctypes.POINTER(c_void_p)]
         L.bullet_set_split.argtypes = [c_void_p, c_int, c_int, c_int, c_int, c_void_p]
@@ -353,6 +356,21 @@ class Bullet:
         ms = (c_float * cap)(); n = c_int()
         _check(lib().bullet_profile_read(self.h, k, p, l, ms, cap, ctypes.byref(n)))
         return [(KERNEL_KINDS[k[i]], p[i], l[i], ms[i]) for i in range(n.value)]
+
+    TRACE_CTAS = 2368   # include/bullet.h BULLET_TRACE_CTAS
+
+    def trace_enable(self, max_launches: int):
+        """Per-CTA timestamps of the next `max_launches` launches (diagnostics)."""
+        _check(lib().bullet_trace_enable(self.h, int(max_launches)))
+
+    def trace_read(self, cap=256):
+        """(records uint64 [n][TRACE_CTAS][8], meta int32 [n][4]) of the traced launches."""
+        import numpy as np
+        rec = np.zeros((cap, self.TRACE_CTAS, 8), dtype=np.uint64)
+        meta = np.zeros((cap, 4), dtype=np.int32)
+        n = c_int()
+        _check(lib().bullet_trace_read(self.h, rec.ctypes.data, meta.ctypes.data, cap, ctypes.byref(n)))
+        return rec[:n.value], meta[:n.value]
 
     def launch_count(self) -> int:
         n = ctypes.c_longlong()

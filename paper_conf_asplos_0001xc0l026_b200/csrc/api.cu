@@ -179,6 +179,10 @@ struct bullet_handle {
   std::vector<cudaEvent_t> ev_pool;
   size_t ev_used = 0;
   long long n_launch = 0;
+  // bullet_trace_enable: per-CTA timestamp records of the next launches
+  unsigned long long* trace = nullptr;
+  int trace_cap = 0, trace_n = 0;
+  std::vector<int> trace_meta;   // [trace_cap][4]
 };
 
 namespace {
@@ -248,6 +252,21 @@ int next_launch(Ctx& c, Launch* L) {
   L->log_cap = c.h->log_cap;
   L->launch_id = c.h->launch_seq++;
   L->phase = c.phase;
+  // Programmatic dependent launch (common.cuh) is OFF by default
+  // (BULLET_PDL=1 enables it, for experiments): an early-launched kernel's
+  // CTAs land on the SMs its predecessor's out-of-range CTAs freed, leave
+  // (gated out), and the next ones land there again — the whole grid can
+  // drain through the wrong SMs before one of its own frees up, leaving the
+  // work to the last CTA (gate_enter).  Measured: prefill layer 2.36 ->
+  // 102 ms on 76 SMs.  Not under BULLET_PROFILE, not for op-level entries.
+  static const bool pdl_on = getenv("BULLET_PDL") && !strcmp(getenv("BULLET_PDL"), "1");
+  L->pdl = pdl_on && !c.op && !c.prof;
+  if (c.h->trace && c.h->trace_n < c.h->trace_cap) {
+    const int i = c.h->trace_n++;
+    L->trace = c.h->trace + (size_t)i * BULLET_TRACE_CTAS * 8;
+    int* m = c.h->trace_meta.data() + 4 * i;
+    m[0] = c.kind; m[1] = c.phase; m[2] = c.layer; m[3] = 0;
+  }
   if (c.op) {
     CK(cudaMemsetAsync(c.h->op_ctr, 0, 2 * sizeof(int), c.st));
     L->ctr = c.h->op_ctr;
@@ -1222,6 +1241,37 @@ int bullet_launch_count(const bullet_handle* h, long long* n) {
   return BULLET_OK;
 }
 
+int bullet_trace_enable(bullet_handle* h, int max_launches) {
+  if (!h || max_launches < 0) return set_err(BULLET_EINVAL, "bad argument");
+  if (h->host_only) return set_err(BULLET_EUNSUPPORTED, "host-only handle");
+  CK(cudaDeviceSynchronize());
+  cudaFree(h->trace);
+  h->trace = nullptr; h->trace_cap = h->trace_n = 0;
+  h->trace_meta.clear();
+  if (max_launches == 0) return BULLET_OK;
+  const size_t bytes = (size_t)max_launches * BULLET_TRACE_CTAS * 8 * sizeof(unsigned long long);
+  if (cudaMalloc(&h->trace, bytes) != cudaSuccess) return set_err(BULLET_ENOMEM, "trace buffer (%zu bytes)", bytes);
+  CK(cudaMemset(h->trace, 0, bytes));
+  h->trace_cap = max_launches;
+  h->trace_meta.assign((size_t)4 * max_launches, 0);
+  return BULLET_OK;
+}
+
+int bullet_trace_read(bullet_handle* h, uint64_t* rec, int32_t* meta, int cap, int* n) {
+  if (!h || !n || cap < 0 || (cap > 0 && (!rec || !meta))) return set_err(BULLET_EINVAL, "bad argument");
+  *n = 0;
+  if (!h->trace) return BULLET_OK;
+  CK(cudaDeviceSynchronize());
+  const int k = std::min(cap, h->trace_n);
+  const size_t per = (size_t)BULLET_TRACE_CTAS * 8;
+  CK(cudaMemcpy(rec, h->trace, (size_t)k * per * sizeof(unsigned long long), cudaMemcpyDeviceToHost));
+  memcpy(meta, h->trace_meta.data(), (size_t)k * 4 * sizeof(int32_t));
+  *n = k;
+  CK(cudaMemset(h->trace, 0, (size_t)h->trace_cap * per * sizeof(unsigned long long)));
+  h->trace_n = 0;
+  return BULLET_OK;
+}
+
 int bullet_sync(bullet_handle* h) {
   if (!h) return set_err(BULLET_EINVAL, "null");
   if (h->host_only) return BULLET_OK;
@@ -1248,6 +1298,7 @@ void bullet_destroy(bullet_handle* h) {
   }
   for (void* p : h->ipc_opened) cudaIpcCloseMemHandle(p);
   cudaFree(h->sym);
+  cudaFree(h->trace);
   cudaFree(h->rope_cs);
   for (auto& P : h->wp) cudaFree(P.base);
   cudaFree(h->op_pack);

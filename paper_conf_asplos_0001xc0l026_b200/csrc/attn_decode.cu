@@ -111,6 +111,9 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
   constexpr int GW = NCW / NG;
   constexpr int NS = 2 * NG;   // unit slots: each group holds <= 2 units (current + next)
   if (!gate_enter(a.L)) return;
+  if (threadIdx.x == 0 && a.L.trace) { trace_at(a.L, 0, smid()); trace_at(a.L, 1, gtimer()); }
+  pdl_wait();      // q and the new token's k / v come from the QKV GEMM
+  pdl_trigger();
   extern __shared__ __align__(128) uint8_t smem[];
   uint8_t* stages = smem;                                                      // [NCW][DEPTH][STAGE]
   uint8_t* qbuf = stages + NCW * DEPTH * STAGE_BYTES;                          // [NS_MAX][QSLOT_BYTES]
@@ -364,6 +367,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
     if (lane == 0) mbar_arrive(uqe + slot);
   }
   cp_async_wait<0>();
+  if (threadIdx.x == 0 && a.L.trace) trace_at(a.L, 5, gtimer());
 }
 
 size_t attn_decode_smem_bytes() {
@@ -389,11 +393,10 @@ cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStrea
     if (e != cudaSuccess) return e;
     set = true;
   }
-  if (ng == 1) k_attn_decode_tc<1><<<grid, THREADS, smem, st>>>(a);
-  else if (ng == 4 && NCW % 4 == 0) k_attn_decode_tc<4><<<grid, THREADS, smem, st>>>(a);
-  else if (ng == 3 && NCW % 3 == 0) k_attn_decode_tc<3><<<grid, THREADS, smem, st>>>(a);
-  else k_attn_decode_tc<2><<<grid, THREADS, smem, st>>>(a);
-  return cudaGetLastError();
+  if (ng == 1) return launch_ex(k_attn_decode_tc<1>, grid, THREADS, smem, st, a.L.pdl, a);
+  if (ng == 4 && NCW % 4 == 0) return launch_ex(k_attn_decode_tc<4>, grid, THREADS, smem, st, a.L.pdl, a);
+  if (ng == 3 && NCW % 3 == 0) return launch_ex(k_attn_decode_tc<3>, grid, THREADS, smem, st, a.L.pdl, a);
+  return launch_ex(k_attn_decode_tc<2>, grid, THREADS, smem, st, a.L.pdl, a);
 }
 
 cudaError_t preload_attn_decode() {

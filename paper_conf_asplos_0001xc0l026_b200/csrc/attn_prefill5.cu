@@ -211,6 +211,8 @@ __device__ __forceinline__ void load_kv_tile(uint8_t* dst, const __nv_bfloat16* 
 
 __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
   if (!gate_enter(a.L)) return;
+  pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
+  pdl_trigger();
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = smem_raw;
   if (smem_u32(sm) & 1023) __trap();   // swizzle atoms need 1024-byte alignment
@@ -501,8 +503,7 @@ cudaError_t launch_attn_prefill5(const AttnArgs& a, int grid, cudaStream_t st) {
     if (e != cudaSuccess) return e;
     set = true;
   }
-  k_attn_prefill5<<<grid, NT, SMEM_BYTES, st>>>(a);
-  return cudaGetLastError();
+  return launch_ex(k_attn_prefill5, grid, NT, SMEM_BYTES, st, a.L.pdl, a);
 }
 
 cudaError_t preload_attn_prefill5() {

@@ -20,6 +20,8 @@ constexpr int WARPS = 4;
 template <typename T, int HD, int HH>
 __global__ void __launch_bounds__(128) k_attn_simt(AttnArgs a) {
   if (!gate_enter(a.L)) return;
+  pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
+  pdl_trigger();
   constexpr int EPC = 16 / sizeof(T);           // elements per 16-byte chunk
   constexpr int CPR = HD / EPC;                 // chunks per key row
   constexpr int SWZ = (CPR < 16 ? CPR : 16) - 1;
@@ -214,7 +216,8 @@ static cudaError_t launch_one(const AttnArgs& a, int grid, cudaStream_t st) {
     if (e != cudaSuccess) return e;
     set = true;
   }
-  k_attn_simt<T, HD, HH><<<grid, 128, smem, st>>>(a);
+  cudaError_t e = launch_ex(k_attn_simt<T, HD, HH>, grid, 128, smem, st, a.L.pdl, a);
+  if (e != cudaSuccess) return e;
   return cudaGetLastError();
 }
 

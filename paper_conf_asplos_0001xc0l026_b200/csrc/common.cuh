@@ -29,7 +29,32 @@ struct Launch {
   int log_cap;
   int launch_id;
   int phase;
+  unsigned long long* trace;   // nullable (BULLET_TRACE): [grid][8] per-CTA timestamps, see trace_at
+  int pdl;                     // host: launched with programmatic stream serialization (launch_ex)
 };
+
+// Programmatic dependent launch (PDL).  Step kernels are launched so that
+// kernel i+1 may start as soon as every CTA of kernel i has passed
+// pdl_wait (its own predecessor is then complete) and triggered: its CTAs
+// take SMs as kernel i's CTAs leave them, run their prologue and stream the
+// static operands (weights) — and only then pdl_wait(), which returns once
+// kernel i has completed and its memory is visible.  Anything that reads a
+// predecessor's output, or writes memory a predecessor may still read, comes
+// after pdl_wait().  Without the launch attribute both are no-ops.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// Per-CTA trace record (BULLET_TRACE, diagnostics only): slot 0 smid,
+// 1 entry, 2 first MMA operand stage ready, 3 MMA issue done, 4 epilogue
+// done, 5 exit, 6 work units, 7 spare.  Written by one thread per slot.
+__device__ __forceinline__ void trace_at(const Launch& L, int slot, unsigned long long v) {
+  if (L.trace) L.trace[(size_t)(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 8 + slot] = v;
+}
 
 __device__ __forceinline__ uint32_t smid() {
   uint32_t r;

@@ -40,6 +40,8 @@ __device__ __forceinline__ void st2(__nv_bfloat16* p, float a, float b) {
 template <typename T, int VPT>
 __global__ void __launch_bounds__(256) k_rmsnorm(NormArgs a) {
   if (!gate_enter(a.L)) return;
+  pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
+  pdl_trigger();
   __shared__ int s_u;
   __shared__ float s_red[8];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -89,6 +91,8 @@ __global__ void __launch_bounds__(256) k_rmsnorm(NormArgs a) {
 template <typename T>
 __global__ void __launch_bounds__(256) k_rmsnorm_warp(NormArgs a) {
   if (!gate_enter(a.L)) return;
+  pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
+  pdl_trigger();
   const int lane = threadIdx.x & 31;
   const T* g = reinterpret_cast<const T*>(a.g);
   T* out = reinterpret_cast<T*>(a.out);
@@ -128,6 +132,8 @@ __global__ void __launch_bounds__(256) k_rmsnorm_warp(NormArgs a) {
 template <typename T>
 __global__ void __launch_bounds__(256) k_rope_kv(RopeArgs a) {
   if (!gate_enter(a.L)) return;
+  pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
+  pdl_trigger();
   __shared__ int s_u;
   const int tid = threadIdx.x;
   const int half = a.hd / 2, hp = half / 2;  // pair-of-pairs per head
@@ -173,6 +179,8 @@ template <typename T>
 __global__ void __launch_bounds__(256) k_gemm_simt(const T* __restrict__ A, const T* __restrict__ B,
                                                    GemmArgs a) {
   if (!gate_enter(a.L)) return;
+  pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
+  pdl_trigger();
   __shared__ float As[16][68], Bs[16][68], Us[16][68];
   __shared__ int s_u;
   const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
@@ -305,28 +313,31 @@ __global__ void k_probe(int* out, int n) {
 // ------------------------------------------------------------- launchers
 template <typename T>
 cudaError_t launch_gemm_simt(const T* A, const T* B, const GemmArgs& a, int grid, cudaStream_t st) {
-  k_gemm_simt<T><<<grid, 256, 0, st>>>(A, B, a);
+  cudaError_t e = launch_ex(k_gemm_simt<T>, grid, 256, 0, st, a.L.pdl, A, B, a);
+  if (e != cudaSuccess) return e;
   return cudaGetLastError();
 }
 template <typename T>
 cudaError_t launch_rmsnorm_warp(const NormArgs& a, int grid, cudaStream_t st) {
   if (a.d % 4) return cudaErrorInvalidValue;
-  k_rmsnorm_warp<T><<<grid, 256, 0, st>>>(a);
+  cudaError_t e = launch_ex(k_rmsnorm_warp<T>, grid, 256, 0, st, a.L.pdl, a);
+  if (e != cudaSuccess) return e;
   return cudaGetLastError();
 }
 template <typename T>
 cudaError_t launch_rmsnorm(const NormArgs& a, int grid, cudaStream_t st) {
   const int v = (a.d / 4 + 255) / 256;
-  if (v <= 1) k_rmsnorm<T, 1><<<grid, 256, 0, st>>>(a);
-  else if (v <= 2) k_rmsnorm<T, 2><<<grid, 256, 0, st>>>(a);
-  else if (v <= 4) k_rmsnorm<T, 4><<<grid, 256, 0, st>>>(a);
-  else if (v <= 8) k_rmsnorm<T, 8><<<grid, 256, 0, st>>>(a);
+  if (v <= 1) return launch_ex(k_rmsnorm<T, 1>, grid, 256, 0, st, a.L.pdl, a);
+  else if (v <= 2) return launch_ex(k_rmsnorm<T, 2>, grid, 256, 0, st, a.L.pdl, a);
+  else if (v <= 4) return launch_ex(k_rmsnorm<T, 4>, grid, 256, 0, st, a.L.pdl, a);
+  else if (v <= 8) return launch_ex(k_rmsnorm<T, 8>, grid, 256, 0, st, a.L.pdl, a);
   else return cudaErrorInvalidValue;
   return cudaGetLastError();
 }
 template <typename T>
 cudaError_t launch_rope_kv(const RopeArgs& a, int grid, cudaStream_t st) {
-  k_rope_kv<T><<<grid, 256, 0, st>>>(a);
+  cudaError_t e = launch_ex(k_rope_kv<T>, grid, 256, 0, st, a.L.pdl, a);
+  if (e != cudaSuccess) return e;
   return cudaGetLastError();
 }
 cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st) {

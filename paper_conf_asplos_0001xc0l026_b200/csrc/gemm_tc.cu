@@ -417,6 +417,7 @@ __global__ void __launch_bounds__(NT, 1)
     k_gemm_tc(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
               GemmArgs a, int n_stages) {
   if (!gate_enter(a.L)) return;  // not this phase's SM: touch nothing
+  if (threadIdx.x == 0 && a.L.trace) { trace_at(a.L, 0, smid()); trace_at(a.L, 1, gtimer()); }
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~uintptr_t(1023));
@@ -464,6 +465,7 @@ __global__ void __launch_bounds__(NT, 1)
       const uint64_t pol_a = policy_evict_last(), pol_b = a.b_evict_first ? policy_evict_first() : policy_evict_normal();
       int it = 0, s = 0;
       uint32_t ph = 0;
+      bool waited = false;
       for (;;) {
         const int slot = it & 3;
         mbar_wait(tqe + slot, ((it >> 2) & 1) ^ 1);
@@ -483,6 +485,11 @@ __global__ void __launch_bounds__(NT, 1)
         int r0, r1;
         if (a.epi == EPI_SILU) { r0 = n_blk * (bn / 2); r1 = a.silu_half + r0; }
         else { r0 = n_blk * bn; r1 = r0 + bn / 2; }
+        if (!waited) {   // activations are the predecessor's output (warp 3 streams weights meanwhile)
+          pdl_wait();
+          pdl_trigger();
+          waited = true;
+        }
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(empty + s, ph ^ 1);
           uint8_t* sa = smem + s * st_bytes;
@@ -560,6 +567,7 @@ __global__ void __launch_bounds__(NT, 1)
                              ((uint32_t)(BM >> 4) << 24);
       int it = 0, s = 0, as = 0;
       uint32_t ph = 0, aph = 0;
+      bool first = true;
       for (;;) {
         const int slot = it & 3;
         mbar_wait(tqf + slot, (it >> 2) & 1);
@@ -568,6 +576,7 @@ __global__ void __launch_bounds__(NT, 1)
         if (u < 0) break;
         const UnitInfo ui = unit_info(a, u);
         const int kb0 = ui.sp * k_blocks / ui.ns, kb1 = (ui.sp + 1) * k_blocks / ui.ns;
+        if (first && a.L.trace) { mbar_wait(full + s, ph); trace_at(a.L, 2, gtimer()); first = false; }
         mbar_wait(acce + as, aph ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tmem + as * acc_cols;
@@ -601,8 +610,10 @@ __global__ void __launch_bounds__(NT, 1)
         if (++as == n_acc) { as = 0; aph ^= 1; }
         ++it;
       }
+      if (a.L.trace) { trace_at(a.L, 3, gtimer()); trace_at(a.L, 6, it); }
     }
   } else if (warp >= 4) {  // ---------------- epilogue (warps 4..7 = TMEM lane quadrants 0..3)
+    pdl_wait();   // reads residual / bias / token table, writes outputs and partials
     const int et = threadIdx.x - 128, eq = warp & 3;
     int it = 0, as = 0;
     uint32_t aph = 0;
@@ -759,7 +770,9 @@ __global__ void __launch_bounds__(NT, 1)
       if (++as == n_acc) { as = 0; aph ^= 1; }
       ++it;
     }
+    if (et == 0 && a.L.trace) trace_at(a.L, 4, gtimer());
   }
+  pdl_wait();   // (no-op once passed) the tails below read and write predecessor-visible memory
   if (a.ar.n) {   // fused all-reduce: this CTA's GEMM units are done
     __syncthreads();
     ar_phase(a, s_last + 1);
@@ -779,6 +792,7 @@ __global__ void __launch_bounds__(NT, 1)
   }
   tc_fence_before();
   __syncthreads();
+  if (threadIdx.x == 0 && a.L.trace) trace_at(a.L, 5, gtimer());
   if (warp == 2) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
@@ -825,10 +839,10 @@ cudaError_t launch_gemm_tc(const CUtensorMap& mapA, const CUtensorMap& mapB, con
   if (a.mh < 1 || a.mh > 2 || a.splits < 1) return cudaErrorInvalidValue;
   if (a.kcb) {
     if (a.mh != 1 || a.bn != 128 || a.n_full != (a.M + BM - 1) / BM * (a.N / 128)) return cudaErrorInvalidValue;
-    k_gemm_tc<1, true><<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn, 1));
-  } else if (a.mh == 2) k_gemm_tc<2><<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn, 2));
-  else k_gemm_tc<1><<<grid, NT, smem, st>>>(mapA, mapB, a, gemm_tc_stages(a.bn, 1));
-  return cudaGetLastError();
+    return launch_ex(k_gemm_tc<1, true>, grid, NT, smem, st, a.L.pdl, mapA, mapB, a, gemm_tc_stages(a.bn, 1));
+  }
+  if (a.mh == 2) return launch_ex(k_gemm_tc<2>, grid, NT, smem, st, a.L.pdl, mapA, mapB, a, gemm_tc_stages(a.bn, 2));
+  return launch_ex(k_gemm_tc<1>, grid, NT, smem, st, a.L.pdl, mapA, mapB, a, gemm_tc_stages(a.bn, 1));
 }
 
 cudaError_t preload_gemm_tc() {

@@ -1,6 +1,7 @@
 // kernels.h — argument structs and launchers of the Bullet sm_100a kernels.
 #pragma once
 #include "common.cuh"
+#include <utility>
 
 namespace bl {
 
@@ -139,6 +140,21 @@ struct PlanArgs {
   // decode attention's units (the longest rows start first, the tail is short)
   int4* order; int order_base;
 };
+
+// Launch helper: `pdl` = programmatic stream serialization (common.cuh
+// pdl_wait / pdl_trigger) so the kernel may start while its predecessor on
+// the stream drains.
+template <typename... P, typename... A>
+inline cudaError_t launch_ex(void (*k)(P...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, bool pdl,
+                             A&&... args) {
+  cudaLaunchConfig_t c = {};
+  c.gridDim = grid; c.blockDim = block; c.dynamicSmemBytes = smem; c.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  c.attrs = at; c.numAttrs = pdl ? 1 : 0;
+  return cudaLaunchKernelEx(&c, k, std::forward<A>(args)...);
+}
 
 // launchers (return cudaError_t of the launch)
 cudaError_t launch_gemm_tc(const CUtensorMap& mapA, const CUtensorMap& mapB, const GemmArgs& a,

@@ -288,8 +288,11 @@ def test_attention_vs_oracle(B, m, kind):
                                      h // grp, cl + i)
                 g = got[row, h * hd:(h + 1) * hd].astype(np.float64)
                 worst = max(worst, float(np.abs(g - ref).max()))
-                if m.dtype == "bf16":   # error in units of the bf16 spacing at |ref| (2^-7 |ref| >= 1 ulp)
-                    ulps = max(ulps, float((np.abs(g - ref) / (np.abs(ref) * 2.0 ** -7 + 1e-12)).max()))
+                if m.dtype == "bf16":
+                    # error in units of the bf16 spacing at |ref| (2^-7 |ref| >= 1 ulp), with an
+                    # absolute floor for outputs that cancel to ~0: fp32 sums of p_j v_j carry
+                    # ~1e-7 sum_j p_j |v_j| and P = hi + lo leaves 2^-16 of it (R-4b)
+                    ulps = max(ulps, float((np.abs(g - ref) / (np.abs(ref) * 2.0 ** -7 + 5e-5)).max()))
                     rr = O.round_bf16(ref)   # R3: the oracle's own bf16 rounding of o
                     err_l1 += float(np.abs(g - rr).sum()); ref_l1 += float(np.abs(rr).sum())
             row += 1
@@ -298,6 +301,5 @@ def test_attention_vs_oracle(B, m, kind):
         # o = RNE(exact + fp32 noise): within one bf16 spacing of the exact
         # value everywhere, and equal to the oracle's R3-rounded o except
         # where the noise straddles a rounding boundary (mean-rel vs that)
-        assert ulps <= 1.0, ulps
-        assert err_l1 / ref_l1 <= 2e-4, err_l1 / ref_l1
+        assert ulps <= 1.0 and err_l1 / ref_l1 <= 2e-4, (ulps, err_l1 / ref_l1)
 
