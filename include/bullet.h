@@ -180,7 +180,12 @@ typedef struct {
   double percentile;             /* 0.9 (Alg. 1 "P90") */
   int objective;                 /* 0: Alg. 1 as read (DESIGN R-14..R-17); 1: when both SLOs hold,
                                     the split with the most predicted tokens/s among the SLO-feasible
-                                    ones instead of the fewest decode SMs (R-21) */
+                                    ones instead of the fewest decode SMs, or the time-sliced cycle
+                                    if it beats them (R-21, R-22); 2: when both SLOs hold, the
+                                    SLO-feasible split and decode layer-steps k with the largest
+                                    predicted gain of the co-run cycle over the same work
+                                    time-sliced, or the time-sliced cycle (prefill_sm_count = N,
+                                    k > 0) when no split gains (R-23) */
 } bullet_slo;
 
 /* Create a handle on the current CUDA device.  Probes the live SM ids

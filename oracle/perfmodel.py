@@ -242,7 +242,42 @@ def choose_split(P, model, state, slo, gran=2):
             return 0, -1.0
         return k, (float(sum(state["prefill_lens"])) + len(state["decode_tokens"]) * k) / cyc
 
-    if ok_t and ok_d and slo.get("objective", 0) == 1:
+    def max_gain():
+        # R-23 (objective 2): among SLO-feasible splits and k in {floor(r),
+        # floor(r) + 1}, r = t_p / t_d (k >= 1), the largest predicted gain
+        # (t_p(N) + k t_d(N)) / max(t_p(u), k t_d(v)) of co-running the cycle
+        # over time-slicing the same work; ties: larger gain, then larger
+        # prefill share (smaller v), then smaller k
+        pre = _phase_shape(model, list(state["prefill_lens"]), [0] * len(state["prefill_lens"]))
+        dec = _phase_shape(model, [1] * len(state["decode_tokens"]),
+                           [int(math.floor(state["decode_mean_ctx"] + 0.5))] * len(state["decode_tokens"]))
+        tpN = layer_time(pre, P, N, 0) * 1e3 if state["prefill_lens"] else 0.0
+        tdN = layer_time(dec, P, N, 0) * 1e3
+        best, best_g = (None, 1), -1.0
+        for v in cands:
+            if ev[v][0] > 1.0 or ev[v][1] > 1.0:
+                continue
+            t_p, t_d = ev[v][2], layer_time(dec, P, v, N - v) * 1e3
+            if t_d <= 0:
+                continue
+            k0 = max(1, int(math.floor(t_p / t_d)))
+            for k in (k0, k0 + 1):
+                g = (tpN + k * tdN) / max(t_p, k * t_d)
+                if g > best_g:
+                    best, best_g = (v, k), g
+        return best, best_g
+
+    if ok_t and ok_d and slo.get("objective", 0) == 2:
+        (vb, kb), g = max_gain()
+        if vb is not None and g > 1.0:
+            return N - vb, kb
+        k_ts, _ = timesliced()
+        if k_ts > 0:
+            return N, k_ts                             # co-running does not pay: time-sliced cycle
+        if vb is not None:
+            return N - vb, kb
+        v = reduce_decode()
+    elif ok_t and ok_d and slo.get("objective", 0) == 1:
         vb, t_co = max_throughput_t()                  # R-21
         k_ts, t_ts = timesliced()                      # R-22
         if k_ts > 0 and t_ts > t_co:

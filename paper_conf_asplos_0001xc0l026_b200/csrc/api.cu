@@ -380,7 +380,7 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   }
   if (h->cfg.dtype == BULLET_DTYPE_FP32) {
     if (K % 16) return set_err(BULLET_EUNSUPPORTED, "fp32 GEMM needs K %% 16 == 0");
-    a.bn = 64; a.mh = 1; a.splits = 1; a.n_full = 0; a.band = 1;
+    a.bn = 64; a.mh = 1; a.n_full = 0; a.band = 1;
     LAUNCH(c, launch_gemm_simt<float>((const float*)A, (const float*)B, a, h->n_sms * 4, c.st));
     return BULLET_OK;
   }
@@ -391,19 +391,20 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
     if (epi == EPI_QKV) return bn % 128 == 0 && N % bn == 0;   // tiles hold whole heads
     return epi == EPI_SILU ? ((N / 2) % (bn / 2) == 0 && N % 2 == 0) : (N % bn == 0);
   };
-  // Plan (mh, bn, tail split) on the phase's m SMs.  A tile costs
-  // max(bytes streamed / per-SM copy bandwidth, MMA flops / per-SM tensor
-  // rate) plus a fixed pipeline fill (at M >= 256 decode GEMMs are
-  // compute-bound per SM; at M <= 128 the weight stream binds).  Tiles fill
-  // full waves of m SMs; the ragged remainder may be split `ts` ways over K,
-  // paying an fp32 partial round trip: the writes, then the last unit's
-  // latency-bound sum (one ~1.3 us round trip per 2 splits x 32 columns).
-  // A single accumulator stage
-  // (mh * bn > 256 columns) exposes the epilogue.  mh = 2 only for
-  // decode-sized M.  Rates: KI2.
-  constexpr double BW_SM = 90e9, FL_SM = 10.5e12, EPI_BW = 100e9, RTT = 1.3e-6, T0 = 0.6e-6;
+  // Plan (mh, bn, work split) on the phase's m SMs.  A k-block step of a
+  // tile costs max(bytes streamed / per-SM copy bandwidth, MMA flops / per-SM
+  // tensor rate); whole tiles fill full waves of the partition; the ragged
+  // remainder (for decode-sized GEMMs: every tile) is either run as whole
+  // tiles (a partly idle last wave) or streamed over K in m equal ranges
+  // (stream-K: every SM streams the same k-blocks, partial tiles pay an fp32
+  // partial round trip and a fixup that reads the tile's other segments
+  // through one SM).  A single accumulator stage (mh * bn > 256 columns)
+  // exposes the epilogue.  mh = 2 only for decode-sized M.  Rates: KI2 and
+  // the per-CTA traces.
+  constexpr double BW_SM = 110e9, FL_SM = 10.5e12, EPI_BW = 100e9, RTT = 1.0e-6, T0 = 0.6e-6;
   const int k_blocks = K / 64;
-  int mh = 1, bn = 0, ts = 1, n_full = 0;
+  const size_t pf = h->ph[c.phase].partial_floats;
+  int mh = 1, bn = 0, n_full = 0, sk_tiles = 0, sk_chunks = 0;
   double best = 1e300;
   for (int cmh = (M > 128 && M <= 512) ? 2 : 1; cmh >= 1; --cmh) {
     const int m_tiles = (M + 128 * cmh - 1) / (128 * cmh);
@@ -411,24 +412,19 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
       if (!fits(cand)) continue;
       const int tiles = m_tiles * (N / cand);
       const double out_b = 128.0 * cmh * cand * 4.0;
-      const double t_tile = std::max((double)k_blocks * (cmh * 16384.0 + cand * 128.0) / BW_SM,
-                                     2.0 * 128 * cmh * cand * K / FL_SM) +
-                            (2 * cmh * cand > 512 ? out_b / EPI_BW : 0.0) + T0;
-      const int full_waves = tiles / c.m_sms, rem = tiles % c.m_sms;
-      const int max_ts = rem ? std::max(1, std::min(16, k_blocks / 4)) : 1;
-      for (int cts = 1; cts <= max_ts; ++cts) {
-        if (cts > 1 && ((size_t)rem * cts * 128 * cmh * cand > h->ph[c.phase].partial_floats || rem > N_TILE_SEMS))
-          break;
-        const double tail = rem == 0 ? 0.0
-                            : cts == 1 ? t_tile
-                                       : std::ceil((double)rem * cts / c.m_sms) *
-                                                 ((t_tile - T0) / cts + T0 + out_b / EPI_BW) +
-                                             std::ceil(cts / 2.0) * (cmh * cand / 32) * RTT;
-        const double cost = full_waves * t_tile + tail;
-        if (cost < best * 0.999) {
-          best = cost; mh = cmh; bn = cand; ts = cts;
-          n_full = cts > 1 ? tiles - rem : tiles;
-        }
+      const double t_kb = std::max((cmh * 16384.0 + cand * 128.0) / BW_SM, 2.0 * 128 * cmh * cand * 64 / FL_SM);
+      const double t_tile = k_blocks * t_kb + (2 * cmh * cand > 512 ? out_b / EPI_BW : 0.0) + T0;
+      const double cost_a = std::ceil((double)tiles / c.m_sms) * t_tile;   // whole tiles only
+      if (cost_a < best * 0.999) { best = cost_a; mh = cmh; bn = cand; n_full = tiles; sk_tiles = 0; sk_chunks = 0; }
+      const int fw = tiles / c.m_sms, rem = tiles % c.m_sms;
+      if (rem == 0) continue;
+      const int chunks = std::min(c.m_sms, rem * k_blocks);
+      if ((size_t)2 * chunks * 128 * cmh * cand > pf || rem > N_TILE_SEMS) continue;
+      const double segs = std::ceil((double)chunks / rem) + 1.0;   // segments per streamed tile
+      const double cost_b = fw * t_tile + (double)rem * k_blocks / chunks * t_kb + T0 +
+                            (segs - 1.0) * out_b / BW_SM + out_b / EPI_BW + 2 * RTT;
+      if (cost_b < best * 0.999) {
+        best = cost_b; mh = cmh; bn = cand; n_full = fw * c.m_sms; sk_tiles = rem; sk_chunks = chunks;
       }
     }
   }
@@ -437,12 +433,14 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   snprintf(kenv, sizeof kenv, "BULLET_GEMM_PLAN_K%d", c.kind);   // per kernel kind (experiments)
   const char* ov = getenv(kenv);
   if (!ov) ov = getenv("BULLET_GEMM_PLAN");
-  if (ov) {   // experiments: "mh,bn,ts"
-    int omh = 0, obn = 0, ots = 0;
-    if (sscanf(ov, "%d,%d,%d", &omh, &obn, &ots) == 3 && fits(obn) && omh >= 1 && omh <= 2 && ots >= 1) {
+  if (ov) {   // experiments: "mh,bn,sk" (sk 1: stream the ragged remainder over K)
+    int omh = 0, obn = 0, osk = 0;
+    if (sscanf(ov, "%d,%d,%d", &omh, &obn, &osk) == 3 && fits(obn) && omh >= 1 && omh <= 2) {
       const int tiles = ((M + 128 * omh - 1) / (128 * omh)) * (N / obn), rem = tiles % c.m_sms;
-      if (ots == 1 || (rem && (size_t)rem * ots * 128 * omh * obn <= h->ph[c.phase].partial_floats)) {
-        mh = omh; bn = obn; ts = ots; n_full = (ts > 1) ? tiles - rem : tiles;
+      const int chunks = std::min(c.m_sms, rem * k_blocks);
+      if (!osk || !rem) { mh = omh; bn = obn; n_full = tiles; sk_tiles = 0; sk_chunks = 0; }
+      else if ((size_t)2 * chunks * 128 * omh * obn <= pf && rem <= N_TILE_SEMS) {
+        mh = omh; bn = obn; n_full = tiles - rem; sk_tiles = rem; sk_chunks = chunks;
       }
     }
   }
@@ -462,27 +460,29 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
     const bool sel = kind >= 0 ? ((kp.mask >> kind) & 1u) != 0 : kp.mask == KC_ALL;
     if (kc >= 64 && K > kc && sel) {
       bool done = false;
-      if (kp.splitk) {
+      const int kcb_ = std::max(1, kc / 64);
+      if (kp.splitk) {   // every tile's K range streamed in ranges of <= kc, summed by the fixup
         const int tiles = ((M + 128 * mh - 1) / (128 * mh)) * (N / bn);
-        const size_t per = (size_t)tiles * 128 * mh * bn;
-        const int want = std::min((K + kc - 1) / kc, k_blocks);
-        const size_t cap = h->ph[c.phase].partial_floats / per;
-        // every chunk must get its own split: when the partials do not fit
+        const long long Ts = (long long)tiles * k_blocks;
+        const int chunks = (int)((Ts + kcb_ - 1) / kcb_);
+        // every range must get its own partial: when they do not fit
         // (prefill-sized M) fall through to the on-chip mode instead of
-        // silently running fewer, longer chunks
-        if ((size_t)want <= cap && tiles <= N_TILE_SEMS) { ts = want; n_full = 0; done = true; }
+        // silently running fewer, longer ranges
+        if ((size_t)2 * chunks * 128 * mh * bn <= h->ph[c.phase].partial_floats && tiles <= N_TILE_SEMS) {
+          n_full = 0; sk_tiles = tiles; sk_chunks = chunks; done = true;
+        }
       }
       if (!done && fits(128)) {
-        mh = 1; bn = 128; ts = 1;
+        mh = 1; bn = 128; sk_tiles = 0; sk_chunks = 0;
         n_full = ((M + 127) / 128) * (N / 128);
-        kcb = std::max(1, kc / 64);
+        kcb = kcb_;
       }
     }
   }
   if (getenv("BULLET_GEMM_DEBUG"))
-    fprintf(stderr, "gemm M=%d N=%d K=%d m_sms=%d -> mh=%d bn=%d n_full=%d kcb=%d ts=%d\n", M, N, K, c.m_sms, mh, bn,
-            n_full, kcb, ts);
-  a.bn = bn; a.mh = mh; a.splits = ts; a.n_full = n_full; a.kcb = kcb;
+    fprintf(stderr, "gemm M=%d N=%d K=%d m_sms=%d -> mh=%d bn=%d n_full=%d sk_tiles=%d sk_chunks=%d kcb=%d\n", M, N,
+            K, c.m_sms, mh, bn, n_full, sk_tiles, sk_chunks, kcb);
+  a.bn = bn; a.mh = mh; a.n_full = n_full; a.sk_tiles = sk_tiles; a.sk_chunks = sk_chunks; a.kcb = kcb;
   {   // second copy issuer for the weight tiles (BULLET_GEMM_SPLIT_B=0/1 overrides; default: on)
     static const int sb = getenv("BULLET_GEMM_SPLIT_B") ? atoi(getenv("BULLET_GEMM_SPLIT_B")) : 1;
     a.split_b = sb ? 1 : 0;
@@ -1195,7 +1195,7 @@ int bullet_choose_split(const bullet_handle* h, const bullet_sched_state* s, con
   for (int i = 0; i < s->n_decode; ++i) { S.decode_tokens.push_back(s->decode_tokens[i]); S.decode_elapsed_ms.push_back(s->decode_elapsed_ms[i]); }
   S.decode_mean_ctx = s->decode_mean_ctx;
   S.u_k = s->u_k; S.v_k = s->v_k;
-  if (slo->objective < 0 || slo->objective > 1) return set_err(BULLET_EINVAL, "slo objective");
+  if (slo->objective < 0 || slo->objective > 2) return set_err(BULLET_EINVAL, "slo objective");
   Slo sl{slo->ttft_norm_ms_per_tok, slo->tpot_ms, slo->w_max, slo->v_min, slo->percentile, slo->objective};
   PerfParams P = h->perf;
   P.M = h->n_sms;

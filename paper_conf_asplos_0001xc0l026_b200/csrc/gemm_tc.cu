@@ -16,11 +16,12 @@
 // mh = 2 (decode-sized M <= 512): a unit covers 256 rows with two M=128
 // accumulators that share every B stage, so weights stream through an SM
 // once per 256 rows instead of once per 128.
-// Tail split: units [0, n_full) are whole tiles; each remaining tile (the
-// ragged last wave) is split `splits` ways over K so that wave fills the
-// partition.  A split unit writes an fp32 partial; the last unit of its tile
-// (atomic ticket) sums the partials in split order (deterministic) and runs
-// the epilogue.
+// Work: units [0, n_full) are whole tiles; the remaining tiles (the ragged
+// last wave, or all tiles of a decode-sized GEMM) are streamed over K in
+// equal ranges (stream-K, see Seg below) so every SM of the partition
+// streams the same number of k-blocks.  Partial segments write fp32
+// partials; the tile's last segment (atomic ticket) sums them in k order
+// (deterministic) and runs the epilogue.
 #include "kernels.h"
 
 namespace bl {
@@ -42,18 +43,27 @@ __device__ __forceinline__ void tile_coords(int tile, int m_tiles, int n_tiles, 
   m_blk = b * band + r % rows;
   n_blk = r / rows;
 }
-struct UnitInfo {
-  int tile, sp, ns, tail;   // tail: index among split units (partials slot), -1 for whole tiles
+// ---------------------------------------------------------------- work decomposition
+// Units [0, n_full) are whole tiles (rasterised by tile_coords).  The other
+// sk_tiles tiles (the ragged remainder, or every tile of a decode-sized
+// GEMM) are streamed: their sk_tiles * k_blocks k-block iterations are cut
+// into sk_chunks equal ranges ("stream-K"), unit n_full + c = range c.  A
+// range covers the pieces ("segments") of the tiles it overlaps; a segment
+// covering a whole tile runs the epilogue itself, the others store an fp32
+// partial in slot 2c (the range's first segment) or 2c + 1 (its last) and
+// the tile's last-arriving segment sums the partials in k order
+// (deterministic) and runs the epilogue.  So a GEMM with fewer tiles than
+// SMs still keeps every SM streaming the same number of k-blocks.
+struct Seg {   // one entry of the CTA's work queue
+  int tile, kb0, kb1, slot;   // slot: partial slot, -1 = whole tile (direct epilogue); tile -1 = end
 };
-__device__ __forceinline__ UnitInfo unit_info(const GemmArgs& a, int u) {
-  UnitInfo r;
-  if (u < a.n_full) {
-    r.tile = u; r.sp = 0; r.ns = 1; r.tail = -1;
-  } else {
-    const int t = u - a.n_full;
-    r.tile = a.n_full + t / a.splits; r.sp = t % a.splits; r.ns = a.splits; r.tail = t;
-  }
-  return r;
+__device__ __forceinline__ int sk_bound(const GemmArgs& a, int k_blocks, int c) {
+  return (int)((long long)c * a.sk_tiles * k_blocks / a.sk_chunks);
+}
+// chunk holding stream iteration x (the largest c with sk_bound(c) <= x)
+__device__ __forceinline__ int sk_chunk_of(const GemmArgs& a, int k_blocks, int x) {
+  const long long Ts = (long long)a.sk_tiles * k_blocks;
+  return (int)(((long long)(x + 1) * a.sk_chunks - 1) / Ts);
 }
 
 __device__ __forceinline__ uint64_t sw128_desc(uint32_t addr) {
@@ -432,14 +442,14 @@ __global__ void __launch_bounds__(NT, 1)
   uint64_t* acce = accf + 2;
   uint64_t* tqf = acce + 2;
   uint64_t* tqe = tqf + 4;
-  int* tile_q = reinterpret_cast<int*>(tqe + 4);
+  Seg* tile_q = reinterpret_cast<Seg*>(tqe + 4);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tile_q + 4);
   int* s_last = reinterpret_cast<int*>(tmem_slot + 1);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int m_tiles = (a.M + BM * mh - 1) / (BM * mh);
   const int n_tiles = a.N / bn;
-  const int units = a.n_full + (m_tiles * n_tiles - a.n_full) * a.splits;
+  const int units = a.n_full + (a.sk_tiles ? a.sk_chunks : 0);
   const int k_blocks = a.K / BK;
 
   if (threadIdx.x == 0) {
@@ -460,37 +470,36 @@ __global__ void __launch_bounds__(NT, 1)
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
 
+  // B rows of tile column n_blk (SiLU tiles take bn/2 gate rows and the
+  // matching bn/2 up rows)
+  auto b_rows_of = [&](int n_blk, int& r0, int& r1) {
+    if (a.epi == EPI_SILU) { r0 = n_blk * (bn / 2); r1 = a.silu_half + r0; }
+    else { r0 = n_blk * bn; r1 = r0 + bn / 2; }
+  };
+
   if (warp == 0) {
     if (lane == 0) {  // ---------------- scheduler + TMA producer
       const uint64_t pol_a = policy_evict_last(), pol_b = a.b_evict_first ? policy_evict_first() : policy_evict_normal();
       int it = 0, s = 0;
       uint32_t ph = 0;
       bool waited = false;
-      for (;;) {
+      // publish one queue entry and stream its operands
+      auto issue = [&](const Seg& g) {
         const int slot = it & 3;
         mbar_wait(tqe + slot, ((it >> 2) & 1) ^ 1);
-        // claim just in time: only once a smem stage is free to load into, so
-        // early CTAs cannot hoard units while others idle (load balance)
-        mbar_wait(empty + s, ph ^ 1);
-        int u = atomicAdd(a.L.ctr, 1);
-        if (u >= units) u = -1;
-        tile_q[slot] = u;
+        tile_q[slot] = g;
         mbar_arrive(tqf + slot);
-        if (u < 0) break;
-        log_unit(a.L, u);
-        const UnitInfo ui = unit_info(a, u);
-        int m_blk, n_blk;
-        tile_coords(ui.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
-        const int kb0 = ui.sp * k_blocks / ui.ns, kb1 = (ui.sp + 1) * k_blocks / ui.ns;
-        int r0, r1;
-        if (a.epi == EPI_SILU) { r0 = n_blk * (bn / 2); r1 = a.silu_half + r0; }
-        else { r0 = n_blk * bn; r1 = r0 + bn / 2; }
+        ++it;
+        if (g.tile < 0) return;
+        int m_blk, n_blk, r0, r1;
+        tile_coords(g.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
+        b_rows_of(n_blk, r0, r1);
         if (!waited) {   // activations are the predecessor's output (warp 3 streams weights meanwhile)
           pdl_wait();
           pdl_trigger();
           waited = true;
         }
-        for (int kb = kb0; kb < kb1; ++kb) {
+        for (int kb = g.kb0; kb < g.kb1; ++kb) {
           mbar_wait(empty + s, ph ^ 1);
           uint8_t* sa = smem + s * st_bytes;
           mbar_arrive_expect_tx(full + s, a.split_b ? a_bytes : st_bytes);
@@ -498,23 +507,40 @@ __global__ void __launch_bounds__(NT, 1)
           for (int hh = 0; hh < mh; ++hh)   // rows past M are zero-filled by TMA
             tma_load_2d_hint(sa + hh * A_BYTES, &mapA, full + s, kb * BK, (m_blk * mh + hh) * BM, pol_a);
           uint8_t* sb = sa + a_bytes;
-          if (a.split_b) {
-            // B comes from warp 3's issuer
-          } else if (a.b_packed) {   // pre-swizzled tiles: contiguous bulk copies
-            const uint8_t* kbase = a.b_packed + (size_t)kb * (a.b_rows / 64) * 8192;
-            if (r1 == r0 + bn / 2) {
-              bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s, pol_b);
+          if (!a.split_b) {   // (else B comes from warp 3's issuer)
+            if (a.b_packed) {
+              const uint8_t* kbase = a.b_packed + (size_t)kb * (a.b_rows / 64) * 8192;
+              if (r1 == r0 + bn / 2) {
+                bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s, pol_b);
+              } else {
+                bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes / 2, full + s, pol_b);
+                bulk_g2s(sb + b_bytes / 2, kbase + (size_t)(r1 / 64) * 8192, b_bytes / 2, full + s, pol_b);
+              }
             } else {
-              bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes / 2, full + s, pol_b);
-              bulk_g2s(sb + b_bytes / 2, kbase + (size_t)(r1 / 64) * 8192, b_bytes / 2, full + s, pol_b);
+              tma_load_2d_hint(sb, &mapB, full + s, kb * BK, r0, pol_b);
+              tma_load_2d_hint(sb + b_bytes / 2, &mapB, full + s, kb * BK, r1, pol_b);
             }
-          } else {
-            tma_load_2d_hint(sb, &mapB, full + s, kb * BK, r0, pol_b);
-            tma_load_2d_hint(sb + b_bytes / 2, &mapB, full + s, kb * BK, r1, pol_b);
           }
           if (++s == n_stages) { s = 0; ph ^= 1; }
         }
-        ++it;
+      };
+      for (;;) {
+        // claim just in time: only once a smem stage is free to load into, so
+        // early CTAs cannot hoard units while others idle (load balance)
+        mbar_wait(empty + s, ph ^ 1);
+        const int u = atomicAdd(a.L.ctr, 1);
+        if (u >= units) { issue(Seg{-1, 0, 0, -1}); break; }
+        log_unit(a.L, u);
+        if (u < a.n_full) { issue(Seg{u, 0, k_blocks, -1}); continue; }
+        const int c = u - a.n_full;   // stream range c: its segments in k order
+        const int xb = sk_bound(a, k_blocks, c), xe = sk_bound(a, k_blocks, c + 1);
+        for (int x = xb; x < xe;) {
+          const int t = x / k_blocks, k0 = x - t * k_blocks, se = min(xe, (t + 1) * k_blocks);
+          const int k1 = se - t * k_blocks;
+          const bool whole = k0 == 0 && k1 == k_blocks;
+          issue(Seg{a.n_full + t, k0, k1, whole ? -1 : (x == xb ? 2 * c : 2 * c + 1)});
+          x = se;
+        }
       }
     }
   } else if (warp == 3) {
@@ -522,25 +548,23 @@ __global__ void __launch_bounds__(NT, 1)
       // one thread's issue loop (wait for a free stage, arm, issue) caps the
       // copy stream it can keep in flight; a second issuing thread for the
       // weight operand lifts the per-SM ceiling (KI2: 99 -> 123 GB/s/SM,
-      // profiles/r01c_ki2_issuers.jsonl).  Same unit / k-block / stage
+      // profiles/r01c_ki2_issuers.jsonl).  Same entry / k-block / stage
       // sequence as warp 0, its own arrival on each full barrier (count 2).
+      // Weights are static: no dependency on the predecessor kernel.
       const uint64_t pol_b = a.b_evict_first ? policy_evict_first() : policy_evict_normal();
       int it = 0, s = 0;
       uint32_t ph = 0;
       for (;;) {
         const int slot = it & 3;
         mbar_wait(tqf + slot, (it >> 2) & 1);
-        const int u = tile_q[slot];
+        const Seg g = tile_q[slot];
         mbar_arrive(tqe + slot);
-        if (u < 0) break;
-        const UnitInfo ui = unit_info(a, u);
-        int m_blk, n_blk;
-        tile_coords(ui.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
-        const int kb0 = ui.sp * k_blocks / ui.ns, kb1 = (ui.sp + 1) * k_blocks / ui.ns;
-        int r0, r1;
-        if (a.epi == EPI_SILU) { r0 = n_blk * (bn / 2); r1 = a.silu_half + r0; }
-        else { r0 = n_blk * bn; r1 = r0 + bn / 2; }
-        for (int kb = kb0; kb < kb1; ++kb) {
+        ++it;
+        if (g.tile < 0) break;
+        int m_blk, n_blk, r0, r1;
+        tile_coords(g.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
+        b_rows_of(n_blk, r0, r1);
+        for (int kb = g.kb0; kb < g.kb1; ++kb) {
           mbar_wait(empty + s, ph ^ 1);
           uint8_t* sb = smem + s * st_bytes + a_bytes;
           mbar_arrive_expect_tx(full + s, b_bytes);
@@ -558,7 +582,6 @@ __global__ void __launch_bounds__(NT, 1)
           }
           if (++s == n_stages) { s = 0; ph ^= 1; }
         }
-        ++it;
       }
     }
   } else if (warp == 1) {
@@ -571,11 +594,10 @@ __global__ void __launch_bounds__(NT, 1)
       for (;;) {
         const int slot = it & 3;
         mbar_wait(tqf + slot, (it >> 2) & 1);
-        const int u = tile_q[slot];
+        const Seg g = tile_q[slot];
         mbar_arrive(tqe + slot);
-        if (u < 0) break;
-        const UnitInfo ui = unit_info(a, u);
-        const int kb0 = ui.sp * k_blocks / ui.ns, kb1 = (ui.sp + 1) * k_blocks / ui.ns;
+        if (g.tile < 0) break;
+        const int kb0 = g.kb0, kb1 = g.kb1;
         if (first && a.L.trace) { mbar_wait(full + s, ph); trace_at(a.L, 2, gtimer()); first = false; }
         mbar_wait(acce + as, aph ^ 1);
         tc_fence_after();
@@ -621,13 +643,12 @@ __global__ void __launch_bounds__(NT, 1)
     for (;;) {
       const int slot = it & 3;
       mbar_wait(tqf + slot, (it >> 2) & 1);
-      const int u = tile_q[slot];
+      const Seg g = tile_q[slot];
       __syncwarp();
       if (lane == 0) mbar_arrive(tqe + slot);
-      if (u < 0) break;
-      const UnitInfo ui = unit_info(a, u);
+      if (g.tile < 0) break;
       int m_blk, n_blk;
-      tile_coords(ui.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
+      tile_coords(g.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
       const int col0 = (a.epi == EPI_SILU) ? n_blk * (bn / 2) : n_blk * bn;
       const int out_chunks = (a.epi == EPI_SILU) ? bn / 64 : bn / 32;
       if constexpr (KC) {   // mh == 1, bn == 128, whole tiles (plan guarantees)
@@ -669,7 +690,7 @@ __global__ void __launch_bounds__(NT, 1)
       mbar_wait(accf + as, aph);
       tc_fence_after();
       const uint32_t tb = tmem + ((uint32_t)(eq * 32) << 16) + as * acc_cols;
-      if (ui.ns == 1) {
+      if (g.slot < 0) {   // whole tile: epilogue straight from TMEM
         for (int hh = 0; hh < mh; ++hh) {
           const int m = (m_blk * mh + hh) * BM + et;
           if (a.epi == EPI_QKV) {   // per head: column chunks (c, c + 2) are rotate-half partners
@@ -698,7 +719,7 @@ __global__ void __launch_bounds__(NT, 1)
         // float4 and a warp's 32 rows are 512 contiguous bytes, so stores
         // and the fixup's loads are vectorised and coalesced
         const size_t tile_f4 = (size_t)mh * BM * bn / 4;
-        float4* P = reinterpret_cast<float4*>(a.partials) + (size_t)ui.tail * tile_f4 + et;
+        float4* P = reinterpret_cast<float4*>(a.partials) + (size_t)g.slot * tile_f4 + et;
         for (int hh = 0; hh < mh; ++hh)
           for (int c = 0; c < bn / 32; ++c) {
             tmem_ld32(tb + hh * bn + c * 32, v);
@@ -710,44 +731,57 @@ __global__ void __launch_bounds__(NT, 1)
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(acce + as);
+        // the tile's segments: stream ranges c_lo .. c_hi (non-empty ones), in k order
+        const int st_idx = g.tile - a.n_full;
+        const int x0 = st_idx * k_blocks, x1 = x0 + k_blocks - 1;
+        const int c_lo = sk_chunk_of(a, k_blocks, x0), c_hi = sk_chunk_of(a, k_blocks, x1);
+        int nseg = 0;
+        for (int c = c_lo; c <= c_hi; ++c) nseg += sk_bound(a, k_blocks, c + 1) > sk_bound(a, k_blocks, c);
         __threadfence();
         named_bar_sync(1, 128);
-        const int sem = ui.tile - a.n_full;
         if (et == 0) {
-          const int old = atomicAdd(a.tile_sems + sem, 1);
-          const int last = (old == ui.ns - 1);
-          if (last) a.tile_sems[sem] = 0;  // self-reset for the next launch
+          const int old = atomicAdd(a.tile_sems + st_idx, 1);
+          const int last = (old == nseg - 1);
+          if (last) a.tile_sems[st_idx] = 0;  // self-reset for the next launch
           *s_last = last;
         }
         named_bar_sync(1, 128);
         const bool last = *s_last;
         if (last) {
           __threadfence();
-          const float4* T0 = reinterpret_cast<const float4*>(a.partials) + (size_t)(ui.tail - ui.sp) * tile_f4 + et;
-          // sum 32 columns of all splits (fixed split order: deterministic),
-          // two splits per batch so 16 float4 loads are in flight per thread
-          auto sum32 = [&](const float4* base, float* acc) {
+          const float4* T0 = reinterpret_cast<const float4*>(a.partials) + et;
+          // sum 32 columns over the tile's segments (k order: deterministic),
+          // two segments per batch so 16 float4 loads are in flight per thread
+          auto sum32 = [&](size_t off, float* acc) {
 #pragma unroll
             for (int i = 0; i < 32; ++i) acc[i] = 0.f;
-            for (int sp = 0; sp < ui.ns; sp += 2) {
+            int c = c_lo;
+            for (;;) {
+              while (c <= c_hi && sk_bound(a, k_blocks, c + 1) == sk_bound(a, k_blocks, c)) ++c;
+              if (c > c_hi) break;
+              const int s0 = sk_bound(a, k_blocks, c) < x0 ? 2 * c + 1 : 2 * c;
+              int c2 = c + 1;
+              while (c2 <= c_hi && sk_bound(a, k_blocks, c2 + 1) == sk_bound(a, k_blocks, c2)) ++c2;
+              const bool two = c2 <= c_hi;
+              const int s1 = two ? (sk_bound(a, k_blocks, c2) < x0 ? 2 * c2 + 1 : 2 * c2) : s0;
               float4 x[8], y[8];
-              const bool two = sp + 1 < ui.ns;
 #pragma unroll
               for (int i = 0; i < 8; ++i) {
-                x[i] = __ldcg(base + (size_t)sp * tile_f4 + (size_t)i * BM);
-                y[i] = two ? __ldcg(base + (size_t)(sp + 1) * tile_f4 + (size_t)i * BM) : make_float4(0.f, 0.f, 0.f, 0.f);
+                x[i] = __ldcg(T0 + (size_t)s0 * tile_f4 + off + (size_t)i * BM);
+                y[i] = two ? __ldcg(T0 + (size_t)s1 * tile_f4 + off + (size_t)i * BM) : make_float4(0.f, 0.f, 0.f, 0.f);
               }
 #pragma unroll
-              for (int i = 0; i < 8; ++i) {   // split sp first, then sp + 1
+              for (int i = 0; i < 8; ++i) {   // segment c first, then c2
                 acc[4 * i] += x[i].x; acc[4 * i + 1] += x[i].y; acc[4 * i + 2] += x[i].z; acc[4 * i + 3] += x[i].w;
                 acc[4 * i] += y[i].x; acc[4 * i + 1] += y[i].y; acc[4 * i + 2] += y[i].z; acc[4 * i + 3] += y[i].w;
               }
+              c = c2 + 1;
             }
           };
           for (int hh = 0; hh < mh; ++hh) {
             const int m = (m_blk * mh + hh) * BM + et;
             if (m >= a.M) continue;
-            const float4* H = T0 + (size_t)hh * BM * bn / 4;
+            const size_t H = (size_t)hh * BM * bn / 4;
             if (a.epi == EPI_QKV) {
               for (int c0 = 0; c0 < bn; c0 += 128)
                 for (int c = 0; c < 64; c += 32) {
@@ -836,9 +870,10 @@ cudaError_t launch_gemm_tc(const CUtensorMap& mapA, const CUtensorMap& mapB, con
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  if (a.mh < 1 || a.mh > 2 || a.splits < 1) return cudaErrorInvalidValue;
+  if (a.mh < 1 || a.mh > 2 || (a.sk_tiles && a.sk_chunks < 1)) return cudaErrorInvalidValue;
   if (a.kcb) {
-    if (a.mh != 1 || a.bn != 128 || a.n_full != (a.M + BM - 1) / BM * (a.N / 128)) return cudaErrorInvalidValue;
+    if (a.mh != 1 || a.bn != 128 || a.sk_tiles || a.n_full != (a.M + BM - 1) / BM * (a.N / 128))
+      return cudaErrorInvalidValue;
     return launch_ex(k_gemm_tc<1, true>, grid, NT, smem, st, a.L.pdl, mapA, mapB, a, gemm_tc_stages(a.bn, 1));
   }
   if (a.mh == 2) return launch_ex(k_gemm_tc<2>, grid, NT, smem, st, a.L.pdl, mapA, mapB, a, gemm_tc_stages(a.bn, 2));

@@ -56,7 +56,8 @@ struct GemmArgs {
   int bn;             // tile width in B rows (tcgen05: 64/128/256; SIMT: 64)
   int mh;             // tcgen05: 128-row halves per unit (1, or 2 = 256 rows sharing each B stage)
   int n_full;         // tcgen05: units [0, n_full) are whole tiles over all of K ...
-  int splits;         // ... the remaining tiles are split `splits` ways over K (tail split)
+  int sk_tiles;       // ... the remaining sk_tiles tiles are streamed: their k-block iterations
+  int sk_chunks;      //     cut into sk_chunks equal ranges (units n_full + c), gemm_tc.cu
   int band;           // tcgen05: M tiles per rasterisation band (see tile_coords)
   int epi;
   int silu_half;      // row offset of the "up" rows in B (EPI_SILU)
@@ -65,15 +66,15 @@ struct GemmArgs {
   float* out_f32;     // [M][ldo] (EPI_F32, EPI_RESID)
   void* out_t;        // [M][ldo] of the element type (EPI_SILU)
   int ldo;
-  float* partials;    // tail split: [tail units][mh][bn/4][128][4] (float4 groups interleaved by row)
-  int* tile_sems;     // tail split: [tail tiles], zero between launches (self-resetting)
+  float* partials;    // stream part: [2 sk_chunks slots][mh][bn/4][128][4] (float4 groups interleaved by row)
+  int* tile_sems;     // stream part: [sk_tiles], zero between launches (self-resetting)
   const uint8_t* b_packed;  // B pre-packed by pack_weight (else B comes through mapB)
   int b_evict_first;        // one M tile: the weight stream is used once (L2 evict-first)
   int b_rows;               // rows of B (packed layout stride)
   int split_b;              // 1: warp 3 issues the B tiles (second copy issuer), warp 0 the A tiles
   int kcb;                  // two-level accumulation (DESIGN R-4e): K chunk in k-blocks (0 = off);
                             // each chunk accumulates in TMEM, the chunks are summed in fp32
-                            // registers by the epilogue (requires mh == 1, bn == 128, splits == 1)
+                            // registers by the epilogue (requires mh == 1, bn == 128, whole tiles)
   // EPI_QKV (bf16, head_dim 128; fuses SURVEY §8a S3 into S2): the epilogue
   // adds the bias, rotates q / k heads (rotate-half RoPE from the (cos, sin)
   // table), rounds to bf16 (point R2) and stores q -> q_out[t][H][128],

@@ -332,8 +332,46 @@ void choose_split(const PerfParams& P, const PhaseShape& model, const SchedState
     *tput = (n_pre + (double)S.decode_tokens.size() * k) / cyc;
     return k;
   };
+  // R-23 (objective 2): the split that makes co-running pay most — among
+  // the SLO-feasible splits and k in {floor(r), ceil(r)} (r = t_p / t_d at
+  // the split, k >= 1), the largest predicted co-location gain
+  // G = (t_p(N) + k t_d(N)) / max(t_p(u), k t_d(v)): the time-sliced cycle
+  // of the same work over the co-run cycle (north_star's target ratio, the
+  // paper's co-run-vs-time-sliced axis, P:L7 / P:L155).  Ties: larger gain,
+  // then the larger prefill share, then the smaller k.  Returns the gain.
+  auto max_gain = [&](int* best_v, int* best_k) -> double {
+    PhaseShape pre = model, dec = model;
+    pre.q_lens = S.prefill_lens; pre.ctx_lens.assign(S.prefill_lens.size(), 0);
+    const int mctx = (int)std::lround(S.decode_mean_ctx);
+    dec.q_lens.assign(S.decode_tokens.size(), 1); dec.ctx_lens.assign(S.decode_tokens.size(), mctx);
+    const double tpN = S.prefill_lens.empty() ? 0.0 : layer_time(pre, P, N, 0) * 1e3;
+    const double tdN = layer_time(dec, P, N, 0) * 1e3;
+    double best_g = -1.0;
+    *best_v = -1; *best_k = 1;
+    for (int v : cands) {
+      if (ev[v].ttft > 1.0 || ev[v].tpot > 1.0) continue;
+      const double t_p = ev[v].t_p, t_d = layer_time(dec, P, v, N - v) * 1e3;
+      if (t_d <= 0.0) continue;
+      const int k0 = std::max(1, (int)std::floor(t_p / t_d));
+      for (int k = k0; k <= k0 + 1; ++k) {
+        const double g = (tpN + k * tdN) / std::max(t_p, k * t_d);
+        if (g > best_g) { best_g = g; *best_v = v; *best_k = k; }
+      }
+    }
+    return best_g;
+  };
   int v;
-  if (ok_t && ok_d && slo.objective == 1) {
+  if (ok_t && ok_d && slo.objective == 2) {
+    int vb, kb;
+    const double g = max_gain(&vb, &kb);
+    if (vb >= 0 && g > 1.0) { *prefill_sms = N - vb; *decode_steps = kb; return; }
+    double t_ts = -1.0;
+    const int k_ts = timesliced(&t_ts);
+    if (k_ts > 0) { *prefill_sms = N; *decode_steps = k_ts; return; }   // co-running does not pay
+    if (vb >= 0) { *prefill_sms = N - vb; *decode_steps = kb; return; }
+    v = reduce_decode();
+  }
+  else if (ok_t && ok_d && slo.objective == 1) {
     double t_co = -1.0, t_ts = -1.0;
     const int vb = max_throughput(&t_co);
     const int k_ts = timesliced(&t_ts);

@@ -39,7 +39,8 @@ struct Slo {
   double ttft_norm, tpot_ms;
   int w_max, v_min;
   double percentile;
-  int objective;   // 0: Alg. 1 as read (R-14..R-17); 1: + throughput among SLO-feasible splits (R-21)
+  int objective;   // 0: Alg. 1 as read (R-14..R-17); 1: + throughput among SLO-feasible splits (R-21, R-22);
+                   // 2: + largest predicted co-location gain over time-slicing (R-23)
 };
 
 double wave_idle(double g, double M);

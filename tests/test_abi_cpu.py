@@ -73,7 +73,7 @@ def test_choose_split_equals_oracle_on_random_states():
     model = MODELS["llama8b"]
     rng = np.random.default_rng(1)
     seen = set()
-    for trial in range(80):
+    for trial in range(120):
         n_pre = int(rng.integers(0, 3)); n_pend = int(rng.integers(0, 6)); n_dec = int(rng.integers(0, 40))
         st = dict(layers_done=int(rng.integers(0, 32)), total_layers=32,
                   prefill_lens=[int(x) for x in rng.integers(128, 8192, n_pre)],
@@ -88,7 +88,7 @@ def test_choose_split_equals_oracle_on_random_states():
         slo = {"ttft_norm_ms_per_tok": float(rng.choice([3.0, 1.5, 0.3])),
                "tpot_ms": float(rng.choice([150.0, 200.0, 175.0, 30.0])),
                "w_max": int(rng.integers(0, 5)), "v_min": int(rng.choice([8, 16, 24])),
-               "percentile": 0.9, "objective": int(trial % 2)}   # both objectives (R-21)
+               "percentile": 0.9, "objective": int(trial % 3)}   # all objectives (R-21, R-23)
         ref = PM.choose_split(P, model, st, slo)
         got = pm.choose_split(st, slo)
         assert got == ref, (trial, got, ref)

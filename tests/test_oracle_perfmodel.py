@@ -345,3 +345,37 @@ def test_max_throughput_and_timesliced_hand_derived(monkeypatch):
     assert PM.choose_split(P, MODEL, _hand_state(), slo) == (82, 2)
     monkeypatch.setattr(PM, "layer_time", _stub_layer_time(2.0))
     assert PM.choose_split(P, MODEL, _hand_state(), slo) == (100, 10)
+
+
+def _stub_saturating(f):
+    """Decode that saturates HBM from 40 SMs on (the non-linearity co-running
+    exploits, §8d feasibility): decode layer = 0.1 x max(1, 40 / m) ms, prefill
+    layer = n / 3 / m ms, both x f under co-location."""
+    def lt(shape, P, m, corun_m):
+        if m <= 0:
+            return math.inf
+        g = f if corun_m > 0 else 1.0
+        q = shape["q_lens"]
+        ms = 0.1 * max(1.0, 40.0 / m) * g if all(x == 1 for x in q) else sum(q) / 3.0 / m * g
+        return ms / 1e3
+    return lt
+
+
+def test_max_gain_hand_derived(monkeypatch):
+    """R-23 (objective 2), M = 100, 300 prefill tokens, f = 1.25.  Alone on
+    all SMs: t_p(N) = 1 ms, t_d(N) = 0.1 ms.  At decode SMs v:
+    t_p = 125/(100 - v), t_d = 0.125 max(1, 40/v), gain(k) = (1 + 0.1k)/max(t_p, k t_d):
+      v = 36: t_d 0.1389, r 14.06 -> k 14: 2.4/1.953 = 1.229;  k 15: 2.5/2.083 = 1.200
+      v = 38: t_d 0.1316, r 15.32 -> k 15: 2.5/2.016 = 1.240;  k 16: 2.6/2.105 = 1.235
+      v = 40: t_d 0.125,  r 16.67 -> k 16: 2.6/2.083 = 1.248;  k 17: 2.7/2.125 = 1.271  (best)
+      v = 42: t_p 2.155,  r 17.24 -> k 17: 2.7/2.155 = 1.253;  k 18: 2.8/2.25 = 1.244
+      v = 44: t_p 2.232,  r 17.86 -> k 17: 2.7/2.232 = 1.210;  k 18: 2.8/2.25 = 1.244
+    (below 40 the decode is slower than linear, above it prefill loses SMs for
+    nothing) -> (u, k) = (60, 17).  With f = 2 the best gain is 2.7/3.4 =
+    0.79 < 1: co-running does not pay -> the time-sliced cycle (100, 10)."""
+    P = PM.default_params(M=100)
+    slo = dict(HAND_SLO_LOOSE, objective=2)
+    monkeypatch.setattr(PM, "layer_time", _stub_saturating(1.25))
+    assert PM.choose_split(P, MODEL, _hand_state(), slo) == (60, 17)
+    monkeypatch.setattr(PM, "layer_time", _stub_saturating(2.0))
+    assert PM.choose_split(P, MODEL, _hand_state(), slo) == (100, 10)
