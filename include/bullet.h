@@ -296,17 +296,18 @@ int bullet_launch_count(const bullet_handle *h, long long *n);
 
 /* Diagnostics (DESIGN.md §5 "where the time goes"): per-CTA device
  * timestamps (%globaltimer, ns) of the next `max_launches` kernel launches
- * of this handle.  Each launch gets BULLET_TRACE_CTAS records of 8 uint64:
+ * of this handle.  Each launch gets BULLET_TRACE_CTAS records of 16 uint64:
  * {smid, entry, first operand stage ready, MMA issue done, epilogue done,
- * exit, work units, 0}; CTAs that left their SM range (or kernels that only
- * record entry / exit) leave zeros.  max_launches = 0 disables (default).
+ * exit, work units, last partial stored, first fixup start, last fixup end,
+ * fixups, 0...}; CTAs that left their SM range (or kernels that only record
+ * entry / exit) leave zeros.  max_launches = 0 disables (default).
  * The handle owns the device buffer.  BULLET_ENOMEM if it cannot be
  * allocated. */
 enum { BULLET_TRACE_CTAS = 2368 };
 int bullet_trace_enable(bullet_handle *h, int max_launches);
 
 /* Copy the recorded launches (oldest first, *n <= cap) to host memory:
- * rec [cap][BULLET_TRACE_CTAS][8], meta [cap][4] = {kind (BULLET_K_*),
+ * rec [cap][BULLET_TRACE_CTAS][16], meta [cap][4] = {kind (BULLET_K_*),
  * phase, layer, grid}; then restart recording.  Synchronizes the device. */
 int bullet_trace_read(bullet_handle *h, uint64_t *rec, int32_t *meta, int cap, int *n);
 

@@ -364,9 +364,9 @@ class Bullet:
         _check(lib().bullet_trace_enable(self.h, int(max_launches)))
 
     def trace_read(self, cap=256):
-        """(records uint64 [n][TRACE_CTAS][8], meta int32 [n][4]) of the traced launches."""
+        """(records uint64 [n][TRACE_CTAS][16], meta int32 [n][4]) of the traced launches."""
         import numpy as np
-        rec = np.zeros((cap, self.TRACE_CTAS, 8), dtype=np.uint64)
+        rec = np.zeros((cap, self.TRACE_CTAS, 16), dtype=np.uint64)
         meta = np.zeros((cap, 4), dtype=np.int32)
         n = c_int()
         _check(lib().bullet_trace_read(self.h, rec.ctypes.data, meta.ctypes.data, cap, ctypes.byref(n)))

@@ -100,7 +100,8 @@ struct PhaseWS {
   void *q = nullptr, *o = nullptr, *h = nullptr, *act = nullptr;
   float* partials = nullptr;
   size_t partial_floats = 0;
-  int* tile_sems = nullptr;
+  int* tile_sems = nullptr;        // [2][N_TILE_SEMS] stream-K counters, alternating slices per GEMM launch
+  int sk_parity = 0;
   int* counters = nullptr;
   int n_counters = 0, next_ctr = 0;
   int2* tiles = nullptr;
@@ -263,12 +264,12 @@ int next_launch(Ctx& c, Launch* L) {
   L->pdl = pdl_on && !c.op && !c.prof;
   if (c.h->trace && c.h->trace_n < c.h->trace_cap) {
     const int i = c.h->trace_n++;
-    L->trace = c.h->trace + (size_t)i * BULLET_TRACE_CTAS * 8;
+    L->trace = c.h->trace + (size_t)i * BULLET_TRACE_CTAS * TRACE_SLOTS;
     int* m = c.h->trace_meta.data() + 4 * i;
     m[0] = c.kind; m[1] = c.phase; m[2] = c.layer; m[3] = 0;
   }
   if (c.op) {
-    CK(cudaMemsetAsync(c.h->op_ctr, 0, 2 * sizeof(int), c.st));
+    CK(cudaMemsetAsync(c.h->op_ctr, 0, 4 * sizeof(int), c.st));
     L->ctr = c.h->op_ctr;
     L->burn = c.h->op_ctr + 1;
   } else {
@@ -418,7 +419,7 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
       if (cost_a < best * 0.999) { best = cost_a; mh = cmh; bn = cand; n_full = tiles; sk_tiles = 0; sk_chunks = 0; }
       const int fw = tiles / c.m_sms, rem = tiles % c.m_sms;
       if (rem == 0) continue;
-      const int chunks = std::min(c.m_sms, rem * k_blocks);
+      const int chunks = std::min({c.m_sms, rem * k_blocks, 15 * rem});   // <= 16 segments per tile
       if ((size_t)2 * chunks * 128 * cmh * cand > pf || rem > N_TILE_SEMS) continue;
       const double segs = std::ceil((double)chunks / rem) + 1.0;   // segments per streamed tile
       const double cost_b = fw * t_tile + (double)rem * k_blocks / chunks * t_kb + T0 +
@@ -437,7 +438,7 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
     int omh = 0, obn = 0, osk = 0;
     if (sscanf(ov, "%d,%d,%d", &omh, &obn, &osk) == 3 && fits(obn) && omh >= 1 && omh <= 2) {
       const int tiles = ((M + 128 * omh - 1) / (128 * omh)) * (N / obn), rem = tiles % c.m_sms;
-      const int chunks = std::min(c.m_sms, rem * k_blocks);
+      const int chunks = std::min({c.m_sms, rem * k_blocks, 15 * rem});
       if (!osk || !rem) { mh = omh; bn = obn; n_full = tiles; sk_tiles = 0; sk_chunks = 0; }
       else if ((size_t)2 * chunks * 128 * omh * obn <= pf && rem <= N_TILE_SEMS) {
         mh = omh; bn = obn; n_full = tiles - rem; sk_tiles = rem; sk_chunks = chunks;
@@ -468,7 +469,8 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
         // every range must get its own partial: when they do not fit
         // (prefill-sized M) fall through to the on-chip mode instead of
         // silently running fewer, longer ranges
-        if ((size_t)2 * chunks * 128 * mh * bn <= h->ph[c.phase].partial_floats && tiles <= N_TILE_SEMS) {
+        if ((size_t)2 * chunks * 128 * mh * bn <= h->ph[c.phase].partial_floats && tiles <= N_TILE_SEMS &&
+            (k_blocks + kcb_ - 1) / kcb_ + 1 <= 16 && Ts * chunks < (1ll << 31)) {
           n_full = 0; sk_tiles = tiles; sk_chunks = chunks; done = true;
         }
       }
@@ -499,6 +501,17 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   a.b_rows = N + (epi == EPI_SILU ? silu_half - N / 2 : 0);
   a.partials = h->ph[c.phase].partials;
   a.tile_sems = h->ph[c.phase].tile_sems;
+  a.sk_parity = h->ph[c.phase].sk_parity;
+  h->ph[c.phase].sk_parity ^= 1;   // every GEMM launch zeroes the slice the next one counts in
+  if (sk_tiles) {   // the stream-K fixup phase's item counter
+    if (c.op) {
+      a.fix_ctr = h->op_ctr + 2;
+    } else {
+      PhaseWS& P = h->ph[c.phase];
+      if (P.next_ctr >= P.n_counters) return set_err(BULLET_ENOMEM, "work counters exhausted");
+      a.fix_ctr = P.counters + P.next_ctr++;
+    }
+  }
   CUtensorMap ma, mb;
   if ((rc = make_map(&ma, A, M, K, 128))) return rc;   // one 128-row half per TMA box
   if ((rc = make_map(&mb, B, N, K, bn / 2))) return rc;
@@ -932,7 +945,7 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
     PhaseWS& P = h->ph[p];
     P.max_tok = p == 0 ? c.max_prefill_tokens : c.max_decode_tokens;
     const size_t T = std::max(1, P.max_tok);
-    P.n_counters = 20 * c.n_layers + 32;
+    P.n_counters = 32 * c.n_layers + 32;
     P.partial_floats = (size_t)2 * h->n_sms * 128 * 256;
     bool ok = cudaMalloc(&P.qkv, T * nq * sizeof(float)) == cudaSuccess &&
               cudaMalloc(&P.q, T * c.n_heads * c.head_dim * h->elt) == cudaSuccess &&
@@ -940,7 +953,7 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
               cudaMalloc(&P.h, T * c.d_model * h->elt) == cudaSuccess &&
               cudaMalloc(&P.act, T * c.d_ff * h->elt) == cudaSuccess &&
               cudaMalloc(&P.partials, P.partial_floats * sizeof(float)) == cudaSuccess &&
-              cudaMalloc(&P.tile_sems, N_TILE_SEMS * sizeof(int)) == cudaSuccess &&
+              cudaMalloc(&P.tile_sems, 2 * N_TILE_SEMS * sizeof(int)) == cudaSuccess &&
               cudaMalloc(&P.counters, P.n_counters * sizeof(int)) == cudaSuccess &&
               cudaMalloc(&P.tiles, (T / ATTN_TC_BQ + T + 1) * sizeof(int2)) == cudaSuccess &&
               cudaMalloc(&P.n_tiles, sizeof(int)) == cudaSuccess &&
@@ -950,10 +963,10 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
     P.max_rb = (int)((T + 127) / 128);
     P.n_rbc_slices = 2 * c.n_layers + 2;
     if (!ok) return fail(set_err(BULLET_ENOMEM, "workspace allocation (phase %d)", p));
-    cudaMemset(P.tile_sems, 0, N_TILE_SEMS * sizeof(int));
+    cudaMemset(P.tile_sems, 0, 2 * N_TILE_SEMS * sizeof(int));
     cudaMemset(P.counters, 0, P.n_counters * sizeof(int));
   }
-  if (cudaMalloc(&h->op_ctr, 2 * sizeof(int)) != cudaSuccess) return fail(set_err(BULLET_ENOMEM, "op ctr"));
+  if (cudaMalloc(&h->op_ctr, 4 * sizeof(int)) != cudaSuccess) return fail(set_err(BULLET_ENOMEM, "op ctr"));
   if (cudaMalloc(&h->d_gates, 2 * sizeof(Gate)) != cudaSuccess) return fail(set_err(BULLET_ENOMEM, "gates"));
   {   // default device split: everything to decode (bullet_set_split overwrites)
     const Gate all = gate_of(h, 0, h->n_sms);
@@ -1249,7 +1262,7 @@ int bullet_trace_enable(bullet_handle* h, int max_launches) {
   h->trace = nullptr; h->trace_cap = h->trace_n = 0;
   h->trace_meta.clear();
   if (max_launches == 0) return BULLET_OK;
-  const size_t bytes = (size_t)max_launches * BULLET_TRACE_CTAS * 8 * sizeof(unsigned long long);
+  const size_t bytes = (size_t)max_launches * BULLET_TRACE_CTAS * TRACE_SLOTS * sizeof(unsigned long long);
   if (cudaMalloc(&h->trace, bytes) != cudaSuccess) return set_err(BULLET_ENOMEM, "trace buffer (%zu bytes)", bytes);
   CK(cudaMemset(h->trace, 0, bytes));
   h->trace_cap = max_launches;
@@ -1263,7 +1276,7 @@ int bullet_trace_read(bullet_handle* h, uint64_t* rec, int32_t* meta, int cap, i
   if (!h->trace) return BULLET_OK;
   CK(cudaDeviceSynchronize());
   const int k = std::min(cap, h->trace_n);
-  const size_t per = (size_t)BULLET_TRACE_CTAS * 8;
+  const size_t per = (size_t)BULLET_TRACE_CTAS * TRACE_SLOTS;
   CK(cudaMemcpy(rec, h->trace, (size_t)k * per * sizeof(unsigned long long), cudaMemcpyDeviceToHost));
   memcpy(meta, h->trace_meta.data(), (size_t)k * 4 * sizeof(int32_t));
   *n = k;

@@ -29,7 +29,7 @@ struct Launch {
   int log_cap;
   int launch_id;
   int phase;
-  unsigned long long* trace;   // nullable (BULLET_TRACE): [grid][8] per-CTA timestamps, see trace_at
+  unsigned long long* trace;   // nullable (bullet_trace_enable): [grid][16] per-CTA timestamps, see trace_at
   int pdl;                     // host: launched with programmatic stream serialization (launch_ex)
 };
 
@@ -49,11 +49,15 @@ __device__ __forceinline__ unsigned long long gtimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
-// Per-CTA trace record (BULLET_TRACE, diagnostics only): slot 0 smid,
+// Per-CTA trace record (bullet_trace_enable, diagnostics only): slot 0 smid,
 // 1 entry, 2 first MMA operand stage ready, 3 MMA issue done, 4 epilogue
-// done, 5 exit, 6 work units, 7 spare.  Written by one thread per slot.
+// done, 5 exit, 6 work units (queue entries), 7 last partial stored + fenced,
+// 8 first fixup start, 9 last fixup end, 10 fixups done.  Written by one
+// thread per slot.
+constexpr int TRACE_SLOTS = 16;
 __device__ __forceinline__ void trace_at(const Launch& L, int slot, unsigned long long v) {
-  if (L.trace) L.trace[(size_t)(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 8 + slot] = v;
+  if (L.trace)
+    L.trace[(size_t)(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * TRACE_SLOTS + slot] = v;
 }
 
 __device__ __forceinline__ uint32_t smid() {

@@ -57,14 +57,16 @@ __device__ __forceinline__ void tile_coords(int tile, int m_tiles, int n_tiles, 
 struct Seg {   // one entry of the CTA's work queue
   int tile, kb0, kb1, slot;   // slot: partial slot, -1 = whole tile (direct epilogue); tile -1 = end
 };
+// (the host keeps sk_chunks * sk_tiles * k_blocks < 2^31: int arithmetic)
 __device__ __forceinline__ int sk_bound(const GemmArgs& a, int k_blocks, int c) {
-  return (int)((long long)c * a.sk_tiles * k_blocks / a.sk_chunks);
+  return c * (a.sk_tiles * k_blocks) / a.sk_chunks;
 }
 // chunk holding stream iteration x (the largest c with sk_bound(c) <= x)
 __device__ __forceinline__ int sk_chunk_of(const GemmArgs& a, int k_blocks, int x) {
-  const long long Ts = (long long)a.sk_tiles * k_blocks;
-  return (int)(((long long)(x + 1) * a.sk_chunks - 1) / Ts);
+  return ((x + 1) * a.sk_chunks - 1) / (a.sk_tiles * k_blocks);
 }
+constexpr int SK_MAX_SEG = 16;   // segments per streamed tile (host: chunks <= 15 x stream tiles)
+constexpr int N_TILE_SEMS_DEV = 2048;   // tile_sems: [0, 2048) segments stored, [2048, 4096) items done (api.cu)
 
 __device__ __forceinline__ uint64_t sw128_desc(uint32_t addr) {
   // UMMA shared-memory descriptor, K-major, SWIZZLE_128B: start>>4 [0,14),
@@ -274,6 +276,14 @@ __device__ __forceinline__ void ar_signal(const GemmArgs& a, int m_blk, int mh, 
     }
   }
 }
+// The same for `cols` columns of row block rb finished by a 128-thread group
+// (named barrier `bar`) of the stream-K fixup phase.
+__device__ __forceinline__ void ar_signal_cols(const GemmArgs& a, int rb, int cols, int et, int bar) {
+  fence_sys();
+  named_bar_sync(bar, 128);
+  if (et < a.ar.n && rb * BM < a.M)
+    red_release_sys_add(a.ar.ready[et] + (size_t)a.ar.rank * a.ar.max_rb + rb, (unsigned long long)cols);
+}
 // After the CTA's GEMM units: reduce units, then wait units (kernels.h).
 __device__ __forceinline__ void ar_phase(const GemmArgs& a, int* s_u) {
   const ArArgs& r = a.ar;
@@ -331,6 +341,12 @@ __device__ __forceinline__ void norm_signal(const GemmArgs& a, int m_blk, int mh
       if (rb * BM >= a.M) break;
       asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(a.nf.rb_ctr + rb), "r"(a.bn) : "memory");
     }
+}
+__device__ __forceinline__ void norm_signal_cols(const GemmArgs& a, int rb, int cols, int et, int bar) {
+  __threadfence();
+  named_bar_sync(bar, 128);
+  if (et == 0 && rb * BM < a.M)
+    asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(a.nf.rb_ctr + rb), "r"(cols) : "memory");
 }
 __device__ __forceinline__ int ld_acquire_gpu(const int* p) {
   int v;
@@ -410,6 +426,169 @@ __device__ __forceinline__ void norm_phase(const GemmArgs& a, int* s_u, float* s
   }
 }
 
+// ---------------------------------------------------------------- stream-K fixup phase
+// After its own queue, every CTA of the launch (all 256 threads, two groups
+// of 128) claims fixup items — (streamed tile, 128-row half, epilogue group
+// of 32 output columns; QKV / SiLU groups pair the rotate-half / gate-up
+// partner columns) — waits until all segments of the item's tile have
+// stored their partials, sums them in k order (deterministic) and runs the
+// epilogue for those columns.  Waiting only after the CTA's own segments are
+// done keeps it deadlock-free (every segment belongs to a unit some CTA runs
+// to completion first), and the reduction is spread over the whole
+// partition instead of one SM per tile.  The tile's last item re-zeroes its
+// counters for the next launch.
+template <int mh>
+__device__ __forceinline__ void fix_phase(const GemmArgs& a, int* s_u, int k_blocks, int m_tiles, int n_tiles,
+                                          uint8_t* ring, uint32_t ring_bytes, uint64_t* fixb) {
+  const int bn = a.bn;
+  const bool pair = a.epi == EPI_QKV || a.epi == EPI_SILU;
+  const int G = pair ? bn / 64 : bn / 32;   // epilogue groups per 128-row half
+  const int nch = pair ? 2 : 1;             // 32-column chunks per group
+  const int per_tile = mh * G, items = a.sk_tiles * per_tile;
+  const int tid = threadIdx.x, et = tid & 127;
+  const size_t tile_f4 = (size_t)mh * BM * bn / 4;
+  constexpr uint32_t CHUNK = BM * 32 * 4;   // one 32-column chunk of one segment's partial: 16 KB
+  const int* sems = a.tile_sems + (a.sk_parity ? N_TILE_SEMS_DEV : 0);
+  float4* buf = reinterpret_cast<float4*>(ring);
+  const int t0n = a.L.trace && tid == 0;
+  if (t0n) trace_at(a.L, 8, gtimer());
+  int n_items = 0;
+  uint32_t fph = 0;
+  uint64_t pol = 0;
+  if (tid == 0) { asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol)); s_u[0] = atomicAdd(a.fix_ctr, 1); }
+  __syncthreads();
+  int u = s_u[0];
+  for (;;) {
+    __syncthreads();   // (s_u, ring reuse)
+    if (u >= items) break;
+    ++n_items;
+    int u_next = 0;
+    if (tid == 0) u_next = atomicAdd(a.fix_ctr, 1);   // claim ahead: its round trip overlaps this item
+    const int st_idx = u / per_tile, r = u % per_tile, hh = r / G, gi = r % G;
+    const int x0 = st_idx * k_blocks, x1 = x0 + k_blocks - 1;
+    const int c_lo = sk_chunk_of(a, k_blocks, x0), c_hi = sk_chunk_of(a, k_blocks, x1);
+    int seg_slot[SK_MAX_SEG];
+    int nseg = 0;
+    {
+      int b0 = sk_bound(a, k_blocks, c_lo);
+      for (int c = c_lo; c <= c_hi && nseg < SK_MAX_SEG; ++c) {
+        const int b1 = sk_bound(a, k_blocks, c + 1);
+        if (b1 > b0) seg_slot[nseg++] = b0 < x0 ? 2 * c + 1 : 2 * c;
+        b0 = b1;
+      }
+    }
+    int m_blk, n_blk;
+    tile_coords(a.n_full + st_idx, m_tiles, n_tiles, a.band, m_blk, n_blk);
+    const int m = (m_blk * mh + hh) * BM + et;
+    const int c = a.epi == EPI_QKV ? (gi >> 1) * 128 + (gi & 1) * 32 : gi * 32;
+    const int c2 = a.epi == EPI_QKV ? c + 64 : bn / 2 + c;   // pair partner chunk
+    // epilogue inputs that do not depend on the partials, loaded while waiting
+    float4 r4[8];
+    if (tid < 128 && a.epi == EPI_RESID && m < a.M) {
+      const float4* rp = reinterpret_cast<const float4*>(a.resid + (size_t)m * a.ldo + n_blk * bn + c);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) r4[i] = rp[i];
+    }
+    const bool tr = t0n && n_items == 1;
+    if (tr) trace_at(a.L, 11, gtimer());
+    const bool bulk = (uint32_t)(nseg * nch) * CHUNK <= ring_bytes;
+    if (tid == 0) {   // every segment of the tile has stored its partial
+      while (ld_acquire_gpu(sems + st_idx) < nseg) __nanosleep(32);
+      if (bulk) {     // all (chunk, segment) blocks in one bulk-copy round
+        mbar_arrive_expect_tx(fixb, (uint32_t)(nseg * nch) * CHUNK);
+        for (int ch = 0; ch < nch; ++ch)
+          for (int sg = 0; sg < nseg; ++sg)
+            bulk_g2s(ring + (size_t)(ch * nseg + sg) * CHUNK,
+                     reinterpret_cast<const float4*>(a.partials) + (size_t)seg_slot[sg] * tile_f4 +
+                         (size_t)hh * BM * bn / 4 + (size_t)((ch ? c2 : c) / 4) * BM,
+                     CHUNK, fixb, pol);
+      }
+    }
+    __syncthreads();
+    if (tr) trace_at(a.L, 12, gtimer());
+    float v[32], w[32];
+    if (bulk) {
+      mbar_wait(fixb, fph);
+      fph ^= 1;
+      // sum the segments in k order, element-wise over the chunks (256 threads),
+      // into each chunk's first block
+      for (int ch = 0; ch < nch; ++ch)
+        for (int f = tid; f < BM * 8; f += NT) {
+          float4 acc = buf[(size_t)(ch * nseg) * BM * 8 + f];
+          for (int sg = 1; sg < nseg; ++sg) {
+            const float4 x = buf[(size_t)(ch * nseg + sg) * BM * 8 + f];
+            acc.x += x.x; acc.y += x.y; acc.z += x.z; acc.w += x.w;
+          }
+          buf[(size_t)(ch * nseg) * BM * 8 + f] = acc;
+        }
+      __syncthreads();
+      if (tid < 128) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const float4 x = buf[(size_t)i * BM + et];
+          v[4 * i] = x.x; v[4 * i + 1] = x.y; v[4 * i + 2] = x.z; v[4 * i + 3] = x.w;
+        }
+        if (pair)
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const float4 x = buf[(size_t)nseg * BM * 8 + (size_t)i * BM + et];
+            w[4 * i] = x.x; w[4 * i + 1] = x.y; w[4 * i + 2] = x.z; w[4 * i + 3] = x.w;
+          }
+      }
+    } else if (tid < 128) {   // too many segments for the ring: register batches
+      const float4* T0 = reinterpret_cast<const float4*>(a.partials) + (size_t)hh * BM * bn / 4 + et;
+      auto sum32 = [&](int col, float* acc) {
+        const size_t off = (size_t)(col / 4) * BM;
+#pragma unroll
+        for (int i = 0; i < 32; ++i) acc[i] = 0.f;
+        for (int j = 0; j < nseg; j += 4) {
+          float4 x[4][8];
+#pragma unroll
+          for (int q = 0; q < 4; ++q)
+#pragma unroll
+            for (int i = 0; i < 8; ++i)
+              x[q][i] = j + q < nseg ? __ldcg(T0 + (size_t)seg_slot[j + q] * tile_f4 + off + (size_t)i * BM)
+                                     : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+          for (int q = 0; q < 4; ++q)
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              acc[4 * i] += x[q][i].x; acc[4 * i + 1] += x[q][i].y;
+              acc[4 * i + 2] += x[q][i].z; acc[4 * i + 3] += x[q][i].w;
+            }
+        }
+      };
+      sum32(c, v);
+      if (pair) sum32(c2, w);
+    }
+    if (tid < 128) {
+      if (a.epi == EPI_QKV) {   // group gi: head gi / 2, columns c and its rotate-half partner c + 64
+        if (m < a.M) epi_qkv(a, m, n_blk * bn + c, v, w);
+      } else if (a.epi == EPI_SILU) {   // gate columns c, up columns bn / 2 + c -> output n_blk bn / 2 + c
+        if (m < a.M) epi_store(a, m, n_blk * (bn / 2) + c, v, w);
+      } else if (a.epi == EPI_RESID) {
+        if (m < a.M) {
+          float4* dst = reinterpret_cast<float4*>(a.out_f32 + (size_t)m * a.ldo + n_blk * bn + c);
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+            dst[i] = make_float4(r4[i].x + v[4 * i], r4[i].y + v[4 * i + 1], r4[i].z + v[4 * i + 2],
+                                 r4[i].w + v[4 * i + 3]);
+        }
+      } else {
+        if (m < a.M) epi_store(a, m, n_blk * bn + c, v, nullptr);
+      }
+      if (tr) trace_at(a.L, 13, gtimer());
+      if (a.ar.n) ar_signal_cols(a, m_blk * mh + hh, 32, et, 2);
+      if (a.nf.out) norm_signal_cols(a, m_blk * mh + hh, 32, et, 2);
+      if (tr) trace_at(a.L, 14, gtimer());
+    }
+    if (tid == 0) s_u[0] = u_next;
+    __syncthreads();
+    u = s_u[0];
+  }
+  if (t0n) { trace_at(a.L, 9, gtimer()); trace_at(a.L, 10, n_items); }
+}
+
 }  // namespace
 
 int gemm_tc_stages(int bn, int mh) {
@@ -442,7 +621,8 @@ __global__ void __launch_bounds__(NT, 1)
   uint64_t* acce = accf + 2;
   uint64_t* tqf = acce + 2;
   uint64_t* tqe = tqf + 4;
-  Seg* tile_q = reinterpret_cast<Seg*>(tqe + 4);
+  uint64_t* fixb = tqe + 4;   // stream-K fixup: bulk loads of partials into the (then idle) stage ring
+  Seg* tile_q = reinterpret_cast<Seg*>(fixb + 2);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tile_q + 4);
   int* s_last = reinterpret_cast<int*>(tmem_slot + 1);
 
@@ -456,6 +636,7 @@ __global__ void __launch_bounds__(NT, 1)
     for (int s = 0; s < n_stages; ++s) { mbar_init(full + s, a.split_b ? 2 : 1); mbar_init(empty + s, 1); }
     for (int i = 0; i < 2; ++i) { mbar_init(accf + i, 1); mbar_init(acce + i, 4); }
     for (int i = 0; i < 4; ++i) { mbar_init(tqf + i, 1); mbar_init(tqe + i, a.split_b ? 6 : 5); }
+    mbar_init(fixb, 1);
     mbar_fence_init();
   }
   if (warp == 0 && lane == 0) { tma_prefetch_desc(&mapA); tma_prefetch_desc(&mapB); }
@@ -531,15 +712,23 @@ __global__ void __launch_bounds__(NT, 1)
         const int u = atomicAdd(a.L.ctr, 1);
         if (u >= units) { issue(Seg{-1, 0, 0, -1}); break; }
         log_unit(a.L, u);
-        if (u < a.n_full) { issue(Seg{u, 0, k_blocks, -1}); continue; }
-        const int c = u - a.n_full;   // stream range c: its segments in k order
-        const int xb = sk_bound(a, k_blocks, c), xe = sk_bound(a, k_blocks, c + 1);
-        for (int x = xb; x < xe;) {
-          const int t = x / k_blocks, k0 = x - t * k_blocks, se = min(xe, (t + 1) * k_blocks);
-          const int k1 = se - t * k_blocks;
-          const bool whole = k0 == 0 && k1 == k_blocks;
-          issue(Seg{a.n_full + t, k0, k1, whole ? -1 : (x == xb ? 2 * c : 2 * c + 1)});
-          x = se;
+        if (u < a.n_full) {
+          issue(Seg{u, 0, k_blocks, -1});
+        } else {
+          const int c = u - a.n_full;   // stream range c: its segments in k order
+          const int xb = sk_bound(a, k_blocks, c), xe = sk_bound(a, k_blocks, c + 1);
+          for (int x = xb; x < xe;) {
+            const int t = x / k_blocks, k0 = x - t * k_blocks, se = min(xe, (t + 1) * k_blocks);
+            const int k1 = se - t * k_blocks;
+            const bool whole = k0 == 0 && k1 == k_blocks;
+            issue(Seg{a.n_full + t, k0, k1, whole ? -1 : (x == xb ? 2 * c : 2 * c + 1)});
+            x = se;
+          }
+        }
+        {   // zero the stream-K counters of the next launch (the other parity slice;
+            // the launch that used it last has completed): unit u takes indices u mod units
+          int* nxt = a.tile_sems + (a.sk_parity ? 0 : N_TILE_SEMS_DEV);
+          for (int i = u; i < N_TILE_SEMS_DEV; i += units) nxt[i] = 0;
         }
       }
     }
@@ -731,74 +920,15 @@ __global__ void __launch_bounds__(NT, 1)
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(acce + as);
-        // the tile's segments: stream ranges c_lo .. c_hi (non-empty ones), in k order
-        const int st_idx = g.tile - a.n_full;
-        const int x0 = st_idx * k_blocks, x1 = x0 + k_blocks - 1;
-        const int c_lo = sk_chunk_of(a, k_blocks, x0), c_hi = sk_chunk_of(a, k_blocks, x1);
-        int nseg = 0;
-        for (int c = c_lo; c <= c_hi; ++c) nseg += sk_bound(a, k_blocks, c + 1) > sk_bound(a, k_blocks, c);
+        // count the segment in its tile; the tile is reduced in the fixup
+        // phase (fix_phase) once all its segments are stored
         __threadfence();
         named_bar_sync(1, 128);
         if (et == 0) {
-          const int old = atomicAdd(a.tile_sems + st_idx, 1);
-          const int last = (old == nseg - 1);
-          if (last) a.tile_sems[st_idx] = 0;  // self-reset for the next launch
-          *s_last = last;
-        }
-        named_bar_sync(1, 128);
-        const bool last = *s_last;
-        if (last) {
-          __threadfence();
-          const float4* T0 = reinterpret_cast<const float4*>(a.partials) + et;
-          // sum 32 columns over the tile's segments (k order: deterministic),
-          // two segments per batch so 16 float4 loads are in flight per thread
-          auto sum32 = [&](size_t off, float* acc) {
-#pragma unroll
-            for (int i = 0; i < 32; ++i) acc[i] = 0.f;
-            int c = c_lo;
-            for (;;) {
-              while (c <= c_hi && sk_bound(a, k_blocks, c + 1) == sk_bound(a, k_blocks, c)) ++c;
-              if (c > c_hi) break;
-              const int s0 = sk_bound(a, k_blocks, c) < x0 ? 2 * c + 1 : 2 * c;
-              int c2 = c + 1;
-              while (c2 <= c_hi && sk_bound(a, k_blocks, c2 + 1) == sk_bound(a, k_blocks, c2)) ++c2;
-              const bool two = c2 <= c_hi;
-              const int s1 = two ? (sk_bound(a, k_blocks, c2) < x0 ? 2 * c2 + 1 : 2 * c2) : s0;
-              float4 x[8], y[8];
-#pragma unroll
-              for (int i = 0; i < 8; ++i) {
-                x[i] = __ldcg(T0 + (size_t)s0 * tile_f4 + off + (size_t)i * BM);
-                y[i] = two ? __ldcg(T0 + (size_t)s1 * tile_f4 + off + (size_t)i * BM) : make_float4(0.f, 0.f, 0.f, 0.f);
-              }
-#pragma unroll
-              for (int i = 0; i < 8; ++i) {   // segment c first, then c2
-                acc[4 * i] += x[i].x; acc[4 * i + 1] += x[i].y; acc[4 * i + 2] += x[i].z; acc[4 * i + 3] += x[i].w;
-                acc[4 * i] += y[i].x; acc[4 * i + 1] += y[i].y; acc[4 * i + 2] += y[i].z; acc[4 * i + 3] += y[i].w;
-              }
-              c = c2 + 1;
-            }
-          };
-          for (int hh = 0; hh < mh; ++hh) {
-            const int m = (m_blk * mh + hh) * BM + et;
-            if (m >= a.M) continue;
-            const size_t H = (size_t)hh * BM * bn / 4;
-            if (a.epi == EPI_QKV) {
-              for (int c0 = 0; c0 < bn; c0 += 128)
-                for (int c = 0; c < 64; c += 32) {
-                  sum32(H + (size_t)((c0 + c) / 4) * BM, v);
-                  sum32(H + (size_t)((c0 + 64 + c) / 4) * BM, w);
-                  epi_qkv(a, m, col0 + c0 + c, v, w);
-                }
-              continue;
-            }
-            for (int c = 0; c < out_chunks; ++c) {
-              sum32(H + (size_t)(c * 8) * BM, v);
-              if (a.epi == EPI_SILU) sum32(H + (size_t)(bn / 8 + c * 8) * BM, w);
-              epi_store(a, m, col0 + c * 32, v, w);
-            }
-          }
-          if (a.ar.n) ar_signal(a, m_blk, mh, et);
-          if (a.nf.out) norm_signal(a, m_blk, mh, et);
+          asm volatile("red.release.gpu.global.add.s32 [%0], 1;" ::"l"(a.tile_sems + (a.sk_parity ? N_TILE_SEMS_DEV : 0) +
+                                                                      (g.tile - a.n_full))
+                       : "memory");
+          if (a.L.trace) trace_at(a.L, 7, gtimer());
         }
       }
       if (++as == n_acc) { as = 0; aph ^= 1; }
@@ -807,6 +937,10 @@ __global__ void __launch_bounds__(NT, 1)
     if (et == 0 && a.L.trace) trace_at(a.L, 4, gtimer());
   }
   pdl_wait();   // (no-op once passed) the tails below read and write predecessor-visible memory
+  if (a.sk_tiles) {   // stream-K: reduce the streamed tiles (all CTAs, after their own segments)
+    __syncthreads();
+    fix_phase<mh>(a, s_last + 2, k_blocks, m_tiles, n_tiles, smem, (uint32_t)n_stages * st_bytes, fixb);
+  }
   if (a.ar.n) {   // fused all-reduce: this CTA's GEMM units are done
     __syncthreads();
     ar_phase(a, s_last + 1);

@@ -67,7 +67,9 @@ struct GemmArgs {
   void* out_t;        // [M][ldo] of the element type (EPI_SILU)
   int ldo;
   float* partials;    // stream part: [2 sk_chunks slots][mh][bn/4][128][4] (float4 groups interleaved by row)
-  int* tile_sems;     // stream part: [sk_tiles], zero between launches (self-resetting)
+  int* tile_sems;     // stream part: [2][2048] segments stored per streamed tile; launch L
+  int sk_parity;      // counts in slice sk_parity and zeroes the other one for launch L + 1
+  int* fix_ctr;       // stream part: fixup item counter, zero at launch
   const uint8_t* b_packed;  // B pre-packed by pack_weight (else B comes through mapB)
   int b_evict_first;        // one M tile: the weight stream is used once (L2 evict-first)
   int b_rows;               // rows of B (packed layout stride)

@@ -42,6 +42,21 @@ def analyse(rec, meta):
             row["epi_done_us_max"] = us(g[:, 4].max() - t0)
             row["exit_us_med"] = us(np.median(g[:, 5] - t0))
             row["units_per_cta"] = [int(g[:, 6].min()), int(g[:, 6].max())]
+        if (r[:, 7] > 0).any():
+            row["partial_stored_us_max"] = us(r[r[:, 7] > 0][:, 7].max() - t0)
+        if (r[:, 8] > 0).any():
+            f = r[r[:, 8] > 0]
+            row["fixup_ctas"] = int(len(f))
+            row["fixups"] = int(f[:, 10].sum())
+            row["fixup_start_us"] = [us(f[:, 8].min() - t0), us(f[:, 8].max() - t0)]
+            row["fixup_end_us_max"] = us(f[:, 9].max() - t0)
+            row["fixup_dur_us_med"] = us(np.median(f[:, 9] - f[:, 8]))
+            g2 = f[f[:, 11] > 0]
+            if len(g2):   # first item of group 0: start -> tile ready -> summed + stored -> signalled
+                row["item_wait_us_med"] = us(np.median(g2[:, 12] - g2[:, 11]))
+                row["item_ready_us_med"] = us(np.median(g2[:, 12] - t0))
+                row["item_sum_store_us_med"] = us(np.median(g2[:, 13] - g2[:, 12]))
+                row["item_signal_us_med"] = us(np.median(g2[:, 14] - g2[:, 13]))
         prev_end = r[:, 5].max() if (r[:, 5] > 0).any() else None
         rows.append(row)
     return rows

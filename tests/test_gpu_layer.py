@@ -287,7 +287,11 @@ def test_fused_qkv_pool_vs_oracle(bias):
         assert np.array_equal(g_s[~mask], o_s[~mask])          # untouched slots: bit-identical
         assert not np.any(np.isnan(g_s[mask]))                # every named slot written
         gw, rw = g_s[mask].astype(np.float64), r_s[mask].astype(np.float64)   # oracle: already R2-rounded
-        assert np.all(np.abs(gw - rw) <= np.abs(rw) * 2.0 ** -7)   # equal, or one bf16 step apart (a flip)
+        # equal, or one bf16 step apart (an R2 rounding flip); plus, for values
+        # near 0, what an R1 flip of the token's normed input moves them by
+        # (one bf16 step of h_i times |w_ij|: up to ~5e-4 per flipped h_i at d = 1024)
+        bad = np.abs(gw - rw) > np.abs(rw) * 2.0 ** -7 + 2e-3
+        assert not bad.any(), (int(bad.sum()), gw[bad][:8], rw[bad][:8], np.argwhere(bad)[:4])
         assert np.mean(gw == rw) > 0.99
 
 
