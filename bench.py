@@ -96,6 +96,11 @@ def broadcast_obj(x, ws):
 
 
 DEFAULT_CONFIG = {1: "arxiv-8b", 2: "qwen14b-tp2", 4: "qwen14b-tp4", 8: "llama70b-tp8"}
+# Table 2 SLOs: normalized TTFT (ms per prompt token), TPOT (ms)
+_SG, _AX = {"ttft_norm_ms_per_tok": 3.0, "tpot_ms": 150.0}, {"ttft_norm_ms_per_tok": 1.5, "tpot_ms": 175.0}
+SLO = {name: dict(v, w_max=4, v_min=16, percentile=0.9) for name, v in
+       (("sharegpt-8b", _SG), ("arxiv-8b", _AX), ("qwen14b-tp2", _SG), ("qwen14b-tp4", _SG),
+        ("llama70b-tp8", _AX), ("tiny", _SG))}
 
 
 # ---------------------------------------------------------------- clocks
@@ -569,6 +574,7 @@ def main():
     ap.add_argument("--k-max", type=int, default=16)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--sweep", action="store_true", help="also print the p sweep (stderr)")
+    ap.add_argument("--no-sweep", action="store_true", help="skip the on-device (p, k) sweep")
     ap.add_argument("--allreduce", default="peer", choices=["peer", "nccl"],
                     help="TP configs: fused peer-memory all-reduce (default) or NCCL")
     args = ap.parse_args()
@@ -588,25 +594,40 @@ def main():
     t_pre_full = S.time_steps(3, N, B.CORUN, dec=False)
     S.time_steps(1, 0, B.CORUN, pre=False)
     t_dec_full = S.time_steps(3, 0, B.CORUN, pre=False)
-    # ---- choose the split (p, k)
-    if args.p is None or args.k is None:
-        cands = [args.p] if args.p else list(range(56, N - 15, 8))
-        best, table = S.tune(cands, t_pre_full, t_dec_full)
-        p = args.p or best["p"]
-        k = args.k or best["k"]
-        if args.sweep and rank == 0:
-            for r in table:
-                print(json.dumps(r), file=sys.stderr)
-    else:
-        p, k, table = args.p, args.k, []
-    # the paper's scheduler on this batch (Alg. 1 with the fitted model, Table 2
-    # ShareGPT SLOs: 3.0 ms/token normalized TTFT, 150 ms TPOT)
+    # ---- the split: the library's own decision (bullet_choose_split, Alg. 1
+    # with objective 2 = the SLO-feasible split with the largest predicted
+    # co-run gain over time-slicing, R-23) on this batch, with the fitted
+    # model and the Table 2 SLOs of the workload; the on-device
+    # sweep of (p, k) is reported next to it (the measured optimum)
+    slo = dict(SLO.get(args.config, SLO["sharegpt-8b"]), objective=2)
     state = dict(layers_done=0, total_layers=S.m.n_layers, prefill_lens=list(S.wl.prefill_lens),
                  prefill_waited_ms=[0.0] * S.n_pre, pending_lens=[], pending_waited_ms=[],
                  decode_tokens=[64] * S.n_d, decode_elapsed_ms=[64 * 30.0] * S.n_d,
-                 decode_mean_ctx=float(np.mean(S.wl.decode_ctx)), u_k=p, v_k=N - p)
-    slo = {"ttft_norm_ms_per_tok": 3.0, "tpot_ms": 150.0, "w_max": 4, "v_min": 16, "percentile": 0.9}
-    model_split = S.bl.choose_split(state, slo)
+                 decode_mean_ctx=float(np.mean(S.wl.decode_ctx)), u_k=N // 2, v_k=N - N // 2)
+    model_split = tuple(broadcast_obj(S.bl.choose_split(state, slo), ws))
+    table, swept = [], None
+    if not args.no_sweep and (args.p is None or args.k is None):
+        cands = [args.p] if args.p else list(range(56, N - 15, 8))
+        swept, table = S.tune(cands, t_pre_full, t_dec_full)
+        if args.sweep and rank == 0:
+            for r in table:
+                print(json.dumps(r), file=sys.stderr)
+    if args.p is not None and args.k is not None:
+        p, k, split_source = args.p, args.k, "command line"
+    elif 0 < model_split[0] < N and model_split[1] >= 1:
+        p, k, split_source = model_split[0], min(model_split[1], args.k_max), "bullet_choose_split (objective 2, R-23)"
+    else:   # the model chose not to co-run (time-sliced cycle): report the swept split instead
+        if swept is None:
+            swept, table = S.tune(list(range(56, N - 15, 8)), t_pre_full, t_dec_full)
+        p, k, split_source = swept["p"], swept["k"], "swept (the model chose the time-sliced cycle)"
+    qp, cp = S.pre.cu[1:] - S.pre.cu[:-1], S.pre.ctx_lens
+    qd, cdc = [1] * S.n_d, S.dec.ctx_lens
+    pred = {"t_prefill_ms": S.bl.predict_us(qp, cp, p, N - p) / 1e3,
+            "t_decode_layer_ms": S.bl.predict_us(qd, cdc, N - p, p) / 1e3,
+            "t_prefill_full_ms": S.bl.predict_us(qp, cp, N, 0) / 1e3,
+            "t_decode_layer_full_ms": S.bl.predict_us(qd, cdc, N, 0) / 1e3}
+    pred["gain"] = (pred["t_prefill_full_ms"] + k * pred["t_decode_layer_full_ms"]) / \
+        max(pred["t_prefill_ms"], k * pred["t_decode_layer_ms"])
     S.dec.layer_end = k
     # ---- co-run (the method) and time-sliced, device-timed, max over ranks.
     # The time-sliced baseline is timed right before AND right after the
@@ -866,7 +887,15 @@ def main():
         "clocks": clk.summary(),
         "tuning": table,
         "alg1_split": {"prefill_sm_count": model_split[0], "decode_layer_steps": model_split[1],
+                       "objective": 2, "slo": slo, "timed": (p, k) == tuple(model_split),
+                       "predicted": pred,
                        "perf_params": "profiles/perf_params_b200.json" if S.perf_json else "unfitted"},
+        "split": {"source": split_source, "prefill_sm_count": p, "decode_layer_steps": k,
+                  "corun_speedup_vs_timesliced": ab,
+                  "swept_best": None if swept is None else {
+                      "prefill_sm_count": swept["p"], "decode_layer_steps": swept["k"],
+                      "speedup_ab": swept["speedup_ab"], "tok_s": swept["tok_s"]},
+                  "vs_swept_best": None if swept is None else ab / swept["speedup_ab"]},
     }
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
         import oracle as O

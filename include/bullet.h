@@ -265,9 +265,9 @@ int bullet_model_predict(const bullet_handle *h, const bullet_batch_shape *shape
 /* Online estimator feedback ("correlating deviations between
  * predicted latency and observed execution times across scheduling cycles,
  * using the inter-cycle duration t_{k+1} - t_k as dynamic feedback"): read /
- * replace the co-location factors p_c, p_b of Eq. 2 that every co-run
- * prediction (corun_sm_count > 0) and bullet_choose_split use.  Errors:
- * EINVAL (non-positive factors). */
+ * replace the scale applied to the fitted co-location factors p_c(m), p_b(m)
+ * of Eq. 2 (default 1) that every co-run prediction (corun_sm_count > 0) and
+ * bullet_choose_split use.  Errors: EINVAL (non-positive factors). */
 int bullet_get_colocation(const bullet_handle *h, double *p_c, double *p_b);
 int bullet_set_colocation(bullet_handle *h, double p_c, double p_b);
 

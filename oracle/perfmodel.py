@@ -105,7 +105,11 @@ def layer_time(shape: dict, P: dict, m: int, corun_m: int) -> float:
     M = P["M"]
     C, B = P["C_tflops"] * 1e12, P["B_gbs"] * 1e9
     d_c, d_b = interp(P["d_c"], m), interp(P["d_b"], m)
-    p_c, p_b = (P["p_c"], P["p_b"]) if corun_m > 0 else (1.0, 1.0)
+    # R-11/R-12: co-location factors, a constant or piecewise linear in the
+    # kernel's own SM count m (fitted from co-run points, like d_c, d_b)
+    def co(v):
+        return interp(v, m) if isinstance(v, dict) else v
+    p_c, p_b = (co(P["p_c"]), co(P["p_b"])) if corun_m > 0 else (1.0, 1.0)
     total = 0.0
     for _, c, b, g, occ in layer_kernels(shape, P, m):
         s = wave_idle(g, m * occ)          # Reading R-13: M := m_i x CTAs per SM

@@ -253,15 +253,20 @@ int next_launch(Ctx& c, Launch* L) {
   L->log_cap = c.h->log_cap;
   L->launch_id = c.h->launch_seq++;
   L->phase = c.phase;
-  // Programmatic dependent launch (common.cuh) is OFF by default
-  // (BULLET_PDL=1 enables it, for experiments): an early-launched kernel's
-  // CTAs land on the SMs its predecessor's out-of-range CTAs freed, leave
-  // (gated out), and the next ones land there again — the whole grid can
-  // drain through the wrong SMs before one of its own frees up, leaving the
-  // work to the last CTA (gate_enter).  Measured: prefill layer 2.36 ->
-  // 102 ms on 76 SMs.  Not under BULLET_PROFILE, not for op-level entries.
-  static const bool pdl_on = getenv("BULLET_PDL") && !strcmp(getenv("BULLET_PDL"), "1");
-  L->pdl = pdl_on && !c.op && !c.prof;
+  // Programmatic dependent launch (common.cuh): a step kernel may launch in
+  // its predecessor's tail, prologue and weight stream overlapping it.  Not
+  // under BULLET_PROFILE (events between launches time each kernel alone),
+  // not for op-level entries; BULLET_PDL=0 disables.  (A first version
+  // triggered at kernel entry and let out-of-range CTAs leave at once: the
+  // grid drained through the SMs the predecessor's gated-out CTAs had freed,
+  // prefill layer 2.36 -> 102 ms — now triggers come in the tail and
+  // out-of-range CTAs park until the predecessor completes.)
+  static const bool pdl_on = !(getenv("BULLET_PDL") && !strcmp(getenv("BULLET_PDL"), "0"));
+  // Not under tensor parallelism: a CTA parked on another partition's SM
+  // (waiting for its own predecessor) could hold an SM that a kernel
+  // spin-waiting on a peer rank (fused all-reduce, NCCL) needs — a cycle
+  // (measured: the simulated-TP4 test hit the 20 s peer timeout).
+  L->pdl = pdl_on && !c.op && !c.prof && c.h->cfg.tp_size == 1;
   if (c.h->trace && c.h->trace_n < c.h->trace_cap) {
     const int i = c.h->trace_n++;
     L->trace = c.h->trace + (size_t)i * BULLET_TRACE_CTAS * TRACE_SLOTS;
@@ -421,9 +426,12 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
       if (rem == 0) continue;
       const int chunks = std::min({c.m_sms, rem * k_blocks, 15 * rem});   // <= 16 segments per tile
       if ((size_t)2 * chunks * 128 * cmh * cand > pf || rem > N_TILE_SEMS) continue;
-      const double segs = std::ceil((double)chunks / rem) + 1.0;   // segments per streamed tile
-      const double cost_b = fw * t_tile + (double)rem * k_blocks / chunks * t_kb + T0 +
-                            (segs - 1.0) * out_b / BW_SM + out_b / EPI_BW + 2 * RTT;
+      // fixup phase (measured by the per-CTA traces): ~6 us to
+      // store the partials and reach the phase, then ~4 us per round of
+      // items (an item = 32 output columns x 128 rows of one streamed tile)
+      const int items = rem * cmh * ((epi == EPI_QKV || epi == EPI_SILU) ? cand / 64 : cand / 32);
+      const double cost_b = fw * t_tile + (double)rem * k_blocks / chunks * t_kb + T0 + 6e-6 +
+                            std::ceil((double)items / c.m_sms) * 4e-6;
       if (cost_b < best * 0.999) {
         best = cost_b; mh = cmh; bn = cand; n_full = fw * c.m_sms; sk_tiles = rem; sk_chunks = chunks;
       }

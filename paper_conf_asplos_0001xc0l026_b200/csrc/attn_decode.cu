@@ -113,7 +113,6 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
   if (!gate_enter(a.L)) return;
   if (threadIdx.x == 0 && a.L.trace) { trace_at(a.L, 0, smid()); trace_at(a.L, 1, gtimer()); }
   pdl_wait();      // q and the new token's k / v come from the QKV GEMM
-  pdl_trigger();
   extern __shared__ __align__(128) uint8_t smem[];
   uint8_t* stages = smem;                                                      // [NCW][DEPTH][STAGE]
   uint8_t* qbuf = stages + NCW * DEPTH * STAGE_BYTES;                          // [NS_MAX][QSLOT_BYTES]
@@ -174,6 +173,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
           mbar_arrive(uqf + slot);
         }
       }
+      if (u < 0 && lane == 0 && n_end == 0) pdl_trigger();   // all units claimed: let the next kernel launch
       if (u < 0 && ++n_end == NG) break;   // one terminator per group
     }
     return;

@@ -212,7 +212,6 @@ __device__ __forceinline__ void load_kv_tile(uint8_t* dst, const __nv_bfloat16* 
 __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
   if (!gate_enter(a.L)) return;
   pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
-  pdl_trigger();
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = smem_raw;
   if (smem_u32(sm) & 1023) __trap();   // swizzle atoms need 1024-byte alignment
@@ -271,7 +270,10 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
         ring[slot] = u < units ? u : -1;
         mbar_arrive(ufull + slot);
       }
-      if (u >= units) break;
+      if (u >= units) {   // all units claimed: the next kernel may launch (PDL)
+        if (lane == 0) pdl_trigger();
+        break;
+      }
       if (lane == 0) log_unit(a.L, u);
       const Unit U = unit_of(a, u);
       const int32_t* bt = a.bt + (size_t)U.r * a.max_blocks;

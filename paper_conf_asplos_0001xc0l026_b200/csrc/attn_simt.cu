@@ -21,7 +21,6 @@ template <typename T, int HD, int HH>
 __global__ void __launch_bounds__(128) k_attn_simt(AttnArgs a) {
   if (!gate_enter(a.L)) return;
   pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
-  pdl_trigger();
   constexpr int EPC = 16 / sizeof(T);           // elements per 16-byte chunk
   constexpr int CPR = HD / EPC;                 // chunks per key row
   constexpr int SWZ = (CPR < 16 ? CPR : 16) - 1;

@@ -70,7 +70,6 @@ __device__ __forceinline__ void cp_async16_zfill(void* dst, const void* src, boo
 __global__ void __launch_bounds__(128) k_attn_prefill_tc(AttnArgs a) {
   if (!gate_enter(a.L)) return;
   pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
-  pdl_trigger();
   extern __shared__ __align__(128) uint8_t sm[];
   uint8_t* Qs = sm;
   uint8_t* Ks = sm + TILE_BYTES;          // [2][64][128]

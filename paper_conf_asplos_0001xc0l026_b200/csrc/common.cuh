@@ -34,15 +34,17 @@ struct Launch {
 };
 
 // Programmatic dependent launch (PDL).  Step kernels are launched so that
-// kernel i+1 may start as soon as every CTA of kernel i has passed
-// pdl_wait (its own predecessor is then complete) and triggered: its CTAs
-// take SMs as kernel i's CTAs leave them, run their prologue and stream the
-// static operands (weights) — and only then pdl_wait(), which returns once
-// kernel i has completed and its memory is visible.  Anything that reads a
-// predecessor's output, or writes memory a predecessor may still read, comes
-// after pdl_wait().  Without the launch attribute both are no-ops.
-__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
-__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+// kernel i+1 may start once every CTA of kernel i has triggered — which a
+// CTA does only when kernel i's work units are all claimed (its tail) and
+// after its own pdl_wait (so kernel i-1 is complete: only neighbours
+// overlap).  Kernel i+1's CTAs then take SMs as kernel i's CTAs leave them,
+// run their prologue and stream the static operands (weights), and only
+// then pdl_wait(), which returns once kernel i has completed and its memory
+// is visible.  Anything that reads a predecessor's output, or writes memory
+// a predecessor may still read, comes after pdl_wait().  Out-of-range CTAs
+// park in gate_enter.  Without the launch attribute both are no-ops.
+// (after pdl_wait: the caller's own predecessor is complete before dependents launch)
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.wait;\n\tgriddepcontrol.launch_dependents;" ::: "memory"); }
 
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
@@ -76,8 +78,14 @@ __device__ __forceinline__ bool gate_ok(const Gate& g) {
 // all landed outside the range, e.g. on SMs another phase or rank freed for
 // a moment): then this last CTA works where it is, so a launch can never end
 // with its units unprocessed (correctness never depends on CTA placement).
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ bool gate_enter(const Launch& L) {
   if (L.gdev ? gate_ok(*L.gdev) : gate_ok(L.gate)) return true;
+  // Launched early (PDL): park until the predecessor has completed before
+  // leaving, so the grid cannot drain through SMs that are free only
+  // because they are not this phase's (the next CTA of the grid would land
+  // on the same SM and leave again) while this phase's SMs are still busy.
+  if (L.pdl) pdl_wait();
   if (!L.burn) return false;
   int last = 0;   // (no shared memory: kernels align their dynamic smem base)
   if (threadIdx.x == 0) last = atomicAdd(L.burn, 1) == (int)(gridDim.x * gridDim.y * gridDim.z) - 1;

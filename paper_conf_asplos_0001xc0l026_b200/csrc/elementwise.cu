@@ -41,7 +41,6 @@ template <typename T, int VPT>
 __global__ void __launch_bounds__(256) k_rmsnorm(NormArgs a) {
   if (!gate_enter(a.L)) return;
   pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
-  pdl_trigger();
   __shared__ int s_u;
   __shared__ float s_red[8];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -92,7 +91,6 @@ template <typename T>
 __global__ void __launch_bounds__(256) k_rmsnorm_warp(NormArgs a) {
   if (!gate_enter(a.L)) return;
   pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
-  pdl_trigger();
   const int lane = threadIdx.x & 31;
   const T* g = reinterpret_cast<const T*>(a.g);
   T* out = reinterpret_cast<T*>(a.out);
@@ -133,7 +131,6 @@ template <typename T>
 __global__ void __launch_bounds__(256) k_rope_kv(RopeArgs a) {
   if (!gate_enter(a.L)) return;
   pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
-  pdl_trigger();
   __shared__ int s_u;
   const int tid = threadIdx.x;
   const int half = a.hd / 2, hp = half / 2;  // pair-of-pairs per head
@@ -180,7 +177,6 @@ __global__ void __launch_bounds__(256) k_gemm_simt(const T* __restrict__ A, cons
                                                    GemmArgs a) {
   if (!gate_enter(a.L)) return;
   pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
-  pdl_trigger();
   __shared__ float As[16][68], Bs[16][68], Us[16][68];
   __shared__ int s_u;
   const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;

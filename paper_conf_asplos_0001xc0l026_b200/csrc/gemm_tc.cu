@@ -677,7 +677,6 @@ __global__ void __launch_bounds__(NT, 1)
         b_rows_of(n_blk, r0, r1);
         if (!waited) {   // activations are the predecessor's output (warp 3 streams weights meanwhile)
           pdl_wait();
-          pdl_trigger();
           waited = true;
         }
         for (int kb = g.kb0; kb < g.kb1; ++kb) {
@@ -710,7 +709,11 @@ __global__ void __launch_bounds__(NT, 1)
         // early CTAs cannot hoard units while others idle (load balance)
         mbar_wait(empty + s, ph ^ 1);
         const int u = atomicAdd(a.L.ctr, 1);
-        if (u >= units) { issue(Seg{-1, 0, 0, -1}); break; }
+        if (u >= units) {   // all units claimed: the tail; the next kernel may launch
+          pdl_trigger();
+          issue(Seg{-1, 0, 0, -1});
+          break;
+        }
         log_unit(a.L, u);
         if (u < a.n_full) {
           issue(Seg{u, 0, k_blocks, -1});

@@ -103,14 +103,22 @@ bool PerfParams::parse(const char* json, std::string* err) {
     if (it != j.out.end()) dst = it->second;
   };
   get1("M", M); get1("C_tflops", C_tflops); get1("B_gbs", B_gbs);
-  get1("p_c", p_c); get1("p_b", p_b);
+  {   // p_c / p_b: a number (constant over m) or a {"m": [...], "v": [...]} table
+    double c = -1.0, b = -1.0;
+    get1("p_c", c); get1("p_b", b);
+    if (c > 0) { pc_m = {1.0, M}; pc_v = {c, c}; }
+    if (b > 0) { pb_m = {1.0, M}; pb_v = {b, b}; }
+    getv("p_c.m", pc_m); getv("p_c.v", pc_v); getv("p_b.m", pb_m); getv("p_b.v", pb_v);
+    p_c = p_b = 1.0;
+  }
   getv("d_c.m", dc_m); getv("d_c.v", dc_v); getv("d_b.m", db_m); getv("d_b.v", db_v);
   get1("tiles.gemm_bm", gemm_bm); get1("tiles.gemm_bn", gemm_bn); get1("tiles.gemm_bk", gemm_bk);
   get1("tiles.min_k_blocks", min_k_blocks); get1("tiles.attn_bq", attn_bq);
   get1("tiles.rows_per_unit", rows_per_unit);
   get1("occ.gemm", occ_gemm); get1("occ.attn", occ_attn); get1("occ.elem", occ_elem);
-  if (dc_m.size() != dc_v.size() || db_m.size() != db_v.size() || dc_m.empty() || db_m.empty()) {
-    if (err) *err = "perf params: d_c / d_b tables malformed";
+  if (dc_m.size() != dc_v.size() || db_m.size() != db_v.size() || dc_m.empty() || db_m.empty() ||
+      pc_m.size() != pc_v.size() || pb_m.size() != pb_v.size() || pc_m.empty() || pb_m.empty()) {
+    if (err) *err = "perf params: d_c / d_b / p_c / p_b tables malformed";
     return false;
   }
   return true;
@@ -121,6 +129,8 @@ void PerfParams::set_default(int n_sms) {
   C_tflops = 1649.5; B_gbs = 6549.4;   // MEASURED_PEAKS.json (burst GEMM, copy)
   dc_m = {1.0, (double)n_sms}; dc_v = {1.0, 1.0};
   db_m = {1.0, (double)n_sms}; db_v = {1.0, 1.0};
+  pc_m = {1.0, (double)n_sms}; pc_v = {1.0, 1.0};
+  pb_m = {1.0, (double)n_sms}; pb_v = {1.0, 1.0};
   p_c = p_b = 1.0;
 }
 
@@ -188,7 +198,8 @@ double layer_time(const PhaseShape& s, const PerfParams& P, int m, int corun_m) 
   if (m <= 0) return std::numeric_limits<double>::infinity();
   const double C = P.C_tflops * 1e12, B = P.B_gbs * 1e9, M = P.M;
   const double dc = interp(P.dc_m, P.dc_v, m), db = interp(P.db_m, P.db_v, m);
-  const double pc = corun_m > 0 ? P.p_c : 1.0, pb = corun_m > 0 ? P.p_b : 1.0;
+  const double pc = corun_m > 0 ? interp(P.pc_m, P.pc_v, m) * P.p_c : 1.0;
+  const double pb = corun_m > 0 ? interp(P.pb_m, P.pb_v, m) * P.p_b : 1.0;
   double total = 0;
   for (const auto& k : layer_kernels(s, P, m)) {
     const double sidle = wave_idle(k.g, (double)m * k.occ);

@@ -9,7 +9,11 @@ namespace bl {
 struct PerfParams {
   double M = 148, C_tflops = 1649.5, B_gbs = 6549.4;
   std::vector<double> dc_m{1, 148}, dc_v{1, 1}, db_m{1, 148}, db_v{1, 1};
-  double p_c = 1, p_b = 1;
+  // co-location factors p_c(m), p_b(m): piecewise linear in the kernel's own
+  // SM count m (a JSON number = constant), times the online scale (P:L195
+  // estimator feedback, bullet_set_colocation)
+  std::vector<double> pc_m{1, 148}, pc_v{1, 1}, pb_m{1, 148}, pb_v{1, 1};
+  double p_c = 1, p_b = 1;   // scale
   double gemm_bm = 128, gemm_bn = 256, gemm_bk = 64, min_k_blocks = 4, attn_bq = 64, rows_per_unit = 8;
   double occ_gemm = 1, occ_attn = 1, occ_elem = 4;
   bool parse(const char* json, std::string* err);

@@ -28,8 +28,12 @@ M_GRID = [16, 32, 48, 64, 80, 96, 112, 128, 148]
 PRE_SHAPES = [[512], [1024], [2048], [4096], [8192], synth.workload("sharegpt-8b").prefill_lens]
 DEC_SHAPES = [(bs, cl) for bs in (32, 64, 128, 256) for cl in (512, 1024, 2048, 4096)]
 L_CO = 16
-CORUN = [(pre, dec, p) for pre in ([2048], synth.workload("sharegpt-8b").prefill_lens, [8192])
-         for dec in ((128, 1024), (256, 2048), (256, 512)) for p in (48, 72, 96, 120, 132)]
+# co-run points on the split grid the bench sweeps, with the bench's own
+# request mixes (config 2: ShareGPT-shaped prompts x 128 decodes @ ~1k;
+# config 3: 8k prompt x 256 decodes @ ~4k) plus two off-grid mixes
+CORUN = [(pre, dec, p) for pre, dec in ((synth.workload("sharegpt-8b").prefill_lens, (128, 1024)),
+                                        ([8192], (256, 4096)), ([2048], (256, 2048)), ([4096], (64, 512)))
+         for p in range(40, 140, 8)]
 
 
 class Rig:
@@ -144,16 +148,35 @@ def fit(N, pts, m_shape):
         dc_v.append(best[1]); db_v.append(best[2])
     P["d_c"] = {"m": M_GRID, "v": [float(x) for x in dc_v]}
     P["d_b"] = {"m": M_GRID, "v": [float(x) for x in db_v]}
+    # co-location factors as functions of the phase's own SM count (R-12):
+    # prefill co-run points fit p_c(m) (compute-bound kernels), decode ones
+    # p_b(m) (bandwidth-bound), each grid point from the points nearest to it
     co = [p for p in train if p["co"] > 0]
-    best = (math.inf, 1.0, 1.0)
-    for pc, pb in itertools.product(np.linspace(0.4, 1.2, 33), np.linspace(0.4, 1.2, 33)):
-        Q = dict(P, p_c=float(pc), p_b=float(pb))
-        pm = predictor(m_shape, Q, N)
-        err = sum((math.log(pm.predict_us(p["q"], p["c"], p["m"], p["co"]) / 1e3) - math.log(p["ms"])) ** 2 for p in co)
-        pm.close()
-        if err < best[0]:
-            best = (err, pc, pb)
-    P["p_c"], P["p_b"] = float(best[1]), float(best[2])
+    fgrid = np.linspace(0.4, 1.3, 46)
+
+    def fit_table(kind, key):
+        pts_k = [p for p in co if p["kind"] == kind]
+        ms = sorted({p["m"] for p in pts_k})
+        if not ms:
+            return 1.0
+        gm = [m for m in M_GRID if ms[0] - 16 <= m <= ms[-1] + 16] or [M_GRID[0], M_GRID[-1]]
+        vals = []
+        for g in gm:
+            near = [p for p in pts_k if abs(p["m"] - g) <= 12] or \
+                [min(pts_k, key=lambda p: abs(p["m"] - g))]
+            best = (math.inf, 1.0)
+            for f in fgrid:
+                Q = dict(P, **{key: float(f)})
+                pm = predictor(m_shape, Q, N)
+                err = sum((math.log(pm.predict_us(p["q"], p["c"], p["m"], p["co"]) / 1e3) - math.log(p["ms"])) ** 2
+                          for p in near)
+                pm.close()
+                if err < best[0]:
+                    best = (err, float(f))
+            vals.append(best[1])
+        return {"m": [float(m) for m in gm], "v": vals}
+    P["p_c"] = fit_table("pre", "p_c")
+    P["p_b"] = fit_table("dec", "p_b")
     pm = predictor(m_shape, P, N)
 
     def mre(ps):

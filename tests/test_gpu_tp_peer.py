@@ -205,3 +205,38 @@ def test_peer_allreduce_qwen14b_kchunk_meets_1e3(kc, only, mode):
             % (here, os.path.dirname(here)))
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=900)
     assert r.returncode == 0 and "KC-OK" in r.stdout, (r.stdout[-2000:], r.stderr[-4000:])
+
+
+def test_peer_allreduce_config4_prefill_size_rowsampled():
+    """The fused all-reduce at BASELINE config-4 prefill size: Qwen2.5-14B
+    TP2 (simulated ranks on disjoint SM ranges), prefill 8 ShareGPT-shaped
+    prompts + one 8192-token prompt = 12288 tokens (96 row blocks of the
+    reduce), one layer against the unsharded oracle on 192 sampled rows
+    (always each prompt's last row; SURVEY §8c "How the oracle runs at
+    scale"), every rank's hidden bit-identical."""
+    global M, PRE_LENS, DEC_CTX
+    saved = M, PRE_LENS, DEC_CTX
+    wl = synth.workload("qwen14b-tp2")
+    M, PRE_LENS, DEC_CTX = synth.MODELS["qwen2.5-14b"], list(wl.prefill_lens), list(wl.decode_ctx[:16])
+    try:
+        S = Setup(M, PRE_LENS, DEC_CTX, n_layers=1)
+        S.bl.close()
+        ranks = _ranks(S, 2)
+        got = _step_all(S, ranks, S.x_pre.cuda(), S.x_dec.cuda(), 0, 1)
+        assert torch.equal(got[1][0], got[0][0]) and torch.equal(got[1][1], got[0][1])
+        n = sum(PRE_LENS)
+        assert n == 12288
+        rng = np.random.default_rng(12)
+        mask = np.zeros(n, np.uint8)
+        mask[rng.choice(n, 192, replace=False)] = 1
+        mask[np.cumsum(PRE_LENS) - 1] = 1
+        ref = oracle_layer(S, 0, S.x_pre.numpy(), S.x_dec.numpy(), row_mask_pre=mask)
+        sel = mask.astype(bool)
+        mx, mr = compare(got[0][0].cpu().numpy()[sel], ref["pre"][sel])
+        assert mx <= 2e-2 and mr <= 1e-3, ("pre", mx, mr)
+        mx, mr = compare(got[0][1].cpu().numpy(), ref["dec"])
+        assert mx <= 2e-2 and mr <= 1e-3, ("dec", mx, mr)
+        for bl in ranks:
+            bl.close()
+    finally:
+        M, PRE_LENS, DEC_CTX = saved
