@@ -112,6 +112,9 @@ struct PhaseWS {
   int max_rb = 0, n_rbc_slices = 0, next_rbc = 0;
   int4* order = nullptr;           // decode rows in LPT order (plan kernel), valid this step if order_ok
   bool order_ok = false;
+  float* kv_part = nullptr;        // decode phase, split-KV decode attention: partial softmax states
+  int* kv_tick = nullptr;          //   and per-unit arrival tickets (contexts > one block window)
+  int kv_cap = 1;                  //   KV chunks per unit the scratch holds
 };
 
 constexpr int GRAN = 2;            // split granularity: one TPC
@@ -603,6 +606,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
   if (b->n_tokens == 0) return BULLET_OK;
   AttnArgs a;
   memset(&a, 0, sizeof a);
+  a.kv_chunks = 1;
   a.q = q; a.o = o; a.pool_k = h->pk[layer]; a.pool_v = h->pv[layer];
   a.cu = b->d_cu_seqlens; a.ctx = b->d_ctx_lens; a.bt = b->d_block_table;
   a.n_reqs = b->n_reqs; a.max_blocks = b->max_blocks_per_req; a.n_tok = b->n_tokens;
@@ -630,11 +634,20 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     return BULLET_OK;
   }
   if (kind == 0) kind = (bf16 && a.hd == 128) ? (max_qlen(b) > 1 ? 4 : 3) : 1;
-  if (kind == 3 && max_kv(b) > attn_decode_max_blocks() * h->block_size) kind = c.op ? -1 : 1;
-  if (kind == -1) return set_err(BULLET_EUNSUPPORTED, "tensor-core decode attention: context too long");
   if (kind == 3) {
     if (!bf16 || a.hd != 128)
       return set_err(BULLET_EUNSUPPORTED, "tensor-core decode attention: bf16, hd 128 only");
+    // contexts longer than one unit's block window are split over KV chunks
+    // (partial softmax states merged in chunk order, attn_decode.cu)
+    const int span = attn_decode_max_blocks() * h->block_size;
+    a.kv_chunks = std::max(1, (max_kv(b) + span - 1) / span);
+    if (a.kv_chunks > 1) {
+      PhaseWS& P = h->ph[1];   // the decode phase owns the split scratch
+      if (!P.kv_part || a.kv_chunks > P.kv_cap || b->n_tokens > P.max_tok)
+        return set_err(BULLET_EUNSUPPORTED, "decode attention: context %d needs %d KV chunks (capacity %d, "
+                       "from max_position)", max_kv(b), a.kv_chunks, P.kv_cap);
+      a.kv_part = P.kv_part; a.kv_tick = P.kv_tick;
+    }
     int rc = next_launch(c, &a.L);
     if (rc) return rc;
     // four consumer groups of 3 warps per SM on partitions (68 SMs: 78.6 vs
@@ -971,6 +984,17 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
     P.max_rb = (int)((T + 127) / 128);
     P.n_rbc_slices = 2 * c.n_layers + 2;
     if (!ok) return fail(set_err(BULLET_ENOMEM, "workspace allocation (phase %d)", p));
+    if (p == 1 && c.dtype == BULLET_DTYPE_BF16 && c.head_dim == 128) {   // split-KV decode attention scratch
+      const int span = attn_decode_max_blocks() * pool->block_size;
+      P.kv_cap = std::max(1, (c.max_position + span - 1) / span);
+      if (P.kv_cap > 1) {
+        const size_t units = T * c.n_kv_heads;
+        if (cudaMalloc(&P.kv_part, units * P.kv_cap * 8 * 130 * sizeof(float)) != cudaSuccess ||
+            cudaMalloc(&P.kv_tick, units * sizeof(int)) != cudaSuccess ||
+            cudaMemset(P.kv_tick, 0, units * sizeof(int)) != cudaSuccess)
+          return fail(set_err(BULLET_ENOMEM, "split-KV scratch"));
+      }
+    }
     cudaMemset(P.tile_sems, 0, 2 * N_TILE_SEMS * sizeof(int));
     cudaMemset(P.counters, 0, P.n_counters * sizeof(int));
   }
@@ -1314,7 +1338,7 @@ void bullet_destroy(bullet_handle* h) {
     PhaseWS& P = h->ph[p];
     cudaFree(P.qkv); cudaFree(P.q); cudaFree(P.o); cudaFree(P.h); cudaFree(P.act);
     cudaFree(P.partials); cudaFree(P.tile_sems); cudaFree(P.counters); cudaFree(P.tiles);
-    cudaFree(P.n_tiles); cudaFree(P.tok); cudaFree(P.rbc); cudaFree(P.order);
+    cudaFree(P.n_tiles); cudaFree(P.tok); cudaFree(P.rbc); cudaFree(P.order); cudaFree(P.kv_part); cudaFree(P.kv_tick);
     if (h->comm[p] && g_nccl.commDestroy) g_nccl.commDestroy(h->comm[p]);
   }
   for (void* p : h->ipc_opened) cudaIpcCloseMemHandle(p);

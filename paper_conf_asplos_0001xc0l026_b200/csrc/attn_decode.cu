@@ -98,8 +98,8 @@ __device__ __forceinline__ void cp_async16_ef(void* dst, const void* src, uint64
                : "memory");
 }
 
-struct Slot {  // one published unit
-  int u, t, pos, nb;
+struct Slot {  // one published unit: blocks [b0, b0 + nb) of (token t, kv head u % Hkv)
+  int u, t, pos, nb, b0, c;   // c: KV chunk of a split unit (kv_chunks > 1), else 0
 };
 }  // namespace
 
@@ -141,12 +141,16 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
       // the same group (load balance across CTAs; 4 slots = 2 NG)
       if (lane == 0 && it >= NS) mbar_wait(uqe + ((it - NS) % NS), ((it - NS) / NS) & 1);
       __syncwarp();
-      int u = 0;
-      if (lane == 0) u = n_end ? units : atomicAdd(a.L.ctr, 1);
-      u = __shfl_sync(0xffffffffu, u, 0);
-      if (u >= units) u = -1;
-      Slot sl{u, 0, 0, 0};
-      if (u >= 0) {
+      // sub-unit v = c * units + u: KV chunk c (MAXNB blocks) of unit u;
+      // chunks past a row's length are empty and skipped
+      Slot sl{-1, 0, 0, 0, 0, 0};
+      int32_t const* bt = nullptr;
+      for (;;) {
+        int v = 0;
+        if (lane == 0) v = n_end ? units * a.kv_chunks : atomicAdd(a.L.ctr, 1);
+        v = __shfl_sync(0xffffffffu, v, 0);
+        if (v >= units * a.kv_chunks) break;
+        const int u = v % units, c = v / units;
         int r;
         if (a.order) {   // (row, request, position) from the plan kernel: one load
           const int4 od = __ldg(a.order + u / a.Hkv);
@@ -156,10 +160,15 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
           r = find_req(a.cu, a.n_reqs, sl.t);
           sl.pos = __ldg(a.ctx + r) + (sl.t - __ldg(a.cu + r));
         }
-        sl.nb = sl.pos / KB + 1;
-        const int32_t* bt = a.bt + (size_t)r * a.max_blocks;
-        for (int b = lane; b < sl.nb; b += 32) btbuf[slot * MAXNB + b] = __ldg(bt + b);
+        const int nb_all = sl.pos / KB + 1;
+        if (c * MAXNB >= nb_all) continue;   // empty chunk of a short row
+        sl.u = u; sl.c = c; sl.b0 = c * MAXNB; sl.nb = min(MAXNB, nb_all - sl.b0);
+        bt = a.bt + (size_t)r * a.max_blocks + sl.b0;
+        break;
       }
+      const int u = sl.u;
+      if (u >= 0)
+        for (int b = lane; b < sl.nb; b += 32) btbuf[slot * MAXNB + b] = __ldg(bt + b);
       __syncwarp();
       if (lane == 0) {
         uq[slot] = sl;
@@ -277,7 +286,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
       }
       s[0] += s2[0]; s[1] += s2[1]; s[2] += s2[2]; s[3] += s2[3];
       // s[0] (key gq, head 2tq), s[1] (gq, 2tq+1), s[2] (gq+8, 2tq), s[3] (gq+8, 2tq+1)
-      const int k0 = b * KB + gq, k1 = k0 + 8;
+      const int k0 = (S.b0 + b) * KB + gq, k1 = k0 + 8;
       s[0] = k0 <= S.pos ? s[0] * sl2 : -INFINITY;
       s[1] = k0 <= S.pos ? s[1] * sl2 : -INFINITY;
       s[2] = k1 <= S.pos ? s[2] * sl2 : -INFINITY;
@@ -348,6 +357,9 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
     const float* recs[GW];
 #pragma unroll
     for (int w = 0; w < GW; ++w) recs[w] = reinterpret_cast<const float*>(stages + rec_stage[gw * GW + w] * STAGE_BYTES);
+    const int n_ch = a.kv_chunks > 1 ? (S.pos / KB + 1 + MAXNB - 1) / MAXNB : 1;   // chunks of this unit
+    // split unit: [unit][chunk] records of grp x (O[128], m, l) in the scratch
+    float* part = n_ch > 1 ? a.kv_part + ((size_t)S.u * a.kv_chunks + S.c) * 8 * (HD + 2) : nullptr;
     for (int e = threadIdx.x - gw * GW * 32; e < grp * HD; e += GW * 32) {
       const int h = e / HD, d = e % HD;
       float M = -INFINITY;
@@ -361,7 +373,42 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
         L += rw[HD * 8 + 8 + h] * f;
         O += rw[d * 8 + h] * f;
       }
-      og[(size_t)S.t * a.H * HD + (size_t)(g * grp + h) * HD + d] = __float2bfloat16_rn(O / L);
+      if (part) {
+        part[h * (HD + 2) + d] = O;
+        if (d == 0) { part[h * (HD + 2) + HD] = M; part[h * (HD + 2) + HD + 1] = L; }
+      } else {
+        og[(size_t)S.t * a.H * HD + (size_t)(g * grp + h) * HD + d] = __float2bfloat16_rn(O / L);
+      }
+    }
+    if (part) {   // the unit's last chunk to finish merges all chunks in chunk order (deterministic)
+      __threadfence();
+      named_bar_sync(1 + gw, GW * 32);
+      int* s_flag = rec_stage + NCW + gw;
+      if (threadIdx.x == gw * GW * 32) {
+        const int old = atomicAdd(a.kv_tick + S.u, 1);
+        *s_flag = old == n_ch - 1;
+        if (old == n_ch - 1) a.kv_tick[S.u] = 0;   // self-reset for the next launch
+      }
+      named_bar_sync(1 + gw, GW * 32);
+      if (*s_flag) {
+        __threadfence();
+        const float* P0 = a.kv_part + (size_t)S.u * a.kv_chunks * 8 * (HD + 2);
+        for (int e = threadIdx.x - gw * GW * 32; e < grp * HD; e += GW * 32) {
+          const int h = e / HD, d = e % HD;
+          float M = -INFINITY;
+          for (int c = 0; c < n_ch; ++c) M = fmaxf(M, __ldcg(P0 + ((size_t)c * 8 + h) * (HD + 2) + HD));
+          float L = 0.f, O = 0.f;
+          for (int c = 0; c < n_ch; ++c) {
+            const float* pc = P0 + ((size_t)c * 8 + h) * (HD + 2);
+            const float mc = __ldcg(pc + HD);
+            if (mc == -INFINITY) continue;
+            const float f = exp2f(mc - M);
+            L += __ldcg(pc + HD + 1) * f;
+            O += __ldcg(pc + d) * f;
+          }
+          og[(size_t)S.t * a.H * HD + (size_t)(g * grp + h) * HD + d] = __float2bfloat16_rn(O / L);
+        }
+      }
     }
     named_bar_sync(1 + gw, GW * 32);
     if (lane == 0) mbar_arrive(uqe + slot);
@@ -372,7 +419,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
 
 size_t attn_decode_smem_bytes() {
   return (size_t)NCW * DEPTH * STAGE_BYTES + NS_MAX * QSLOT_BYTES + NS_MAX * MAXNB * 4 + NS_MAX * sizeof(Slot) +
-         2 * NS_MAX * 8 + NCW * 4;
+         2 * NS_MAX * 8 + (NCW + 4) * 4;
 }
 int attn_decode_max_blocks() { return MAXNB; }
 

@@ -122,6 +122,10 @@ struct AttnArgs {
   int tok_base;           // decode kernel: its rows are tokens [tok_base, n_tok) (mixed batches)
   const int4* order;      // decode kernel (nullable): unit row i -> (token - tok_base, request, position, -),
                           // longest context first; saves the claimer its per-unit request search
+  int kv_chunks;          // decode kernel: KV chunks of attn_decode_max_blocks() blocks per unit (split-KV
+                          // for longer contexts; 1 = none); partial (O, m, l) per chunk merged in order
+  float* kv_part;         // [units][kv_chunks][8][128 + 2] (kv_chunks > 1)
+  int* kv_tick;           // [units], zero between launches (self-resetting)
   Launch L;
 };
 

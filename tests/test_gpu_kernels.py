@@ -303,3 +303,56 @@ def test_attention_vs_oracle(B, m, kind):
         # where the noise straddles a rounding boundary (mean-rel vs that)
         assert ulps <= 1.0 and err_l1 / ref_l1 <= 2e-4, (ulps, err_l1 / ref_l1)
 
+
+
+def test_decode_attention_long_contexts_split_kv(B):
+    """Decode attention beyond one unit's block window (8192 tokens): the
+    context is split over KV chunks whose partial softmax states are merged
+    in chunk order (attn_decode.cu) — on tensor cores, no SIMT fallback.
+    Contexts straddling the window edges, 16k and 32k, against the oracle's
+    plain softmax attention through the block table."""
+    m = SMALL
+    ctx = [16383, 32767, 9000, 100, 8191, 8192, 0, 20000]
+    q_lens = [1] * len(ctx)
+    lay = synth.paged_layout(q_lens, ctx, 16, seed_offset=6)
+    bl, pools = _handle(B, m, n_blocks=lay.n_blocks, max_tok=64, max_pos=33000)
+    pk_cpu, pv_cpu = synth.kv_pool(m, lay.n_blocks, 16, 0)
+    pools[0][0].copy_(pk_cpu.to(bf16)); pools[0][1].copy_(pv_cpu.to(bf16))
+    n, H, hd = len(ctx), m.n_heads, m.head_dim
+    rng = np.random.default_rng(13)
+    q = O.round_bf16(rng.standard_normal((n, H * hd)))
+    o = torch.zeros(n, H * hd, dtype=bf16, device="cuda")
+    b = B.Batch(q_lens, ctx, lay.block_table, torch.zeros(n, m.d_model, device="cuda"))
+    for rep in range(2):   # twice: the per-unit tickets reset themselves
+        o.zero_()
+        bl.op_attention(b, 0, torch.from_numpy(q.astype(np.float32)).to("cuda", bf16), o, kind=3)
+        torch.cuda.synchronize()
+        got = o.float().cpu().numpy()
+        pk, pv = pk_cpu.numpy(), pv_cpu.numpy()
+        grp = H // m.n_kv_heads
+        err_l1 = ref_l1 = 0.0
+        for r in range(n):
+            for h in range(H):
+                ref = O.attend_paged(q[r, h * hd:(h + 1) * hd], pk, pv, lay.block_table[r], 16, h // grp, ctx[r])
+                g = got[r, h * hd:(h + 1) * hd].astype(np.float64)
+                assert np.all(np.abs(g - ref) <= np.abs(ref) * 2.0 ** -7 + 5e-5), (r, ctx[r], h)
+                rr = O.round_bf16(ref)
+                err_l1 += float(np.abs(g - rr).sum()); ref_l1 += float(np.abs(rr).sum())
+        assert err_l1 / ref_l1 <= 2e-4, err_l1 / ref_l1
+    bl.close()
+
+
+def test_decode_layer_long_contexts_vs_oracle():
+    """A co-run layer step whose decode batch has 16k / 30k contexts (split-KV
+    decode attention inside bullet_step) meets the north-star bar."""
+    from harness import Setup, compare, phase_streams
+    m = synth.ModelShape("small-bf16-long", 1024, 8, 2, 128, 2816, 1)
+    S = Setup(m, [200], [16000, 33, 30000, 8191], n_layers=1)
+    ref = S.oracle()
+    pre, dec = S.batches()
+    S.bl.step(pre, dec, 74, S.B.CORUN, *phase_streams())
+    torch.cuda.synchronize()
+    for name, b in (("pre", pre), ("dec", dec)):
+        mx, mr = compare(b.hidden.cpu().numpy(), ref[name])
+        assert mx <= 2e-2 and mr <= 1e-3, (name, mx, mr)
+    S.bl.close()

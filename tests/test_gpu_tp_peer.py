@@ -221,6 +221,7 @@ def test_peer_allreduce_config4_prefill_size_rowsampled():
     try:
         S = Setup(M, PRE_LENS, DEC_CTX, n_layers=1)
         S.bl.close()
+        S.bl_max_position = max(max(PRE_LENS), max(DEC_CTX) + 1) + 16
         ranks = _ranks(S, 2)
         got = _step_all(S, ranks, S.x_pre.cuda(), S.x_dec.cuda(), 0, 1)
         assert torch.equal(got[1][0], got[0][0]) and torch.equal(got[1][1], got[0][1])
