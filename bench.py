@@ -884,6 +884,7 @@ def main():
                         "step i's copies with the neighbouring steps' compute (two device input sets, copy "
                         "streams), 'serial' copies, computes and reads back one step at a time"},
         "gpu_launches": int(launches),
+        "gate_fallbacks": S.bl.gate_fallbacks(),
         "clocks": clk.summary(),
         "tuning": table,
         "alg1_split": {"prefill_sm_count": model_split[0], "decode_layer_steps": model_split[1],

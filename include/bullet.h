@@ -215,8 +215,22 @@ int bullet_set_layer_weights(bullet_handle *h, int layer, const bullet_layer_wei
 int bullet_num_sms(const bullet_handle *h, int *n_sms, int *granularity);
 
 /* Copy the probed ordered SM list sigma (host int32 [N]) — prefill gets
- * sigma[0:p), decode sigma[p:N) for prefill_sm_count p. */
+ * sigma[0:p), decode sigma[p:N) for prefill_sm_count p.  Order (SURVEY §8a
+ * SG; env BULLET_SIGMA read at create): "sorted" smid order (default; TPC
+ * pairs adjacent), "die" (the TPCs of one die, then the other's) or
+ * "interleave" (alternating dies TPC by TPC), dies from the die probe. */
 int bullet_sm_order(const bullet_handle *h, int32_t *h_sigma, int cap);
+
+/* Die (0 / 1) of each SM of sigma, in sigma order (host int32 [N]), from the
+ * die probe at create: an L2 hit on an SM's own die is faster than one on
+ * the other die; -1 everywhere when the probe was inconclusive. */
+int bullet_sm_dies(const bullet_handle *h, int32_t *h_die, int cap);
+
+/* Number of kernel launches so far whose last CTA found every other CTA of
+ * its grid outside the phase's SM range and did the work where it landed
+ * (gate_enter's liveness guard: correct, but off-range).  0 in a healthy
+ * run; synchronizes the device. */
+int bullet_gate_fallbacks(bullet_handle *h, long long *n);
 
 /* One layer step: the prefill batch runs its layers on stream s_prefill and
  * the decode batch runs its layers on stream s_decode.  With BULLET_CORUN

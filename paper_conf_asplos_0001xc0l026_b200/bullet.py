@@ -91,7 +91,7 @@ def lib():
                      "bullet_profile_read", "bullet_launch_count", "bullet_tp_base", "bullet_tp_ipc_handle",
                      "bullet_tp_connect", "bullet_tp_connect_ipc", "bullet_tp_hidden", "bullet_set_split",
                      "bullet_get_colocation", "bullet_set_colocation", "bullet_trace_enable",
-                     "bullet_trace_read"):
+                     "bullet_trace_read", "bullet_sm_dies", "bullet_gate_fallbacks"):
             getattr(L, name).restype = c_int
         L.bullet_create.argtypes = [ctypes.POINTER(ModelCfg), ctypes.POINTER(KvPool), c_void_p,
                                     ctypes.c_char_p, ctypes.POINTER(c_void_p)]
@@ -100,6 +100,8 @@ def lib():
         L.bullet_set_layer_weights.argtypes = [c_void_p, c_int, ctypes.POINTER(LayerWeights)]
         L.bullet_num_sms.argtypes = [c_void_p, ctypes.POINTER(c_int), ctypes.POINTER(c_int)]
         L.bullet_sm_order.argtypes = [c_void_p, P_i32, c_int]
+        L.bullet_sm_dies.argtypes = [c_void_p, P_i32, c_int]
+        L.bullet_gate_fallbacks.argtypes = [c_void_p, ctypes.POINTER(ctypes.c_longlong)]
         L.bullet_step.argtypes = [c_void_p, ctypes.POINTER(CBatch), ctypes.POINTER(CBatch), c_int, c_int,
                                   c_void_p, c_void_p]
         L.bullet_step_ranges.argtypes = [c_void_p, ctypes.POINTER(CBatch), ctypes.POINTER(CBatch), c_int, c_int,
@@ -371,6 +373,17 @@ class Bullet:
         n = c_int()
         _check(lib().bullet_trace_read(self.h, rec.ctypes.data, meta.ctypes.data, cap, ctypes.byref(n)))
         return rec[:n.value], meta[:n.value]
+
+    def sm_dies(self):
+        """Die (0 / 1, -1 unknown) of each SM of sigma, in sigma order."""
+        d = (ctypes.c_int32 * self.n_sms)()
+        _check(lib().bullet_sm_dies(self.h, d, self.n_sms))
+        return list(d)
+
+    def gate_fallbacks(self) -> int:
+        n = ctypes.c_longlong()
+        _check(lib().bullet_gate_fallbacks(self.h, ctypes.byref(n)))
+        return n.value
 
     def launch_count(self) -> int:
         n = ctypes.c_longlong()

@@ -25,6 +25,7 @@ struct Launch {
                      // a captured graph then follows bullet_set_split at replay
   int* ctr;        // work counter, zero at launch
   int* burn;       // CTAs that left out of range (zero at launch; nullable)
+  int* fallback;   // handle-wide count of launches whose last CTA worked off-range (nullable)
   int32_t* log;    // smid log (nullable): [0] = count, then {launch, unit, smid, phase}
   int log_cap;
   int launch_id;
@@ -88,7 +89,10 @@ __device__ __forceinline__ bool gate_enter(const Launch& L) {
   if (L.pdl) pdl_wait();
   if (!L.burn) return false;
   int last = 0;   // (no shared memory: kernels align their dynamic smem base)
-  if (threadIdx.x == 0) last = atomicAdd(L.burn, 1) == (int)(gridDim.x * gridDim.y * gridDim.z) - 1;
+  if (threadIdx.x == 0) {
+    last = atomicAdd(L.burn, 1) == (int)(gridDim.x * gridDim.y * gridDim.z) - 1;
+    if (last && L.fallback) atomicAdd(L.fallback, 1);   // reported by bullet_gate_fallbacks
+  }
   return __syncthreads_or(last) != 0;
 }
 

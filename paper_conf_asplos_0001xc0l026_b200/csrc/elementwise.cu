@@ -351,6 +351,42 @@ cudaError_t launch_set_gates(Gate* d_gates, const Gate& pre, const Gate& dec, cu
   return cudaGetLastError();
 }
 
+// Die probe (KI1b): the B200 is two dies, each with half of the L2; an L2
+// hit on the SM's own die is ~10 % faster than one on the other die
+// (B300_MICROARCH: 234 vs 262 cycles).  Every CTA spins (so the first wave
+// spreads over all SMs), touches the n lines once, then times a dependent
+// ld.global.cg to each line (min of 8) and records the cycles under its smid.
+__global__ void k_die_probe(const uint4* lines, int n_lines, int stride4, uint32_t* lat) {
+  const long long t0 = clock64();
+  while (clock64() - t0 < 100000) {
+  }
+  if (threadIdx.x != 0) return;
+  const uint32_t s = smid();
+  if (s >= 256) return;
+  // the lines hold zeros: acc stays 0 at run time, but every address depends
+  // on the previous load's value (no overlap), and each clock read follows
+  // the add that consumes the load (volatile asm keeps the order)
+  uint32_t acc = 0;
+  for (int j = 0; j < n_lines; ++j) acc += __ldcg(lines + (size_t)j * stride4).x;
+  for (int j = 0; j < n_lines; ++j) {
+    uint32_t best = 0xffffffffu;
+    for (int r = 0; r < 8; ++r) {
+      const uint4* p = lines + (size_t)j * stride4 + acc;
+      long long c0, c1;
+      asm volatile("mov.u64 %0, %%clock64;" : "=l"(c0) :: "memory");
+      const uint4 v = __ldcg(p);
+      asm volatile("add.u32 %0, %0, %1;" : "+r"(acc) : "r"(v.x) : "memory");
+      asm volatile("mov.u64 %0, %%clock64;" : "=l"(c1) :: "memory");
+      best = min(best, (uint32_t)(c1 - c0));
+    }
+    lat[s * n_lines + j] = best;
+  }
+  if (acc == 0x12345678u) lat[0] = 0;
+}
+cudaError_t launch_die_probe(const void* lines, int n_lines, int stride_bytes, uint32_t* lat, int grid, cudaStream_t st) {
+  k_die_probe<<<grid, 32, 0, st>>>(reinterpret_cast<const uint4*>(lines), n_lines, stride_bytes / 16, lat);
+  return cudaGetLastError();
+}
 cudaError_t launch_probe(int* out, int n, cudaStream_t st) {
   k_probe<<<n, 32, 0, st>>>(out, n);
   return cudaGetLastError();
@@ -373,6 +409,7 @@ cudaError_t preload_elementwise() {
   cudaError_t e = cudaFuncGetAttributes(&f, k_plan);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_set_gates);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_probe);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_die_probe);
   if (e == cudaSuccess) e = preload_elt_t<float>();
   if (e == cudaSuccess) e = preload_elt_t<__nv_bfloat16>();
   return e;

@@ -187,6 +187,7 @@ cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);   // grid sized to 
 cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_stream_mc(const uint8_t* src, size_t bytes, int mc, int grid, uint32_t* sink, cudaStream_t st);
 cudaError_t launch_probe(int* out_smid, int n, cudaStream_t st);
+cudaError_t launch_die_probe(const void* lines, int n_lines, int stride_bytes, uint32_t* lat, int grid, cudaStream_t st);
 cudaError_t launch_set_gates(Gate* d_gates, const Gate& pre, const Gate& dec, cudaStream_t st);
 
 // Lazy module loading (CUDA default) loads a kernel at its first launch

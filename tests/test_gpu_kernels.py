@@ -356,3 +356,42 @@ def test_decode_layer_long_contexts_vs_oracle():
         mx, mr = compare(b.hidden.cpu().numpy(), ref[name])
         assert mx <= 2e-2 and mr <= 1e-3, (name, mx, mr)
     S.bl.close()
+
+
+def test_die_probe_and_sigma_orders(B):
+    """Die probe (KI1b): every SM is assigned one of the two dies, both dies
+    hold a plausible share of the 148 SMs, the two SMs of a TPC pair agree,
+    a second probe agrees SM by SM, and the sigma orders keep the probed SM
+    set and the TPC pairs: "die" puts one die's SMs first, "interleave"
+    alternates dies pair by pair (BULLET_SIGMA, read at create)."""
+    import os
+    from collections import Counter
+    bl, _ = _handle(B, SMALL)
+    sig, dies = bl.sm_order(), bl.sm_dies()
+    assert set(dies) == {0, 1}, Counter(dies)
+    c = Counter(dies)
+    assert 50 <= c[0] <= 98 and 50 <= c[1] <= 98, c
+    by_sm = dict(zip(sig, dies))
+    for i in range(0, len(sig) - 1, 2):
+        assert by_sm[sig[i]] == by_sm[sig[i + 1]], (sig[i], sig[i + 1])
+    bl.close()
+    try:
+        for pol in ("die", "interleave", "sorted"):
+            os.environ["BULLET_SIGMA"] = pol
+            b2, _ = _handle(B, SMALL)
+            s2, d2 = b2.sm_order(), b2.sm_dies()
+            b2.close()
+            assert sorted(s2) == sorted(sig)
+            assert all(dict(zip(s2, d2))[s] == by_sm[s] for s in s2)   # the probe is reproducible
+            pairs = [(s2[i], s2[i + 1]) for i in range(0, len(s2) - 1, 2)]
+            assert all(abs(a - b) == 1 for a, b in pairs) or pol == "sorted"
+            pd = [d2[i] for i in range(0, len(d2) - 1, 2)]
+            if pol == "die":
+                assert pd == sorted(pd)                       # one die, then the other
+            elif pol == "interleave":
+                n = 2 * min(pd.count(0), pd.count(1))
+                assert all(pd[i] != pd[i + 1] for i in range(0, n - 1, 2))
+            else:
+                assert s2 == sorted(s2)
+    finally:
+        os.environ.pop("BULLET_SIGMA", None)
