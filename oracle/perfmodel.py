@@ -105,15 +105,19 @@ def layer_time(shape: dict, P: dict, m: int, corun_m: int) -> float:
     M = P["M"]
     C, B = P["C_tflops"] * 1e12, P["B_gbs"] * 1e9
     d_c, d_b = interp(P["d_c"], m), interp(P["d_b"], m)
+    # R-12b: the attention kernel's own decay tables (default: the same)
+    d_ca = interp(P["d_c_attn"], m) if "d_c_attn" in P else d_c
+    d_ba = interp(P["d_b_attn"], m) if "d_b_attn" in P else d_b
     # R-11/R-12: co-location factors, a constant or piecewise linear in the
     # kernel's own SM count m (fitted from co-run points, like d_c, d_b)
     def co(v):
         return interp(v, m) if isinstance(v, dict) else v
     p_c, p_b = (co(P["p_c"]), co(P["p_b"])) if corun_m > 0 else (1.0, 1.0)
     total = 0.0
-    for _, c, b, g, occ in layer_kernels(shape, P, m):
+    for name, c, b, g, occ in layer_kernels(shape, P, m):
         s = wave_idle(g, m * occ)          # Reading R-13: M := m_i x CTAs per SM
-        total += kernel_time(c, b, C, B, M, m, d_c, d_b, p_c, p_b, s)
+        dc, db = (d_ca, d_ba) if name == "attn" else (d_c, d_b)
+        total += kernel_time(c, b, C, B, M, m, dc, db, p_c, p_b, s)
     return total
 
 

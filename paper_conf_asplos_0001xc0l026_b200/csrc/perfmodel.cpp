@@ -112,12 +112,17 @@ bool PerfParams::parse(const char* json, std::string* err) {
     p_c = p_b = 1.0;
   }
   getv("d_c.m", dc_m); getv("d_c.v", dc_v); getv("d_b.m", db_m); getv("d_b.v", db_v);
+  dca_m.clear(); dca_v.clear(); dba_m.clear(); dba_v.clear();
+  getv("d_c_attn.m", dca_m); getv("d_c_attn.v", dca_v); getv("d_b_attn.m", dba_m); getv("d_b_attn.v", dba_v);
+  if (dca_m.empty()) { dca_m = dc_m; dca_v = dc_v; }   // not given: the attention kernel shares d_c / d_b
+  if (dba_m.empty()) { dba_m = db_m; dba_v = db_v; }
   get1("tiles.gemm_bm", gemm_bm); get1("tiles.gemm_bn", gemm_bn); get1("tiles.gemm_bk", gemm_bk);
   get1("tiles.min_k_blocks", min_k_blocks); get1("tiles.attn_bq", attn_bq);
   get1("tiles.rows_per_unit", rows_per_unit);
   get1("occ.gemm", occ_gemm); get1("occ.attn", occ_attn); get1("occ.elem", occ_elem);
   if (dc_m.size() != dc_v.size() || db_m.size() != db_v.size() || dc_m.empty() || db_m.empty() ||
-      pc_m.size() != pc_v.size() || pb_m.size() != pb_v.size() || pc_m.empty() || pb_m.empty()) {
+      pc_m.size() != pc_v.size() || pb_m.size() != pb_v.size() || pc_m.empty() || pb_m.empty() ||
+      dca_m.size() != dca_v.size() || dba_m.size() != dba_v.size()) {
     if (err) *err = "perf params: d_c / d_b / p_c / p_b tables malformed";
     return false;
   }
@@ -131,6 +136,7 @@ void PerfParams::set_default(int n_sms) {
   db_m = {1.0, (double)n_sms}; db_v = {1.0, 1.0};
   pc_m = {1.0, (double)n_sms}; pc_v = {1.0, 1.0};
   pb_m = {1.0, (double)n_sms}; pb_v = {1.0, 1.0};
+  dca_m = dc_m; dca_v = dc_v; dba_m = db_m; dba_v = db_v;
   p_c = p_b = 1.0;
 }
 
@@ -197,11 +203,15 @@ std::vector<KernelCost> layer_kernels(const PhaseShape& s, const PerfParams& P, 
 double layer_time(const PhaseShape& s, const PerfParams& P, int m, int corun_m) {
   if (m <= 0) return std::numeric_limits<double>::infinity();
   const double C = P.C_tflops * 1e12, B = P.B_gbs * 1e9, M = P.M;
-  const double dc = interp(P.dc_m, P.dc_v, m), db = interp(P.db_m, P.db_v, m);
+  const double dc0 = interp(P.dc_m, P.dc_v, m), db0 = interp(P.db_m, P.db_v, m);
+  const double dca = P.dca_m.empty() ? dc0 : interp(P.dca_m, P.dca_v, m);
+  const double dba = P.dba_m.empty() ? db0 : interp(P.dba_m, P.dba_v, m);
   const double pc = corun_m > 0 ? interp(P.pc_m, P.pc_v, m) * P.p_c : 1.0;
   const double pb = corun_m > 0 ? interp(P.pb_m, P.pb_v, m) * P.p_b : 1.0;
   double total = 0;
   for (const auto& k : layer_kernels(s, P, m)) {
+    const bool attn = !strcmp(k.name, "attn");
+    const double dc = attn ? dca : dc0, db = attn ? dba : db0;
     const double sidle = wave_idle(k.g, (double)m * k.occ);
     const double tc = k.c / C * M / (m * dc * pc);
     const double tb = k.b / B * M / (m * db * pb);

@@ -9,6 +9,10 @@ namespace bl {
 struct PerfParams {
   double M = 148, C_tflops = 1649.5, B_gbs = 6549.4;
   std::vector<double> dc_m{1, 148}, dc_v{1, 1}, db_m{1, 148}, db_v{1, 1};
+  // the attention kernel's own d_c(m), d_b(m) (R-12b; default: the tables
+  // above): its roofline efficiency differs from the GEMMs', so batches
+  // with different KV / weight byte mixes need both
+  std::vector<double> dca_m, dca_v, dba_m, dba_v;
   // co-location factors p_c(m), p_b(m): piecewise linear in the kernel's own
   // SM count m (a JSON number = constant), times the online scale (P:L195
   // estimator feedback, bullet_set_colocation)

@@ -28,6 +28,7 @@ M_GRID = [16, 32, 48, 64, 80, 96, 112, 128, 148]
 PRE_SHAPES = [[512], [1024], [2048], [4096], [8192], synth.workload("sharegpt-8b").prefill_lens]
 DEC_SHAPES = [(bs, cl) for bs in (32, 64, 128, 256) for cl in (512, 1024, 2048, 4096)]
 L_CO = 16
+L_DEC = 4   # decode layer-steps per isolated decode point
 # co-run points on the split grid the bench sweeps, with the bench's own
 # request mixes (config 2: ShareGPT-shaped prompts x 128 decodes @ ~1k;
 # config 3: 8k prompt x 256 decodes @ ~4k) plus two off-grid mixes
@@ -95,9 +96,10 @@ def measure():
             pts.append({"kind": "pre", "q": lens, "c": [0] * len(lens), "m": m, "co": 0, "ms": tp})
     for bs, cl in DEC_SHAPES:
         d, _ = R.batch([1] * bs, [cl] * bs, 0)
+        d.layer_end = L_DEC   # per-layer time of a multi-layer decode step, as the co-run step runs it
         for m in M_GRID:
             _, td = R.time(None, d, R.N - m)
-            pts.append({"kind": "dec", "q": [1] * bs, "c": [cl] * bs, "m": m, "co": 0, "ms": td})
+            pts.append({"kind": "dec", "q": [1] * bs, "c": [cl] * bs, "m": m, "co": 0, "ms": td / L_DEC})
     for lens, (bs, cl), p in CORUN:
         pre, used = R.batch(lens, [0] * len(lens))
         dec, _ = R.batch([1] * bs, [cl] * bs, used)
@@ -134,20 +136,31 @@ def fit(N, pts, m_shape):
     test = [p for i, p in enumerate(pts) if i in held]
     P = base_params(N)
     grid = np.exp(np.linspace(np.log(0.05), np.log(3.0), 48))
-    dc_v, db_v = [], []
+    # per SM count m: the decode points fix the bandwidth decays of the GEMMs
+    # and of the attention kernel (d_b, d_b_attn: the KV / weight byte mix
+    # varies over the shapes), then the prefill points the compute decays
+    # (d_c, d_c_attn) — R-12 / R-12b
+    dc_v, db_v, dca_v, dba_v = [], [], [], []
     for m in M_GRID:
-        iso = [p for p in train if p["co"] == 0 and p["m"] == m]
-        best = (math.inf, 1.0, 1.0)
-        for dc, db in itertools.product(grid, grid):
-            Q = dict(P, d_c={"m": [1, N], "v": [dc, dc]}, d_b={"m": [1, N], "v": [db, db]})
-            pm = predictor(m_shape, Q, N)
-            err = sum((math.log(pm.predict_us(p["q"], p["c"], m, 0) / 1e3) - math.log(p["ms"])) ** 2 for p in iso)
-            pm.close()
-            if err < best[0]:
-                best = (err, dc, db)
-        dc_v.append(best[1]); db_v.append(best[2])
+        def search(kind, keys, fixed):
+            iso = [p for p in train if p["co"] == 0 and p["m"] == m and p["kind"] == kind]
+            best = (math.inf, 1.0, 1.0)
+            for x, y in itertools.product(grid, grid):
+                Q = dict(P, **fixed, **{keys[0]: {"m": [1, N], "v": [x, x]}, keys[1]: {"m": [1, N], "v": [y, y]}})
+                pm = predictor(m_shape, Q, N)
+                err = sum((math.log(pm.predict_us(p["q"], p["c"], m, 0) / 1e3) - math.log(p["ms"])) ** 2 for p in iso)
+                pm.close()
+                if err < best[0]:
+                    best = (err, x, y)
+            return best[1], best[2]
+        db, dba = search("dec", ("d_b", "d_b_attn"), {})
+        fixed = {"d_b": {"m": [1, N], "v": [db, db]}, "d_b_attn": {"m": [1, N], "v": [dba, dba]}}
+        dc, dca = search("pre", ("d_c", "d_c_attn"), fixed)
+        dc_v.append(dc); db_v.append(db); dca_v.append(dca); dba_v.append(dba)
     P["d_c"] = {"m": M_GRID, "v": [float(x) for x in dc_v]}
     P["d_b"] = {"m": M_GRID, "v": [float(x) for x in db_v]}
+    P["d_c_attn"] = {"m": M_GRID, "v": [float(x) for x in dca_v]}
+    P["d_b_attn"] = {"m": M_GRID, "v": [float(x) for x in dba_v]}
     # co-location factors as functions of the phase's own SM count (R-12):
     # prefill co-run points fit p_c(m) (compute-bound kernels), decode ones
     # p_b(m) (bandwidth-bound), each grid point from the points nearest to it
@@ -229,6 +242,14 @@ def main():
     if len(sys.argv) > 1 and sys.argv[1] == "--evaluate":
         pp = os.path.join(ROOT, "profiles", "perf_params_b200.json")
         print(json.dumps(evaluate(pp, pp.replace(".json", "_points.json"))))
+        return
+    if len(sys.argv) > 2 and sys.argv[1] == "--refit":   # fit again from saved points (host only)
+        pts = json.load(open(sys.argv[2]))
+        out = sys.argv[3] if len(sys.argv) > 3 else sys.argv[2].replace("_points.json", ".json")
+        P = fit(148, pts, synth.MODELS["llama3.1-8b"])
+        P["fit"]["points"] = os.path.basename(sys.argv[2])
+        json.dump(P, open(out, "w"), indent=1)
+        print(json.dumps(P["fit"]))
         return
     out = sys.argv[1] if len(sys.argv) > 1 else os.path.join(ROOT, "profiles", "perf_params_b200.json")
     t0 = time.time()
