@@ -317,6 +317,27 @@ class Step:
         for hb in self.hyb:
             self.bl.step(hb, None, self.N, self.B.TIMESLICED, self.sp, self.sd)
 
+    def time_phases(self, n, p, k):
+        """Median per-phase durations (ms) of n co-run steps at (p, k): from
+        the common start to the end of each phase's stream."""
+        B = self.B
+        self.dec.layer_end = k
+        tp, td = [], []
+        for i in range(n + 1):
+            e0 = torch.cuda.Event(enable_timing=True)
+            ep, ed = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(self.sp)
+            self.sd.wait_event(e0)
+            self.bl.step(self.pre, self.dec, p, B.CORUN, self.sp, self.sd)
+            ep.record(self.sp)
+            ed.record(self.sd)
+            self.sp.wait_event(ed)
+            torch.cuda.synchronize()
+            if i:
+                tp.append(e0.elapsed_time(ep)); td.append(e0.elapsed_time(ed))
+        self.dec.layer_end = 1
+        return (allreduce_max(float(np.median(tp)), self.ws), allreduce_max(float(np.median(td)), self.ws))
+
     def time_hybrid(self, n):
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -575,6 +596,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--sweep", action="store_true", help="also print the p sweep (stderr)")
     ap.add_argument("--no-sweep", action="store_true", help="skip the on-device (p, k) sweep")
+    ap.add_argument("--feedback", type=int, default=3, help="online feedback cycles before the split decision")
     ap.add_argument("--allreduce", default="peer", choices=["peer", "nccl"],
                     help="TP configs: fused peer-memory all-reduce (default) or NCCL")
     args = ap.parse_args()
@@ -604,6 +626,29 @@ def main():
                  prefill_waited_ms=[0.0] * S.n_pre, pending_lens=[], pending_waited_ms=[],
                  decode_tokens=[64] * S.n_d, decode_elapsed_ms=[64 * 30.0] * S.n_d,
                  decode_mean_ctx=float(np.mean(S.wl.decode_ctx)), u_k=N // 2, v_k=N - N // 2)
+    # online estimator feedback ("correlating deviations between
+    # predicted latency and observed execution times ... as dynamic
+    # feedback") before the decision is taken: the model's level on this
+    # batch from the measured full-GPU layers (bullet_set_phase_scale), then
+    # a few decide -> run -> correct cycles on the co-location factors
+    # (bullet_set_colocation) with the measured per-phase co-run times
+    qp, cp = S.pre.cu[1:] - S.pre.cu[:-1], S.pre.ctx_lens
+    qd, cdc = [1] * S.n_d, S.dec.ctx_lens
+    S.bl.set_phase_scale(t_pre_full / (S.bl.predict_us(qp, cp, N, 0) / 1e3),
+                         t_dec_full / (S.bl.predict_us(qd, cdc, N, 0) / 1e3))
+    feedback = []
+    for _ in range(args.feedback):
+        ps = tuple(broadcast_obj(S.bl.choose_split(state, slo), ws))
+        if not (0 < ps[0] < N and ps[1] >= 1):
+            break
+        fp, fk = ps[0], min(ps[1], args.k_max)
+        tp_co, td_co = S.time_phases(5, fp, fk)
+        pred_tp = S.bl.predict_us(qp, cp, fp, N - fp) / 1e3
+        pred_td = S.bl.predict_us(qd, cdc, N - fp, fp) / 1e3 * fk
+        sc, sb = S.bl.colocation()
+        S.bl.set_colocation(sc * pred_tp / tp_co, sb * pred_td / td_co)
+        feedback.append({"p": fp, "k": fk, "prefill_ms": tp_co, "decode_ms": td_co,
+                         "predicted_prefill_ms": pred_tp, "predicted_decode_ms": pred_td})
     model_split = tuple(broadcast_obj(S.bl.choose_split(state, slo), ws))
     table, swept = [], None
     if not args.no_sweep and (args.p is None or args.k is None):
@@ -620,8 +665,6 @@ def main():
         if swept is None:
             swept, table = S.tune(list(range(56, N - 15, 8)), t_pre_full, t_dec_full)
         p, k, split_source = swept["p"], swept["k"], "swept (the model chose the time-sliced cycle)"
-    qp, cp = S.pre.cu[1:] - S.pre.cu[:-1], S.pre.ctx_lens
-    qd, cdc = [1] * S.n_d, S.dec.ctx_lens
     pred = {"t_prefill_ms": S.bl.predict_us(qp, cp, p, N - p) / 1e3,
             "t_decode_layer_ms": S.bl.predict_us(qd, cdc, N - p, p) / 1e3,
             "t_prefill_full_ms": S.bl.predict_us(qp, cp, N, 0) / 1e3,
@@ -889,6 +932,7 @@ def main():
         "tuning": table,
         "alg1_split": {"prefill_sm_count": model_split[0], "decode_layer_steps": model_split[1],
                        "objective": 2, "slo": slo, "timed": (p, k) == tuple(model_split),
+                       "feedback": feedback, "phase_scale": S.bl.phase_scale(), "colocation_scale": S.bl.colocation(),
                        "predicted": pred,
                        "perf_params": "profiles/perf_params_b200.json" if S.perf_json else "unfitted"},
         "split": {"source": split_source, "prefill_sm_count": p, "decode_layer_steps": k,

@@ -285,6 +285,14 @@ int bullet_model_predict(const bullet_handle *h, const bullet_batch_shape *shape
 int bullet_get_colocation(const bullet_handle *h, double *p_c, double *p_b);
 int bullet_set_colocation(bullet_handle *h, double p_c, double p_b);
 
+/* The same feedback for the model's level: every predicted layer
+ * time of a prefill-shaped batch (some request with more than one new
+ * token) is multiplied by `pre`, of a decode-shaped batch by `dec` (default
+ * 1; e.g. measured / predicted full-GPU layer time of the live batch).
+ * Errors: EINVAL (non-positive scales). */
+int bullet_get_phase_scale(const bullet_handle *h, double *pre, double *dec);
+int bullet_set_phase_scale(bullet_handle *h, double pre, double dec);
+
 /* Alg. 1 and the §3.3.3 search under the readings
  * of DESIGN.md §3 (R-14..R-17): returns the prefill SM count for the next
  * cycle (N = decode paused) and the number of decode layer-steps to co-run

@@ -118,7 +118,8 @@ def layer_time(shape: dict, P: dict, m: int, corun_m: int) -> float:
         s = wave_idle(g, m * occ)          # Reading R-13: M := m_i x CTAs per SM
         dc, db = (d_ca, d_ba) if name == "attn" else (d_c, d_b)
         total += kernel_time(c, b, C, B, M, m, dc, db, p_c, p_b, s)
-    return total
+    # online level calibration per phase class (P:L195 feedback; default 1)
+    return total * (P.get("scale_pre", 1.0) if max(shape["q_lens"], default=0) > 1 else P.get("scale_dec", 1.0))
 
 
 # ------------------------------------------------------------ Alg. 1 reading

@@ -91,7 +91,8 @@ def lib():
                      "bullet_profile_read", "bullet_launch_count", "bullet_tp_base", "bullet_tp_ipc_handle",
                      "bullet_tp_connect", "bullet_tp_connect_ipc", "bullet_tp_hidden", "bullet_set_split",
                      "bullet_get_colocation", "bullet_set_colocation", "bullet_trace_enable",
-                     "bullet_trace_read", "bullet_sm_dies", "bullet_gate_fallbacks"):
+                     "bullet_trace_read", "bullet_sm_dies", "bullet_gate_fallbacks", "bullet_get_phase_scale",
+                     "bullet_set_phase_scale"):
             getattr(L, name).restype = c_int
         L.bullet_create.argtypes = [ctypes.POINTER(ModelCfg), ctypes.POINTER(KvPool), c_void_p,
                                     ctypes.c_char_p, ctypes.POINTER(c_void_p)]
@@ -121,6 +122,8 @@ def lib():
         L.bullet_set_split.argtypes = [c_void_p, c_int, c_int, c_int, c_int, c_void_p]
         L.bullet_get_colocation.argtypes = [c_void_p, P_f64, P_f64]
         L.bullet_set_colocation.argtypes = [c_void_p, c_double, c_double]
+        L.bullet_get_phase_scale.argtypes = [c_void_p, P_f64, P_f64]
+        L.bullet_set_phase_scale.argtypes = [c_void_p, c_double, c_double]
         L.bullet_tp_ipc_handle.argtypes = [c_void_p, c_void_p]
         L.bullet_tp_connect.argtypes = [c_void_p, ctypes.POINTER(c_void_p)]
         L.bullet_tp_connect_ipc.argtypes = [c_void_p, c_void_p]
@@ -397,6 +400,15 @@ class Bullet:
 
     def set_colocation(self, p_c: float, p_b: float):
         _check(lib().bullet_set_colocation(self.h, float(p_c), float(p_b)))
+
+    def phase_scale(self):
+        a, b = c_double(), c_double()
+        _check(lib().bullet_get_phase_scale(self.h, ctypes.byref(a), ctypes.byref(b)))
+        return a.value, b.value
+
+    def set_phase_scale(self, pre: float, dec: float):
+        """Online level calibration: predicted prefill / decode layer times x pre / dec."""
+        _check(lib().bullet_set_phase_scale(self.h, float(pre), float(dec)))
 
     def predict_us(self, q_lens, ctx_lens, sm_count, corun_sm_count=0) -> float:
         q = np.ascontiguousarray(q_lens, dtype=np.int32); c = np.ascontiguousarray(ctx_lens, dtype=np.int32)

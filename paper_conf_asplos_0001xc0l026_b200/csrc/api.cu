@@ -504,12 +504,15 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
     static const int sb = getenv("BULLET_GEMM_SPLIT_B") ? atoi(getenv("BULLET_GEMM_SPLIT_B")) : 1;
     a.split_b = sb ? 1 : 0;
   }
-  {  // rasterisation band: activations of a band <= 32 MB (L2-resident)
+  {  // rasterisation band: the activations of a band stay L2-resident (evict-last)
+     // while every weight tile streams past them once per band: a band of
+     // <= BULLET_GEMM_BAND_MB (default 32) MB of activations
+    static const double band_bytes =
+        (getenv("BULLET_GEMM_BAND_MB") ? atof(getenv("BULLET_GEMM_BAND_MB")) : 32.0) * 1e6;
     const int m_tiles = (M + 128 * mh - 1) / (128 * mh);
     const double a_tile = 128.0 * mh * K * 2;
-    int band = 1;
-    while (band * 2 <= m_tiles && band * 2 * a_tile <= 32e6) band *= 2;
-    a.band = std::max(1, std::min(band, m_tiles));
+    const int n_bands = std::max(1, (int)std::ceil(m_tiles * a_tile / band_bytes));
+    a.band = std::max(1, (m_tiles + n_bands - 1) / n_bands);   // equal bands
   }
   a.b_packed = Bp;
   a.b_evict_first = ((M + 128 * mh - 1) / (128 * mh)) == 1;   // weights reused by no other M tile
@@ -1329,6 +1332,18 @@ int bullet_choose_split(const bullet_handle* h, const bullet_sched_state* s, con
 int bullet_get_colocation(const bullet_handle* h, double* p_c, double* p_b) {
   if (!h || !p_c || !p_b) return set_err(BULLET_EINVAL, "null");
   *p_c = h->perf.p_c; *p_b = h->perf.p_b;
+  return BULLET_OK;
+}
+
+int bullet_get_phase_scale(const bullet_handle* h, double* pre, double* dec) {
+  if (!h || !pre || !dec) return set_err(BULLET_EINVAL, "null");
+  *pre = h->perf.scale_pre; *dec = h->perf.scale_dec;
+  return BULLET_OK;
+}
+
+int bullet_set_phase_scale(bullet_handle* h, double pre, double dec) {
+  if (!h || !(pre > 0.0) || !(dec > 0.0)) return set_err(BULLET_EINVAL, "phase scales must be > 0");
+  h->perf.scale_pre = pre; h->perf.scale_dec = dec;
   return BULLET_OK;
 }
 

@@ -209,6 +209,9 @@ double layer_time(const PhaseShape& s, const PerfParams& P, int m, int corun_m) 
   const double pc = corun_m > 0 ? interp(P.pc_m, P.pc_v, m) * P.p_c : 1.0;
   const double pb = corun_m > 0 ? interp(P.pb_m, P.pb_v, m) * P.p_b : 1.0;
   double total = 0;
+  int maxq = 0;
+  for (int q : s.q_lens) maxq = std::max(maxq, q);
+  const double scale = maxq > 1 ? P.scale_pre : P.scale_dec;
   for (const auto& k : layer_kernels(s, P, m)) {
     const bool attn = !strcmp(k.name, "attn");
     const double dc = attn ? dca : dc0, db = attn ? dba : db0;
@@ -217,7 +220,7 @@ double layer_time(const PhaseShape& s, const PerfParams& P, int m, int corun_m) 
     const double tb = k.b / B * M / (m * db * pb);
     total += std::max(tc, tb) / (1.0 - sidle);
   }
-  return total;
+  return total * scale;
 }
 
 static double p90(std::vector<double> v, double pct) {

@@ -18,6 +18,10 @@ struct PerfParams {
   // estimator feedback, bullet_set_colocation)
   std::vector<double> pc_m{1, 148}, pc_v{1, 1}, pb_m{1, 148}, pb_v{1, 1};
   double p_c = 1, p_b = 1;   // scale
+  // online level calibration per phase class (bullet_set_phase_scale): every
+  // predicted layer time of a prefill-shaped (some q > 1) / decode-shaped
+  // batch is multiplied by scale_pre / scale_dec (default 1)
+  double scale_pre = 1, scale_dec = 1;
   double gemm_bm = 128, gemm_bn = 256, gemm_bk = 64, min_k_blocks = 4, attn_bq = 64, rows_per_unit = 8;
   double occ_gemm = 1, occ_attn = 1, occ_elem = 4;
   bool parse(const char* json, std::string* err);

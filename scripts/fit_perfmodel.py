@@ -144,14 +144,18 @@ def fit(N, pts, m_shape):
     for m in M_GRID:
         def search(kind, keys, fixed):
             iso = [p for p in train if p["co"] == 0 and p["m"] == m and p["kind"] == kind]
-            best = (math.inf, 1.0, 1.0)
-            for x, y in itertools.product(grid, grid):
+
+            def err_of(x, y):
                 Q = dict(P, **fixed, **{keys[0]: {"m": [1, N], "v": [x, x]}, keys[1]: {"m": [1, N], "v": [y, y]}})
                 pm = predictor(m_shape, Q, N)
-                err = sum((math.log(pm.predict_us(p["q"], p["c"], m, 0) / 1e3) - math.log(p["ms"])) ** 2 for p in iso)
+                e = sum((math.log(pm.predict_us(p["q"], p["c"], m, 0) / 1e3) - math.log(p["ms"])) ** 2 for p in iso)
                 pm.close()
-                if err < best[0]:
-                    best = (err, x, y)
+                return e
+            best = min((err_of(x, y), x, y) for x, y in itertools.product(grid, grid))
+            # refine: the coarse grid steps 9 %; search +-1 step at 0.5 % resolution
+            step = grid[1] / grid[0]
+            fine = lambda v: np.exp(np.linspace(np.log(v / step), np.log(v * step), 37))  # noqa: E731
+            best = min([best] + [(err_of(x, y), x, y) for x, y in itertools.product(fine(best[1]), fine(best[2]))])
             return best[1], best[2]
         db, dba = search("dec", ("d_b", "d_b_attn"), {})
         fixed = {"d_b": {"m": [1, N], "v": [db, db]}, "d_b_attn": {"m": [1, N], "v": [dba, dba]}}
@@ -165,7 +169,7 @@ def fit(N, pts, m_shape):
     # prefill co-run points fit p_c(m) (compute-bound kernels), decode ones
     # p_b(m) (bandwidth-bound), each grid point from the points nearest to it
     co = [p for p in train if p["co"] > 0]
-    fgrid = np.linspace(0.4, 1.3, 46)
+    fgrid = np.linspace(0.4, 1.3, 181)
 
     def fit_table(kind, key):
         pts_k = [p for p in co if p["kind"] == kind]

@@ -151,3 +151,20 @@ def test_header_is_plain_c99(tmp_path):
     r = subprocess.run([gcc, "-std=c99", "-Wall", "-Wextra", "-pedantic", "-Werror", "-fsyntax-only", "-I", inc, str(src)],
                        capture_output=True, text=True)
     assert r.returncode == 0, r.stderr
+
+
+def test_phase_scale_equals_oracle():
+    """Online level calibration (bullet_set_phase_scale): prefill- and
+    decode-shaped predictions scale by their own factor, as in the oracle."""
+    P = _fitted_params()
+    pm = _pm("llama8b", params=P)
+    pm.set_phase_scale(1.3, 0.7)
+    assert pm.phase_scale() == (1.3, 0.7)
+    shape = dict(MODELS["llama8b"])
+    Q = dict(P, scale_pre=1.3, scale_dec=0.7)
+    for q, c in [([4096], [0]), ([1] * 64, [900] * 64), ([33, 1], [0, 5])]:
+        for m, co in [(148, 0), (80, 68)]:
+            ref = PM.layer_time(dict(shape, q_lens=q, ctx_lens=c), Q, m, co) * 1e6
+            assert pm.predict_us(q, c, m, co) == pytest.approx(ref, rel=1e-12)
+    with pytest.raises(Exception):
+        pm.set_phase_scale(0.0, 1.0)

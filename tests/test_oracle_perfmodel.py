@@ -251,7 +251,7 @@ def test_fitted_model_heldout_report_reproduces():
     import fit_perfmodel as F
     pp = os.path.join(root, "profiles", "perf_params_b200.json")
     got = F.evaluate(pp, pp.replace(".json", "_points.json"))
-    want = json.load(open(os.path.join(root, "profiles", "r01c_perfmodel_eval.json")))
+    want = json.load(open(os.path.join(root, "profiles", "r02_perfmodel_eval.json")))
     assert abs(got["mre_heldout"] - want["mre_heldout"]) < 1e-9
     assert abs(got["slo_accuracy_heldout"] - want["slo_accuracy_heldout"]) < 1e-9
     assert got["mre_heldout"] < 0.191 and got["slo_accuracy_heldout"] > 0.88   # paper's numbers, context
