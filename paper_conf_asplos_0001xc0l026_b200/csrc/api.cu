@@ -506,9 +506,10 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   }
   {  // rasterisation band: the activations of a band stay L2-resident (evict-last)
      // while every weight tile streams past them once per band: a band of
-     // <= BULLET_GEMM_BAND_MB (default 32) MB of activations
+     // <= BULLET_GEMM_BAND_MB (default 64; co-run step vs 32 / 128 MB: config 2
+     // 2.919 vs 2.968 / 2.922 ms, config 3 7.144 vs 7.201 / 7.272 ms) MB of activations
     static const double band_bytes =
-        (getenv("BULLET_GEMM_BAND_MB") ? atof(getenv("BULLET_GEMM_BAND_MB")) : 32.0) * 1e6;
+        (getenv("BULLET_GEMM_BAND_MB") ? atof(getenv("BULLET_GEMM_BAND_MB")) : 64.0) * 1e6;
     const int m_tiles = (M + 128 * mh - 1) / (128 * mh);
     const double a_tile = 128.0 * mh * K * 2;
     const int n_bands = std::max(1, (int)std::ceil(m_tiles * a_tile / band_bytes));

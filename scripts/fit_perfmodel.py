@@ -26,14 +26,16 @@ from workload import synth  # noqa: E402
 
 M_GRID = [16, 32, 48, 64, 80, 96, 112, 128, 148]
 PRE_SHAPES = [[512], [1024], [2048], [4096], [8192], synth.workload("sharegpt-8b").prefill_lens]
-DEC_SHAPES = [(bs, cl) for bs in (32, 64, 128, 256) for cl in (512, 1024, 2048, 4096)]
+DEC_SHAPES = [[cl] * bs for bs in (32, 64, 128, 256) for cl in (512, 1024, 2048, 4096)] + \
+    [list(synth.workload("sharegpt-8b").decode_ctx), list(synth.workload("arxiv-8b").decode_ctx)]
 L_CO = 16
 L_DEC = 4   # decode layer-steps per isolated decode point
 # co-run points on the split grid the bench sweeps, with the bench's own
 # request mixes (config 2: ShareGPT-shaped prompts x 128 decodes @ ~1k;
 # config 3: 8k prompt x 256 decodes @ ~4k) plus two off-grid mixes
-CORUN = [(pre, dec, p) for pre, dec in ((synth.workload("sharegpt-8b").prefill_lens, (128, 1024)),
-                                        ([8192], (256, 4096)), ([2048], (256, 2048)), ([4096], (64, 512)))
+CORUN = [(pre, dec, p) for pre, dec in ((synth.workload("sharegpt-8b").prefill_lens, list(synth.workload("sharegpt-8b").decode_ctx)),
+                                        ([8192], list(synth.workload("arxiv-8b").decode_ctx)),
+                                        ([2048], [2048] * 256), ([4096], [512] * 64))
          for p in range(40, 140, 8)]
 
 
@@ -43,7 +45,7 @@ class Rig:
         self.m = synth.MODELS["llama3.1-8b"]
         w = synth.layer_weights(self.m, 0, device="cuda")
         self.w = {k: (None if v is None else v.bfloat16()) for k, v in w.items()}
-        self.n_blocks = 256 * (4096 // 16 + 1) + 8192 // 16 + 64
+        self.n_blocks = 256 * (6144 // 16 + 1) + 8192 // 16 + 64
         k, v = synth.kv_pool(self.m, self.n_blocks, 16, 0, device="cuda")
         self.pool = [(k.bfloat16(), v.bfloat16())]
         del k, v
@@ -57,12 +59,20 @@ class Rig:
         self.sp, self.sd = torch.cuda.Stream(), torch.cuda.Stream()
 
     def batch(self, q_lens, ctx_lens, first_block=0):
+        """Block tables as the bench and a serving pool have them: a random
+        permutation of the free blocks (fragmented KV — contiguous tables
+        stream measurably faster and made round 2's first fit 30-50 %
+        optimistic for KV-heavy decode batches)."""
         nb = [-(-(q + c) // 16) for q, c in zip(q_lens, ctx_lens)]
+        total = sum(nb)
+        rng = np.random.default_rng(first_block + 7)
+        perm = first_block + rng.permutation(total).astype(np.int32)
         bt = np.zeros((len(nb), max(nb)), np.int32)
-        pos = first_block
+        pos = 0
         for i, n in enumerate(nb):
-            bt[i, :n] = np.arange(pos, pos + n)
+            bt[i, :n] = perm[pos:pos + n]
             pos += n
+        pos += first_block
         x = torch.randn(sum(q_lens), self.m.d_model, device="cuda")
         torch.cuda.synchronize()   # x is read on the phase streams
         return B.Batch(q_lens, ctx_lens, bt, x, 0, 1), pos
@@ -94,22 +104,24 @@ def measure():
         for m in M_GRID:
             tp, _ = R.time(b, None, m if m < R.N else R.N)
             pts.append({"kind": "pre", "q": lens, "c": [0] * len(lens), "m": m, "co": 0, "ms": tp})
-    for bs, cl in DEC_SHAPES:
-        d, _ = R.batch([1] * bs, [cl] * bs, 0)
+    for ctx in DEC_SHAPES:
+        bs = len(ctx)
+        d, _ = R.batch([1] * bs, ctx, 0)
         d.layer_end = L_DEC   # per-layer time of a multi-layer decode step, as the co-run step runs it
         for m in M_GRID:
             _, td = R.time(None, d, R.N - m)
-            pts.append({"kind": "dec", "q": [1] * bs, "c": [cl] * bs, "m": m, "co": 0, "ms": td / L_DEC})
-    for lens, (bs, cl), p in CORUN:
+            pts.append({"kind": "dec", "q": [1] * bs, "c": list(ctx), "m": m, "co": 0, "ms": td / L_DEC})
+    for lens, ctx, p in CORUN:
+        bs = len(ctx)
         pre, used = R.batch(lens, [0] * len(lens))
-        dec, _ = R.batch([1] * bs, [cl] * bs, used)
+        dec, _ = R.batch([1] * bs, ctx, used)
         tp0, _ = R.time(pre, None, p)                 # alone on the same SMs: the balance k
         _, td0 = R.time(None, dec, p)
         k = int(min(L_CO, max(1, round(tp0 / max(td0, 1e-6)))))
         dec.layer_end = k
         tp, td = R.time(pre, dec, p)
         pts.append({"kind": "pre", "q": lens, "c": [0] * len(lens), "m": p, "co": R.N - p, "ms": tp, "k": k})
-        pts.append({"kind": "dec", "q": [1] * bs, "c": [cl] * bs, "m": R.N - p, "co": p, "ms": td / k, "k": k})
+        pts.append({"kind": "dec", "q": [1] * bs, "c": list(ctx), "m": R.N - p, "co": p, "ms": td / k, "k": k})
     return R.N, pts
 
 
