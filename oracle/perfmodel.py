@@ -166,6 +166,9 @@ def evaluate_split(P, model, state, slo, u, v):
     return p90(ttft, pct), p90(tpot, pct), t_p
 
 
+GAIN_TOL = 0.03   # R-23: the model's resolution for the gain objective
+
+
 def candidates(P, slo, gran):
     """Decode SM counts v (prefill gets N - v) with v >= v_min and u >= gran."""
     N = P["M"]
@@ -262,7 +265,7 @@ def choose_split(P, model, state, slo, gran=2):
                            [int(math.floor(state["decode_mean_ctx"] + 0.5))] * len(state["decode_tokens"]))
         tpN = layer_time(pre, P, N, 0) * 1e3 if state["prefill_lens"] else 0.0
         tdN = layer_time(dec, P, N, 0) * 1e3
-        best, best_g = (None, 1), -1.0
+        cs = []
         for v in cands:
             if ev[v][0] > 1.0 or ev[v][1] > 1.0:
                 continue
@@ -271,10 +274,15 @@ def choose_split(P, model, state, slo, gran=2):
                 continue
             k0 = max(1, int(math.floor(t_p / t_d)))
             for k in (k0, k0 + 1):
-                g = (tpN + k * tdN) / max(t_p, k * t_d)
-                if g > best_g:
-                    best, best_g = (v, k), g
-        return best, best_g
+                cs.append((v, k, (tpN + k * tdN) / max(t_p, k * t_d)))
+        if not cs:
+            return (None, 1), -1.0
+        best_g = max(c[2] for c in cs)
+        # gains within GAIN_TOL of the best are within the model's resolution:
+        # the larger prefill share wins, then the larger gain, then smaller k
+        near = [c for c in cs if c[2] >= (1.0 - GAIN_TOL) * best_g]
+        v, k, _ = min(near, key=lambda c: (c[0], -c[2], c[1]))
+        return (v, k), best_g
 
     if ok_t and ok_d and slo.get("objective", 0) == 2:
         (vb, kb), g = max_gain()

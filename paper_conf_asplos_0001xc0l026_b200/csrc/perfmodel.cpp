@@ -262,6 +262,10 @@ static Eval evaluate(const PerfParams& P, const PhaseShape& model, const SchedSt
   return {p90(ttft, slo.percentile), p90(tpot, slo.percentile), t_p};
 }
 
+// R-23: gains within this fraction of the best are within the model's
+// resolution (held-out MRE ~5 %); among them prefill is prioritised
+constexpr double GAIN_TOL = 0.03;
+
 void choose_split(const PerfParams& P, const PhaseShape& model, const SchedState& S,
                   const Slo& slo, int gran, int* prefill_sms, int* decode_steps) {
   const int N = (int)P.M, L = S.total_layers;
@@ -363,6 +367,9 @@ void choose_split(const PerfParams& P, const PhaseShape& model, const SchedState
   // of the same work over the co-run cycle (north_star's target ratio, the
   // paper's co-run-vs-time-sliced axis, P:L7 / P:L155).  Ties: larger gain,
   // then the larger prefill share, then the smaller k.  Returns the gain.
+  // Ties within the model's resolution (R-23: gains within GAIN_TOL of the
+  // best) go to the larger prefill share ("prioritize prefill"), then
+  // the larger gain, then the smaller k.  Returns the best gain.
   auto max_gain = [&](int* best_v, int* best_k) -> double {
     PhaseShape pre = model, dec = model;
     pre.q_lens = S.prefill_lens; pre.ctx_lens.assign(S.prefill_lens.size(), 0);
@@ -370,8 +377,9 @@ void choose_split(const PerfParams& P, const PhaseShape& model, const SchedState
     dec.q_lens.assign(S.decode_tokens.size(), 1); dec.ctx_lens.assign(S.decode_tokens.size(), mctx);
     const double tpN = S.prefill_lens.empty() ? 0.0 : layer_time(pre, P, N, 0) * 1e3;
     const double tdN = layer_time(dec, P, N, 0) * 1e3;
+    struct Cand { int v, k; double g; };
+    std::vector<Cand> cs;
     double best_g = -1.0;
-    *best_v = -1; *best_k = 1;
     for (int v : cands) {
       if (ev[v].ttft > 1.0 || ev[v].tpot > 1.0) continue;
       const double t_p = ev[v].t_p, t_d = layer_time(dec, P, v, N - v) * 1e3;
@@ -379,8 +387,15 @@ void choose_split(const PerfParams& P, const PhaseShape& model, const SchedState
       const int k0 = std::max(1, (int)std::floor(t_p / t_d));
       for (int k = k0; k <= k0 + 1; ++k) {
         const double g = (tpN + k * tdN) / std::max(t_p, k * t_d);
-        if (g > best_g) { best_g = g; *best_v = v; *best_k = k; }
+        cs.push_back({v, k, g});
+        best_g = std::max(best_g, g);
       }
+    }
+    *best_v = -1; *best_k = 1;
+    double pick_g = -1.0;
+    for (const Cand& c : cs) {   // candidates in ascending v (cands order), k ascending
+      if (c.g < (1.0 - GAIN_TOL) * best_g) continue;
+      if (*best_v < 0 || c.v < *best_v || (c.v == *best_v && c.g > pick_g)) { *best_v = c.v; *best_k = c.k; pick_g = c.g; }
     }
     return best_g;
   };
