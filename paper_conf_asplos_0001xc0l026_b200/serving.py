@@ -23,6 +23,9 @@ Policies:
               tuned split; a diagnostic of the decision layer, not a policy
   bullet_tput the same with objective 1: when both SLOs hold, the split with
               the most predicted tokens/s among the SLO-feasible ones (R-21)
+  bullet_gain the same with objective 2: when both SLOs hold, the split with
+              the largest predicted gain of the co-run cycle over the same
+              work time-sliced, or a time-sliced cycle when none gains (R-23)
   timesliced  same cycle structure, both phases on all SMs one after the
               other (BULLET_TIMESLICED), k from the model's full-GPU balance
   prefill_first  vLLM-style: while a prefill batch exists decode is paused
@@ -127,11 +130,11 @@ class ServingLoop:
                  slo: Slo = Slo(), prefill_layers_per_cycle: int = 1, max_prefill_tokens: int = 8192,
                  max_decodes: int = 256, k_full: int = 4, chunk_tokens: int = 2048, feedback_model=None,
                  feedback_alpha: float = 0.2, static_split=(88, 6)):
-        assert policy in ("bullet", "bullet_tput", "static", "timesliced", "prefill_first", "chunked")
+        assert policy in ("bullet", "bullet_tput", "bullet_gain", "static", "timesliced", "prefill_first", "chunked")
         self.static_split = static_split   # policy "static": fixed (prefill SMs, decode layer-steps) co-run
-        if policy == "bullet_tput":   # Alg. 1 with the throughput objective among feasible splits (R-21)
+        if policy in ("bullet_tput", "bullet_gain"):   # Alg. 1 with objective 1 (R-21 / R-22) or 2 (R-23)
+            slo = Slo(**{**slo.__dict__, "objective": 1 if policy == "bullet_tput" else 2})
             policy = "bullet"
-            slo = Slo(**{**slo.__dict__, "objective": 1})
         self.L, self.N = n_layers, n_sms
         self.step, self.choose, self.policy = step, choose, policy
         self.alloc, self.slo = allocator, slo

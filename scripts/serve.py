@@ -97,7 +97,7 @@ def main():
     ap.add_argument("--rate", type=float, default=60.0, help="requests / s (Poisson)")
     ap.add_argument("--duration", type=float, default=10.0, help="seconds of arrivals")
     ap.add_argument("--layers", type=int, default=32)
-    ap.add_argument("--policies", nargs="+", default=["bullet", "bullet_tput", "timesliced", "prefill_first",
+    ap.add_argument("--policies", nargs="+", default=["bullet", "bullet_tput", "bullet_gain", "timesliced", "prefill_first",
                                                        "chunked"])
     ap.add_argument("--chunk-tokens", type=int, default=2048, help="chunked policy: token budget per iteration")
     ap.add_argument("--max-decodes", type=int, default=256)

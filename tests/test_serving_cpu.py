@@ -54,7 +54,7 @@ def _run(pm, policy, rate=40.0, dur=1.0):
     return trace, rec, alloc, loop, res
 
 
-@pytest.mark.parametrize("policy", ["bullet", "bullet_tput", "static", "timesliced", "prefill_first", "chunked"])
+@pytest.mark.parametrize("policy", ["bullet", "bullet_tput", "bullet_gain", "static", "timesliced", "prefill_first", "chunked"])
 def test_every_request_completes_and_blocks_return(pm, policy):
     trace, rec, alloc, loop, res = _run(pm, policy)
     assert res["finished"] == len(trace) > 10
