@@ -516,6 +516,10 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
     a.band = std::max(1, (m_tiles + n_bands - 1) / n_bands);   // equal bands
   }
   a.b_packed = Bp;
+  {   // L2 prefetch distance of the weight stream (experiments; BULLET_GEMM_PF k-blocks)
+    static const int pf = getenv("BULLET_GEMM_PF") ? atoi(getenv("BULLET_GEMM_PF")) : 0;
+    a.b_pf = pf;
+  }
   a.b_evict_first = ((M + 128 * mh - 1) / (128 * mh)) == 1;   // weights reused by no other M tile
   a.b_rows = N + (epi == EPI_SILU ? silu_half - N / 2 : 0);
   a.partials = h->ph[c.phase].partials;
@@ -615,6 +619,8 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
   AttnArgs a;
   memset(&a, 0, sizeof a);
   a.kv_chunks = 1;
+  static const int dec_pf = getenv("BULLET_DEC_PF") ? atoi(getenv("BULLET_DEC_PF")) : 0;
+  a.dec_pf = dec_pf;
   a.q = q; a.o = o; a.pool_k = h->pk[layer]; a.pool_v = h->pv[layer];
   a.cu = b->d_cu_seqlens; a.ctx = b->d_ctx_lens; a.bt = b->d_block_table;
   a.n_reqs = b->n_reqs; a.max_blocks = b->max_blocks_per_req; a.n_tok = b->n_tokens;

@@ -210,6 +210,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
     v_off[i] = BLK_BYTES + tile_off(((lane >> 3) >> 1) * 8 + (lane & 7), i * 2 + ((lane >> 3) & 1));
   }
 
+  const int pf = a.dec_pf;   // L2 prefetch distance in this warp's blocks (0 = off)
   // issue cursor over this warp's block sequence (units in claim order,
   // my blocks warp, warp + 8, ... of each), never beyond unit `limit`
   int iu = gw, ij = 0, n_issued = 0, n_cons = 0;
@@ -227,6 +228,14 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
       const int blk = btbuf[sl * MAXNB + wl + ij * GW];
       const uint8_t* ks = reinterpret_cast<const uint8_t*>(pk + ((size_t)blk * a.Hkv + cur_g) * KB * HD) + lane * 16;
       const uint8_t* vs = reinterpret_cast<const uint8_t*>(pv + ((size_t)blk * a.Hkv + cur_g) * KB * HD) + lane * 16;
+      if (pf > 0 && lane == 0 && ij + pf < cur_nb) {
+        // L2 prefetch pf blocks ahead of this warp's stream: the cp.async that
+        // follows hits L2, so the smem ring (the bytes a warp can keep in
+        // flight) covers the L2 latency instead of the DRAM latency
+        const int b2 = btbuf[sl * MAXNB + wl + (ij + pf) * GW];
+        prefetch_l2(pk + ((size_t)b2 * a.Hkv + cur_g) * KB * HD, BLK_BYTES);
+        prefetch_l2(pv + ((size_t)b2 * a.Hkv + cur_g) * KB * HD, BLK_BYTES);
+      }
       uint8_t* dk = my + (n_issued % DEPTH) * STAGE_BYTES;
 #pragma unroll
       for (int i = 0; i < 8; ++i) {

@@ -757,6 +757,16 @@ __global__ void __launch_bounds__(NT, 1)
         tile_coords(g.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
         b_rows_of(n_blk, r0, r1);
         for (int kb = g.kb0; kb < g.kb1; ++kb) {
+          if (a.b_pf && a.b_packed && kb + a.b_pf < g.kb1) {
+            // L2 prefetch b_pf k-blocks ahead of the ring (BULLET_GEMM_PF)
+            const uint8_t* kp = a.b_packed + (size_t)(kb + a.b_pf) * (a.b_rows / 64) * 8192;
+            if (r1 == r0 + bn / 2) {
+              prefetch_l2(kp + (size_t)(r0 / 64) * 8192, b_bytes);
+            } else {
+              prefetch_l2(kp + (size_t)(r0 / 64) * 8192, b_bytes / 2);
+              prefetch_l2(kp + (size_t)(r1 / 64) * 8192, b_bytes / 2);
+            }
+          }
           mbar_wait(empty + s, ph ^ 1);
           uint8_t* sb = smem + s * st_bytes + a_bytes;
           mbar_arrive_expect_tx(full + s, b_bytes);

@@ -74,6 +74,7 @@ struct GemmArgs {
   int b_evict_first;        // one M tile: the weight stream is used once (L2 evict-first)
   int b_rows;               // rows of B (packed layout stride)
   int split_b;              // 1: warp 3 issues the B tiles (second copy issuer), warp 0 the A tiles
+  int b_pf;                 // warp 3 prefetches packed B k-block kb + b_pf into L2 (0 = off)
   int kcb;                  // two-level accumulation (DESIGN R-4e): K chunk in k-blocks (0 = off);
                             // each chunk accumulates in TMEM, the chunks are summed in fp32
                             // registers by the epilogue (requires mh == 1, bn == 128, whole tiles)
@@ -126,6 +127,7 @@ struct AttnArgs {
                           // for longer contexts; 1 = none); partial (O, m, l) per chunk merged in order
   float* kv_part;         // [units][kv_chunks][8][128 + 2] (kv_chunks > 1)
   int* kv_tick;           // [units], zero between launches (self-resetting)
+  int dec_pf;             // decode kernel: L2 prefetch distance (blocks of a warp's stream; 0 = off)
   Launch L;
 };
 
