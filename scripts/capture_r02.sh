@@ -8,9 +8,12 @@ set -u
 P2=${1:-76}; K2=${2:-8}; P3=${3:-84}; K3=${4:-5}
 O=gpurun_out/ncu2; mkdir -p $O
 F="ncu --set full --clock-control none --import-source on"
-cap() { # name, kernel regex, skip, prof_step args...
+cap() { # name, kernel regex, skip, prof_step args...  (raw metrics exported as csv; the .ncu-rep is
+         # dropped unless KEEP_REP names it: gpurun brings back <= 64 MiB)
   local name=$1 k=$2 s=$3; shift 3
   timeout 300 $F -k regex:$k -s $s -c 1 -o $O/$name python scripts/prof_step.py --reps 2 --quiet "$@" > $O/$name.log 2>&1
+  ncu -i $O/$name.ncu-rep --page raw --csv > $O/$name.raw.csv 2>/dev/null
+  case " ${KEEP_REP:-} " in *" $name "*) ;; *) rm -f $O/$name.ncu-rep ;; esac
 }
 # decode layer GEMM order: qkv(0) o_proj(1) gate_up(2) down(3) (second step: +4)
 i=0

@@ -1,5 +1,6 @@
-"""Summarise ncu reports (.ncu-rep) into a markdown table: duration, SM
-clock, tensor-pipe %, DRAM bytes read/written, DRAM %, achieved occupancy."""
+"""Summarise ncu reports (.ncu-rep, or their `--page raw --csv` exports) into
+a markdown table: duration, SM clock, tensor-pipe %, DRAM bytes read/written,
+DRAM %, achieved occupancy."""
 import csv, io, subprocess, sys
 
 KEYS = [("gpu__time_duration.sum", "us"), ("sm__cycles_elapsed.avg.per_second", "GHz"),
@@ -11,7 +12,11 @@ KEYS = [("gpu__time_duration.sum", "us"), ("sm__cycles_elapsed.avg.per_second", 
 
 
 def rows(path):
-    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    """Rows of a report (.ncu-rep, read through ncu) or of its exported raw page (.csv)."""
+    if path.endswith(".csv"):
+        out = open(path).read()
+    else:
+        out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     r = list(csv.reader(io.StringIO(out)))
     hdr, units = r[0], r[1]
     for row in r[2:]:

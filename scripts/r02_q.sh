@@ -1,6 +1,4 @@
 O=gpurun_out/r02; mkdir -p $O
-bash scripts/capture_r02.sh 84 7 84 5 > $O/q_capture.log 2>&1
-for rate in 120 240; do
-  timeout 900 python scripts/serve.py --rate $rate --duration 3 --policies bullet_gain bullet timesliced prefill_first chunked --log-cycles $O/q_serve_cycles_$rate > $O/q_serve_rate$rate.jsonl 2> $O/q_serve_rate$rate.err
-done
+KEEP_REP="r02_c3_attn_dec_p84 r02_c2_down_dec_p84" bash scripts/capture_r02.sh 84 7 84 5 > $O/q_capture.log 2>&1
+du -sh gpurun_out/ncu2 >> $O/q_capture.log
 echo done
