@@ -118,6 +118,30 @@ def main():
     # typical batch against one decode layer-step of a typical decode batch
     k_ts = a.k_ts or max(1, round(g.bl.predict_us([400] * 8, [0] * 8, g.N) /
                                   g.bl.predict_us([1] * 128, [600] * 128, g.N)))
+    # online level calibration (bullet_set_phase_scale): a typical
+    # prefill layer and decode layer-step timed alone on the full GPU against
+    # the model's prediction, before any policy runs
+    cal = {}
+    if not a.no_feedback:
+        meas = {}
+        for name, q, c in (("pre", [400] * 8, [0] * 8), ("dec", [1] * 128, [600] * 128)):
+            blocks = list(range(sum(-(-(x + y) // 16) for x, y in zip(q, c))))
+            reqs, pos = [], 0
+            for x, y in zip(q, c):
+                n = -(-(x + y) // 16)
+                reqs.append(SV.Request(len(reqs), 0.0, max(x, 2), 2, blocks[pos:pos + n]))
+                pos += n
+            pw = SV.PhaseWork(reqs, q, c, 0, 4, -10 - len(meas))
+            ts = []
+            for _ in range(4):
+                ts.append(g(pw if name == "pre" else None, pw if name == "dec" else None,
+                            g.N if name == "pre" else 0, "corun"))
+            g.rec = []
+            meas[name] = float(np.median(ts[1:])) / 4
+        pre_s = meas["pre"] / (g.bl.predict_us([400] * 8, [0] * 8, g.N) / 1e3)
+        dec_s = meas["dec"] / (g.bl.predict_us([1] * 128, [600] * 128, g.N) / 1e3)
+        g.bl.set_phase_scale(pre_s, dec_s)
+        cal = {"prefill_layer_ms": meas["pre"], "decode_layer_ms": meas["dec"], "phase_scale": [pre_s, dec_s]}
     base = g.bl.colocation()
     for pol in a.policies:
         trace = SV.poisson_trace(a.rate, a.duration, seed=a.seed)
@@ -131,7 +155,7 @@ def main():
         res["policy"] = pol
         res["estimator_feedback"] = None if fb is None else {"corun_ratio": loop.fb_ratio,
                                                              "p_c_p_b": list(g.bl.colocation())}
-        res.update(rate_req_s=a.rate, arrivals_s=a.duration, layers=a.layers, k_timesliced=k_ts,
+        res.update(rate_req_s=a.rate, arrivals_s=a.duration, layers=a.layers, k_timesliced=k_ts, calibration=cal,
                    wall_s=time.perf_counter() - t0, model="llama3.1-8b", data="synthetic Poisson trace")
         ps = [c[1] for c in loop.log if 0 < c[1] < g.N]
         res["mean_prefill_sms_when_corun"] = float(np.mean(ps)) if ps else None
