@@ -72,8 +72,9 @@ def test_gemm_f32_epilogue_bit_exact(B, M, N, K, lo, hi, packed):
 
 
 # Every plan shape of the tcgen05 GEMM, forced through BULLET_GEMM_PLAN
-# ("mh,bn,ts"): 256-row units (mh=2) with a ragged second half, tail splits
-# of the last wave on a 20-SM partition, both combined, every epilogue.
+# ("mh,bn,sk"; sk != 0: the ragged remainder streamed over K, stream-K with
+# the fixup phase): 256-row units (mh=2) with a ragged second half, streamed
+# remainders on a 20-SM partition, both combined, every epilogue.
 @pytest.mark.parametrize("plan", ["1,256,1", "2,256,1", "2,128,1", "1,128,5", "2,128,3", "2,64,7", "2,256,2"])
 @pytest.mark.parametrize("epi", ["f32", "resid", "silu"])
 def test_gemm_plans_bit_exact(B, plan, epi, monkeypatch):
@@ -104,6 +105,40 @@ def test_gemm_plans_bit_exact(B, plan, epi, monkeypatch):
         ref = g / (1 + np.exp(-g)) * u
         got = out.float().cpu().numpy()
         assert np.all(np.abs(got - ref) <= np.maximum(np.abs(ref), 1e-30) * 2.0 ** -7 + 1e-6)
+
+
+@pytest.mark.parametrize("epi,N", [("f32", 512), ("resid", 512), ("silu", 1024)])
+def test_gemm_stream_k_many_segments_bit_exact(B, epi, N, monkeypatch):
+    """Stream-K with up to 16 segments per tile (2-4 tiles streamed over 60-64
+    SMs): the fixup phase's register-batch path (too many segments for one
+    bulk round through the stage ring) and its 16-segment limit, bit-exact
+    on integer operands, twice in a row (the counter slices alternate)."""
+    monkeypatch.setenv("BULLET_GEMM_PLAN", "1,256,1")
+    bl, _ = _handle(B, SMALL)
+    rng = np.random.default_rng(21)
+    M, K = 128, 4096
+    A, W = _int_operands(rng, M, K, N)
+    if epi == "silu":
+        W = W * 0.0625
+    At, Wt = torch.from_numpy(A).to("cuda", bf16), torch.from_numpy(W).to("cuda", bf16)
+    gu = (torch.from_numpy(A).double() @ torch.from_numpy(W).double().T).numpy()
+    for rep in range(2):
+        if epi == "f32":
+            out = torch.full((M, N), float("nan"), device="cuda")
+            bl.op_gemm(B.EPI_F32, At, Wt, out, lo=20, hi=84)
+            assert np.array_equal(out.cpu().numpy(), gu.astype(np.float32)), rep
+        elif epi == "resid":
+            R = rng.integers(-50, 50, size=(M, N)).astype(np.float32)
+            h = torch.from_numpy(R).cuda()
+            bl.op_gemm(B.EPI_RESID, At, Wt, h, resid=h, lo=20, hi=84)
+            assert np.array_equal(h.cpu().numpy(), (R + gu).astype(np.float32)), rep
+        else:
+            I = N // 2
+            out = torch.zeros(M, I, dtype=bf16, device="cuda")
+            bl.op_gemm(B.EPI_SILU, At, Wt, out, silu_half=I, lo=20, hi=80)
+            g, u = gu[:, :I], gu[:, I:]
+            ref = g / (1 + np.exp(-g)) * u
+            assert np.all(np.abs(out.float().cpu().numpy() - ref) <= np.maximum(np.abs(ref), 1e-30) * 2.0 ** -7 + 1e-6)
 
 
 def test_gemm_matches_oracle_linear_small(B):
