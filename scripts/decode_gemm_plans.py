@@ -1,6 +1,6 @@
 """Per-kind GEMM plan sweep on the decode side of the bench workload:
 time the decode layer-step with BULLET_PROFILE for each forced plan
-(BULLET_GEMM_PLAN_K<kind> = "mh,bn,ts") and print the GEMM's event time.
+(BULLET_GEMM_PLAN_K<kind> = "mh,bn,sk") and print the GEMM's event time.
 
   python scripts/decode_gemm_plans.py --p 80 0
 """
@@ -17,11 +17,11 @@ import torch  # noqa: E402
 import bench  # noqa: E402
 
 KINDS = {"qkv": 2, "o_proj": 5, "gate_up": 7, "down": 8}
-PLANS = {
-    "qkv": ["", "1,128,1", "1,64,1", "1,64,2", "1,128,2", "1,128,3", "1,256,2", "1,256,3", "1,256,4"],
-    "o_proj": ["", "1,64,1", "1,64,2", "1,128,1", "1,128,2", "1,256,4", "1,256,3", "1,128,3", "1,256,6"],
-    "gate_up": ["", "1,256,1", "1,128,1", "1,256,2"],
-    "down": ["", "1,128,2", "1,256,4", "1,256,3", "1,128,3", "1,256,6", "1,256,8", "1,64,1"],
+PLANS = {   # "mh,bn,sk": sk 1 streams the ragged remainder over K (stream-K + fixup phase)
+    "qkv": ["", "1,256,0", "1,256,1", "1,128,0", "1,128,1"],
+    "o_proj": ["", "1,64,0", "1,64,1", "1,128,0", "1,128,1", "1,256,1"],
+    "gate_up": ["", "1,256,0", "1,256,1", "1,128,0", "1,128,1"],
+    "down": ["", "1,128,0", "1,128,1", "1,256,1", "1,64,0"],
 }
 
 
