@@ -458,17 +458,17 @@ def test_pdl_on_off_bit_identical():
     import subprocess
     import sys
     here = os.path.dirname(os.path.abspath(__file__))
-    code = ("import sys; sys.path[:0] = [%r, %r]\\n"
-            "import torch, hashlib\\n"
-            "from harness import Setup, phase_streams\\n"
-            "from workload import synth\\n"
-            "m = synth.ModelShape('pdl', 1024, 8, 2, 128, 2816, 2)\\n"
-            "S = Setup(m, [300, 77, 1], [64, 1, 500, 31], n_layers=2)\\n"
-            "pre, dec = S.batches()\\n"
-            "S.bl.step(pre, dec, 64, S.B.CORUN, *phase_streams())\\n"
-            "torch.cuda.synchronize()\\n"
-            "h = hashlib.sha256(pre.hidden.cpu().numpy().tobytes() + dec.hidden.cpu().numpy().tobytes())\\n"
-            "print('DIGEST', h.hexdigest())\\n") % (here, os.path.dirname(here))
+    code = ("import sys; sys.path[:0] = [%r, %r]\n"
+            "import torch, hashlib\n"
+            "from harness import Setup, phase_streams\n"
+            "from workload import synth\n"
+            "m = synth.ModelShape('pdl', 1024, 8, 2, 128, 2816, 2)\n"
+            "S = Setup(m, [300, 77, 1], [64, 1, 500, 31], n_layers=2)\n"
+            "pre, dec = S.batches()\n"
+            "S.bl.step(pre, dec, 64, S.B.CORUN, *phase_streams())\n"
+            "torch.cuda.synchronize()\n"
+            "h = hashlib.sha256(pre.hidden.cpu().numpy().tobytes() + dec.hidden.cpu().numpy().tobytes())\n"
+            "print('DIGEST', h.hexdigest())\n") % (here, os.path.dirname(here))
     digests = []
     for pdl in ("1", "0"):
         r = subprocess.run([sys.executable, "-c", code], env=dict(os.environ, BULLET_PDL=pdl),
