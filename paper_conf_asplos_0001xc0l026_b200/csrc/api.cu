@@ -414,7 +414,9 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   // through one SM).  A single accumulator stage (mh * bn > 256 columns)
   // exposes the epilogue.  mh = 2 only for decode-sized M.  Rates: KI2 and
   // the per-CTA traces.
-  constexpr double BW_SM = 110e9, FL_SM = 10.5e12, EPI_BW = 100e9, RTT = 1.0e-6, T0 = 0.6e-6;
+  // FL_SM: the per-SM bf16 rate a decode-sized tile sustains (9 TF/s: 256-row units at M = 256 measured
+  // 7-9 % slower than two 128-row tiles, scripts/decode_gemm_plans.py, profiles/r02_decode_gemm_plans.log)
+  constexpr double BW_SM = 110e9, FL_SM = 9.0e12, EPI_BW = 100e9, RTT = 1.0e-6, T0 = 0.6e-6;
   const int k_blocks = K / 64;
   const size_t pf = h->ph[c.phase].partial_floats;
   int mh = 1, bn = 0, n_full = 0, sk_tiles = 0, sk_chunks = 0;
