@@ -321,21 +321,25 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
       }
     }
   } else if (warp == W_MMA) {
-    // ---------------- MMA issuer (one thread): S(g) then PV(g-1)
-    if (lane == 0) {
-      // f32 accumulate, bf16 A/B; S: N = 64, B K-major; O: N = 128, B MN-major
-      const uint32_t id_s = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(BKV >> 3) << 17) | ((uint32_t)(BQ >> 4) << 24);
-      const uint32_t id_o = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(HD >> 3) << 17) |
-                            ((uint32_t)(BQ >> 4) << 24);
-      uint32_t g = 0;
-      auto issue_pv = [&](uint32_t gp, bool first, int n) {
-        const int b = gp & 1;
-        wait(pfull + b, (gp >> 1) & 1);
-        wait(vfull + b, (gp >> 1) & 1);
-        if (first && n >= 1) wait(oempty, (n - 1) & 1);   // previous unit's O read out
-        tc_after();
-        fence_async_smem();
-        const uint32_t va = sbase + OFF_V + b * 16384, pa = t_s + b * 64;
+    // ---------------- MMA issuer: the whole warp runs the loop (descriptors
+    // stay warp-uniform, in uniform registers) and one elected lane issues
+    // each tcgen05 op; an issuer in a lane-0 branch made the compiler wrap
+    // every MMA in a per-lane waterfall loop (R2UR + ELECT + BRA.U.ANY), and
+    // that issue chain, not the tensor pipe, paced the kernel
+    // f32 accumulate, bf16 A/B; S: N = 64, B K-major; O: N = 128, B MN-major
+    const uint32_t id_s = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(BKV >> 3) << 17) | ((uint32_t)(BQ >> 4) << 24);
+    const uint32_t id_o = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(HD >> 3) << 17) |
+                          ((uint32_t)(BQ >> 4) << 24);
+    uint32_t g = 0;
+    auto issue_pv = [&](uint32_t gp, bool first, int n) {
+      const int b = gp & 1;
+      wait(pfull + b, (gp >> 1) & 1);
+      wait(vfull + b, (gp >> 1) & 1);
+      if (first && n >= 1) wait(oempty, (n - 1) & 1);   // previous unit's O read out
+      tc_after();
+      fence_async_smem();
+      const uint32_t va = sbase + OFF_V + b * 16384, pa = t_s + b * 64;
+      if (elect_one()) {
         // A = P from TMEM: keys 16kk..16kk+15 hi at column 32(kk/2) + 8(kk%2), lo 16 further
 #pragma unroll
         for (int kk = 0; kk < BKV / 16; ++kk)
@@ -344,22 +348,26 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
         for (int kk = 0; kk < BKV / 16; ++kk)
           tc_mma_ts(t_o, pa + (kk >> 1) * 32 + 16 + (kk & 1) * 8, desc_mn(va + kk * 2048), id_o, 1u);
         tc_commit(pvdone + b);
-      };
-      for (int n = 0;; ++n) {
-        const int slot = n & 1;
-        wait(ufull + slot, (n >> 1) & 1);
-        const int u = ring[slot];
-        mbar_arrive(uempty + slot);
-        if (u < 0) break;
-        const Unit U = unit_of(a, u);
-        wait(qfull, n & 1);
-        for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
-          const int b = g & 1, kb = g % NKB;
-          wait(kfull + kb, (g / NKB) & 1);
-          if (g >= 2) wait(pvdone + b, ((g - 2) >> 1) & 1);   // P(g-2) consumed: S buffer b free
-          tc_after();
-          fence_async_smem();
-          const uint32_t qa = sbase + OFF_Q, ka = sbase + OFF_K + kb * 16384;
+      }
+      __syncwarp();
+    };
+    for (int n = 0;; ++n) {
+      const int slot = n & 1;
+      wait(ufull + slot, (n >> 1) & 1);
+      const int u = ring[slot];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(uempty + slot);
+      if (u < 0) break;
+      const Unit U = unit_of(a, u);
+      wait(qfull, n & 1);
+      for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
+        const int b = g & 1, kb = g % NKB;
+        wait(kfull + kb, (g / NKB) & 1);
+        if (g >= 2) wait(pvdone + b, ((g - 2) >> 1) & 1);   // P(g-2) consumed: S buffer b free
+        tc_after();
+        fence_async_smem();
+        const uint32_t qa = sbase + OFF_Q, ka = sbase + OFF_K + kb * 16384;
+        if (elect_one()) {
 #pragma unroll
           for (int kk = 0; kk < HD / 16; ++kk)
             tc_mma(t_s + b * 64, desc_k(qa + (kk >> 2) * 16384 + (kk & 3) * 32),
@@ -367,10 +375,11 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
           tc_commit(sfull + b);
           tc_commit(kempty + kb);
           if (kt == U.n_kt - 1) tc_commit(qempty);
-          if (kt > 0) issue_pv(g - 1, kt == 1, n);
         }
-        issue_pv(g - 1, U.n_kt == 1, n);
+        __syncwarp();
+        if (kt > 0) issue_pv(g - 1, kt == 1, n);
       }
+      issue_pv(g - 1, U.n_kt == 1, n);
     }
   } else {
     // ---------------- softmax + epilogue: thread tid owns query row tid (TMEM lane tid)

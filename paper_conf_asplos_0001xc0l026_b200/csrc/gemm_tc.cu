@@ -454,8 +454,8 @@ __device__ __forceinline__ void fix_phase(const GemmArgs& a, int* s_u, int k_blo
   if (t0n) trace_at(a.L, 8, gtimer());
   int n_items = 0;
   uint32_t fph = 0;
-  uint64_t pol = 0;
-  if (tid == 0) { asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol)); s_u[0] = atomicAdd(a.fix_ctr, 1); }
+  const uint64_t pol = policy_evict_first();
+  if (tid == 0) s_u[0] = atomicAdd(a.fix_ctr, 1);
   __syncthreads();
   int u = s_u[0];
   for (;;) {
@@ -492,9 +492,13 @@ __device__ __forceinline__ void fix_phase(const GemmArgs& a, int* s_u, int k_blo
     const bool tr = t0n && n_items == 1;
     if (tr) trace_at(a.L, 11, gtimer());
     const bool bulk = (uint32_t)(nseg * nch) * CHUNK <= ring_bytes;
-    if (tid == 0) {   // every segment of the tile has stored its partial
-      while (ld_acquire_gpu(sems + st_idx) < nseg) __nanosleep(32);
-      if (bulk) {     // all (chunk, segment) blocks in one bulk-copy round
+    if (tid < 32) {   // every segment of the tile has stored its partial
+      if (tid == 0)
+        while (ld_acquire_gpu(sems + st_idx) < nseg) __nanosleep(32);
+      __syncwarp();
+      // all (chunk, segment) blocks in one bulk-copy round, issued by one
+      // elected lane of the converged warp (uniform operands, no waterfall)
+      if (bulk && elect_one()) {
         mbar_arrive_expect_tx(fixb, (uint32_t)(nseg * nch) * CHUNK);
         for (int ch = 0; ch < nch; ++ch)
           for (int sg = 0; sg < nseg; ++sg)
@@ -503,6 +507,7 @@ __device__ __forceinline__ void fix_phase(const GemmArgs& a, int* s_u, int k_blo
                          (size_t)hh * BM * bn / 4 + (size_t)((ch ? c2 : c) / 4) * BM,
                      CHUNK, fixb, pol);
       }
+      __syncwarp();
     }
     __syncthreads();
     if (tr) trace_at(a.L, 12, gtimer());
@@ -659,7 +664,8 @@ __global__ void __launch_bounds__(NT, 1)
   };
 
   if (warp == 0) {
-    if (lane == 0) {  // ---------------- scheduler + TMA producer
+    {  // ---------------- scheduler + TMA producer (whole warp; one elected lane
+       // issues, so the copy operands stay in uniform registers: see the MMA issuer)
       const uint64_t pol_a = policy_evict_last(), pol_b = a.b_evict_first ? policy_evict_first() : policy_evict_normal();
       int it = 0, s = 0;
       uint32_t ph = 0;
@@ -668,8 +674,11 @@ __global__ void __launch_bounds__(NT, 1)
       auto issue = [&](const Seg& g) {
         const int slot = it & 3;
         mbar_wait(tqe + slot, ((it >> 2) & 1) ^ 1);
-        tile_q[slot] = g;
-        mbar_arrive(tqf + slot);
+        if (lane == 0) {
+          tile_q[slot] = g;
+          mbar_arrive(tqf + slot);
+        }
+        __syncwarp();
         ++it;
         if (g.tile < 0) return;
         int m_blk, n_blk, r0, r1;
@@ -682,25 +691,28 @@ __global__ void __launch_bounds__(NT, 1)
         for (int kb = g.kb0; kb < g.kb1; ++kb) {
           mbar_wait(empty + s, ph ^ 1);
           uint8_t* sa = smem + s * st_bytes;
-          mbar_arrive_expect_tx(full + s, a.split_b ? a_bytes : st_bytes);
+          if (elect_one()) {
+            mbar_arrive_expect_tx(full + s, a.split_b ? a_bytes : st_bytes);
 #pragma unroll
-          for (int hh = 0; hh < mh; ++hh)   // rows past M are zero-filled by TMA
-            tma_load_2d_hint(sa + hh * A_BYTES, &mapA, full + s, kb * BK, (m_blk * mh + hh) * BM, pol_a);
-          uint8_t* sb = sa + a_bytes;
-          if (!a.split_b) {   // (else B comes from warp 3's issuer)
-            if (a.b_packed) {
-              const uint8_t* kbase = a.b_packed + (size_t)kb * (a.b_rows / 64) * 8192;
-              if (r1 == r0 + bn / 2) {
-                bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s, pol_b);
+            for (int hh = 0; hh < mh; ++hh)   // rows past M are zero-filled by TMA
+              tma_load_2d_hint(sa + hh * A_BYTES, &mapA, full + s, kb * BK, (m_blk * mh + hh) * BM, pol_a);
+            uint8_t* sb = sa + a_bytes;
+            if (!a.split_b) {   // (else B comes from warp 3's issuer)
+              if (a.b_packed) {
+                const uint8_t* kbase = a.b_packed + (size_t)kb * (a.b_rows / 64) * 8192;
+                if (r1 == r0 + bn / 2) {
+                  bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s, pol_b);
+                } else {
+                  bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes / 2, full + s, pol_b);
+                  bulk_g2s(sb + b_bytes / 2, kbase + (size_t)(r1 / 64) * 8192, b_bytes / 2, full + s, pol_b);
+                }
               } else {
-                bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes / 2, full + s, pol_b);
-                bulk_g2s(sb + b_bytes / 2, kbase + (size_t)(r1 / 64) * 8192, b_bytes / 2, full + s, pol_b);
+                tma_load_2d_hint(sb, &mapB, full + s, kb * BK, r0, pol_b);
+                tma_load_2d_hint(sb + b_bytes / 2, &mapB, full + s, kb * BK, r1, pol_b);
               }
-            } else {
-              tma_load_2d_hint(sb, &mapB, full + s, kb * BK, r0, pol_b);
-              tma_load_2d_hint(sb + b_bytes / 2, &mapB, full + s, kb * BK, r1, pol_b);
             }
           }
+          __syncwarp();
           if (++s == n_stages) { s = 0; ph ^= 1; }
         }
       };
@@ -708,13 +720,15 @@ __global__ void __launch_bounds__(NT, 1)
         // claim just in time: only once a smem stage is free to load into, so
         // early CTAs cannot hoard units while others idle (load balance)
         mbar_wait(empty + s, ph ^ 1);
-        const int u = atomicAdd(a.L.ctr, 1);
+        int u = 0;
+        if (lane == 0) u = atomicAdd(a.L.ctr, 1);
+        u = __shfl_sync(0xffffffffu, u, 0);
         if (u >= units) {   // all units claimed: the tail; the next kernel may launch
-          pdl_trigger();
+          if (lane == 0) pdl_trigger();
           issue(Seg{-1, 0, 0, -1});
           break;
         }
-        log_unit(a.L, u);
+        if (lane == 0) log_unit(a.L, u);
         if (u < a.n_full) {
           issue(Seg{u, 0, k_blocks, -1});
         } else {
@@ -731,12 +745,12 @@ __global__ void __launch_bounds__(NT, 1)
         {   // zero the stream-K counters of the next launch (the other parity slice;
             // the launch that used it last has completed): unit u takes indices u mod units
           int* nxt = a.tile_sems + (a.sk_parity ? 0 : N_TILE_SEMS_DEV);
-          for (int i = u; i < N_TILE_SEMS_DEV; i += units) nxt[i] = 0;
+          for (int i = u + lane * units; i < N_TILE_SEMS_DEV; i += 32 * units) nxt[i] = 0;
         }
       }
     }
   } else if (warp == 3) {
-    if (lane == 0 && a.split_b) {  // ---------------- second issuer: B (weight) tiles
+    if (a.split_b) {  // ---------------- second issuer: B (weight) tiles (whole warp, elected issue)
       // one thread's issue loop (wait for a free stage, arm, issue) caps the
       // copy stream it can keep in flight; a second issuing thread for the
       // weight operand lifts the per-SM ceiling (KI2: 99 -> 123 GB/s/SM,
@@ -750,14 +764,15 @@ __global__ void __launch_bounds__(NT, 1)
         const int slot = it & 3;
         mbar_wait(tqf + slot, (it >> 2) & 1);
         const Seg g = tile_q[slot];
-        mbar_arrive(tqe + slot);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(tqe + slot);
         ++it;
         if (g.tile < 0) break;
         int m_blk, n_blk, r0, r1;
         tile_coords(g.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
         b_rows_of(n_blk, r0, r1);
         for (int kb = g.kb0; kb < g.kb1; ++kb) {
-          if (a.b_pf && a.b_packed && kb + a.b_pf < g.kb1) {
+          if (a.b_pf && a.b_packed && kb + a.b_pf < g.kb1 && lane == 0) {
             // L2 prefetch b_pf k-blocks ahead of the ring (BULLET_GEMM_PF)
             const uint8_t* kp = a.b_packed + (size_t)(kb + a.b_pf) * (a.b_rows / 64) * 8192;
             if (r1 == r0 + bn / 2) {
@@ -769,25 +784,31 @@ __global__ void __launch_bounds__(NT, 1)
           }
           mbar_wait(empty + s, ph ^ 1);
           uint8_t* sb = smem + s * st_bytes + a_bytes;
-          mbar_arrive_expect_tx(full + s, b_bytes);
-          if (a.b_packed) {
-            const uint8_t* kbase = a.b_packed + (size_t)kb * (a.b_rows / 64) * 8192;
-            if (r1 == r0 + bn / 2) {
-              bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s, pol_b);
+          if (elect_one()) {
+            mbar_arrive_expect_tx(full + s, b_bytes);
+            if (a.b_packed) {
+              const uint8_t* kbase = a.b_packed + (size_t)kb * (a.b_rows / 64) * 8192;
+              if (r1 == r0 + bn / 2) {
+                bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes, full + s, pol_b);
+              } else {
+                bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes / 2, full + s, pol_b);
+                bulk_g2s(sb + b_bytes / 2, kbase + (size_t)(r1 / 64) * 8192, b_bytes / 2, full + s, pol_b);
+              }
             } else {
-              bulk_g2s(sb, kbase + (size_t)(r0 / 64) * 8192, b_bytes / 2, full + s, pol_b);
-              bulk_g2s(sb + b_bytes / 2, kbase + (size_t)(r1 / 64) * 8192, b_bytes / 2, full + s, pol_b);
+              tma_load_2d_hint(sb, &mapB, full + s, kb * BK, r0, pol_b);
+              tma_load_2d_hint(sb + b_bytes / 2, &mapB, full + s, kb * BK, r1, pol_b);
             }
-          } else {
-            tma_load_2d_hint(sb, &mapB, full + s, kb * BK, r0, pol_b);
-            tma_load_2d_hint(sb + b_bytes / 2, &mapB, full + s, kb * BK, r1, pol_b);
           }
+          __syncwarp();
           if (++s == n_stages) { s = 0; ph ^= 1; }
         }
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {  // ---------------- MMA issuer
+    {  // ---------------- MMA issuer: the whole warp runs the loop (descriptors
+       // warp-uniform, in uniform registers) and one elected lane issues the
+       // tcgen05 ops; a lane-0 branch made the compiler wrap every MMA in a
+       // per-lane waterfall loop (R2UR + ELECT + BRA.U.ANY, ~20 instructions)
       const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(bn >> 3) << 17) |
                              ((uint32_t)(BM >> 4) << 24);
       int it = 0, s = 0, as = 0;
@@ -797,10 +818,15 @@ __global__ void __launch_bounds__(NT, 1)
         const int slot = it & 3;
         mbar_wait(tqf + slot, (it >> 2) & 1);
         const Seg g = tile_q[slot];
-        mbar_arrive(tqe + slot);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(tqe + slot);
         if (g.tile < 0) break;
         const int kb0 = g.kb0, kb1 = g.kb1;
-        if (first && a.L.trace) { mbar_wait(full + s, ph); trace_at(a.L, 2, gtimer()); first = false; }
+        if (first && a.L.trace) {
+          mbar_wait(full + s, ph);
+          if (lane == 0) trace_at(a.L, 2, gtimer());
+          first = false;
+        }
         mbar_wait(acce + as, aph ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tmem + as * acc_cols;
@@ -811,7 +837,8 @@ __global__ void __launch_bounds__(NT, 1)
             // two-level accumulation: hand the finished chunk to the epilogue
             // (it adds it to its fp32 registers) and start the next chunk in
             // the other accumulator stage
-            tc_commit(accf + as);
+            if (elect_one()) tc_commit(accf + as);
+            __syncwarp();
             if (++as == n_acc) { as = 0; aph ^= 1; }
             mbar_wait(acce + as, aph ^ 1);
             tc_fence_after();
@@ -821,20 +848,24 @@ __global__ void __launch_bounds__(NT, 1)
           mbar_wait(full + s, ph);
           tc_fence_after();
           const uint32_t a_addr = smem_u32(smem + s * st_bytes), b_addr = a_addr + a_bytes;
+          if (elect_one()) {
 #pragma unroll
-          for (int k = 0; k < BK / 16; ++k)
+            for (int k = 0; k < BK / 16; ++k)
 #pragma unroll
-            for (int hh = 0; hh < mh; ++hh)
-              tc_mma(d_tmem_c + hh * bn, sw128_desc(a_addr + hh * A_BYTES + k * 32), sw128_desc(b_addr + k * 32),
-                     idesc, (kb > kc0 || k > 0) ? 1u : 0u);
-          tc_commit(empty + s);
+              for (int hh = 0; hh < mh; ++hh)
+                tc_mma(d_tmem_c + hh * bn, sw128_desc(a_addr + hh * A_BYTES + k * 32), sw128_desc(b_addr + k * 32),
+                       idesc, (kb > kc0 || k > 0) ? 1u : 0u);
+            tc_commit(empty + s);
+          }
+          __syncwarp();
           if (++s == n_stages) { s = 0; ph ^= 1; }
         }
-        tc_commit(accf + as);
+        if (elect_one()) tc_commit(accf + as);
+        __syncwarp();
         if (++as == n_acc) { as = 0; aph ^= 1; }
         ++it;
       }
-      if (a.L.trace) { trace_at(a.L, 3, gtimer()); trace_at(a.L, 6, it); }
+      if (a.L.trace && lane == 0) { trace_at(a.L, 3, gtimer()); trace_at(a.L, 6, it); }
     }
   } else if (warp >= 4) {  // ---------------- epilogue (warps 4..7 = TMEM lane quadrants 0..3)
     pdl_wait();   // reads residual / bias / token table, writes outputs and partials

@@ -6,6 +6,7 @@ BULLET_DEC_GROUPS (consumer groups per SM).
   python scripts/attn_dec_bench.py --config arxiv-8b --kind 3 --sms 60 148
 """
 import argparse
+import hashlib
 import json
 import os
 import sys
@@ -39,6 +40,7 @@ def main():
 def run(a, m, ctx):
     n = len(ctx)
     lay = synth.paged_layout([1] * n, ctx, 16)
+    torch.manual_seed(0)
     pk = torch.randn(lay.n_blocks, m.n_kv_heads, 16, m.head_dim, device="cuda").to(torch.bfloat16)
     pv = torch.randn_like(pk)
     bl = B.Bullet(B.Model.of(m), [(pk, pv)], n, n, max(ctx) + 32)
@@ -59,7 +61,8 @@ def run(a, m, ctx):
         torch.cuda.synchronize()
         us = e0.elapsed_time(e1) / a.reps * 1e3
         gbs = kv_bytes / us / 1e3
-        print(json.dumps({"config": a.config, "kind": a.kind, "tag": a.tag, "ctx": ctx[0] if a.uniform else "mix",
+        sha = hashlib.sha256(o.view(torch.int16).cpu().numpy().tobytes()).hexdigest()[:16]   # A/B bit identity
+        print(json.dumps({"sha": sha, "config": a.config, "kind": a.kind, "tag": a.tag, "ctx": ctx[0] if a.uniform else "mix",
                           "n": n, "units": n * m.n_kv_heads, "sms": msm, "us": round(us, 1),
                           "gbs": round(gbs), "gbs_per_sm": round(gbs / msm, 1)}), flush=True)
 

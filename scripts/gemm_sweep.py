@@ -58,7 +58,7 @@ def main():
                     us = e0.elapsed_time(e1) * 1e3 / a.reps
                     gbs = N * K * 2 / us / 1e3
                     print(f"plan={plan or 'auto':7s} M={M:4d} {name:8s} sms={n_sm:3d} {us:8.1f} us  "
-                          f"{gbs:7.0f} GB/s  {gbs / n_sm:6.1f} GB/s/SM", flush=True)
+                          f"{gbs:7.0f} GB/s  {gbs / n_sm:6.1f} GB/s/SM  {2 * M * N * K / us / 1e6:7.1f} TFLOP/s", flush=True)
 
 
 if __name__ == "__main__":
