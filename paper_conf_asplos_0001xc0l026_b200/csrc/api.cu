@@ -641,7 +641,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     a.tiles = P.tiles; a.n_tiles = P.n_tiles;   // the plan listed tiles of requests [0, r0) only
     int rc = next_launch(c, &a.L);
     if (rc) return rc;
-    LAUNCH(c, launch_attn_prefill5(a, persist_grid(c, 2), c.st));
+    LAUNCH(c, launch_attn_prefill5(a, persist_grid(c, attn_prefill5_ctas_per_sm(a.H, a.Hkv)), c.st));
     AttnArgs d = a;
     d.tok_base = t0;
     d.order = P.order_ok ? P.order : nullptr;
@@ -685,7 +685,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     }
     int rc = next_launch(c, &a.L);
     if (rc) return rc;
-    if (kind == 4) LAUNCH(c, launch_attn_prefill5(a, persist_grid(c, 2), c.st));
+    if (kind == 4) LAUNCH(c, launch_attn_prefill5(a, persist_grid(c, attn_prefill5_ctas_per_sm(a.H, a.Hkv)), c.st));
     else LAUNCH(c, launch_attn_prefill_tc(a, persist_grid(c, 2), c.st));
     return BULLET_OK;
   }

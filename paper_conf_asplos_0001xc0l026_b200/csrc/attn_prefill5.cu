@@ -2,39 +2,54 @@
 // (tcgen05 + TMEM), bf16, head_dim 128 (the paper's
 // FlashAttention).
 //
-// Work unit = (request, 128-row query tile, query head), LPT order from the
-// plan kernel.  Two CTAs per SM (96 KB smem, 256 TMEM columns each).  Per
-// 64-key KV tile t:
-//   S(t) = Q K(t)^T   tcgen05.mma M=128 (queries) N=64 (keys) -> TMEM fp32,
+// Work unit = (request, 128-row query tile, NQ query heads of one KV
+// group), LPT order from the plan kernel.  NQ = 2 (GQA groups of even size):
+// one CTA per SM, two query tiles share every K / V tile in shared memory
+// (half the gather traffic per MMA; 512 TMEM columns); NQ = 1: two CTAs per
+// SM (112 KB smem, 256 TMEM columns each).  Per 64-key KV tile t and query
+// tile q:
+//   S_q(t) = Q_q K(t)^T  tcgen05.mma M=128 (queries) N=64 (keys) -> TMEM fp32,
 //                     double-buffered so S(t+1) runs during softmax(t)
-//   softmax           4 warps, thread r owns query row r = TMEM lane r:
-//                     tcgen05.ld, causal mask, exp2 against a lazily moved
-//                     reference max, P = hi + lo (two bf16 halves, R-4b)
+//   softmax           4 warps per query tile, thread r owns query row r = TMEM
+//                     lane r: tcgen05.ld, causal mask, exp2 against a lazily
+//                     moved reference max, P = hi + lo (two bf16 halves, R-4b)
 //                     tcgen05.st'd over S(t) in TMEM
-//   O += P V          tcgen05.mma with A = P from TMEM, B = V(t) used as an
+//   O_q += P V        tcgen05.mma with A = P from TMEM, B = V(t) used as an
 //                     MN-major operand straight from its [key][dim] tile; O
 //                     stays in TMEM, rescaled only when a row max grows > 2^8
-// One __syncthreads per tile: after it one thread issues S(t+1) and PV(t)
-// back to back.  K/V rows are gathered through the block table with coalesced
-// cp.async into the 128-byte-swizzled layouts the UMMA descriptors describe,
-// two buffers each: K(t+2) loads from tile t on, V(t+1) during tile t.
+// One warp issues S(t+1) and PV(t) back to back (an elected lane of the
+// converged warp).  K/V rows are gathered through the block table with
+// coalesced cp.async into the 128-byte-swizzled layouts the UMMA descriptors
+// describe: NKB K buffers (K(t) loads once S(t-NKB) is done), two V buffers.
+// Measured (round 2, scripts/attn_pre_bench.py): the gathers, not the MMAs,
+// bound the NQ = 1 kernel (without them it runs at 0.65 of the bf16 peak,
+// with them 0.47; loading every other tile only: 0.55), hence NQ = 2.
 #include "kernels.h"
 
 namespace bl {
 
 namespace {
 constexpr int BQ = 128, BKV = 64, HD = 128, KB = 16;
-// warps 0-3 softmax + epilogue, 4 K/Q loader + unit claimer, 5 V loader, 6 MMA issuer
-constexpr int NT = 224, W_LOAD = 4, W_VLOAD = 5, W_MMA = 6;
-// smem: Q [2][128][128 B] | K[2 buffers] [2][64][128 B] | V[2 buffers] [2][64][128 B]
-// = 96 KB + barriers: two CTAs per SM.  The dynamic window must start
-// 1024-byte aligned (128-byte swizzle atoms); checked at entry.
-constexpr int NKB = 3;   // K buffers (K(g) may load once S(g-3) is done); V has 2
-constexpr int OFF_Q = 0, OFF_K = 32768, OFF_V = OFF_K + NKB * 16384, OFF_BAR = OFF_V + 2 * 16384;
-constexpr int SMEM_BYTES = OFF_BAR + 256;   // 20 mbarriers, TMEM slot, unit ring
-// TMEM: S/P double buffer in columns [0,64) and [64,128) (P = bf16 hi|lo
-// packed two per column, written over the S it came from), O in [128,256)
-constexpr uint32_t TMEM_COLS = 256;
+template <int NQ>
+struct Cfg {
+  // warps [0, 4 NQ) softmax + epilogue (query tile w / 4), then the K/Q
+  // loader + unit claimer, the V loader, one MMA issuer per query tile (the
+  // tiles' S -> softmax -> PV chains stay independent, as with two CTAs)
+  static constexpr int NSW = 4 * NQ, W_LOAD = NSW, W_VLOAD = NSW + 1, W_MMA = NSW + 2, NT = (NSW + 2 + NQ) * 32;
+  static constexpr int CTAS = 2 / NQ;   // per SM
+  // smem: Q [NQ][2][128][128 B] | K [NKB][2][64][128 B] | V [2][2][64][128 B] | barriers.
+  // The dynamic window must start 1024-byte aligned (128-byte swizzle atoms); checked at entry.
+#ifndef PF5_NKB2
+#define PF5_NKB2 4
+#endif
+  static constexpr int NKB = NQ == 2 ? PF5_NKB2 : 3;
+  static constexpr int OFF_Q = 0, OFF_K = NQ * 32768, OFF_V = OFF_K + NKB * 16384, OFF_BAR = OFF_V + 2 * 16384;
+  static constexpr int SMEM_BYTES = OFF_BAR + 512;   // mbarriers, TMEM slot, unit ring
+  // TMEM per query tile q (256 columns from 256 q): S/P double buffer in
+  // [0,64) and [64,128) (P = bf16 hi|lo packed two per column, written over
+  // the S it came from), O in [128,256)
+  static constexpr uint32_t TMEM_COLS = 256 * NQ;
+};
 
 // 128-byte swizzled offset of 16-byte chunk c of `row` in a tile whose
 // 64-element halves are `half` bytes apart
@@ -141,13 +156,15 @@ __device__ __forceinline__ uint32_t pack_bf2(float a, float b) {
 }
 
 struct Unit {
-  int h, g, q0, tok0, q_len, ctx, kv_len, n_kt, r;
+  int h, g, q0, tok0, q_len, ctx, kv_len, n_kt, r;   // h: first of the unit's NQ query heads
 };
+template <int NQ>
 __device__ __forceinline__ Unit unit_of(const AttnArgs& a, int u) {
   Unit U;
-  const int2 rt = a.tiles[u / a.H];
-  U.h = u % a.H;
-  U.g = U.h / (a.H / a.Hkv);
+  const int hq = a.H / NQ;
+  const int2 rt = a.tiles[u / hq];
+  U.h = (u % hq) * NQ;
+  U.g = U.h / (a.H / a.Hkv);   // NQ = 2 only for even groups: both heads read KV head g
   U.r = rt.x;
   U.q0 = rt.y * BQ;
   U.tok0 = __ldg(a.cu + U.r);
@@ -209,54 +226,60 @@ __device__ __forceinline__ void load_kv_tile(uint8_t* dst, const __nv_bfloat16* 
 }
 }  // namespace
 
-__global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
+template <int NQ>
+__global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS) k_attn_prefill5(AttnArgs a) {
+  using C = Cfg<NQ>;
+  constexpr int NKB = C::NKB, W_LOAD = C::W_LOAD, W_VLOAD = C::W_VLOAD, W_MMA = C::W_MMA;
+  constexpr int OFF_Q = C::OFF_Q, OFF_K = C::OFF_K, OFF_V = C::OFF_V;
   if (!gate_enter(a.L)) return;
   pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = smem_raw;
   if (smem_u32(sm) & 1023) __trap();   // swizzle atoms need 1024-byte alignment
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + OFF_BAR);
-  uint64_t *vfull = bars, *sfull = bars + 2, *pfull = bars + 4, *pvdone = bars + 6;
-  uint64_t *qfull = bars + 8, *qempty = bars + 9, *oempty = bars + 10, *ufull = bars + 11, *uempty = bars + 13;
-  uint64_t *kfull = bars + 15, *kempty = bars + 18;
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 21);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + C::OFF_BAR);
+  // sfull / pfull / pvdone: [query tile][S/P or V buffer]; oempty: [query tile]
+  uint64_t *vfull = bars, *pvdone = bars + 2, *sfull = pvdone + 2 * NQ, *pfull = sfull + 2 * NQ;
+  uint64_t *oempty = pfull + 2 * NQ, *qfull = oempty + NQ, *qempty = qfull + 1, *ufull = qfull + 2, *uempty = ufull + 2;
+  uint64_t *kfull = uempty + 2, *kempty = kfull + NKB;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(kempty + NKB);
   volatile int* ring = reinterpret_cast<volatile int*>(tslot + 1);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const uint32_t sbase = smem_u32(sm);
   if (tid == 0) {
     for (int i = 0; i < 2; ++i) {
       mbar_init(vfull + i, 32);   // one cp.async-completion arrive per loader lane
-      mbar_init(sfull + i, 1);    // tcgen05.commit
-      mbar_init(pfull + i, 4);    // one arrive per softmax warp
-      mbar_init(pvdone + i, 1);
       mbar_init(ufull + i, 1);
-      mbar_init(uempty + i, 6);   // MMA thread, V loader, 4 softmax warps
+      mbar_init(uempty + i, 1 + NQ + C::NSW);   // V loader, MMA warps, softmax warps
+    }
+    for (int i = 0; i < 2 * NQ; ++i) {
+      mbar_init(sfull + i, 1);    // tcgen05.commit
+      mbar_init(pfull + i, 4);    // one arrive per softmax warp of the tile
+      mbar_init(pvdone + i, 1);
     }
     for (int i = 0; i < NKB; ++i) {
       mbar_init(kfull + i, 32);
-      mbar_init(kempty + i, 1);
+      mbar_init(kempty + i, NQ);  // each query tile's S
     }
+    for (int i = 0; i < NQ; ++i) mbar_init(oempty + i, 4);
     mbar_init(qfull, 32);
-    mbar_init(qempty, 1);
-    mbar_init(oempty, 4);
+    mbar_init(qempty, NQ);
     mbar_fence_init();
   }
   if (warp == W_MMA) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tslot)), "r"(TMEM_COLS));
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tslot)), "r"(C::TMEM_COLS));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   tc_before();
   __syncthreads();
   tc_after();
   const uint32_t tmem = *tslot;
-  const uint32_t t_s = tmem, t_o = tmem + 128;
   const __nv_bfloat16* pk = reinterpret_cast<const __nv_bfloat16*>(a.pool_k);
   const __nv_bfloat16* pv = reinterpret_cast<const __nv_bfloat16*>(a.pool_v);
-  const int units = (*a.n_tiles) * a.H;
+  const int units = (*a.n_tiles) * (a.H / NQ);
 
   if (warp == W_LOAD) {
-    // ---------------- K/Q loader: claims units, gathers Q and K(g) as soon as
-    // S(g-3) has released K buffer g % 3
+    // ---------------- K/Q loader: claims units, gathers Q (NQ heads) and K(g)
+    // as soon as S(g-NKB) has released K buffer g % NKB
     const __nv_bfloat16* qg = reinterpret_cast<const __nv_bfloat16*>(a.q);
     const int r0 = lane >> 4, c = lane & 15;   // this lane: rows r0 + 2j, 16-byte chunk c
     uint32_t g = 0;
@@ -275,7 +298,7 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
         break;
       }
       if (lane == 0) log_unit(a.L, u);
-      const Unit U = unit_of(a, u);
+      const Unit U = unit_of<NQ>(a, u);
       const int32_t* bt = a.bt + (size_t)U.r * a.max_blocks;
       const int n_blk = (U.kv_len + KB - 1) / KB;   // blocks this sequence owns
       BtWin w;
@@ -287,12 +310,15 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
         load_kv_tile(sm + OFF_K + kb * 16384, pk, a, U, kt, lane, kfull + kb, w);
         if (kt == 0) {
           if (n >= 1) wait(qempty, (n - 1) & 1);         // last S of the previous unit done
+#pragma unroll
+          for (int q = 0; q < NQ; ++q) {
 #pragma unroll 8
-          for (int j = 0; j < BQ / 2; ++j) {
-            const int row = r0 + 2 * j;
-            const bool ok = U.q0 + row < U.q_len;
-            cp_async16_zfill(sm + OFF_Q + sw(row, c, 16384),
-                             qg + (size_t)(U.tok0 + (ok ? U.q0 + row : 0)) * a.H * HD + U.h * HD + c * 8, ok);
+            for (int j = 0; j < BQ / 2; ++j) {
+              const int row = r0 + 2 * j;
+              const bool ok = U.q0 + row < U.q_len;
+              cp_async16_zfill(sm + OFF_Q + q * 32768 + sw(row, c, 16384),
+                               qg + (size_t)(U.tok0 + (ok ? U.q0 + row : 0)) * a.H * HD + (U.h + q) * HD + c * 8, ok);
+            }
           }
           cp_async_arrive_noinc(qfull);
         }
@@ -308,7 +334,7 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
       __syncwarp();
       if (lane == 0) mbar_arrive(uempty + slot);
       if (u < 0) break;
-      const Unit U = unit_of(a, u);
+      const Unit U = unit_of<NQ>(a, u);
       const int32_t* bt = a.bt + (size_t)U.r * a.max_blocks;
       const int n_blk = (U.kv_len + KB - 1) / KB;   // blocks this sequence owns
       BtWin w;
@@ -316,29 +342,32 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
       for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
         const int b = g & 1;
         if (kt > 0 && kt % 8 == 0) w.advance(bt, n_blk, kt, lane);
-        if (g >= 2) wait(pvdone + b, ((g - 2) >> 1) & 1);
+        if (g >= 2)
+#pragma unroll
+          for (int q = 0; q < NQ; ++q) wait(pvdone + q * 2 + b, ((g - 2) >> 1) & 1);
         load_kv_tile(sm + OFF_V + b * 16384, pv, a, U, kt, lane, vfull + b, w);
       }
     }
-  } else if (warp == W_MMA) {
-    // ---------------- MMA issuer: the whole warp runs the loop (descriptors
-    // stay warp-uniform, in uniform registers) and one elected lane issues
-    // each tcgen05 op; an issuer in a lane-0 branch made the compiler wrap
-    // every MMA in a per-lane waterfall loop (R2UR + ELECT + BRA.U.ANY), and
-    // that issue chain, not the tensor pipe, paced the kernel
+  } else if (warp >= W_MMA) {
+    // ---------------- MMA issuer of query tile qm: the whole warp runs the
+    // loop (descriptors stay warp-uniform, in uniform registers) and one
+    // elected lane issues each tcgen05 op; an issuer in a lane-0 branch made
+    // the compiler wrap every MMA in a per-lane waterfall loop
     // f32 accumulate, bf16 A/B; S: N = 64, B K-major; O: N = 128, B MN-major
+    const int qm = warp - W_MMA;
     const uint32_t id_s = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(BKV >> 3) << 17) | ((uint32_t)(BQ >> 4) << 24);
     const uint32_t id_o = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(HD >> 3) << 17) |
                           ((uint32_t)(BQ >> 4) << 24);
+    const uint32_t t_q = tmem + qm * 256, t_o = t_q + 128, qa = sbase + OFF_Q + qm * 32768;
     uint32_t g = 0;
     auto issue_pv = [&](uint32_t gp, bool first, int n) {
       const int b = gp & 1;
-      wait(pfull + b, (gp >> 1) & 1);
       wait(vfull + b, (gp >> 1) & 1);
-      if (first && n >= 1) wait(oempty, (n - 1) & 1);   // previous unit's O read out
+      if (first && n >= 1) wait(oempty + qm, (n - 1) & 1);   // previous unit's O read out
+      wait(pfull + qm * 2 + b, (gp >> 1) & 1);
       tc_after();
       fence_async_smem();
-      const uint32_t va = sbase + OFF_V + b * 16384, pa = t_s + b * 64;
+      const uint32_t va = sbase + OFF_V + b * 16384, pa = t_q + b * 64;
       if (elect_one()) {
         // A = P from TMEM: keys 16kk..16kk+15 hi at column 32(kk/2) + 8(kk%2), lo 16 further
 #pragma unroll
@@ -347,7 +376,7 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
 #pragma unroll
         for (int kk = 0; kk < BKV / 16; ++kk)
           tc_mma_ts(t_o, pa + (kk >> 1) * 32 + 16 + (kk & 1) * 8, desc_mn(va + kk * 2048), id_o, 1u);
-        tc_commit(pvdone + b);
+        tc_commit(pvdone + qm * 2 + b);
       }
       __syncwarp();
     };
@@ -358,21 +387,21 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
       __syncwarp();
       if (lane == 0) mbar_arrive(uempty + slot);
       if (u < 0) break;
-      const Unit U = unit_of(a, u);
+      const Unit U = unit_of<NQ>(a, u);
       wait(qfull, n & 1);
       for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
         const int b = g & 1, kb = g % NKB;
         wait(kfull + kb, (g / NKB) & 1);
-        if (g >= 2) wait(pvdone + b, ((g - 2) >> 1) & 1);   // P(g-2) consumed: S buffer b free
+        if (g >= 2) wait(pvdone + qm * 2 + b, ((g - 2) >> 1) & 1);   // P(g-2) consumed: S buffer b free
         tc_after();
         fence_async_smem();
-        const uint32_t qa = sbase + OFF_Q, ka = sbase + OFF_K + kb * 16384;
+        const uint32_t ka = sbase + OFF_K + kb * 16384;
         if (elect_one()) {
 #pragma unroll
           for (int kk = 0; kk < HD / 16; ++kk)
-            tc_mma(t_s + b * 64, desc_k(qa + (kk >> 2) * 16384 + (kk & 3) * 32),
+            tc_mma(t_q + b * 64, desc_k(qa + (kk >> 2) * 16384 + (kk & 3) * 32),
                    desc_k(ka + (kk >> 2) * 8192 + (kk & 3) * 32), id_s, kk > 0 ? 1u : 0u);
-          tc_commit(sfull + b);
+          tc_commit(sfull + qm * 2 + b);
           tc_commit(kempty + kb);
           if (kt == U.n_kt - 1) tc_commit(qempty);
         }
@@ -382,10 +411,13 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
       issue_pv(g - 1, U.n_kt == 1, n);
     }
   } else {
-    // ---------------- softmax + epilogue: thread tid owns query row tid (TMEM lane tid)
+    // ---------------- softmax + epilogue: warp w serves query tile w / 4;
+    // thread owns query row (w % 4) * 32 + lane = its TMEM lane
     __nv_bfloat16* og = reinterpret_cast<__nv_bfloat16*>(a.o);
     const float sl2 = a.scale * 1.4426950408889634f;
-    const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
+    const int qt = warp >> 2, row = tid & 127;
+    const uint32_t lane_off = (uint32_t)((warp & 3) * 32) << 16;
+    const uint32_t t_s = tmem + qt * 256, t_o = t_s + 128;
     uint32_t g = 0;
     for (int n = 0;; ++n) {
       const int slot = n & 1;
@@ -394,13 +426,13 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
       __syncwarp();
       if (lane == 0) mbar_arrive(uempty + slot);
       if (u < 0) break;
-      const Unit U = unit_of(a, u);
-      const int qpos = U.ctx + U.q0 + tid;
+      const Unit U = unit_of<NQ>(a, u);
+      const int qpos = U.ctx + U.q0 + row;
       float m_ref = -INFINITY, l_run = 0.f;
       for (int kt = 0; kt < U.n_kt; ++kt, ++g) {
         const int b = g & 1;
         const uint32_t t_sb = t_s + b * 64 + lane_off;
-        wait(sfull + b, (g >> 1) & 1);
+        wait(sfull + qt * 2 + b, (g >> 1) & 1);
         tc_after();
         // two passes over S in TMEM (32 columns at a time) keep ~32 scores live:
         // pass 1 row max, pass 2 P.  Only tiles crossing the causal diagonal or
@@ -425,7 +457,7 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
         const float m_new = move ? mx_s : m_ref;
         const float alpha = move ? ex2(m_ref - m_new) : 1.f;
         if (kt > 0 && __any_sync(0xffffffffu, move)) {   // lazy rescale of O: PV(g-1) must be done
-          wait(pvdone + ((g - 1) & 1), ((g - 1) >> 1) & 1);
+          wait(pvdone + qt * 2 + ((g - 1) & 1), ((g - 1) >> 1) & 1);
           tc_after();
 #pragma unroll 1
           for (int c = 0; c < 4; ++c) {
@@ -474,14 +506,14 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
         asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
         tc_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(pfull + b);
+        if (lane == 0) mbar_arrive(pfull + qt * 2 + b);
       }
-      // ---- normalise and store row tid (bf16, point R3) once the last PV is done
-      wait(pvdone + ((g - 1) & 1), ((g - 1) >> 1) & 1);
+      // ---- normalise and store row `row` of head U.h + qt (bf16, point R3) once the last PV is done
+      wait(pvdone + qt * 2 + ((g - 1) & 1), ((g - 1) >> 1) & 1);
       tc_after();
       const float inv = 1.f / l_run;
-      const bool ok = U.q0 + tid < U.q_len;
-      __nv_bfloat16* dst = og + (size_t)(U.tok0 + U.q0 + (ok ? tid : 0)) * a.H * HD + U.h * HD;
+      const bool ok = U.q0 + row < U.q_len;
+      __nv_bfloat16* dst = og + (size_t)(U.tok0 + U.q0 + (ok ? row : 0)) * a.H * HD + (U.h + qt) * HD;
 #pragma unroll
       for (int c = 0; c < 4; ++c) {
         float w[32];
@@ -496,30 +528,48 @@ __global__ void __launch_bounds__(NT, 2) k_attn_prefill5(AttnArgs a) {
       }
       tc_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(oempty);
+      if (lane == 0) mbar_arrive(oempty + qt);
     }
   }
   tc_before();
   __syncthreads();
   if (warp == W_MMA) {
     tc_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS));
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(C::TMEM_COLS));
   }
 }
 
-cudaError_t launch_attn_prefill5(const AttnArgs& a, int grid, cudaStream_t st) {
+// Query tiles per CTA: 2 when the GQA group size is even (the two heads
+// share their K / V tiles), else 1; BULLET_PF5_NQ=1 forces the single-tile
+// kernel (A/B).
+int attn_prefill5_nq(int H, int Hkv) {
+  static const int forced = getenv("BULLET_PF5_NQ") ? atoi(getenv("BULLET_PF5_NQ")) : 0;
+  if (forced == 1) return 1;
+  return (H / Hkv) % 2 == 0 ? 2 : 1;
+}
+int attn_prefill5_ctas_per_sm(int H, int Hkv) { return attn_prefill5_nq(H, Hkv) == 2 ? 1 : 2; }
+
+template <int NQ>
+static cudaError_t launch_nq(const AttnArgs& a, int grid, cudaStream_t st) {
   static bool set = false;
   if (!set) {
-    cudaError_t e = cudaFuncSetAttribute(k_attn_prefill5, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+    cudaError_t e = cudaFuncSetAttribute(k_attn_prefill5<NQ>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<NQ>::SMEM_BYTES);
     if (e != cudaSuccess) return e;
     set = true;
   }
-  return launch_ex(k_attn_prefill5, grid, NT, SMEM_BYTES, st, a.L.pdl, a);
+  return launch_ex(k_attn_prefill5<NQ>, grid, Cfg<NQ>::NT, Cfg<NQ>::SMEM_BYTES, st, a.L.pdl, a);
+}
+
+// `grid` must be n_sms * attn_prefill5_ctas_per_sm(H, Hkv) (persistent, gated).
+cudaError_t launch_attn_prefill5(const AttnArgs& a, int grid, cudaStream_t st) {
+  return attn_prefill5_nq(a.H, a.Hkv) == 2 ? launch_nq<2>(a, grid, st) : launch_nq<1>(a, grid, st);
 }
 
 cudaError_t preload_attn_prefill5() {
   cudaFuncAttributes f;
-  return cudaFuncGetAttributes(&f, k_attn_prefill5);
+  cudaError_t e = cudaFuncGetAttributes(&f, k_attn_prefill5<1>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&f, k_attn_prefill5<2>);
+  return e;
 }
 
 }  // namespace bl

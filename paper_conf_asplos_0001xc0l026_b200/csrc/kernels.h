@@ -182,6 +182,7 @@ template <typename T>
 cudaError_t launch_attn_simt(const AttnArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_attn_prefill_tc(const AttnArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_attn_prefill5(const AttnArgs& a, int grid, cudaStream_t st);
+int attn_prefill5_ctas_per_sm(int H, int Hkv);   // grid = n_sms * this (2 query tiles per CTA for even GQA groups)
 cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStream_t st);
 size_t attn_decode_smem_bytes();
 int attn_decode_max_blocks();
