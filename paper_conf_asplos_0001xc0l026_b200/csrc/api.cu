@@ -416,12 +416,16 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   // the per-CTA traces.
   // FL_SM: the per-SM bf16 rate a decode-sized tile sustains (9 TF/s: 256-row units at M = 256 measured
   // 7-9 % slower than two 128-row tiles, scripts/decode_gemm_plans.py, profiles/r02_decode_gemm_plans.log)
-  constexpr double BW_SM = 110e9, FL_SM = 9.0e12, EPI_BW = 100e9, RTT = 1.0e-6, T0 = 0.6e-6;
+  constexpr double BW_SM = 110e9, FL_SM = 9.0e12, EPI_BW = 100e9, T0 = 0.6e-6;
   const int k_blocks = K / 64;
   const size_t pf = h->ph[c.phase].partial_floats;
   int mh = 1, bn = 0, n_full = 0, sk_tiles = 0, sk_chunks = 0;
   double best = 1e300;
-  for (int cmh = (M > 128 && M <= 512) ? 2 : 1; cmh >= 1; --cmh) {
+  // mh = 1 is tried first and mh = 2 pays 5 %: with the warp-wide issue,
+  // 128 x 256 tiles measured 10-13 % faster than the 256-row units the model
+  // ranked equal or better at M = 256 (profiles/r02_decode_gemm_plans_v2.log)
+  for (int cmh = 1; cmh <= ((M > 128 && M <= 512) ? 2 : 1); ++cmh) {
+    const double pen = cmh == 2 ? 1.05 : 1.0;
     const int m_tiles = (M + 128 * cmh - 1) / (128 * cmh);
     for (int cand : {256, 128, 64}) {
       if (!fits(cand)) continue;
@@ -429,7 +433,7 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
       const double out_b = 128.0 * cmh * cand * 4.0;
       const double t_kb = std::max((cmh * 16384.0 + cand * 128.0) / BW_SM, 2.0 * 128 * cmh * cand * 64 / FL_SM);
       const double t_tile = k_blocks * t_kb + (2 * cmh * cand > 512 ? out_b / EPI_BW : 0.0) + T0;
-      const double cost_a = std::ceil((double)tiles / c.m_sms) * t_tile;   // whole tiles only
+      const double cost_a = pen * std::ceil((double)tiles / c.m_sms) * t_tile;   // whole tiles only
       if (cost_a < best * 0.999) { best = cost_a; mh = cmh; bn = cand; n_full = tiles; sk_tiles = 0; sk_chunks = 0; }
       const int fw = tiles / c.m_sms, rem = tiles % c.m_sms;
       if (rem == 0) continue;
@@ -439,8 +443,8 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
       // store the partials and reach the phase, then ~4 us per round of
       // items (an item = 32 output columns x 128 rows of one streamed tile)
       const int items = rem * cmh * ((epi == EPI_QKV || epi == EPI_SILU) ? cand / 64 : cand / 32);
-      const double cost_b = fw * t_tile + (double)rem * k_blocks / chunks * t_kb + T0 + 6e-6 +
-                            std::ceil((double)items / c.m_sms) * 4e-6;
+      const double cost_b = pen * (fw * t_tile + (double)rem * k_blocks / chunks * t_kb + T0 + 6e-6 +
+                                   std::ceil((double)items / c.m_sms) * 4e-6);
       if (cost_b < best * 0.999) {
         best = cost_b; mh = cmh; bn = cand; n_full = fw * c.m_sms; sk_tiles = rem; sk_chunks = chunks;
       }
