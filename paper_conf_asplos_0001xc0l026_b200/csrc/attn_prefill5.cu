@@ -35,7 +35,13 @@ struct Cfg {
   // warps [0, 4 NQ) softmax + epilogue (query tile w / 4), then the K/Q
   // loader + unit claimer, the V loader, one MMA issuer per query tile (the
   // tiles' S -> softmax -> PV chains stay independent, as with two CTAs)
-  static constexpr int NSW = 4 * NQ, W_LOAD = NSW, W_VLOAD = NSW + 1, W_MMA = NSW + 2, NT = (NSW + 2 + NQ) * 32;
+  // NLW warps gather each of K (and Q) and V (the first K warp claims units)
+#ifndef PF5_NLW
+#define PF5_NLW 2
+#endif
+  static constexpr int NLW = NQ == 2 ? PF5_NLW : 1;
+  static constexpr int NSW = 4 * NQ, W_LOAD = NSW, W_VLOAD = NSW + NLW, W_MMA = NSW + 2 * NLW,
+                       NT = (NSW + 2 * NLW + NQ) * 32;
   static constexpr int CTAS = 2 / NQ;   // per SM
   // smem: Q [NQ][2][128][128 B] | K [NKB][2][64][128 B] | V [2][2][64][128 B] | barriers.
   // The dynamic window must start 1024-byte aligned (128-byte swizzle atoms); checked at entry.
@@ -204,15 +210,17 @@ struct BtWin {
     nxt = e < n_blk ? __ldg(bt + e) : 0;
   }
 };
-// One warp gathers KV tile kt (64 rows of head U.g through the block table)
-// into a 128-byte-swizzled [2][64][128 B] tile; `bar` completes when it lands.
+// One warp gathers blocks [b0, b0 + NB) of KV tile kt (16 rows each, of head
+// U.g through the block table) into a 128-byte-swizzled [2][64][128 B] tile;
+// `bar` gets this warp's arrivals when they land.
+template <int NB>
 __device__ __forceinline__ void load_kv_tile(uint8_t* dst, const __nv_bfloat16* pool, const AttnArgs& a,
-                                             const Unit& U, int kt, int lane, uint64_t* bar, const BtWin& w) {
+                                             const Unit& U, int kt, int lane, uint64_t* bar, const BtWin& w, int b0) {
   const int r0 = lane >> 4, c = lane & 15;   // this lane: rows r0 + 2j, 16-byte chunk c
   const int kb = kt * BKV;
   const bool full = kb + BKV <= U.kv_len;
 #pragma unroll
-  for (int b = 0; b < BKV / KB; ++b) {
+  for (int b = b0; b < b0 + NB; ++b) {
     const int blk = __shfl_sync(0xffffffffu, w.cur, (kt % 8) * (BKV / KB) + b);
     const __nv_bfloat16* src = pool + (((size_t)blk * a.Hkv + U.g) * KB + r0) * HD + c * 8;
 #pragma unroll
@@ -229,7 +237,8 @@ __device__ __forceinline__ void load_kv_tile(uint8_t* dst, const __nv_bfloat16* 
 template <int NQ>
 __global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS) k_attn_prefill5(AttnArgs a) {
   using C = Cfg<NQ>;
-  constexpr int NKB = C::NKB, W_LOAD = C::W_LOAD, W_VLOAD = C::W_VLOAD, W_MMA = C::W_MMA;
+  constexpr int NKB = C::NKB, W_LOAD = C::W_LOAD, W_VLOAD = C::W_VLOAD, W_MMA = C::W_MMA, NLW = C::NLW;
+  constexpr int NBW = BKV / KB / NLW;   // blocks of a KV tile per loader warp
   constexpr int OFF_Q = C::OFF_Q, OFF_K = C::OFF_K, OFF_V = C::OFF_V;
   if (!gate_enter(a.L)) return;
   pdl_wait();      // inputs are the predecessor's outputs (common.cuh, PDL)
@@ -247,9 +256,9 @@ __global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS) k_attn_prefill5(At
   const uint32_t sbase = smem_u32(sm);
   if (tid == 0) {
     for (int i = 0; i < 2; ++i) {
-      mbar_init(vfull + i, 32);   // one cp.async-completion arrive per loader lane
+      mbar_init(vfull + i, 32 * NLW);   // one cp.async-completion arrive per loader lane
       mbar_init(ufull + i, 1);
-      mbar_init(uempty + i, 1 + NQ + C::NSW);   // V loader, MMA warps, softmax warps
+      mbar_init(uempty + i, 2 * NLW - 1 + NQ + C::NSW);   // loaders but the claimer, MMA warps, softmax warps
     }
     for (int i = 0; i < 2 * NQ; ++i) {
       mbar_init(sfull + i, 1);    // tcgen05.commit
@@ -257,11 +266,11 @@ __global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS) k_attn_prefill5(At
       mbar_init(pvdone + i, 1);
     }
     for (int i = 0; i < NKB; ++i) {
-      mbar_init(kfull + i, 32);
+      mbar_init(kfull + i, 32 * NLW);
       mbar_init(kempty + i, NQ);  // each query tile's S
     }
     for (int i = 0; i < NQ; ++i) mbar_init(oempty + i, 4);
-    mbar_init(qfull, 32);
+    mbar_init(qfull, 32 * NLW);
     mbar_init(qempty, NQ);
     mbar_fence_init();
   }
@@ -277,27 +286,37 @@ __global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS) k_attn_prefill5(At
   const __nv_bfloat16* pv = reinterpret_cast<const __nv_bfloat16*>(a.pool_v);
   const int units = (*a.n_tiles) * (a.H / NQ);
 
-  if (warp == W_LOAD) {
-    // ---------------- K/Q loader: claims units, gathers Q (NQ heads) and K(g)
+  if (warp >= W_LOAD && warp < W_VLOAD) {
+    // ---------------- K/Q loaders: warp W_LOAD claims units (the others read
+    // them from the ring); each gathers its share of Q (NQ heads) and of K(g)
     // as soon as S(g-NKB) has released K buffer g % NKB
+    const int lw = warp - W_LOAD;
     const __nv_bfloat16* qg = reinterpret_cast<const __nv_bfloat16*>(a.q);
     const int r0 = lane >> 4, c = lane & 15;   // this lane: rows r0 + 2j, 16-byte chunk c
     uint32_t g = 0;
     for (int n = 0;; ++n) {
-      int u = 0;
-      if (lane == 0) u = atomicAdd(a.L.ctr, 1);
-      u = __shfl_sync(0xffffffffu, u, 0);
       const int slot = n & 1;
-      if (n >= 2) wait(uempty + slot, ((n - 2) >> 1) & 1);
-      if (lane == 0) {
-        ring[slot] = u < units ? u : -1;
-        mbar_arrive(ufull + slot);
+      int u = 0;
+      if (lw == 0) {
+        if (lane == 0) u = atomicAdd(a.L.ctr, 1);
+        u = __shfl_sync(0xffffffffu, u, 0);
+        if (n >= 2) wait(uempty + slot, ((n - 2) >> 1) & 1);
+        if (lane == 0) {
+          ring[slot] = u < units ? u : -1;
+          mbar_arrive(ufull + slot);
+        }
+        if (u >= units) {   // all units claimed: the next kernel may launch (PDL)
+          if (lane == 0) pdl_trigger();
+          break;
+        }
+        if (lane == 0) log_unit(a.L, u);
+      } else {
+        wait(ufull + slot, (n >> 1) & 1);
+        u = ring[slot];
+        __syncwarp();
+        if (lane == 0) mbar_arrive(uempty + slot);
+        if (u < 0) break;
       }
-      if (u >= units) {   // all units claimed: the next kernel may launch (PDL)
-        if (lane == 0) pdl_trigger();
-        break;
-      }
-      if (lane == 0) log_unit(a.L, u);
       const Unit U = unit_of<NQ>(a, u);
       const int32_t* bt = a.bt + (size_t)U.r * a.max_blocks;
       const int n_blk = (U.kv_len + KB - 1) / KB;   // blocks this sequence owns
@@ -307,13 +326,13 @@ __global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS) k_attn_prefill5(At
         const int kb = g % NKB;
         if (kt > 0 && kt % 8 == 0) w.advance(bt, n_blk, kt, lane);
         if (g >= NKB) wait(kempty + kb, (g / NKB - 1) & 1);
-        load_kv_tile(sm + OFF_K + kb * 16384, pk, a, U, kt, lane, kfull + kb, w);
+        load_kv_tile<NBW>(sm + OFF_K + kb * 16384, pk, a, U, kt, lane, kfull + kb, w, lw * NBW);
         if (kt == 0) {
           if (n >= 1) wait(qempty, (n - 1) & 1);         // last S of the previous unit done
 #pragma unroll
           for (int q = 0; q < NQ; ++q) {
 #pragma unroll 8
-            for (int j = 0; j < BQ / 2; ++j) {
+            for (int j = lw * (BQ / 2 / NLW); j < (lw + 1) * (BQ / 2 / NLW); ++j) {
               const int row = r0 + 2 * j;
               const bool ok = U.q0 + row < U.q_len;
               cp_async16_zfill(sm + OFF_Q + q * 32768 + sw(row, c, 16384),
@@ -324,8 +343,9 @@ __global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS) k_attn_prefill5(At
         }
       }
     }
-  } else if (warp == W_VLOAD) {
-    // ---------------- V loader: V(g) as soon as PV(g-2) has released buffer g & 1
+  } else if (warp >= W_VLOAD && warp < W_MMA) {
+    // ---------------- V loaders: their share of V(g) as soon as PV(g-2) has released buffer g & 1
+    const int lw = warp - W_VLOAD;
     uint32_t g = 0;
     for (int n = 0;; ++n) {
       const int slot = n & 1;
@@ -345,7 +365,7 @@ __global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS) k_attn_prefill5(At
         if (g >= 2)
 #pragma unroll
           for (int q = 0; q < NQ; ++q) wait(pvdone + q * 2 + b, ((g - 2) >> 1) & 1);
-        load_kv_tile(sm + OFF_V + b * 16384, pv, a, U, kt, lane, vfull + b, w);
+        load_kv_tile<NBW>(sm + OFF_V + b * 16384, pv, a, U, kt, lane, vfull + b, w, lw * NBW);
       }
     }
   } else if (warp >= W_MMA) {

@@ -476,3 +476,33 @@ def test_pdl_on_off_bit_identical():
         assert r.returncode == 0, r.stderr[-3000:]
         digests.append([l for l in r.stdout.splitlines() if l.startswith("DIGEST")][0])
     assert digests[0] == digests[1]
+
+
+def test_prefill_attention_gqa_pair_bit_identical():
+    """Two query heads of a GQA group per CTA (k_attn_prefill5<2>, the
+    default for even group sizes) change which CTA computes a head, never the
+    per-row arithmetic: a two-layer co-run step with ragged prompts (partial
+    query tiles, a 1-token prompt) gives the same bits as the one-head kernel
+    (BULLET_PF5_NQ=1, fresh process)."""
+    import os
+    import subprocess
+    import sys
+    here = os.path.dirname(os.path.abspath(__file__))
+    code = ("import sys; sys.path[:0] = [%r, %r]\n"
+            "import torch, hashlib\n"
+            "from harness import Setup, phase_streams\n"
+            "from workload import synth\n"
+            "m = synth.ModelShape('gqa', 1024, 8, 2, 128, 2816, 2)\n"
+            "S = Setup(m, [300, 77, 1, 129], [64, 1, 500, 31], n_layers=2)\n"
+            "pre, dec = S.batches()\n"
+            "S.bl.step(pre, dec, 64, S.B.CORUN, *phase_streams())\n"
+            "torch.cuda.synchronize()\n"
+            "h = hashlib.sha256(pre.hidden.cpu().numpy().tobytes() + dec.hidden.cpu().numpy().tobytes())\n"
+            "print('DIGEST', h.hexdigest())\n") % (here, os.path.dirname(here))
+    digests = []
+    for nq in ("0", "1"):
+        r = subprocess.run([sys.executable, "-c", code], env=dict(os.environ, BULLET_PF5_NQ=nq),
+                           capture_output=True, text=True, timeout=600)
+        assert r.returncode == 0, r.stderr[-3000:]
+        digests.append([l for l in r.stdout.splitlines() if l.startswith("DIGEST")][0])
+    assert digests[0] == digests[1]
