@@ -619,6 +619,23 @@ int mixed_split(const bullet_batch* b, int* t0) {
   return *t0 < b->n_tokens ? r0 : 0;
 }
 
+// TMA maps of the layer's K / V pool for the tcgen05 prefill attention: the
+// pool [blocks][Hkv][16][128] bf16 viewed as [blocks * Hkv * 16][128], boxes
+// of 16 rows (one block of one head) x 64 dims, 128-byte swizzle (the UMMA
+// operand layout).  BULLET_PF5_TMA=0 keeps every tile on cp.async (A/B).
+static int pf5_maps(bullet_handle* h, int layer, AttnArgs* a, CUtensorMap* mk, CUtensorMap* mv) {
+  static const int on = getenv("BULLET_PF5_TMA") ? atoi(getenv("BULLET_PF5_TMA")) : 1;
+  memset(mk, 0, sizeof *mk);
+  memset(mv, 0, sizeof *mv);
+  a->kv_tma = on && h->block_size == 16;
+  if (!a->kv_tma) return BULLET_OK;
+  const long long rows = (long long)h->n_blocks * h->cfg.n_kv_heads * 16;
+  if (rows >= (1ll << 31)) { a->kv_tma = 0; return BULLET_OK; }
+  int rc = make_map(mk, h->pk[layer], (int)rows, 128, 16);
+  if (!rc) rc = make_map(mv, h->pv[layer], (int)rows, 128, 16);
+  return rc;
+}
+
 int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* o, int kind) {
   bullet_handle* h = c.h;
   if (b->n_tokens == 0) return BULLET_OK;
@@ -643,9 +660,11 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
         return set_err(BULLET_EUNSUPPORTED, "hybrid batch: decode context too long");
     PhaseWS& P = h->ph[c.phase];
     a.tiles = P.tiles; a.n_tiles = P.n_tiles;   // the plan listed tiles of requests [0, r0) only
-    int rc = next_launch(c, &a.L);
+    CUtensorMap mk, mv;
+    int rc = pf5_maps(h, layer, &a, &mk, &mv);
     if (rc) return rc;
-    LAUNCH(c, launch_attn_prefill5(a, persist_grid(c, attn_prefill5_ctas_per_sm(a.H, a.Hkv)), c.st));
+    if ((rc = next_launch(c, &a.L))) return rc;
+    LAUNCH(c, launch_attn_prefill5(mk, mv, a, persist_grid(c, attn_prefill5_ctas_per_sm(a.H, a.Hkv)), c.st));
     AttnArgs d = a;
     d.tok_base = t0;
     d.order = P.order_ok ? P.order : nullptr;
@@ -687,9 +706,11 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
       prof_begin(c);
       LAUNCH(c, launch_plan(pa, c.st));
     }
-    int rc = next_launch(c, &a.L);
+    CUtensorMap mk, mv;
+    int rc = kind == 4 ? pf5_maps(h, layer, &a, &mk, &mv) : 0;
     if (rc) return rc;
-    if (kind == 4) LAUNCH(c, launch_attn_prefill5(a, persist_grid(c, attn_prefill5_ctas_per_sm(a.H, a.Hkv)), c.st));
+    if ((rc = next_launch(c, &a.L))) return rc;
+    if (kind == 4) LAUNCH(c, launch_attn_prefill5(mk, mv, a, persist_grid(c, attn_prefill5_ctas_per_sm(a.H, a.Hkv)), c.st));
     else LAUNCH(c, launch_attn_prefill_tc(a, persist_grid(c, 2), c.st));
     return BULLET_OK;
   }

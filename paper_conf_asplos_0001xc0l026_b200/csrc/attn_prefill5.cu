@@ -18,9 +18,15 @@
 //                     MN-major operand straight from its [key][dim] tile; O
 //                     stays in TMEM, rescaled only when a row max grows > 2^8
 // One warp issues S(t+1) and PV(t) back to back (an elected lane of the
-// converged warp).  K/V rows are gathered through the block table with
-// coalesced cp.async into the 128-byte-swizzled layouts the UMMA descriptors
-// describe: NKB K buffers (K(t) loads once S(t-NKB) is done), two V buffers.
+// converged warp).  K/V tiles are fed by TMA: the pool viewed as a 2-D tensor
+// [blocks * Hkv * 16 rows][128 dims] with 16 x 64-element boxes and the
+// 128-byte swizzle, so a (block, head) half-chunk lands in exactly the
+// swizzled layout the UMMA descriptors describe — 8 copies of 2 KB per 64-key
+// operand tile, issued by one elected lane, completion counted in bytes on
+// the tile's mbarrier.  The last tile of a sequence (rows past its end must
+// read as zeros: P = 0 times a stale non-finite V would poison O) is gathered
+// with zero-filling cp.async instead, as is every tile when a.kv_tma = 0.
+// NKB K buffers (K(t) loads once S(t-NKB) is done), two V buffers.
 // Measured (round 2, scripts/attn_pre_bench.py): the gathers, not the MMAs,
 // bound the NQ = 1 kernel (without them it runs at 0.65 of the bf16 peak,
 // with them 0.47; loading every other tile only: 0.55), hence NQ = 2.
@@ -232,10 +238,32 @@ __device__ __forceinline__ void load_kv_tile(uint8_t* dst, const __nv_bfloat16* 
   }
   cp_async_arrive_noinc(bar);
 }
+// KV tile kt by TMA (a full tile: every row inside the sequence).  The whole
+// warp calls it: the block ids come from the lanes' window, one elected lane
+// arms the barrier with the tile's bytes and issues the 8 copies (4 blocks x
+// 2 halves of 64 dims), the other lanes arrive plainly (the barrier counts
+// 32 arrivals per loader warp whichever path fed the tile).
+__device__ __forceinline__ void tma_kv_tile(uint8_t* dst, const CUtensorMap* map, const AttnArgs& a,
+                                            const Unit& U, int kt, uint64_t* bar, const BtWin& w) {
+  int blk[BKV / KB];
+#pragma unroll
+  for (int b = 0; b < BKV / KB; ++b) blk[b] = __shfl_sync(0xffffffffu, w.cur, (kt % 8) * (BKV / KB) + b);
+  if (elect_one()) {
+    mbar_arrive_expect_tx(bar, BKV * HD * 2);
+#pragma unroll
+    for (int b = 0; b < BKV / KB; ++b)
+#pragma unroll
+      for (int half = 0; half < 2; ++half)
+        tma_load_2d(dst + half * 8192 + b * KB * 128, map, bar, half * 64, (blk[b] * a.Hkv + U.g) * KB);
+  } else {
+    mbar_arrive(bar);
+  }
+}
 }  // namespace
 
 template <int NQ>
-__global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS) k_attn_prefill5(AttnArgs a) {
+__global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS)
+    k_attn_prefill5(const __grid_constant__ CUtensorMap mk, const __grid_constant__ CUtensorMap mv, AttnArgs a) {
   using C = Cfg<NQ>;
   constexpr int NKB = C::NKB, W_LOAD = C::W_LOAD, W_VLOAD = C::W_VLOAD, W_MMA = C::W_MMA, NLW = C::NLW;
   constexpr int NBW = BKV / KB / NLW;   // blocks of a KV tile per loader warp
@@ -326,7 +354,12 @@ __global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS) k_attn_prefill5(At
         const int kb = g % NKB;
         if (kt > 0 && kt % 8 == 0) w.advance(bt, n_blk, kt, lane);
         if (g >= NKB) wait(kempty + kb, (g / NKB - 1) & 1);
-        load_kv_tile<NBW>(sm + OFF_K + kb * 16384, pk, a, U, kt, lane, kfull + kb, w, lw * NBW);
+        if (a.kv_tma && (kt + 1) * BKV <= U.kv_len) {
+          if (lw == 0) tma_kv_tile(sm + OFF_K + kb * 16384, &mk, a, U, kt, kfull + kb, w);
+          else mbar_arrive(kfull + kb);
+        } else {
+          load_kv_tile<NBW>(sm + OFF_K + kb * 16384, pk, a, U, kt, lane, kfull + kb, w, lw * NBW);
+        }
         if (kt == 0) {
           if (n >= 1) wait(qempty, (n - 1) & 1);         // last S of the previous unit done
 #pragma unroll
@@ -365,7 +398,12 @@ __global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS) k_attn_prefill5(At
         if (g >= 2)
 #pragma unroll
           for (int q = 0; q < NQ; ++q) wait(pvdone + q * 2 + b, ((g - 2) >> 1) & 1);
-        load_kv_tile<NBW>(sm + OFF_V + b * 16384, pv, a, U, kt, lane, vfull + b, w, lw * NBW);
+        if (a.kv_tma && (kt + 1) * BKV <= U.kv_len) {
+          if (lw == 0) tma_kv_tile(sm + OFF_V + b * 16384, &mv, a, U, kt, vfull + b, w);
+          else mbar_arrive(vfull + b);
+        } else {
+          load_kv_tile<NBW>(sm + OFF_V + b * 16384, pv, a, U, kt, lane, vfull + b, w, lw * NBW);
+        }
       }
     }
   } else if (warp >= W_MMA) {
@@ -570,19 +608,23 @@ int attn_prefill5_nq(int H, int Hkv) {
 int attn_prefill5_ctas_per_sm(int H, int Hkv) { return attn_prefill5_nq(H, Hkv) == 2 ? 1 : 2; }
 
 template <int NQ>
-static cudaError_t launch_nq(const AttnArgs& a, int grid, cudaStream_t st) {
+static cudaError_t launch_nq(const CUtensorMap& mk, const CUtensorMap& mv, const AttnArgs& a, int grid,
+                             cudaStream_t st) {
   static bool set = false;
   if (!set) {
     cudaError_t e = cudaFuncSetAttribute(k_attn_prefill5<NQ>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<NQ>::SMEM_BYTES);
     if (e != cudaSuccess) return e;
     set = true;
   }
-  return launch_ex(k_attn_prefill5<NQ>, grid, Cfg<NQ>::NT, Cfg<NQ>::SMEM_BYTES, st, a.L.pdl, a);
+  return launch_ex(k_attn_prefill5<NQ>, grid, Cfg<NQ>::NT, Cfg<NQ>::SMEM_BYTES, st, a.L.pdl, mk, mv, a);
 }
 
 // `grid` must be n_sms * attn_prefill5_ctas_per_sm(H, Hkv) (persistent, gated).
-cudaError_t launch_attn_prefill5(const AttnArgs& a, int grid, cudaStream_t st) {
-  return attn_prefill5_nq(a.H, a.Hkv) == 2 ? launch_nq<2>(a, grid, st) : launch_nq<1>(a, grid, st);
+// mk / mv: the layer's K / V pool as [blocks * Hkv * 16][128] bf16 tensors,
+// box {64, 16}, 128-byte swizzle (used when a.kv_tma != 0).
+cudaError_t launch_attn_prefill5(const CUtensorMap& mk, const CUtensorMap& mv, const AttnArgs& a, int grid,
+                                 cudaStream_t st) {
+  return attn_prefill5_nq(a.H, a.Hkv) == 2 ? launch_nq<2>(mk, mv, a, grid, st) : launch_nq<1>(mk, mv, a, grid, st);
 }
 
 cudaError_t preload_attn_prefill5() {

@@ -506,3 +506,37 @@ def test_prefill_attention_gqa_pair_bit_identical():
         assert r.returncode == 0, r.stderr[-3000:]
         digests.append([l for l in r.stdout.splitlines() if l.startswith("DIGEST")][0])
     assert digests[0] == digests[1]
+
+
+def test_prefill_attention_tma_kv_bit_identical():
+    """K / V tiles fed by TMA (the default: a full 64-key tile is 8 boxes of
+    16 pool rows x 64 dims, 128-byte swizzle) land in the same swizzled
+    shared-memory layout as the cp.async gathers: a two-layer co-run step with
+    ragged prompts (full tiles, partial last tiles, a 1-token prompt, a
+    16-aligned prompt) gives the same bits with BULLET_PF5_TMA=0 (every tile
+    gathered by cp.async, fresh process), for both the GQA-pair and the
+    one-head kernel."""
+    import os
+    import subprocess
+    import sys
+    here = os.path.dirname(os.path.abspath(__file__))
+    code = ("import sys; sys.path[:0] = [%r, %r]\n"
+            "import torch, hashlib\n"
+            "from harness import Setup, phase_streams\n"
+            "from workload import synth\n"
+            "m = synth.ModelShape('gqa', 1024, 8, 2, 128, 2816, 2)\n"
+            "S = Setup(m, [300, 77, 1, 129, 256], [64, 1, 500, 31], n_layers=2)\n"
+            "pre, dec = S.batches()\n"
+            "S.bl.step(pre, dec, 64, S.B.CORUN, *phase_streams())\n"
+            "torch.cuda.synchronize()\n"
+            "h = hashlib.sha256(pre.hidden.cpu().numpy().tobytes() + dec.hidden.cpu().numpy().tobytes())\n"
+            "print('DIGEST', h.hexdigest())\n") % (here, os.path.dirname(here))
+    for nq in ("0", "1"):
+        digests = []
+        for tma in ("1", "0"):
+            r = subprocess.run([sys.executable, "-c", code],
+                               env=dict(os.environ, BULLET_PF5_TMA=tma, BULLET_PF5_NQ=nq),
+                               capture_output=True, text=True, timeout=600)
+            assert r.returncode == 0, r.stderr[-3000:]
+            digests.append([l for l in r.stdout.splitlines() if l.startswith("DIGEST")][0])
+        assert digests[0] == digests[1], nq
