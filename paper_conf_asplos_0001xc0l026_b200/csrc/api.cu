@@ -522,6 +522,12 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
     a.band = std::max(1, (m_tiles + n_bands - 1) / n_bands);   // equal bands
   }
   a.b_packed = Bp;
+  {   // epilogue-input L2 prefetch (BULLET_GEMM_EPI_PF=0 disables, A/B) and diagnostics
+    static const int epf = getenv("BULLET_GEMM_EPI_PF") ? atoi(getenv("BULLET_GEMM_EPI_PF")) : 1;
+    static const int edbg = getenv("BULLET_GEMM_EPI_DBG") ? atoi(getenv("BULLET_GEMM_EPI_DBG")) : 0;
+    static const int ecoal = getenv("BULLET_GEMM_EPI_COAL") ? atoi(getenv("BULLET_GEMM_EPI_COAL")) : 1;
+    a.epi_pf = epf; a.epi_dbg = edbg; a.epi_coal = ecoal;
+  }
   {   // L2 prefetch distance of the weight stream (experiments; BULLET_GEMM_PF k-blocks)
     static const int pf = getenv("BULLET_GEMM_PF") ? atoi(getenv("BULLET_GEMM_PF")) : 0;
     a.b_pf = pf;
@@ -623,17 +629,28 @@ int mixed_split(const bullet_batch* b, int* t0) {
 // pool [blocks][Hkv][16][128] bf16 viewed as [blocks * Hkv * 16][128], boxes
 // of 16 rows (one block of one head) x 64 dims, 128-byte swizzle (the UMMA
 // operand layout).  BULLET_PF5_TMA=0 keeps every tile on cp.async (A/B).
-static int pf5_maps(bullet_handle* h, int layer, AttnArgs* a, CUtensorMap* mk, CUtensorMap* mv) {
+static int pf5_maps(bullet_handle* h, int layer, AttnArgs* a, CUtensorMap* mk, CUtensorMap* mv, CUtensorMap* mq) {
   static const int on = getenv("BULLET_PF5_TMA") ? atoi(getenv("BULLET_PF5_TMA")) : 1;
   memset(mk, 0, sizeof *mk);
   memset(mv, 0, sizeof *mv);
+  memset(mq, 0, sizeof *mq);
   a->kv_tma = on && h->block_size == 16;
   if (!a->kv_tma) return BULLET_OK;
   const long long rows = (long long)h->n_blocks * h->cfg.n_kv_heads * 16;
   if (rows >= (1ll << 31)) { a->kv_tma = 0; return BULLET_OK; }
   int rc = make_map(mk, h->pk[layer], (int)rows, 128, 16);
   if (!rc) rc = make_map(mv, h->pv[layer], (int)rows, 128, 16);
-  return rc;
+  if (rc) return rc;
+  // q [T][H][128] bf16: box {64 dims, 1 head, 128 tokens}
+  cuuint64_t dims[3] = {128, (cuuint64_t)a->H, (cuuint64_t)a->n_tok};
+  cuuint64_t strides[2] = {128 * 2, (cuuint64_t)a->H * 128 * 2};
+  cuuint32_t box[3] = {64, 1, 128};
+  cuuint32_t es[3] = {1, 1, 1};
+  CUresult r = g_encode(mq, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(a->q), dims, strides, box, es,
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_err(BULLET_ECUDA, "cuTensorMapEncodeTiled (q) failed (%d)", (int)r);
+  return BULLET_OK;
 }
 
 int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* o, int kind) {
@@ -660,11 +677,11 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
         return set_err(BULLET_EUNSUPPORTED, "hybrid batch: decode context too long");
     PhaseWS& P = h->ph[c.phase];
     a.tiles = P.tiles; a.n_tiles = P.n_tiles;   // the plan listed tiles of requests [0, r0) only
-    CUtensorMap mk, mv;
-    int rc = pf5_maps(h, layer, &a, &mk, &mv);
+    CUtensorMap mk, mv, mq;
+    int rc = pf5_maps(h, layer, &a, &mk, &mv, &mq);
     if (rc) return rc;
     if ((rc = next_launch(c, &a.L))) return rc;
-    LAUNCH(c, launch_attn_prefill5(mk, mv, a, persist_grid(c, attn_prefill5_ctas_per_sm(a.H, a.Hkv)), c.st));
+    LAUNCH(c, launch_attn_prefill5(mk, mv, mq, a, persist_grid(c, attn_prefill5_ctas_per_sm(a.H, a.Hkv)), c.st));
     AttnArgs d = a;
     d.tok_base = t0;
     d.order = P.order_ok ? P.order : nullptr;
@@ -706,11 +723,11 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
       prof_begin(c);
       LAUNCH(c, launch_plan(pa, c.st));
     }
-    CUtensorMap mk, mv;
-    int rc = kind == 4 ? pf5_maps(h, layer, &a, &mk, &mv) : 0;
+    CUtensorMap mk, mv, mq;
+    int rc = kind == 4 ? pf5_maps(h, layer, &a, &mk, &mv, &mq) : 0;
     if (rc) return rc;
     if ((rc = next_launch(c, &a.L))) return rc;
-    if (kind == 4) LAUNCH(c, launch_attn_prefill5(mk, mv, a, persist_grid(c, attn_prefill5_ctas_per_sm(a.H, a.Hkv)), c.st));
+    if (kind == 4) LAUNCH(c, launch_attn_prefill5(mk, mv, mq, a, persist_grid(c, attn_prefill5_ctas_per_sm(a.H, a.Hkv)), c.st));
     else LAUNCH(c, launch_attn_prefill_tc(a, persist_grid(c, 2), c.st));
     return BULLET_OK;
   }

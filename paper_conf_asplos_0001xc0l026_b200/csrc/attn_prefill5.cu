@@ -18,7 +18,9 @@
 //                     MN-major operand straight from its [key][dim] tile; O
 //                     stays in TMEM, rescaled only when a row max grows > 2^8
 // One warp issues S(t+1) and PV(t) back to back (an elected lane of the
-// converged warp).  K/V tiles are fed by TMA: the pool viewed as a 2-D tensor
+// converged warp).  Q, K and V tiles are fed by TMA (Q: [T][H][128] boxes of
+// 128 tokens x 64 dims of one head; rows past the batch read as zeros, rows
+// of the next request are never stored): the pool viewed as a 2-D tensor
 // [blocks * Hkv * 16 rows][128 dims] with 16 x 64-element boxes and the
 // 128-byte swizzle, so a (block, head) half-chunk lands in exactly the
 // swizzled layout the UMMA descriptors describe — 8 copies of 2 KB per 64-key
@@ -263,7 +265,8 @@ __device__ __forceinline__ void tma_kv_tile(uint8_t* dst, const CUtensorMap* map
 
 template <int NQ>
 __global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS)
-    k_attn_prefill5(const __grid_constant__ CUtensorMap mk, const __grid_constant__ CUtensorMap mv, AttnArgs a) {
+    k_attn_prefill5(const __grid_constant__ CUtensorMap mk, const __grid_constant__ CUtensorMap mv,
+                    const __grid_constant__ CUtensorMap mq, AttnArgs a) {
   using C = Cfg<NQ>;
   constexpr int NKB = C::NKB, W_LOAD = C::W_LOAD, W_VLOAD = C::W_VLOAD, W_MMA = C::W_MMA, NLW = C::NLW;
   constexpr int NBW = BKV / KB / NLW;   // blocks of a KV tile per loader warp
@@ -360,7 +363,19 @@ __global__ void __launch_bounds__(Cfg<NQ>::NT, Cfg<NQ>::CTAS)
         } else {
           load_kv_tile<NBW>(sm + OFF_K + kb * 16384, pk, a, U, kt, lane, kfull + kb, w, lw * NBW);
         }
-        if (kt == 0) {
+        if (kt == 0 && a.kv_tma) {   // Q tiles by TMA: [T][H][128] boxes {64 dims, 1 head, 128 tokens}
+          if (n >= 1) wait(qempty, (n - 1) & 1);         // last S of the previous unit done
+          if (lw == 0 && elect_one()) {
+            mbar_arrive_expect_tx(qfull, NQ * BQ * HD * 2);
+#pragma unroll
+            for (int q = 0; q < NQ; ++q)
+#pragma unroll
+              for (int half = 0; half < 2; ++half)
+                tma_load_3d(sm + OFF_Q + q * 32768 + half * 16384, &mq, qfull, half * 64, U.h + q, U.tok0 + U.q0);
+          } else {
+            mbar_arrive(qfull);
+          }
+        } else if (kt == 0) {
           if (n >= 1) wait(qempty, (n - 1) & 1);         // last S of the previous unit done
 #pragma unroll
           for (int q = 0; q < NQ; ++q) {
@@ -608,23 +623,25 @@ int attn_prefill5_nq(int H, int Hkv) {
 int attn_prefill5_ctas_per_sm(int H, int Hkv) { return attn_prefill5_nq(H, Hkv) == 2 ? 1 : 2; }
 
 template <int NQ>
-static cudaError_t launch_nq(const CUtensorMap& mk, const CUtensorMap& mv, const AttnArgs& a, int grid,
-                             cudaStream_t st) {
+static cudaError_t launch_nq(const CUtensorMap& mk, const CUtensorMap& mv, const CUtensorMap& mq, const AttnArgs& a,
+                             int grid, cudaStream_t st) {
   static bool set = false;
   if (!set) {
     cudaError_t e = cudaFuncSetAttribute(k_attn_prefill5<NQ>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<NQ>::SMEM_BYTES);
     if (e != cudaSuccess) return e;
     set = true;
   }
-  return launch_ex(k_attn_prefill5<NQ>, grid, Cfg<NQ>::NT, Cfg<NQ>::SMEM_BYTES, st, a.L.pdl, mk, mv, a);
+  return launch_ex(k_attn_prefill5<NQ>, grid, Cfg<NQ>::NT, Cfg<NQ>::SMEM_BYTES, st, a.L.pdl, mk, mv, mq, a);
 }
 
 // `grid` must be n_sms * attn_prefill5_ctas_per_sm(H, Hkv) (persistent, gated).
 // mk / mv: the layer's K / V pool as [blocks * Hkv * 16][128] bf16 tensors,
-// box {64, 16}, 128-byte swizzle (used when a.kv_tma != 0).
-cudaError_t launch_attn_prefill5(const CUtensorMap& mk, const CUtensorMap& mv, const AttnArgs& a, int grid,
-                                 cudaStream_t st) {
-  return attn_prefill5_nq(a.H, a.Hkv) == 2 ? launch_nq<2>(mk, mv, a, grid, st) : launch_nq<1>(mk, mv, a, grid, st);
+// box {64, 16}; mq: q as [T][H][128], box {64, 1, 128}; 128-byte swizzle
+// (used when a.kv_tma != 0).
+cudaError_t launch_attn_prefill5(const CUtensorMap& mk, const CUtensorMap& mv, const CUtensorMap& mq,
+                                 const AttnArgs& a, int grid, cudaStream_t st) {
+  return attn_prefill5_nq(a.H, a.Hkv) == 2 ? launch_nq<2>(mk, mv, mq, a, grid, st)
+                                           : launch_nq<1>(mk, mv, mq, a, grid, st);
 }
 
 cudaError_t preload_attn_prefill5() {

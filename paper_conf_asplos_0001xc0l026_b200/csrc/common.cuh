@@ -55,7 +55,8 @@ __device__ __forceinline__ unsigned long long gtimer() {
 // Per-CTA trace record (bullet_trace_enable, diagnostics only): slot 0 smid,
 // 1 entry, 2 first MMA operand stage ready, 3 MMA issue done, 4 epilogue
 // done, 5 exit, 6 work units (queue entries), 7 last partial stored + fenced,
-// 8 first fixup start, 9 last fixup end, 10 fixups done.  Written by one
+// 8 first fixup start, 9 last fixup end, 10 fixups done, 15 the epilogue's
+// last accumulator ready (GEMM).  Written by one
 // thread per slot.
 constexpr int TRACE_SLOTS = 16;
 __device__ __forceinline__ void trace_at(const Launch& L, int slot, unsigned long long v) {
@@ -174,6 +175,14 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, u
       "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
       " [%0], [%1, {%3, %4}], [%2];" ::"r"(smem_u32(dst)),
       "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, uint64_t* bar,
+                                            int c0, int c1, int c2) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2)
       : "memory");
 }
 __device__ __forceinline__ void tma_prefetch_desc(const CUtensorMap* map) {

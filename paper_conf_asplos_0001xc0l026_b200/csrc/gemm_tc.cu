@@ -111,7 +111,12 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
   for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
 }
 
-__device__ __forceinline__ float silu_f(float z) { return z / (1.0f + __expf(-z)); }
+// silu(z) = z / (1 + e^-z) with the MUFU exponential and reciprocal (~1e-7
+// relative error, far below the bf16 rounding R5 that follows; the IEEE
+// division's slow path made the SiLU epilogue of a decode gate_up tile cost
+// ~6 us, scripts/trace_step.py with BULLET_GEMM_EPI_DBG=1).  e^-z = inf for
+// z < -88 gives z * 0 = -0, as the exact expression does.
+__device__ __forceinline__ float silu_f(float z) { return __fdividef(z, 1.0f + __expf(-z)); }
 
 // L2 cache policies: activation tiles are re-read by every N tile (evict
 // last); decode-sized GEMMs (one M tile) stream each weight tile once (evict
@@ -168,23 +173,31 @@ __device__ __forceinline__ void epi_store(const GemmArgs& a, int m, int col, con
   } else if (a.epi == EPI_RESID) {
     const float4* r = reinterpret_cast<const float4*>(a.resid + o);
     float4* dst = reinterpret_cast<float4*>(a.out_f32 + o);
+    const bool ld = !(a.epi_dbg & 4), st = !(a.epi_dbg & 2);
+    // all loads before the first store: resid may alias out, so a load after
+    // a store could not be hoisted and each would pay its own L2 round trip
+    float4 rr[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) rr[i] = ld ? r[i] : make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
-      float4 w = r[i];
+      float4 w = rr[i];
       w.x += v[4 * i]; w.y += v[4 * i + 1]; w.z += v[4 * i + 2]; w.w += v[4 * i + 3];
-      dst[i] = w;
+      if (st) dst[i] = w;
     }
   } else {  // EPI_SILU: out = silu(gate) * up, bf16
     uint32_t p[16];
+    const bool math = !(a.epi_dbg & 1);
 #pragma unroll
     for (int i = 0; i < 16; ++i) {
-      __nv_bfloat162 h = __floats2bfloat162_rn(silu_f(v[2 * i]) * u[2 * i],
-                                              silu_f(v[2 * i + 1]) * u[2 * i + 1]);
+      __nv_bfloat162 h = math ? __floats2bfloat162_rn(silu_f(v[2 * i]) * u[2 * i], silu_f(v[2 * i + 1]) * u[2 * i + 1])
+                              : __floats2bfloat162_rn(v[2 * i], u[2 * i + 1]);
       p[i] = *reinterpret_cast<uint32_t*>(&h);
     }
     uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(a.out_t) + o);
+    if (!(a.epi_dbg & 2))
 #pragma unroll
-    for (int i = 0; i < 4; ++i) dst[i] = make_uint4(p[4 * i], p[4 * i + 1], p[4 * i + 2], p[4 * i + 3]);
+      for (int i = 0; i < 4; ++i) dst[i] = make_uint4(p[4 * i], p[4 * i + 1], p[4 * i + 2], p[4 * i + 3]);
   }
 }
 
@@ -203,9 +216,10 @@ __device__ __forceinline__ void epi_qkv(const GemmArgs& a, int m, int col, float
   __nv_bfloat16* dst;
   if (head < a.H + a.Hkv) {
     const float4* cs = reinterpret_cast<const float4*>(a.cs + (size_t)ti.x * 64 + i0);
+    const bool ld = !(a.epi_dbg & 8);
 #pragma unroll
     for (int j = 0; j < 16; ++j) {
-      const float4 c = cs[j];   // (cos, sin) of frequencies i0 + 2j, i0 + 2j + 1
+      const float4 c = ld ? cs[j] : make_float4(1.f, 0.f, 1.f, 0.f);   // (cos, sin) of frequencies i0 + 2j, i0 + 2j + 1
       const float x0 = v[2 * j], x1 = w[2 * j], y0 = v[2 * j + 1], y1 = w[2 * j + 1];
       v[2 * j] = x0 * c.x - x1 * c.y;
       w[2 * j] = x1 * c.x + x0 * c.y;
@@ -229,11 +243,89 @@ __device__ __forceinline__ void epi_qkv(const GemmArgs& a, int m, int col, float
   }
   uint4* d0 = reinterpret_cast<uint4*>(dst + i0);
   uint4* d1 = reinterpret_cast<uint4*>(dst + 64 + i0);
+  if (a.epi_dbg & 2) return;
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
     d0[i] = make_uint4(p[4 * i], p[4 * i + 1], p[4 * i + 2], p[4 * i + 3]);
     d1[i] = make_uint4(q[4 * i], q[4 * i + 1], q[4 * i + 2], q[4 * i + 3]);
   }
+}
+
+// Epilogue inputs of row m of a tile at output column col0 (w columns), pulled
+// into L2 by the epilogue thread that owns the row as soon as it learns the
+// unit — the mainloop then hides their DRAM latency (the decode attention
+// that precedes the O-proj / QKV GEMMs streams GBs of KV past them, so the
+// residual rows and the RoPE rows are usually gone from L2 by then; measured:
+// 4-13 us epilogues on decode-sized GEMMs, scripts/trace_step.py).
+__device__ __forceinline__ void epi_prefetch(const GemmArgs& a, int m, int col0, int w) {
+  if (m >= a.M) return;
+  if (a.epi == EPI_RESID) {
+    prefetch_l2(a.resid + (size_t)m * a.ldo + col0, (uint32_t)w * 4);
+  } else if (a.epi == EPI_QKV) {
+    const TokInfo ti = a.tok[m];
+    prefetch_l2(a.cs + (size_t)ti.x * 64, 64 * sizeof(float2));
+  }
+}
+
+// Coalesced epilogue of one 32-column chunk for EPI_RESID / EPI_SILU: the
+// warp's 32 rows (one per lane, as they come out of TMEM) are transposed
+// through a 32 x 33-word shared-memory buffer so every global access of the
+// warp covers whole row segments — the residual loads and fp32 stores as
+// 4 rows x 128 B per instruction, the bf16 SiLU stores as 8 rows x 64 B —
+// instead of 32 rows x 16 B (per-row vectors: 8x the L2 transactions,
+// measured 5-11 us per decode-sized O-proj / down tile, BULLET_GEMM_EPI_DBG).
+// Same arithmetic per element as epi_store (out = resid + acc; silu(g) * u
+// rounded once to bf16): bit-identical.
+// residual of the warp's rows [m0, m0 + 32) at columns [col, col + 32) in the
+// transposed layout (lane: column quad lane & 7 of rows it * 4 + lane / 8)
+__device__ __forceinline__ void epi_resid_load(const GemmArgs& a, int m0, int col, int lane, float4* rr) {
+  const int cq = lane & 7;
+#pragma unroll
+  for (int it = 0; it < 8; ++it) {
+    const int m = m0 + it * 4 + (lane >> 3);
+    rr[it] = (m < a.M && !(a.epi_dbg & 4)) ? *reinterpret_cast<const float4*>(a.resid + (size_t)m * a.ldo + col + 4 * cq)
+                                           : make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+}
+// rr: the chunk's residual from epi_resid_load (loaded ahead: resid may alias
+// out_f32, so loads issued after a store could not be hoisted)
+__device__ __forceinline__ void epi_chunk_coalesced(const GemmArgs& a, float* wb, int m0, int col, int lane,
+                                                    const float* v, const float* u, const float4* rr) {
+  if (a.epi == EPI_RESID) {
+#pragma unroll
+    for (int j = 0; j < 32; ++j) wb[lane * 33 + j] = v[j];
+    __syncwarp();
+    const int cq = lane & 7;
+#pragma unroll
+    for (int it = 0; it < 8; ++it) {
+      const int r = it * 4 + (lane >> 3), m = m0 + r;
+      if (m < a.M) {
+        float4 w = rr[it];
+        w.x += wb[r * 33 + 4 * cq]; w.y += wb[r * 33 + 4 * cq + 1];
+        w.z += wb[r * 33 + 4 * cq + 2]; w.w += wb[r * 33 + 4 * cq + 3];
+        if (!(a.epi_dbg & 2)) *reinterpret_cast<float4*>(a.out_f32 + (size_t)m * a.ldo + col + 4 * cq) = w;
+      }
+    }
+  } else {   // EPI_SILU: 32 bf16 outputs per row, 16 words
+    uint32_t* wu = reinterpret_cast<uint32_t*>(wb);
+    const bool math = !(a.epi_dbg & 1);
+#pragma unroll
+    for (int i = 0; i < 16; ++i) {
+      __nv_bfloat162 h = math ? __floats2bfloat162_rn(silu_f(v[2 * i]) * u[2 * i], silu_f(v[2 * i + 1]) * u[2 * i + 1])
+                              : __floats2bfloat162_rn(v[2 * i], u[2 * i + 1]);
+      wu[lane * 17 + i] = *reinterpret_cast<uint32_t*>(&h);
+    }
+    __syncwarp();
+    const int q = lane & 3;
+#pragma unroll
+    for (int it = 0; it < 4; ++it) {
+      const int r = it * 8 + (lane >> 2), m = m0 + r;
+      if (m < a.M && !(a.epi_dbg & 2))
+        *reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(a.out_t) + (size_t)m * a.ldo + col + 8 * q) =
+            make_uint4(wu[r * 17 + 4 * q], wu[r * 17 + 4 * q + 1], wu[r * 17 + 4 * q + 2], wu[r * 17 + 4 * q + 3]);
+    }
+  }
+  __syncwarp();   // the buffer is reused by the next chunk
 }
 
 // ---------------------------------------------------------------- fused all-reduce (kernels.h ArArgs)
@@ -603,7 +695,7 @@ int gemm_tc_stages(int bn, int mh) {
 }
 size_t gemm_tc_smem_bytes(int bn, int mh) {
   const int st = mh * A_BYTES + bn * BK * 2;
-  return (size_t)gemm_tc_stages(bn, mh) * st + 1024 /*align*/ + 512 /*barriers etc.*/;
+  return (size_t)gemm_tc_stages(bn, mh) * st + 1024 /*align*/ + 512 /*barriers etc.*/ + 4 * 32 * 33 * 4 /*epilogue*/;
 }
 
 template <int mh, bool KC = false>
@@ -621,6 +713,7 @@ __global__ void __launch_bounds__(NT, 1)
   const uint32_t acc_cols = mh * bn;
   const int n_acc = 2 * acc_cols <= 512 ? 2 : 1;
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + n_stages * st_bytes);
+  const uint32_t epi_off = n_stages * st_bytes + 512;   // 4 x [32][33] words: coalesced epilogue
   uint64_t* empty = full + n_stages;
   uint64_t* accf = empty + n_stages;
   uint64_t* acce = accf + 2;
@@ -884,6 +977,14 @@ __global__ void __launch_bounds__(NT, 1)
       tile_coords(g.tile, m_tiles, n_tiles, a.band, m_blk, n_blk);
       const int col0 = (a.epi == EPI_SILU) ? n_blk * (bn / 2) : n_blk * bn;
       const int out_chunks = (a.epi == EPI_SILU) ? bn / 64 : bn / 32;
+      if (a.epi_pf && (g.slot < 0 || KC))   // this unit's epilogue runs here: warm its inputs in L2
+        for (int hh = 0; hh < (KC ? 1 : mh); ++hh) epi_prefetch(a, (m_blk * mh + hh) * BM + et, col0, bn);
+      // coalesced residual epilogue: the first chunk's residual is loaded
+      // before the accumulator wait (it does not depend on it), each next
+      // chunk's while the current one is stored
+      const bool coal_resid = !KC && g.slot < 0 && a.epi == EPI_RESID && a.epi_coal;
+      float4 rr[8];
+      if (coal_resid) epi_resid_load(a, m_blk * mh * BM + eq * 32, col0, lane, rr);
       if constexpr (KC) {   // mh == 1, bn == 128, whole tiles (plan guarantees)
         const int n_ch = (k_blocks + a.kcb - 1) / a.kcb;
         float R[128];
@@ -922,6 +1023,7 @@ __global__ void __launch_bounds__(NT, 1)
       }
       mbar_wait(accf + as, aph);
       tc_fence_after();
+      if (et == 0 && a.L.trace) trace_at(a.L, 15, gtimer());   // (last) accumulator ready
       const uint32_t tb = tmem + ((uint32_t)(eq * 32) << 16) + as * acc_cols;
       if (g.slot < 0) {   // whole tile: epilogue straight from TMEM
         for (int hh = 0; hh < mh; ++hh) {
@@ -933,6 +1035,31 @@ __global__ void __launch_bounds__(NT, 1)
                 tmem_ld32(tb + hh * bn + c0 + 64 + c, w);
                 if (m < a.M) epi_qkv(a, m, col0 + c0 + c, v, w);
               }
+            continue;
+          }
+          if (coal_resid) {
+            float* wb = reinterpret_cast<float*>(smem + epi_off) + eq * (32 * 33);
+            for (int c = 0; c < out_chunks; ++c) {
+              float4 rn[8];
+              const bool more = c + 1 < out_chunks || hh + 1 < mh;
+              if (more)   // next chunk (or the next 128-row half's first) in flight now
+                epi_resid_load(a, (c + 1 < out_chunks ? m : m + BM) - lane, col0 + (c + 1 < out_chunks ? (c + 1) * 32 : 0),
+                               lane, rn);
+              tmem_ld32(tb + hh * bn + c * 32, v);
+              epi_chunk_coalesced(a, wb, m - lane, col0 + c * 32, lane, v, nullptr, rr);
+              if (more)
+#pragma unroll
+                for (int i = 0; i < 8; ++i) rr[i] = rn[i];
+            }
+            continue;
+          }
+          if (a.epi == EPI_SILU && a.epi_coal) {
+            float* wb = reinterpret_cast<float*>(smem + epi_off) + eq * (32 * 33);
+            for (int c = 0; c < out_chunks; ++c) {
+              tmem_ld32(tb + hh * bn + c * 32, v);
+              tmem_ld32(tb + hh * bn + bn / 2 + c * 32, w);
+              epi_chunk_coalesced(a, wb, m - lane, col0 + c * 32, lane, v, w, nullptr);
+            }
             continue;
           }
           for (int c = 0; c < out_chunks; ++c) {

@@ -75,6 +75,12 @@ struct GemmArgs {
   int b_rows;               // rows of B (packed layout stride)
   int split_b;              // 1: warp 3 issues the B tiles (second copy issuer), warp 0 the A tiles
   int b_pf;                 // warp 3 prefetches packed B k-block kb + b_pf into L2 (0 = off)
+  int epi_coal;             // EPI_RESID / EPI_SILU whole tiles: rows transposed through shared memory so the
+                            // warp's global loads / stores cover whole row segments (1 = on)
+  int epi_pf;               // epilogue warps L2-prefetch their tile's inputs (residual rows, RoPE rows)
+                            // when they learn the unit, i.e. while the mainloop streams (1 = on)
+  int epi_dbg;              // diagnostics (BULLET_GEMM_EPI_DBG; wrong results): bit 0 no SiLU math,
+                            // bit 1 no output stores, bit 2 no residual loads, bit 3 no RoPE-table loads
   int kcb;                  // two-level accumulation (DESIGN R-4e): K chunk in k-blocks (0 = off);
                             // each chunk accumulates in TMEM, the chunks are summed in fp32
                             // registers by the epilogue (requires mh == 1, bn == 128, whole tiles)
@@ -128,7 +134,7 @@ struct AttnArgs {
   float* kv_part;         // [units][kv_chunks][8][128 + 2] (kv_chunks > 1)
   int* kv_tick;           // [units], zero between launches (self-resetting)
   int dec_pf;             // decode kernel: L2 prefetch distance (blocks of a warp's stream; 0 = off)
-  int kv_tma;             // prefill tcgen05 kernel: full K/V tiles by TMA (else cp.async gathers)
+  int kv_tma;             // prefill tcgen05 kernel: Q and full K/V tiles by TMA (else cp.async gathers)
   Launch L;
 };
 
@@ -182,8 +188,8 @@ cudaError_t launch_rope_kv(const RopeArgs& a, int grid, cudaStream_t st);
 template <typename T>
 cudaError_t launch_attn_simt(const AttnArgs& a, int grid, cudaStream_t st);
 cudaError_t launch_attn_prefill_tc(const AttnArgs& a, int grid, cudaStream_t st);
-cudaError_t launch_attn_prefill5(const CUtensorMap& mk, const CUtensorMap& mv, const AttnArgs& a, int grid,
-                                 cudaStream_t st);
+cudaError_t launch_attn_prefill5(const CUtensorMap& mk, const CUtensorMap& mv, const CUtensorMap& mq,
+                                 const AttnArgs& a, int grid, cudaStream_t st);
 int attn_prefill5_ctas_per_sm(int H, int Hkv);   // grid = n_sms * this (2 query tiles per CTA for even GQA groups)
 cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStream_t st);
 size_t attn_decode_smem_bytes();

@@ -40,6 +40,9 @@ def analyse(rec, meta):
             row["mma_done_us_med"] = us(np.median(g[:, 3] - t0))
             row["mma_done_us_max"] = us(g[:, 3].max() - t0)
             row["epi_done_us_max"] = us(g[:, 4].max() - t0)
+            if (g[:, 15] > 0).any():   # last accumulator ready (the MMAs of the CTA's last unit complete)
+                row["acc_ready_us_med"] = us(np.median(g[g[:, 15] > 0][:, 15] - t0))
+                row["acc_ready_us_max"] = us(g[:, 15].max() - t0)
             row["exit_us_med"] = us(np.median(g[:, 5] - t0))
             row["units_per_cta"] = [int(g[:, 6].min()), int(g[:, 6].max())]
         if (r[:, 7] > 0).any():
