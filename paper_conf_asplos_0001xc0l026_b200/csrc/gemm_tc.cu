@@ -251,6 +251,62 @@ __device__ __forceinline__ void epi_qkv(const GemmArgs& a, int m, int col, float
   }
 }
 
+// EPI_QKV, coalesced: the same arithmetic as epi_qkv (bias, rotation with the
+// (cos, sin) rows `cs` loaded ahead by the caller, one bf16 rounding) for
+// the warp's 32 rows, then the rows' two 64-byte segments are written through
+// the warp's shared-memory buffer so each store instruction covers 4 rows x
+// 2 segments x 64 B instead of 32 rows x 16 B.
+__device__ __forceinline__ const float4* qkv_cs_row(const GemmArgs& a, const TokInfo& ti, int i0) {
+  return reinterpret_cast<const float4*>(a.cs + (size_t)ti.x * 64 + i0);
+}
+__device__ __forceinline__ void epi_qkv_coal(const GemmArgs& a, uint32_t* wu, int m, int col, int lane, float* v,
+                                             float* w, const TokInfo& ti, const float4* csv) {
+  const int head = col >> 7, i0 = col & 127;
+  if (a.bias) {
+    const __nv_bfloat16* b = reinterpret_cast<const __nv_bfloat16*>(a.bias);
+#pragma unroll
+    for (int j = 0; j < 32; ++j) { v[j] += __bfloat162float(b[col + j]); w[j] += __bfloat162float(b[col + 64 + j]); }
+  }
+  __nv_bfloat16* dst;
+  if (head < a.H + a.Hkv) {
+#pragma unroll
+    for (int j = 0; j < 16; ++j) {
+      const float4 c = csv[j];   // (cos, sin) of frequencies i0 + 2j, i0 + 2j + 1
+      const float x0 = v[2 * j], x1 = w[2 * j], y0 = v[2 * j + 1], y1 = w[2 * j + 1];
+      v[2 * j] = x0 * c.x - x1 * c.y;
+      w[2 * j] = x1 * c.x + x0 * c.y;
+      v[2 * j + 1] = y0 * c.z - y1 * c.w;
+      w[2 * j + 1] = y1 * c.z + y0 * c.w;
+    }
+    dst = head < a.H ? reinterpret_cast<__nv_bfloat16*>(a.q_out) + ((size_t)m * a.H + head) * 128
+                     : reinterpret_cast<__nv_bfloat16*>(a.pool_k) +
+                           (((size_t)(ti.y / a.kvB) * a.Hkv + (head - a.H)) * a.kvB + ti.y % a.kvB) * 128;
+  } else {
+    dst = reinterpret_cast<__nv_bfloat16*>(a.pool_v) +
+          (((size_t)(ti.y / a.kvB) * a.Hkv + (head - a.H - a.Hkv)) * a.kvB + ti.y % a.kvB) * 128;
+  }
+#pragma unroll
+  for (int i = 0; i < 16; ++i) {
+    __nv_bfloat162 h = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
+    __nv_bfloat162 g = __floats2bfloat162_rn(w[2 * i], w[2 * i + 1]);
+    wu[lane * 33 + i] = *reinterpret_cast<uint32_t*>(&h);
+    wu[lane * 33 + 16 + i] = *reinterpret_cast<uint32_t*>(&g);
+  }
+  __syncwarp();
+  const unsigned long long dp = m < a.M ? reinterpret_cast<unsigned long long>(dst + i0) : 0ull;
+  const int k = lane & 7, seg = k >> 2, qd = k & 3;
+#pragma unroll
+  for (int it = 0; it < 8; ++it) {
+    const int r = it * 4 + (lane >> 3);
+    const unsigned long long d = __shfl_sync(0xffffffffu, dp, r);
+    if (d && !(a.epi_dbg & 2))
+      *reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(d) + seg * 64 + qd * 8) =
+          make_uint4(wu[r * 33 + seg * 16 + qd * 4], wu[r * 33 + seg * 16 + qd * 4 + 1],
+                     wu[r * 33 + seg * 16 + qd * 4 + 2], wu[r * 33 + seg * 16 + qd * 4 + 3]);
+  }
+  __syncwarp();
+}
+
 // Epilogue inputs of row m of a tile at output column col0 (w columns), pulled
 // into L2 by the epilogue thread that owns the row as soon as it learns the
 // unit — the mainloop then hides their DRAM latency (the decode attention
@@ -984,7 +1040,12 @@ __global__ void __launch_bounds__(NT, 1)
       // chunk's while the current one is stored
       const bool coal_resid = !KC && g.slot < 0 && a.epi == EPI_RESID && a.epi_coal;
       float4 rr[8];
-      if (coal_resid) epi_resid_load(a, m_blk * mh * BM + eq * 32, col0, lane, rr);
+
+      // coalesced QKV epilogue: the first head's token info and (cos, sin)
+      // rows are loaded before the accumulator wait
+      const bool coal_qkv = !KC && g.slot < 0 && a.epi == EPI_QKV && a.epi_coal;
+      TokInfo qti{0, 0};
+      if (coal_qkv) qti = m_blk * mh * BM + et < a.M ? a.tok[m_blk * mh * BM + et] : TokInfo{0, 0};
       if constexpr (KC) {   // mh == 1, bn == 128, whole tiles (plan guarantees)
         const int n_ch = (k_blocks + a.kcb - 1) / a.kcb;
         float R[128];
@@ -1026,19 +1087,33 @@ __global__ void __launch_bounds__(NT, 1)
       if (et == 0 && a.L.trace) trace_at(a.L, 15, gtimer());   // (last) accumulator ready
       const uint32_t tb = tmem + ((uint32_t)(eq * 32) << 16) + as * acc_cols;
       if (g.slot < 0) {   // whole tile: epilogue straight from TMEM
-        for (int hh = 0; hh < mh; ++hh) {
-          const int m = (m_blk * mh + hh) * BM + et;
-          if (a.epi == EPI_QKV) {   // per head: column chunks (c, c + 2) are rotate-half partners
+        // one hh loop per epilogue kind: the residual carried from one 128-row
+        // half to the next (rr) must not stay live through the QKV path
+        // (register pressure: spills)
+        if (coal_qkv) {   // per head: column chunks (c, c + 2) are rotate-half partners
+          uint32_t* wu = reinterpret_cast<uint32_t*>(smem + epi_off) + eq * (32 * 33);
+          for (int hh = 0; hh < mh; ++hh) {
+            const int m = (m_blk * mh + hh) * BM + et;
             for (int c0 = 0; c0 < bn; c0 += 128)
               for (int c = 0; c < 64; c += 32) {
+                if (hh && !c0 && !c) qti = m < a.M ? a.tok[m] : TokInfo{0, 0};
+                float4 csv[16];
+                if (((col0 + c0 + c) >> 7) < a.H + a.Hkv) {
+                  const float4* cs = qkv_cs_row(a, qti, c);
+                  const bool ld = !(a.epi_dbg & 8);
+#pragma unroll
+                  for (int j = 0; j < 16; ++j) csv[j] = ld ? cs[j] : make_float4(1.f, 0.f, 1.f, 0.f);
+                }
                 tmem_ld32(tb + hh * bn + c0 + c, v);
                 tmem_ld32(tb + hh * bn + c0 + 64 + c, w);
-                if (m < a.M) epi_qkv(a, m, col0 + c0 + c, v, w);
+                epi_qkv_coal(a, wu, m, col0 + c0 + c, lane, v, w, qti, csv);
               }
-            continue;
           }
-          if (coal_resid) {
-            float* wb = reinterpret_cast<float*>(smem + epi_off) + eq * (32 * 33);
+        } else if (coal_resid) {
+          epi_resid_load(a, m_blk * mh * BM + eq * 32, col0, lane, rr);
+          float* wb = reinterpret_cast<float*>(smem + epi_off) + eq * (32 * 33);
+          for (int hh = 0; hh < mh; ++hh) {
+            const int m = (m_blk * mh + hh) * BM + et;
             for (int c = 0; c < out_chunks; ++c) {
               float4 rn[8];
               const bool more = c + 1 < out_chunks || hh + 1 < mh;
@@ -1051,21 +1126,34 @@ __global__ void __launch_bounds__(NT, 1)
 #pragma unroll
                 for (int i = 0; i < 8; ++i) rr[i] = rn[i];
             }
-            continue;
           }
-          if (a.epi == EPI_SILU && a.epi_coal) {
-            float* wb = reinterpret_cast<float*>(smem + epi_off) + eq * (32 * 33);
+        } else if (a.epi == EPI_SILU && a.epi_coal) {
+          float* wb = reinterpret_cast<float*>(smem + epi_off) + eq * (32 * 33);
+          for (int hh = 0; hh < mh; ++hh) {
+            const int m = (m_blk * mh + hh) * BM + et;
             for (int c = 0; c < out_chunks; ++c) {
               tmem_ld32(tb + hh * bn + c * 32, v);
               tmem_ld32(tb + hh * bn + bn / 2 + c * 32, w);
               epi_chunk_coalesced(a, wb, m - lane, col0 + c * 32, lane, v, w, nullptr);
             }
-            continue;
           }
-          for (int c = 0; c < out_chunks; ++c) {
-            tmem_ld32(tb + hh * bn + c * 32, v);
-            if (a.epi == EPI_SILU) tmem_ld32(tb + hh * bn + bn / 2 + c * 32, w);
-            if (m < a.M) epi_store(a, m, col0 + c * 32, v, w);
+        } else {
+          for (int hh = 0; hh < mh; ++hh) {
+            const int m = (m_blk * mh + hh) * BM + et;
+            if (a.epi == EPI_QKV) {   // per head: column chunks (c, c + 2) are rotate-half partners
+              for (int c0 = 0; c0 < bn; c0 += 128)
+                for (int c = 0; c < 64; c += 32) {
+                  tmem_ld32(tb + hh * bn + c0 + c, v);
+                  tmem_ld32(tb + hh * bn + c0 + 64 + c, w);
+                  if (m < a.M) epi_qkv(a, m, col0 + c0 + c, v, w);
+                }
+              continue;
+            }
+            for (int c = 0; c < out_chunks; ++c) {
+              tmem_ld32(tb + hh * bn + c * 32, v);
+              if (a.epi == EPI_SILU) tmem_ld32(tb + hh * bn + bn / 2 + c * 32, w);
+              if (m < a.M) epi_store(a, m, col0 + c * 32, v, w);
+            }
           }
         }
         tc_fence_before();
