@@ -653,6 +653,20 @@ static int pf5_maps(bullet_handle* h, int layer, AttnArgs* a, CUtensorMap* mk, C
   return BULLET_OK;
 }
 
+// K / V maps of the decode attention's stream (the same pool view and boxes as
+// pf5_maps); BULLET_DEC_TMA=0 keeps the cp.async stream (A/B).
+static int dec_maps(bullet_handle* h, int layer, AttnArgs* a, CUtensorMap* mk, CUtensorMap* mv) {
+  static const int on = getenv("BULLET_DEC_TMA") ? atoi(getenv("BULLET_DEC_TMA")) : 1;
+  memset(mk, 0, sizeof *mk);
+  memset(mv, 0, sizeof *mv);
+  a->kv_tma = on && h->block_size == 16;
+  if (!a->kv_tma) return BULLET_OK;
+  const long long rows = (long long)h->n_blocks * h->cfg.n_kv_heads * 16;
+  if (rows >= (1ll << 31)) { a->kv_tma = 0; return BULLET_OK; }
+  int rc = make_map(mk, h->pk[layer], (int)rows, 128, 16);
+  return rc ? rc : make_map(mv, h->pv[layer], (int)rows, 128, 16);
+}
+
 int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* o, int kind) {
   bullet_handle* h = c.h;
   if (b->n_tokens == 0) return BULLET_OK;
@@ -685,8 +699,9 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     AttnArgs d = a;
     d.tok_base = t0;
     d.order = P.order_ok ? P.order : nullptr;
+    if ((rc = dec_maps(h, layer, &d, &mk, &mv))) return rc;
     if ((rc = next_launch(c, &d.L))) return rc;
-    LAUNCH(c, launch_attn_decode_tc(d, persist_grid(c, 1), c.m_sms <= 100 ? 4 : 1, c.st));
+    LAUNCH(c, launch_attn_decode_tc(mk, mv, d, persist_grid(c, 1), c.m_sms <= 100 ? 4 : 1, c.st));
     return BULLET_OK;
   }
   if (kind == 0) kind = (bf16 && a.hd == 128) ? (max_qlen(b) > 1 ? 4 : 3) : 1;
@@ -704,13 +719,15 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
                        "from max_position)", max_kv(b), a.kv_chunks, P.kv_cap);
       a.kv_part = P.kv_part; a.kv_tick = P.kv_tick;
     }
-    int rc = next_launch(c, &a.L);
+    CUtensorMap mk, mv;
+    int rc = dec_maps(h, layer, &a, &mk, &mv);
     if (rc) return rc;
+    if ((rc = next_launch(c, &a.L))) return rc;
     // four consumer groups of 3 warps per SM on partitions (68 SMs: 78.6 vs
     // 72.3 GB/s/SM with two groups at 1k contexts), one on the full GPU (tail
     // balance) — scripts/attn_dec_bench.py, DESIGN.md §5
     if (!c.op && h->ph[c.phase].order_ok) a.order = h->ph[c.phase].order;
-    LAUNCH(c, launch_attn_decode_tc(a, persist_grid(c, 1), c.m_sms <= 100 ? 4 : 1, c.st));
+    LAUNCH(c, launch_attn_decode_tc(mk, mv, a, persist_grid(c, 1), c.m_sms <= 100 ? 4 : 1, c.st));
     return BULLET_OK;
   }
   if (kind == 2 || kind == 4) {

@@ -90,6 +90,21 @@ __device__ __forceinline__ uint32_t tile_off(int row, int c) {
   return row * 256 + ((c ^ (row & 7)) << 4);
 }
 
+// byte offset of 16-byte chunk c (0..15) of key row `row` in the layout the
+// TMA boxes produce: [2 halves of 64 dims][16 rows][128 B], 128-byte swizzle
+__device__ __forceinline__ uint32_t tile_off_sw128(int row, int c) {
+  return (c >> 3) * 2048 + row * 128 + (((c & 7) ^ (row & 7)) << 4);
+}
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void tma_load_2d_hint(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
+                                                 uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1, {%3, %4}], [%2], %5;" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "l"(pol)
+      : "memory");
+}
+
 // KV is streamed once per launch: evict-first keeps it from displacing the
 // other phase's L2-resident activation tiles.
 __device__ __forceinline__ void cp_async16_ef(void* dst, const void* src, uint64_t pol) {
@@ -107,7 +122,8 @@ struct Slot {  // one published unit: blocks [b0, b0 + nb) of (token t, kv head 
 // gw + NG, ... (units alternate between groups), so a unit's blocks are
 // split over fewer warps and the per-unit merge is paid over more blocks.
 template <int NG>
-__global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
+__global__ void __launch_bounds__(THREADS, 1)
+    k_attn_decode_tc(const __grid_constant__ CUtensorMap mk, const __grid_constant__ CUtensorMap mv, AttnArgs a) {
   constexpr int GW = NCW / NG;
   constexpr int NS = 2 * NG;   // unit slots: each group holds <= 2 units (current + next)
   if (!gate_enter(a.L)) return;
@@ -120,13 +136,15 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
   Slot* uq = reinterpret_cast<Slot*>(btbuf + NS_MAX * MAXNB);
   uint64_t* uqf = reinterpret_cast<uint64_t*>(uq + NS_MAX);
   uint64_t* uqe = uqf + NS_MAX;
-  int* rec_stage = reinterpret_cast<int*>(uqe + NS_MAX);                       // [NCW]
+  int* rec_stage = reinterpret_cast<int*>(uqe + NS_MAX);                       // [NCW] (+ NG merge flags)
+  uint64_t* sfull = reinterpret_cast<uint64_t*>(rec_stage + NCW + 4);          // [NCW][DEPTH] (a.kv_tma)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int grp = a.H / a.Hkv;
   const int units = (a.n_tok - a.tok_base) * a.Hkv;   // decode rows are tokens [tok_base, n_tok)
   if (threadIdx.x == 0) {
     for (int i = 0; i < NS; ++i) { mbar_init(uqf + i, 1); mbar_init(uqe + i, GW); }
+    for (int i = 0; i < NCW * DEPTH; ++i) mbar_init(sfull + i, 1);
     mbar_fence_init();
   }
   __syncthreads();
@@ -202,13 +220,18 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
   auto my_count = [&](int nb) { return nb > wl ? (nb - wl + GW - 1) / GW : 0; };
   // per-lane swizzled offsets (loop invariant): cp.async destinations and
   // ldmatrix sources for the QK (K, by k-step) and PV (V^T, by m-tile) MMAs
+  // (a.kv_tma: the TMA boxes land K / V as [2 halves of 64 dims][16 rows][128 B]
+  // with the 128-byte swizzle — also conflict-free for ldmatrix)
+  const bool tma = a.kv_tma != 0;
+  auto off = [&](int row, int c) { return tma ? tile_off_sw128(row, c) : tile_off(row, c); };
   uint32_t cp_off[8], k_off[8], v_off[8];
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
     cp_off[i] = tile_off(2 * i + (lane >> 4), lane & 15);
-    k_off[i] = tile_off(lane & 15, i * 2 + (lane >> 4));
-    v_off[i] = BLK_BYTES + tile_off(((lane >> 3) >> 1) * 8 + (lane & 7), i * 2 + ((lane >> 3) & 1));
+    k_off[i] = off(lane & 15, i * 2 + (lane >> 4));
+    v_off[i] = BLK_BYTES + off(((lane >> 3) >> 1) * 8 + (lane & 7), i * 2 + ((lane >> 3) & 1));
   }
+  uint64_t* my_full = sfull + warp * DEPTH;
 
   const int pf = a.dec_pf;   // L2 prefetch distance in this warp's blocks (0 = off)
   // issue cursor over this warp's block sequence (units in claim order,
@@ -237,12 +260,26 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
         prefetch_l2(pv + ((size_t)b2 * a.Hkv + cur_g) * KB * HD, BLK_BYTES);
       }
       uint8_t* dk = my + (n_issued % DEPTH) * STAGE_BYTES;
+      if (tma) {   // one elected lane: K and V as 2 boxes each (16 rows x 64 dims), bytes counted on the stage barrier
+        const int row = (blk * a.Hkv + cur_g) * KB;
+        if (elect_one()) {
+          uint64_t* bar = my_full + (n_issued % DEPTH);
+          fence_proxy_async();   // this warp's generic reads / merge-record writes of the stage come first
+          mbar_arrive_expect_tx(bar, STAGE_BYTES);
+          tma_load_2d_hint(dk, &mk, bar, 0, row, pol_kv);
+          tma_load_2d_hint(dk + BLK_BYTES / 2, &mk, bar, 64, row, pol_kv);
+          tma_load_2d_hint(dk + BLK_BYTES, &mv, bar, 0, row, pol_kv);
+          tma_load_2d_hint(dk + BLK_BYTES + BLK_BYTES / 2, &mv, bar, 64, row, pol_kv);
+        }
+        __syncwarp();
+      } else {
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
         cp_async16_ef(dk + cp_off[i], ks + 512 * i, pol_kv);
         cp_async16_ef(dk + BLK_BYTES + cp_off[i], vs + 512 * i, pol_kv);
       }
       cp_async_commit();
+      }
       ++n_issued;
       ++ij;
     }
@@ -273,9 +310,13 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
     const int mine = my_count(S.nb);
     for (int j = 0; j < mine; ++j) {
       fill(it + NG, DEPTH);
+      if (tma) {
+        mbar_wait(my_full + (n_cons % DEPTH), (n_cons / DEPTH) & 1);
+      } else {
       const int pend = n_issued - n_cons;   // groups in flight; the oldest is block j
       if (pend >= 5) cp_async_wait<4>(); else if (pend == 4) cp_async_wait<3>();
       else if (pend == 3) cp_async_wait<2>(); else if (pend == 2) cp_async_wait<1>(); else cp_async_wait<0>();
+      }
       __syncwarp();
       const int b = wl + j * GW;
       const uint32_t kt = my_s + (n_cons % DEPTH) * STAGE_BYTES;
@@ -428,12 +469,13 @@ __global__ void __launch_bounds__(THREADS, 1) k_attn_decode_tc(AttnArgs a) {
 
 size_t attn_decode_smem_bytes() {
   return (size_t)NCW * DEPTH * STAGE_BYTES + NS_MAX * QSLOT_BYTES + NS_MAX * MAXNB * 4 + NS_MAX * sizeof(Slot) +
-         2 * NS_MAX * 8 + (NCW + 4) * 4;
+         2 * NS_MAX * 8 + (NCW + 4) * 4 + NCW * DEPTH * 8;
 }
 int attn_decode_max_blocks() { return MAXNB; }
 
 // `ng` consumer groups per CTA (1, 2 or 4; BULLET_DEC_GROUPS overrides).
-cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStream_t st) {
+cudaError_t launch_attn_decode_tc(const CUtensorMap& mk, const CUtensorMap& mv, const AttnArgs& a, int grid, int ng,
+                                  cudaStream_t st) {
   const size_t smem = attn_decode_smem_bytes();
   static const int forced = getenv("BULLET_DEC_GROUPS") ? atoi(getenv("BULLET_DEC_GROUPS")) : 0;
   if (forced >= 1 && forced <= 4) ng = forced;
@@ -449,10 +491,10 @@ cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStrea
     if (e != cudaSuccess) return e;
     set = true;
   }
-  if (ng == 1) return launch_ex(k_attn_decode_tc<1>, grid, THREADS, smem, st, a.L.pdl, a);
-  if (ng == 4 && NCW % 4 == 0) return launch_ex(k_attn_decode_tc<4>, grid, THREADS, smem, st, a.L.pdl, a);
-  if (ng == 3 && NCW % 3 == 0) return launch_ex(k_attn_decode_tc<3>, grid, THREADS, smem, st, a.L.pdl, a);
-  return launch_ex(k_attn_decode_tc<2>, grid, THREADS, smem, st, a.L.pdl, a);
+  if (ng == 1) return launch_ex(k_attn_decode_tc<1>, grid, THREADS, smem, st, a.L.pdl, mk, mv, a);
+  if (ng == 4 && NCW % 4 == 0) return launch_ex(k_attn_decode_tc<4>, grid, THREADS, smem, st, a.L.pdl, mk, mv, a);
+  if (ng == 3 && NCW % 3 == 0) return launch_ex(k_attn_decode_tc<3>, grid, THREADS, smem, st, a.L.pdl, mk, mv, a);
+  return launch_ex(k_attn_decode_tc<2>, grid, THREADS, smem, st, a.L.pdl, mk, mv, a);
 }
 
 cudaError_t preload_attn_decode() {

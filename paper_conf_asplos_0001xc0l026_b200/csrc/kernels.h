@@ -134,7 +134,7 @@ struct AttnArgs {
   float* kv_part;         // [units][kv_chunks][8][128 + 2] (kv_chunks > 1)
   int* kv_tick;           // [units], zero between launches (self-resetting)
   int dec_pf;             // decode kernel: L2 prefetch distance (blocks of a warp's stream; 0 = off)
-  int kv_tma;             // prefill tcgen05 kernel: Q and full K/V tiles by TMA (else cp.async gathers)
+  int kv_tma;             // tcgen05 prefill: Q and full K/V tiles by TMA; decode: K/V blocks by TMA (else cp.async)
   Launch L;
 };
 
@@ -191,7 +191,8 @@ cudaError_t launch_attn_prefill_tc(const AttnArgs& a, int grid, cudaStream_t st)
 cudaError_t launch_attn_prefill5(const CUtensorMap& mk, const CUtensorMap& mv, const CUtensorMap& mq,
                                  const AttnArgs& a, int grid, cudaStream_t st);
 int attn_prefill5_ctas_per_sm(int H, int Hkv);   // grid = n_sms * this (2 query tiles per CTA for even GQA groups)
-cudaError_t launch_attn_decode_tc(const AttnArgs& a, int grid, int ng, cudaStream_t st);
+cudaError_t launch_attn_decode_tc(const CUtensorMap& mk, const CUtensorMap& mv, const AttnArgs& a, int grid, int ng,
+                                  cudaStream_t st);   // mk / mv as for launch_attn_prefill5 (a.kv_tma)
 size_t attn_decode_smem_bytes();
 int attn_decode_max_blocks();
 cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);   // grid sized to n_tok
