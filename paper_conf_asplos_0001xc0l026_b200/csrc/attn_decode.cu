@@ -2,14 +2,18 @@
 // (the paper's PagedAttention decode: "irregular
 // memory access" — here every (block, kv head) is one contiguous 4 KB chunk).
 //
-// Memory side: each of the 8 consumer warps streams its own blocks with
-// 16-byte cp.async (coalesced 4 KB chunks, XOR-swizzled into shared memory),
-// DEPTH blocks in flight per warp.  A claimer warp takes units from the
+// Memory side: each of the 12 consumer warps streams its own blocks, DEPTH
+// blocks in flight per warp: by TMA (default, a.kv_tma: the pool viewed as a
+// [blocks * Hkv * 16][128] tensor, K and V of a block as two 16-row x 64-dim
+// boxes each with the 128-byte swizzle, issued by one elected lane, completion
+// in bytes on the stage's mbarrier) or with 16-byte cp.async (coalesced 4 KB
+// chunks, XOR-swizzled; BULLET_DEC_TMA=0).  Round 2 measured the TMA stream
+// 1.5-2.5 % faster on 64-70 SMs and bit-identical (round 1's TMA attempt,
+// capped near 27 GB/s per SM, issued from a single thread).  A claimer warp takes units from the
 // gated work counter and publishes each unit's block-table row and Q rows in
 // shared memory up to 4 units ahead, so no consumer waits on a dependent
 // global load; warps prefetch the next unit's first blocks before merging the
-// current one.  (A TMA version was capped near 27 GB/s per SM by the
-// per-operation cost of 2 KB paged boxes — DESIGN.md §5.)
+// current one.
 // Math side: swap-AB so the 16 keys of a block fill the MMA M dimension and
 // the GQA group (<= 8 query heads) fills N = 8:
 //   S^T[16 keys x 8 heads] = K[16 x 128] . Q^T[128 x 8]   (mma.m16n8k16 bf16)
