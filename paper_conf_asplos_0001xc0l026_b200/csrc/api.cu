@@ -655,16 +655,28 @@ static int pf5_maps(bullet_handle* h, int layer, AttnArgs* a, CUtensorMap* mk, C
 
 // K / V maps of the decode attention's stream (the same pool view and boxes as
 // pf5_maps); BULLET_DEC_TMA=0 keeps the cp.async stream (A/B).
-static int dec_maps(bullet_handle* h, int layer, AttnArgs* a, CUtensorMap* mk, CUtensorMap* mv) {
+static int dec_maps(bullet_handle* h, int layer, AttnArgs* a, CUtensorMap* mk, CUtensorMap* mv, bool force = false) {
   static const int on = getenv("BULLET_DEC_TMA") ? atoi(getenv("BULLET_DEC_TMA")) : 1;
   memset(mk, 0, sizeof *mk);
   memset(mv, 0, sizeof *mv);
-  a->kv_tma = on && h->block_size == 16;
+  a->kv_tma = (on || force) && h->block_size == 16;
   if (!a->kv_tma) return BULLET_OK;
   const long long rows = (long long)h->n_blocks * h->cfg.n_kv_heads * 16;
   if (rows >= (1ll << 31)) { a->kv_tma = 0; return BULLET_OK; }
   int rc = make_map(mk, h->pk[layer], (int)rows, 128, 16);
   return rc ? rc : make_map(mv, h->pv[layer], (int)rows, 128, 16);
+}
+
+// BULLET_DEC_KERNEL=5 selects the tcgen05 decode attention (attn_decode5.cu;
+// bf16, head_dim 128, block 16, GQA groups <= 8) instead of the default
+// mma.sync kernel (attn_decode.cu): parity-green but measured slower on
+// partitions (its 64 KB stages are held through the whole
+// S -> softmax -> PV chain, so fewer bytes stay in flight per SM).
+static bool use_decode5(bullet_handle* h) {
+  static const int k = getenv("BULLET_DEC_KERNEL") ? atoi(getenv("BULLET_DEC_KERNEL")) : 3;
+  const int grp = h->cfg.n_heads / std::max(1, h->cfg.n_kv_heads);
+  return k == 5 && h->cfg.dtype == BULLET_DTYPE_BF16 && h->cfg.head_dim == 128 && h->block_size == 16 && grp <= 8 &&
+         (long long)h->n_blocks * h->cfg.n_kv_heads * 16 < (1ll << 31);
 }
 
 int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* o, int kind) {
@@ -699,12 +711,23 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
     AttnArgs d = a;
     d.tok_base = t0;
     d.order = P.order_ok ? P.order : nullptr;
-    if ((rc = dec_maps(h, layer, &d, &mk, &mv))) return rc;
+    const bool d5 = use_decode5(h);
+    if ((rc = dec_maps(h, layer, &d, &mk, &mv, d5))) return rc;
     if ((rc = next_launch(c, &d.L))) return rc;
-    LAUNCH(c, launch_attn_decode_tc(mk, mv, d, persist_grid(c, 1), c.m_sms <= 100 ? 4 : 1, c.st));
+    if (d5) LAUNCH(c, launch_attn_decode5(mk, mv, d, persist_grid(c, 1), c.st));
+    else LAUNCH(c, launch_attn_decode_tc(mk, mv, d, persist_grid(c, 1), c.m_sms <= 100 ? 4 : 1, c.st));
     return BULLET_OK;
   }
   if (kind == 0) kind = (bf16 && a.hd == 128) ? (max_qlen(b) > 1 ? 4 : 3) : 1;
+  if (kind == 3 && use_decode5(h)) {   // tcgen05 decode attention (any context length: no KV chunks)
+    CUtensorMap mk, mv;
+    int rc = dec_maps(h, layer, &a, &mk, &mv, true);
+    if (rc) return rc;
+    if ((rc = next_launch(c, &a.L))) return rc;
+    if (!c.op && h->ph[c.phase].order_ok) a.order = h->ph[c.phase].order;
+    LAUNCH(c, launch_attn_decode5(mk, mv, a, persist_grid(c, 1), c.st));
+    return BULLET_OK;
+  }
   if (kind == 3) {
     if (!bf16 || a.hd != 128)
       return set_err(BULLET_EUNSUPPORTED, "tensor-core decode attention: bf16, hd 128 only");
@@ -968,7 +991,7 @@ int bullet_create(const bullet_model_cfg* cfg, const bullet_kv_pool* pool, const
   if (prop.major != 10) return set_err(BULLET_EUNSUPPORTED, "needs an sm_100 (Blackwell) GPU, got sm_%d%d", prop.major, prop.minor);
   int rc = get_encode();
   if (rc) return rc;
-  for (auto pre : {preload_attn_decode, preload_attn_prefill5, preload_attn_tc, preload_attn_simt,
+  for (auto pre : {preload_attn_decode, preload_attn_decode5, preload_attn_prefill5, preload_attn_tc, preload_attn_simt,
                    preload_elementwise, preload_gemm_tc, preload_stream}) {
     cudaError_t e = pre();
     if (e != cudaSuccess) return set_err(BULLET_ECUDA, "kernel preload: %s", cudaGetErrorString(e));

@@ -194,6 +194,11 @@ int attn_prefill5_ctas_per_sm(int H, int Hkv);   // grid = n_sms * this (2 query
 cudaError_t launch_attn_decode_tc(const CUtensorMap& mk, const CUtensorMap& mv, const AttnArgs& a, int grid, int ng,
                                   cudaStream_t st);   // mk / mv as for launch_attn_prefill5 (a.kv_tma)
 size_t attn_decode_smem_bytes();
+// tcgen05 decode attention (attn_decode5.cu): grid = n_sms, GQA group <= 8, head_dim 128, block 16;
+// mk / mv as for launch_attn_prefill5
+cudaError_t launch_attn_decode5(const CUtensorMap& mk, const CUtensorMap& mv, const AttnArgs& a, int grid,
+                                cudaStream_t st);
+cudaError_t preload_attn_decode5();
 int attn_decode_max_blocks();
 cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);   // grid sized to n_tok
 cudaError_t launch_stream(const StreamArgs& a, int grid, cudaStream_t st);

@@ -447,3 +447,18 @@ def test_die_probe_and_sigma_orders(B):
                 assert all(pd[i] != pd[i + 1] for i in range(0, n - 1, 2))
     finally:
         os.environ.pop("BULLET_SIGMA", None)
+
+
+def test_decode5_tcgen05_kernel_vs_oracle():
+    """The opt-in tcgen05 decode attention (BULLET_DEC_KERNEL=5, fresh
+    process): the decode-attention oracle checks (GQA groups 4 / 5 / 8,
+    contexts 0..2047, and 100..32767 with no KV chunking) and a co-run layer
+    step with 16k / 30k decode contexts."""
+    import os
+    import subprocess
+    import sys
+    here = os.path.dirname(os.path.abspath(__file__))
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", os.path.join(here, "test_gpu_kernels.py"),
+                        "-k", "(attention_vs_oracle and -3]) or long_contexts"],
+                       env=dict(os.environ, BULLET_DEC_KERNEL="5"), capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0 and " passed" in r.stdout, r.stdout[-3000:] + r.stderr[-2000:]
