@@ -758,7 +758,7 @@ def main():
     bound, work = kernel_work(S, dom[0], dom[1])
     avg_ms = float(np.mean(by[dom]))
     P, src = peaks()
-    tf = os.path.join(ROOT, "profiles", "r02_traffic.json")   # ncu --set full capture of the same kernel
+    tf = os.path.join(ROOT, "profiles", "r02b_traffic.json")   # ncu --set full capture of the same kernel
     dom_name = f"{dom[0]} ({'prefill' if dom[1] == 0 else 'decode'})"
     traffic = (json.load(open(tf))["bytes"].get(args.config, {}).get(dom_name)
                if os.path.exists(tf) else None)

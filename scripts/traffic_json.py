@@ -3,7 +3,7 @@ DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum), keyed by
 bench config and the bench's kernel name ("<kind> (prefill|decode)"), which
 bench.py reads for roofline.traffic.
 
-  python scripts/traffic_json.py gpurun_out/ncu2/*.raw.csv > profiles/r02_traffic.json
+  python scripts/traffic_json.py profiles/r02b/ncu/*.raw.csv > profiles/r02b_traffic.json
 """
 import csv
 import io
@@ -20,7 +20,7 @@ CFG = {"c2": "sharegpt-8b", "c3": "arxiv-8b"}
 def main():
     out = {}
     for p in sys.argv[1:]:
-        m = re.match(r"r02_(c\d)_(\w+?)_(dec|pre)_p\d+\.raw\.csv", os.path.basename(p))
+        m = re.match(r"r02b?_(c\d)_(\w+?)_(dec|pre)_p\d+\.raw\.csv", os.path.basename(p))
         if not m:
             continue
         r = list(csv.reader(io.StringIO(open(p).read())))
