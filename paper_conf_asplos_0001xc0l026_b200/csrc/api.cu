@@ -451,9 +451,16 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
     }
   }
   if (!bn) return set_err(BULLET_EUNSUPPORTED, "GEMM N=%d not tileable", N);
-  char kenv[32];
-  snprintf(kenv, sizeof kenv, "BULLET_GEMM_PLAN_K%d", c.kind);   // per kernel kind (experiments)
-  const char* ov = getenv(kenv);
+  char kenv[32];   // per kernel kind (experiments): BULLET_GEMM_PLAN_K<kind>, prefill phase only: ..._K<kind>P
+  const char* ov = nullptr;
+  if (c.phase == 0) {
+    snprintf(kenv, sizeof kenv, "BULLET_GEMM_PLAN_K%dP", c.kind);
+    ov = getenv(kenv);
+  }
+  if (!ov) {
+    snprintf(kenv, sizeof kenv, "BULLET_GEMM_PLAN_K%d", c.kind);
+    ov = getenv(kenv);
+  }
   if (!ov) ov = getenv("BULLET_GEMM_PLAN");
   if (ov) {   // experiments: "mh,bn,sk" (sk 1: stream the ragged remainder over K)
     int omh = 0, obn = 0, osk = 0;
@@ -514,8 +521,11 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
      // while every weight tile streams past them once per band: a band of
      // <= BULLET_GEMM_BAND_MB (default 64; co-run step vs 32 / 128 MB: config 2
      // 2.919 vs 2.968 / 2.922 ms, config 3 7.144 vs 7.201 / 7.272 ms) MB of activations
-    static const double band_bytes =
+    static const double band_all =
         (getenv("BULLET_GEMM_BAND_MB") ? atof(getenv("BULLET_GEMM_BAND_MB")) : 64.0) * 1e6;
+    char benv[40];   // per kernel kind (experiments): BULLET_GEMM_BAND_MB_K<kind>
+    snprintf(benv, sizeof benv, "BULLET_GEMM_BAND_MB_K%d", c.kind);   // (one M tile in decode: no effect)
+    const double band_bytes = getenv(benv) ? atof(getenv(benv)) * 1e6 : band_all;
     const int m_tiles = (M + 128 * mh - 1) / (128 * mh);
     const double a_tile = 128.0 * mh * K * 2;
     const int n_bands = std::max(1, (int)std::ceil(m_tiles * a_tile / band_bytes));
