@@ -250,6 +250,15 @@ void prof_end(Ctx& c) {
     prof_end(c);      \
   } while (0)
 
+// Kernels with several CTAs per SM (the row grids, the fp32 SIMT kernels) are
+// launched without PDL: launched early, their whole grid can fit on the SMs
+// outside a small partition whose SMs the predecessor still holds, park
+// there, and leave the gate's liveness fallback to run a unit off-range (seen
+// with a 2-SM decode partition, test_smid_gating_invariants[146]).  The
+// one-CTA-per-SM persistent kernels always leave CTAs queued for the
+// partition's SMs (grid = SMs x occupancy).
+static inline void no_pdl(Launch& L) { L.pdl = 0; }
+
 int next_launch(Ctx& c, Launch* L) {
   prof_begin(c);
   memset(L, 0, sizeof *L);
@@ -394,6 +403,7 @@ int do_gemm(Ctx& c, int epi, const void* A, int M, int K, const void* B, int N, 
   if (h->cfg.dtype == BULLET_DTYPE_FP32) {
     if (K % 16) return set_err(BULLET_EUNSUPPORTED, "fp32 GEMM needs K %% 16 == 0");
     a.bn = 64; a.mh = 1; a.n_full = 0; a.band = 1;
+    no_pdl(a.L);
     LAUNCH(c, launch_gemm_simt<float>((const float*)A, (const float*)B, a, h->n_sms * 4, c.st));
     return BULLET_OK;
   }
@@ -579,6 +589,7 @@ int do_rmsnorm(Ctx& c, const float* x, int n, const void* g, void* out) {
   a.x = x; a.g = g; a.out = out; a.n = n; a.d = c.h->cfg.d_model; a.eps = c.h->cfg.rms_eps;
   int rc = next_launch(c, &a.L);
   if (rc) return rc;
+  no_pdl(a.L);
   // one CTA per row (BULLET_NORM=warp: warp per row — measured slower, 9.6 -> 24 us
   // for 128 decode rows on 68 SMs: the per-warp row loads are latency-bound)
   static const bool warp = getenv("BULLET_NORM") && !strcmp(getenv("BULLET_NORM"), "warp");
@@ -604,6 +615,7 @@ int do_rope(Ctx& c, const bullet_batch* b, int layer, const float* qkv, void* q)
   a.max_pos = h->cfg.max_position;
   int rc = next_launch(c, &a.L);
   if (rc) return rc;
+  no_pdl(a.L);
   if (h->cfg.dtype == BULLET_DTYPE_FP32) LAUNCH(c, launch_rope_kv<float>(a, row_grid(c, b->n_tokens), c.st));
   else LAUNCH(c, launch_rope_kv<__nv_bfloat16>(a, row_grid(c, b->n_tokens), c.st));
   return BULLET_OK;
@@ -783,6 +795,7 @@ int do_attention(Ctx& c, const bullet_batch* b, int layer, const void* q, void* 
   }
   int rc = next_launch(c, &a.L);
   if (rc) return rc;
+  no_pdl(a.L);
   if (bf16) LAUNCH(c, launch_attn_simt<__nv_bfloat16>(a, h->n_sms * 4, c.st));
   else LAUNCH(c, launch_attn_simt<float>(a, h->n_sms * 4, c.st));
   return BULLET_OK;
