@@ -540,3 +540,36 @@ def test_prefill_attention_tma_kv_bit_identical():
             assert r.returncode == 0, r.stderr[-3000:]
             digests.append([l for l in r.stdout.splitlines() if l.startswith("DIGEST")][0])
         assert digests[0] == digests[1], nq
+
+
+@pytest.mark.parametrize("knob", ["BULLET_GEMM_EPI_COAL=0", "BULLET_DEC_TMA=0"])
+def test_layout_knobs_bit_identical(knob):
+    """Round-2 data-movement changes that must not touch the arithmetic: the
+    GEMM epilogues' shared-memory transposed loads / stores (off:
+    BULLET_GEMM_EPI_COAL=0, per-row vectors) and the decode attention's TMA
+    stream (off: BULLET_DEC_TMA=0, cp.async) — a two-layer co-run step with
+    ragged prompts and decodes gives the same bits either way (fresh
+    processes)."""
+    import os
+    import subprocess
+    import sys
+    here = os.path.dirname(os.path.abspath(__file__))
+    code = ("import sys; sys.path[:0] = [%r, %r]\n"
+            "import torch, hashlib\n"
+            "from harness import Setup, phase_streams\n"
+            "from workload import synth\n"
+            "m = synth.ModelShape('gqa', 1024, 8, 2, 128, 2816, 2)\n"
+            "S = Setup(m, [300, 77, 1, 129, 256], [64, 1, 500, 31, 2047, 16], n_layers=2)\n"
+            "pre, dec = S.batches()\n"
+            "S.bl.step(pre, dec, 64, S.B.CORUN, *phase_streams())\n"
+            "torch.cuda.synchronize()\n"
+            "h = hashlib.sha256(pre.hidden.cpu().numpy().tobytes() + dec.hidden.cpu().numpy().tobytes())\n"
+            "print('DIGEST', h.hexdigest())\n") % (here, os.path.dirname(here))
+    k, v = knob.split("=")
+    digests = []
+    for env in ({}, {k: v}):
+        r = subprocess.run([sys.executable, "-c", code], env=dict(os.environ, **env),
+                           capture_output=True, text=True, timeout=600)
+        assert r.returncode == 0, r.stderr[-3000:]
+        digests.append([l for l in r.stdout.splitlines() if l.startswith("DIGEST")][0])
+    assert digests[0] == digests[1], knob
