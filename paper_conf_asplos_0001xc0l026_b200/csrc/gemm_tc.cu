@@ -9,7 +9,10 @@
 //   warp 0 lane 0  tile scheduler (atomic claim, gated) + TMA producer
 //   warp 1 lane 0  MMA issuer: tcgen05.mma.cta_group::1.kind::f16, M=128
 //   warp 2         TMEM allocator (512 columns = 2 accumulator stages)
-//   warps 4..7     epilogue: tcgen05.ld 32x32b -> registers -> global
+//   warps 4..7     epilogue: tcgen05.ld 32x32b -> registers -> global (whole
+//                  tiles of EPI_RESID / EPI_SILU / EPI_QKV: rows transposed
+//                  through a 4 x [32][33]-word smem buffer so each warp access
+//                  covers whole row segments; residual loads issued ahead)
 // Pipelines: smem stage ring (full/empty mbarriers, TMA complete_tx and
 // tcgen05.commit), accumulator ring (2 stages), work-unit queue (4 slots).
 // Operand tiles: A mh x (128 x 64), B bn x 64 (bf16, 128-byte swizzle, TMA).
@@ -20,7 +23,8 @@
 // last wave, or all tiles of a decode-sized GEMM) are streamed over K in
 // equal ranges (stream-K, see Seg below) so every SM of the partition
 // streams the same number of k-blocks.  Partial segments write fp32
-// partials; the tile's last segment (atomic ticket) sums them in k order
+// partials; after its own queue every CTA runs the fixup phase (fix_phase):
+// claims items of streamed tiles, sums their partials in k order
 // (deterministic) and runs the epilogue.
 #include "kernels.h"
 
