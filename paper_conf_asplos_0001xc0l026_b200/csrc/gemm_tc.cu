@@ -115,6 +115,34 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
   for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
 }
 
+// Two 32-column TMEM loads in flight under one wait (the KC merge: chunk and
+// running sum together)
+__device__ __forceinline__ void tmem_ld32x2(uint32_t ta, uint32_t tb, float* va, float* vb) {
+  uint32_t r[64];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%64];\n\t"
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%32,%33,%34,%35,%36,%37,%38,%39,%40,%41,%42,%43,%44,%45,%46,%47,%48,%49,%50,%51,%52,%53,%54,%55,%56,%57,%58,%59,%60,%61,%62,%63}, [%65];\n\t"
+      "tcgen05.wait::ld.sync.aligned;"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31]), "=r"(r[32]), "=r"(r[33]), "=r"(r[34]), "=r"(r[35]), "=r"(r[36]), "=r"(r[37]), "=r"(r[38]), "=r"(r[39]), "=r"(r[40]), "=r"(r[41]), "=r"(r[42]), "=r"(r[43]), "=r"(r[44]), "=r"(r[45]), "=r"(r[46]), "=r"(r[47]), "=r"(r[48]), "=r"(r[49]), "=r"(r[50]), "=r"(r[51]), "=r"(r[52]), "=r"(r[53]), "=r"(r[54]), "=r"(r[55]), "=r"(r[56]), "=r"(r[57]), "=r"(r[58]), "=r"(r[59]), "=r"(r[60]), "=r"(r[61]), "=r"(r[62]), "=r"(r[63])
+      : "r"(ta), "r"(tb));
+#pragma unroll
+  for (int i = 0; i < 32; ++i) { va[i] = __uint_as_float(r[i]); vb[i] = __uint_as_float(r[32 + i]); }
+}
+
+// 32 fp32 columns of this warp's 32 TMEM lanes (the KC running sum); the
+// caller waits (tcgen05.wait::st) before reading them back
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const float* v) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%"
+      "14,%15,%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+      "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7]),
+      "f"(v[8]), "f"(v[9]), "f"(v[10]), "f"(v[11]), "f"(v[12]), "f"(v[13]), "f"(v[14]), "f"(v[15]),
+      "f"(v[16]), "f"(v[17]), "f"(v[18]), "f"(v[19]), "f"(v[20]), "f"(v[21]), "f"(v[22]),
+      "f"(v[23]), "f"(v[24]), "f"(v[25]), "f"(v[26]), "f"(v[27]), "f"(v[28]), "f"(v[29]),
+      "f"(v[30]), "f"(v[31])
+      : "memory");
+}
+
 // silu(z) = z / (1 + e^-z) with the MUFU exponential and reciprocal (~1e-7
 // relative error, far below the bf16 rounding R5 that follows; the IEEE
 // division's slow path made the SiLU epilogue of a decode gate_up tile cost
@@ -771,13 +799,17 @@ __global__ void __launch_bounds__(NT, 1)
   const uint32_t a_bytes = mh * A_BYTES, b_bytes = bn * BK * 2, st_bytes = a_bytes + b_bytes;
   // accumulator ring: mh * bn TMEM columns per stage, two stages when they fit
   const uint32_t acc_cols = mh * bn;
-  const int n_acc = 2 * acc_cols <= 512 ? 2 : 1;
+  // two-level accumulation (KC): three 128-column chunk stages and the running
+  // fp32 sum in TMEM columns [384, 512) (not in registers: 128 live floats per
+  // thread spilled, and with two stages the per-chunk merge paced the MMA —
+  // QKV at 8k tokens was 1.68x a plain 128-wide tile)
+  const int n_acc = KC ? 3 : 2 * acc_cols <= 512 ? 2 : 1;
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + n_stages * st_bytes);
   const uint32_t epi_off = n_stages * st_bytes + 512;   // 4 x [32][33] words: coalesced epilogue
   uint64_t* empty = full + n_stages;
   uint64_t* accf = empty + n_stages;
-  uint64_t* acce = accf + 2;
-  uint64_t* tqf = acce + 2;
+  uint64_t* acce = accf + 4;
+  uint64_t* tqf = acce + 4;
   uint64_t* tqe = tqf + 4;
   uint64_t* fixb = tqe + 4;   // stream-K fixup: bulk loads of partials into the (then idle) stage ring
   Seg* tile_q = reinterpret_cast<Seg*>(fixb + 2);
@@ -792,7 +824,7 @@ __global__ void __launch_bounds__(NT, 1)
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < n_stages; ++s) { mbar_init(full + s, a.split_b ? 2 : 1); mbar_init(empty + s, 1); }
-    for (int i = 0; i < 2; ++i) { mbar_init(accf + i, 1); mbar_init(acce + i, 4); }
+    for (int i = 0; i < 4; ++i) { mbar_init(accf + i, 1); mbar_init(acce + i, 4); }
     for (int i = 0; i < 4; ++i) { mbar_init(tqf + i, 1); mbar_init(tqe + i, a.split_b ? 6 : 5); }
     mbar_init(fixb, 1);
     mbar_fence_init();
@@ -1051,35 +1083,56 @@ __global__ void __launch_bounds__(NT, 1)
       TokInfo qti{0, 0};
       if (coal_qkv) qti = m_blk * mh * BM + et < a.M ? a.tok[m_blk * mh * BM + et] : TokInfo{0, 0};
       if constexpr (KC) {   // mh == 1, bn == 128, whole tiles (plan guarantees)
+        // chunk sums in IEEE fp32 in chunk order: R = R + chunk, R in TMEM
+        // columns [384, 512) of this warp's lane quadrant; the last chunk's
+        // sums go straight to the epilogue (column pairs c / c + 64: the QKV
+        // rotate-half partners, the SiLU gate / up halves)
         const int n_ch = (k_blocks + a.kcb - 1) / a.kcb;
-        float R[128];
+        const uint32_t t_r = tmem + ((uint32_t)(eq * 32) << 16) + 3 * acc_cols;
+        const int m = m_blk * BM + et;
         for (int ch = 0; ch < n_ch; ++ch) {
           mbar_wait(accf + as, aph);
           tc_fence_after();
           const uint32_t tb = tmem + ((uint32_t)(eq * 32) << 16) + as * acc_cols;
+          if (ch + 1 < n_ch) {
+#pragma unroll 1
+            for (int c = 0; c < 4; ++c) {
+              if (ch) {
+                tmem_ld32x2(tb + c * 32, t_r + c * 32, v, w);
 #pragma unroll
-          for (int c = 0; c < 4; ++c) {
-            tmem_ld32(tb + c * 32, v);
+                for (int i = 0; i < 32; ++i) v[i] = w[i] + v[i];   // chunk order: fixed
+              } else {
+                tmem_ld32(tb + c * 32, v);
+              }
+              tmem_st32(t_r + c * 32, v);
+            }
+            asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+          } else {
+#pragma unroll 1
+            for (int c = 0; c < 64; c += 32) {
+              tmem_ld32x2(tb + c, tb + c + 64, v, w);
+              if (ch) {
+                float x[32], y[32];
+                tmem_ld32x2(t_r + c, t_r + c + 64, x, y);
 #pragma unroll
-            for (int i = 0; i < 32; ++i) R[c * 32 + i] = ch ? R[c * 32 + i] + v[i] : v[i];   // chunk order: fixed
+                for (int i = 0; i < 32; ++i) { v[i] = x[i] + v[i]; w[i] = y[i] + w[i]; }
+              }
+              if (m < a.M) {
+                if (a.epi == EPI_QKV) {
+                  epi_qkv(a, m, col0 + c, v, w);
+                } else if (a.epi == EPI_SILU) {
+                  epi_store(a, m, col0 + c, v, w);
+                } else {
+                  epi_store(a, m, col0 + c, v, nullptr);
+                  epi_store(a, m, col0 + c + 64, w, nullptr);
+                }
+              }
+            }
           }
           tc_fence_before();
           __syncwarp();
           if (lane == 0) mbar_arrive(acce + as);
           if (++as == n_acc) { as = 0; aph ^= 1; }
-        }
-        const int m = m_blk * BM + et;
-        if (m < a.M) {
-          if (a.epi == EPI_QKV) {
-            epi_qkv(a, m, col0, R, R + 64);
-            epi_qkv(a, m, col0 + 32, R + 32, R + 96);
-          } else if (a.epi == EPI_SILU) {
-            epi_store(a, m, col0, R, R + 64);
-            epi_store(a, m, col0 + 32, R + 32, R + 96);
-          } else {
-#pragma unroll
-            for (int c = 0; c < 4; ++c) epi_store(a, m, col0 + c * 32, R + c * 32, nullptr);
-          }
         }
         if (a.ar.n) ar_signal(a, m_blk, mh, et);
         if (a.nf.out) norm_signal(a, m_blk, mh, et);
