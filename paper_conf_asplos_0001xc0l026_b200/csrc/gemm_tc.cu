@@ -1094,46 +1094,41 @@ __global__ void __launch_bounds__(NT, 1)
           mbar_wait(accf + as, aph);
           tc_fence_after();
           const uint32_t tb = tmem + ((uint32_t)(eq * 32) << 16) + as * acc_cols;
-          if (ch + 1 < n_ch) {
 #pragma unroll 1
-            for (int c = 0; c < 4; ++c) {
-              if (ch) {
-                tmem_ld32x2(tb + c * 32, t_r + c * 32, v, w);
+          for (int c = 0; c < 4; ++c) {
+            if (ch) {
+              tmem_ld32x2(tb + c * 32, t_r + c * 32, v, w);
 #pragma unroll
-                for (int i = 0; i < 32; ++i) v[i] = w[i] + v[i];   // chunk order: fixed
-              } else {
-                tmem_ld32(tb + c * 32, v);
-              }
-              tmem_st32(t_r + c * 32, v);
+              for (int i = 0; i < 32; ++i) v[i] = w[i] + v[i];   // chunk order: fixed
+            } else {
+              tmem_ld32(tb + c * 32, v);
             }
-            asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
-          } else {
-#pragma unroll 1
-            for (int c = 0; c < 64; c += 32) {
-              tmem_ld32x2(tb + c, tb + c + 64, v, w);
-              if (ch) {
-                float x[32], y[32];
-                tmem_ld32x2(t_r + c, t_r + c + 64, x, y);
-#pragma unroll
-                for (int i = 0; i < 32; ++i) { v[i] = x[i] + v[i]; w[i] = y[i] + w[i]; }
-              }
-              if (m < a.M) {
-                if (a.epi == EPI_QKV) {
-                  epi_qkv(a, m, col0 + c, v, w);
-                } else if (a.epi == EPI_SILU) {
-                  epi_store(a, m, col0 + c, v, w);
-                } else {
-                  epi_store(a, m, col0 + c, v, nullptr);
-                  epi_store(a, m, col0 + c + 64, w, nullptr);
-                }
-              }
-            }
+            tmem_st32(t_r + c * 32, v);
           }
+          asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+          // the stage goes back to the MMA at once — also after the last
+          // chunk, so the next tile's chunks run during this tile's stores
           tc_fence_before();
           __syncwarp();
           if (lane == 0) mbar_arrive(acce + as);
           if (++as == n_acc) { as = 0; aph ^= 1; }
         }
+        tc_fence_after();
+#pragma unroll 1
+        for (int c = 0; c < 64; c += 32) {
+          tmem_ld32x2(t_r + c, t_r + c + 64, v, w);
+          if (m < a.M) {
+            if (a.epi == EPI_QKV) {
+              epi_qkv(a, m, col0 + c, v, w);
+            } else if (a.epi == EPI_SILU) {
+              epi_store(a, m, col0 + c, v, w);
+            } else {
+              epi_store(a, m, col0 + c, v, nullptr);
+              epi_store(a, m, col0 + c + 64, w, nullptr);
+            }
+          }
+        }
+        tc_fence_before();
         if (a.ar.n) ar_signal(a, m_blk, mh, et);
         if (a.nf.out) norm_signal(a, m_blk, mh, et);
         ++it;
