@@ -1018,7 +1018,7 @@ __global__ void __launch_bounds__(NT, 1)
         uint32_t d_tmem_c = d_tmem;
         int kc0 = kb0;   // first k-block of the current accumulation chunk
         for (int kb = kb0; kb < kb1; ++kb) {
-          if (KC && kb > kb0 && (kb - kb0) % a.kcb == 0) {
+          if (KC && kb > kb0 && (kb - kb0) % a.kcb == 0 && !(a.epi_dbg & 32)) {   // (bit 5: one chunk, diagnostics)
             // two-level accumulation: hand the finished chunk to the epilogue
             // (it adds it to its fp32 registers) and start the next chunk in
             // the other accumulator stage
@@ -1087,7 +1087,7 @@ __global__ void __launch_bounds__(NT, 1)
         // columns [384, 512) of this warp's lane quadrant; the last chunk's
         // sums go straight to the epilogue (column pairs c / c + 64: the QKV
         // rotate-half partners, the SiLU gate / up halves)
-        const int n_ch = (k_blocks + a.kcb - 1) / a.kcb;
+        const int n_ch = (a.epi_dbg & 32) ? 1 : (k_blocks + a.kcb - 1) / a.kcb;
         const uint32_t t_r = tmem + ((uint32_t)(eq * 32) << 16) + 3 * acc_cols;
         const int m = m_blk * BM + et;
         for (int ch = 0; ch < n_ch; ++ch) {
@@ -1095,7 +1095,7 @@ __global__ void __launch_bounds__(NT, 1)
           tc_fence_after();
           const uint32_t tb = tmem + ((uint32_t)(eq * 32) << 16) + as * acc_cols;
 #pragma unroll 1
-          for (int c = 0; c < 4; ++c) {
+          for (int c = 0; c < ((a.epi_dbg & 16) ? 0 : 4); ++c) {   // (diagnostics: bit 4 skips the merge)
             if (ch) {
               tmem_ld32x2(tb + c * 32, t_r + c * 32, v, w);
 #pragma unroll
@@ -1114,10 +1114,31 @@ __global__ void __launch_bounds__(NT, 1)
           if (++as == n_acc) { as = 0; aph ^= 1; }
         }
         tc_fence_after();
+        // the tile's stores: the coalesced (shared-memory transposed) forms of
+        // the whole-tile epilogues where they exist — per-row stores here made
+        // the 128-wide KC tile 27 % slower than a plain one even with a single chunk
+        float* wb = reinterpret_cast<float*>(smem + epi_off) + eq * (32 * 33);
+        const TokInfo ti = (a.epi == EPI_QKV && a.epi_coal && m < a.M) ? a.tok[m] : TokInfo{0, 0};
 #pragma unroll 1
         for (int c = 0; c < 64; c += 32) {
           tmem_ld32x2(t_r + c, t_r + c + 64, v, w);
-          if (m < a.M) {
+          if (a.epi_coal && a.epi == EPI_QKV) {
+            float4 csv[16];
+            if (((col0 + c) >> 7) < a.H + a.Hkv) {
+              const float4* cs = qkv_cs_row(a, ti, c);
+#pragma unroll
+              for (int j = 0; j < 16; ++j) csv[j] = cs[j];
+            }
+            epi_qkv_coal(a, reinterpret_cast<uint32_t*>(wb), m, col0 + c, lane, v, w, ti, csv);
+          } else if (a.epi_coal && a.epi == EPI_SILU) {
+            epi_chunk_coalesced(a, wb, m - lane, col0 + c, lane, v, w, nullptr);
+          } else if (a.epi_coal && a.epi == EPI_RESID) {
+            float4 rr[8];
+            epi_resid_load(a, m - lane, col0 + c, lane, rr);
+            epi_chunk_coalesced(a, wb, m - lane, col0 + c, lane, v, nullptr, rr);
+            epi_resid_load(a, m - lane, col0 + c + 64, lane, rr);
+            epi_chunk_coalesced(a, wb, m - lane, col0 + c + 64, lane, w, nullptr, rr);
+          } else if (m < a.M) {
             if (a.epi == EPI_QKV) {
               epi_qkv(a, m, col0 + c, v, w);
             } else if (a.epi == EPI_SILU) {

@@ -80,7 +80,8 @@ struct GemmArgs {
   int epi_pf;               // epilogue warps L2-prefetch their tile's inputs (residual rows, RoPE rows)
                             // when they learn the unit, i.e. while the mainloop streams (1 = on)
   int epi_dbg;              // diagnostics (BULLET_GEMM_EPI_DBG; wrong results): bit 0 no SiLU math,
-                            // bit 1 no output stores, bit 2 no residual loads, bit 3 no RoPE-table loads
+                            // bit 1 no output stores, bit 2 no residual loads, bit 3 no RoPE-table loads,
+                            // bit 4 no two-level-accumulation merge, bit 5 one accumulation chunk per tile
   int kcb;                  // two-level accumulation (DESIGN R-4e): K chunk in k-blocks (0 = off);
                             // each chunk accumulates in TMEM, the chunks are summed in fp32
                             // registers by the epilogue (requires mh == 1, bn == 128, whole tiles)

@@ -1,0 +1,13 @@
+#!/bin/bash
+# KC GEMM diagnosis 3: one chunk with / without the TMEM copy of the sum (bits 5 / 4+5), stores off (bit 1).
+set -u
+O=gpurun_out/s40; mkdir -p $O
+run() { local tag=$1; shift; echo "== $tag" >> $O/prof.log; env "$@" timeout 300 python scripts/prof_step.py --reps 3 --mode pre --p 148 --config arxiv-8b >> $O/prof.log 2>&1; }
+for rep in 1 2; do
+  run bn128 BULLET_GEMM_PLAN_K2P=1,128,0 BULLET_GEMM_PLAN_K5P=1,128,0
+  run bn128_nostore BULLET_GEMM_PLAN_K2P=1,128,0 BULLET_GEMM_PLAN_K5P=1,128,0 BULLET_GEMM_EPI_DBG=2
+  run kc_one BULLET_GEMM_KCHUNK=256 BULLET_GEMM_EPI_DBG=32
+  run kc_one_nocopy BULLET_GEMM_KCHUNK=256 BULLET_GEMM_EPI_DBG=48
+  run kc_one_nocopy_nostore BULLET_GEMM_KCHUNK=256 BULLET_GEMM_EPI_DBG=50
+done
+grep -E "==|qkv|o_proj" $O/prof.log
