@@ -637,6 +637,7 @@ def main():
     S.bl.set_phase_scale(t_pre_full / (S.bl.predict_us(qp, cp, N, 0) / 1e3),
                          t_dec_full / (S.bl.predict_us(qd, cdc, N, 0) / 1e3))
     feedback = []
+    sc0, sb0 = S.bl.colocation()
     for _ in range(args.feedback):
         ps = tuple(broadcast_obj(S.bl.choose_split(state, slo), ws))
         if not (0 < ps[0] < N and ps[1] >= 1):
@@ -645,8 +646,14 @@ def main():
         tp_co, td_co = S.time_phases(5, fp, fk)
         pred_tp = S.bl.predict_us(qp, cp, fp, N - fp) / 1e3
         pred_td = S.bl.predict_us(qd, cdc, N - fp, fp) / 1e3 * fk
+        # damped (half steps in log space) and bounded to [0.8, 1.25] x the
+        # fitted factors: one cycle measured in a different power state must
+        # not walk the decision off to a degenerate split (seen once: p_c at
+        # 0.73 after three full-step cycles, split (52, 11) at 1.12x)
         sc, sb = S.bl.colocation()
-        S.bl.set_colocation(sc * pred_tp / tp_co, sb * pred_td / td_co)
+        nc = min(1.25 * sc0, max(0.8 * sc0, sc * math.sqrt(pred_tp / tp_co)))
+        nb = min(1.25 * sb0, max(0.8 * sb0, sb * math.sqrt(pred_td / td_co)))
+        S.bl.set_colocation(nc, nb)
         feedback.append({"p": fp, "k": fk, "prefill_ms": tp_co, "decode_ms": td_co,
                          "predicted_prefill_ms": pred_tp, "predicted_decode_ms": pred_td})
     model_split = tuple(broadcast_obj(S.bl.choose_split(state, slo), ws))

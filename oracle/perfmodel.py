@@ -166,7 +166,7 @@ def evaluate_split(P, model, state, slo, u, v):
     return p90(ttft, pct), p90(tpot, pct), t_p
 
 
-GAIN_TOL = 0.03   # R-23: the model's resolution for the gain objective
+GAIN_TOL = 0.06   # R-23: the model's resolution for the gain objective (held-out MRE ~6 %)
 
 
 def candidates(P, slo, gran):
