@@ -1017,11 +1017,15 @@ __global__ void __launch_bounds__(NT, 1)
         const uint32_t d_tmem = tmem + as * acc_cols;
         uint32_t d_tmem_c = d_tmem;
         int kc0 = kb0;   // first k-block of the current accumulation chunk
+        // k-blocks left in the current chunk (a countdown: no integer division
+        // on the MMA issuer's path)
+        int kc_left = (KC && !(a.epi_dbg & 32)) ? a.kcb : 1 << 30;   // (bit 5: one chunk, diagnostics)
         for (int kb = kb0; kb < kb1; ++kb) {
-          if (KC && kb > kb0 && (kb - kb0) % a.kcb == 0 && !(a.epi_dbg & 32)) {   // (bit 5: one chunk, diagnostics)
+          if (KC && kc_left == 0) {
             // two-level accumulation: hand the finished chunk to the epilogue
-            // (it adds it to its fp32 registers) and start the next chunk in
-            // the other accumulator stage
+            // (it adds it to the running sum) and start the next chunk in the
+            // next accumulator stage
+            kc_left = a.kcb;
             if (elect_one()) tc_commit(accf + as);
             __syncwarp();
             if (++as == n_acc) { as = 0; aph ^= 1; }
@@ -1030,6 +1034,7 @@ __global__ void __launch_bounds__(NT, 1)
             d_tmem_c = tmem + as * acc_cols;
             kc0 = kb;
           }
+          if (KC) --kc_left;
           mbar_wait(full + s, ph);
           tc_fence_after();
           const uint32_t a_addr = smem_u32(smem + s * st_bytes), b_addr = a_addr + a_bytes;
