@@ -1038,12 +1038,15 @@ __global__ void __launch_bounds__(NT, 1)
           mbar_wait(full + s, ph);
           tc_fence_after();
           const uint32_t a_addr = smem_u32(smem + s * st_bytes), b_addr = a_addr + a_bytes;
+          // two descriptors per stage; the k steps / row halves only move the
+          // start-address field (addr >> 4 < 2^14: no carry out of it)
+          const uint64_t da = sw128_desc(a_addr), db = sw128_desc(b_addr);
           if (elect_one()) {
 #pragma unroll
             for (int k = 0; k < BK / 16; ++k)
 #pragma unroll
               for (int hh = 0; hh < mh; ++hh)
-                tc_mma(d_tmem_c + hh * bn, sw128_desc(a_addr + hh * A_BYTES + k * 32), sw128_desc(b_addr + k * 32),
+                tc_mma(d_tmem_c + hh * bn, da + (uint64_t)((hh * A_BYTES + k * 32) >> 4), db + (uint64_t)(k * 2),
                        idesc, (kb > kc0 || k > 0) ? 1u : 0u);
             tc_commit(empty + s);
           }
